@@ -1,0 +1,486 @@
+"""ORACLE (test infrastructure) -- C2: scheduling-policy reference + discrete-event
+simulator, step by step in the paper's order.
+
+Paper: §6 "Scheduling Strategy" (PAPER.md P1222-1323): (1) SRPT on the remaining
+time  remaining = sum_{i in K} max(0, C_i - c_i) * T_i  (P1257-1261), (2) deficit
+counters -- the scheduled user's deficit drops by (1 - 1/#users), every other
+user's rises by 1/#users; above a threshold the oldest job of the highest-deficit
+client is chosen (P1287-1298), (3) B blocks of slack beyond full utilisation
+(P1300-1304), and the dispatch loop (P1306-1314).  Notification semantics: Fig. 6
+(P848-870), flow control (P1115-1119), block groups of <=16 (P1138-1142).  Resource
+accounting: Table 1 (P782-802).  Every reading of a silent/garbled passage is
+SURVEY.md §8(c) C2-Q1..Q20, restated in DESIGN.md §"Readings".
+
+The state machine ``Policy`` is the reference for the C++ dispatcher: replaying the
+dispatcher's event log through it (``replay``) must reproduce the dispatcher's issue
+sequence (uid, job, layer, stream) bit-exactly (pin S6).  All quantities are
+integers: times in ns, deficits in units of 1/N with a global offset Omega
+(the paper's O(1) threshold-shift trick, P1316-1323, in integer form).
+
+``SyntheticGPU`` + ``simulate`` model a GPU (S SMs with Table-1 resources, H FIFO
+hardware queues, greedy placement, launch/notification delays) driving either the
+Paella dispatcher (``Policy``) or the naive submit-everything-at-arrival baseline.
+It backs the brute-force and closed-form pins (S1-S3), the invariants (S5) and
+what-if sweeps; it is not expected to reproduce B200 timing.
+"""
+from __future__ import annotations
+
+import heapq
+import itertools
+from dataclasses import dataclass, field
+
+PLACEMENT, COMPLETION = 1, 2
+SRPT_DEFICIT, FIFO = 0, 1
+RESOURCES = ("blocks", "warps", "regs", "smem", "tmem")
+INF_THETA = (1 << 63) - 1
+
+
+@dataclass
+class Layer:
+    grid: int
+    demand: tuple          # per-block demand, one int per RESOURCES entry (blocks=1)
+    tbar: int              # profiled mean kernel time, ns (frozen)
+    dur: int = 0           # synthetic-mode block duration, ns
+
+
+@dataclass
+class Config:
+    num_clients: int
+    policy: int = SRPT_DEFICIT
+    theta: int = 100                  # fairness threshold in kernel dispatches
+    slack: int = 148                  # B, in blocks
+    group: int = 16                   # G
+    ring_capacity: int = 65536
+    streams: int = 32                 # P
+    capacity: tuple = (148 * 32, 148 * 64, 148 * 65536, 148 * 233472, 148 * 512)
+
+
+def groups(g, G):
+    return -(-g // G)
+
+
+@dataclass
+class Job:
+    id: int
+    client: int
+    model: int
+    seq: int
+    R: int
+    cursor: int = 0
+    inflight: bool = False
+    last_stream: int = -1
+
+
+@dataclass
+class Launch:
+    uid: int
+    job: int
+    layer: int
+    grid: int
+    demand: tuple
+    stream: int
+    p: int = 0
+    f: int = 0
+
+
+class Policy:
+    """The dispatcher state machine of SURVEY.md §8(c) C2, integer-exact."""
+
+    def __init__(self, cfg: Config, models: list[list[Layer]]):
+        self.cfg = cfg
+        self.models = models
+        self.jobs: dict[int, Job] = {}
+        self.launches: dict[int, Launch] = {}
+        self.U = [0] * len(RESOURCES)
+        self.Q = 0
+        self.O = 0
+        self.free = set(range(cfg.streams))
+        self.Dt = [0] * cfg.num_clients      # stored deficits D~_c
+        self.Omega = 0                       # global offset
+        self.unfinished = [0] * cfg.num_clients
+        self.next_uid = 0
+        self.next_seq = 0
+        self.completed: list[int] = []
+        self.issues: list[tuple] = []
+        self.checks = True                   # assert invariants (c),(d),(g) as we go
+        self.log: list[tuple] | None = None  # consumed-event log in replay format
+
+    # effective deficit, units of 1/N
+    def D(self, c):
+        return self.Dt[c] + self.Omega
+
+    def remaining(self, model, cursor):
+        """R_j = sum of T-bar over kernels not yet dispatched (C2-Q8, C2-Q9)."""
+        return sum(l.tbar for l in self.models[model][cursor:])
+
+    # --- events -------------------------------------------------------------
+    def arrival(self, job_id, client, model):
+        if self.unfinished[client] == 0:          # C2-Q11: idle client restarts at 0
+            self.Dt[client] = -self.Omega
+        self.unfinished[client] += 1
+        if self.log is not None:
+            self.log.append((EV_ARRIVAL, job_id, client, model))
+        j = Job(job_id, client, model, self.next_seq, self.remaining(model, 0))
+        self.next_seq += 1
+        self.jobs[job_id] = j
+        return j
+
+    def record(self, typ, uid, n):
+        """Consume one notification record (type, launch uid, block count)."""
+        L = self.launches[uid]
+        self.O -= 1
+        if self.log is not None:
+            self.log.append((EV_RECORD, typ, uid, n))
+        old = max(L.p, L.f)
+        if typ == PLACEMENT:
+            L.p += n
+        elif typ == COMPLETION:
+            L.f += n
+            for r in range(len(RESOURCES)):
+                self.U[r] -= n * L.demand[r]
+        else:
+            raise ValueError(typ)
+        self.Q -= max(L.p, L.f) - old
+        assert L.p <= L.grid and L.f <= L.grid
+        done = None
+        if L.f == L.grid:
+            del self.launches[uid]
+            self.free.add(L.stream)
+            j = self.jobs[L.job]
+            j.inflight = False
+            j.cursor += 1
+            j.last_stream = L.stream
+            if j.cursor == len(self.models[j.model]):
+                if self.checks:
+                    assert j.R == 0
+                del self.jobs[j.id]
+                self.unfinished[j.client] -= 1
+                self.completed.append(j.id)
+                if self.log is not None:
+                    self.log.append((EV_COMPLETE, j.id))
+                done = j.id
+        return done
+
+    def ready(self):
+        return [j for j in self.jobs.values()
+                if not j.inflight and j.cursor < len(self.models[j.model])]
+
+    def pick(self, rdy):
+        cfg = self.cfg
+        if cfg.policy == FIFO:
+            return min(rdy, key=lambda j: j.seq)
+        clients = sorted({j.client for j in rdy})
+        cstar = max(clients, key=lambda c: (self.D(c), -c))
+        if cfg.theta != INF_THETA and self.D(cstar) > cfg.theta * cfg.num_clients:
+            return min((j for j in rdy if j.client == cstar), key=lambda j: j.seq)
+        return min(rdy, key=lambda j: (j.R, j.seq, j.id))
+
+    def predicate(self, grid):
+        cfg = self.cfg
+        fits = self.Q < cfg.slack or all(u < c for u, c in zip(self.U, cfg.capacity))
+        ring_ok = self.O + 2 * groups(grid, cfg.group) <= cfg.ring_capacity
+        return fits and ring_ok
+
+    def decide(self):
+        """Dispatch loop (P1306-1314). Returns the list of issues made."""
+        cfg = self.cfg
+        out = []
+        if self.log is not None:
+            self.log.append((EV_BATCH_END,))
+        while True:
+            if not self.free:
+                break
+            rdy = self.ready()
+            if not rdy:
+                break
+            j = self.pick(rdy)
+            layer = self.models[j.model][j.cursor]
+            if not self.predicate(layer.grid):
+                break
+            uid = self.next_uid
+            self.next_uid += 1
+            stream = j.last_stream if j.last_stream in self.free else min(self.free)
+            self.free.remove(stream)
+            self.launches[uid] = Launch(uid, j.id, j.cursor, layer.grid, layer.demand, stream)
+            for r in range(len(RESOURCES)):
+                self.U[r] += layer.grid * layer.demand[r]
+            self.Q += layer.grid
+            self.O += 2 * groups(layer.grid, cfg.group)
+            j.R -= layer.tbar
+            j.inflight = True
+            if self.checks:
+                assert j.R >= 0
+            self.Dt[j.client] -= cfg.num_clients
+            self.Omega += 1
+            rec = (uid, j.id, j.cursor, stream)
+            if self.log is not None:
+                self.log.append((EV_ISSUE,) + rec)
+            out.append(rec)
+            self.issues.append(rec)
+        return out
+
+
+# ---------------------------------------------------------------------------
+# Replay mode (pin S6)
+# ---------------------------------------------------------------------------
+
+EV_ARRIVAL, EV_RECORD, EV_BATCH_END, EV_ISSUE, EV_COMPLETE = 1, 2, 3, 4, 5
+
+
+def replay(cfg: Config, models, events):
+    """Drive ``Policy`` with a recorded event sequence.
+
+    events: iterable of tuples
+      (EV_ARRIVAL, job_id, client, model) | (EV_RECORD, type, uid, n) |
+      (EV_BATCH_END,) | (EV_ISSUE, uid, job, layer, stream) | (EV_COMPLETE, job_id)
+    Inputs (arrivals, records, batch ends) are applied in order; the policy's own
+    issues / completions are compared with the logged ones.  Returns
+    (ok, first_divergence_message, n_issues_checked).
+    """
+    pol = Policy(cfg, models)
+    expect = []            # issues the policy produced, awaiting the logged ones
+    expect_done = []
+    n = 0
+    for ev in events:
+        k = ev[0]
+        if k == EV_ARRIVAL:
+            pol.arrival(ev[1], ev[2], ev[3])
+        elif k == EV_RECORD:
+            d = pol.record(ev[1], ev[2], ev[3])
+            if d is not None:
+                expect_done.append(d)
+        elif k == EV_BATCH_END:
+            if expect:
+                return False, f"dispatcher issued fewer kernels than the reference: missing {expect[0]}", n
+            expect = list(pol.decide())
+        elif k == EV_ISSUE:
+            got = tuple(ev[1:5])
+            if not expect:
+                return False, f"dispatcher issued {got} where the reference issues nothing", n
+            want = expect.pop(0)
+            if want != got:
+                return False, f"issue #{n}: dispatcher {got} != reference {want}", n
+            n += 1
+        elif k == EV_COMPLETE:
+            if not expect_done or expect_done[0] != ev[1]:
+                return False, f"completion {ev[1]} != reference {expect_done[:1]}", n
+            expect_done.pop(0)
+    if expect:
+        return False, f"log ends with reference issues pending: {expect[0]}", n
+    return True, "", n
+
+
+# ---------------------------------------------------------------------------
+# Synthetic mode: a GPU model
+# ---------------------------------------------------------------------------
+
+@dataclass
+class GPUModel:
+    sms: int = 148
+    per_sm: tuple = (32, 64, 65536, 233472, 512)   # Table 1 + TMEM, per SM
+    hw_queues: int = 32                            # H
+    launch_delay: int = 0                          # delta_l, ns
+    notif_delay: int = 0                           # delta_n, ns
+
+
+@dataclass
+class SimResult:
+    arrival: dict = field(default_factory=dict)
+    finish: dict = field(default_factory=dict)
+    issues: list = field(default_factory=list)
+    records: list = field(default_factory=list)    # (t, type, uid, n, group)
+    blocks: list = field(default_factory=list)     # (uid, sm, t_start, t_end)
+    max_running_blocks: int = 0
+    busy_block_time: int = 0
+    violations: list = field(default_factory=list)
+    policy: Policy | None = None
+
+    def jct(self):
+        return {j: self.finish[j] - self.arrival[j] for j in self.finish}
+
+
+class _Kernel:
+    __slots__ = ("uid", "job", "layer", "grid", "demand", "dur", "stream", "placed", "done",
+                 "start_count", "end_count")
+
+    def __init__(self, uid, job, layer, grid, demand, dur, stream):
+        self.uid, self.job, self.layer = uid, job, layer
+        self.grid, self.demand, self.dur, self.stream = grid, demand, dur, stream
+        self.placed = self.done = 0
+        self.start_count = self.end_count = 0
+
+
+def simulate(cfg: Config, models, trace, gpu: GPUModel, system="paella", naive_streams=None,
+             check=True, horizon=None):
+    """Event-driven simulation.
+
+    trace: list of (t_arrival_ns, client, model).  system: 'paella' (Policy drives
+    issue) or 'naive' (every kernel of a job enters stream job % naive_streams at
+    arrival; the hardware model decides everything).  Returns SimResult.
+    """
+    res = SimResult()
+    S = gpu.sms
+    free_sm = [list(gpu.per_sm) for _ in range(S)]
+    hwq = [[] for _ in range(gpu.hw_queues)]       # FIFO of _Kernel per hardware queue
+    stream_busy_until_done = {}                    # stream -> kernel currently ahead
+    stream_fifo = {}                               # stream -> list of kernels (stream order)
+    evq = []
+    cnt = itertools.count()
+
+    def push(t, kind, *a):
+        heapq.heappush(evq, (t, next(cnt), kind, a))
+
+    pol = Policy(cfg, models) if system == "paella" else None
+    if pol is not None:
+        pol.checks = check
+    res.policy = pol
+    naive_streams = naive_streams or cfg.streams
+    running_blocks = 0
+    uid_counter = itertools.count()
+
+    for jid, (t, c, m) in enumerate(trace):
+        push(t, "arrival", jid, c, m)
+
+    def enqueue_kernel(k):
+        # CUDA stream semantics: a kernel waits for its stream predecessor; the
+        # stream is bound to hardware queue stream % H (FIFO, head-of-line).
+        stream_fifo.setdefault(k.stream, []).append(k)
+        hwq[k.stream % gpu.hw_queues].append(k)
+
+    def try_place(t):
+        nonlocal running_blocks
+        progress = True
+        while progress:
+            progress = False
+            for q in hwq:
+                if not q:
+                    continue
+                k = q[0]
+                # the head kernel must also be the head of its stream
+                if stream_fifo[k.stream][0] is not k:
+                    continue
+                while k.placed < k.grid:
+                    sm = next((i for i in range(S)
+                               if all(free_sm[i][r] >= k.demand[r] for r in range(len(RESOURCES)))), None)
+                    if sm is None:
+                        break
+                    for r in range(len(RESOURCES)):
+                        free_sm[sm][r] -= k.demand[r]
+                    k.placed += 1
+                    running_blocks += 1
+                    res.max_running_blocks = max(res.max_running_blocks, running_blocks)
+                    progress = True
+                    push(t, "block_start", k, sm)
+                    push(t + k.dur, "block_end", k, sm, t)
+                if k.placed == k.grid:
+                    q.pop(0)
+                    progress = True
+
+    def emit(t, typ, k, count):
+        G = cfg.group
+        if count % G == 0 or count == k.grid:
+            n = G if count % G == 0 else count % G
+            grp = (count - 1) // G
+            res.records.append((t, typ, k.uid, n, grp))
+            if pol is not None:
+                push(t + gpu.notif_delay, "record", typ, k.uid, n)
+
+    def dispatch(t):
+        for (uid, jid, layer, stream) in pol.decide():
+            m = pol.jobs[jid].model
+            L = models[m][layer]
+            res.issues.append((t, uid, jid, layer, stream))
+            push(t + gpu.launch_delay, "launch",
+                 _Kernel(uid, jid, layer, L.grid, L.demand, L.dur, stream))
+
+    kernels_left = {}
+    while evq:
+        t, _, kind, a = heapq.heappop(evq)
+        if horizon is not None and t > horizon:
+            break
+        if kind == "arrival":
+            jid, c, m = a
+            res.arrival[jid] = t
+            if pol is not None:
+                pol.arrival(jid, c, m)
+            else:
+                s = jid % naive_streams
+                kernels_left[jid] = len(models[m])
+                for li, L in enumerate(models[m]):
+                    k = _Kernel(next(uid_counter), jid, li, L.grid, L.demand, L.dur, s)
+                    res.issues.append((t, k.uid, jid, li, s))
+                    enqueue_kernel(k)
+                try_place(t)
+        elif kind == "launch":
+            enqueue_kernel(a[0])
+            try_place(t)
+        elif kind == "block_start":
+            k, sm = a
+            k.start_count += 1
+            emit(t, PLACEMENT, k, k.start_count)
+        elif kind == "block_end":
+            k, sm, t0 = a
+            for r in range(len(RESOURCES)):
+                free_sm[sm][r] += k.demand[r]
+            running_blocks -= 1
+            res.busy_block_time += t - t0
+            res.blocks.append((k.uid, sm, t0, t))
+            k.end_count += 1
+            emit(t, COMPLETION, k, k.end_count)
+            if k.end_count == k.grid:
+                fifo = stream_fifo[k.stream]
+                assert fifo[0] is k
+                fifo.pop(0)
+                if pol is None:
+                    kernels_left[k.job] -= 1
+                    if kernels_left[k.job] == 0:
+                        res.finish[k.job] = t
+            try_place(t)
+        elif kind == "record":
+            typ, uid, n = a
+            done = pol.record(typ, uid, n)
+            if done is not None:
+                res.finish[done] = t
+        # the dispatcher decides once every event of this instant is consumed
+        if pol is not None and (not evq or evq[0][0] > t):
+            dispatch(t)
+        if check:
+            for i in range(S):
+                if any(v < 0 for v in free_sm[i]):
+                    res.violations.append(("capacity", t, i))
+    return res
+
+
+# ---------------------------------------------------------------------------
+# Invariants (pin S5), usable on simulator results and on GPU event logs
+# ---------------------------------------------------------------------------
+
+def check_exactly_once(records, grids, G):
+    """(b): per uid, sum of PLACEMENT counts = sum of COMPLETION counts = grid,
+    ceil(grid/G) records per type, group indices unique and covering [0, ceil)."""
+    per = {}
+    for rec in records:
+        _, typ, uid, n, grp = rec
+        per.setdefault((uid, typ), []).append((grp, n))
+    bad = []
+    for uid, g in grids.items():
+        for typ in (PLACEMENT, COMPLETION):
+            lst = per.get((uid, typ), [])
+            ng = groups(g, G)
+            gs = sorted(x[0] for x in lst)
+            if gs != list(range(ng)) or sum(x[1] for x in lst) != g:
+                bad.append((uid, typ, lst))
+    return bad
+
+
+def deficit_bound_holds(trace_of_D, N, theta):
+    """(f): for a client continuously ready since s, D(t) <= max(D(s), theta*N) + N."""
+    bad = []
+    for c, series in trace_of_D.items():
+        if not series:
+            continue
+        d0 = series[0]
+        for d in series:
+            if d > max(d0, theta * N) + N:
+                bad.append((c, d0, d))
+    return bad

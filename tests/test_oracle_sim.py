@@ -1,0 +1,342 @@
+"""Pins for oracle C2 (policy reference + discrete-event simulator), SURVEY.md §8(c):
+
+S1a  brute force: single server, all releases at 0 -> SRPT total JCT = exhaustive min
+S1b  brute force: unit kernels, integer releases -> SRPT = exhaustive min incl. idling
+S1c  SRPT is NOT optimal in general (counterexample kept as a regression guard)
+S2   Fig. 1 setup (P214-219): 4 jobs x 3 unit kernels, 2 SMs -> mean JCT 4.5
+S3   Fig. 2 closed form (P431-442): naive job-by-job submission caps running
+     kernels at H = 32 of 176; the dispatcher reaches 176
+S4   special cases: theta=inf / N=1 => SRPT; theta=0 => round-robin windows; FIFO order
+S5   invariants: capacity, exactly-once records, dependency, predicate, deficit
+     rule and bound, R_j >= 0
+S6   replay of the policy's own consumed-event log reproduces its issue sequence
+"""
+import itertools
+import random
+from functools import lru_cache
+
+import pytest
+
+from oracle import sim
+from oracle.sim import Config, GPUModel, Layer
+
+UNIT = 1000  # ns per time unit
+
+
+def whole_sm_models(job_lens_units):
+    """Each kernel = 1 block that takes a whole SM (per-SM block capacity 1)."""
+    return [[Layer(1, (1, 1, 1, 1, 0), d * UNIT, d * UNIT) for d in lens] for lens in job_lens_units]
+
+
+def single_server_cfg(n_clients=1, sms=1):
+    return Config(num_clients=n_clients, theta=sim.INF_THETA, slack=0, group=16,
+                  capacity=(sms, 10**9, 10**12, 10**12, 10**9))
+
+
+ONE_SM = GPUModel(sms=1, per_sm=(1, 64, 65536, 233472, 512), hw_queues=32)
+
+
+def brute_min_total_completion(jobs):
+    """All interleavings (each job's kernels in order), single server, no idling."""
+    best = None
+    n = len(jobs)
+    seq = [i for i, lens in enumerate(jobs) for _ in lens]
+    for perm in set(itertools.permutations(seq)):
+        t, cur, fin = 0, [0] * n, [0] * n
+        for i in perm:
+            t += jobs[i][cur[i]]
+            cur[i] += 1
+            if cur[i] == len(jobs[i]):
+                fin[i] = t
+        tot = sum(fin)
+        best = tot if best is None else min(best, tot)
+    return best
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_S1a_srpt_optimal_all_released_at_zero(seed):
+    r = random.Random(seed)
+    jobs = [[r.randint(1, 9) for _ in range(r.randint(1, 3))] for _ in range(r.randint(2, 4))]
+    models = whole_sm_models(jobs)
+    trace = [(0, 0, m) for m in range(len(jobs))]
+    res = sim.simulate(single_server_cfg(), models, trace, ONE_SM)
+    assert sum(res.jct().values()) == brute_min_total_completion(jobs) * UNIT
+
+
+def brute_unit_with_releases(lens, rel):
+    """Exact min total JCT for unit kernels with integer releases, idling allowed."""
+    n = len(lens)
+
+    @lru_cache(None)
+    def go(t, rem):
+        if all(x == 0 for x in rem):
+            return 0
+        best = None
+        opts = [i for i in range(n) if rem[i] > 0 and rel[i] <= t]
+        choices = opts + [None]
+        for c in choices:
+            if c is None:
+                if all(rel[i] <= t for i in range(n) if rem[i] > 0):
+                    continue   # idling only helps while something is unreleased
+                v = go(t + 1, rem)
+            else:
+                nr = list(rem)
+                nr[c] -= 1
+                v = go(t + 1, tuple(nr)) + ((t + 1 - rel[c]) if nr[c] == 0 else 0)
+            best = v if best is None else min(best, v)
+        return best
+
+    return go(0, tuple(lens))
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_S1b_srpt_optimal_unit_kernels_with_releases(seed):
+    r = random.Random(1000 + seed)
+    n = r.randint(2, 4)
+    lens = [r.randint(1, 3) for _ in range(n)]
+    rel = [r.randint(0, 4) for _ in range(n)]
+    models = whole_sm_models([[1] * k for k in lens])
+    trace = sorted([(rel[i] * UNIT, 0, i) for i in range(n)], key=lambda x: x[0])
+    res = sim.simulate(single_server_cfg(), models, trace, ONE_SM)
+    assert sum(res.jct().values()) == brute_unit_with_releases(tuple(lens), tuple(rel)) * UNIT
+
+
+def test_S1c_srpt_not_optimal_in_general():
+    # jobs [[4],[3,7]] released at [6,5]: SRPT total 20 vs optimum 19 (optimum idles)
+    models = whole_sm_models([[4], [3, 7]])
+    trace = [(5 * UNIT, 0, 1), (6 * UNIT, 0, 0)]
+    res = sim.simulate(single_server_cfg(), models, trace, ONE_SM)
+    assert sum(res.jct().values()) == 20 * UNIT
+
+
+def test_S2_fig1_setup():
+    models = whole_sm_models([[1, 1, 1]] * 4)
+    trace = [(0, 0, i) for i in range(4)]
+    gpu = GPUModel(sms=2, per_sm=(1, 64, 65536, 233472, 512))
+    res = sim.simulate(single_server_cfg(sms=2), models, trace, gpu)
+    jct = sorted(res.jct().values())
+    assert sum(jct) / 4 == 4.5 * UNIT
+    assert jct == [3 * UNIT, 3 * UNIT, 6 * UNIT, 6 * UNIT]
+
+
+def test_S3_fig2_hol_blocking_closed_form():
+    # GTX 1660 SUPER: 22 SMs x 1024 threads, 32 HW queues; jobs of 8 kernels, each
+    # 1 block x 128 threads (4 warps), 9 regs, no smem, ~300 us.  176 could run.
+    per_sm = (32, 32, 65536, 100 * 1024, 512)
+    gpu = GPUModel(sms=22, per_sm=per_sm, hw_queues=32)
+    regs = -(-9 * 32 // 256) * 256 * 4
+    layer = Layer(1, (1, 4, regs, 0, 0), 300_000, 300_000)
+    models = [[layer] * 8]
+    trace = [(0, 0, 0)] * 400
+    naive = sim.simulate(Config(num_clients=1), models, trace, gpu, system="naive",
+                         naive_streams=400, horizon=2_000_000)
+    assert naive.max_running_blocks == 32          # 32/176 = 18%
+    cap = tuple(22 * x for x in per_sm)
+    cfg = Config(num_clients=1, slack=0, capacity=cap, streams=176)
+    gpu176 = GPUModel(sms=22, per_sm=per_sm, hw_queues=176)
+    paella = sim.simulate(cfg, models, trace, gpu176, horizon=2_000_000)
+    assert paella.max_running_blocks == 176        # 176/176
+
+
+def random_models(r, n_models=3):
+    ms = []
+    for _ in range(n_models):
+        ms.append([Layer(r.randint(1, 40), (1, r.choice([4, 8]), 4096 * r.randint(1, 4),
+                                            r.choice([0, 8192, 40960]), r.choice([0, 0, 32])),
+                         tb, tb)
+                   for tb in (r.randint(1, 20) * 500 for _ in range(r.randint(1, 6)))])
+    return ms
+
+
+def random_trace(r, n, n_clients, n_models, rate_ns=3000):
+    t, out = 0, []
+    for _ in range(n):
+        t += int(r.expovariate(1.0 / rate_ns))
+        out.append((t, r.randrange(n_clients), r.randrange(n_models)))
+    return out
+
+
+@pytest.mark.parametrize("policy", [sim.SRPT_DEFICIT, sim.FIFO])
+@pytest.mark.parametrize("seed", range(6))
+def test_S5_invariants_and_S6_self_replay(seed, policy):
+    r = random.Random(seed)
+    models = random_models(r)
+    gpu = GPUModel(sms=8, per_sm=(32, 64, 65536, 233472, 512), launch_delay=700, notif_delay=900)
+    N = 3
+    cfg = Config(num_clients=N, policy=policy, theta=r.choice([0, 1, 5, 100]), slack=r.choice([0, 8, 16]),
+                 group=r.choice([1, 4, 16]), ring_capacity=256, streams=r.choice([4, 32]),
+                 capacity=tuple(8 * x for x in (32, 64, 65536, 233472, 512)))
+    trace = random_trace(r, 150, N, len(models))
+    res = sim.simulate(cfg, models, trace, gpu)
+    assert not res.violations                                  # (a) per-SM capacity
+    assert len(res.finish) == len(trace)                       # everything completes
+    # (b) exactly once
+    grids = {}
+    for (t, uid, jid, layer, stream) in res.issues:
+        grids[uid] = models[trace[jid][2]][layer].grid
+    assert sim.check_exactly_once(res.records, grids, cfg.group) == []
+    # (c) dependency: kernel k+1 of a job issued after kernel k's last completion
+    last_done = {}
+    for (t, typ, uid, n, grp) in res.records:
+        if typ == sim.COMPLETION:
+            last_done[uid] = t
+    by_job = {}
+    for (t, uid, jid, layer, stream) in res.issues:
+        by_job.setdefault(jid, []).append((layer, t, uid))
+    for jid, lst in by_job.items():
+        lst.sort()
+        assert [x[0] for x in lst] == list(range(len(models[trace[jid][2]])))
+        for (l0, t0, u0), (l1, t1, u1) in zip(lst, lst[1:]):
+            assert t1 >= last_done[u0]
+
+
+def _run_policy_with_log(cfg, models, trace, gpu):
+    """simulate() with the Policy event log switched on."""
+    orig = sim.Policy.__init__
+
+    def init(self, *a, **k):
+        orig(self, *a, **k)
+        self.log = []
+    sim.Policy.__init__ = init
+    try:
+        return sim.simulate(cfg, models, trace, gpu)
+    finally:
+        sim.Policy.__init__ = orig
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_S6_replay_reproduces_issue_order(seed):
+    r = random.Random(50 + seed)
+    models = random_models(r)
+    gpu = GPUModel(sms=4, per_sm=(32, 64, 65536, 233472, 512), launch_delay=300, notif_delay=1100)
+    cfg = Config(num_clients=4, theta=r.choice([0, 3, 100]), slack=4, group=r.choice([1, 16]),
+                 ring_capacity=128, streams=8, capacity=tuple(4 * x for x in (32, 64, 65536, 233472, 512)))
+    trace = random_trace(r, 120, 4, len(models), rate_ns=2000)
+    res = _run_policy_with_log(cfg, models, trace, gpu)
+    log = res.policy.log
+    ok, msg, n = sim.replay(cfg, models, log)
+    assert ok, msg
+    assert n == len(res.issues) > 0
+    # a corrupted log (one record's count changed) must be detected as a divergence
+    # or an inconsistency
+    bad = list(log)
+    idx = next(i for i, e in enumerate(bad) if e[0] == sim.EV_ISSUE and i > len(bad) // 2)
+    e = bad[idx]
+    bad[idx] = (e[0], e[1], e[2], e[3], (e[4] + 1) % cfg.streams)
+    ok2, msg2, _ = sim.replay(cfg, models, bad)
+    assert not ok2 and "issue" in msg2
+
+
+def test_S4_theta_inf_and_single_client_are_srpt():
+    r = random.Random(3)
+    models = random_models(r)
+    trace = random_trace(r, 100, 1, len(models))
+    gpu = GPUModel(sms=2)
+    base = Config(num_clients=1, theta=sim.INF_THETA, slack=0,
+                  capacity=tuple(2 * x for x in (32, 64, 65536, 233472, 512)))
+    a = sim.simulate(base, models, trace, gpu)
+    for th in (0, 1, 7):
+        b = sim.simulate(Config(num_clients=1, theta=th, slack=0, capacity=base.capacity), models, trace, gpu)
+        assert [i[1:] for i in a.issues] == [i[1:] for i in b.issues]
+
+
+@pytest.mark.parametrize("N", [2, 3, 4, 8])
+def test_S4_theta_zero_round_robin_windows(N):
+    """theta = 0, all clients always ready: every aligned window of N dispatches
+    serves each client exactly once and deficits return to 0 at window ends."""
+    r = random.Random(N)
+    models = [[Layer(1, (1, 1, 1, 1, 0), 1000 * r.randint(1, 9), 1)] * 3 for _ in range(3)]
+    cfg = Config(num_clients=N, theta=0, slack=10**9, streams=8,
+                 capacity=(10**9,) * 5)
+    pol = sim.Policy(cfg, models)
+    jid = 0
+    for c in range(N):
+        for _ in range(400):
+            pol.arrival(jid, c, r.randrange(3))
+            jid += 1
+    clients = []
+    for w in range(200):
+        for _ in range(N):
+            # one dispatch at a time: issue, then complete it immediately
+            (uid, job, layer, stream), = _issue_one(pol)
+            clients.append(pol.jobs[job].client if job in pol.jobs else None)
+            pol.record(sim.PLACEMENT, uid, 1)
+            pol.record(sim.COMPLETION, uid, 1)
+        assert all(pol.D(c) == 0 for c in range(N))
+    for w in range(200):
+        win = clients[w * N:(w + 1) * N]
+        assert None not in win and sorted(win) == list(range(N))
+
+
+def _issue_one(pol):
+    saved = set(pol.free)
+    pol.free = {min(saved)}
+    out = pol.decide()
+    pol.free = saved - {o[3] for o in out}
+    return out
+
+
+def test_S4_fifo_order():
+    r = random.Random(9)
+    models = random_models(r)
+    trace = random_trace(r, 120, 3, len(models), rate_ns=500)
+    cfg = Config(num_clients=3, policy=sim.FIFO, slack=0, streams=4,
+                 capacity=tuple(2 * x for x in (32, 64, 65536, 233472, 512)))
+    res = _run_policy_with_log(cfg, models, trace, GPUModel(sms=2))
+    assert len(res.finish) == len(trace)
+    # at each issue the chosen job is the oldest ready job: replay the log and check
+    pol = sim.Policy(cfg, models)
+    for ev in res.policy.log:
+        if ev[0] == sim.EV_ARRIVAL:
+            pol.arrival(*ev[1:])
+        elif ev[0] == sim.EV_RECORD:
+            pol.record(*ev[1:])
+        elif ev[0] == sim.EV_ISSUE:
+            rdy = pol.ready()
+            assert ev[2] == min(rdy, key=lambda j: j.seq).id
+            _force_issue(pol, ev[2], ev[4])
+
+
+def _force_issue(pol, job_id, stream):
+    saved = set(pol.free)
+    pol.free = {stream}
+    (out,) = pol.decide()
+    assert out[1] == job_id
+    pol.free = saved - {stream}
+
+
+@pytest.mark.parametrize("N,theta", [(2, 0), (3, 1), (4, 5), (8, 20), (3, 0)])
+def test_S5_deficit_rule_and_bound(N, theta):
+    """(e) when some ready client has D > theta*N the pick is the oldest ready job of
+    the max-D client; (f) a continuously-ready client never exceeds
+    max(D(s), theta*N) + N."""
+    r = random.Random(N * 100 + theta)
+    models = [[Layer(1, (1, 1, 1, 1, 0), 100 * r.randint(1, 50), 1)] * r.randint(1, 5) for _ in range(4)]
+    cfg = Config(num_clients=N, theta=theta, slack=10**9, streams=8, capacity=(10**9,) * 5)
+    pol = sim.Policy(cfg, models)
+    jid = 0
+    for c in range(N):
+        for _ in range(300):
+            pol.arrival(jid, c, r.randrange(4))
+            jid += 1
+    series = {c: [] for c in range(N)}
+    for step in range(280):  # every client stays ready (>= 300 kernels each)
+        rdy = pol.ready()
+        if not rdy:
+            break
+        ds = {c: pol.D(c) for c in {j.client for j in rdy}}
+        cstar = max(sorted(ds), key=lambda c: (ds[c], -c))
+        srpt = min(rdy, key=lambda j: (j.R, j.seq, j.id)).id
+        (uid, job, layer, stream), = _issue_one(pol)
+        picked = pol.jobs[job]
+        if ds[cstar] > theta * N:
+            assert picked.client == cstar
+            assert picked.seq == min(j.seq for j in rdy if j.client == cstar)
+        else:
+            assert picked.id == srpt
+        pol.record(sim.PLACEMENT, uid, 1)
+        pol.record(sim.COMPLETION, uid, 1)
+        for c in range(N):
+            series[c].append(pol.D(c))
+    assert sim.deficit_bound_holds(series, N, theta) == []
+    assert max(max(s) for s in series.values()) <= max(0, theta * N) + N
