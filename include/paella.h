@@ -1,0 +1,233 @@
+/*
+ * paella.h -- C ABI of the B200-native Paella hot path.
+ *
+ * Paella (SOSP '23, "Low-latency Model Serving with Software-defined GPU
+ * Scheduling"): many concurrent batch-1 inference jobs run on instrumented kernels
+ * that report thread-block placement and completion through a host-mapped
+ * notification ring; a software dispatcher (one pinned core per GPU) tracks SM
+ * occupancy and decides kernel issue order with SRPT on remaining-time estimates
+ * bounded by deficit-counter fairness, instead of the GPU's FIFO hardware queues.
+ *
+ * Citations are PAPER.md line numbers ("P123") with the section they fall in.
+ *
+ *   paella_init           -- service start-up; one dispatcher thread per GPU (P1024-1033 §5)
+ *   paella_register_model -- "users add new job definitions to the Paella service"
+ *                            (P1036-1038 §5.1); profiling runs fix T-bar (P1249-1254 §6)
+ *   paella_submit         -- predict(model_name, len, io_ptr, options) -> req_id
+ *                            (P1039-1056 §5.1); range check [io, io+len) (P1060-1061)
+ *   paella_poll_completion-- readResult(options) -> first available completion id,
+ *                            NONBLOCK -> negative EAGAIN (P1144-1155 §5.3)
+ *   paella_shutdown       -- stop admitting, drain, free
+ *
+ * Conventions: every call returns >= 0 on success and -errno on failure ("it may
+ * return the negative code EAGAIN", P1155).  No call takes or returns framework
+ * (torch) types: plain host pointers and sizes only.
+ *
+ * Threading: one thread per client_id at a time (each client's submission and
+ * completion queues are single-producer/single-consumer); different clients may
+ * call concurrently.  The dispatcher threads are internal.
+ *
+ * Ownership: the io buffer passed to paella_submit is LENT to the library from
+ * submit until paella_poll_completion returns that req_id; its layout is
+ * [input | output] (Fig. 8, P992-996: output = io_ptr + INPUT_SIZE).  The input is
+ * fp32 NCHW (1 x C x H x W); the output is fp32 logits.  The ingest kernel reads
+ * the input straight from that (page-locked, device-mapped) client memory and the
+ * last kernel writes the output in place ("pinned output", P1016).  The library
+ * owns device weights, per-job workspaces, rings and streams.
+ */
+#ifndef PAELLA_H_
+#define PAELLA_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define PAELLA_ABI_VERSION 1u
+
+/* policies (P1222-1323 §6; FIFO = the Paella-SS-like ablation of Table 3, P1349) */
+#define PAELLA_POLICY_SRPT_DEFICIT 0u
+#define PAELLA_POLICY_FIFO         1u
+
+/* routing across GPUs */
+#define PAELLA_ROUTE_LEAST_WORK    0u
+#define PAELLA_ROUTE_ROUND_ROBIN   1u
+
+/* device backends */
+#define PAELLA_DEVICE_CUDA 0u   /* real sm_100a GPUs */
+#define PAELLA_DEVICE_FAKE 1u   /* CPU model of a GPU that synthesises ring records
+                                   (tests of dispatcher / router / replay without a GPU) */
+
+/* dtypes of a model's compute path */
+#define PAELLA_DTYPE_BF16 0u    /* bf16 activations, fp32 accumulate, tcgen05 for conv */
+#define PAELLA_DTYPE_FP32 1u    /* fp32 everything, SIMT FFMA, no TF32 */
+
+/* flags */
+#define PAELLA_NONBLOCK 1u      /* submit: -EAGAIN if the ring is full; poll: -EAGAIN if none */
+
+/* maximum sizes */
+#define PAELLA_MAX_GPUS    8u
+#define PAELLA_MAX_CLIENTS 64u
+
+typedef struct paella_s paella_t;  /* opaque, owned by the library */
+
+typedef struct {
+  uint32_t abi_version;          /* = PAELLA_ABI_VERSION */
+  uint32_t device;               /* PAELLA_DEVICE_CUDA | PAELLA_DEVICE_FAKE */
+  uint32_t num_gpus;             /* 1..8; one dispatcher thread per GPU */
+  uint32_t first_gpu;            /* CUDA ordinal of GPU 0 of this instance */
+  uint32_t num_clients;          /* N of the deficit rule (P1290-1296); fixed */
+  uint32_t policy;               /* PAELLA_POLICY_* */
+  int64_t  fairness_threshold;   /* theta, in kernel dispatches; INT64_MAX = pure SRPT */
+  uint32_t slack_blocks;         /* B (P1300-1304); 0 = default (SM count) */
+  uint32_t group_size;           /* G in 1..16 (P1138-1142); 0 = default 16 */
+  uint32_t ring_capacity;        /* notification ring slots, power of two; 0 = 65536 */
+  uint32_t stream_pool;          /* P CUDA streams per GPU (P1090-1098); 0 = 32 */
+  uint32_t route;                /* PAELLA_ROUTE_* */
+  uint32_t submit_slots;         /* per-(client,GPU) submission ring slots, pow2; 0 = 1024 */
+  uint32_t max_jobs_per_model;   /* in-flight job workspaces per model per GPU; 0 = 128 */
+  uint32_t instrument;           /* 1 = instrumented kernels (Paella); 0 = uninstrumented twin */
+  uint32_t naive;                /* 1 = naive baseline: no dispatcher decisions, every kernel
+                                    of a job is launched at admission onto stream
+                                    job % stream_pool (CUDA-MS, Table 3 P1343-1344) */
+  size_t   client_region_bytes;  /* shared io region per client, created here; 0 = 64 MiB */
+  const int32_t* dispatcher_cpus;/* num_gpus core ids to pin the dispatchers to, or NULL */
+  const char* event_log_path;    /* binary event log for replay (printf pattern "%u" = GPU
+                                    index), or NULL */
+  uint32_t fake_sms;             /* FAKE device: SM count (0 = 148) */
+  uint32_t fake_time_scale_ns;   /* FAKE device: virtual ns per poll iteration (0 = 500) */
+} paella_config_t;
+
+/* ---- model description (input to paella_register_model) ---------------- */
+#define PAELLA_OP_INPUT   0u
+#define PAELLA_OP_CONV    1u
+#define PAELLA_OP_MAXPOOL 2u
+#define PAELLA_OP_AVGPOOL 3u   /* count_include_pad = True */
+#define PAELLA_OP_GAP     4u   /* global average pool */
+#define PAELLA_OP_FC      5u
+#define PAELLA_OP_CONCAT  6u   /* channel concat, realised by channel-offset stores */
+
+#define PAELLA_ACT_NONE  0u
+#define PAELLA_ACT_RELU  1u
+#define PAELLA_ACT_RELU6 2u
+
+#define PAELLA_NODE_PROLOGUE 1u  /* relu(pro_scale[c]*x + pro_shift[c]) on the input (DenseNet) */
+#define PAELLA_NODE_CEIL     2u  /* maxpool ceil_mode */
+
+typedef struct {
+  uint32_t op;                 /* PAELLA_OP_* */
+  uint32_t n_inputs;           /* 1, or the number of concat inputs; 0 for INPUT */
+  const int32_t* inputs;       /* node ids (earlier nodes) */
+  int32_t  residual;           /* conv: node id added before the activation, or -1 */
+  uint32_t c, h, w;            /* output shape (C, H, W), batch 1 */
+  uint32_t cout, kh, kw, sh, sw, ph, pw, groups;  /* conv; pools use kh=kw=k, sh=sw=s, ph=pw=p;
+                                                     fc uses cout */
+  uint32_t act;                /* PAELLA_ACT_* */
+  uint32_t flags;              /* PAELLA_NODE_* */
+  const float* weight;         /* conv [cout][cin/groups][kh][kw], fc [cout][cin]; fp32 host
+                                  values (the bf16 path requires bf16-representable values
+                                  and stores them as bf16 exactly) */
+  const float* bias;           /* [cout] or NULL (zero) */
+  const float* pro_scale;      /* [cin] if PROLOGUE */
+  const float* pro_shift;      /* [cin] if PROLOGUE */
+} paella_node_t;
+
+typedef struct {
+  const char* name;            /* unique */
+  uint32_t dtype;              /* PAELLA_DTYPE_* */
+  uint32_t n_nodes;
+  const paella_node_t* nodes;  /* topologically ordered; node 0 is the INPUT; the last node
+                                  produces the logits */
+  uint32_t profile_runs;       /* isolated profiling runs for T-bar (0 = 20) */
+} paella_model_desc_t;
+
+/* ---- calls --------------------------------------------------------------- */
+
+int paella_init(const paella_config_t* cfg, paella_t** out);
+/* -EINVAL bad cfg; -ENODEV fewer than num_gpus sm_100 GPUs (CUDA backend);
+   -ENOMEM.  Creates the client regions, rings, stream pools and starts one
+   dispatcher thread per GPU. */
+
+int paella_register_model(paella_t* p, const paella_model_desc_t* desc, uint32_t* model_id);
+/* Copies the parameters (library owns the device copies on every GPU), builds the
+   kernel chain (one kernel per non-concat node + ingest), queries each kernel's
+   resource attributes (Table 1, P782-802; P814-830), profiles T-bar per kernel
+   with isolated instrumented runs (P1249-1254) and freezes it.
+   -EEXIST name taken; -EINVAL malformed graph or a kernel needing more records
+   than the ring holds; -ENOMEM; -EIO CUDA failure. */
+
+int64_t paella_submit(paella_t* p, uint32_t client_id, uint32_t model_id,
+                      void* io, size_t len, uint32_t flags);
+/* Zero-copy request: [io, io+len) must lie inside client_id's region
+   (paella_client_region), else -EFAULT (P1060-1061).  -EINVAL unknown model or
+   len < input_bytes + output_bytes; -EAGAIN ring full and PAELLA_NONBLOCK;
+   -ESHUTDOWN.  Returns req_id = (client_id << 48) | seq. */
+
+int64_t paella_submit_at(paella_t* p, uint32_t client_id, uint32_t model_id,
+                         void* io, size_t len, uint32_t flags, int64_t t_sched_ns);
+/* paella_submit with the request's scheduled arrival time (CLOCK_MONOTONIC ns),
+   recorded in the event log; paella_submit uses "now". */
+
+int64_t paella_poll_completion(paella_t* p, uint32_t client_id, uint32_t flags, int32_t* status);
+/* Returns the req_id of the FIRST available completion of this client (completion
+   order, not submission order, P1149).  PAELLA_NONBLOCK: -EAGAIN if none (P1155);
+   otherwise spins until one is available.  *status (if non-NULL): 0 ok, -EIO CUDA
+   error on that GPU, -ECANCELED shutdown. */
+
+int paella_shutdown(paella_t* p);
+/* Stop admitting; drain in-flight kernels; requests not yet admitted complete with
+   -ECANCELED; join dispatchers; free everything. */
+
+int paella_client_region(paella_t* p, uint32_t client_id, void** base, size_t* bytes);
+/* The shared io region of a client (page-locked, device-mapped on every GPU). */
+
+/* ---- introspection (tests, bench) ---------------------------------------- */
+
+typedef struct {
+  uint32_t n_kernels;          /* kernels per job (incl. ingest) */
+  size_t   input_bytes, output_bytes;
+  uint64_t weight_bytes;       /* device bytes of parameters */
+  int64_t  total_tbar_ns;      /* sum of frozen T-bar */
+} paella_model_info_t;
+
+int paella_model_info(paella_t* p, uint32_t model_id, paella_model_info_t* info);
+
+typedef struct {
+  uint32_t grid, block, smem, regs, tmem_cols;
+  uint32_t kind;               /* kernel kind id (paella_kernel_name) */
+  int64_t  tbar_ns;            /* frozen profile */
+  uint64_t flops, bytes;       /* algorithmic work per launch */
+} paella_kernel_info_t;
+
+int paella_kernel_info(paella_t* p, uint32_t model_id, uint32_t k, paella_kernel_info_t* info);
+const char* paella_kernel_name(uint32_t kind);
+
+typedef struct {
+  uint64_t admitted, completed, launches, records, torn_retries, decide_calls;
+  uint64_t loop_iters;
+  int64_t  outstanding_work_ns;   /* W_g published for the router */
+} paella_stats_t;
+
+int paella_stats(paella_t* p, uint32_t gpu, paella_stats_t* st);
+
+/* Flush and close the event logs (also done by shutdown). */
+int paella_flush_log(paella_t* p);
+
+/* Run one job of model_id synchronously on GPU `gpu`, outside the dispatcher
+   (no other work must be in flight): every kernel in order on one stream, with
+   instrumentation as configured.  Used by parity tests and the device-only
+   roofline (summed isolated kernel time).  If kernel_ns is non-NULL it receives
+   n_kernels per-kernel device times (CUDA events).  Returns 0 or -errno. */
+int paella_run_isolated(paella_t* p, uint32_t gpu, uint32_t model_id, const void* input,
+                        void* output, int64_t* kernel_ns);
+
+/* Debug: copy node `node`'s activation of the last isolated run to host as fp32
+   NCHW (C*H*W floats).  Returns 0 or -errno. */
+int paella_debug_node(paella_t* p, uint32_t gpu, uint32_t model_id, uint32_t node, float* out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PAELLA_H_ */

@@ -1,0 +1,87 @@
+"""ORACLE (test infrastructure): reader of the dispatcher's binary event log, for
+replay parity (pin S6) and the GPU-log invariants (S5).
+
+Format (DESIGN.md §"Event log"): a sequence of 32-byte little-endian records
+``{u32 type, u32 a, u64 b, u64 c, u64 d}``:
+
+  100 CONFIG    a=N clients, b=policy, c=theta, d=(B << 32) | G
+  100 CONFIG    a=0xFFFFFFFF, b=ring capacity, c=stream pool P
+  101 CAPACITY  a=resource r, b=C_r
+  110 MODEL     a=model, b=#kernels
+  111 LAYER     a=model, b=layer, c=grid, d=T-bar ns
+  112 DEMAND    a=model, b=layer, c=(warps << 32) | regs, d=(smem << 32) | tmem
+    1 ARRIVAL   a=client, b=job, c=model, d=t_sched ns
+    2 RECORD    a=type, b=uid, c=count, d=globaltimer:40 | group:16 | smid:8
+    3 BATCH_END
+    4 ISSUE     a=stream, b=uid, c=job, d=layer
+    5 COMPLETE  b=job, c=t ns
+"""
+import numpy as np
+
+from . import sim
+
+DT = np.dtype([("type", "<u4"), ("a", "<u4"), ("b", "<u8"), ("c", "<u8"), ("d", "<u8")])
+
+
+def read(path):
+    """Returns (Config, models, events, extras) where events are in sim.replay's format."""
+    raw = np.fromfile(path, dtype=DT)
+    cfg_kw = {}
+    cap = [0] * 5
+    layers = {}
+    demands = {}
+    nlayers = {}
+    events = []
+    arrivals = {}
+    records = []
+    issues = []
+    completes = []
+    narrivals = 0
+    for r in raw:
+        t, a, b, c, d = int(r["type"]), int(r["a"]), int(r["b"]), int(r["c"]), int(r["d"])
+        if t == 100:
+            if a == 0xFFFFFFFF:
+                cfg_kw["ring_capacity"] = b
+                cfg_kw["streams"] = c
+            else:
+                cfg_kw["num_clients"] = a
+                cfg_kw["policy"] = b
+                cfg_kw["theta"] = c if c < (1 << 63) else c - (1 << 64)
+                cfg_kw["slack"] = d >> 32
+                cfg_kw["group"] = d & 0xFFFFFFFF
+        elif t == 101:
+            cap[a] = b
+        elif t == 110:
+            nlayers[a] = b
+        elif t == 111:
+            layers[(a, b)] = (c, d)
+        elif t == 112:
+            demands[(a, b)] = (c >> 32, c & 0xFFFFFFFF, d >> 32, d & 0xFFFFFFFF)
+        elif t == 1:
+            events.append((sim.EV_ARRIVAL, b, a, c))
+            arrivals[b] = (a, c, d)        # latest job with this id (ids are recycled)
+            narrivals += 1
+        elif t == 2:
+            events.append((sim.EV_RECORD, a, b, c))
+            # (t, type, uid, n, group) as sim.check_exactly_once expects, + smid
+            records.append((d & ((1 << 40) - 1), a, b, c, (d >> 40) & 0xFFFF, d >> 56))
+        elif t == 3:
+            events.append((sim.EV_BATCH_END,))
+        elif t == 4:
+            events.append((sim.EV_ISSUE, b, c, d, a))
+            issues.append((b, c, d, a, arrivals[c][1]))   # (uid, job, layer, stream, model)
+        elif t == 5:
+            events.append((sim.EV_COMPLETE, b))
+            completes.append((b, c))
+    cfg = sim.Config(capacity=tuple(cap), **cfg_kw)
+    models = []
+    for m in range(len(nlayers)):
+        ms = []
+        for l in range(nlayers[m]):
+            grid, tbar = layers[(m, l)]
+            w, rg, sm, tm = demands[(m, l)]
+            ms.append(sim.Layer(grid, (1, w, rg, sm, tm), tbar))
+        models.append(ms)
+    extras = dict(records=records, issues=issues, completes=completes, arrivals=arrivals,
+                  n_arrivals=narrivals)
+    return cfg, models, events, extras

@@ -460,7 +460,7 @@ def check_exactly_once(records, grids, G):
     ceil(grid/G) records per type, group indices unique and covering [0, ceil)."""
     per = {}
     for rec in records:
-        _, typ, uid, n, grp = rec
+        _, typ, uid, n, grp = rec[:5]
         per.setdefault((uid, typ), []).append((grp, n))
     bad = []
     for uid, g in grids.items():

@@ -1,0 +1,73 @@
+"""Build the in-tree C-ABI library ``libpaella.so`` for sm_100a.
+
+    python -m paella_conf_sosp_ngd023_b200.build
+
+Host C++ (runtime, dispatcher, planner, policy) is compiled with g++; kernels with
+nvcc ``-gencode arch=compute_100a,code=sm_100a -lineinfo``; everything is linked by
+nvcc into one shared library with the static CUDA runtime.  Incremental: objects
+are rebuilt when their source or any header is newer.
+"""
+from __future__ import annotations
+
+import glob
+import os
+import subprocess
+import sys
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+CSRC = os.path.join(HERE, "csrc")
+ROOT = os.path.dirname(HERE)
+OUT = os.path.join(HERE, "libpaella.so")
+BUILD = os.path.join(HERE, "_build")
+CUDA = os.environ.get("CUDA_HOME", "/usr/local/cuda")
+NVCC = os.path.join(CUDA, "bin", "nvcc")
+ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+
+
+def _newer(src, obj, headers):
+    if not os.path.exists(obj):
+        return True
+    t = os.path.getmtime(obj)
+    return os.path.getmtime(src) > t or any(os.path.getmtime(h) > t for h in headers)
+
+
+def _run(cmd, verbose):
+    if verbose:
+        print(" ".join(cmd), file=sys.stderr)
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if r.returncode != 0:
+        sys.stderr.write(r.stdout + r.stderr)
+        raise RuntimeError(f"build failed: {' '.join(cmd[:3])} ...")
+    if verbose and (r.stdout or r.stderr):
+        sys.stderr.write(r.stdout + r.stderr)
+
+
+def build(verbose=False, ptxas_v=False):
+    os.makedirs(BUILD, exist_ok=True)
+    headers = glob.glob(os.path.join(CSRC, "*.h")) + glob.glob(os.path.join(CSRC, "*.cuh")) + \
+        [os.path.join(ROOT, "include", "paella.h")]
+    objs = []
+    inc = ["-I", CSRC, "-I", os.path.join(ROOT, "include"), "-I", os.path.join(CUDA, "include")]
+    for src in sorted(glob.glob(os.path.join(CSRC, "*.cpp"))):
+        obj = os.path.join(BUILD, os.path.basename(src) + ".o")
+        objs.append(obj)
+        if _newer(src, obj, headers):
+            _run(["g++", "-O2", "-g", "-fPIC", "-std=c++17", "-Wall", "-Wno-unused-function",
+                  "-Wno-sign-compare", *inc, "-c", src, "-o", obj], verbose)
+    for src in sorted(glob.glob(os.path.join(CSRC, "*.cu"))):
+        obj = os.path.join(BUILD, os.path.basename(src) + ".o")
+        objs.append(obj)
+        if _newer(src, obj, headers):
+            extra = ["-Xptxas", "-v"] if ptxas_v else []
+            _run([NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", *inc, *extra,
+                  "-c", src, "-o", obj], verbose or ptxas_v)
+    if not os.path.exists(OUT) or any(os.path.getmtime(o) > os.path.getmtime(OUT) for o in objs):
+        tmp = OUT + ".tmp"
+        _run([NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lpthread", "-lrt", "-ldl"], verbose)
+        os.replace(tmp, OUT)
+    return OUT
+
+
+if __name__ == "__main__":
+    build(verbose="-v" in sys.argv, ptxas_v="--ptxas" in sys.argv)
+    print(OUT)

@@ -1,0 +1,109 @@
+// Internal definitions shared by the host runtime and the device kernels of the
+// CUDA path (never by the oracle).
+//
+// Notification record (readings C2-Q3/Q4/Q5 in DESIGN.md).
+// The paper's entry is one 64-bit word {type:8, smId:8, kernId:32} (P1126-1133);
+// we keep those fields and use a 16-byte record written with ONE vector store so
+// it carries the block count, the group index, %globaltimer and a lap tag that
+// detects torn / stale reads without an INVALID reset race:
+//   w0 = type:8 | count:8 | smid:8 | tag:8 | uid:32
+//   w1 = gtimer_ns:40 | group:16 | tag:8          tag = 0x80 | (lap & 0x7f)
+// where lap = ring index >> log2(capacity).  type 0 = INVALID (P1110-1113).
+#pragma once
+#include <stdint.h>
+
+#ifndef __CUDACC__
+#define PAELLA_HD
+#else
+#define PAELLA_HD __host__ __device__
+#endif
+
+namespace paella {
+
+enum : uint32_t { REC_INVALID = 0, REC_PLACEMENT = 1, REC_COMPLETION = 2 };
+
+struct alignas(16) Rec {
+  uint64_t w0, w1;
+};
+
+PAELLA_HD inline uint32_t rec_tag(uint32_t lap) { return 0x80u | (lap & 0x7fu); }
+
+PAELLA_HD inline Rec rec_encode(uint32_t type, uint32_t count, uint32_t smid, uint32_t lap,
+                                uint32_t uid, uint64_t gtimer, uint32_t group) {
+  uint64_t tag = rec_tag(lap);
+  Rec r;
+  r.w0 = (uint64_t)(type & 0xff) | ((uint64_t)(count & 0xff) << 8) | ((uint64_t)(smid & 0xff) << 16) |
+         (tag << 24) | ((uint64_t)uid << 32);
+  r.w1 = (gtimer & ((1ull << 40) - 1)) | ((uint64_t)(group & 0xffff) << 40) | (tag << 56);
+  return r;
+}
+
+struct RecFields {
+  uint32_t type, count, smid, tag0, uid, group, tag1;
+  uint64_t gtimer;
+};
+
+PAELLA_HD inline RecFields rec_decode(uint64_t w0, uint64_t w1) {
+  RecFields f;
+  f.type = (uint32_t)(w0 & 0xff);
+  f.count = (uint32_t)((w0 >> 8) & 0xff);
+  f.smid = (uint32_t)((w0 >> 16) & 0xff);
+  f.tag0 = (uint32_t)((w0 >> 24) & 0xff);
+  f.uid = (uint32_t)(w0 >> 32);
+  f.gtimer = w1 & ((1ull << 40) - 1);
+  f.group = (uint32_t)((w1 >> 40) & 0xffff);
+  f.tag1 = (uint32_t)(w1 >> 56);
+  return f;
+}
+
+// Per-launch instrumentation arguments (Fig. 6's extra parameters notifQ, kernId,
+// P887-895, plus the per-launch counter slot -- reading C2-Q1).
+enum : uint32_t { INSTR_ON = 1u, INSTR_LAST = 2u };
+
+struct InstrArgs {
+  Rec* ring;          // device-visible pointer to the pinned, mapped ring
+  uint32_t* tail;     // device counter: next ring index
+  uint32_t* ctr;      // {start, end} block counters of this launch's slot (uid mod NCTR)
+  uint32_t mask;      // capacity - 1
+  uint32_t log2cap;
+  uint32_t base;      // counter value of the slot before this launch (never reset)
+  uint32_t uid;       // unique launch id (kernel id of the paper)
+  uint32_t group;     // G
+  uint32_t flags;     // INSTR_*
+};
+
+constexpr uint32_t NCTR = 4096;   // counter slots; > max in-flight launches (<= P)
+
+// Kernel-side arguments of one layer.  Activations are NHWC with an explicit
+// channel stride/offset so that a concat is just producers writing into disjoint
+// channel ranges of one buffer (zero-copy concat).
+enum : uint32_t {
+  LF_PROLOGUE = 1u,   // relu(scale*x + shift) on the input (DenseNet pre-activation)
+  LF_CEIL = 2u,       // maxpool ceil mode
+  LF_FINAL = 4u,      // output is the fp32 logits in client memory
+  LF_RESIDUAL = 8u,
+};
+
+struct LayerArgs {
+  const void* in;       // NHWC, element type of the model (ingest: fp32 NCHW client memory)
+  void* out;
+  const void* res;      // residual (same layout as out)
+  const void* w;        // packed weights (layout depends on the kernel)
+  const float* bias;    // [cout] fp32
+  const float* pro_scale;
+  const float* pro_shift;
+  uint32_t in_cs, in_co;    // channel stride / offset of the input buffer
+  uint32_t out_cs, out_co;
+  uint32_t res_cs, res_co;
+  uint32_t cin, h, w_;      // input (channels used, H, W)
+  uint32_t cout, oh, ow;
+  uint32_t kh, kw, sh, sw, ph, pw, groups;
+  uint32_t act, flags;
+  uint32_t kpad;            // packed K (conv) / row pitch (fc), in elements
+  uint32_t tiles_m, tiles_n;// tcgen05 conv: tile grid
+  uint32_t ksplit;          // split-K factor (1 = none)
+  float* ws;                // fp32 split-K workspace
+  uint32_t* ws_ctr;         // split-K arrival counters (one per output tile)
+};
+
+}  // namespace paella

@@ -1,0 +1,1089 @@
+// Paella runtime: C ABI, per-GPU dispatcher threads, notification-ring drain,
+// client channels, router, event log, CUDA and fake backends.
+//
+// Paper map:  dispatcher on a dedicated core (§5 P1024-1033, §7 P1331-1332);
+// client->Paella shm queues polled round-robin (§5.1 P1062-1068); Paella->GPU
+// launches with the original config + instrumentation params + a substituted
+// stream from a pool (§5.2 P1080-1098); notifQ polling and INVALID reset
+// (P1100-1113); flow control by delaying dispatch (P1115-1119); readResult with
+// NONBLOCK / EAGAIN (§5.3 P1144-1155); scheduling policy (§6, policy.cpp).
+#include <errno.h>
+#include <fcntl.h>
+#include <pthread.h>
+#include <sched.h>
+#include <sys/mman.h>
+#include <time.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <array>
+#include <climits>
+#include <cstdarg>
+#include <cstdlib>
+#include <cstring>
+#include <deque>
+#include <queue>
+
+#include <cuda_runtime.h>
+
+#include "engine.h"
+
+namespace paella {
+
+int64_t now_ns() {
+  timespec ts;
+  clock_gettime(CLOCK_MONOTONIC, &ts);
+  return (int64_t)ts.tv_sec * 1000000000ll + ts.tv_nsec;
+}
+
+// ---------------------------------------------------------------------------
+// event log (replay input for oracle/sim.py::replay; format in DESIGN.md)
+// ---------------------------------------------------------------------------
+enum : uint32_t { EV_ARRIVAL = 1, EV_RECORD = 2, EV_BATCH_END = 3, EV_ISSUE = 4, EV_COMPLETE = 5,
+                  EV_CONFIG = 100, EV_CAPACITY = 101, EV_MODEL = 110, EV_LAYER = 111, EV_DEMAND = 112 };
+
+struct LogEv {
+  uint32_t type, a;
+  uint64_t b, c, d;
+};
+static_assert(sizeof(LogEv) == 32, "log event");
+
+static inline void logev(Gpu* g, uint32_t type, uint32_t a, uint64_t b, uint64_t c, uint64_t d) {
+  if (!g->log) return;
+  LogEv e{type, a, b, c, d};
+  fwrite(&e, sizeof e, 1, g->log);
+}
+
+// ---------------------------------------------------------------------------
+// fake backend: a CPU model of a GPU that synthesises ring records
+// ---------------------------------------------------------------------------
+struct FakeBackend : Backend {
+  struct FK {
+    uint32_t uid, grid, stream, placed = 0, sc = 0, ec = 0;
+    int64_t demand[NRES];
+    int64_t dur;
+  };
+  uint32_t sms, cap, log2cap, G, nstreams;
+  int64_t per_sm[NRES] = {32, 64, 65536, 233472, 512};
+  std::vector<std::array<int64_t, NRES>> freeres;
+  std::vector<Rec> ringmem;
+  uint32_t tail = 0;
+  std::vector<uint32_t> ctr;
+  std::vector<std::deque<FK*>> streams;
+  struct End {
+    int64_t t;
+    uint64_t seq;
+    FK* k;
+    uint32_t sm;
+    bool operator>(const End& o) const { return t != o.t ? t > o.t : seq > o.seq; }
+  };
+  std::priority_queue<End, std::vector<End>, std::greater<End>> ends;
+  uint64_t seq = 0;
+  int64_t now = 0, dt;
+  std::vector<void*> evs;
+
+  FakeBackend(uint32_t s, uint32_t c, uint32_t l2, uint32_t g, uint32_t P, int64_t d)
+      : sms(s), cap(c), log2cap(l2), G(g), nstreams(P), dt(d) {}
+  int init() override {
+    freeres.assign(sms, {});
+    for (auto& f : freeres)
+      for (int r = 0; r < NRES; ++r) f[r] = per_sm[r];
+    ringmem.assign(cap, Rec{0, 0});
+    ctr.assign(2 * NCTR, 0);
+    streams.resize(nstreams + 1);
+    return 0;
+  }
+  Rec* ring() override { return ringmem.data(); }
+  uint32_t* tail_dev() override { return &tail; }
+  uint32_t* ctr_dev() override { return ctr.data(); }
+  void* ring_dev() override { return ringmem.data(); }
+  void emit(FK* k, uint32_t type, uint32_t count) {
+    uint32_t r = count % G;
+    if (r == 0 || count == k->grid) {
+      uint32_t idx = tail++;
+      ringmem[idx & (cap - 1)] = rec_encode(type, r == 0 ? G : r, 0, idx >> log2cap, k->uid,
+                                            (uint64_t)now, (count - 1) / G);
+    }
+  }
+  void launch(const KernelInst& k, const LayerArgs&, const InstrArgs& ia, uint32_t stream, uint32_t,
+              bool) override {
+    FK* f = new FK();
+    f->uid = ia.uid;
+    f->grid = k.grid_total();
+    f->stream = stream;
+    for (int r = 0; r < NRES; ++r) f->demand[r] = k.demand[r];
+    f->dur = k.tbar > 0 ? k.tbar : 1000;
+    streams[stream].push_back(f);
+  }
+  void place() {
+    for (auto& q : streams) {
+      if (q.empty()) continue;
+      FK* k = q.front();
+      while (k->placed < k->grid) {
+        int sm = -1;
+        for (uint32_t i = 0; i < sms && sm < 0; ++i) {
+          bool ok = true;
+          for (int r = 0; r < NRES; ++r) ok &= freeres[i][r] >= k->demand[r];
+          if (ok) sm = (int)i;
+        }
+        if (sm < 0) break;
+        for (int r = 0; r < NRES; ++r) freeres[sm][r] -= k->demand[r];
+        k->placed++;
+        k->sc++;
+        emit(k, REC_PLACEMENT, k->sc);
+        ends.push(End{now + k->dur, seq++, k, (uint32_t)sm});
+      }
+    }
+  }
+  void advance() override {
+    now += dt;
+    while (!ends.empty() && ends.top().t <= now) {
+      End e = ends.top();
+      ends.pop();
+      for (int r = 0; r < NRES; ++r) freeres[e.sm][r] += e.k->demand[r];
+      e.k->ec++;
+      emit(e.k, REC_COMPLETION, e.k->ec);
+      if (e.k->ec == e.k->grid) {
+        streams[e.k->stream].pop_front();
+        delete e.k;
+      }
+    }
+    place();
+  }
+  // naive mode is a CUDA-only baseline; on the fake device jobs finish at once
+  void record_event(uint32_t, void** ev) override { *ev = nullptr; }
+  bool event_done(void*) override { return true; }
+  void release_event(void*) override {}
+};
+
+// ---------------------------------------------------------------------------
+// CUDA backend
+// ---------------------------------------------------------------------------
+struct CudaBackend : Backend {
+  int dev;
+  uint32_t cap, nstreams;
+  Rec* ring_h = nullptr;
+  Rec* ring_d = nullptr;
+  uint32_t* tail = nullptr;   // device
+  uint32_t* ctr = nullptr;    // device, 2*NCTR
+  std::vector<cudaStream_t> streams;
+  KernelFn tab[2][2][KIND_COUNT];   // [dtype][instr][kind]
+  int err_ = 0;
+  CudaBackend(int d, uint32_t c, uint32_t P) : dev(d), cap(c), nstreams(P) {}
+  int init() override {
+    if (cudaSetDevice(dev) != cudaSuccess) return -ENODEV;
+    if (cudaHostAlloc((void**)&ring_h, (size_t)cap * sizeof(Rec), cudaHostAllocMapped | cudaHostAllocPortable) !=
+        cudaSuccess)
+      return -ENOMEM;
+    std::memset(ring_h, 0, (size_t)cap * sizeof(Rec));
+    if (cudaHostGetDevicePointer((void**)&ring_d, ring_h, 0) != cudaSuccess) return -EIO;
+    if (cudaMalloc(&tail, 256) != cudaSuccess) return -ENOMEM;
+    if (cudaMalloc(&ctr, 2 * NCTR * sizeof(uint32_t)) != cudaSuccess) return -ENOMEM;
+    cudaMemset(tail, 0, 256);
+    cudaMemset(ctr, 0, 2 * NCTR * sizeof(uint32_t));
+    streams.resize(nstreams);
+    for (auto& s : streams)
+      if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess) return -EIO;
+    KernelFn tc_i[1], tc_p[1];
+    simt_kernel_table(tab[0][1], tab[0][0], tab[1][1], tab[1][0]);
+    tc_kernel_table(tc_i, tc_p);
+    tab[0][1][KIND_CONV_TC] = tc_i[0];
+    tab[0][0][KIND_CONV_TC] = tc_p[0];
+    tab[1][1][KIND_CONV_TC] = nullptr;
+    tab[1][0][KIND_CONV_TC] = nullptr;
+    return cudaDeviceSynchronize() == cudaSuccess ? 0 : -EIO;
+  }
+  ~CudaBackend() override {
+    cudaSetDevice(dev);
+    for (auto& s : streams) cudaStreamDestroy(s);
+    if (ring_h) cudaFreeHost(ring_h);
+    if (tail) cudaFree(tail);
+    if (ctr) cudaFree(ctr);
+  }
+  Rec* ring() override { return ring_h; }
+  uint32_t* tail_dev() override { return tail; }
+  uint32_t* ctr_dev() override { return ctr; }
+  void* ring_dev() override { return ring_d; }
+  KernelFn fn(uint32_t kind, uint32_t dtype, bool instr) { return tab[dtype][instr ? 1 : 0][kind]; }
+  void launch(const KernelInst& k, const LayerArgs& a, const InstrArgs& ia, uint32_t stream, uint32_t dtype,
+              bool instr) override {
+    void* args[3] = {(void*)&a, (void*)&ia, (void*)k_tmap(k)};
+    cudaError_t e = cudaLaunchKernel((const void*)fn(k.kind, dtype, instr), dim3(k.grid[0], k.grid[1], k.grid[2]),
+                                     dim3(k.block), args, k.smem, streams[stream]);
+    if (e != cudaSuccess && !err_) err_ = (int)e;
+  }
+  // the tensor map of a tcgen05 conv is stored right after its KernelInst's proto
+  // in per-GPU storage; set by the engine before launch through this hook
+  const void* cur_tmap = nullptr;
+  const void* k_tmap(const KernelInst&) { return cur_tmap; }
+  int error() override {
+    if (err_) return err_;
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) err_ = (int)e;
+    return err_;
+  }
+  void record_event(uint32_t stream, void** ev) override {
+    cudaEvent_t e;
+    cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+    cudaEventRecord(e, streams[stream]);
+    *ev = e;
+  }
+  bool event_done(void* ev) override { return cudaEventQuery((cudaEvent_t)ev) == cudaSuccess; }
+  void release_event(void* ev) override { cudaEventDestroy((cudaEvent_t)ev); }
+  void sync() override { cudaDeviceSynchronize(); }
+};
+
+// per-(model, gpu) tensor maps for tcgen05 weights (defined in kernels_tc.cu)
+int make_weight_tmap(void* weights, uint32_t rows, uint32_t kpad, void* out128);
+
+
+// ---------------------------------------------------------------------------
+// helpers
+// ---------------------------------------------------------------------------
+static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last) {
+  InstrArgs ia;
+  ia.ring = (Rec*)g->be->ring_dev();
+  ia.tail = g->be->tail_dev();
+  uint32_t slot = uid % NCTR;
+  ia.ctr = g->be->ctr_dev() + 2 * slot;
+  ia.mask = g->cap - 1;
+  ia.log2cap = g->log2cap;
+  ia.base = g->ctr_base[slot];
+  g->ctr_base[slot] += grid;
+  ia.uid = uid;
+  ia.group = g->P->cfg.group_size;
+  ia.flags = INSTR_ON | (last ? INSTR_LAST : 0);
+  return ia;
+}
+
+static void do_launch(Gpu* g, Model* m, uint32_t slot, uint32_t layer, uint32_t uid, uint32_t stream, bool instr) {
+  const KernelInst& k = m->kernels[layer];
+  InstrArgs ia = make_instr(g, uid, k.grid_total(), layer + 1 == m->kernels.size());
+  if (g->P->cfg.device == PAELLA_DEVICE_CUDA) {
+    auto* cb = static_cast<CudaBackend*>(g->be.get());
+    cb->cur_tmap = (k.kind == KIND_CONV_TC) ? m->gpu[g->index].tmaps[layer].b : nullptr;
+  }
+  g->be->launch(k, m->gpu[g->index].args[slot][layer], ia, stream, m->dtype, instr);
+}
+
+static void push_completion(Gpu* g, const JobRec& j, int32_t status) {
+  CompleteSlot cs{};
+  cs.req_id = j.req_id;
+  cs.status = status;
+  cs.gpu = g->index;
+  cs.t_done_ns = now_ns();
+  while (!g->done[j.client]->push(cs)) {
+    // completion ring full: the client is not polling; spin (bounded by client)
+    if (g->stop.load(std::memory_order_relaxed)) break;
+  }
+}
+
+static void finish_job(Gpu* g, uint32_t jid, int32_t status) {
+  JobRec& j = g->jobs[jid];
+  Model* m = g->P->models[j.model].get();
+  push_completion(g, j, status);
+  m->gpu[g->index].free_slots.push_back(j.slot);
+  j.live = false;
+  g->free_job_ids.push_back(jid);
+  g->stats.completed++;
+  logev(g, EV_COMPLETE, 0, jid, (uint64_t)now_ns(), 0);
+}
+
+// admit one submission; false = no workspace (leave it in the ring)
+static bool admit(Gpu* g, uint32_t client, const SubmitSlot& s) {
+  Paella* P = g->P;
+  Model* m = P->models[s.model_id].get();
+  ModelGpu& mg = m->gpu[g->index];
+  if (mg.free_slots.empty()) return false;
+  uint32_t slot = mg.free_slots.back();
+  mg.free_slots.pop_back();
+  uint32_t jid;
+  if (!g->free_job_ids.empty()) {
+    jid = g->free_job_ids.back();
+    g->free_job_ids.pop_back();
+  } else {
+    jid = g->next_job++;
+    g->jobs.resize(g->next_job);
+  }
+  // The policy requires job ids in admission order only for tie-breaks via seq;
+  // ids themselves may be reused once a job is done.
+  JobRec& j = g->jobs[jid];
+  j.req_id = s.req_id;
+  j.client = client;
+  j.model = s.model_id;
+  j.slot = slot;
+  j.io = P->region[client] + s.io_off;
+  j.t_sched = s.t_sched_ns;
+  j.live = true;
+  auto& args = mg.args[slot];
+  args.front().in = j.io;                           // ingest reads client memory
+  args.back().out = j.io + m->input_bytes;           // last kernel writes the logits in place
+  g->stats.admitted++;
+  logev(g, EV_ARRIVAL, client, jid, s.model_id, (uint64_t)s.t_sched_ns);
+  if (P->cfg.naive) {
+    // CUDA-MS baseline: every kernel of the job enters stream jid % P now
+    uint32_t st = jid % P->cfg.stream_pool;
+    j.stream = st;
+    for (uint32_t l = 0; l < m->kernels.size(); ++l) {
+      do_launch(g, m, slot, l, 0, st, false);
+      g->stats.launches++;
+    }
+    g->be->record_event(st, &j.event);
+    g->naive_inflight.push_back(jid);
+  } else {
+    g->policy->arrival(jid, client, s.model_id);
+  }
+  return true;
+}
+
+static uint32_t drain_ring(Gpu* g) {
+  Rec* ring = g->be->ring();
+  uint32_t n = 0;
+  for (;;) {
+    Rec* r = ring + (g->head & (g->cap - 1));
+    uint32_t lap = (uint32_t)(g->head >> g->log2cap);
+    uint32_t want = rec_tag(lap);
+    volatile uint64_t* vr = reinterpret_cast<volatile uint64_t*>(r);
+    uint64_t w0 = vr[0];
+    if ((w0 & 0xff) == REC_INVALID || ((w0 >> 24) & 0xff) != want) break;
+    uint64_t w1 = vr[1];
+    if ((w1 >> 56) != want) {   // torn: the second half has not landed yet
+      g->stats.torn_retries++;
+      break;
+    }
+    RecFields f = rec_decode(w0, w1);
+    vr[0] = 0;                  // INVALID (P1110-1113)
+    vr[1] = 0;
+    g->head++;
+    n++;
+    g->stats.records++;
+    logev(g, EV_RECORD, f.type, f.uid, f.count, f.gtimer | ((uint64_t)f.group << 40) | ((uint64_t)f.smid << 56));
+    int64_t done = -1;
+    g->policy->record(f.type, f.uid, f.count, &done);
+    if (done >= 0) finish_job(g, (uint32_t)done, 0);
+  }
+  return n;
+}
+
+static void decide_and_launch(Gpu* g) {
+  g->issues.clear();
+  g->policy->decide(&g->issues);
+  g->stats.decide_calls++;
+  for (const Issue& is : g->issues) {
+    JobRec& j = g->jobs[is.job];
+    Model* m = g->P->models[j.model].get();
+    logev(g, EV_ISSUE, is.stream, is.uid, is.job, is.layer);
+    do_launch(g, m, j.slot, is.layer, is.uid, is.stream, g->P->cfg.instrument != 0);
+    g->stats.launches++;
+  }
+}
+
+static void dispatcher_main(Gpu* g) {
+  Paella* P = g->P;
+  if (P->cfg.device == PAELLA_DEVICE_CUDA) cudaSetDevice(g->device);
+  if (P->cfg.dispatcher_cpus) {
+    cpu_set_t cs;
+    CPU_ZERO(&cs);
+    CPU_SET(P->cfg.dispatcher_cpus[g->index], &cs);
+    pthread_setaffinity_np(pthread_self(), sizeof cs, &cs);
+  }
+  const uint32_t N = P->cfg.num_clients;
+  for (;;) {
+    g->stats.loop_iters++;
+    g->be->advance();
+    uint32_t nev = 0;
+    // 1. client rings, round-robin, starting after the last client served (C2-Q16)
+    bool stopping = g->stop.load(std::memory_order_acquire);
+    if (!stopping) {
+      uint32_t nm = P->nmodels.load(std::memory_order_acquire);
+      for (uint32_t k = 0; k < N; ++k) {
+        uint32_t c = (g->rr_start + k) % N;
+        SpscRing<SubmitSlot>* q = g->sub[c];
+        const SubmitSlot* s;
+        bool served = false;
+        while ((s = q->peek()) != nullptr) {
+          if (s->model_id >= nm) {   // cannot happen through the API; drop defensively
+            q->pop();
+            continue;
+          }
+          if (!admit(g, c, *s)) break;
+          q->pop();
+          nev++;
+          served = true;
+        }
+        if (served) g->rr_start = (c + 1) % N;
+      }
+      g->admitted_pub.store(g->stats.admitted, std::memory_order_release);
+    }
+    if (P->cfg.naive) {
+      for (size_t i = 0; i < g->naive_inflight.size();) {
+        uint32_t jid = g->naive_inflight[i];
+        if (g->be->event_done(g->jobs[jid].event)) {
+          g->be->release_event(g->jobs[jid].event);
+          finish_job(g, jid, 0);
+          g->naive_inflight[i] = g->naive_inflight.back();
+          g->naive_inflight.pop_back();
+        } else {
+          ++i;
+        }
+      }
+      if (stopping && g->naive_inflight.empty()) break;
+      continue;
+    }
+    // 2. notification ring
+    nev += drain_ring(g);
+    // 3. decide (the batch boundary is logged for replay, C2-Q17)
+    if (nev) {
+      logev(g, EV_BATCH_END, 0, 0, 0, 0);
+      decide_and_launch(g);
+      g->work_published.store(g->policy->outstanding_work(), std::memory_order_release);
+    }
+    int e = g->be->error();
+    if (e) {
+      g->err.store(-EIO);
+      // fail every live job of this GPU with -EIO
+      for (uint32_t jid = 0; jid < g->jobs.size(); ++jid)
+        if (g->jobs[jid].live) finish_job(g, jid, -EIO);
+      break;
+    }
+    if (stopping && g->policy->live_jobs() == 0) break;
+  }
+}
+
+// ---------------------------------------------------------------------------
+// shared memory helpers
+// ---------------------------------------------------------------------------
+static void* shm_alloc(Paella* P, size_t bytes) {
+  void* p = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_SHARED | MAP_ANONYMOUS, -1, 0);
+  if (p == MAP_FAILED) return nullptr;
+  P->shm_maps.push_back(p);
+  P->shm_sizes.push_back(bytes);
+  return p;
+}
+
+static uint32_t ilog2(uint32_t x) {
+  uint32_t l = 0;
+  while ((1u << l) < x) ++l;
+  return l;
+}
+
+static int setup_model_gpu(Paella* P, Model* m, Gpu* g);
+
+}  // namespace paella
+
+using namespace paella;
+
+// ===========================================================================
+// C ABI
+// ===========================================================================
+extern "C" {
+
+int paella_init(const paella_config_t* cfg_in, paella_t** out) {
+  if (!cfg_in || !out || cfg_in->abi_version != PAELLA_ABI_VERSION) return -EINVAL;
+  paella_config_t cfg = *cfg_in;
+  if (cfg.num_gpus < 1 || cfg.num_gpus > PAELLA_MAX_GPUS) return -EINVAL;
+  if (cfg.num_clients < 1 || cfg.num_clients > PAELLA_MAX_CLIENTS) return -EINVAL;
+  if (cfg.policy > PAELLA_POLICY_FIFO || cfg.device > PAELLA_DEVICE_FAKE) return -EINVAL;
+  if (cfg.group_size == 0) cfg.group_size = 16;
+  if (cfg.group_size > 16) return -EINVAL;
+  if (cfg.ring_capacity == 0) cfg.ring_capacity = 65536;
+  if (cfg.ring_capacity & (cfg.ring_capacity - 1)) return -EINVAL;
+  if (cfg.stream_pool == 0) cfg.stream_pool = 32;
+  if (cfg.stream_pool > 1024) return -EINVAL;
+  if (cfg.submit_slots == 0) cfg.submit_slots = 1024;
+  if (cfg.submit_slots & (cfg.submit_slots - 1)) return -EINVAL;
+  if (cfg.max_jobs_per_model == 0) cfg.max_jobs_per_model = 128;
+  if (cfg.client_region_bytes == 0) cfg.client_region_bytes = 64ull << 20;
+  if (cfg.fake_time_scale_ns == 0) cfg.fake_time_scale_ns = 500;
+  if (cfg.fairness_threshold < 0) return -EINVAL;
+
+  auto P = std::make_unique<Paella>();
+  P->cfg = cfg;
+  if (cfg.device == PAELLA_DEVICE_CUDA) {
+    int n = 0;
+    if (cudaGetDeviceCount(&n) != cudaSuccess || n < (int)(cfg.first_gpu + cfg.num_gpus)) return -ENODEV;
+    cudaDeviceProp prop;
+    cudaGetDeviceProperties(&prop, cfg.first_gpu);
+    if (prop.major != 10) return -ENODEV;
+    P->sms = prop.multiProcessorCount;
+    int smem_sm = prop.sharedMemPerMultiprocessor;
+    P->capacity[0] = (int64_t)P->sms * prop.maxBlocksPerMultiProcessor;
+    P->capacity[1] = (int64_t)P->sms * (prop.maxThreadsPerMultiProcessor / 32);
+    P->capacity[2] = (int64_t)P->sms * prop.regsPerMultiprocessor;
+    P->capacity[3] = (int64_t)P->sms * smem_sm;
+    P->capacity[4] = (int64_t)P->sms * 512;
+  } else {
+    P->sms = cfg.fake_sms ? cfg.fake_sms : 148;
+    int64_t per[NRES] = {32, 64, 65536, 233472, 512};
+    for (int r = 0; r < NRES; ++r) P->capacity[r] = (int64_t)P->sms * per[r];
+  }
+  if (cfg.slack_blocks == 0) P->cfg.slack_blocks = P->sms;
+  P->models.resize(256);
+
+  // client regions (shared, page-locked and mapped into every GPU)
+  P->region_bytes = cfg.client_region_bytes;
+  for (uint32_t c = 0; c < cfg.num_clients; ++c) {
+    void* r = shm_alloc(P.get(), P->region_bytes);
+    if (!r) return -ENOMEM;
+    if (cfg.device == PAELLA_DEVICE_CUDA) {
+      cudaSetDevice(cfg.first_gpu);
+      if (cudaHostRegister(r, P->region_bytes, cudaHostRegisterPortable | cudaHostRegisterMapped) != cudaSuccess)
+        return -ENOMEM;
+    }
+    P->region.push_back((uint8_t*)r);
+    P->client_seq.push_back(new std::atomic<uint64_t>(0));
+  }
+  P->rr_next.assign(cfg.num_clients, 0);
+  P->poll_rr.assign(cfg.num_clients, 0);
+
+  for (uint32_t gi = 0; gi < cfg.num_gpus; ++gi) {
+    auto g = std::make_unique<Gpu>();
+    g->P = P.get();
+    g->index = gi;
+    g->device = (int)(cfg.first_gpu + gi);
+    g->cap = cfg.ring_capacity;
+    g->log2cap = ilog2(cfg.ring_capacity);
+    g->ctr_base.assign(NCTR, 0);
+    if (cfg.device == PAELLA_DEVICE_CUDA)
+      g->be.reset(new CudaBackend(g->device, g->cap, cfg.stream_pool));
+    else
+      g->be.reset(new FakeBackend(P->sms, g->cap, g->log2cap, cfg.group_size, cfg.stream_pool,
+                                  cfg.fake_time_scale_ns));
+    int rc = g->be->init();
+    if (rc) return rc;
+    Policy::Cfg pc;
+    pc.num_clients = cfg.num_clients;
+    pc.policy = cfg.policy;
+    pc.theta = cfg.fairness_threshold;
+    pc.slack = P->cfg.slack_blocks;
+    pc.group = cfg.group_size;
+    pc.ring_capacity = cfg.ring_capacity;
+    pc.streams = cfg.stream_pool;
+    for (int r = 0; r < NRES; ++r) pc.capacity[r] = P->capacity[r];
+    g->policy.reset(new Policy(pc));
+    for (uint32_t c = 0; c < cfg.num_clients; ++c) {
+      auto* s = (SpscRing<SubmitSlot>*)shm_alloc(P.get(), SpscRing<SubmitSlot>::bytes(cfg.submit_slots));
+      auto* d = (SpscRing<CompleteSlot>*)shm_alloc(P.get(), SpscRing<CompleteSlot>::bytes(cfg.submit_slots));
+      if (!s || !d) return -ENOMEM;
+      s->init(cfg.submit_slots);
+      d->init(cfg.submit_slots);
+      g->sub.push_back(s);
+      g->done.push_back(d);
+    }
+    if (cfg.event_log_path) {
+      char path[4096];
+      snprintf(path, sizeof path, cfg.event_log_path, gi);
+      g->log = fopen(path, "wb");
+      if (!g->log) return -EINVAL;
+      setvbuf(g->log, nullptr, _IOFBF, 1 << 20);
+      logev(g.get(), EV_CONFIG, cfg.num_clients, cfg.policy, (uint64_t)cfg.fairness_threshold,
+            ((uint64_t)P->cfg.slack_blocks << 32) | cfg.group_size);
+      logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFFu, cfg.ring_capacity, cfg.stream_pool, 0);
+      for (int r = 0; r < NRES; ++r) logev(g.get(), EV_CAPACITY, (uint32_t)r, (uint64_t)P->capacity[r], 0, 0);
+    }
+    P->gpus.push_back(std::move(g));
+  }
+  for (auto& g : P->gpus) g->thread = std::thread(dispatcher_main, g.get());
+  *out = (paella_t*)P.release();
+  return 0;
+}
+
+int paella_client_region(paella_t* p, uint32_t client_id, void** base, size_t* bytes) {
+  Paella* P = (Paella*)p;
+  if (!P || client_id >= P->cfg.num_clients) return -EINVAL;
+  if (base) *base = P->region[client_id];
+  if (bytes) *bytes = P->region_bytes;
+  return 0;
+}
+
+int paella_register_model(paella_t* p, const paella_model_desc_t* desc, uint32_t* model_id) {
+  Paella* P = (Paella*)p;
+  if (!P || !desc || !desc->name) return -EINVAL;
+  std::lock_guard<std::mutex> lk(P->reg_mu);
+  uint32_t nm = P->nmodels.load();
+  for (uint32_t i = 0; i < nm; ++i)
+    if (P->models[i]->name == desc->name) return -EEXIST;
+  if (nm >= P->models.size()) return -ENOMEM;
+  auto m = std::make_unique<Model>();
+  m->id = nm;
+  int rc = plan_model(P, desc, m.get());
+  if (rc) return rc;
+  for (auto& k : m->kernels) {
+    if (2ull * ((k.grid_total() + P->cfg.group_size - 1) / P->cfg.group_size) > P->cfg.ring_capacity)
+      return -EINVAL;
+  }
+  m->gpu.resize(P->gpus.size());
+  for (auto& g : P->gpus) {
+    rc = setup_model_gpu(P, m.get(), g.get());
+    if (rc) return rc;
+  }
+  // policy tables + log (identical T-bar on every GPU: profiled on GPU 0)
+  std::vector<PolicyLayer> layers;
+  m->total_tbar = 0;
+  for (auto& k : m->kernels) {
+    PolicyLayer L;
+    L.grid = k.grid_total();
+    for (int r = 0; r < NRES; ++r) L.demand[r] = k.demand[r];
+    L.tbar = k.tbar;
+    m->total_tbar += k.tbar;
+    layers.push_back(L);
+  }
+  Model* mp = m.get();
+  P->models[nm] = std::move(m);
+  for (auto& g : P->gpus) {
+    // the dispatcher thread only reads a model once nmodels covers it; the policy
+    // table is written before publication
+    g->policy->add_model(nm, layers);
+    logev(g.get(), EV_MODEL, nm, layers.size(), 0, 0);
+    for (uint32_t l = 0; l < layers.size(); ++l) {
+      logev(g.get(), EV_LAYER, nm, l, layers[l].grid, (uint64_t)layers[l].tbar);
+      logev(g.get(), EV_DEMAND, nm, l, ((uint64_t)layers[l].demand[1] << 32) | (uint64_t)layers[l].demand[2],
+            ((uint64_t)layers[l].demand[3] << 32) | (uint64_t)layers[l].demand[4]);
+    }
+    if (g->log) fflush(g->log);
+  }
+  (void)mp;
+  P->nmodels.store(nm + 1, std::memory_order_release);
+  if (model_id) *model_id = nm;
+  return 0;
+}
+
+static int64_t submit_impl(Paella* P, uint32_t client_id, uint32_t model_id, void* io, size_t len, uint32_t flags,
+                           int64_t t_sched) {
+  if (!P) return -EINVAL;
+  if (P->shutting.load()) return -ESHUTDOWN;
+  if (client_id >= P->cfg.num_clients) return -EINVAL;
+  if (model_id >= P->nmodels.load(std::memory_order_acquire)) return -EINVAL;
+  Model* m = P->models[model_id].get();
+  uint8_t* base = P->region[client_id];
+  uint8_t* b = (uint8_t*)io;
+  if (b < base || b + len > base + P->region_bytes || b + len < b) return -EFAULT;
+  if (len < m->input_bytes + m->output_bytes) return -EINVAL;
+  if (((uintptr_t)io & 15) != 0) return -EINVAL;
+  // route: least outstanding work, ties to the lowest index
+  uint32_t gsel = 0;
+  uint32_t ng = (uint32_t)P->gpus.size();
+  if (ng > 1) {
+    if (P->cfg.route == PAELLA_ROUTE_ROUND_ROBIN) {
+      gsel = P->rr_next[client_id]++ % ng;
+    } else {
+      int64_t best = INT64_MAX;
+      for (uint32_t g = 0; g < ng; ++g) {
+        Gpu* G = P->gpus[g].get();
+        int64_t pending = (int64_t)(G->submitted.load(std::memory_order_relaxed) -
+                                    G->admitted_pub.load(std::memory_order_acquire));
+        int64_t w = G->work_published.load(std::memory_order_acquire) + pending * m->total_tbar;
+        if (w < best) {
+          best = w;
+          gsel = g;
+        }
+      }
+    }
+  }
+  Gpu* G = P->gpus[gsel].get();
+  SubmitSlot s{};
+  uint64_t seq = P->client_seq[client_id]->fetch_add(1);
+  s.req_id = ((uint64_t)client_id << 48) | (seq & ((1ull << 48) - 1));
+  s.model_id = model_id;
+  s.flags = flags;
+  s.io_off = (uint64_t)(b - base);
+  s.len = len;
+  s.t_sched_ns = t_sched;
+  for (;;) {
+    if (G->sub[client_id]->push(s)) break;
+    if (flags & PAELLA_NONBLOCK) return -EAGAIN;
+    if (P->shutting.load()) return -ESHUTDOWN;
+  }
+  G->submitted.fetch_add(1, std::memory_order_relaxed);
+  return (int64_t)s.req_id;
+}
+
+int64_t paella_submit(paella_t* p, uint32_t client_id, uint32_t model_id, void* io, size_t len, uint32_t flags) {
+  return submit_impl((Paella*)p, client_id, model_id, io, len, flags, now_ns());
+}
+
+int64_t paella_submit_at(paella_t* p, uint32_t client_id, uint32_t model_id, void* io, size_t len, uint32_t flags,
+                         int64_t t_sched_ns) {
+  return submit_impl((Paella*)p, client_id, model_id, io, len, flags, t_sched_ns);
+}
+
+int64_t paella_poll_completion(paella_t* p, uint32_t client_id, uint32_t flags, int32_t* status) {
+  Paella* P = (Paella*)p;
+  if (!P || client_id >= P->cfg.num_clients) return -EINVAL;
+  uint32_t ng = (uint32_t)P->gpus.size();
+  for (;;) {
+    for (uint32_t k = 0; k < ng; ++k) {
+      uint32_t g = (P->poll_rr[client_id] + k) % ng;
+      SpscRing<CompleteSlot>* q = P->gpus[g]->done[client_id];
+      const CompleteSlot* c = q->peek();
+      if (c) {
+        int64_t id = (int64_t)c->req_id;
+        if (status) *status = c->status;
+        q->pop();
+        P->poll_rr[client_id] = (g + 1) % ng;
+        return id;
+      }
+    }
+    if (flags & PAELLA_NONBLOCK) return -EAGAIN;
+    bool alive = false;
+    for (auto& g : P->gpus) alive |= g->thread.joinable() && !g->stop.load();
+    if (!alive) return -ESHUTDOWN;
+  }
+}
+
+int paella_shutdown(paella_t* p) {
+  Paella* P = (Paella*)p;
+  if (!P) return -EINVAL;
+  P->shutting.store(true);
+  for (auto& g : P->gpus) g->stop.store(true, std::memory_order_release);
+  for (auto& g : P->gpus)
+    if (g->thread.joinable()) g->thread.join();
+  // requests never admitted complete with -ECANCELED
+  for (auto& g : P->gpus) {
+    for (uint32_t c = 0; c < P->cfg.num_clients; ++c) {
+      const SubmitSlot* s;
+      while ((s = g->sub[c]->peek()) != nullptr) {
+        CompleteSlot cs{};
+        cs.req_id = s->req_id;
+        cs.status = -ECANCELED;
+        g->done[c]->push(cs);
+        g->sub[c]->pop();
+      }
+    }
+    if (g->log) {
+      fclose(g->log);
+      g->log = nullptr;
+    }
+  }
+  for (uint32_t i = 0; i < P->nmodels.load(); ++i) {
+    Model* m = P->models[i].get();
+    for (size_t gi = 0; gi < P->gpus.size(); ++gi) {
+      if (P->cfg.device == PAELLA_DEVICE_CUDA) {
+        cudaSetDevice(P->gpus[gi]->device);
+        cudaFree(m->gpu[gi].weights);
+        cudaFree(m->gpu[gi].workspace);
+        if (m->gpu[gi].splitk_ws) cudaFree(m->gpu[gi].splitk_ws);
+        if (m->gpu[gi].splitk_ctr) cudaFree(m->gpu[gi].splitk_ctr);
+      } else {
+        free(m->gpu[gi].weights);
+        free(m->gpu[gi].workspace);
+      }
+    }
+  }
+  if (P->cfg.device == PAELLA_DEVICE_CUDA)
+    for (auto* r : P->region) cudaHostUnregister(r);
+  P->gpus.clear();
+  for (size_t i = 0; i < P->shm_maps.size(); ++i) munmap(P->shm_maps[i], P->shm_sizes[i]);
+  for (auto* a : P->client_seq) delete a;
+  delete P;
+  return 0;
+}
+
+int paella_flush_log(paella_t* p) {
+  Paella* P = (Paella*)p;
+  if (!P) return -EINVAL;
+  for (auto& g : P->gpus)
+    if (g->log) fflush(g->log);
+  return 0;
+}
+
+int paella_model_info(paella_t* p, uint32_t model_id, paella_model_info_t* info) {
+  Paella* P = (Paella*)p;
+  if (!P || !info || model_id >= P->nmodels.load()) return -EINVAL;
+  Model* m = P->models[model_id].get();
+  info->n_kernels = (uint32_t)m->kernels.size();
+  info->input_bytes = m->input_bytes;
+  info->output_bytes = m->output_bytes;
+  info->weight_bytes = m->blob.size();
+  info->total_tbar_ns = m->total_tbar;
+  return 0;
+}
+
+int paella_kernel_info(paella_t* p, uint32_t model_id, uint32_t k, paella_kernel_info_t* info) {
+  Paella* P = (Paella*)p;
+  if (!P || !info || model_id >= P->nmodels.load()) return -EINVAL;
+  Model* m = P->models[model_id].get();
+  if (k >= m->kernels.size()) return -EINVAL;
+  const KernelInst& ki = m->kernels[k];
+  info->grid = ki.grid_total();
+  info->block = ki.block;
+  info->smem = ki.smem + ki.static_smem;
+  info->regs = ki.regs;
+  info->tmem_cols = ki.tmem_cols;
+  info->kind = ki.kind;
+  info->tbar_ns = ki.tbar;
+  info->flops = ki.flops;
+  info->bytes = ki.bytes;
+  return 0;
+}
+
+const char* paella_kernel_name(uint32_t kind) {
+  static const char* names[] = {"ingest", "conv_simt", "conv_tcgen05", "dwconv", "maxpool",
+                                "avgpool", "gap", "fc_gemv", "empty"};
+  return kind < KIND_COUNT ? names[kind] : "?";
+}
+
+int paella_stats(paella_t* p, uint32_t gpu, paella_stats_t* st) {
+  Paella* P = (Paella*)p;
+  if (!P || !st || gpu >= P->gpus.size()) return -EINVAL;
+  *st = P->gpus[gpu]->stats;   // racy snapshot of counters, fine for reporting
+  st->outstanding_work_ns = P->gpus[gpu]->work_published.load();
+  return 0;
+}
+
+}  // extern "C"
+
+// ===========================================================================
+// per-GPU model setup, isolated runs, profiling
+// ===========================================================================
+namespace paella {
+
+static int ensure_iso(Gpu* g) {
+  if (g->prof_ring_h) return 0;
+  const uint32_t cap = 1u << 16;
+  if (cudaSetDevice(g->device) != cudaSuccess) return -EIO;
+  if (cudaHostAlloc((void**)&g->prof_ring_h, cap * sizeof(Rec), cudaHostAllocMapped | cudaHostAllocPortable))
+    return -ENOMEM;
+  std::memset(g->prof_ring_h, 0, cap * sizeof(Rec));
+  cudaHostGetDevicePointer(&g->prof_ring_d, g->prof_ring_h, 0);
+  if (cudaMalloc(&g->prof_tail, 256) || cudaMalloc(&g->prof_ctr, 2 * NCTR * sizeof(uint32_t))) return -ENOMEM;
+  cudaMemset(g->prof_tail, 0, 256);
+  cudaMemset(g->prof_ctr, 0, 2 * NCTR * sizeof(uint32_t));
+  g->prof_base.assign(NCTR, 0);
+  cudaStream_t s;
+  cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
+  g->prof_stream = s;
+  g->stage_bytes = 16u << 20;
+  if (cudaHostAlloc(&g->stage_in, g->stage_bytes, cudaHostAllocMapped | cudaHostAllocPortable)) return -ENOMEM;
+  return cudaDeviceSynchronize() == cudaSuccess ? 0 : -EIO;
+}
+
+// launch kernel `l` of model m from the isolated slot on the profiling stream
+static void iso_launch(Gpu* g, Model* m, uint32_t l, bool instr) {
+  const KernelInst& k = m->kernels[l];
+  InstrArgs ia;
+  ia.ring = (Rec*)g->prof_ring_d;
+  ia.tail = g->prof_tail;
+  uint32_t uid = g->prof_uid++;
+  uint32_t slot = uid % NCTR;
+  ia.ctr = g->prof_ctr + 2 * slot;
+  ia.mask = (1u << 16) - 1;
+  ia.log2cap = 16;
+  ia.base = g->prof_base[slot];
+  g->prof_base[slot] += k.grid_total();
+  ia.uid = uid;
+  ia.group = g->P->cfg.group_size;
+  ia.flags = INSTR_ON | (l + 1 == m->kernels.size() ? INSTR_LAST : 0);
+  uint32_t iso_slot = (uint32_t)m->gpu[g->index].args.size() - 1;
+  auto* cb = static_cast<CudaBackend*>(g->be.get());
+  const void* tm = (k.kind == KIND_CONV_TC) ? m->gpu[g->index].tmaps[l].b : nullptr;
+  void* args[3] = {(void*)&m->gpu[g->index].args[iso_slot][l], (void*)&ia, (void*)tm};
+  cudaLaunchKernel((const void*)cb->fn(k.kind, m->dtype, instr), dim3(k.grid[0], k.grid[1], k.grid[2]),
+                   dim3(k.block), args, k.smem, (cudaStream_t)g->prof_stream);
+}
+
+static int iso_run(Gpu* g, Model* m, const void* input, void* output, int64_t* kernel_ns, bool instr) {
+  int rc = ensure_iso(g);
+  if (rc) return rc;
+  cudaSetDevice(g->device);
+  uint8_t* st = (uint8_t*)g->stage_in;
+  if (m->input_bytes + m->output_bytes > g->stage_bytes) return -ENOMEM;
+  if (input) std::memcpy(st, input, m->input_bytes);
+  std::memset(st + m->input_bytes, 0, m->output_bytes);
+  ModelGpu& mg = m->gpu[g->index];
+  auto& args = mg.args.back();
+  args.front().in = st;
+  args.back().out = st + m->input_bytes;
+  cudaStream_t s = (cudaStream_t)g->prof_stream;
+  std::vector<cudaEvent_t> ev;
+  volatile uint32_t* gate = (volatile uint32_t*)(st + g->stage_bytes - 64);
+  if (kernel_ns) {
+    // gate the stream so the chain runs back to back: events then time the device,
+    // not the host's launch rate
+    *gate = 0;
+    const volatile uint32_t* gd = nullptr;
+    cudaHostGetDevicePointer((void**)&gd, (void*)gate, 0);
+    void* gargs[1] = {(void*)&gd};
+    cudaLaunchKernel((const void*)gate_kernel(), dim3(1), dim3(1), gargs, 0, s);
+    ev.resize(m->kernels.size() + 1);
+    for (auto& e : ev) cudaEventCreate(&e);
+    cudaEventRecord(ev[0], s);
+  }
+  for (uint32_t l = 0; l < m->kernels.size(); ++l) {
+    iso_launch(g, m, l, instr);
+    if (kernel_ns) cudaEventRecord(ev[l + 1], s);
+  }
+  if (kernel_ns) {
+    std::atomic_thread_fence(std::memory_order_seq_cst);
+    *gate = 1;
+  }
+  cudaError_t e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) {
+    fprintf(stderr, "paella: isolated run failed: %s\n", cudaGetErrorString(e));
+    return -EIO;
+  }
+  if (kernel_ns) {
+    for (uint32_t l = 0; l < m->kernels.size(); ++l) {
+      float ms = 0;
+      cudaEventElapsedTime(&ms, ev[l], ev[l + 1]);
+      kernel_ns[l] = (int64_t)((double)ms * 1e6);
+    }
+    for (auto& x : ev) cudaEventDestroy(x);
+  }
+  if (output) std::memcpy(output, st + m->input_bytes, m->output_bytes);
+  return 0;
+}
+
+static int setup_model_gpu(Paella* P, Model* m, Gpu* g) {
+  ModelGpu& mg = m->gpu[g->index];
+  const uint32_t slots = P->cfg.max_jobs_per_model;
+  const size_t nslot = slots + 1;   // + the isolated slot
+  const bool cuda = P->cfg.device == PAELLA_DEVICE_CUDA;
+  uint8_t* wdev;
+  uint8_t* wsp;
+  if (cuda) {
+    cudaSetDevice(g->device);
+    if (cudaMalloc((void**)&wdev, m->blob.size() + 256)) return -ENOMEM;
+    cudaMemcpy(wdev, m->blob.data(), m->blob.size(), cudaMemcpyHostToDevice);
+    if (cudaMalloc((void**)&wsp, nslot * m->slot_bytes)) return -ENOMEM;
+    cudaMemset(wsp, 0, nslot * m->slot_bytes);
+    if (m->splitk_floats) {
+      if (cudaMalloc((void**)&mg.splitk_ws, nslot * m->splitk_floats * 4)) return -ENOMEM;
+      if (cudaMalloc((void**)&mg.splitk_ctr, nslot * m->splitk_ctrs * 4)) return -ENOMEM;
+      cudaMemset(mg.splitk_ctr, 0, nslot * m->splitk_ctrs * 4);
+    }
+  } else {
+    wdev = (uint8_t*)malloc(m->blob.size() + 256);
+    wsp = (uint8_t*)calloc(1, 256);   // the fake device never touches activations
+  }
+  mg.weights = wdev;
+  mg.workspace = wsp;
+  auto& tmaps = mg.tmaps;
+  tmaps.resize(m->kernels.size());
+  // per-kernel attributes -> Table-1 demand
+  for (uint32_t l = 0; l < m->kernels.size(); ++l) {
+    KernelInst& k = m->kernels[l];
+    if (cuda) {
+      auto* cb = static_cast<CudaBackend*>(g->be.get());
+      KernelFn f = cb->fn(k.kind, m->dtype, true);
+      if (!f) return -EINVAL;
+      cudaFuncAttributes fa;
+      if (cudaFuncGetAttributes(&fa, (const void*)f)) return -EIO;
+      if (k.smem > 48 * 1024) {
+        cudaFuncSetAttribute((const void*)f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k.smem);
+        cudaFuncSetAttribute((const void*)cb->fn(k.kind, m->dtype, false),
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k.smem);
+      }
+      // constant per-SM capacity for Table-1 accounting: maximum carveout (hard part #4)
+      cudaFuncSetAttribute((const void*)f, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+      cudaFuncSetAttribute((const void*)cb->fn(k.kind, m->dtype, false),
+                           cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+      k.regs = (uint32_t)fa.numRegs;
+      k.static_smem = (uint32_t)fa.sharedSizeBytes;
+      if (k.kind == KIND_CONV_TC) {
+        if (make_weight_tmap(wdev + k.w_off, k.proto.tiles_m * TC_BM, k.proto.kpad, tmaps[l].b)) return -EIO;
+      }
+    } else {
+      k.regs = 64;
+      k.static_smem = 0;
+    }
+    uint32_t warps = (k.block + 31) / 32;
+    uint32_t regs_warp = (k.regs * 32 + 255) / 256 * 256;
+    k.demand[0] = 1;
+    k.demand[1] = warps;
+    k.demand[2] = (int64_t)regs_warp * warps;
+    k.demand[3] = (int64_t)((k.static_smem + k.smem + 1024 + 127) / 128 * 128);
+    k.demand[4] = k.tmem_cols;
+  }
+  // per-slot argument blocks
+  mg.args.assign(nslot, {});
+  for (size_t s = 0; s < nslot; ++s) {
+    uint8_t* base = wsp + (cuda ? s * m->slot_bytes : 0);
+    auto& A = mg.args[s];
+    A.resize(m->kernels.size());
+    for (uint32_t l = 0; l < m->kernels.size(); ++l) {
+      const KernelInst& k = m->kernels[l];
+      LayerArgs a = k.proto;
+      auto bp = [&](int32_t b) -> void* { return b >= 0 ? (void*)(base + m->bufs[b].off) : nullptr; };
+      if (k.kind != KIND_INGEST) a.in = bp(k.in_buf);
+      a.out = bp(k.out_buf);
+      a.res = bp(k.res_buf);
+      a.w = wdev + k.w_off;
+      a.bias = (const float*)(wdev + k.b_off);
+      a.pro_scale = k.has_pro ? (const float*)(wdev + k.ps_off) : nullptr;
+      a.pro_shift = k.has_pro ? (const float*)(wdev + k.pz_off) : nullptr;
+      if (cuda && mg.splitk_ws) {
+        a.ws = mg.splitk_ws + s * m->splitk_floats;
+        a.ws_ctr = mg.splitk_ctr + s * m->splitk_ctrs;
+      }
+      A[l] = a;
+    }
+  }
+  mg.free_slots.clear();
+  for (uint32_t s = slots; s-- > 0;) mg.free_slots.push_back(s);
+  // profile T-bar (P1249-1254; reading C2-Q15): GPU 0 measures, others copy
+  if (g->index == 0) {
+    uint32_t runs = 20;
+    if (cuda) {
+      std::vector<int64_t> t(m->kernels.size()), acc(m->kernels.size(), 0);
+      for (int w = 0; w < 5; ++w)
+        if (iso_run(g, m, nullptr, nullptr, nullptr, true)) return -EIO;
+      for (uint32_t r = 0; r < runs; ++r) {
+        if (iso_run(g, m, nullptr, nullptr, t.data(), true)) return -EIO;
+        for (size_t l = 0; l < t.size(); ++l) acc[l] += t[l];
+      }
+      for (size_t l = 0; l < t.size(); ++l) m->kernels[l].tbar = std::max<int64_t>(1, acc[l] / runs);
+    } else {
+      // fake device: analytic block duration, used as its own "profile"
+      for (auto& k : m->kernels) k.tbar = 2000 + 40 * (int64_t)((k.grid_total() + P->sms - 1) / P->sms) * 1000 / 1000;
+    }
+  }
+  return 0;
+}
+
+}  // namespace paella
+
+extern "C" {
+
+int paella_run_isolated(paella_t* p, uint32_t gpu, uint32_t model_id, const void* input, void* output,
+                        int64_t* kernel_ns) {
+  Paella* P = (Paella*)p;
+  if (!P || gpu >= P->gpus.size() || model_id >= P->nmodels.load()) return -EINVAL;
+  if (P->cfg.device != PAELLA_DEVICE_CUDA) return -ENODEV;
+  Gpu* g = P->gpus[gpu].get();
+  std::lock_guard<std::mutex> lk(g->iso_mu);
+  return iso_run(g, P->models[model_id].get(), input, output, kernel_ns, P->cfg.instrument != 0);
+}
+
+int paella_debug_node(paella_t* p, uint32_t gpu, uint32_t model_id, uint32_t node, float* out) {
+  Paella* P = (Paella*)p;
+  if (!P || gpu >= P->gpus.size() || model_id >= P->nmodels.load() || !out) return -EINVAL;
+  if (P->cfg.device != PAELLA_DEVICE_CUDA) return -ENODEV;
+  Model* m = P->models[model_id].get();
+  if (node >= m->nodes.size() || m->buf_of[node] < 0) return -EINVAL;
+  Gpu* g = P->gpus[gpu].get();
+  const paella_node_t& nd = m->nodes[node];
+  const Buffer& b = m->bufs[m->buf_of[node]];
+  const size_t es = m->dtype == PAELLA_DTYPE_BF16 ? 2 : 4;
+  std::vector<uint8_t> h(b.bytes);
+  cudaSetDevice(g->device);
+  uint8_t* base = (uint8_t*)m->gpu[gpu].workspace + (m->gpu[gpu].args.size() - 1) * m->slot_bytes;
+  if (cudaMemcpy(h.data(), base + b.off, b.bytes, cudaMemcpyDeviceToHost)) return -EIO;
+  uint32_t C = nd.op == PAELLA_OP_INPUT ? nd.c : nd.c;
+  uint32_t co = m->coff[node];
+  for (uint32_t c = 0; c < C; ++c)
+    for (uint32_t p2 = 0; p2 < nd.h * nd.w; ++p2) {
+      size_t idx = (size_t)p2 * b.c + co + c;
+      float v;
+      if (es == 2) {
+        uint32_t u = (uint32_t)((uint16_t*)h.data())[idx] << 16;
+        std::memcpy(&v, &u, 4);
+      } else {
+        v = ((float*)h.data())[idx];
+      }
+      out[(size_t)c * nd.h * nd.w + p2] = v;
+    }
+  return 0;
+}
+
+}  // extern "C"

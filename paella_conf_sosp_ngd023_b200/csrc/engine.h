@@ -1,0 +1,172 @@
+// Internal structures of the Paella runtime (host side).
+#pragma once
+#include <atomic>
+#include <cstdint>
+#include <cstdio>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "../../include/paella.h"
+#include "common.h"
+#include "kernels.h"
+#include "policy.h"
+#include "spsc.h"
+
+namespace paella {
+
+// one kernel of a model's chain (one per non-concat node, plus the ingest)
+struct KernelInst {
+  uint32_t kind = 0;
+  int32_t node = -1;           // graph node it computes (-1 = ingest)
+  uint32_t grid[3] = {1, 1, 1};
+  uint32_t block = 256;
+  uint32_t smem = 0;           // dynamic shared memory
+  uint32_t regs = 32, static_smem = 0, tmem_cols = 0;
+  LayerArgs proto{};           // shapes/flags; pointers patched per GPU / slot
+  int32_t in_buf = -1, out_buf = -1, res_buf = -1;
+  size_t w_off = 0, w_bytes = 0;       // packed weights in the model's weight blob
+  size_t b_off = 0, ps_off = 0, pz_off = 0;   // fp32 bias / prologue scale / shift
+  bool has_pro = false;
+  int64_t tbar = 0;
+  uint64_t flops = 0, bytes = 0;
+  int64_t demand[NRES] = {1, 0, 0, 0, 0};
+  uint32_t grid_total() const { return grid[0] * grid[1] * grid[2]; }
+};
+
+struct Buffer {
+  uint32_t c, h, w;
+  size_t off, bytes;
+};
+
+struct TmapStore {           // CUtensorMap storage (64-byte aligned, 128 bytes)
+  alignas(64) uint8_t b[128];
+};
+
+struct ModelGpu {
+  void* weights = nullptr;     // device blob (packed weights + fp32 vectors)
+  void* workspace = nullptr;   // slots * slot_bytes (+1 isolated slot)
+  float* splitk_ws = nullptr;  // split-K fp32 partials, per slot
+  uint32_t* splitk_ctr = nullptr;
+  std::vector<std::vector<LayerArgs>> args;   // [slot][kernel]
+  std::vector<uint32_t> free_slots;
+  std::vector<TmapStore> tmaps;   // per kernel (tcgen05 conv weights)
+};
+
+struct Model {
+  std::string name;
+  uint32_t id = 0, dtype = 0;
+  std::vector<paella_node_t> nodes;       // shapes/attrs (host param pointers not kept)
+  std::vector<std::vector<int32_t>> node_inputs;
+  std::vector<int32_t> buf_of;            // node -> buffer
+  std::vector<uint32_t> coff;             // node -> channel offset in its buffer
+  std::vector<Buffer> bufs;
+  size_t slot_bytes = 0;
+  size_t splitk_floats = 0, splitk_ctrs = 0;
+  std::vector<KernelInst> kernels;
+  std::vector<uint8_t> blob;              // host copy of the packed parameters
+  size_t input_bytes = 0, output_bytes = 0;
+  uint32_t in_c = 0, in_h = 0, in_w = 0, out_n = 0;
+  std::vector<ModelGpu> gpu;
+  int64_t total_tbar = 0;
+};
+
+struct JobRec {
+  uint64_t req_id = 0;
+  uint32_t client = 0, model = 0, slot = 0;
+  uint8_t* io = nullptr;
+  int64_t t_sched = 0;
+  bool live = false;
+  // naive mode
+  uint32_t stream = 0;
+  void* event = nullptr;
+};
+
+struct Paella;
+
+// device backend: real CUDA GPU or CPU fake
+struct Backend {
+  virtual ~Backend() {}
+  virtual int init() = 0;
+  virtual Rec* ring() = 0;          // host view of the notification ring
+  virtual void launch(const KernelInst& k, const LayerArgs& a, const InstrArgs& ia, uint32_t stream,
+                      uint32_t dtype, bool instr) = 0;
+  virtual void advance() {}         // fake: progress virtual time
+  virtual int error() { return 0; }
+  virtual uint32_t* tail_dev() = 0;
+  virtual uint32_t* ctr_dev() = 0;
+  virtual void* ring_dev() = 0;
+  // naive mode completion detection
+  virtual void record_event(uint32_t stream, void** ev) = 0;
+  virtual bool event_done(void* ev) = 0;
+  virtual void release_event(void* ev) = 0;
+  virtual void sync() {}
+};
+
+struct Gpu {
+  Paella* P = nullptr;
+  uint32_t index = 0;       // instance-local index
+  int device = 0;           // CUDA ordinal
+  std::unique_ptr<Backend> be;
+  std::unique_ptr<Policy> policy;
+  uint64_t head = 0;        // notification ring consumer index
+  uint32_t cap = 0, log2cap = 0;
+  std::vector<uint32_t> ctr_base;   // running base per counter slot
+  std::vector<JobRec> jobs;         // indexed by job id (dense)
+  std::vector<uint32_t> free_job_ids;
+  uint32_t next_job = 0;
+  std::vector<SpscRing<SubmitSlot>*> sub;     // per client
+  std::vector<SpscRing<CompleteSlot>*> done;  // per client
+  std::thread thread;
+  std::atomic<bool> stop{false};
+  std::atomic<int64_t> work_published{0};
+  std::atomic<uint64_t> admitted_pub{0};
+  std::atomic<uint64_t> submitted{0};
+  std::atomic<int> err{0};
+  uint32_t rr_start = 0;
+  FILE* log = nullptr;
+  std::mutex log_mu;
+  paella_stats_t stats{};
+  std::vector<Issue> issues;
+  // isolated runs (profiling, parity tests): private ring, counters and stream
+  Rec* prof_ring_h = nullptr;
+  void* prof_ring_d = nullptr;
+  uint32_t* prof_tail = nullptr;
+  uint32_t* prof_ctr = nullptr;
+  std::vector<uint32_t> prof_base;
+  uint32_t prof_uid = 0;
+  void* prof_stream = nullptr;
+  void* stage_in = nullptr;    // pinned mapped staging for isolated-run io
+  size_t stage_bytes = 0;
+  std::mutex iso_mu;
+  std::vector<uint32_t> naive_inflight;   // job ids in naive mode
+};
+
+struct Paella {
+  paella_config_t cfg{};
+  uint32_t sms = 148;
+  std::vector<std::unique_ptr<Gpu>> gpus;
+  std::vector<std::unique_ptr<Model>> models;   // capacity reserved; published via nmodels
+  std::atomic<uint32_t> nmodels{0};
+  std::mutex reg_mu;
+  std::vector<uint8_t*> region;                 // client io regions
+  size_t region_bytes = 0;
+  std::vector<void*> shm_maps;
+  std::vector<size_t> shm_sizes;
+  std::vector<std::atomic<uint64_t>*> client_seq;
+  std::vector<uint32_t> rr_next;                // per-client round-robin router state
+  std::vector<uint32_t> poll_rr;                // per-client completion ring scan start
+  std::atomic<bool> shutting{false};
+  int64_t capacity[NRES];
+};
+
+// planner (plan.cpp)
+int plan_model(Paella* P, const paella_model_desc_t* d, Model* m);
+uint32_t tc_tmem_cols();
+
+// time
+int64_t now_ns();
+
+}  // namespace paella

@@ -1,0 +1,84 @@
+// Block entry / exit instrumentation (K1) -- Paella Fig. 6 (PAPER.md P848-870, §4.1
+// P872-899) re-designed for sm_100a:
+//
+//  * one elected thread per block does the counter atomic; the other warps never
+//    wait on it at entry (they start computing immediately);
+//  * per-launch counters {start, end} in device memory, slot = uid mod NCTR, never
+//    reset -- the dispatcher passes the slot's running base (reading C2-Q1);
+//  * the block whose count reaches a multiple of G or the grid total claims a ring
+//    index with one atomicAdd on the tail (power-of-two ring + lap tag, C2-Q2/Q3) and
+//    writes ONE 16-byte record {type, count, smid, uid | globaltimer, group} with a
+//    single vector store straight into pinned, mapped host memory (P1104-1106);
+//  * exit: __syncthreads (all outputs of the block written), a release fence
+//    (gpu scope; system scope for a job's last kernel, whose output lives in client
+//    host memory) before the end-counter atomic, so a successor kernel launched after
+//    the dispatcher saw the final COMPLETION reads complete data (reading C2-Q19);
+//  * %smid is re-read at exit (reading C2-Q4).
+//
+// Compiled out entirely in the uninstrumented twin (INSTR = false).
+#pragma once
+#include "common.h"
+
+namespace paella {
+
+__device__ __forceinline__ uint32_t smid_reg() {
+  uint32_t s;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(s));
+  return s;
+}
+
+__device__ __forceinline__ uint64_t globaltimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+__device__ __forceinline__ void put_record(const InstrArgs& ia, uint32_t type, uint32_t count_in_group,
+                                           uint32_t group) {
+  uint32_t idx = atomicAdd(ia.tail, 1u);
+  uint32_t slot = idx & ia.mask;
+  uint32_t lap = idx >> ia.log2cap;
+  Rec r = rec_encode(type, count_in_group, smid_reg(), lap, ia.uid, globaltimer(), group);
+  asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(ia.ring + slot), "l"(r.w0), "l"(r.w1)
+               : "memory");
+}
+
+// count = 1-based index of this block's arrival at the counter
+__device__ __forceinline__ void maybe_record(const InstrArgs& ia, uint32_t type, uint32_t count,
+                                             uint32_t total) {
+  uint32_t G = ia.group;
+  uint32_t r = count % G;
+  if (r == 0 || count == total) {
+    uint32_t n = (r == 0) ? G : r;
+    put_record(ia, type, n, (count - 1) / G);
+  }
+}
+
+template <bool INSTR>
+__device__ __forceinline__ void instr_enter(const InstrArgs& ia) {
+  if constexpr (INSTR) {
+    if (threadIdx.x == 0 && threadIdx.y == 0 && threadIdx.z == 0) {
+      uint32_t total = gridDim.x * gridDim.y * gridDim.z;
+      uint32_t c = atomicAdd(&ia.ctr[0], 1u) + 1u - ia.base;
+      maybe_record(ia, REC_PLACEMENT, c, total);
+    }
+  }
+}
+
+template <bool INSTR>
+__device__ __forceinline__ void instr_exit(const InstrArgs& ia) {
+  if constexpr (INSTR) {
+    __syncthreads();
+    if (threadIdx.x == 0 && threadIdx.y == 0 && threadIdx.z == 0) {
+      if (ia.flags & INSTR_LAST)
+        __threadfence_system();
+      else
+        __threadfence();
+      uint32_t total = gridDim.x * gridDim.y * gridDim.z;
+      uint32_t c = atomicAdd(&ia.ctr[1], 1u) + 1u - ia.base;
+      maybe_record(ia, REC_COMPLETION, c, total);
+    }
+  }
+}
+
+}  // namespace paella

@@ -1,0 +1,36 @@
+// Kernel kinds of the CUDA path and their launch table.
+#pragma once
+#include <stdint.h>
+
+namespace paella {
+
+enum KernelKind : uint32_t {
+  KIND_INGEST = 0,
+  KIND_CONV_SIMT = 1,
+  KIND_CONV_TC = 2,     // tcgen05 implicit-GEMM conv (bf16)
+  KIND_DWCONV = 3,
+  KIND_MAXPOOL = 4,
+  KIND_AVGPOOL = 5,
+  KIND_GAP = 6,
+  KIND_FC = 7,
+  KIND_EMPTY = 8,
+  KIND_COUNT = 9,
+};
+
+typedef void (*KernelFn)();
+
+void simt_kernel_table(KernelFn (&bf16_instr)[KIND_COUNT], KernelFn (&bf16_plain)[KIND_COUNT],
+                       KernelFn (&f32_instr)[KIND_COUNT], KernelFn (&f32_plain)[KIND_COUNT]);
+
+KernelFn gate_kernel();   // k_gate(const volatile uint32_t* flag)
+
+// tcgen05 conv: instrumented / plain instantiations and their launch geometry
+void tc_kernel_table(KernelFn* instr, KernelFn* plain);
+constexpr uint32_t TC_BM = 128;       // Cout rows per CTA (UMMA M, TMEM lanes)
+constexpr uint32_t TC_BN = 64;        // output pixels per CTA (UMMA N)
+constexpr uint32_t TC_BK = 64;        // K per pipeline stage (128 B of bf16 = one swizzle row)
+constexpr uint32_t TC_STAGES = 4;
+constexpr uint32_t TC_THREADS = 160;    // 4 producer/epilogue warps + 1 MMA warp
+uint32_t tc_smem_bytes();
+
+}  // namespace paella

@@ -1,0 +1,392 @@
+// SIMT inference kernels (K2b-K2e, and the fp32 / fallback-free SIMT conv K2a-simt).
+//
+// All activations are NHWC with an explicit channel stride (LayerArgs::*_cs) and
+// channel offset (*_co): channel counts are multiples of 8 after the ingest pads the
+// image to 8 channels, so every thread moves 8 channels = one 16-byte vector (bf16)
+// or two (fp32).  Every kernel is built twice (INSTR = true: Paella-instrumented,
+// false: the uninstrumented twin used by the naive baseline and the overhead
+// microbenchmark).  No kernel returns early: instr_exit needs every thread.
+#include <cuda_bf16.h>
+
+#include "common.h"
+#include "instr.cuh"
+#include "kernels.h"
+
+namespace paella {
+
+// ---------------------------------------------------------------------------
+// 8-element vector load / store
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void load8(const __nv_bfloat16* p, float (&v)[8]) {
+  uint4 u = *reinterpret_cast<const uint4*>(p);
+  const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&u);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    float2 f = __bfloat1622float2(h[i]);
+    v[2 * i] = f.x;
+    v[2 * i + 1] = f.y;
+  }
+}
+__device__ __forceinline__ void load8(const float* p, float (&v)[8]) {
+  float4 a = reinterpret_cast<const float4*>(p)[0];
+  float4 b = reinterpret_cast<const float4*>(p)[1];
+  v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
+  v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
+}
+__device__ __forceinline__ void store8(__nv_bfloat16* p, const float (&v)[8]) {
+  uint4 u;
+  __nv_bfloat162* h = reinterpret_cast<__nv_bfloat162*>(&u);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) h[i] = __floats2bfloat162_rn(v[2 * i], v[2 * i + 1]);  // RNE
+  *reinterpret_cast<uint4*>(p) = u;
+}
+__device__ __forceinline__ void store8(float* p, const float (&v)[8]) {
+  reinterpret_cast<float4*>(p)[0] = make_float4(v[0], v[1], v[2], v[3]);
+  reinterpret_cast<float4*>(p)[1] = make_float4(v[4], v[5], v[6], v[7]);
+}
+
+__device__ __forceinline__ float act_f(float x, uint32_t act) {
+  if (act == 1) return fmaxf(x, 0.f);
+  if (act == 2) return fminf(fmaxf(x, 0.f), 6.f);
+  return x;
+}
+
+// ---------------------------------------------------------------------------
+// K2e ingest: client fp32 NCHW (pinned, mapped host memory) -> model dtype NHWC,
+// channels padded to 8 with zeros.  bf16 rounding is RNE (reading C1-Q7).
+// ---------------------------------------------------------------------------
+template <typename T, bool INSTR>
+__global__ void __launch_bounds__(256) k_ingest(const __grid_constant__ LayerArgs a,
+                                                const __grid_constant__ InstrArgs ia) {
+  instr_enter<INSTR>(ia);
+  const float* in = static_cast<const float*>(a.in);
+  T* out = static_cast<T*>(a.out);
+  uint32_t hw = a.h * a.w_;
+  uint32_t p = blockIdx.x * blockDim.x + threadIdx.x;
+  if (p < hw) {
+    float v[8];
+#pragma unroll
+    for (int c = 0; c < 8; ++c) v[c] = (c < (int)a.cin) ? __ldcs(in + (size_t)c * hw + p) : 0.f;
+    store8(out + (size_t)p * a.out_cs + a.out_co, v);
+  }
+  instr_exit<INSTR>(ia);
+}
+
+// ---------------------------------------------------------------------------
+// K2a (SIMT): conv as implicit GEMM  D[Cout x P] = W[Cout x K] . im2col(X)[K x P],
+// K = kh*kw*cin ordered (r, s, ci) so 8 consecutive k are 8 consecutive channels.
+// Tile 64 (cout) x 64 (pixels) x 32 (k), 256 threads, 4x4 outputs per thread.
+// Weights packed [cout][Kpad] (Kpad = K rounded up to 64, zero-filled).
+// Used for the fp32 path (SIMT FFMA, no TF32 -- reading C1-Q3) and for convs the
+// tcgen05 kernel does not take.  Epilogue: bias, residual (fp32), activation, one
+// rounding.
+// ---------------------------------------------------------------------------
+template <typename T, bool INSTR>
+__global__ void __launch_bounds__(256) k_conv_simt(const __grid_constant__ LayerArgs a,
+                                                   const __grid_constant__ InstrArgs ia) {
+  instr_enter<INSTR>(ia);
+  constexpr int BM = 64, BN = 64, BK = 32;
+  __shared__ float As[BK][BM + 4];
+  __shared__ float Bs[BK][BN + 4];
+  const T* X = static_cast<const T*>(a.in);
+  const T* W = static_cast<const T*>(a.w);
+  const int tid = threadIdx.x;
+  const int co0 = blockIdx.y * BM;
+  const int p0 = blockIdx.x * BN;
+  const int P = a.oh * a.ow;
+  const int K = a.kh * a.kw * a.cin;
+  const int tm = tid % 16, tn = tid / 16;
+  float acc[4][4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int j = 0; j < 4; ++j) acc[i][j] = 0.f;
+
+  // this thread's B-load pixel
+  const int lp = tid % 64, lkg = tid / 64;   // pixel, k-granule (0..3)
+  const int gp = p0 + lp;
+  const int oh = gp / a.ow, ow = gp % a.ow;
+  // this thread's A-load row
+  const int arow = tid / 4, akg = tid % 4;
+
+  for (int k0 = 0; k0 < (int)a.kpad; k0 += BK) {
+    {  // A: 64 rows x 32 k
+      float v[8];
+      int co = co0 + arow;
+      if (co < (int)a.cout) {
+        load8(W + (size_t)co * a.kpad + k0 + akg * 8, v);
+      } else {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) v[i] = 0.f;
+      }
+#pragma unroll
+      for (int i = 0; i < 8; ++i) As[akg * 8 + i][arow] = v[i];
+    }
+    {  // B: 32 k x 64 pixels, im2col gather
+      float v[8];
+      int k = k0 + lkg * 8;
+      bool ok = (gp < P) && (k < K);
+      int ci = 0, ih = 0, iw = 0;
+      if (ok) {
+        ci = k % a.cin;
+        int rs = k / a.cin;
+        int s = rs % a.kw, r = rs / a.kw;
+        ih = oh * a.sh - a.ph + r;
+        iw = ow * a.sw - a.pw + s;
+        ok = ih >= 0 && ih < (int)a.h && iw >= 0 && iw < (int)a.w_;
+      }
+      if (ok) {
+        load8(X + ((size_t)ih * a.w_ + iw) * a.in_cs + a.in_co + ci, v);
+        if (a.flags & LF_PROLOGUE) {
+#pragma unroll
+          for (int i = 0; i < 8; ++i) v[i] = fmaxf(fmaf(a.pro_scale[ci + i], v[i], a.pro_shift[ci + i]), 0.f);
+        }
+      } else {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) v[i] = 0.f;
+      }
+#pragma unroll
+      for (int i = 0; i < 8; ++i) Bs[lkg * 8 + i][lp] = v[i];
+    }
+    __syncthreads();
+#pragma unroll 8
+    for (int k = 0; k < BK; ++k) {
+      float4 av = *reinterpret_cast<const float4*>(&As[k][tm * 4]);
+      float4 bv = *reinterpret_cast<const float4*>(&Bs[k][tn * 4]);
+      float am[4] = {av.x, av.y, av.z, av.w};
+      float bn[4] = {bv.x, bv.y, bv.z, bv.w};
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(am[i], bn[j], acc[i][j]);
+    }
+    __syncthreads();
+  }
+  // epilogue
+  T* Y = static_cast<T*>(a.out);
+  const T* Rz = static_cast<const T*>(a.res);
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    int p = p0 + tn * 4 + j;
+    if (p >= P) continue;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      int co = co0 + tm * 4 + i;
+      if (co >= (int)a.cout) continue;
+      float v = acc[i][j] + a.bias[co];
+      if (a.flags & LF_RESIDUAL) v += (float)Rz[(size_t)p * a.res_cs + a.res_co + co];
+      v = act_f(v, a.act);
+      Y[(size_t)p * a.out_cs + a.out_co + co] = (T)v;
+    }
+  }
+  instr_exit<INSTR>(ia);
+}
+
+// ---------------------------------------------------------------------------
+// K2c depthwise conv (groups == cin == cout), any kh x kw, stride, pad.  One thread
+// per (output pixel, 8-channel granule).  Weights packed [kh][kw][c].
+// ---------------------------------------------------------------------------
+template <typename T, bool INSTR>
+__global__ void __launch_bounds__(256) k_dwconv(const __grid_constant__ LayerArgs a,
+                                                const __grid_constant__ InstrArgs ia) {
+  instr_enter<INSTR>(ia);
+  const T* X = static_cast<const T*>(a.in);
+  const T* W = static_cast<const T*>(a.w);
+  T* Y = static_cast<T*>(a.out);
+  uint32_t ng = a.cout / 8;
+  uint32_t idx = blockIdx.x * blockDim.x + threadIdx.x;
+  uint32_t P = a.oh * a.ow;
+  if (idx < P * ng) {
+    uint32_t g = idx % ng, p = idx / ng;
+    int oh = p / a.ow, ow = p % a.ow;
+    int c = g * 8;
+    float acc[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) acc[i] = a.bias[c + i];
+    for (int r = 0; r < (int)a.kh; ++r) {
+      int ih = oh * a.sh - a.ph + r;
+      if (ih < 0 || ih >= (int)a.h) continue;
+      for (int s = 0; s < (int)a.kw; ++s) {
+        int iw = ow * a.sw - a.pw + s;
+        if (iw < 0 || iw >= (int)a.w_) continue;
+        float xv[8], wv[8];
+        load8(X + ((size_t)ih * a.w_ + iw) * a.in_cs + a.in_co + c, xv);
+        load8(W + ((size_t)r * a.kw + s) * a.cout + c, wv);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) acc[i] = fmaf(wv[i], xv[i], acc[i]);
+      }
+    }
+    if (a.flags & LF_RESIDUAL) {
+      float rv[8];
+      load8(static_cast<const T*>(a.res) + (size_t)p * a.res_cs + a.res_co + c, rv);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) acc[i] += rv[i];
+    }
+#pragma unroll
+    for (int i = 0; i < 8; ++i) acc[i] = act_f(acc[i], a.act);
+    store8(Y + (size_t)p * a.out_cs + a.out_co + c, acc);
+  }
+  instr_exit<INSTR>(ia);
+}
+
+// ---------------------------------------------------------------------------
+// K2d pooling.  max: padding = -inf, ceil-mode windows clipped to the input;
+// avg: count_include_pad (divisor k*k).  One thread per (pixel, granule).
+// ---------------------------------------------------------------------------
+template <typename T, bool INSTR, bool MAX>
+__global__ void __launch_bounds__(256) k_pool(const __grid_constant__ LayerArgs a,
+                                              const __grid_constant__ InstrArgs ia) {
+  instr_enter<INSTR>(ia);
+  const T* X = static_cast<const T*>(a.in);
+  T* Y = static_cast<T*>(a.out);
+  uint32_t ng = a.cout / 8;
+  uint32_t idx = blockIdx.x * blockDim.x + threadIdx.x;
+  uint32_t P = a.oh * a.ow;
+  if (idx < P * ng) {
+    uint32_t g = idx % ng, p = idx / ng;
+    int oh = p / a.ow, ow = p % a.ow;
+    int c = g * 8;
+    float acc[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) acc[i] = MAX ? -INFINITY : 0.f;
+    for (int r = 0; r < (int)a.kh; ++r) {
+      int ih = oh * a.sh - a.ph + r;
+      if (ih < 0 || ih >= (int)a.h) continue;
+      for (int s = 0; s < (int)a.kw; ++s) {
+        int iw = ow * a.sw - a.pw + s;
+        if (iw < 0 || iw >= (int)a.w_) continue;
+        float xv[8];
+        load8(X + ((size_t)ih * a.w_ + iw) * a.in_cs + a.in_co + c, xv);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) acc[i] = MAX ? fmaxf(acc[i], xv[i]) : acc[i] + xv[i];
+      }
+    }
+    if (!MAX) {
+      float inv = 1.f / (float)(a.kh * a.kw);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) acc[i] *= inv;
+    }
+    store8(Y + (size_t)p * a.out_cs + a.out_co + c, acc);
+  }
+  instr_exit<INSTR>(ia);
+}
+
+// ---------------------------------------------------------------------------
+// Global average pool (+ optional DenseNet prologue).  One thread per channel
+// granule; output either an activation (C,1,1) or, if final, fp32 logits in client
+// memory.
+// ---------------------------------------------------------------------------
+template <typename T, bool INSTR>
+__global__ void __launch_bounds__(128) k_gap(const __grid_constant__ LayerArgs a,
+                                             const __grid_constant__ InstrArgs ia) {
+  instr_enter<INSTR>(ia);
+  const T* X = static_cast<const T*>(a.in);
+  uint32_t ng = a.cout / 8;
+  uint32_t g = blockIdx.x * blockDim.x + threadIdx.x;
+  if (g < ng) {
+    int c = g * 8;
+    float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    uint32_t HW = a.h * a.w_;
+    for (uint32_t p = 0; p < HW; ++p) {
+      float xv[8];
+      load8(X + (size_t)p * a.in_cs + a.in_co + c, xv);
+      if (a.flags & LF_PROLOGUE) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) xv[i] = fmaxf(fmaf(a.pro_scale[c + i], xv[i], a.pro_shift[c + i]), 0.f);
+      }
+#pragma unroll
+      for (int i = 0; i < 8; ++i) acc[i] += xv[i];
+    }
+    float inv = 1.f / (float)HW;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) acc[i] *= inv;
+    if (a.flags & LF_FINAL) {
+      store8(static_cast<float*>(a.out) + c, acc);
+    } else {
+      store8(static_cast<T*>(a.out) + a.out_co + c, acc);
+    }
+  }
+  instr_exit<INSTR>(ia);
+}
+
+// ---------------------------------------------------------------------------
+// K2b FC at batch 1 = weight-streaming GEMV (HBM-bound: no tensor cores, reading of
+// the north star "do not reshape HBM-bound work into GEMMs").  One warp per output
+// row, 16-byte weight loads, fp32 accumulate, warp-shuffle reduction.  Weights
+// [cout][kpad] in NHWC-flatten order (the planner permutes torch's NCHW flatten).
+// ---------------------------------------------------------------------------
+template <typename T, bool INSTR>
+__global__ void __launch_bounds__(256) k_fc(const __grid_constant__ LayerArgs a,
+                                            const __grid_constant__ InstrArgs ia) {
+  instr_enter<INSTR>(ia);
+  const T* X = static_cast<const T*>(a.in);
+  const T* W = static_cast<const T*>(a.w);
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int row = blockIdx.x * 8 + warp;
+  const int K = a.cin;   // multiple of 8, input contiguous (checked by the planner)
+  if (row < (int)a.cout) {
+    float acc = 0.f;
+    const T* wr = W + (size_t)row * a.kpad;
+    for (int k = lane * 8; k < K; k += 32 * 8) {
+      float wv[8], xv[8];
+      load8(wr + k, wv);
+      load8(X + a.in_co + k, xv);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) acc = fmaf(wv[i], xv[i], acc);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (lane == 0) {
+      float v = act_f(acc + a.bias[row], a.act);
+      if (a.flags & LF_FINAL)
+        static_cast<float*>(a.out)[row] = v;
+      else
+        static_cast<T*>(a.out)[a.out_co + row] = (T)v;
+    }
+  }
+  instr_exit<INSTR>(ia);
+}
+
+// ---------------------------------------------------------------------------
+// Empty instrumented kernel for the notification microbenchmark (K5, Fig. 15).
+// ---------------------------------------------------------------------------
+template <bool INSTR>
+__global__ void k_empty(const __grid_constant__ LayerArgs a, const __grid_constant__ InstrArgs ia) {
+  instr_enter<INSTR>(ia);
+  instr_exit<INSTR>(ia);
+}
+
+// ---------------------------------------------------------------------------
+// Gate: holds a stream until the host sets *flag (mapped host memory), so that the
+// kernels queued behind it run back to back and CUDA events time the device only.
+// ---------------------------------------------------------------------------
+__global__ void k_gate(const volatile uint32_t* flag) {
+  while (*flag == 0) __nanosleep(1000);
+}
+
+KernelFn gate_kernel() { return (KernelFn)k_gate; }
+
+// ---------------------------------------------------------------------------
+// kernel table
+// ---------------------------------------------------------------------------
+template <typename T, bool I>
+static void fill(KernelFn (&t)[KIND_COUNT]) {
+  t[KIND_INGEST] = (KernelFn)k_ingest<T, I>;
+  t[KIND_CONV_SIMT] = (KernelFn)k_conv_simt<T, I>;
+  t[KIND_DWCONV] = (KernelFn)k_dwconv<T, I>;
+  t[KIND_MAXPOOL] = (KernelFn)k_pool<T, I, true>;
+  t[KIND_AVGPOOL] = (KernelFn)k_pool<T, I, false>;
+  t[KIND_GAP] = (KernelFn)k_gap<T, I>;
+  t[KIND_FC] = (KernelFn)k_fc<T, I>;
+  t[KIND_EMPTY] = (KernelFn)k_empty<I>;
+}
+
+void simt_kernel_table(KernelFn (&bf16_instr)[KIND_COUNT], KernelFn (&bf16_plain)[KIND_COUNT],
+                       KernelFn (&f32_instr)[KIND_COUNT], KernelFn (&f32_plain)[KIND_COUNT]) {
+  fill<__nv_bfloat16, true>(bf16_instr);
+  fill<__nv_bfloat16, false>(bf16_plain);
+  fill<float, true>(f32_instr);
+  fill<float, false>(f32_plain);
+}
+
+}  // namespace paella

@@ -1,0 +1,362 @@
+// K2a: convolution as implicit GEMM on the 5th-generation tensor cores (sm_100a).
+//
+//   D[Cout x P] = W[Cout x K] . im2col(X)[K x P],   K = kh*kw*cin ordered (r, s, ci)
+//
+// Batch-1 CNN layers have small P (HW down to 49) and Cout >= 64, so the GEMM is
+// "swap-AB": Cout is the 128-row UMMA M (= TMEM lanes), output pixels are N = 64.
+//
+//  * A (weights, [Cout_pad][Kpad] bf16, K-major) is fed by TMA: a 2D tiled tensor
+//    map, box 64 (k) x 128 (rows), 128-byte swizzle -- exactly the UMMA K-major
+//    SWIZZLE_128B canonical layout;
+//  * B (the im2col gather of NHWC activations, with padding, stride, channel stride
+//    and channel offset of concat buffers) is gathered by 4 producer warps with
+//    16-byte cp.async (zero-fill for padding) into the same swizzled layout;
+//  * one elected thread of the MMA warp issues tcgen05.mma.cta_group::1.kind::f16
+//    (bf16 x bf16 -> fp32 in TMEM), 4 x K=16 per 64-wide k-block, and releases each
+//    smem stage with tcgen05.commit -> mbarrier (4-stage ring);
+//  * epilogue: the 4 producer warps read the accumulator with tcgen05.ld (warp w
+//    owns TMEM lanes 32w..32w+31 = 32 output channels), add bias, residual (fp32),
+//    activation, round once to bf16 (reading C1-Q7) and store NHWC;
+//  * split-K over blockIdx.z for the deep, narrow late layers: fp32 partials to a
+//    per-job workspace, the last-arriving CTA of a tile reduces and runs the epilogue.
+//
+// Block instrumentation (K1) wraps the whole CTA (instr.cuh).
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include "common.h"
+#include "instr.cuh"
+#include "kernels.h"
+
+namespace paella {
+
+namespace {
+
+constexpr uint32_t A_BYTES = TC_BM * TC_BK * 2;   // 16 KiB
+constexpr uint32_t B_BYTES = TC_BN * TC_BK * 2;   // 8 KiB
+constexpr uint32_t LOOK = 2;                      // cp.async groups in flight per producer
+constexpr uint32_t NPROD = 128;                   // producer threads (warps 0-3)
+
+__device__ __forceinline__ uint32_t su32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(su32(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(su32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint64_t* b, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(su32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n}" ::"r"(su32(b)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, uint64_t* bar, int x, int y) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(
+          su32(dst)),
+      "l"(map), "r"(su32(bar)), "r"(x), "r"(y)
+      : "memory");
+}
+__device__ __forceinline__ void cp_async16(uint32_t dst, const void* src, uint32_t src_bytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+
+// UMMA shared-memory descriptor, K-major, SWIZZLE_128B: 8-row x 128-byte atoms,
+// stride between 8-row groups (SBO) 1024 B; version 1 (sm_100); layout type 2.
+__device__ __forceinline__ uint64_t sdesc_sw128(uint32_t saddr) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr & 0x3FFFF) >> 4);        // start address
+  d |= (uint64_t)(16 >> 4) << 16;                  // LBO (unused for SW128 K-major)
+  d |= (uint64_t)(1024 >> 4) << 32;                // SBO
+  d |= (uint64_t)1 << 46;                          // descriptor version (sm_100)
+  d |= (uint64_t)2 << 61;                          // SWIZZLE_128B
+  return d;
+}
+
+// instruction descriptor, kind::f16: D=F32, A=B=BF16, both K-major, N, M
+__host__ __device__ constexpr uint32_t idesc_bf16(uint32_t M, uint32_t N) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | ((N >> 3) << 17) | ((M >> 4) << 24);
+}
+
+__device__ __forceinline__ void umma_bf16(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                          uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}" ::"r"(tmem_d),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+__device__ __forceinline__ void umma_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(su32(bar))
+               : "memory");
+}
+
+// 32 lanes x 32 bit, 16 consecutive columns per thread
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, float (&v)[16]) {
+  uint32_t r[16];
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+  for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
+}
+
+__device__ __forceinline__ float act_tc(float x, uint32_t act) {
+  if (act == 1) return fmaxf(x, 0.f);
+  if (act == 2) return fminf(fmaxf(x, 0.f), 6.f);
+  return x;
+}
+
+}  // namespace
+
+template <bool INSTR>
+__global__ void __launch_bounds__(TC_THREADS, 1)
+    k_conv_tc(const __grid_constant__ LayerArgs a, const __grid_constant__ InstrArgs ia,
+              const __grid_constant__ CUtensorMap wmap) {
+  instr_enter<INSTR>(ia);
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* sA = smem;                                  // STAGES x 16 KiB
+  uint8_t* sB = smem + TC_STAGES * A_BYTES;            // STAGES x 8 KiB
+  uint64_t* full = (uint64_t*)(sB + TC_STAGES * B_BYTES);
+  uint64_t* empty = full + TC_STAGES;
+  uint64_t* accb = empty + TC_STAGES;
+  uint32_t* tmem_slot = (uint32_t*)(accb + 1);
+  uint32_t* flag = tmem_slot + 1;
+
+  const uint32_t warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const uint32_t tile_n = blockIdx.x, tile_m = blockIdx.y, split = blockIdx.z;
+  const uint32_t P = a.oh * a.ow;
+  const uint32_t n0 = tile_n * TC_BN, m0 = tile_m * TC_BM;
+  const uint32_t nk = a.kpad / TC_BK;
+  const uint32_t per = (nk + a.ksplit - 1) / a.ksplit;
+  const uint32_t kb0 = split * per;
+  const uint32_t kb1 = min(nk, kb0 + per);
+  const uint32_t nkl = kb1 > kb0 ? kb1 - kb0 : 0;
+
+  if (threadIdx.x == 0) {
+    for (uint32_t s = 0; s < TC_STAGES; ++s) {
+      mbar_init(&full[s], NPROD + 1);
+      mbar_init(&empty[s], 1);
+    }
+    mbar_init(accb, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&wmap) : "memory");
+  }
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(su32(tmem_slot)),
+                 "r"(64u)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp < 4) {
+    // ------------------------------------------------------------ producers
+    const __nv_bfloat16* X = static_cast<const __nv_bfloat16*>(a.in);
+    const uint32_t t = threadIdx.x;
+    // rows (pixels) of this thread: n = t/8 + 16*j, chunk = t%8
+    const uint32_t chunk = t % 8;
+    int ohs[4], ows[4];
+    bool pv[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      uint32_t n = t / 8 + 16 * j;
+      uint32_t p = n0 + n;
+      pv[j] = p < P;
+      ohs[j] = pv[j] ? (int)(p / a.ow) : 0;
+      ows[j] = pv[j] ? (int)(p % a.ow) : 0;
+    }
+    const uint32_t K = a.kh * a.kw * a.cin;
+    for (uint32_t it = 0; it < nkl; ++it) {
+      const uint32_t s = it % TC_STAGES;
+      const uint32_t ph = (it / TC_STAGES) & 1;
+      mbar_wait(&empty[s], ph ^ 1);
+      const uint32_t kbase = (kb0 + it) * TC_BK;
+      if (t == 0) {
+        mbar_arrive_tx(&full[s], A_BYTES);
+        tma_load_2d(sA + s * A_BYTES, &wmap, &full[s], (int)kbase, (int)m0);
+      }
+      const uint32_t k = kbase + chunk * 8;
+      int r = 0, sx = 0, ci = 0;
+      const bool kv = k < K;
+      if (kv) {
+        ci = (int)(k % a.cin);
+        int rs = (int)(k / a.cin);
+        sx = rs % (int)a.kw;
+        r = rs / (int)a.kw;
+      }
+      const uint32_t bstage = su32(sB + s * B_BYTES);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint32_t n = t / 8 + 16 * j;
+        const int ih = ohs[j] * (int)a.sh - (int)a.ph + r;
+        const int iw = ows[j] * (int)a.sw - (int)a.pw + sx;
+        const bool ok = kv && pv[j] && ih >= 0 && ih < (int)a.h && iw >= 0 && iw < (int)a.w_;
+        const __nv_bfloat16* src = ok ? X + ((size_t)ih * a.w_ + iw) * a.in_cs + a.in_co + ci : X;
+        const uint32_t dst = bstage + n * 128 + ((chunk ^ (n & 7)) << 4);
+        cp_async16(dst, src, ok ? 16u : 0u);
+      }
+      cp_async_commit();
+      if (it >= LOOK) {
+        cp_async_wait<LOOK>();
+        fence_proxy_async();
+        mbar_arrive(&full[(it - LOOK) % TC_STAGES]);
+      }
+    }
+    cp_async_wait<0>();
+    fence_proxy_async();
+    for (uint32_t it = (nkl > LOOK ? nkl - LOOK : 0); it < nkl; ++it) mbar_arrive(&full[it % TC_STAGES]);
+  } else if (lane == 0) {
+    // ------------------------------------------------------------ MMA issuer
+    constexpr uint32_t IDESC = idesc_bf16(TC_BM, TC_BN);
+    for (uint32_t it = 0; it < nkl; ++it) {
+      const uint32_t s = it % TC_STAGES;
+      mbar_wait(&full[s], (it / TC_STAGES) & 1);
+      tc_fence_after();
+      const uint32_t abase = su32(sA + s * A_BYTES), bbase = su32(sB + s * B_BYTES);
+#pragma unroll
+      for (uint32_t kk = 0; kk < TC_BK / 16; ++kk) {
+        umma_bf16(tmem, sdesc_sw128(abase + kk * 32), sdesc_sw128(bbase + kk * 32), IDESC,
+                  (it | kk) != 0 ? 1u : 0u);
+      }
+      umma_commit(&empty[s]);
+    }
+    umma_commit(accb);
+  }
+
+  // ---------------------------------------------------------------- epilogue
+  if (warp < 4) {
+    const uint32_t row = warp * 32 + lane;          // output channel within the tile
+    const uint32_t co = m0 + row;
+    const uint32_t taddr = tmem + ((warp * 32) << 16);
+    float acc[64];
+    if (nkl > 0) {
+      mbar_wait(accb, 0);
+      tc_fence_after();
+#pragma unroll
+      for (int c = 0; c < 4; ++c) {
+        float v[16];
+        tmem_ld16(taddr + c * 16, v);
+#pragma unroll
+        for (int i = 0; i < 16; ++i) acc[c * 16 + i] = v[i];
+      }
+    } else {
+#pragma unroll
+      for (int i = 0; i < 64; ++i) acc[i] = 0.f;
+    }
+    bool do_epi = true;
+    if (a.ksplit > 1) {
+      const uint32_t tiles = a.tiles_m * a.tiles_n;
+      const uint32_t tile = tile_m * a.tiles_n + tile_n;
+      float* part = a.ws + ((size_t)split * tiles + tile) * (TC_BM * TC_BN) + (size_t)row * TC_BN;
+#pragma unroll
+      for (int i = 0; i < 64; i += 4) __stcg(reinterpret_cast<float4*>(part + i), make_float4(acc[i], acc[i + 1], acc[i + 2], acc[i + 3]));
+      __threadfence();
+      asm volatile("bar.sync 1, 128;" ::: "memory");
+      if (threadIdx.x == 0) {
+        uint32_t old = atomicAdd(&a.ws_ctr[tile], 1u);
+        uint32_t last = (old == a.ksplit - 1) ? 1u : 0u;
+        if (last) a.ws_ctr[tile] = 0;   // reset for the next launch on this slot
+        *flag = last;
+      }
+      asm volatile("bar.sync 1, 128;" ::: "memory");
+      do_epi = *flag != 0;
+      if (do_epi) {
+        __threadfence();
+#pragma unroll
+        for (int i = 0; i < 64; ++i) acc[i] = 0.f;
+        for (uint32_t sp = 0; sp < a.ksplit; ++sp) {
+          const float* q = a.ws + ((size_t)sp * tiles + tile) * (TC_BM * TC_BN) + (size_t)row * TC_BN;
+#pragma unroll
+          for (int i = 0; i < 64; i += 4) {
+            float4 f = __ldcg(reinterpret_cast<const float4*>(q + i));
+            acc[i] += f.x;
+            acc[i + 1] += f.y;
+            acc[i + 2] += f.z;
+            acc[i + 3] += f.w;
+          }
+        }
+      }
+    }
+    if (do_epi && co < a.cout) {
+      const float b = a.bias[co];
+      __nv_bfloat16* Y = static_cast<__nv_bfloat16*>(a.out);
+      const __nv_bfloat16* R = static_cast<const __nv_bfloat16*>(a.res);
+      const bool has_res = (a.flags & LF_RESIDUAL) != 0;
+#pragma unroll
+      for (int j = 0; j < 64; ++j) {
+        const uint32_t p = n0 + j;
+        if (p < P) {
+          float v = acc[j] + b;
+          if (has_res) v += __bfloat162float(R[(size_t)p * a.res_cs + a.res_co + co]);
+          Y[(size_t)p * a.out_cs + a.out_co + co] = __float2bfloat16_rn(act_tc(v, a.act));
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 0) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(64u) : "memory");
+  }
+  instr_exit<INSTR>(ia);
+}
+
+uint32_t tc_smem_bytes() { return 1024 + TC_STAGES * (A_BYTES + B_BYTES) + 128; }
+
+void tc_kernel_table(KernelFn* instr, KernelFn* plain) {
+  instr[0] = (KernelFn)k_conv_tc<true>;
+  plain[0] = (KernelFn)k_conv_tc<false>;
+}
+
+// Host: tensor map for the packed weights [rows][kpad] bf16, box 64 x 128, SW128.
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+int make_weight_tmap(void* weights, uint32_t rows, uint32_t kpad, void* out128) {
+  static EncodeTiledFn enc = nullptr;
+  if (!enc) {
+    cudaDriverEntryPointQueryResult q;
+    void* fn = nullptr;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess || !fn)
+      return -1;
+    enc = (EncodeTiledFn)fn;
+  }
+  cuuint64_t dims[2] = {kpad, rows};
+  cuuint64_t strides[1] = {(cuuint64_t)kpad * 2};
+  cuuint32_t box[2] = {TC_BK, TC_BM};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = enc((CUtensorMap*)out128, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, weights, dims, strides, box, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? 0 : -1;
+}
+
+}  // namespace paella

@@ -1,0 +1,362 @@
+// Model planner: graph -> kernel chain, NHWC buffer plan, packed parameters.
+//
+// Paper: a job is the ordered sequence of its model's kernels (TVM's graph executor
+// runs ops in order on one stream; §4.2 P943-951 waitlists follow stream semantics).
+// Each kernel's static resource demand is known before launch (§4.1 P814-830:
+// grid, block, shared memory, registers) -- the planner fixes grid/block/smem here
+// and the CUDA backend reads registers from the compiled function.
+//
+//  * one kernel per non-concat node, plus the ingest (fp32 NCHW client input ->
+//    NHWC, channels padded to 8) -- BN/ReLU/residual add are fused into the conv,
+//    DenseNet's pre-activation BN+ReLU into the consuming conv/GAP as a prologue;
+//  * concat = producers write disjoint channel ranges of one buffer (zero-copy);
+//  * conv: groups==1 -> tcgen05 implicit GEMM (bf16) or SIMT implicit GEMM (fp32);
+//    depthwise -> K2c;  FC -> GEMV;  pools / GAP -> SIMT.
+#include <cmath>
+#include <cstdlib>
+#include <cstring>
+#include <stdexcept>
+#include <string>
+
+#include "engine.h"
+
+namespace paella {
+
+static size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+static uint16_t f32_to_bf16_exact(float f, bool* exact) {
+  uint32_t u;
+  std::memcpy(&u, &f, 4);
+  // RNE (inputs are required to be bf16-representable; flag otherwise)
+  uint32_t r = (u + 0x7FFFu + ((u >> 16) & 1u)) >> 16;
+  if ((u & 0xFFFFu) != 0) *exact = false;
+  return (uint16_t)r;
+}
+
+struct Blob {
+  std::vector<uint8_t>& b;
+  size_t put(const void* p, size_t n) {
+    size_t off = align_up(b.size(), 256);
+    b.resize(off + n);
+    if (p) std::memcpy(b.data() + off, p, n);
+    return off;
+  }
+};
+
+static bool use_tc() {
+  const char* e = std::getenv("PAELLA_CONV");
+  return !(e && std::string(e) == "simt");
+}
+
+uint32_t tc_tmem_cols() { return TC_BN < 32 ? 32 : TC_BN; }
+
+int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
+  const uint32_t n = d->n_nodes;
+  if (n < 2 || !d->nodes || d->nodes[0].op != PAELLA_OP_INPUT) return -EINVAL;
+  if (d->dtype != PAELLA_DTYPE_BF16 && d->dtype != PAELLA_DTYPE_FP32) return -EINVAL;
+  const size_t es = d->dtype == PAELLA_DTYPE_BF16 ? 2 : 4;
+  m->name = d->name;
+  m->dtype = d->dtype;
+  m->nodes.assign(d->nodes, d->nodes + n);
+  m->node_inputs.resize(n);
+  for (uint32_t i = 0; i < n; ++i) {
+    const paella_node_t& nd = d->nodes[i];
+    for (uint32_t k = 0; k < nd.n_inputs; ++k) {
+      int32_t s = nd.inputs[k];
+      if (s < 0 || (uint32_t)s >= i) return -EINVAL;
+      m->node_inputs[i].push_back(s);
+    }
+    if (nd.op != PAELLA_OP_INPUT && nd.n_inputs == 0) return -EINVAL;
+    if (nd.op != PAELLA_OP_CONCAT && nd.op != PAELLA_OP_INPUT && nd.n_inputs != 1) return -EINVAL;
+    if (nd.residual >= (int32_t)i) return -EINVAL;
+    if (nd.op != PAELLA_OP_INPUT && nd.c % 8 != 0 && !(i == n - 1)) return -EINVAL;
+  }
+  const paella_node_t& in = d->nodes[0];
+  if (in.c > 8) return -EINVAL;
+  m->in_c = in.c;
+  m->in_h = in.h;
+  m->in_w = in.w;
+  m->input_bytes = (size_t)in.c * in.h * in.w * 4;
+  const paella_node_t& last = d->nodes[n - 1];
+  if (last.op != PAELLA_OP_FC && last.op != PAELLA_OP_GAP) return -EINVAL;
+  m->out_n = last.c;
+  m->output_bytes = (size_t)last.c * 4;
+  if (last.c % 8 != 0 && last.op == PAELLA_OP_GAP) return -EINVAL;
+
+  // ---- buffer plan: concat aliasing, processed from the last node backwards ----
+  m->buf_of.assign(n, -1);
+  m->coff.assign(n, 0);
+  auto new_buf = [&](uint32_t c, uint32_t h, uint32_t w) {
+    m->bufs.push_back(Buffer{c, h, w, 0, 0});
+    return (int32_t)m->bufs.size() - 1;
+  };
+  for (int32_t i = (int32_t)n - 1; i >= 0; --i) {
+    const paella_node_t& nd = d->nodes[i];
+    if (nd.op != PAELLA_OP_CONCAT) continue;
+    if (m->buf_of[i] < 0) {
+      int32_t first = m->node_inputs[i][0];
+      if (m->buf_of[first] >= 0) {
+        // a prefix of a later concat (DenseNet: every layer's input is a prefix of
+        // the block's concat buffer): alias it
+        m->buf_of[i] = m->buf_of[first];
+        m->coff[i] = m->coff[first];
+      } else {
+        m->buf_of[i] = new_buf(nd.c, nd.h, nd.w);
+        m->coff[i] = 0;
+      }
+    }
+    uint32_t off = m->coff[i];
+    for (int32_t s : m->node_inputs[i]) {
+      const paella_node_t& sn = d->nodes[s];
+      if (sn.op == PAELLA_OP_INPUT) return -EINVAL;
+      if (m->buf_of[s] < 0) {
+        m->buf_of[s] = m->buf_of[i];
+        m->coff[s] = off;
+      } else if (m->buf_of[s] != m->buf_of[i] || m->coff[s] != off) {
+        return -EINVAL;   // a tensor in two non-prefix concats: unsupported layout
+      }
+      off += sn.c;
+    }
+    if (off != m->coff[i] + nd.c) return -EINVAL;
+  }
+  for (uint32_t i = 0; i < n; ++i) {
+    const paella_node_t& nd = d->nodes[i];
+    if (m->buf_of[i] >= 0) continue;
+    if (i == n - 1) continue;                     // final output goes to client memory
+    if (nd.op == PAELLA_OP_INPUT)
+      m->buf_of[i] = new_buf(8, nd.h, nd.w);      // ingest pads channels to 8
+    else
+      m->buf_of[i] = new_buf(nd.c, nd.h, nd.w);
+  }
+  size_t ws = 0;
+  for (auto& b : m->bufs) {
+    b.bytes = (size_t)b.c * b.h * b.w * es;
+    b.off = ws;
+    ws = align_up(ws + b.bytes, 256);
+  }
+  m->slot_bytes = std::max<size_t>(ws, 256);
+
+  // ---- kernels + packed parameters ----
+  Blob blob{m->blob};
+  const bool tc = use_tc() && d->dtype == PAELLA_DTYPE_BF16;
+  bool exact = true;
+  auto cs_of = [&](int32_t node) { return m->bufs[m->buf_of[node]].c; };
+
+  {  // ingest
+    KernelInst k;
+    k.kind = KIND_INGEST;
+    k.node = 0;
+    k.out_buf = m->buf_of[0];
+    LayerArgs& a = k.proto;
+    a.cin = in.c;
+    a.h = in.h;
+    a.w_ = in.w;
+    a.cout = 8;
+    a.oh = in.h;
+    a.ow = in.w;
+    a.out_cs = 8;
+    a.out_co = 0;
+    k.grid[0] = (in.h * in.w + 255) / 256;
+    k.block = 256;
+    k.bytes = (uint64_t)in.c * in.h * in.w * 4 + (uint64_t)8 * in.h * in.w * es;
+    m->kernels.push_back(k);
+  }
+
+  size_t max_splitk = 0, max_tiles = 0;
+  for (uint32_t i = 1; i < n; ++i) {
+    const paella_node_t& nd = d->nodes[i];
+    if (nd.op == PAELLA_OP_CONCAT) continue;
+    int32_t src = m->node_inputs[i][0];
+    const paella_node_t& sn = d->nodes[src];
+    const bool is_first = sn.op == PAELLA_OP_INPUT;
+    const uint32_t cin = is_first ? 8 : sn.c;   // channels the kernel reads
+    KernelInst k;
+    k.node = (int32_t)i;
+    k.in_buf = m->buf_of[src];
+    k.out_buf = (i == n - 1) ? -1 : m->buf_of[i];
+    LayerArgs& a = k.proto;
+    a.in_cs = cs_of(src);
+    a.in_co = m->coff[src];
+    if (k.out_buf >= 0) {
+      a.out_cs = cs_of(i);
+      a.out_co = m->coff[i];
+    }
+    a.cin = cin;
+    a.h = sn.h;
+    a.w_ = sn.w;
+    a.cout = nd.c;
+    a.oh = nd.h;
+    a.ow = nd.w;
+    a.kh = nd.kh;
+    a.kw = nd.kw;
+    a.sh = nd.sh;
+    a.sw = nd.sw;
+    a.ph = nd.ph;
+    a.pw = nd.pw;
+    a.groups = nd.groups ? nd.groups : 1;
+    a.act = nd.act;
+    a.ksplit = 1;
+    if (i == n - 1) a.flags |= LF_FINAL;
+    if (nd.flags & PAELLA_NODE_PROLOGUE) {
+      if (!nd.pro_scale || !nd.pro_shift) return -EINVAL;
+      a.flags |= LF_PROLOGUE;
+      k.has_pro = true;
+      k.ps_off = blob.put(nd.pro_scale, sn.c * 4);
+      k.pz_off = blob.put(nd.pro_shift, sn.c * 4);
+    }
+    if (nd.residual >= 0) {
+      if (nd.op != PAELLA_OP_CONV) return -EINVAL;
+      a.flags |= LF_RESIDUAL;
+      k.res_buf = m->buf_of[nd.residual];
+      a.res_cs = cs_of(nd.residual);
+      a.res_co = m->coff[nd.residual];
+    }
+    const uint32_t P_out = nd.h * nd.w;
+    switch (nd.op) {
+      case PAELLA_OP_CONV: {
+        const uint32_t g = a.groups;
+        const uint32_t cin_real = sn.c;
+        if (!nd.weight) return -EINVAL;
+        std::vector<float> bias(nd.c, 0.f);
+        if (nd.bias) std::memcpy(bias.data(), nd.bias, nd.c * 4);
+        k.b_off = blob.put(bias.data(), nd.c * 4);
+        if (g == 1) {
+          const uint32_t K = nd.kh * nd.kw * cin;
+          const uint32_t kpad = (uint32_t)align_up(K, 64);
+          a.kpad = kpad;
+          const bool use_tc_here = tc && (a.flags & LF_PROLOGUE) == 0;
+          const uint32_t rows = use_tc_here ? (uint32_t)align_up(nd.c, TC_BM) : nd.c;
+          // pack [rows][kpad], k = (r, s, ci)
+          std::vector<float> wp((size_t)rows * kpad, 0.f);
+          for (uint32_t co = 0; co < nd.c; ++co)
+            for (uint32_t r = 0; r < nd.kh; ++r)
+              for (uint32_t s = 0; s < nd.kw; ++s)
+                for (uint32_t ci = 0; ci < cin_real; ++ci)
+                  wp[(size_t)co * kpad + (r * nd.kw + s) * cin + ci] =
+                      nd.weight[(((size_t)co * cin_real + ci) * nd.kh + r) * nd.kw + s];
+          if (es == 2) {
+            std::vector<uint16_t> wb(wp.size());
+            for (size_t q = 0; q < wp.size(); ++q) wb[q] = f32_to_bf16_exact(wp[q], &exact);
+            k.w_off = blob.put(wb.data(), wb.size() * 2);
+            k.w_bytes = wb.size() * 2;
+          } else {
+            k.w_off = blob.put(wp.data(), wp.size() * 4);
+            k.w_bytes = wp.size() * 4;
+          }
+          if (use_tc_here) {
+            k.kind = KIND_CONV_TC;
+            a.tiles_m = rows / TC_BM;
+            a.tiles_n = (P_out + TC_BN - 1) / TC_BN;
+            uint32_t nk = kpad / TC_BK;
+            uint32_t tiles = a.tiles_m * a.tiles_n;
+            // split K so the grid approaches one wave of SMs, >= 2 k-blocks per split
+            uint32_t split = 1;
+            const char* e = std::getenv("PAELLA_NOSPLIT");
+            if (!e) {
+              while (tiles * split * 2 <= P->sms && nk / (split * 2) >= 2) split *= 2;
+            }
+            a.ksplit = split;
+            k.grid[0] = a.tiles_n;
+            k.grid[1] = a.tiles_m;
+            k.grid[2] = split;
+            k.block = TC_THREADS;
+            k.smem = tc_smem_bytes();
+            k.tmem_cols = tc_tmem_cols();
+            if (split > 1) {
+              max_splitk = std::max<size_t>(max_splitk, (size_t)split * tiles * TC_BM * TC_BN);
+              max_tiles = std::max<size_t>(max_tiles, tiles);
+            }
+          } else {
+            k.kind = KIND_CONV_SIMT;
+            k.grid[0] = (P_out + 63) / 64;
+            k.grid[1] = (nd.c + 63) / 64;
+            k.block = 256;
+          }
+          k.flops = 2ull * nd.c * P_out * nd.kh * nd.kw * cin_real;
+          k.bytes = (uint64_t)nd.c * nd.kh * nd.kw * cin_real * es + (uint64_t)sn.h * sn.w * cin_real * es +
+                    (uint64_t)P_out * nd.c * es * ((a.flags & LF_RESIDUAL) ? 2 : 1);
+        } else if (g == cin_real && g == nd.c) {
+          // depthwise: pack [kh][kw][c]
+          std::vector<float> wp((size_t)nd.kh * nd.kw * nd.c);
+          for (uint32_t c = 0; c < nd.c; ++c)
+            for (uint32_t r = 0; r < nd.kh; ++r)
+              for (uint32_t s = 0; s < nd.kw; ++s)
+                wp[((size_t)r * nd.kw + s) * nd.c + c] = nd.weight[((size_t)c * nd.kh + r) * nd.kw + s];
+          if (es == 2) {
+            std::vector<uint16_t> wb(wp.size());
+            for (size_t q = 0; q < wp.size(); ++q) wb[q] = f32_to_bf16_exact(wp[q], &exact);
+            k.w_off = blob.put(wb.data(), wb.size() * 2);
+          } else {
+            k.w_off = blob.put(wp.data(), wp.size() * 4);
+          }
+          k.kind = KIND_DWCONV;
+          k.grid[0] = (P_out * (nd.c / 8) + 255) / 256;
+          k.block = 256;
+          k.flops = 2ull * nd.c * P_out * nd.kh * nd.kw;
+          k.bytes = (uint64_t)nd.c * nd.kh * nd.kw * es + (uint64_t)sn.h * sn.w * nd.c * es +
+                    (uint64_t)P_out * nd.c * es * ((a.flags & LF_RESIDUAL) ? 2 : 1);
+        } else {
+          return -EINVAL;   // grouped conv other than depthwise: not in the model mix
+        }
+        break;
+      }
+      case PAELLA_OP_MAXPOOL:
+      case PAELLA_OP_AVGPOOL: {
+        k.kind = nd.op == PAELLA_OP_MAXPOOL ? KIND_MAXPOOL : KIND_AVGPOOL;
+        if (nd.flags & PAELLA_NODE_CEIL) a.flags |= LF_CEIL;
+        if (nd.c != sn.c) return -EINVAL;
+        k.grid[0] = (P_out * (nd.c / 8) + 255) / 256;
+        k.block = 256;
+        k.bytes = (uint64_t)sn.h * sn.w * sn.c * es + (uint64_t)P_out * nd.c * es;
+        break;
+      }
+      case PAELLA_OP_GAP: {
+        k.kind = KIND_GAP;
+        if (nd.c != sn.c || sn.c % 8) return -EINVAL;
+        k.grid[0] = (nd.c / 8 + 127) / 128;
+        k.block = 128;
+        k.bytes = (uint64_t)sn.h * sn.w * sn.c * es + (uint64_t)nd.c * ((a.flags & LF_FINAL) ? 4 : es);
+        break;
+      }
+      case PAELLA_OP_FC: {
+        k.kind = KIND_FC;
+        const uint32_t K = sn.c * sn.h * sn.w;
+        if (K % 8 || (sn.h * sn.w > 1 && a.in_cs != sn.c)) return -EINVAL;
+        if (!nd.weight) return -EINVAL;
+        a.cin = K;
+        a.kpad = K;
+        // torch flattens NCHW (c*HW + p); our activation is NHWC (p*C + c)
+        const uint32_t HW = sn.h * sn.w, C = sn.c;
+        std::vector<float> wp((size_t)nd.c * K);
+        for (uint32_t o = 0; o < nd.c; ++o)
+          for (uint32_t c = 0; c < C; ++c)
+            for (uint32_t p = 0; p < HW; ++p)
+              wp[(size_t)o * K + (size_t)p * C + c] = nd.weight[(size_t)o * K + (size_t)c * HW + p];
+        if (es == 2) {
+          std::vector<uint16_t> wb(wp.size());
+          for (size_t q = 0; q < wp.size(); ++q) wb[q] = f32_to_bf16_exact(wp[q], &exact);
+          k.w_off = blob.put(wb.data(), wb.size() * 2);
+        } else {
+          k.w_off = blob.put(wp.data(), wp.size() * 4);
+        }
+        std::vector<float> bias(nd.c, 0.f);
+        if (nd.bias) std::memcpy(bias.data(), nd.bias, nd.c * 4);
+        k.b_off = blob.put(bias.data(), nd.c * 4);
+        k.grid[0] = (nd.c + 7) / 8;
+        k.block = 256;
+        k.flops = 2ull * nd.c * K;
+        k.bytes = (uint64_t)nd.c * K * es + (uint64_t)K * es + (uint64_t)nd.c * ((a.flags & LF_FINAL) ? 4 : es);
+        break;
+      }
+      default:
+        return -EINVAL;
+    }
+    m->kernels.push_back(k);
+  }
+  if (!exact && es == 2) return -EINVAL;   // bf16 path requires bf16-representable weights
+  m->splitk_floats = max_splitk;
+  m->splitk_ctrs = max_tiles;
+  return 0;
+}
+
+}  // namespace paella

@@ -1,0 +1,175 @@
+// See policy.h.  Rule-for-rule the state machine of SURVEY.md §8(c) C2.
+#include "policy.h"
+
+#include <cassert>
+#include <climits>
+#include <stdexcept>
+
+namespace paella {
+
+Policy::Policy(const Cfg& c) : cfg_(c) {
+  launches_.resize(kLaunchSlots);
+  free_.assign((c.streams + 63) / 64, 0);
+  for (uint32_t s = 0; s < c.streams; ++s) free_[s / 64] |= 1ull << (s % 64);
+  Dt_.assign(c.num_clients, 0);
+  unfinished_.assign(c.num_clients, 0);
+  per_client_.resize(c.num_clients);
+  models_.resize(kMaxModels);   // never reallocated: models are added while dispatching
+}
+
+void Policy::add_model(uint32_t mid, const std::vector<PolicyLayer>& layers) {
+  if (mid >= kMaxModels) throw std::runtime_error("too many models");
+  models_[mid] = layers;
+}
+
+void Policy::make_ready(PolicyJob& j) {
+  srpt_.emplace(j.R, j.seq, j.id);
+  fifo_.emplace(j.seq, j.id);
+  per_client_[j.client].emplace(j.seq, j.id);
+}
+
+void Policy::make_unready(PolicyJob& j) {
+  srpt_.erase(std::make_tuple(j.R, j.seq, j.id));
+  fifo_.erase(std::make_pair(j.seq, j.id));
+  per_client_[j.client].erase(std::make_pair(j.seq, j.id));
+}
+
+void Policy::arrival(uint32_t job_id, uint32_t client, uint32_t model) {
+  if (unfinished_[client] == 0) Dt_[client] = -Omega_;   // C2-Q11: idle client restarts at 0
+  unfinished_[client] += 1;
+  if (jobs_.size() <= job_id) jobs_.resize(job_id + 1 + jobs_.size());
+  PolicyJob& j = jobs_[job_id];
+  j = PolicyJob();
+  j.id = job_id;
+  j.client = client;
+  j.model = model;
+  j.seq = next_seq_++;
+  int64_t R = 0;
+  for (const auto& l : models_[model]) R += l.tbar;
+  j.R = R;
+  j.live = true;
+  work_ += R;
+  live_jobs_ += 1;
+  make_ready(j);
+}
+
+bool Policy::record(uint32_t type, uint32_t uid, uint32_t n, int64_t* job_done) {
+  *job_done = -1;
+  PolicyLaunch& L = launches_[uid % kLaunchSlots];
+  if (!L.live || L.uid != uid) throw std::runtime_error("record for unknown launch");
+  O_ -= 1;
+  uint32_t old = L.p > L.f ? L.p : L.f;
+  const PolicyLayer& lay = models_[jobs_[L.job].model][L.layer];
+  if (type == 1) {
+    L.p += n;
+  } else if (type == 2) {
+    L.f += n;
+    for (int r = 0; r < NRES; ++r) U_[r] -= (int64_t)n * lay.demand[r];
+  } else {
+    throw std::runtime_error("bad record type");
+  }
+  uint32_t now = L.p > L.f ? L.p : L.f;
+  Q_ -= (int64_t)(now - old);
+  if (L.p > L.grid || L.f > L.grid) throw std::runtime_error("record count exceeds grid");
+  if (L.f != L.grid) return false;
+  L.live = false;
+  free_[L.stream / 64] |= 1ull << (L.stream % 64);
+  PolicyJob& j = jobs_[L.job];
+  j.inflight = false;
+  j.cursor += 1;
+  j.last_stream = (int32_t)L.stream;
+  if (j.cursor == models_[j.model].size()) {
+    j.live = false;
+    unfinished_[j.client] -= 1;
+    live_jobs_ -= 1;
+    *job_done = j.id;
+  } else {
+    make_ready(j);
+  }
+  return true;
+}
+
+int Policy::lowest_free() const {
+  for (size_t w = 0; w < free_.size(); ++w)
+    if (free_[w]) return (int)(w * 64 + __builtin_ctzll(free_[w]));
+  return -1;
+}
+
+bool Policy::pick(uint32_t* job_id) {
+  if (srpt_.empty()) return false;
+  if (cfg_.policy == POL_FIFO) {
+    *job_id = fifo_.begin()->second;
+    return true;
+  }
+  // c* = argmax (D_c, -c) over clients with a ready job
+  int cstar = -1;
+  int64_t best = 0;
+  for (uint32_t c = 0; c < cfg_.num_clients; ++c) {
+    if (per_client_[c].empty()) continue;
+    int64_t d = Dt_[c] + Omega_;
+    if (cstar < 0 || d > best) {
+      cstar = (int)c;
+      best = d;
+    }
+  }
+  bool over = false;
+  if (cfg_.theta != INT64_MAX) {
+    // theta * N without overflow: huge thresholds are never exceeded
+    if (cfg_.theta <= INT64_MAX / (int64_t)cfg_.num_clients)
+      over = best > cfg_.theta * (int64_t)cfg_.num_clients;
+  }
+  if (over) {
+    *job_id = per_client_[cstar].begin()->second;   // oldest ready job of c*
+  } else {
+    *job_id = std::get<2>(*srpt_.begin());           // SRPT: (R, seq, id)
+  }
+  return true;
+}
+
+bool Policy::predicate(uint32_t grid) const {
+  bool all_below = true;
+  for (int r = 0; r < NRES; ++r)
+    if (!(U_[r] < cfg_.capacity[r])) all_below = false;
+  bool fits = (Q_ < cfg_.slack) || all_below;
+  int64_t recs = 2 * (int64_t)((grid + cfg_.group - 1) / cfg_.group);
+  bool ring_ok = O_ + recs <= cfg_.ring_capacity;
+  return fits && ring_ok;
+}
+
+void Policy::decide(std::vector<Issue>* out) {
+  for (;;) {
+    int s0 = lowest_free();
+    if (s0 < 0) break;
+    uint32_t jid;
+    if (!pick(&jid)) break;
+    PolicyJob& j = jobs_[jid];
+    const PolicyLayer& lay = models_[j.model][j.cursor];
+    if (!predicate(lay.grid)) break;
+    uint32_t uid = next_uid_++;
+    uint32_t stream = (uint32_t)s0;
+    if (j.last_stream >= 0 && (free_[j.last_stream / 64] >> (j.last_stream % 64) & 1))
+      stream = (uint32_t)j.last_stream;
+    free_[stream / 64] &= ~(1ull << (stream % 64));
+    PolicyLaunch& L = launches_[uid % kLaunchSlots];
+    if (L.live) throw std::runtime_error("launch slot table overflow");
+    L.uid = uid;
+    L.job = jid;
+    L.layer = j.cursor;
+    L.grid = lay.grid;
+    L.stream = stream;
+    L.p = L.f = 0;
+    L.live = true;
+    for (int r = 0; r < NRES; ++r) U_[r] += (int64_t)lay.grid * lay.demand[r];
+    Q_ += lay.grid;
+    O_ += 2 * (int64_t)((lay.grid + cfg_.group - 1) / cfg_.group);
+    make_unready(j);
+    j.R -= lay.tbar;
+    work_ -= lay.tbar;
+    j.inflight = true;
+    Dt_[j.client] -= (int64_t)cfg_.num_clients;
+    Omega_ += 1;
+    out->push_back(Issue{uid, jid, L.layer, stream});
+  }
+}
+
+}  // namespace paella

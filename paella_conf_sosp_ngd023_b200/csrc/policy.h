@@ -1,0 +1,119 @@
+// The dispatcher's scheduling state machine (Paella §6, PAPER.md P1222-1323).
+//
+//   (1) SRPT: remaining = sum_{i in K} max(0, C_i - c_i) * T_i  (P1257-1261).  Our jobs
+//       are static kernel chains, so C_i is an exact count and R_j is the sum of the
+//       frozen T-bar of the kernels not yet dispatched (readings C2-Q8, C2-Q9).
+//   (2) Deficit fairness (P1287-1298): the scheduled client's deficit drops by
+//       (1 - 1/N), every other client's rises by 1/N; if a client's deficit exceeds
+//       theta, the oldest ready job of the highest-deficit client is chosen.  Kept in
+//       integer units of 1/N with a global offset Omega -- the paper's O(1)
+//       threshold-shift trick (P1316-1323) without its floating-point underflow.
+//   (3) Slack B beyond full utilisation (P1300-1304) and the dispatch loop
+//       (P1306-1314): issue while (unplaced blocks Q < B) or (every resource U_r <
+//       C_r), and while the notification ring has room for the launch's records
+//       (flow control, P1115-1119).
+//
+// Exactly the rules of oracle/sim.py::Policy; the replay test
+// checks the issue sequence bit for bit.  Data structures are the fast ones
+// (ordered sets instead of linear scans), the decisions are identical.
+#pragma once
+#include <cstdint>
+#include <set>
+#include <tuple>
+#include <vector>
+
+namespace paella {
+
+constexpr int NRES = 5;   // blocks, warps, regs, smem, tmem (Table 1 + TMEM)
+
+struct PolicyLayer {
+  uint32_t grid;
+  int64_t demand[NRES];
+  int64_t tbar;
+};
+
+struct PolicyJob {
+  uint32_t id = 0;
+  uint32_t client = 0, model = 0;
+  uint64_t seq = 0;
+  int64_t R = 0;
+  uint32_t cursor = 0;
+  bool inflight = false;
+  bool live = false;
+  int32_t last_stream = -1;
+};
+
+struct PolicyLaunch {
+  uint32_t uid = 0, job = 0, layer = 0, grid = 0, stream = 0;
+  uint32_t p = 0, f = 0;
+  bool live = false;
+};
+
+struct Issue {
+  uint32_t uid, job, layer, stream;
+};
+
+enum : uint32_t { POL_SRPT_DEFICIT = 0, POL_FIFO = 1 };
+
+class Policy {
+ public:
+  struct Cfg {
+    uint32_t num_clients = 1, policy = POL_SRPT_DEFICIT;
+    int64_t theta = 100;
+    int64_t slack = 148;
+    uint32_t group = 16;
+    int64_t ring_capacity = 65536;
+    uint32_t streams = 32;
+    int64_t capacity[NRES] = {148 * 32, 148 * 64, 148 * 65536, 148 * 233472, 148 * 512};
+  };
+
+  explicit Policy(const Cfg& c);
+
+  void add_model(uint32_t mid, const std::vector<PolicyLayer>& layers);
+  const std::vector<PolicyLayer>& model(uint32_t m) const { return models_[m]; }
+
+  // job ids are dense, assigned by the caller in admission order
+  void arrival(uint32_t job_id, uint32_t client, uint32_t model);
+  // returns true if the launch finished; *job_done set if its job completed
+  bool record(uint32_t type, uint32_t uid, uint32_t n, int64_t* job_done);
+  // dispatch loop; appends issues
+  void decide(std::vector<Issue>* out);
+
+  int64_t outstanding_work() const { return work_; }
+  uint64_t live_jobs() const { return live_jobs_; }
+  const PolicyJob& job(uint32_t id) const { return jobs_[id]; }
+  const PolicyLaunch& launch(uint32_t uid) const { return launches_[uid % kLaunchSlots]; }
+  int64_t deficit(uint32_t c) const { return Dt_[c] + Omega_; }
+  int64_t Q() const { return Q_; }
+  int64_t O() const { return O_; }
+
+ private:
+  static constexpr uint32_t kLaunchSlots = 8192;
+  static constexpr uint32_t kMaxModels = 256;
+  bool pick(uint32_t* job_id);
+  bool predicate(uint32_t grid) const;
+  void make_ready(PolicyJob& j);
+  void make_unready(PolicyJob& j);
+  int lowest_free() const;
+
+  Cfg cfg_;
+  std::vector<std::vector<PolicyLayer>> models_;
+  std::vector<PolicyJob> jobs_;
+  std::vector<PolicyLaunch> launches_;
+  int64_t U_[NRES] = {0, 0, 0, 0, 0};
+  int64_t Q_ = 0, O_ = 0;
+  std::vector<uint64_t> free_;   // bitmap of free streams
+  std::vector<int64_t> Dt_;
+  int64_t Omega_ = 0;
+  std::vector<uint32_t> unfinished_;
+  uint32_t next_uid_ = 0;
+  uint64_t next_seq_ = 0;
+  int64_t work_ = 0;             // sum of R over live jobs (router's W_g)
+  uint64_t live_jobs_ = 0;
+  // ready structures
+  std::set<std::tuple<int64_t, uint64_t, uint32_t>> srpt_;     // (R, seq, id)
+  std::set<std::pair<uint64_t, uint32_t>> fifo_;               // (seq, id)
+  std::vector<std::set<std::pair<uint64_t, uint32_t>>> per_client_;  // (seq, id)
+};
+
+}  // namespace paella

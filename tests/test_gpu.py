@@ -1,0 +1,175 @@
+"""GPU parity tests (need a B200 and the built libpaella.so; run with -m gpu).
+
+* kernels: every model of the mix, run isolated through the C ABI, vs the float64
+  oracle (oracle/infer.py) -- bf16 path within max-abs 2e-2 / rel 1e-2, fp32 path
+  within 1e-4 (BASELINE.json north_star tolerances, reading C1-Q6: atol + rtol|ref|);
+* serving: mixed concurrent requests through paella_submit / poll_completion on the
+  real dispatcher; every output checked against the oracle; the GPU event log
+  replayed through the oracle policy reproduces the issue order bit-exactly (S6);
+  every launch's notification records tile its grid exactly once (S5 b);
+* the naive baseline path produces the same outputs;
+* ring wrap-around (small ring, many laps), G = 1, a single stream.
+"""
+import time
+
+import numpy as np
+import pytest
+
+from oracle import eventlog, infer, sim
+from workload import archs, rng
+
+pytestmark = pytest.mark.gpu
+
+L = pytest.importorskip("paella_conf_sosp_ngd023_b200._lib")
+
+BF16_TOL = (2e-2, 1e-2)
+FP32_TOL = (1e-4, 1e-4)
+_ORACLE = {}
+
+
+def oracle_out(name, i, dtype):
+    key = (name, i, dtype)
+    if key not in _ORACLE:
+        g = archs.build(name)
+        _ORACLE[key] = infer.forward(g, rng.model_params(g), rng.image(g, i), dtype=dtype)
+    return _ORACLE[key]
+
+
+def within(out, ref, tol):
+    atol, rtol = tol
+    return np.abs(out - ref) <= atol + rtol * np.abs(ref)
+
+
+@pytest.fixture(scope="module")
+def engine():
+    from paella_conf_sosp_ngd023_b200 import build
+    build.build()
+    e = L.Engine(num_clients=1)
+    yield e
+    e.shutdown()
+
+
+MODELS = ["toy", "resnet18", "mobilenet_v2", "squeezenet1_1", "resnet50", "densenet121", "inception_v3"]
+
+
+@pytest.mark.parametrize("name", MODELS)
+def test_isolated_bf16_parity(engine, name):
+    g = archs.build(name)
+    mid = engine.register_model(g, rng.model_params(g), dtype=L.DTYPE_BF16, name=name + "-iso")
+    for i in (0, 1):
+        out = engine.run_isolated(mid, rng.image(g, i))
+        ref = oracle_out(name, i, "bf16")
+        ok = within(out, ref, BF16_TOL)
+        assert ok.all(), f"{name} input {i}: {np.sum(~ok)} logits out of tolerance, max err {np.abs(out-ref).max()}"
+
+
+@pytest.mark.parametrize("name", ["toy", "resnet18", "mobilenet_v2", "squeezenet1_1", "densenet121"])
+def test_isolated_fp32_parity(engine, name):
+    g = archs.build(name)
+    mid = engine.register_model(g, rng.model_params(g), dtype=L.DTYPE_FP32, name=name + "-f32")
+    out = engine.run_isolated(mid, rng.image(g, 0))
+    ref = oracle_out(name, 0, "fp32")
+    assert within(out, ref, FP32_TOL).all(), np.abs(out - ref).max()
+
+
+def _serve_and_check(e, specs, n, n_clients, seed, rate_us=30.0):
+    """specs: list of (model id, model name, graph).  Submits n requests with Poisson
+    gaps, distinct pooled inputs, checks all outputs against the oracle."""
+    r = np.random.default_rng(seed)
+    infos = {mid: e.model_info(mid) for mid, _, _ in specs}
+    stride = max(i["input_bytes"] + i["output_bytes"] for i in infos.values())
+    stride = (stride + 4095) // 4096 * 4096
+    slots = 64
+    free = {c: list(range(slots)) for c in range(n_clients)}
+    pending = {}
+    done = 0
+    sent = 0
+    t0 = time.time()
+    while done < n:
+        assert time.time() - t0 < 120, f"timeout: {done}/{n} completed"
+        if sent < n:
+            c = int(r.integers(n_clients))
+            if free[c]:
+                mid, name, g = specs[int(r.integers(len(specs)))]
+                slot = free[c].pop()
+                off = slot * stride
+                idx = int(r.integers(4))
+                x = rng.image(g, idx)
+                _, reg = e.region(c)
+                reg[off:off + x.nbytes] = np.frombuffer(x.tobytes(), np.uint8)
+                rid = e.submit(c, mid, off, infos[mid]["input_bytes"] + infos[mid]["output_bytes"])
+                assert rid >= 0
+                pending[rid] = (c, slot, off, mid, name, idx)
+                sent += 1
+                time.sleep(r.exponential(rate_us) * 1e-6)
+        for c in range(n_clients):
+            while True:
+                rid, st = e.poll(c)
+                if rid < 0:
+                    break
+                assert st == 0
+                c2, slot, off, mid, name, idx = pending.pop(rid)
+                _, reg = e.region(c2)
+                ib = infos[mid]["input_bytes"]
+                out = np.frombuffer(reg[off + ib:off + ib + infos[mid]["output_bytes"]].tobytes(), np.float32)
+                ref = oracle_out(name, idx, "bf16")
+                assert within(out, ref, BF16_TOL).all(), (name, np.abs(out - ref).max())
+                free[c2].append(slot)
+                done += 1
+
+
+@pytest.mark.parametrize("policy,group,streams,ring", [
+    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536),
+    (L.POLICY_FIFO, 16, 32, 65536),
+    (L.POLICY_SRPT_DEFICIT, 1, 8, 256),      # G = 1 debug mode, ring wraps many laps
+    (L.POLICY_SRPT_DEFICIT, 16, 1, 1024),    # a single stream
+])
+def test_serving_parity_and_replay(tmp_path, policy, group, streams, ring):
+    log = str(tmp_path / "gpu_%u.log")
+    names = ["toy", "resnet18", "mobilenet_v2", "squeezenet1_1"]
+    with L.Engine(num_clients=3, policy=policy, group=group, streams=streams, ring_capacity=ring,
+                  event_log=log, max_jobs_per_model=32) as e:
+        specs = []
+        for nm in names:
+            g = archs.build(nm)
+            specs.append((e.register_model(g, rng.model_params(g)), nm, g))
+        _serve_and_check(e, specs, 120, 3, seed=policy * 7 + group)
+        st = e.stats()
+        assert st["completed"] == 120
+    cfg, ms, events, ex = eventlog.read(log % 0)
+    ok, msg, n = sim.replay(cfg, ms, events)
+    assert ok, msg
+    assert n == len(ex["issues"]) == st["launches"]
+    grids = {uid: ms[model][layer].grid for (uid, job, layer, stream, model) in ex["issues"]}
+    assert sim.check_exactly_once(ex["records"], grids, cfg.group) == []
+
+
+def test_naive_baseline_outputs():
+    names = ["toy", "squeezenet1_1"]
+    with L.Engine(num_clients=2, naive=True, instrument=False) as e:
+        specs = []
+        for nm in names:
+            g = archs.build(nm)
+            specs.append((e.register_model(g, rng.model_params(g)), nm, g))
+        _serve_and_check(e, specs, 60, 2, seed=3)
+
+
+def test_ring_records_carry_sm_and_time(tmp_path):
+    """G=1: one PLACEMENT and one COMPLETION per block, SM ids < 148, completion time
+    of a block's group never before the first placement of its launch."""
+    log = str(tmp_path / "g1_%u.log")
+    g = archs.toy()
+    with L.Engine(num_clients=1, group=1, event_log=log) as e:
+        mid = e.register_model(g, rng.model_params(g))
+        _serve_and_check(e, [(mid, "toy", g)], 10, 1, seed=1)
+    cfg, ms, events, ex = eventlog.read(log % 0)
+    recs = ex["records"]
+    assert all(r[3] == 1 for r in recs)
+    assert all(r[5] < 148 for r in recs)
+    first_place = {}
+    for (t, typ, uid, n, grp, sm) in recs:
+        if typ == sim.PLACEMENT:
+            first_place[uid] = min(first_place.get(uid, t), t)
+    for (t, typ, uid, n, grp, sm) in recs:
+        if typ == sim.COMPLETION:
+            assert (t - first_place[uid]) % (1 << 40) < (1 << 39)

@@ -1,0 +1,171 @@
+"""CPU tests of the C-ABI library (no GPU): exported symbols, argument checking,
+and the dispatcher / router / replay path driven by the FAKE device backend (a CPU
+model of a GPU that synthesises notification records in the same ring format).
+
+Replay parity (pin S6): the C++ dispatcher's event log, replayed
+through the oracle policy (oracle/sim.py), reproduces its issue sequence bit for bit.
+"""
+import errno
+import os
+import re
+import subprocess
+import time
+
+import numpy as np
+import pytest
+
+from oracle import eventlog, sim
+from workload import archs, rng
+
+L = pytest.importorskip("paella_conf_sosp_ngd023_b200._lib")
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module", autouse=True)
+def built():
+    from paella_conf_sosp_ngd023_b200 import build
+    build.build()
+    L.load()
+
+
+def test_exports_every_declared_symbol():
+    hdr = open(os.path.join(ROOT, "include", "paella.h")).read()
+    declared = set(re.findall(r"^\s*(?:int|int64_t|const char\*)\s+(paella_\w+)\s*\(", hdr, re.M))
+    assert declared == set(L.SYMBOLS), declared ^ set(L.SYMBOLS)
+    out = subprocess.run(["nm", "-D", "--defined-only", L.LIB_PATH], capture_output=True, text=True).stdout
+    exported = set(re.findall(r" T (paella_\w+)", out))
+    assert declared <= exported, declared - exported
+    lib = L.load()
+    for s in declared:
+        assert hasattr(lib, s)
+
+
+def _toy_engine(**kw):
+    kw.setdefault("device", L.DEVICE_FAKE)
+    kw.setdefault("fake_sms", 4)
+    return L.Engine(**kw)
+
+
+def test_init_rejects_bad_config():
+    with pytest.raises(OSError) as ei:
+        L.Engine(num_clients=0, device=L.DEVICE_FAKE)
+    assert ei.value.errno == errno.EINVAL
+    with pytest.raises(OSError):
+        L.Engine(num_clients=1, device=L.DEVICE_FAKE, ring_capacity=1000)   # not a power of two
+    with pytest.raises(OSError):
+        L.Engine(num_clients=1, device=L.DEVICE_FAKE, group=17)
+
+
+def test_submit_argument_errors_and_eagain():
+    g = archs.toy()
+    P = rng.model_params(g)
+    with _toy_engine(num_clients=2) as e:
+        mid = e.register_model(g, P)
+        with pytest.raises(OSError) as ei:
+            e.register_model(g, P)
+        assert ei.value.errno == errno.EEXIST
+        info = e.model_info(mid)
+        need = info["input_bytes"] + info["output_bytes"]
+        base, reg = e.region(0)
+        lib = e.lib
+        # outside the client's region -> EFAULT (P1060-1061)
+        assert lib.paella_submit(e.h, 0, mid, base + len(reg) - 16, need, 0) == -errno.EFAULT
+        base1, _ = e.region(1)
+        assert lib.paella_submit(e.h, 0, mid, base1, need, 0) == -errno.EFAULT
+        assert lib.paella_submit(e.h, 0, mid, base, need - 1, 0) == -errno.EINVAL
+        assert lib.paella_submit(e.h, 0, 7, base, need, 0) == -errno.EINVAL
+        assert lib.paella_submit(e.h, 5, mid, base, need, 0) == -errno.EINVAL
+        rid, st = e.poll(0, L.NONBLOCK)
+        assert rid == -errno.EAGAIN    # readResult NONBLOCK (P1150-1155)
+
+
+def _serve(e, mids, n, n_clients, seed, stride=16384, timeout=60):
+    r = np.random.default_rng(seed)
+    infos = {m: e.model_info(m) for m in mids}
+    out = {}
+    pending = set()
+    for i in range(n):
+        c = int(r.integers(n_clients))
+        m = int(r.choice(mids))
+        need = infos[m]["input_bytes"] + infos[m]["output_bytes"]
+        off = (i % 512) * stride
+        rid = e.submit(c, m, off, need)
+        assert rid >= 0, rid
+        assert rid >> 48 == c
+        pending.add(rid)
+        if r.random() < 0.3:
+            time.sleep(0.0002)
+    t0 = time.time()
+    while pending:
+        assert time.time() - t0 < timeout, f"{len(pending)} requests never completed"
+        for c in range(n_clients):
+            rid, st = e.poll(c)
+            if rid >= 0:
+                assert st == 0
+                pending.remove(rid)
+                out[rid] = st
+    return out
+
+
+@pytest.mark.parametrize("policy,theta,group,streams", [
+    (L.POLICY_SRPT_DEFICIT, 100, 16, 8), (L.POLICY_SRPT_DEFICIT, 0, 1, 4),
+    (L.POLICY_SRPT_DEFICIT, None, 4, 32), (L.POLICY_FIFO, 100, 16, 8), (L.POLICY_SRPT_DEFICIT, 3, 16, 2)])
+def test_fake_device_replay_parity(tmp_path, policy, theta, group, streams):
+    log = str(tmp_path / "ev_%u.log")
+    models = [archs.toy(), archs.squeezenet1_1()]
+    with _toy_engine(num_clients=3, policy=policy, theta=theta, group=group, streams=streams,
+                     event_log=log, ring_capacity=1024, slack=8) as e:
+        mids = [e.register_model(g, rng.model_params(g)) for g in models]
+        _serve(e, mids, 300, 3, seed=policy * 10 + group)
+    cfg, ms, events, ex = eventlog.read(log % 0)
+    assert cfg.num_clients == 3 and cfg.policy == policy and cfg.group == group
+    ok, msg, n = sim.replay(cfg, ms, events)
+    assert ok, msg
+    assert n == len(ex["issues"]) > 0 and ex["n_arrivals"] == 300 == len(ex["completes"])
+    # S5 (b) exactly-once coverage of every launch's records
+    grids = {uid: ms[model][layer].grid for (uid, job, layer, stream, model) in ex["issues"]}
+    assert sim.check_exactly_once(ex["records"], grids, cfg.group) == []
+
+
+def test_fake_replay_with_job_id_reuse(tmp_path):
+    """Long run (job ids are recycled) still replays exactly."""
+    log = str(tmp_path / "ev_%u.log")
+    g = archs.toy()
+    with _toy_engine(num_clients=2, event_log=log, max_jobs_per_model=8, streams=4) as e:
+        mid = e.register_model(g, rng.model_params(g))
+        _serve(e, [mid], 600, 2, seed=5)
+        st = e.stats()
+        assert st["completed"] == 600 and st["launches"] == 600 * 5
+    cfg, ms, events, ex = eventlog.read(log % 0)
+    ok, msg, n = sim.replay(cfg, ms, events)
+    assert ok and n == 3000, msg
+
+
+@pytest.mark.parametrize("route", [L.ROUTE_LEAST_WORK, L.ROUTE_ROUND_ROBIN])
+def test_router_multi_gpu_fake(tmp_path, route):
+    log = str(tmp_path / "ev_%u.log")
+    g = archs.toy()
+    with _toy_engine(num_clients=2, num_gpus=4, route=route, event_log=log) as e:
+        mid = e.register_model(g, rng.model_params(g))
+        _serve(e, [mid], 400, 2, seed=11)
+        per = [e.stats(i)["completed"] for i in range(4)]
+    assert sum(per) == 400
+    if route == L.ROUTE_ROUND_ROBIN:
+        assert max(per) - min(per) <= 2 and min(per) > 0
+    else:   # least outstanding work, ties to the lowest index: a burst spreads out
+        assert sum(1 for x in per if x > 0) >= 2
+    for gi in range(4):   # every per-GPU dispatcher replays exactly
+        cfg, ms, events, ex = eventlog.read(log % gi)
+        ok, msg, n = sim.replay(cfg, ms, events)
+        assert ok, (gi, msg)
+
+
+def test_shutdown_cancels_unadmitted():
+    g = archs.toy()
+    e = _toy_engine(num_clients=1, max_jobs_per_model=1, fake_time_scale_ns=1)
+    mid = e.register_model(g, rng.model_params(g))
+    info = e.model_info(mid)
+    need = info["input_bytes"] + info["output_bytes"]
+    for i in range(50):
+        assert e.submit(0, mid, i * 16384, need) >= 0
+    e.shutdown()
