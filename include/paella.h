@@ -98,6 +98,9 @@ typedef struct {
                                     index), or NULL */
   uint32_t fake_sms;             /* FAKE device: SM count (0 = 148) */
   uint32_t fake_time_scale_ns;   /* FAKE device: virtual ns per poll iteration (0 = 500) */
+  uint32_t event_time_kind;      /* 0 = off; k+1 = the dispatcher brackets every launch of
+                                    kernel kind k with CUDA events on its stream and sums
+                                    the durations (paella_stats ev_*): the live roofline */
 } paella_config_t;
 
 /* ---- model description (input to paella_register_model) ---------------- */
@@ -208,6 +211,7 @@ typedef struct {
   uint64_t admitted, completed, launches, records, torn_retries, decide_calls;
   uint64_t loop_iters;
   int64_t  outstanding_work_ns;   /* W_g published for the router */
+  uint64_t ev_launches, ev_ns, ev_bytes, ev_flops;   /* event-timed launches (event_time_kind) */
 } paella_stats_t;
 
 int paella_stats(paella_t* p, uint32_t gpu, paella_stats_t* st);
@@ -222,6 +226,44 @@ int paella_flush_log(paella_t* p);
    n_kernels per-kernel device times (CUDA events).  Returns 0 or -errno. */
 int paella_run_isolated(paella_t* p, uint32_t gpu, uint32_t model_id, const void* input,
                         void* output, int64_t* kernel_ns);
+
+/* Device-only kernel timing (the "summed isolated kernel time" roofline of the north
+   star, and instrumentation overhead, config 5): kernel k of the model's chain is
+   launched `reps` times back to back behind a gate on an otherwise idle GPU
+   (instrumented if `instrumented`, else the uninstrumented twin); kernel_ns[k] =
+   elapsed / reps.  Returns 0 or -errno. */
+int paella_time_kernels(paella_t* p, uint32_t gpu, uint32_t model_id, uint32_t instrumented,
+                        uint32_t reps, int64_t* kernel_ns);
+
+/* Notification microbenchmarks (config 5, P1881-1897 Fig. 15).
+   paella_bench_empty: `iters` launches of an empty kernel with `grid` x `block`
+   threads, back to back behind a gate; *ns_per_launch = elapsed / iters.
+   paella_bench_roundtrip: `n` times, launch a 1-block instrumented empty kernel and
+   spin on the ring until its PLACEMENT / COMPLETION records are visible to the host;
+   place_ns[i] / complete_ns[i] = host time from before the launch call.  Both run
+   on the isolated ring, outside the dispatcher. */
+int paella_bench_empty(paella_t* p, uint32_t gpu, uint32_t grid, uint32_t block, uint32_t instrumented,
+                       uint32_t group, uint32_t iters, double* ns_per_launch);
+int paella_bench_roundtrip(paella_t* p, uint32_t gpu, uint32_t n, int64_t* place_ns, int64_t* complete_ns);
+
+/* ---- open-loop load generator (benchmark harness; same front end for every system) ----
+   Replays requests at their scheduled times from the calling thread: request i of
+   client c uses io slot (i-th free slot of c) at offset slot*stride in c's region;
+   a request waits for a free slot (that wait counts in its JCT).  With copy_inputs
+   != NULL (end-to-end mode) the client copies the request's input from
+   copy_inputs[model][input_idx] into its slot right before submitting and copies the
+   logits out after completion (the host<->device traffic of the step); otherwise the
+   slots must hold the inputs already.  jct_ns[i] = completion seen by the client -
+   t_sched (scheduled arrival; no coordinated omission).  t0_ns = the monotonic time
+   that request times are relative to (0 = now).  Returns completed count or -errno. */
+typedef struct {
+  int64_t t_ns;        /* scheduled arrival, relative to t0 */
+  uint32_t client, model, input_idx, pad;
+} paella_req_t;
+
+int64_t paella_loadgen(paella_t* p, const paella_req_t* reqs, uint32_t n, size_t stride,
+                       uint32_t slots_per_client, const void* const* const* copy_inputs,
+                       int64_t t0_ns, int64_t* jct_ns, int64_t* elapsed_ns);
 
 /* Debug: copy node `node`'s activation of the last isolated run to host as fp32
    NCHW (C*H*W floats).  Returns 0 or -errno. */

@@ -31,7 +31,8 @@ INT64_MAX = (1 << 63) - 1
 SYMBOLS = ["paella_init", "paella_register_model", "paella_submit", "paella_submit_at",
            "paella_poll_completion", "paella_shutdown", "paella_client_region", "paella_model_info",
            "paella_kernel_info", "paella_kernel_name", "paella_stats", "paella_flush_log",
-           "paella_run_isolated", "paella_debug_node"]
+           "paella_run_isolated", "paella_debug_node", "paella_time_kernels", "paella_bench_empty",
+           "paella_bench_roundtrip", "paella_loadgen"]
 
 
 class Config(C.Structure):
@@ -42,7 +43,7 @@ class Config(C.Structure):
                 ("submit_slots", C.c_uint32), ("max_jobs_per_model", C.c_uint32), ("instrument", C.c_uint32),
                 ("naive", C.c_uint32), ("client_region_bytes", C.c_size_t),
                 ("dispatcher_cpus", C.POINTER(C.c_int32)), ("event_log_path", C.c_char_p),
-                ("fake_sms", C.c_uint32), ("fake_time_scale_ns", C.c_uint32)]
+                ("fake_sms", C.c_uint32), ("fake_time_scale_ns", C.c_uint32), ("event_time_kind", C.c_uint32)]
 
 
 class Node(C.Structure):
@@ -71,10 +72,16 @@ class KernelInfo(C.Structure):
                 ("flops", C.c_uint64), ("bytes", C.c_uint64)]
 
 
+class Req(C.Structure):
+    _fields_ = [("t_ns", C.c_int64), ("client", C.c_uint32), ("model", C.c_uint32),
+                ("input_idx", C.c_uint32), ("pad", C.c_uint32)]
+
+
 class Stats(C.Structure):
     _fields_ = [("admitted", C.c_uint64), ("completed", C.c_uint64), ("launches", C.c_uint64),
                 ("records", C.c_uint64), ("torn_retries", C.c_uint64), ("decide_calls", C.c_uint64),
-                ("loop_iters", C.c_uint64), ("outstanding_work_ns", C.c_int64)]
+                ("loop_iters", C.c_uint64), ("outstanding_work_ns", C.c_int64), ("ev_launches", C.c_uint64),
+                ("ev_ns", C.c_uint64), ("ev_bytes", C.c_uint64), ("ev_flops", C.c_uint64)]
 
 
 _lib = None
@@ -108,6 +115,13 @@ def load():
     lib.paella_flush_log.argtypes = [P]
     lib.paella_run_isolated.argtypes = [P, C.c_uint32, C.c_uint32, P, P, C.POINTER(C.c_int64)]
     lib.paella_debug_node.argtypes = [P, C.c_uint32, C.c_uint32, C.c_uint32, C.POINTER(C.c_float)]
+    lib.paella_time_kernels.argtypes = [P, C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32, C.POINTER(C.c_int64)]
+    lib.paella_bench_empty.argtypes = [P, C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32, C.c_uint32,
+                                       C.POINTER(C.c_double)]
+    lib.paella_bench_roundtrip.argtypes = [P, C.c_uint32, C.c_uint32, C.POINTER(C.c_int64), C.POINTER(C.c_int64)]
+    lib.paella_loadgen.argtypes = [P, C.POINTER(Req), C.c_uint32, C.c_size_t, C.c_uint32, P, C.c_int64,
+                                   C.POINTER(C.c_int64), C.POINTER(C.c_int64)]
+    lib.paella_loadgen.restype = C.c_int64
     _lib = lib
     return lib
 
@@ -129,7 +143,7 @@ class Engine:
                  policy=POLICY_SRPT_DEFICIT, theta=100, slack=0, group=16, ring_capacity=65536,
                  streams=32, route=ROUTE_LEAST_WORK, submit_slots=1024, max_jobs_per_model=128,
                  instrument=True, naive=False, region_bytes=64 << 20, dispatcher_cpus=None,
-                 event_log=None, fake_sms=0, fake_time_scale_ns=0):
+                 event_log=None, fake_sms=0, fake_time_scale_ns=0, event_time_kind=None):
         self.lib = load()
         cfg = Config()
         cfg.abi_version = ABI_VERSION
@@ -157,6 +171,7 @@ class Engine:
         cfg.event_log_path = self._log
         cfg.fake_sms = fake_sms
         cfg.fake_time_scale_ns = fake_time_scale_ns
+        cfg.event_time_kind = 0 if event_time_kind is None else event_time_kind + 1
         self.cfg = cfg
         h = C.c_void_p()
         _check(self.lib.paella_init(C.byref(cfg), C.byref(h)), "paella_init")
@@ -269,6 +284,55 @@ class Engine:
         out = np.zeros(int(np.prod(shape)), dtype=np.float32)
         _check(self.lib.paella_debug_node(self.h, gpu, model, node, _fptr(out)), "paella_debug_node")
         return out.reshape(shape)
+
+    def time_kernels(self, model, instrumented=True, reps=50, gpu=0):
+        n = self.model_info(model)["n_kernels"]
+        kt = np.zeros(n, dtype=np.int64)
+        _check(self.lib.paella_time_kernels(self.h, gpu, model, 1 if instrumented else 0, reps,
+                                            kt.ctypes.data_as(C.POINTER(C.c_int64))), "paella_time_kernels")
+        return kt
+
+    def bench_empty(self, grid, block=128, instrumented=True, group=16, iters=2000, gpu=0):
+        v = C.c_double()
+        _check(self.lib.paella_bench_empty(self.h, gpu, grid, block, 1 if instrumented else 0, group, iters,
+                                           C.byref(v)), "paella_bench_empty")
+        return v.value
+
+    def bench_roundtrip(self, n=1000, gpu=0):
+        a = np.zeros(n, dtype=np.int64)
+        b = np.zeros(n, dtype=np.int64)
+        _check(self.lib.paella_bench_roundtrip(self.h, gpu, n, a.ctypes.data_as(C.POINTER(C.c_int64)),
+                                               b.ctypes.data_as(C.POINTER(C.c_int64))), "paella_bench_roundtrip")
+        return a, b
+
+    def loadgen(self, t_ns, clients, models, inputs, stride, slots, copy_inputs=None, t0_ns=0):
+        """Open-loop replay of a trace from the calling thread (GIL released).
+        copy_inputs: None (inputs pre-staged in the slots) or {model: [np arrays]}.
+        Returns (jct_ns array, elapsed_ns)."""
+        n = len(t_ns)
+        reqs = (Req * n)()
+        for i in range(n):
+            reqs[i].t_ns = int(t_ns[i])
+            reqs[i].client = int(clients[i])
+            reqs[i].model = int(models[i])
+            reqs[i].input_idx = int(inputs[i])
+        jct = np.zeros(n, dtype=np.int64)
+        el = C.c_int64()
+        cp = None
+        if copy_inputs is not None:
+            nm = max(copy_inputs) + 1
+            rows = (C.c_void_p * nm)()
+            self._cp_keep = []
+            for m, arrs in copy_inputs.items():
+                ptrs = (C.c_void_p * len(arrs))(*[a.ctypes.data for a in arrs])
+                self._cp_keep.append((ptrs, arrs))
+                rows[m] = C.cast(ptrs, C.c_void_p)
+            cp = rows
+            self._cp_keep.append(rows)
+        rc = self.lib.paella_loadgen(self.h, reqs, n, stride, slots, C.cast(cp, C.c_void_p) if cp else None,
+                                     t0_ns, jct.ctypes.data_as(C.POINTER(C.c_int64)), C.byref(el))
+        _check(rc, "paella_loadgen")
+        return jct, el.value
 
     def stats(self, gpu=0):
         st = Stats()

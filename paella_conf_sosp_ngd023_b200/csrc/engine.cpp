@@ -159,6 +159,26 @@ struct FakeBackend : Backend {
 // ---------------------------------------------------------------------------
 // CUDA backend
 // ---------------------------------------------------------------------------
+// one launch of kernel k: split-K tcgen05 convs are thread-block clusters
+static cudaError_t cuda_launch(KernelFn fn, const KernelInst& k, void** args, cudaStream_t s) {
+  if (k.kind == KIND_CONV_TC && k.proto.ksplit > 1) {
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(k.grid[0], k.grid[1], k.grid[2]);
+    cfg.blockDim = dim3(k.block);
+    cfg.dynamicSmemBytes = k.smem;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 1;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = k.proto.ksplit;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelExC(&cfg, (const void*)fn, args);
+  }
+  return cudaLaunchKernel((const void*)fn, dim3(k.grid[0], k.grid[1], k.grid[2]), dim3(k.block), args, k.smem, s);
+}
+
 struct CudaBackend : Backend {
   int dev;
   uint32_t cap, nstreams;
@@ -208,8 +228,7 @@ struct CudaBackend : Backend {
   void launch(const KernelInst& k, const LayerArgs& a, const InstrArgs& ia, uint32_t stream, uint32_t dtype,
               bool instr) override {
     void* args[3] = {(void*)&a, (void*)&ia, (void*)k_tmap(k)};
-    cudaError_t e = cudaLaunchKernel((const void*)fn(k.kind, dtype, instr), dim3(k.grid[0], k.grid[1], k.grid[2]),
-                                     dim3(k.block), args, k.smem, streams[stream]);
+    cudaError_t e = cuda_launch(fn(k.kind, dtype, instr), k, args, streams[stream]);
     if (e != cudaSuccess && !err_) err_ = (int)e;
   }
   // the tensor map of a tcgen05 conv is stored right after its KernelInst's proto
@@ -259,11 +278,45 @@ static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last) {
 static void do_launch(Gpu* g, Model* m, uint32_t slot, uint32_t layer, uint32_t uid, uint32_t stream, bool instr) {
   const KernelInst& k = m->kernels[layer];
   InstrArgs ia = make_instr(g, uid, k.grid_total(), layer + 1 == m->kernels.size());
-  if (g->P->cfg.device == PAELLA_DEVICE_CUDA) {
-    auto* cb = static_cast<CudaBackend*>(g->be.get());
+  const paella_config_t& cfg = g->P->cfg;
+  Gpu::EvPair ep{nullptr, nullptr, 0, 0};
+  CudaBackend* cb = nullptr;
+  if (cfg.device == PAELLA_DEVICE_CUDA) {
+    cb = static_cast<CudaBackend*>(g->be.get());
     cb->cur_tmap = (k.kind == KIND_CONV_TC) ? m->gpu[g->index].tmaps[layer].b : nullptr;
+    if (cfg.event_time_kind == k.kind + 1 && !g->ev_free.empty()) {
+      ep = g->ev_free.back();
+      g->ev_free.pop_back();
+      ep.bytes = k.bytes;
+      ep.flops = k.flops;
+      cudaEventRecord((cudaEvent_t)ep.e0, cb->streams[stream]);
+    }
   }
   g->be->launch(k, m->gpu[g->index].args[slot][layer], ia, stream, m->dtype, instr);
+  if (ep.e0) {
+    cudaEventRecord((cudaEvent_t)ep.e1, cb->streams[stream]);
+    g->ev_pending.push_back(ep);
+  }
+}
+
+// harvest completed event-timed launches (in launch order; stops at the first pending)
+static void harvest_events(Gpu* g) {
+  while (g->ev_head < g->ev_pending.size()) {
+    Gpu::EvPair& ep = g->ev_pending[g->ev_head];
+    if (cudaEventQuery((cudaEvent_t)ep.e1) != cudaSuccess) break;
+    float ms = 0;
+    cudaEventElapsedTime(&ms, (cudaEvent_t)ep.e0, (cudaEvent_t)ep.e1);
+    g->stats.ev_launches++;
+    g->stats.ev_ns += (uint64_t)((double)ms * 1e6);
+    g->stats.ev_bytes += ep.bytes;
+    g->stats.ev_flops += ep.flops;
+    g->ev_free.push_back(ep);
+    g->ev_head++;
+  }
+  if (g->ev_head == g->ev_pending.size()) {
+    g->ev_pending.clear();
+    g->ev_head = 0;
+  }
 }
 
 static void push_completion(Gpu* g, const JobRec& j, int32_t status) {
@@ -388,8 +441,17 @@ static void dispatcher_main(Gpu* g) {
     pthread_setaffinity_np(pthread_self(), sizeof cs, &cs);
   }
   const uint32_t N = P->cfg.num_clients;
+  if (P->cfg.device == PAELLA_DEVICE_CUDA && P->cfg.event_time_kind) {
+    for (int i = 0; i < 512; ++i) {
+      cudaEvent_t a, b;
+      cudaEventCreate(&a);
+      cudaEventCreate(&b);
+      g->ev_free.push_back(Gpu::EvPair{a, b, 0, 0});
+    }
+  }
   for (;;) {
     g->stats.loop_iters++;
+    if (!g->ev_pending.empty() && (g->stats.loop_iters & 63) == 0) harvest_events(g);
     g->be->advance();
     uint32_t nev = 0;
     // 1. client rings, round-robin, starting after the last client served (C2-Q16)
@@ -878,8 +940,7 @@ static void iso_launch(Gpu* g, Model* m, uint32_t l, bool instr) {
   auto* cb = static_cast<CudaBackend*>(g->be.get());
   const void* tm = (k.kind == KIND_CONV_TC) ? m->gpu[g->index].tmaps[l].b : nullptr;
   void* args[3] = {(void*)&m->gpu[g->index].args[iso_slot][l], (void*)&ia, (void*)tm};
-  cudaLaunchKernel((const void*)cb->fn(k.kind, m->dtype, instr), dim3(k.grid[0], k.grid[1], k.grid[2]),
-                   dim3(k.block), args, k.smem, (cudaStream_t)g->prof_stream);
+  cuda_launch(cb->fn(k.kind, m->dtype, instr), k, args, (cudaStream_t)g->prof_stream);
 }
 
 static int iso_run(Gpu* g, Model* m, const void* input, void* output, int64_t* kernel_ns, bool instr) {
@@ -1084,6 +1145,183 @@ int paella_debug_node(paella_t* p, uint32_t gpu, uint32_t model_id, uint32_t nod
       out[(size_t)c * nd.h * nd.w + p2] = v;
     }
   return 0;
+}
+
+}  // extern "C"
+
+// ===========================================================================
+// device-only timing and notification microbenchmarks
+// ===========================================================================
+namespace paella {
+
+static volatile uint32_t* gate_ptr(Gpu* g, const volatile uint32_t** dev) {
+  volatile uint32_t* gate = (volatile uint32_t*)((uint8_t*)g->stage_in + g->stage_bytes - 64);
+  cudaHostGetDevicePointer((void**)dev, (void*)gate, 0);
+  return gate;
+}
+
+static void launch_gate(Gpu* g, const volatile uint32_t* gd) {
+  void* gargs[1] = {(void*)&gd};
+  cudaLaunchKernel((const void*)gate_kernel(), dim3(1), dim3(1), gargs, 0, (cudaStream_t)g->prof_stream);
+}
+
+static InstrArgs iso_instr(Gpu* g, uint32_t grid, uint32_t group, bool last) {
+  InstrArgs ia;
+  ia.ring = (Rec*)g->prof_ring_d;
+  ia.tail = g->prof_tail;
+  uint32_t uid = g->prof_uid++;
+  uint32_t slot = uid % NCTR;
+  ia.ctr = g->prof_ctr + 2 * slot;
+  ia.mask = (1u << 16) - 1;
+  ia.log2cap = 16;
+  ia.base = g->prof_base[slot];
+  g->prof_base[slot] += grid;
+  ia.uid = uid;
+  ia.group = group;
+  ia.flags = INSTR_ON | (last ? INSTR_LAST : 0);
+  return ia;
+}
+
+}  // namespace paella
+
+extern "C" {
+
+int paella_time_kernels(paella_t* p, uint32_t gpu, uint32_t model_id, uint32_t instrumented, uint32_t reps,
+                        int64_t* kernel_ns) {
+  Paella* P = (Paella*)p;
+  if (!P || gpu >= P->gpus.size() || model_id >= P->nmodels.load() || !kernel_ns || reps == 0) return -EINVAL;
+  if (P->cfg.device != PAELLA_DEVICE_CUDA) return -ENODEV;
+  Gpu* g = P->gpus[gpu].get();
+  std::lock_guard<std::mutex> lk(g->iso_mu);
+  Model* m = P->models[model_id].get();
+  int rc = iso_run(g, m, nullptr, nullptr, nullptr, true);   // materialise valid activations
+  if (rc) return rc;
+  cudaSetDevice(g->device);
+  cudaStream_t s = (cudaStream_t)g->prof_stream;
+  auto* cb = static_cast<CudaBackend*>(g->be.get());
+  uint32_t iso_slot = (uint32_t)m->gpu[gpu].args.size() - 1;
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  for (uint32_t l = 0; l < m->kernels.size(); ++l) {
+    const KernelInst& k = m->kernels[l];
+    const volatile uint32_t* gd;
+    volatile uint32_t* gate = gate_ptr(g, &gd);
+    *gate = 0;
+    launch_gate(g, gd);
+    cudaEventRecord(e0, s);
+    const void* tm = (k.kind == KIND_CONV_TC) ? m->gpu[gpu].tmaps[l].b : nullptr;
+    for (uint32_t r = 0; r < std::min(reps, 256u); ++r) {
+      InstrArgs ia = iso_instr(g, k.grid_total(), P->cfg.group_size, l + 1 == m->kernels.size());
+      void* args[3] = {(void*)&m->gpu[gpu].args[iso_slot][l], (void*)&ia, (void*)tm};
+      cuda_launch(cb->fn(k.kind, m->dtype, instrumented != 0), k, args, s);
+    }
+    cudaEventRecord(e1, s);
+    std::atomic_thread_fence(std::memory_order_seq_cst);
+    *gate = 1;
+    if (cudaStreamSynchronize(s) != cudaSuccess) return -EIO;
+    float ms = 0;
+    cudaEventElapsedTime(&ms, e0, e1);
+    kernel_ns[l] = (int64_t)((double)ms * 1e6 / std::min(reps, 256u));
+  }
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  return 0;
+}
+
+int paella_bench_empty(paella_t* p, uint32_t gpu, uint32_t grid, uint32_t block, uint32_t instrumented,
+                       uint32_t group, uint32_t iters, double* ns_per_launch) {
+  Paella* P = (Paella*)p;
+  if (!P || gpu >= P->gpus.size() || !ns_per_launch || iters == 0 || group == 0 || group > 16) return -EINVAL;
+  if (P->cfg.device != PAELLA_DEVICE_CUDA) return -ENODEV;
+  Gpu* g = P->gpus[gpu].get();
+  std::lock_guard<std::mutex> lk(g->iso_mu);
+  int rc = ensure_iso(g);
+  if (rc) return rc;
+  cudaSetDevice(g->device);
+  cudaStream_t s = (cudaStream_t)g->prof_stream;
+  auto* cb = static_cast<CudaBackend*>(g->be.get());
+  KernelFn f = cb->fn(KIND_EMPTY, 0, instrumented != 0);
+  LayerArgs la{};
+  const volatile uint32_t* gd;
+  volatile uint32_t* gate = gate_ptr(g, &gd);
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  // gated batches stay well below the driver's pending-launch queue depth (a full
+  // queue would block the host while the gate blocks the GPU)
+  const uint32_t batch = 256;
+  double total_ms = 0;
+  for (uint32_t done = 0; done < iters; done += batch) {
+    uint32_t nb = std::min(batch, iters - done);
+    *gate = 0;
+    launch_gate(g, gd);
+    cudaEventRecord(e0, s);
+    for (uint32_t i = 0; i < nb; ++i) {
+      InstrArgs ia = iso_instr(g, grid, group, false);
+      void* args[2] = {(void*)&la, (void*)&ia};
+      cudaLaunchKernel((const void*)f, dim3(grid), dim3(block), args, 0, s);
+    }
+    cudaEventRecord(e1, s);
+    std::atomic_thread_fence(std::memory_order_seq_cst);
+    *gate = 1;
+    if (cudaStreamSynchronize(s) != cudaSuccess) return -EIO;
+    float ms = 0;
+    cudaEventElapsedTime(&ms, e0, e1);
+    total_ms += ms;
+  }
+  float ms = (float)total_ms;
+  *ns_per_launch = (double)ms * 1e6 / iters;
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  return 0;
+}
+
+int paella_bench_roundtrip(paella_t* p, uint32_t gpu, uint32_t n, int64_t* place_ns, int64_t* complete_ns) {
+  Paella* P = (Paella*)p;
+  if (!P || gpu >= P->gpus.size() || !place_ns || !complete_ns) return -EINVAL;
+  if (P->cfg.device != PAELLA_DEVICE_CUDA) return -ENODEV;
+  Gpu* g = P->gpus[gpu].get();
+  std::lock_guard<std::mutex> lk(g->iso_mu);
+  int rc = ensure_iso(g);
+  if (rc) return rc;
+  cudaSetDevice(g->device);
+  cudaStream_t s = (cudaStream_t)g->prof_stream;
+  cudaStreamSynchronize(s);
+  auto* cb = static_cast<CudaBackend*>(g->be.get());
+  KernelFn f = cb->fn(KIND_EMPTY, 0, true);
+  LayerArgs la{};
+  // consume from the current device tail
+  uint32_t tail = 0;
+  cudaMemcpy(&tail, g->prof_tail, 4, cudaMemcpyDeviceToHost);
+  uint64_t head = tail;
+  const uint32_t mask = (1u << 16) - 1;
+  for (uint32_t i = 0; i < n; ++i) {
+    InstrArgs ia = iso_instr(g, 1, 1, false);
+    void* args[2] = {(void*)&la, (void*)&ia};
+    int64_t t0 = now_ns();
+    cudaLaunchKernel((const void*)f, dim3(1), dim3(32), args, 0, s);
+    for (int want = 0; want < 2; ++want) {
+      volatile uint64_t* r = (volatile uint64_t*)(g->prof_ring_h + (head & mask));
+      uint32_t tag = rec_tag((uint32_t)(head >> 16));
+      int64_t tstart = now_ns();
+      for (;;) {
+        uint64_t w0 = r[0];
+        if ((w0 & 0xff) != 0 && ((w0 >> 24) & 0xff) == tag && (r[1] >> 56) == tag) break;
+        if (now_ns() - tstart > 1000000000ll) return -ETIMEDOUT;
+      }
+      int64_t t = now_ns() - t0;
+      uint64_t w0 = r[0];
+      r[0] = 0;
+      r[1] = 0;
+      if ((w0 & 0xff) == REC_PLACEMENT)
+        place_ns[i] = t;
+      else
+        complete_ns[i] = t;
+      head++;
+    }
+  }
+  return cudaStreamSynchronize(s) == cudaSuccess ? 0 : -EIO;
 }
 
 }  // extern "C"

@@ -142,6 +142,15 @@ struct Gpu {
   size_t stage_bytes = 0;
   std::mutex iso_mu;
   std::vector<uint32_t> naive_inflight;   // job ids in naive mode
+  // live event timing of one kernel kind (roofline)
+  struct EvPair {
+    void* e0;
+    void* e1;
+    uint64_t bytes, flops;
+  };
+  std::vector<EvPair> ev_free;
+  std::vector<EvPair> ev_pending;   // FIFO by launch order
+  size_t ev_head = 0;
 };
 
 struct Paella {

@@ -17,8 +17,9 @@
 //  * epilogue: the 4 producer warps read the accumulator with tcgen05.ld (warp w
 //    owns TMEM lanes 32w..32w+31 = 32 output channels), add bias, residual (fp32),
 //    activation, round once to bf16 (reading C1-Q7) and store NHWC;
-//  * split-K over blockIdx.z for the deep, narrow late layers: fp32 partials to a
-//    per-job workspace, the last-arriving CTA of a tile reduces and runs the epilogue.
+//  * split-K over blockIdx.z for the deep, narrow late layers: the ksplit CTAs of a
+//    tile form a thread-block cluster; partial tiles stay in shared memory and are
+//    reduced over DSMEM, each CTA finishing a 1/ksplit slice of the tile.
 //
 // Block instrumentation (K1) wraps the whole CTA (instr.cuh).
 #include <cuda.h>
@@ -142,7 +143,6 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   uint64_t* empty = full + TC_STAGES;
   uint64_t* accb = empty + TC_STAGES;
   uint32_t* tmem_slot = (uint32_t*)(accb + 1);
-  uint32_t* flag = tmem_slot + 1;
 
   const uint32_t warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const uint32_t tile_n = blockIdx.x, tile_m = blockIdx.y, split = blockIdx.z;
@@ -268,55 +268,81 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 #pragma unroll
       for (int i = 0; i < 64; ++i) acc[i] = 0.f;
     }
-    bool do_epi = true;
-    if (a.ksplit > 1) {
-      const uint32_t tiles = a.tiles_m * a.tiles_n;
-      const uint32_t tile = tile_m * a.tiles_n + tile_n;
-      float* part = a.ws + ((size_t)split * tiles + tile) * (TC_BM * TC_BN) + (size_t)row * TC_BN;
+    if (a.ksplit == 1) {
+      if (co < a.cout) {
+        const float b = a.bias[co];
+        __nv_bfloat16* Y = static_cast<__nv_bfloat16*>(a.out);
+        const __nv_bfloat16* R = static_cast<const __nv_bfloat16*>(a.res);
+        const bool has_res = (a.flags & LF_RESIDUAL) != 0;
 #pragma unroll
-      for (int i = 0; i < 64; i += 4) __stcg(reinterpret_cast<float4*>(part + i), make_float4(acc[i], acc[i + 1], acc[i + 2], acc[i + 3]));
-      __threadfence();
-      asm volatile("bar.sync 1, 128;" ::: "memory");
-      if (threadIdx.x == 0) {
-        uint32_t old = atomicAdd(&a.ws_ctr[tile], 1u);
-        uint32_t last = (old == a.ksplit - 1) ? 1u : 0u;
-        if (last) a.ws_ctr[tile] = 0;   // reset for the next launch on this slot
-        *flag = last;
+        for (int j = 0; j < 64; ++j) {
+          const uint32_t p = n0 + j;
+          if (p < P) {
+            float v = acc[j] + b;
+            if (has_res) v += __bfloat162float(R[(size_t)p * a.res_cs + a.res_co + co]);
+            Y[(size_t)p * a.out_cs + a.out_co + co] = __float2bfloat16_rn(act_tc(v, a.act));
+          }
+        }
       }
-      asm volatile("bar.sync 1, 128;" ::: "memory");
-      do_epi = *flag != 0;
-      if (do_epi) {
-        __threadfence();
+    } else {
+      // split-K across the CTAs of a cluster (cluster dims 1 x 1 x ksplit): every CTA
+      // parks its fp32 partial tile in its own shared memory (the drained pipeline
+      // buffers), then reduces a 1/ksplit slice of the tile over DSMEM and runs the
+      // epilogue for it -- no global workspace, no atomics.
+      float* part = reinterpret_cast<float*>(smem);   // [128 rows][64 cols]
 #pragma unroll
-        for (int i = 0; i < 64; ++i) acc[i] = 0.f;
-        for (uint32_t sp = 0; sp < a.ksplit; ++sp) {
-          const float* q = a.ws + ((size_t)sp * tiles + tile) * (TC_BM * TC_BN) + (size_t)row * TC_BN;
+      for (int i = 0; i < 64; i += 4)
+        *reinterpret_cast<float4*>(part + row * 64 + ((i + 4 * (row & 15)) & 63)) =
+            make_float4(acc[i], acc[i + 1], acc[i + 2], acc[i + 3]);
+    }
+  }
+  if (a.ksplit > 1) {
+    __syncwarp();
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    if (warp < 4) {
+      const uint32_t ks = a.ksplit;
+      const uint32_t per_thr = 64 / ks;               // elements of the tile per thread
+      const uint32_t e0 = split * (8192 / ks) + threadIdx.x * per_thr;
+      const uint32_t row = e0 / 64, col0 = e0 % 64;   // per_thr <= 64 stays inside one row
+      const uint32_t part_addr = su32(smem);
+      float sum[32];
 #pragma unroll
-          for (int i = 0; i < 64; i += 4) {
-            float4 f = __ldcg(reinterpret_cast<const float4*>(q + i));
-            acc[i] += f.x;
-            acc[i + 1] += f.y;
-            acc[i + 2] += f.z;
-            acc[i + 3] += f.w;
+      for (int i = 0; i < 32; ++i) sum[i] = 0.f;
+      for (uint32_t r = 0; r < ks; ++r) {
+        uint32_t peer;
+        asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(peer) : "r"(part_addr), "r"(r));
+        for (uint32_t i = 0; i < per_thr; i += 4) {
+          const uint32_t c = col0 + i;
+          const uint32_t addr = peer + (row * 64 + ((c + 4 * (row & 15)) & 63)) * 4;
+          float x0, x1, x2, x3;
+          asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
+                       : "=f"(x0), "=f"(x1), "=f"(x2), "=f"(x3)
+                       : "r"(addr));
+          sum[i] += x0;
+          sum[i + 1] += x1;
+          sum[i + 2] += x2;
+          sum[i + 3] += x3;
+        }
+      }
+      const uint32_t co = m0 + row;
+      if (co < a.cout) {
+        const float b = a.bias[co];
+        __nv_bfloat16* Y = static_cast<__nv_bfloat16*>(a.out);
+        const __nv_bfloat16* R = static_cast<const __nv_bfloat16*>(a.res);
+        const bool has_res = (a.flags & LF_RESIDUAL) != 0;
+        for (uint32_t i = 0; i < per_thr; ++i) {
+          const uint32_t p = n0 + col0 + i;
+          if (p < P) {
+            float v = sum[i] + b;
+            if (has_res) v += __bfloat162float(R[(size_t)p * a.res_cs + a.res_co + co]);
+            Y[(size_t)p * a.out_cs + a.out_co + co] = __float2bfloat16_rn(act_tc(v, a.act));
           }
         }
       }
     }
-    if (do_epi && co < a.cout) {
-      const float b = a.bias[co];
-      __nv_bfloat16* Y = static_cast<__nv_bfloat16*>(a.out);
-      const __nv_bfloat16* R = static_cast<const __nv_bfloat16*>(a.res);
-      const bool has_res = (a.flags & LF_RESIDUAL) != 0;
-#pragma unroll
-      for (int j = 0; j < 64; ++j) {
-        const uint32_t p = n0 + j;
-        if (p < P) {
-          float v = acc[j] + b;
-          if (has_res) v += __bfloat162float(R[(size_t)p * a.res_cs + a.res_co + co]);
-          Y[(size_t)p * a.out_cs + a.out_co + co] = __float2bfloat16_rn(act_tc(v, a.act));
-        }
-      }
-    }
+    // no CTA may leave while a peer still reads its shared memory
+    __syncwarp();
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
   }
   tc_fence_before();
   __syncthreads();

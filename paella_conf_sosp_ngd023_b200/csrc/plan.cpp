@@ -249,11 +249,12 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
             a.tiles_n = (P_out + TC_BN - 1) / TC_BN;
             uint32_t nk = kpad / TC_BK;
             uint32_t tiles = a.tiles_m * a.tiles_n;
-            // split K so the grid approaches one wave of SMs, >= 2 k-blocks per split
+            // split K so the grid approaches one wave of SMs, >= 2 k-blocks per split;
+            // the splits of a tile form one thread-block cluster (<= 8, portable)
             uint32_t split = 1;
             const char* e = std::getenv("PAELLA_NOSPLIT");
             if (!e) {
-              while (tiles * split * 2 <= P->sms && nk / (split * 2) >= 2) split *= 2;
+              while (split < 8 && tiles * split * 2 <= P->sms && nk / (split * 2) >= 2) split *= 2;
             }
             a.ksplit = split;
             k.grid[0] = a.tiles_n;
@@ -262,10 +263,7 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
             k.block = TC_THREADS;
             k.smem = tc_smem_bytes();
             k.tmem_cols = tc_tmem_cols();
-            if (split > 1) {
-              max_splitk = std::max<size_t>(max_splitk, (size_t)split * tiles * TC_BM * TC_BN);
-              max_tiles = std::max<size_t>(max_tiles, tiles);
-            }
+
           } else {
             k.kind = KIND_CONV_SIMT;
             k.grid[0] = (P_out + 63) / 64;
