@@ -50,6 +50,8 @@ def parse():
     ap.add_argument("--rho", type=float, default=0.7)
     ap.add_argument("--reqs", type=int, default=2000, help="requests per step")
     ap.add_argument("--no-baselines", action="store_true")
+    ap.add_argument("--fake", action="store_true",
+                    help="CPU fake device (tests of the multi-rank plumbing; not a measurement)")
     return ap.parse_args()
 
 
@@ -109,6 +111,8 @@ class Clocks:
         self.proc = None
 
     def start(self):
+        if self.gpu < 0:
+            return
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
                                           "--format=csv,noheader,nounits", "-lms", "200"],
@@ -142,8 +146,12 @@ class Clocks:
 # ---------------------------------------------------------------------------
 # the GPU arm
 # ---------------------------------------------------------------------------
-def build_engine(L, specs, gpu, **kw):
-    e = L.Engine(num_clients=len(specs), first_gpu=gpu, **kw)
+def build_engine(L, specs, gpu, fake=False, **kw):
+    if fake:
+        kw.pop("event_time_kind", None)
+        e = L.Engine(num_clients=len(specs), device=L.DEVICE_FAKE, **kw)
+    else:
+        e = L.Engine(num_clients=len(specs), first_gpu=gpu, **kw)
     mids = [e.register_model(g, P) for (g, P) in specs]
     return e, mids
 
@@ -209,7 +217,7 @@ def run_gpu(args, dist):
     region = slots * stride + (1 << 20)
 
     def engine(**kw):
-        e, mids = build_engine(L, specs, gpu, region_bytes=region, max_jobs_per_model=128, **kw)
+        e, mids = build_engine(L, specs, gpu, fake=args.fake, region_bytes=region, max_jobs_per_model=128, **kw)
         stage_inputs(e, specs, mids, slots, stride, pool)
         return e, mids
 
@@ -230,7 +238,10 @@ def run_gpu(args, dist):
     dev_roof = {}
     kinfo = {}
     for m, nm in enumerate(names):
-        kt = e.time_kernels(mids[m], instrumented=False, reps=20)
+        if args.fake:
+            kt = np.array([k["tbar_ns"] for k in e.kernels(mids[m])], dtype=np.int64)
+        else:
+            kt = e.time_kernels(mids[m], instrumented=False, reps=20)
         dev_roof[nm] = float(kt.sum()) / 1e3
         kinfo[nm] = (e.kernels(mids[m]), kt)
     calib_s = time.time() - t_cal
@@ -240,7 +251,7 @@ def run_gpu(args, dist):
         t, mm, ii = make_trace(args.reqs, lam, cfg, len(names), seed=seed0 + w)
         e.loadgen(t, mm, mm, ii, stride, slots)
     st0 = e.stats()
-    clocks = Clocks(gpu)
+    clocks = Clocks(gpu if not args.fake else -1)
     dist.barrier()
     clocks.start()
     t_start = time.perf_counter_ns()
@@ -420,8 +431,10 @@ def main():
         "clocks": res["clocks"],
         "dispatcher": {k: int(v) for k, v in res["stats"].items()},
     }
-    if args.gpus == 1:
+    if args.gpus == 1 and not args.fake:
         line["cpu_baseline"] = cpu_baseline(cfg, seconds=12.0)
+    if args.fake:
+        line["data"] = "synthetic, FAKE CPU device (plumbing test, not a measurement)"
     print(json.dumps(line))
 
 

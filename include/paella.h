@@ -101,6 +101,11 @@ typedef struct {
   uint32_t event_time_kind;      /* 0 = off; k+1 = the dispatcher brackets every launch of
                                     kernel kind k with CUDA events on its stream and sums
                                     the durations (paella_stats ev_*): the live roofline */
+  uint32_t lookahead;            /* NEXT-1 launch-ahead depth: 0 = the paper's semantics (a
+                                    job's next kernel is dispatched after the previous one's
+                                    final COMPLETION); D > 0 = once the previous kernel is
+                                    fully placed and <= D are in flight, the next kernel is
+                                    queued behind it on the same stream */
 } paella_config_t;
 
 /* ---- model description (input to paella_register_model) ---------------- */

@@ -53,6 +53,7 @@ class Config:
     ring_capacity: int = 65536
     streams: int = 32                 # P
     capacity: tuple = (148 * 32, 148 * 64, 148 * 65536, 148 * 233472, 148 * 512)
+    lookahead: int = 0                # NEXT-1 launch-ahead depth (0 = the paper's semantics)
 
 
 def groups(g, G):
@@ -66,9 +67,15 @@ class Job:
     model: int
     seq: int
     R: int
-    cursor: int = 0
-    inflight: bool = False
+    cursor: int = 0          # next kernel to issue (= kernels dispatched, c_i of P1265)
+    done: int = 0            # kernels completed
+    stream: int = -1         # stream held while kernels are in flight
     last_stream: int = -1
+    last_uid: int = -1
+
+    @property
+    def inflight(self):
+        return self.cursor - self.done
 
 
 @dataclass
@@ -84,7 +91,12 @@ class Launch:
 
 
 class Policy:
-    """The dispatcher state machine of SURVEY.md §8(c) C2, integer-exact."""
+    """The dispatcher state machine of SURVEY.md §8(c) C2, integer-exact.
+
+    Launch-ahead (NEXT-1; off by default): with lookahead = D > 0 a
+    job whose most recent kernel is fully placed (p_eff = grid) and that has at most
+    D kernels in flight may issue its next kernel onto the SAME stream (stream order
+    carries the dependency, P947-951); the paper's semantics is D = 0."""
 
     def __init__(self, cfg: Config, models: list[list[Layer]]):
         self.cfg = cfg
@@ -145,12 +157,13 @@ class Policy:
         done = None
         if L.f == L.grid:
             del self.launches[uid]
-            self.free.add(L.stream)
             j = self.jobs[L.job]
-            j.inflight = False
-            j.cursor += 1
-            j.last_stream = L.stream
-            if j.cursor == len(self.models[j.model]):
+            j.done += 1
+            if j.inflight == 0:
+                self.free.add(L.stream)
+                j.stream = -1
+                j.last_stream = L.stream
+            if j.done == len(self.models[j.model]):
                 if self.checks:
                     assert j.R == 0
                 del self.jobs[j.id]
@@ -161,9 +174,18 @@ class Policy:
                 done = j.id
         return done
 
+    def is_ready(self, j):
+        if j.cursor >= len(self.models[j.model]):
+            return False
+        if j.inflight == 0:
+            return True
+        if self.cfg.lookahead <= 0 or j.inflight > self.cfg.lookahead:
+            return False
+        L = self.launches.get(j.last_uid)
+        return L is not None and max(L.p, L.f) >= L.grid
+
     def ready(self):
-        return [j for j in self.jobs.values()
-                if not j.inflight and j.cursor < len(self.models[j.model])]
+        return [j for j in self.jobs.values() if self.is_ready(j)]
 
     def pick(self, rdy):
         cfg = self.cfg
@@ -188,31 +210,36 @@ class Policy:
         if self.log is not None:
             self.log.append((EV_BATCH_END,))
         while True:
-            if not self.free:
-                break
             rdy = self.ready()
             if not rdy:
                 break
             j = self.pick(rdy)
+            if j.inflight == 0 and not self.free:
+                break
             layer = self.models[j.model][j.cursor]
             if not self.predicate(layer.grid):
                 break
             uid = self.next_uid
             self.next_uid += 1
-            stream = j.last_stream if j.last_stream in self.free else min(self.free)
-            self.free.remove(stream)
+            if j.inflight > 0:
+                stream = j.stream            # launch-ahead: behind its predecessor
+            else:
+                stream = j.last_stream if j.last_stream in self.free else min(self.free)
+                self.free.remove(stream)
+                j.stream = stream
             self.launches[uid] = Launch(uid, j.id, j.cursor, layer.grid, layer.demand, stream)
             for r in range(len(RESOURCES)):
                 self.U[r] += layer.grid * layer.demand[r]
             self.Q += layer.grid
             self.O += 2 * groups(layer.grid, cfg.group)
             j.R -= layer.tbar
-            j.inflight = True
+            rec = (uid, j.id, j.cursor, stream)
+            j.cursor += 1
+            j.last_uid = uid
             if self.checks:
                 assert j.R >= 0
             self.Dt[j.client] -= cfg.num_clients
             self.Omega += 1
-            rec = (uid, j.id, j.cursor, stream)
             if self.log is not None:
                 self.log.append((EV_ISSUE,) + rec)
             out.append(rec)

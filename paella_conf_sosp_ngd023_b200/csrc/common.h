@@ -82,6 +82,7 @@ enum : uint32_t {
   LF_CEIL = 2u,       // maxpool ceil mode
   LF_FINAL = 4u,      // output is the fp32 logits in client memory
   LF_RESIDUAL = 8u,
+  LF_TRACE = 16u,     // debug: per-CTA phase timestamps (globaltimer) into ws
 };
 
 struct LayerArgs {

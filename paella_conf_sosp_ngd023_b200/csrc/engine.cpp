@@ -558,6 +558,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
   if (cfg.client_region_bytes == 0) cfg.client_region_bytes = 64ull << 20;
   if (cfg.fake_time_scale_ns == 0) cfg.fake_time_scale_ns = 500;
   if (cfg.fairness_threshold < 0) return -EINVAL;
+  if (cfg.lookahead > 4) return -EINVAL;
 
   auto P = std::make_unique<Paella>();
   P->cfg = cfg;
@@ -621,6 +622,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     pc.group = cfg.group_size;
     pc.ring_capacity = cfg.ring_capacity;
     pc.streams = cfg.stream_pool;
+    pc.lookahead = cfg.lookahead;
     for (int r = 0; r < NRES; ++r) pc.capacity[r] = P->capacity[r];
     g->policy.reset(new Policy(pc));
     for (uint32_t c = 0; c < cfg.num_clients; ++c) {
@@ -640,7 +642,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
       setvbuf(g->log, nullptr, _IOFBF, 1 << 20);
       logev(g.get(), EV_CONFIG, cfg.num_clients, cfg.policy, (uint64_t)cfg.fairness_threshold,
             ((uint64_t)P->cfg.slack_blocks << 32) | cfg.group_size);
-      logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFFu, cfg.ring_capacity, cfg.stream_pool, 0);
+      logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFFu, cfg.ring_capacity, cfg.stream_pool, cfg.lookahead);
       for (int r = 0; r < NRES; ++r) logev(g.get(), EV_CAPACITY, (uint32_t)r, (uint64_t)P->capacity[r], 0, 0);
     }
     P->gpus.push_back(std::move(g));
@@ -965,10 +967,24 @@ static int iso_run(Gpu* g, Model* m, const void* input, void* output, int64_t* k
     const volatile uint32_t* gd = nullptr;
     cudaHostGetDevicePointer((void**)&gd, (void*)gate, 0);
     void* gargs[1] = {(void*)&gd};
-    cudaLaunchKernel((const void*)gate_kernel(), dim3(1), dim3(1), gargs, 0, s);
+    if (!std::getenv("PAELLA_NO_GATE"))
+      cudaLaunchKernel((const void*)gate_kernel(), dim3(1), dim3(1), gargs, 0, s);
     ev.resize(m->kernels.size() + 1);
     for (auto& e : ev) cudaEventCreate(&e);
     cudaEventRecord(ev[0], s);
+  }
+  // debug: PAELLA_TRACE_KERNEL=<k> -> per-CTA phase timestamps of tcgen05 conv k
+  int trace_k = std::getenv("PAELLA_TRACE_KERNEL") ? atoi(std::getenv("PAELLA_TRACE_KERNEL")) : -1;
+  uint64_t* trbuf = nullptr;
+  LayerArgs saved{};
+  if (trace_k >= 0 && trace_k < (int)m->kernels.size() && m->kernels[trace_k].kind == KIND_CONV_TC) {
+    cudaMalloc(&trbuf, 8 * 8 * m->kernels[trace_k].grid_total());
+    cudaMemset(trbuf, 0, 8 * 8 * m->kernels[trace_k].grid_total());
+    saved = args[trace_k];
+    args[trace_k].flags |= LF_TRACE;
+    args[trace_k].ws = (float*)trbuf;
+  } else {
+    trace_k = -1;
   }
   for (uint32_t l = 0; l < m->kernels.size(); ++l) {
     iso_launch(g, m, l, instr);
@@ -982,6 +998,27 @@ static int iso_run(Gpu* g, Model* m, const void* input, void* output, int64_t* k
   if (e != cudaSuccess) {
     fprintf(stderr, "paella: isolated run failed: %s\n", cudaGetErrorString(e));
     return -EIO;
+  }
+  if (trace_k >= 0) {
+    cudaStreamSynchronize(s);
+    uint32_t nb = m->kernels[trace_k].grid_total();
+    std::vector<uint64_t> h(8 * nb);
+    cudaMemcpy(h.data(), trbuf, h.size() * 8, cudaMemcpyDeviceToHost);
+    cudaFree(trbuf);
+    args[trace_k] = saved;
+    uint64_t t0 = UINT64_MAX;
+    for (uint32_t b = 0; b < nb; ++b) t0 = std::min(t0, h[8 * b]);
+    const char* names[8] = {"entry", "setup", "full0", "mma_done", "accb", "epi_done", "pre_exit", "exit"};
+    fprintf(stderr, "trace kernel %d grid %u (ns from first CTA entry): phase min/med/max\n", trace_k, nb);
+    for (int ph = 0; ph < 8; ++ph) {
+      std::vector<int64_t> v;
+      for (uint32_t b = 0; b < nb; ++b)
+        if (h[8 * b + ph]) v.push_back((int64_t)(h[8 * b + ph] - t0));
+      if (v.empty()) continue;
+      std::sort(v.begin(), v.end());
+      fprintf(stderr, "  %-9s %7lld %7lld %7lld\n", names[ph], (long long)v.front(), (long long)v[v.size() / 2],
+              (long long)v.back());
+    }
   }
   if (kernel_ns) {
     for (uint32_t l = 0; l < m->kernels.size(); ++l) {
@@ -1161,6 +1198,7 @@ static volatile uint32_t* gate_ptr(Gpu* g, const volatile uint32_t** dev) {
 }
 
 static void launch_gate(Gpu* g, const volatile uint32_t* gd) {
+  if (std::getenv("PAELLA_NO_GATE")) return;
   void* gargs[1] = {(void*)&gd};
   cudaLaunchKernel((const void*)gate_kernel(), dim3(1), dim3(1), gargs, 0, (cudaStream_t)g->prof_stream);
 }

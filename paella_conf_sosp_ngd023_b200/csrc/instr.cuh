@@ -10,8 +10,8 @@
 //    writes ONE 16-byte record {type, count, smid, uid | globaltimer, group} with a
 //    single vector store straight into pinned, mapped host memory (P1104-1106);
 //  * exit: __syncthreads (all outputs of the block written), a release fence
-//    (gpu scope; system scope for a job's last kernel, whose output lives in client
-//    host memory) before the end-counter atomic, so a successor kernel launched after
+//    (an acq_rel end-counter atomic: gpu scope; system scope for a job's last kernel,
+//    whose output lives in client host memory), so a successor kernel launched after
 //    the dispatcher saw the final COMPLETION reads complete data (reading C2-Q19);
 //  * %smid is re-read at exit (reading C2-Q4).
 //
@@ -54,10 +54,12 @@ __device__ __forceinline__ void maybe_record(const InstrArgs& ia, uint32_t type,
   }
 }
 
-template <bool INSTR>
+// T = the (1-D) thread that does the bookkeeping; kernels pick an otherwise idle
+// thread so that compute never waits on the counter atomics
+template <bool INSTR, uint32_t T = 0>
 __device__ __forceinline__ void instr_enter(const InstrArgs& ia) {
   if constexpr (INSTR) {
-    if (threadIdx.x == 0 && threadIdx.y == 0 && threadIdx.z == 0) {
+    if (threadIdx.x == T && threadIdx.y == 0 && threadIdx.z == 0) {
       uint32_t total = gridDim.x * gridDim.y * gridDim.z;
       uint32_t c = atomicAdd(&ia.ctr[0], 1u) + 1u - ia.base;
       maybe_record(ia, REC_PLACEMENT, c, total);
@@ -65,18 +67,21 @@ __device__ __forceinline__ void instr_enter(const InstrArgs& ia) {
   }
 }
 
-template <bool INSTR>
+template <bool INSTR, uint32_t T = 0>
 __device__ __forceinline__ void instr_exit(const InstrArgs& ia) {
   if constexpr (INSTR) {
     __syncthreads();
-    if (threadIdx.x == 0 && threadIdx.y == 0 && threadIdx.z == 0) {
+    if (threadIdx.x == T && threadIdx.y == 0 && threadIdx.z == 0) {
+      // acq_rel atomic: releases this block's outputs (ordered before by the barrier,
+      // release is cumulative) and acquires the earlier blocks' before the record is
+      // written; system scope for a job's last kernel, whose output is in host memory
+      uint32_t old;
       if (ia.flags & INSTR_LAST)
-        __threadfence_system();
+        asm volatile("atom.acq_rel.sys.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(&ia.ctr[1]) : "memory");
       else
-        __threadfence();
+        asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(&ia.ctr[1]) : "memory");
       uint32_t total = gridDim.x * gridDim.y * gridDim.z;
-      uint32_t c = atomicAdd(&ia.ctr[1], 1u) + 1u - ia.base;
-      maybe_record(ia, REC_COMPLETION, c, total);
+      maybe_record(ia, REC_COMPLETION, old + 1u - ia.base, total);
     }
   }
 }

@@ -183,9 +183,36 @@ __global__ void __launch_bounds__(256) k_conv_simt(const __grid_constant__ Layer
 }
 
 // ---------------------------------------------------------------------------
-// K2c depthwise conv (groups == cin == cout), any kh x kw, stride, pad.  One thread
-// per (output pixel, 8-channel granule).  Weights packed [kh][kw][c].
+// K2c depthwise conv (groups == cin == cout).  One thread per (output pixel, 8-channel
+// granule); for the 3x3 case (every depthwise layer of MobileNetV2) all 9 taps of
+// activations and weights are loaded before any arithmetic so the 18 independent
+// 16-byte loads are in flight together (latency, not bandwidth, bounds batch 1).
+// Weights packed [kh][kw][c].
 // ---------------------------------------------------------------------------
+template <typename T, int KH, int KW>
+__device__ __forceinline__ void dw_taps(const LayerArgs& a, const T* X, const T* W, int oh, int ow, int c,
+                                        float (&acc)[8]) {
+  float xv[KH * KW][8], wv[KH * KW][8];
+#pragma unroll
+  for (int r = 0; r < KH; ++r)
+#pragma unroll
+    for (int s = 0; s < KW; ++s) {
+      const int ih = oh * (int)a.sh - (int)a.ph + r, iw = ow * (int)a.sw - (int)a.pw + s;
+      const bool ok = ih >= 0 && ih < (int)a.h && iw >= 0 && iw < (int)a.w_;
+      if (ok) {
+        load8(X + ((size_t)ih * a.w_ + iw) * a.in_cs + a.in_co + c, xv[r * KW + s]);
+      } else {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) xv[r * KW + s][i] = 0.f;
+      }
+      load8(W + ((size_t)r * KW + s) * a.cout + c, wv[r * KW + s]);
+    }
+#pragma unroll
+  for (int t = 0; t < KH * KW; ++t)
+#pragma unroll
+    for (int i = 0; i < 8; ++i) acc[i] = fmaf(wv[t][i], xv[t][i], acc[i]);
+}
+
 template <typename T, bool INSTR>
 __global__ void __launch_bounds__(256) k_dwconv(const __grid_constant__ LayerArgs a,
                                                 const __grid_constant__ InstrArgs ia) {
@@ -203,17 +230,21 @@ __global__ void __launch_bounds__(256) k_dwconv(const __grid_constant__ LayerArg
     float acc[8];
 #pragma unroll
     for (int i = 0; i < 8; ++i) acc[i] = a.bias[c + i];
-    for (int r = 0; r < (int)a.kh; ++r) {
-      int ih = oh * a.sh - a.ph + r;
-      if (ih < 0 || ih >= (int)a.h) continue;
-      for (int s = 0; s < (int)a.kw; ++s) {
-        int iw = ow * a.sw - a.pw + s;
-        if (iw < 0 || iw >= (int)a.w_) continue;
-        float xv[8], wv[8];
-        load8(X + ((size_t)ih * a.w_ + iw) * a.in_cs + a.in_co + c, xv);
-        load8(W + ((size_t)r * a.kw + s) * a.cout + c, wv);
+    if (a.kh == 3 && a.kw == 3) {
+      dw_taps<T, 3, 3>(a, X, W, oh, ow, c, acc);
+    } else {
+      for (int r = 0; r < (int)a.kh; ++r) {
+        int ih = oh * a.sh - a.ph + r;
+        if (ih < 0 || ih >= (int)a.h) continue;
+        for (int s = 0; s < (int)a.kw; ++s) {
+          int iw = ow * a.sw - a.pw + s;
+          if (iw < 0 || iw >= (int)a.w_) continue;
+          float xv[8], wv[8];
+          load8(X + ((size_t)ih * a.w_ + iw) * a.in_cs + a.in_co + c, xv);
+          load8(W + ((size_t)r * a.kw + s) * a.cout + c, wv);
 #pragma unroll
-        for (int i = 0; i < 8; ++i) acc[i] = fmaf(wv[i], xv[i], acc[i]);
+          for (int i = 0; i < 8; ++i) acc[i] = fmaf(wv[i], xv[i], acc[i]);
+        }
       }
     }
     if (a.flags & LF_RESIDUAL) {
@@ -231,8 +262,29 @@ __global__ void __launch_bounds__(256) k_dwconv(const __grid_constant__ LayerArg
 
 // ---------------------------------------------------------------------------
 // K2d pooling.  max: padding = -inf, ceil-mode windows clipped to the input;
-// avg: count_include_pad (divisor k*k).  One thread per (pixel, granule).
+// avg: count_include_pad (divisor k*k).  One thread per (pixel, granule); square
+// 2x2 / 3x3 windows load every tap before reducing (independent loads in flight).
 // ---------------------------------------------------------------------------
+template <typename T, bool MAX, int K>
+__device__ __forceinline__ void pool_taps(const LayerArgs& a, const T* X, int oh, int ow, int c, float (&acc)[8]) {
+  float xv[K * K][8];
+  bool ok[K * K];
+#pragma unroll
+  for (int r = 0; r < K; ++r)
+#pragma unroll
+    for (int s = 0; s < K; ++s) {
+      const int ih = oh * (int)a.sh - (int)a.ph + r, iw = ow * (int)a.sw - (int)a.pw + s;
+      ok[r * K + s] = ih >= 0 && ih < (int)a.h && iw >= 0 && iw < (int)a.w_;
+      if (ok[r * K + s]) load8(X + ((size_t)ih * a.w_ + iw) * a.in_cs + a.in_co + c, xv[r * K + s]);
+    }
+#pragma unroll
+  for (int t = 0; t < K * K; ++t)
+    if (ok[t]) {
+#pragma unroll
+      for (int i = 0; i < 8; ++i) acc[i] = MAX ? fmaxf(acc[i], xv[t][i]) : acc[i] + xv[t][i];
+    }
+}
+
 template <typename T, bool INSTR, bool MAX>
 __global__ void __launch_bounds__(256) k_pool(const __grid_constant__ LayerArgs a,
                                               const __grid_constant__ InstrArgs ia) {
@@ -249,16 +301,22 @@ __global__ void __launch_bounds__(256) k_pool(const __grid_constant__ LayerArgs 
     float acc[8];
 #pragma unroll
     for (int i = 0; i < 8; ++i) acc[i] = MAX ? -INFINITY : 0.f;
-    for (int r = 0; r < (int)a.kh; ++r) {
-      int ih = oh * a.sh - a.ph + r;
-      if (ih < 0 || ih >= (int)a.h) continue;
-      for (int s = 0; s < (int)a.kw; ++s) {
-        int iw = ow * a.sw - a.pw + s;
-        if (iw < 0 || iw >= (int)a.w_) continue;
-        float xv[8];
-        load8(X + ((size_t)ih * a.w_ + iw) * a.in_cs + a.in_co + c, xv);
+    if (a.kh == 3 && a.kw == 3) {
+      pool_taps<T, MAX, 3>(a, X, oh, ow, c, acc);
+    } else if (a.kh == 2 && a.kw == 2) {
+      pool_taps<T, MAX, 2>(a, X, oh, ow, c, acc);
+    } else {
+      for (int r = 0; r < (int)a.kh; ++r) {
+        int ih = oh * a.sh - a.ph + r;
+        if (ih < 0 || ih >= (int)a.h) continue;
+        for (int s = 0; s < (int)a.kw; ++s) {
+          int iw = ow * a.sw - a.pw + s;
+          if (iw < 0 || iw >= (int)a.w_) continue;
+          float xv[8];
+          load8(X + ((size_t)ih * a.w_ + iw) * a.in_cs + a.in_co + c, xv);
 #pragma unroll
-        for (int i = 0; i < 8; ++i) acc[i] = MAX ? fmaxf(acc[i], xv[i]) : acc[i] + xv[i];
+          for (int i = 0; i < 8; ++i) acc[i] = MAX ? fmaxf(acc[i], xv[i]) : acc[i] + xv[i];
+        }
       }
     }
     if (!MAX) {
@@ -272,31 +330,48 @@ __global__ void __launch_bounds__(256) k_pool(const __grid_constant__ LayerArgs 
 }
 
 // ---------------------------------------------------------------------------
-// Global average pool (+ optional DenseNet prologue).  One thread per channel
-// granule; output either an activation (C,1,1) or, if final, fp32 logits in client
-// memory.
+// Global average pool (+ optional DenseNet prologue).  8 threads per 8-channel
+// granule split the pixels and reduce with shuffles; the output is either an
+// activation (C,1,1) or, if final, fp32 logits in client memory.
 // ---------------------------------------------------------------------------
 template <typename T, bool INSTR>
-__global__ void __launch_bounds__(128) k_gap(const __grid_constant__ LayerArgs a,
+__global__ void __launch_bounds__(256) k_gap(const __grid_constant__ LayerArgs a,
                                              const __grid_constant__ InstrArgs ia) {
   instr_enter<INSTR>(ia);
   const T* X = static_cast<const T*>(a.in);
   uint32_t ng = a.cout / 8;
-  uint32_t g = blockIdx.x * blockDim.x + threadIdx.x;
+  uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
+  uint32_t g = tid / 8, l = tid % 8;
+  float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  const uint32_t HW = a.h * a.w_;
   if (g < ng) {
     int c = g * 8;
-    float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-    uint32_t HW = a.h * a.w_;
-    for (uint32_t p = 0; p < HW; ++p) {
+    float sc[8], sh[8];
+    if (a.flags & LF_PROLOGUE) {
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        sc[i] = a.pro_scale[c + i];
+        sh[i] = a.pro_shift[c + i];
+      }
+    }
+#pragma unroll 4
+    for (uint32_t p = l; p < HW; p += 8) {
       float xv[8];
       load8(X + (size_t)p * a.in_cs + a.in_co + c, xv);
       if (a.flags & LF_PROLOGUE) {
 #pragma unroll
-        for (int i = 0; i < 8; ++i) xv[i] = fmaxf(fmaf(a.pro_scale[c + i], xv[i], a.pro_shift[c + i]), 0.f);
+        for (int i = 0; i < 8; ++i) xv[i] = fmaxf(fmaf(sc[i], xv[i], sh[i]), 0.f);
       }
 #pragma unroll
       for (int i = 0; i < 8; ++i) acc[i] += xv[i];
     }
+  }
+#pragma unroll
+  for (int o = 4; o > 0; o >>= 1)
+#pragma unroll
+    for (int i = 0; i < 8; ++i) acc[i] += __shfl_xor_sync(0xffffffffu, acc[i], o);
+  if (g < ng && l == 0) {
+    int c = g * 8;
     float inv = 1.f / (float)HW;
 #pragma unroll
     for (int i = 0; i < 8; ++i) acc[i] *= inv;

@@ -130,11 +130,44 @@ __device__ __forceinline__ float act_tc(float x, uint32_t act) {
 
 }  // namespace
 
+// epilogue of one (pixel, 8-channel group) item: bias, residual (fp32), activation,
+// one RNE rounding, one 16-byte store
+__device__ __forceinline__ void epi_store8(const LayerArgs& a, uint32_t p, uint32_t co, const float (&v)[8]) {
+  float x[8];
+  const float4 b0 = __ldg(reinterpret_cast<const float4*>(a.bias + co));
+  const float4 b1 = __ldg(reinterpret_cast<const float4*>(a.bias + co + 4));
+  x[0] = v[0] + b0.x; x[1] = v[1] + b0.y; x[2] = v[2] + b0.z; x[3] = v[3] + b0.w;
+  x[4] = v[4] + b1.x; x[5] = v[5] + b1.y; x[6] = v[6] + b1.z; x[7] = v[7] + b1.w;
+  if (a.flags & LF_RESIDUAL) {
+    uint4 u = *reinterpret_cast<const uint4*>(static_cast<const __nv_bfloat16*>(a.res) + (size_t)p * a.res_cs +
+                                              a.res_co + co);
+    const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&u);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      float2 f = __bfloat1622float2(h[i]);
+      x[2 * i] += f.x;
+      x[2 * i + 1] += f.y;
+    }
+  }
+  uint4 o;
+  __nv_bfloat162* oh = reinterpret_cast<__nv_bfloat162*>(&o);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) oh[i] = __floats2bfloat162_rn(act_tc(x[2 * i], a.act), act_tc(x[2 * i + 1], a.act));
+  *reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(a.out) + (size_t)p * a.out_cs + a.out_co + co) = o;
+}
+
 template <bool INSTR>
 __global__ void __launch_bounds__(TC_THREADS, 1)
     k_conv_tc(const __grid_constant__ LayerArgs a, const __grid_constant__ InstrArgs ia,
               const __grid_constant__ CUtensorMap wmap) {
-  instr_enter<INSTR>(ia);
+  const bool trace = (a.flags & LF_TRACE) != 0;
+  uint64_t* tr = trace ? reinterpret_cast<uint64_t*>(a.ws) +
+                             8 * ((blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x)
+                       : nullptr;
+  if (trace && threadIdx.x == 0) tr[0] = globaltimer();
+  // the instrumentation runs on an otherwise idle lane of the MMA warp, so neither
+  // the TMA issuer nor the gather warps wait on its atomics (instr.cuh)
+  instr_enter<INSTR, NPROD + 1>(ia);
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   uint8_t* sA = smem;                                  // STAGES x 16 KiB
@@ -143,6 +176,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   uint64_t* empty = full + TC_STAGES;
   uint64_t* accb = empty + TC_STAGES;
   uint32_t* tmem_slot = (uint32_t*)(accb + 1);
+  float* stage = reinterpret_cast<float*>(smem);       // epilogue tile [64 px][128 ch] fp32 (reuses sA)
 
   const uint32_t warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const uint32_t tile_n = blockIdx.x, tile_m = blockIdx.y, split = blockIdx.z;
@@ -163,22 +197,14 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(&wmap) : "memory");
   }
-  if (warp == 0) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(su32(tmem_slot)),
-                 "r"(64u)
-                 : "memory");
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
-  }
-  tc_fence_before();
   __syncthreads();
-  tc_fence_after();
-  const uint32_t tmem = *tmem_slot;
+  if (trace && threadIdx.x == 0) tr[1] = globaltimer();
 
   if (warp < 4) {
     // ------------------------------------------------------------ producers
     const __nv_bfloat16* X = static_cast<const __nv_bfloat16*>(a.in);
     const uint32_t t = threadIdx.x;
-    // rows (pixels) of this thread: n = t/8 + 16*j, chunk = t%8
+    // rows (pixels) of this thread: n = t/8 + 16*j, 16-byte chunk = t%8
     const uint32_t chunk = t % 8;
     int ohs[4], ows[4];
     bool pv[4];
@@ -230,113 +256,106 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     cp_async_wait<0>();
     fence_proxy_async();
     for (uint32_t it = (nkl > LOOK ? nkl - LOOK : 0); it < nkl; ++it) mbar_arrive(&full[it % TC_STAGES]);
-  } else if (lane == 0) {
-    // ------------------------------------------------------------ MMA issuer
-    constexpr uint32_t IDESC = idesc_bf16(TC_BM, TC_BN);
-    for (uint32_t it = 0; it < nkl; ++it) {
-      const uint32_t s = it % TC_STAGES;
-      mbar_wait(&full[s], (it / TC_STAGES) & 1);
-      tc_fence_after();
-      const uint32_t abase = su32(sA + s * A_BYTES), bbase = su32(sB + s * B_BYTES);
+  } else {
+    // ------------------------------------------------------------ MMA warp
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(su32(tmem_slot)),
+                 "r"(64u)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    tc_fence_before();
+    __syncwarp();
+    tc_fence_after();
+    const uint32_t tmem = *tmem_slot;
+    if (lane == 0) {
+      constexpr uint32_t IDESC = idesc_bf16(TC_BM, TC_BN);
+      for (uint32_t it = 0; it < nkl; ++it) {
+        const uint32_t s = it % TC_STAGES;
+        mbar_wait(&full[s], (it / TC_STAGES) & 1);
+        if (trace && it == 0) tr[2] = globaltimer();
+        tc_fence_after();
+        const uint32_t abase = su32(sA + s * A_BYTES), bbase = su32(sB + s * B_BYTES);
 #pragma unroll
-      for (uint32_t kk = 0; kk < TC_BK / 16; ++kk) {
-        umma_bf16(tmem, sdesc_sw128(abase + kk * 32), sdesc_sw128(bbase + kk * 32), IDESC,
-                  (it | kk) != 0 ? 1u : 0u);
+        for (uint32_t kk = 0; kk < TC_BK / 16; ++kk) {
+          umma_bf16(tmem, sdesc_sw128(abase + kk * 32), sdesc_sw128(bbase + kk * 32), IDESC,
+                    (it | kk) != 0 ? 1u : 0u);
+        }
+        umma_commit(&empty[s]);
       }
-      umma_commit(&empty[s]);
+      umma_commit(accb);   // also orders the TMEM address write before the epilogue's read
+      if (trace) tr[3] = globaltimer();
     }
-    umma_commit(accb);
+    __syncwarp();
   }
 
   // ---------------------------------------------------------------- epilogue
+  // 1. TMEM -> registers (warp w owns lanes = output channels 32w..32w+31) -> fp32
+  //    tile in shared memory [pixel][channel] (conflict-free: a warp writes 32
+  //    consecutive words of one pixel row)
   if (warp < 4) {
-    const uint32_t row = warp * 32 + lane;          // output channel within the tile
-    const uint32_t co = m0 + row;
-    const uint32_t taddr = tmem + ((warp * 32) << 16);
-    float acc[64];
+    const uint32_t row = warp * 32 + lane;
     if (nkl > 0) {
       mbar_wait(accb, 0);
+      if (trace && threadIdx.x == 0) tr[4] = globaltimer();
       tc_fence_after();
+      const uint32_t taddr = *tmem_slot + ((warp * 32) << 16);
 #pragma unroll
       for (int c = 0; c < 4; ++c) {
         float v[16];
         tmem_ld16(taddr + c * 16, v);
 #pragma unroll
-        for (int i = 0; i < 16; ++i) acc[c * 16 + i] = v[i];
+        for (int i = 0; i < 16; ++i) stage[(c * 16 + i) * TC_BM + row] = v[i];
       }
     } else {
-#pragma unroll
-      for (int i = 0; i < 64; ++i) acc[i] = 0.f;
-    }
-    if (a.ksplit == 1) {
-      if (co < a.cout) {
-        const float b = a.bias[co];
-        __nv_bfloat16* Y = static_cast<__nv_bfloat16*>(a.out);
-        const __nv_bfloat16* R = static_cast<const __nv_bfloat16*>(a.res);
-        const bool has_res = (a.flags & LF_RESIDUAL) != 0;
-#pragma unroll
-        for (int j = 0; j < 64; ++j) {
-          const uint32_t p = n0 + j;
-          if (p < P) {
-            float v = acc[j] + b;
-            if (has_res) v += __bfloat162float(R[(size_t)p * a.res_cs + a.res_co + co]);
-            Y[(size_t)p * a.out_cs + a.out_co + co] = __float2bfloat16_rn(act_tc(v, a.act));
-          }
-        }
-      }
-    } else {
-      // split-K across the CTAs of a cluster (cluster dims 1 x 1 x ksplit): every CTA
-      // parks its fp32 partial tile in its own shared memory (the drained pipeline
-      // buffers), then reduces a 1/ksplit slice of the tile over DSMEM and runs the
-      // epilogue for it -- no global workspace, no atomics.
-      float* part = reinterpret_cast<float*>(smem);   // [128 rows][64 cols]
-#pragma unroll
-      for (int i = 0; i < 64; i += 4)
-        *reinterpret_cast<float4*>(part + row * 64 + ((i + 4 * (row & 15)) & 63)) =
-            make_float4(acc[i], acc[i + 1], acc[i + 2], acc[i + 3]);
+#pragma unroll 8
+      for (int j = 0; j < 64; ++j) stage[j * TC_BM + row] = 0.f;
     }
   }
-  if (a.ksplit > 1) {
+  if (a.ksplit == 1) {
+    // 2. coalesced epilogue: item = (pixel, 8-channel group), 16-byte loads/stores
+    if (warp < 4) {
+      asm volatile("bar.sync 1, 128;" ::: "memory");   // the 4 epilogue warps only
+      for (uint32_t item = threadIdx.x; item < TC_BN * (TC_BM / 8); item += NPROD) {
+        const uint32_t px = item / (TC_BM / 8), g = item % (TC_BM / 8);
+        const uint32_t p = n0 + px, co = m0 + g * 8;
+        if (p < P && co < a.cout) {
+          const float4* q = reinterpret_cast<const float4*>(stage + px * TC_BM + g * 8);
+          float4 u0 = q[0], u1 = q[1];
+          float v[8] = {u0.x, u0.y, u0.z, u0.w, u1.x, u1.y, u1.z, u1.w};
+          epi_store8(a, p, co, v);
+        }
+      }
+    }
+  } else {
+    // split-K across the CTAs of a cluster (1 x 1 x ksplit): each CTA reduces a
+    // 1/ksplit slice of the tile's pixel rows over DSMEM (16-byte loads) and runs the
+    // epilogue for it -- no global workspace, no atomics.
     __syncwarp();
     asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
     if (warp < 4) {
       const uint32_t ks = a.ksplit;
-      const uint32_t per_thr = 64 / ks;               // elements of the tile per thread
-      const uint32_t e0 = split * (8192 / ks) + threadIdx.x * per_thr;
-      const uint32_t row = e0 / 64, col0 = e0 % 64;   // per_thr <= 64 stays inside one row
-      const uint32_t part_addr = su32(smem);
-      float sum[32];
-#pragma unroll
-      for (int i = 0; i < 32; ++i) sum[i] = 0.f;
-      for (uint32_t r = 0; r < ks; ++r) {
-        uint32_t peer;
-        asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(peer) : "r"(part_addr), "r"(r));
-        for (uint32_t i = 0; i < per_thr; i += 4) {
-          const uint32_t c = col0 + i;
-          const uint32_t addr = peer + (row * 64 + ((c + 4 * (row & 15)) & 63)) * 4;
-          float x0, x1, x2, x3;
-          asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
-                       : "=f"(x0), "=f"(x1), "=f"(x2), "=f"(x3)
-                       : "r"(addr));
-          sum[i] += x0;
-          sum[i + 1] += x1;
-          sum[i + 2] += x2;
-          sum[i + 3] += x3;
-        }
-      }
-      const uint32_t co = m0 + row;
-      if (co < a.cout) {
-        const float b = a.bias[co];
-        __nv_bfloat16* Y = static_cast<__nv_bfloat16*>(a.out);
-        const __nv_bfloat16* R = static_cast<const __nv_bfloat16*>(a.res);
-        const bool has_res = (a.flags & LF_RESIDUAL) != 0;
-        for (uint32_t i = 0; i < per_thr; ++i) {
-          const uint32_t p = n0 + col0 + i;
-          if (p < P) {
-            float v = sum[i] + b;
-            if (has_res) v += __bfloat162float(R[(size_t)p * a.res_cs + a.res_co + co]);
-            Y[(size_t)p * a.out_cs + a.out_co + co] = __float2bfloat16_rn(act_tc(v, a.act));
+      const uint32_t rows = TC_BN / ks;
+      const uint32_t px0 = split * rows;
+      const uint32_t base = su32(stage);
+      for (uint32_t item = threadIdx.x; item < rows * (TC_BM / 8); item += NPROD) {
+        const uint32_t px = px0 + item / (TC_BM / 8), g = item % (TC_BM / 8);
+        const uint32_t p = n0 + px, co = m0 + g * 8;
+        if (p < P && co < a.cout) {
+          float v[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+          const uint32_t off = (px * TC_BM + g * 8) * 4;
+          for (uint32_t r = 0; r < ks; ++r) {
+            uint32_t peer;
+            asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(peer) : "r"(base + off), "r"(r));
+            float x0, x1, x2, x3, x4, x5, x6, x7;
+            asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
+                         : "=f"(x0), "=f"(x1), "=f"(x2), "=f"(x3)
+                         : "r"(peer));
+            asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
+                         : "=f"(x4), "=f"(x5), "=f"(x6), "=f"(x7)
+                         : "r"(peer + 16));
+            v[0] += x0; v[1] += x1; v[2] += x2; v[3] += x3;
+            v[4] += x4; v[5] += x5; v[6] += x6; v[7] += x7;
           }
+          epi_store8(a, p, co, v);
         }
       }
     }
@@ -344,13 +363,16 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     __syncwarp();
     asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
   }
+  if (trace && threadIdx.x == 0) tr[5] = globaltimer();
   tc_fence_before();
   __syncthreads();
-  if (warp == 0) {
+  if (warp == 4) {
     tc_fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(64u) : "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tmem_slot), "r"(64u) : "memory");
   }
-  instr_exit<INSTR>(ia);
+  if (trace && threadIdx.x == 0) tr[6] = globaltimer();
+  instr_exit<INSTR, NPROD + 1>(ia);
+  if (trace && threadIdx.x == NPROD + 1) tr[7] = globaltimer();
 }
 
 uint32_t tc_smem_bytes() { return 1024 + TC_STAGES * (A_BYTES + B_BYTES) + 128; }

@@ -311,8 +311,8 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
       case PAELLA_OP_GAP: {
         k.kind = KIND_GAP;
         if (nd.c != sn.c || sn.c % 8) return -EINVAL;
-        k.grid[0] = (nd.c / 8 + 127) / 128;
-        k.block = 128;
+        k.grid[0] = (nd.c + 255) / 256;   // 8 threads per 8-channel granule
+        k.block = 256;
         k.bytes = (uint64_t)sn.h * sn.w * sn.c * es + (uint64_t)nd.c * ((a.flags & LF_FINAL) ? 4 : es);
         break;
       }

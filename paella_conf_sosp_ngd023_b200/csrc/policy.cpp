@@ -22,13 +22,32 @@ void Policy::add_model(uint32_t mid, const std::vector<PolicyLayer>& layers) {
   models_[mid] = layers;
 }
 
+bool Policy::is_ready(const PolicyJob& j) const {
+  if (!j.live || j.cursor >= models_[j.model].size()) return false;
+  uint32_t infl = j.inflight();
+  if (infl == 0) return true;
+  if (cfg_.lookahead == 0 || infl > cfg_.lookahead) return false;
+  const PolicyLaunch& L = launches_[j.last_uid % kLaunchSlots];
+  if (!L.live || L.uid != j.last_uid) return false;
+  return (L.p > L.f ? L.p : L.f) >= L.grid;   // most recent kernel fully placed
+}
+
+// bring the ready structures in line with is_ready(j)
+void Policy::refresh(PolicyJob& j) {
+  bool r = is_ready(j);
+  if (r && !j.in_ready) make_ready(j);
+  else if (!r && j.in_ready) make_unready(j);
+}
+
 void Policy::make_ready(PolicyJob& j) {
+  j.in_ready = true;
   srpt_.emplace(j.R, j.seq, j.id);
   fifo_.emplace(j.seq, j.id);
   per_client_[j.client].emplace(j.seq, j.id);
 }
 
 void Policy::make_unready(PolicyJob& j) {
+  j.in_ready = false;
   srpt_.erase(std::make_tuple(j.R, j.seq, j.id));
   fifo_.erase(std::make_pair(j.seq, j.id));
   per_client_[j.client].erase(std::make_pair(j.seq, j.id));
@@ -50,7 +69,7 @@ void Policy::arrival(uint32_t job_id, uint32_t client, uint32_t model) {
   j.live = true;
   work_ += R;
   live_jobs_ += 1;
-  make_ready(j);
+  refresh(j);
 }
 
 bool Policy::record(uint32_t type, uint32_t uid, uint32_t n, int64_t* job_done) {
@@ -71,20 +90,26 @@ bool Policy::record(uint32_t type, uint32_t uid, uint32_t n, int64_t* job_done) 
   uint32_t now = L.p > L.f ? L.p : L.f;
   Q_ -= (int64_t)(now - old);
   if (L.p > L.grid || L.f > L.grid) throw std::runtime_error("record count exceeds grid");
-  if (L.f != L.grid) return false;
-  L.live = false;
-  free_[L.stream / 64] |= 1ull << (L.stream % 64);
   PolicyJob& j = jobs_[L.job];
-  j.inflight = false;
-  j.cursor += 1;
-  j.last_stream = (int32_t)L.stream;
-  if (j.cursor == models_[j.model].size()) {
+  if (L.f != L.grid) {
+    if (cfg_.lookahead) refresh(j);   // a fully placed predecessor may free a launch-ahead
+    return false;
+  }
+  L.live = false;
+  j.done += 1;
+  if (j.inflight() == 0) {
+    free_[L.stream / 64] |= 1ull << (L.stream % 64);
+    j.stream = -1;
+    j.last_stream = (int32_t)L.stream;
+  }
+  if (j.done == models_[j.model].size()) {
+    if (j.in_ready) make_unready(j);
     j.live = false;
     unfinished_[j.client] -= 1;
     live_jobs_ -= 1;
     *job_done = j.id;
   } else {
-    make_ready(j);
+    refresh(j);
   }
   return true;
 }
@@ -138,18 +163,24 @@ bool Policy::predicate(uint32_t grid) const {
 
 void Policy::decide(std::vector<Issue>* out) {
   for (;;) {
-    int s0 = lowest_free();
-    if (s0 < 0) break;
     uint32_t jid;
     if (!pick(&jid)) break;
     PolicyJob& j = jobs_[jid];
+    int s0 = lowest_free();
+    if (j.inflight() == 0 && s0 < 0) break;
     const PolicyLayer& lay = models_[j.model][j.cursor];
     if (!predicate(lay.grid)) break;
     uint32_t uid = next_uid_++;
-    uint32_t stream = (uint32_t)s0;
-    if (j.last_stream >= 0 && (free_[j.last_stream / 64] >> (j.last_stream % 64) & 1))
-      stream = (uint32_t)j.last_stream;
-    free_[stream / 64] &= ~(1ull << (stream % 64));
+    uint32_t stream;
+    if (j.inflight() > 0) {
+      stream = (uint32_t)j.stream;   // launch-ahead: queued behind its predecessor
+    } else {
+      stream = (uint32_t)s0;
+      if (j.last_stream >= 0 && (free_[j.last_stream / 64] >> (j.last_stream % 64) & 1))
+        stream = (uint32_t)j.last_stream;
+      free_[stream / 64] &= ~(1ull << (stream % 64));
+      j.stream = (int32_t)stream;
+    }
     PolicyLaunch& L = launches_[uid % kLaunchSlots];
     if (L.live) throw std::runtime_error("launch slot table overflow");
     L.uid = uid;
@@ -165,10 +196,12 @@ void Policy::decide(std::vector<Issue>* out) {
     make_unready(j);
     j.R -= lay.tbar;
     work_ -= lay.tbar;
-    j.inflight = true;
+    j.cursor += 1;
+    j.last_uid = uid;
     Dt_[j.client] -= (int64_t)cfg_.num_clients;
     Omega_ += 1;
     out->push_back(Issue{uid, jid, L.layer, stream});
+    refresh(j);   // not ready until its new kernel is fully placed
   }
 }
 

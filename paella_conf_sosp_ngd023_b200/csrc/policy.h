@@ -37,10 +37,14 @@ struct PolicyJob {
   uint32_t client = 0, model = 0;
   uint64_t seq = 0;
   int64_t R = 0;
-  uint32_t cursor = 0;
-  bool inflight = false;
-  bool live = false;
+  uint32_t cursor = 0;       // next kernel to issue (kernels dispatched)
+  uint32_t done = 0;         // kernels completed
+  int32_t stream = -1;       // stream held while kernels are in flight
   int32_t last_stream = -1;
+  uint32_t last_uid = 0;
+  bool live = false;
+  bool in_ready = false;
+  uint32_t inflight() const { return cursor - done; }
 };
 
 struct PolicyLaunch {
@@ -65,6 +69,7 @@ class Policy {
     int64_t ring_capacity = 65536;
     uint32_t streams = 32;
     int64_t capacity[NRES] = {148 * 32, 148 * 64, 148 * 65536, 148 * 233472, 148 * 512};
+    uint32_t lookahead = 0;   // NEXT-1 launch-ahead depth (0 = the paper's semantics)
   };
 
   explicit Policy(const Cfg& c);
@@ -94,6 +99,8 @@ class Policy {
   bool predicate(uint32_t grid) const;
   void make_ready(PolicyJob& j);
   void make_unready(PolicyJob& j);
+  bool is_ready(const PolicyJob& j) const;
+  void refresh(PolicyJob& j);
   int lowest_free() const;
 
   Cfg cfg_;

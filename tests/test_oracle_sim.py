@@ -156,16 +156,17 @@ def random_trace(r, n, n_clients, n_models, rate_ns=3000):
     return out
 
 
+@pytest.mark.parametrize("lookahead", [0, 1])
 @pytest.mark.parametrize("policy", [sim.SRPT_DEFICIT, sim.FIFO])
 @pytest.mark.parametrize("seed", range(6))
-def test_S5_invariants_and_S6_self_replay(seed, policy):
+def test_S5_invariants_and_S6_self_replay(seed, policy, lookahead):
     r = random.Random(seed)
     models = random_models(r)
     gpu = GPUModel(sms=8, per_sm=(32, 64, 65536, 233472, 512), launch_delay=700, notif_delay=900)
     N = 3
     cfg = Config(num_clients=N, policy=policy, theta=r.choice([0, 1, 5, 100]), slack=r.choice([0, 8, 16]),
                  group=r.choice([1, 4, 16]), ring_capacity=256, streams=r.choice([4, 32]),
-                 capacity=tuple(8 * x for x in (32, 64, 65536, 233472, 512)))
+                 capacity=tuple(8 * x for x in (32, 64, 65536, 233472, 512)), lookahead=lookahead)
     trace = random_trace(r, 150, N, len(models))
     res = sim.simulate(cfg, models, trace, gpu)
     assert not res.violations                                  # (a) per-SM capacity
@@ -177,9 +178,15 @@ def test_S5_invariants_and_S6_self_replay(seed, policy):
     assert sim.check_exactly_once(res.records, grids, cfg.group) == []
     # (c) dependency: kernel k+1 of a job issued after kernel k's last completion
     last_done = {}
+    placed = {}
+    first_place_done = {}
     for (t, typ, uid, n, grp) in res.records:
         if typ == sim.COMPLETION:
             last_done[uid] = t
+        else:
+            placed[uid] = placed.get(uid, 0) + n
+            if uid in grids and placed[uid] == grids[uid]:
+                first_place_done[uid] = t
     by_job = {}
     for (t, uid, jid, layer, stream) in res.issues:
         by_job.setdefault(jid, []).append((layer, t, uid))
@@ -187,7 +194,10 @@ def test_S5_invariants_and_S6_self_replay(seed, policy):
         lst.sort()
         assert [x[0] for x in lst] == list(range(len(models[trace[jid][2]])))
         for (l0, t0, u0), (l1, t1, u1) in zip(lst, lst[1:]):
-            assert t1 >= last_done[u0]
+            if lookahead == 0:
+                assert t1 >= last_done[u0]
+            else:   # launch-ahead: issued behind a fully placed predecessor on its stream
+                assert t1 >= first_place_done.get(u0, t1) or t1 >= last_done[u0]
 
 
 def _run_policy_with_log(cfg, models, trace, gpu):
@@ -204,13 +214,15 @@ def _run_policy_with_log(cfg, models, trace, gpu):
         sim.Policy.__init__ = orig
 
 
+@pytest.mark.parametrize("lookahead", [0, 1, 2])
 @pytest.mark.parametrize("seed", range(8))
-def test_S6_replay_reproduces_issue_order(seed):
+def test_S6_replay_reproduces_issue_order(seed, lookahead):
     r = random.Random(50 + seed)
     models = random_models(r)
     gpu = GPUModel(sms=4, per_sm=(32, 64, 65536, 233472, 512), launch_delay=300, notif_delay=1100)
     cfg = Config(num_clients=4, theta=r.choice([0, 3, 100]), slack=4, group=r.choice([1, 16]),
-                 ring_capacity=128, streams=8, capacity=tuple(4 * x for x in (32, 64, 65536, 233472, 512)))
+                 ring_capacity=128, streams=8, capacity=tuple(4 * x for x in (32, 64, 65536, 233472, 512)),
+                 lookahead=lookahead)
     trace = random_trace(r, 120, 4, len(models), rate_ns=2000)
     res = _run_policy_with_log(cfg, models, trace, gpu)
     log = res.policy.log
