@@ -106,6 +106,10 @@ typedef struct {
                                     final COMPLETION); D > 0 = once the previous kernel is
                                     fully placed and <= D are in flight, the next kernel is
                                     queued behind it on the same stream */
+  uint32_t launch_threads;       /* 0 = each dispatcher calls cudaLaunchKernel itself; n > 0 =
+                                    n helper threads per GPU perform the launches (stream s is
+                                    owned by helper s % n, so per-stream order is kept); the
+                                    decisions stay on the one dispatcher core */
 } paella_config_t;
 
 /* ---- model description (input to paella_register_model) ---------------- */

@@ -44,7 +44,7 @@ class Config(C.Structure):
                 ("naive", C.c_uint32), ("client_region_bytes", C.c_size_t),
                 ("dispatcher_cpus", C.POINTER(C.c_int32)), ("event_log_path", C.c_char_p),
                 ("fake_sms", C.c_uint32), ("fake_time_scale_ns", C.c_uint32), ("event_time_kind", C.c_uint32),
-                ("lookahead", C.c_uint32)]
+                ("lookahead", C.c_uint32), ("launch_threads", C.c_uint32)]
 
 
 class Node(C.Structure):
@@ -144,7 +144,8 @@ class Engine:
                  policy=POLICY_SRPT_DEFICIT, theta=100, slack=0, group=16, ring_capacity=65536,
                  streams=32, route=ROUTE_LEAST_WORK, submit_slots=1024, max_jobs_per_model=128,
                  instrument=True, naive=False, region_bytes=64 << 20, dispatcher_cpus=None,
-                 event_log=None, fake_sms=0, fake_time_scale_ns=0, event_time_kind=None, lookahead=0):
+                 event_log=None, fake_sms=0, fake_time_scale_ns=0, event_time_kind=None, lookahead=0,
+                 launch_threads=0):
         self.lib = load()
         cfg = Config()
         cfg.abi_version = ABI_VERSION
@@ -174,6 +175,7 @@ class Engine:
         cfg.fake_time_scale_ns = fake_time_scale_ns
         cfg.event_time_kind = 0 if event_time_kind is None else event_time_kind + 1
         cfg.lookahead = lookahead
+        cfg.launch_threads = launch_threads
         self.cfg = cfg
         h = C.c_void_p()
         _check(self.lib.paella_init(C.byref(cfg), C.byref(h)), "paella_init")

@@ -160,8 +160,10 @@ struct FakeBackend : Backend {
 // CUDA backend
 // ---------------------------------------------------------------------------
 // one launch of kernel k: split-K tcgen05 convs are thread-block clusters
+static bool is_tc(uint32_t kind) { return kind == KIND_CONV_TC || kind == KIND_CONV_TC_PRO; }
+
 static cudaError_t cuda_launch(KernelFn fn, const KernelInst& k, void** args, cudaStream_t s) {
-  if (k.kind == KIND_CONV_TC && k.proto.ksplit > 1) {
+  if (is_tc(k.kind) && k.proto.ksplit > 1) {
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3(k.grid[0], k.grid[1], k.grid[2]);
     cfg.blockDim = dim3(k.block);
@@ -204,13 +206,14 @@ struct CudaBackend : Backend {
     streams.resize(nstreams);
     for (auto& s : streams)
       if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess) return -EIO;
-    KernelFn tc_i[1], tc_p[1];
+    KernelFn tc_i[2], tc_p[2];
     simt_kernel_table(tab[0][1], tab[0][0], tab[1][1], tab[1][0]);
     tc_kernel_table(tc_i, tc_p);
     tab[0][1][KIND_CONV_TC] = tc_i[0];
     tab[0][0][KIND_CONV_TC] = tc_p[0];
-    tab[1][1][KIND_CONV_TC] = nullptr;
-    tab[1][0][KIND_CONV_TC] = nullptr;
+    tab[0][1][KIND_CONV_TC_PRO] = tc_i[1];
+    tab[0][0][KIND_CONV_TC_PRO] = tc_p[1];
+    for (int i = 0; i < 2; ++i) tab[1][i][KIND_CONV_TC] = tab[1][i][KIND_CONV_TC_PRO] = nullptr;
     return cudaDeviceSynchronize() == cudaSuccess ? 0 : -EIO;
   }
   ~CudaBackend() override {
@@ -275,15 +278,58 @@ static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last) {
   return ia;
 }
 
+static void launcher_push(Gpu* g, const LaunchDesc& d) {
+  Launcher* L = g->launchers[d.stream % g->launchers.size()].get();
+  while (!L->q.push(d)) {
+  }
+}
+
+// launcher thread: performs the CUDA launches of the streams it owns, in order
+static void launcher_main(Gpu* g, Launcher* L) {
+  cudaSetDevice(g->device);
+  auto* cb = static_cast<CudaBackend*>(g->be.get());
+  for (;;) {
+    LaunchDesc* d = L->q.peek();
+    if (!d) {
+      if (g->launchers_stop.load(std::memory_order_acquire) && !L->q.peek()) break;
+      continue;
+    }
+    if (d->kind == 0) {
+      void* args[3] = {(void*)&d->a, (void*)&d->ia, (void*)d->tmap};
+      cudaError_t e = cuda_launch(cb->fn(d->k->kind, d->dtype, d->instr != 0), *d->k, args, cb->streams[d->stream]);
+      if (e != cudaSuccess) g->launch_err.store((int)e);
+    } else {
+      cudaEventRecord((cudaEvent_t)d->event, cb->streams[d->stream]);
+      __atomic_store_n(d->recorded, (uint8_t)1, __ATOMIC_RELEASE);
+    }
+    L->q.pop();
+  }
+}
+
 static void do_launch(Gpu* g, Model* m, uint32_t slot, uint32_t layer, uint32_t uid, uint32_t stream, bool instr) {
   const KernelInst& k = m->kernels[layer];
   InstrArgs ia = make_instr(g, uid, k.grid_total(), layer + 1 == m->kernels.size());
   const paella_config_t& cfg = g->P->cfg;
+  if (!g->launchers.empty()) {
+    LaunchDesc d;
+    d.k = &k;
+    d.a = m->gpu[g->index].args[slot][layer];
+    d.ia = ia;
+    d.tmap = is_tc(k.kind) ? m->gpu[g->index].tmaps[layer].b : nullptr;
+    d.event = nullptr;
+    d.recorded = nullptr;
+    d.stream = stream;
+    d.dtype = m->dtype;
+    d.instr = instr ? 1 : 0;
+    d.kind = 0;
+    launcher_push(g, d);
+    return;
+  }
   Gpu::EvPair ep{nullptr, nullptr, 0, 0};
   CudaBackend* cb = nullptr;
   if (cfg.device == PAELLA_DEVICE_CUDA) {
     cb = static_cast<CudaBackend*>(g->be.get());
-    cb->cur_tmap = (k.kind == KIND_CONV_TC) ? m->gpu[g->index].tmaps[layer].b : nullptr;
+    cb->cur_tmap = is_tc(k.kind) ? m->gpu[g->index].tmaps[layer].b : nullptr;
     if (cfg.event_time_kind == k.kind + 1 && !g->ev_free.empty()) {
       ep = g->ev_free.back();
       g->ev_free.pop_back();
@@ -355,6 +401,7 @@ static bool admit(Gpu* g, uint32_t client, const SubmitSlot& s) {
     jid = g->free_job_ids.back();
     g->free_job_ids.pop_back();
   } else {
+    if (g->next_job >= g->jobs.capacity()) return false;
     jid = g->next_job++;
     g->jobs.resize(g->next_job);
   }
@@ -381,7 +428,19 @@ static bool admit(Gpu* g, uint32_t client, const SubmitSlot& s) {
       do_launch(g, m, slot, l, 0, st, false);
       g->stats.launches++;
     }
-    g->be->record_event(st, &j.event);
+    if (!g->launchers.empty()) {
+      cudaEventCreateWithFlags((cudaEvent_t*)&j.event, cudaEventDisableTiming);
+      __atomic_store_n(&j.event_recorded, (uint8_t)0, __ATOMIC_RELAXED);
+      LaunchDesc d{};
+      d.event = j.event;
+      d.recorded = &j.event_recorded;
+      d.stream = st;
+      d.kind = 1;
+      launcher_push(g, d);
+    } else {
+      g->be->record_event(st, &j.event);
+      j.event_recorded = 1;
+    }
     g->naive_inflight.push_back(jid);
   } else {
     g->policy->arrival(jid, client, s.model_id);
@@ -480,7 +539,7 @@ static void dispatcher_main(Gpu* g) {
     if (P->cfg.naive) {
       for (size_t i = 0; i < g->naive_inflight.size();) {
         uint32_t jid = g->naive_inflight[i];
-        if (g->be->event_done(g->jobs[jid].event)) {
+        if (__atomic_load_n(&g->jobs[jid].event_recorded, __ATOMIC_ACQUIRE) && g->be->event_done(g->jobs[jid].event)) {
           g->be->release_event(g->jobs[jid].event);
           finish_job(g, jid, 0);
           g->naive_inflight[i] = g->naive_inflight.back();
@@ -501,6 +560,7 @@ static void dispatcher_main(Gpu* g) {
       g->work_published.store(g->policy->outstanding_work(), std::memory_order_release);
     }
     int e = g->be->error();
+    if (!e) e = g->launch_err.load(std::memory_order_relaxed);
     if (e) {
       g->err.store(-EIO);
       // fail every live job of this GPU with -EIO
@@ -559,6 +619,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
   if (cfg.fake_time_scale_ns == 0) cfg.fake_time_scale_ns = 500;
   if (cfg.fairness_threshold < 0) return -EINVAL;
   if (cfg.lookahead > 4) return -EINVAL;
+  if (cfg.launch_threads > 16) return -EINVAL;
 
   auto P = std::make_unique<Paella>();
   P->cfg = cfg;
@@ -607,6 +668,8 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     g->cap = cfg.ring_capacity;
     g->log2cap = ilog2(cfg.ring_capacity);
     g->ctr_base.assign(NCTR, 0);
+    // never reallocated: launcher threads hold pointers into job records
+    g->jobs.reserve(65536);
     if (cfg.device == PAELLA_DEVICE_CUDA)
       g->be.reset(new CudaBackend(g->device, g->cap, cfg.stream_pool));
     else
@@ -647,7 +710,17 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     }
     P->gpus.push_back(std::move(g));
   }
-  for (auto& g : P->gpus) g->thread = std::thread(dispatcher_main, g.get());
+  for (auto& g : P->gpus) {
+    if (cfg.device == PAELLA_DEVICE_CUDA && cfg.launch_threads > 0) {
+      for (uint32_t i = 0; i < cfg.launch_threads; ++i) {
+        auto L = std::make_unique<Launcher>();
+        L->q.init(8192);
+        g->launchers.push_back(std::move(L));
+      }
+      for (auto& L : g->launchers) L->th = std::thread(launcher_main, g.get(), L.get());
+    }
+    g->thread = std::thread(dispatcher_main, g.get());
+  }
   *out = (paella_t*)P.release();
   return 0;
 }
@@ -802,6 +875,15 @@ int paella_shutdown(paella_t* p) {
   for (auto& g : P->gpus) g->stop.store(true, std::memory_order_release);
   for (auto& g : P->gpus)
     if (g->thread.joinable()) g->thread.join();
+  for (auto& g : P->gpus) {
+    g->launchers_stop.store(true, std::memory_order_release);
+    for (auto& L : g->launchers)
+      if (L->th.joinable()) L->th.join();
+    if (P->cfg.device == PAELLA_DEVICE_CUDA) {
+      cudaSetDevice(g->device);
+      cudaDeviceSynchronize();
+    }
+  }
   // requests never admitted complete with -ECANCELED
   for (auto& g : P->gpus) {
     for (uint32_t c = 0; c < P->cfg.num_clients; ++c) {
@@ -883,7 +965,7 @@ int paella_kernel_info(paella_t* p, uint32_t model_id, uint32_t k, paella_kernel
 
 const char* paella_kernel_name(uint32_t kind) {
   static const char* names[] = {"ingest", "conv_simt", "conv_tcgen05", "dwconv", "maxpool",
-                                "avgpool", "gap", "fc_gemv", "empty"};
+                                "avgpool", "gap", "fc_gemv", "empty", "conv_tcgen05_pro"};
   return kind < KIND_COUNT ? names[kind] : "?";
 }
 
@@ -940,7 +1022,7 @@ static void iso_launch(Gpu* g, Model* m, uint32_t l, bool instr) {
   ia.flags = INSTR_ON | (l + 1 == m->kernels.size() ? INSTR_LAST : 0);
   uint32_t iso_slot = (uint32_t)m->gpu[g->index].args.size() - 1;
   auto* cb = static_cast<CudaBackend*>(g->be.get());
-  const void* tm = (k.kind == KIND_CONV_TC) ? m->gpu[g->index].tmaps[l].b : nullptr;
+  const void* tm = is_tc(k.kind) ? m->gpu[g->index].tmaps[l].b : nullptr;
   void* args[3] = {(void*)&m->gpu[g->index].args[iso_slot][l], (void*)&ia, (void*)tm};
   cuda_launch(cb->fn(k.kind, m->dtype, instr), k, args, (cudaStream_t)g->prof_stream);
 }
@@ -977,9 +1059,9 @@ static int iso_run(Gpu* g, Model* m, const void* input, void* output, int64_t* k
   int trace_k = std::getenv("PAELLA_TRACE_KERNEL") ? atoi(std::getenv("PAELLA_TRACE_KERNEL")) : -1;
   uint64_t* trbuf = nullptr;
   LayerArgs saved{};
-  if (trace_k >= 0 && trace_k < (int)m->kernels.size() && m->kernels[trace_k].kind == KIND_CONV_TC) {
-    cudaMalloc(&trbuf, 8 * 8 * m->kernels[trace_k].grid_total());
-    cudaMemset(trbuf, 0, 8 * 8 * m->kernels[trace_k].grid_total());
+  if (trace_k >= 0 && trace_k < (int)m->kernels.size() && is_tc(m->kernels[trace_k].kind)) {
+    cudaMalloc(&trbuf, 16 * 8 * m->kernels[trace_k].grid_total());
+    cudaMemset(trbuf, 0, 16 * 8 * m->kernels[trace_k].grid_total());
     saved = args[trace_k];
     args[trace_k].flags |= LF_TRACE;
     args[trace_k].ws = (float*)trbuf;
@@ -1002,18 +1084,21 @@ static int iso_run(Gpu* g, Model* m, const void* input, void* output, int64_t* k
   if (trace_k >= 0) {
     cudaStreamSynchronize(s);
     uint32_t nb = m->kernels[trace_k].grid_total();
-    std::vector<uint64_t> h(8 * nb);
+    std::vector<uint64_t> h(16 * nb);
     cudaMemcpy(h.data(), trbuf, h.size() * 8, cudaMemcpyDeviceToHost);
     cudaFree(trbuf);
     args[trace_k] = saved;
     uint64_t t0 = UINT64_MAX;
-    for (uint32_t b = 0; b < nb; ++b) t0 = std::min(t0, h[8 * b]);
-    const char* names[8] = {"entry", "setup", "full0", "mma_done", "accb", "epi_done", "pre_exit", "exit"};
+    for (uint32_t b = 0; b < nb; ++b) t0 = std::min(t0, h[16 * b]);
+    const char* names[16] = {"entry", "setup", "full0", "mma_done", "accb", "epi_done", "pre_exit", "exit",
+                             "tmem2smem", "pre_bar", "post_bar", "inited", "tma_issued", "b_issued", "reduced", "-"};
     fprintf(stderr, "trace kernel %d grid %u (ns from first CTA entry): phase min/med/max\n", trace_k, nb);
-    for (int ph = 0; ph < 8; ++ph) {
+    const int order[15] = {0, 11, 12, 13, 1, 2, 3, 4, 8, 9, 10, 14, 5, 6, 7};
+    for (int oi = 0; oi < 15; ++oi) {
+      int ph = order[oi];
       std::vector<int64_t> v;
       for (uint32_t b = 0; b < nb; ++b)
-        if (h[8 * b + ph]) v.push_back((int64_t)(h[8 * b + ph] - t0));
+        if (h[16 * b + ph]) v.push_back((int64_t)(h[16 * b + ph] - t0));
       if (v.empty()) continue;
       std::sort(v.begin(), v.end());
       fprintf(stderr, "  %-9s %7lld %7lld %7lld\n", names[ph], (long long)v.front(), (long long)v[v.size() / 2],
@@ -1072,13 +1157,18 @@ static int setup_model_gpu(Paella* P, Model* m, Gpu* g) {
         cudaFuncSetAttribute((const void*)cb->fn(k.kind, m->dtype, false),
                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k.smem);
       }
+      if (is_tc(k.kind)) {   // split-K clusters of up to 16 CTAs
+        cudaFuncSetAttribute((const void*)f, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+        cudaFuncSetAttribute((const void*)cb->fn(k.kind, m->dtype, false),
+                             cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+      }
       // constant per-SM capacity for Table-1 accounting: maximum carveout (hard part #4)
       cudaFuncSetAttribute((const void*)f, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
       cudaFuncSetAttribute((const void*)cb->fn(k.kind, m->dtype, false),
                            cudaFuncAttributePreferredSharedMemoryCarveout, 100);
       k.regs = (uint32_t)fa.numRegs;
       k.static_smem = (uint32_t)fa.sharedSizeBytes;
-      if (k.kind == KIND_CONV_TC) {
+      if (is_tc(k.kind)) {
         if (make_weight_tmap(wdev + k.w_off, k.proto.tiles_m * TC_BM, k.proto.kpad, tmaps[l].b)) return -EIO;
       }
     } else {
@@ -1248,7 +1338,7 @@ int paella_time_kernels(paella_t* p, uint32_t gpu, uint32_t model_id, uint32_t i
     *gate = 0;
     launch_gate(g, gd);
     cudaEventRecord(e0, s);
-    const void* tm = (k.kind == KIND_CONV_TC) ? m->gpu[gpu].tmaps[l].b : nullptr;
+    const void* tm = is_tc(k.kind) ? m->gpu[gpu].tmaps[l].b : nullptr;
     for (uint32_t r = 0; r < std::min(reps, 256u); ++r) {
       InstrArgs ia = iso_instr(g, k.grid_total(), P->cfg.group_size, l + 1 == m->kernels.size());
       void* args[3] = {(void*)&m->gpu[gpu].args[iso_slot][l], (void*)&ia, (void*)tm};

@@ -82,9 +82,53 @@ struct JobRec {
   // naive mode
   uint32_t stream = 0;
   void* event = nullptr;
+  uint8_t event_recorded = 0;  // set by the launcher thread (__atomic builtins)
 };
 
 struct Paella;
+
+// a launch handed from the dispatcher to a launcher thread
+struct LaunchDesc {
+  const KernelInst* k;
+  LayerArgs a;
+  InstrArgs ia;
+  const void* tmap;
+  void* event;                 // kind 1: record this event on the stream
+  uint8_t* recorded;
+  uint32_t stream, dtype;
+  uint8_t instr, kind;         // kind 0 = kernel, 1 = event record
+};
+
+// plain (in-process) single-producer / single-consumer queue
+template <typename T>
+struct SpscQ {
+  std::vector<T> buf;
+  uint64_t mask = 0;
+  alignas(64) std::atomic<uint64_t> tail{0};
+  alignas(64) std::atomic<uint64_t> head{0};
+  void init(uint64_t cap) {
+    buf.resize(cap);
+    mask = cap - 1;
+  }
+  bool push(const T& v) {
+    uint64_t t = tail.load(std::memory_order_relaxed);
+    if (t - head.load(std::memory_order_acquire) > mask) return false;
+    buf[t & mask] = v;
+    tail.store(t + 1, std::memory_order_release);
+    return true;
+  }
+  T* peek() {
+    uint64_t h = head.load(std::memory_order_relaxed);
+    if (h == tail.load(std::memory_order_acquire)) return nullptr;
+    return &buf[h & mask];
+  }
+  void pop() { head.store(head.load(std::memory_order_relaxed) + 1, std::memory_order_release); }
+};
+
+struct Launcher {
+  SpscQ<LaunchDesc> q;
+  std::thread th;
+};
 
 // device backend: real CUDA GPU or CPU fake
 struct Backend {
@@ -151,6 +195,10 @@ struct Gpu {
   std::vector<EvPair> ev_free;
   std::vector<EvPair> ev_pending;   // FIFO by launch order
   size_t ev_head = 0;
+  // launcher threads (cfg.launch_threads)
+  std::vector<std::unique_ptr<Launcher>> launchers;
+  std::atomic<bool> launchers_stop{false};
+  std::atomic<int> launch_err{0};
 };
 
 struct Paella {

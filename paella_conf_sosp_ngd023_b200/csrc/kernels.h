@@ -14,7 +14,8 @@ enum KernelKind : uint32_t {
   KIND_GAP = 6,
   KIND_FC = 7,
   KIND_EMPTY = 8,
-  KIND_COUNT = 9,
+  KIND_CONV_TC_PRO = 9, // tcgen05 conv with the per-channel affine+ReLU input prologue
+  KIND_COUNT = 10,
 };
 
 typedef void (*KernelFn)();
@@ -24,7 +25,7 @@ void simt_kernel_table(KernelFn (&bf16_instr)[KIND_COUNT], KernelFn (&bf16_plain
 
 KernelFn gate_kernel();   // k_gate(const volatile uint32_t* flag)
 
-// tcgen05 conv: instrumented / plain instantiations and their launch geometry
+// tcgen05 conv: instrumented / plain instantiations [0] plain input, [1] prologue
 void tc_kernel_table(KernelFn* instr, KernelFn* plain);
 constexpr uint32_t TC_BM = 128;       // Cout rows per CTA (UMMA M, TMEM lanes)
 constexpr uint32_t TC_BN = 64;        // output pixels per CTA (UMMA N)

@@ -36,7 +36,6 @@ namespace {
 
 constexpr uint32_t A_BYTES = TC_BM * TC_BK * 2;   // 16 KiB
 constexpr uint32_t B_BYTES = TC_BN * TC_BK * 2;   // 8 KiB
-constexpr uint32_t LOOK = 2;                      // cp.async groups in flight per producer
 constexpr uint32_t NPROD = 128;                   // producer threads (warps 0-3)
 
 __device__ __forceinline__ uint32_t su32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -132,16 +131,13 @@ __device__ __forceinline__ float act_tc(float x, uint32_t act) {
 
 // epilogue of one (pixel, 8-channel group) item: bias, residual (fp32), activation,
 // one RNE rounding, one 16-byte store
-__device__ __forceinline__ void epi_store8(const LayerArgs& a, uint32_t p, uint32_t co, const float (&v)[8]) {
+__device__ __forceinline__ void epi_store8(const LayerArgs& a, uint32_t p, uint32_t co, const float (&v)[8],
+                                           const float (&bias)[8], const uint4& res) {
   float x[8];
-  const float4 b0 = __ldg(reinterpret_cast<const float4*>(a.bias + co));
-  const float4 b1 = __ldg(reinterpret_cast<const float4*>(a.bias + co + 4));
-  x[0] = v[0] + b0.x; x[1] = v[1] + b0.y; x[2] = v[2] + b0.z; x[3] = v[3] + b0.w;
-  x[4] = v[4] + b1.x; x[5] = v[5] + b1.y; x[6] = v[6] + b1.z; x[7] = v[7] + b1.w;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) x[i] = v[i] + bias[i];
   if (a.flags & LF_RESIDUAL) {
-    uint4 u = *reinterpret_cast<const uint4*>(static_cast<const __nv_bfloat16*>(a.res) + (size_t)p * a.res_cs +
-                                              a.res_co + co);
-    const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&u);
+    const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&res);
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
       float2 f = __bfloat1622float2(h[i]);
@@ -156,13 +152,27 @@ __device__ __forceinline__ void epi_store8(const LayerArgs& a, uint32_t p, uint3
   *reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(a.out) + (size_t)p * a.out_cs + a.out_co + co) = o;
 }
 
-template <bool INSTR>
+__device__ __forceinline__ void load_bias8(const LayerArgs& a, uint32_t co, float (&b)[8]) {
+  if (co < a.cout) {
+    const float4 b0 = __ldg(reinterpret_cast<const float4*>(a.bias + co));
+    const float4 b1 = __ldg(reinterpret_cast<const float4*>(a.bias + co + 4));
+    b[0] = b0.x; b[1] = b0.y; b[2] = b0.z; b[3] = b0.w;
+    b[4] = b1.x; b[5] = b1.y; b[6] = b1.z; b[7] = b1.w;
+  }
+}
+
+__device__ __forceinline__ uint4 load_res8(const LayerArgs& a, uint32_t p, uint32_t co) {
+  return __ldg(reinterpret_cast<const uint4*>(static_cast<const __nv_bfloat16*>(a.res) + (size_t)p * a.res_cs +
+                                              a.res_co + co));
+}
+
+template <bool INSTR, bool PRO>
 __global__ void __launch_bounds__(TC_THREADS, 1)
     k_conv_tc(const __grid_constant__ LayerArgs a, const __grid_constant__ InstrArgs ia,
               const __grid_constant__ CUtensorMap wmap) {
   const bool trace = (a.flags & LF_TRACE) != 0;
   uint64_t* tr = trace ? reinterpret_cast<uint64_t*>(a.ws) +
-                             8 * ((blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x)
+                             16 * ((blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x)
                        : nullptr;
   if (trace && threadIdx.x == 0) tr[0] = globaltimer();
   // the instrumentation runs on an otherwise idle lane of the MMA warp, so neither
@@ -188,74 +198,129 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   const uint32_t kb1 = min(nk, kb0 + per);
   const uint32_t nkl = kb1 > kb0 ? kb1 - kb0 : 0;
 
-  if (threadIdx.x == 0) {
+  const uint32_t pre = nkl < TC_STAGES ? nkl : TC_STAGES;
+  if (warp == 4 && lane == 0) {
+    // the MMA warp's leader sets up the barriers and starts the weight stream while
+    // the gather warps compute their addresses
     for (uint32_t s = 0; s < TC_STAGES; ++s) {
       mbar_init(&full[s], NPROD + 1);
       mbar_init(&empty[s], 1);
     }
     mbar_init(accb, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    asm volatile("prefetch.tensormap [%0];" ::"l"(&wmap) : "memory");
+    if (trace) tr[11] = globaltimer();
+    for (uint32_t it = 0; it < pre; ++it) {   // the first stages need no empty-wait
+      mbar_arrive_tx(&full[it], A_BYTES);
+      tma_load_2d(sA + it * A_BYTES, &wmap, &full[it], (int)((kb0 + it) * TC_BK), (int)m0);
+    }
+    if (trace) tr[12] = globaltimer();
+  }
+  // ---- producer state (warps 0-3): this thread gathers 16-byte chunk `chunk` of
+  // pixel rows n = t/8 + 16 j (j < 4) of every B stage
+  const __nv_bfloat16* X = static_cast<const __nv_bfloat16*>(a.in);
+  const uint32_t t = threadIdx.x;
+  const uint32_t chunk = t % 8;
+  int ohs[4], ows[4];
+  bool pv[4];
+  const uint32_t K = a.kh * a.kw * a.cin;
+  // (r, s, ci) of k = kbase + 8*chunk, advanced incrementally by TC_BK per stage
+  int kr = 0, ks_ = 0, kci = 0;
+  auto issue_B = [&](uint32_t it) {
+    const uint32_t s = it % TC_STAGES;
+    const uint32_t k = (kb0 + it) * TC_BK + chunk * 8;
+    const bool kv = k < K;
+    const uint32_t bstage = su32(sB + s * B_BYTES);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const uint32_t n = t / 8 + 16 * j;
+      const int ih = ohs[j] * (int)a.sh - (int)a.ph + kr;
+      const int iw = ows[j] * (int)a.sw - (int)a.pw + ks_;
+      const bool ok = kv && pv[j] && ih >= 0 && ih < (int)a.h && iw >= 0 && iw < (int)a.w_;
+      const __nv_bfloat16* src = ok ? X + ((size_t)ih * a.w_ + iw) * a.in_cs + a.in_co + kci : X;
+      const uint32_t dst = bstage + n * 128 + ((chunk ^ (n & 7)) << 4);
+      if constexpr (!PRO) {
+        cp_async16(dst, src, ok ? 16u : 0u);
+      } else {
+        // DenseNet pre-activation: relu(scale[c] * x + shift[c]) through registers;
+        // padding stays zero (it pads the activated tensor)
+        uint4 u = make_uint4(0, 0, 0, 0);
+        if (ok) {
+          u = __ldg(reinterpret_cast<const uint4*>(src));
+          const float4 s0 = __ldg(reinterpret_cast<const float4*>(a.pro_scale + kci));
+          const float4 s1 = __ldg(reinterpret_cast<const float4*>(a.pro_scale + kci + 4));
+          const float4 z0 = __ldg(reinterpret_cast<const float4*>(a.pro_shift + kci));
+          const float4 z1 = __ldg(reinterpret_cast<const float4*>(a.pro_shift + kci + 4));
+          const float sc[8] = {s0.x, s0.y, s0.z, s0.w, s1.x, s1.y, s1.z, s1.w};
+          const float sh[8] = {z0.x, z0.y, z0.z, z0.w, z1.x, z1.y, z1.z, z1.w};
+          __nv_bfloat162* h = reinterpret_cast<__nv_bfloat162*>(&u);
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            float2 f = __bfloat1622float2(h[i]);
+            h[i] = __floats2bfloat162_rn(fmaxf(fmaf(sc[2 * i], f.x, sh[2 * i]), 0.f),
+                                         fmaxf(fmaf(sc[2 * i + 1], f.y, sh[2 * i + 1]), 0.f));
+          }
+        }
+        asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(dst), "r"(u.x), "r"(u.y), "r"(u.z),
+                     "r"(u.w)
+                     : "memory");
+      }
+    }
+    if constexpr (!PRO) cp_async_commit();
+    // advance (r, s, ci) by TC_BK channels for the next stage
+    kci += TC_BK;
+    while (kci >= (int)a.cin) {
+      kci -= (int)a.cin;
+      if (++ks_ == (int)a.kw) {
+        ks_ = 0;
+        ++kr;
+      }
+    }
+  };
+  if (warp < 4) {
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      uint32_t p = n0 + t / 8 + 16 * j;
+      pv[j] = p < P;
+      ohs[j] = pv[j] ? (int)(p / a.ow) : 0;
+      ows[j] = pv[j] ? (int)(p % a.ow) : 0;
+    }
+    {
+      const uint32_t k0 = kb0 * TC_BK + chunk * 8;
+      kci = (int)(k0 % a.cin);
+      const int rs = (int)(k0 / a.cin);
+      ks_ = rs % (int)a.kw;
+      kr = rs / (int)a.kw;
+    }
+    // ... and the first activation gathers, before the CTA-wide barrier
+    for (uint32_t it = 0; it < pre; ++it) issue_B(it);
+    if (trace && t == 0) tr[13] = globaltimer();
   }
   __syncthreads();
   if (trace && threadIdx.x == 0) tr[1] = globaltimer();
 
   if (warp < 4) {
     // ------------------------------------------------------------ producers
-    const __nv_bfloat16* X = static_cast<const __nv_bfloat16*>(a.in);
-    const uint32_t t = threadIdx.x;
-    // rows (pixels) of this thread: n = t/8 + 16*j, 16-byte chunk = t%8
-    const uint32_t chunk = t % 8;
-    int ohs[4], ows[4];
-    bool pv[4];
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      uint32_t n = t / 8 + 16 * j;
-      uint32_t p = n0 + n;
-      pv[j] = p < P;
-      ohs[j] = pv[j] ? (int)(p / a.ow) : 0;
-      ows[j] = pv[j] ? (int)(p % a.ow) : 0;
-    }
-    const uint32_t K = a.kh * a.kw * a.cin;
     for (uint32_t it = 0; it < nkl; ++it) {
-      const uint32_t s = it % TC_STAGES;
-      const uint32_t ph = (it / TC_STAGES) & 1;
-      mbar_wait(&empty[s], ph ^ 1);
-      const uint32_t kbase = (kb0 + it) * TC_BK;
-      if (t == 0) {
-        mbar_arrive_tx(&full[s], A_BYTES);
-        tma_load_2d(sA + s * A_BYTES, &wmap, &full[s], (int)kbase, (int)m0);
+      // stage `it` has landed for this thread: make it visible to the tensor core
+      if constexpr (!PRO) {
+        if (it + TC_STAGES <= nkl)
+          cp_async_wait<TC_STAGES - 1>();
+        else
+          cp_async_wait<0>();
       }
-      const uint32_t k = kbase + chunk * 8;
-      int r = 0, sx = 0, ci = 0;
-      const bool kv = k < K;
-      if (kv) {
-        ci = (int)(k % a.cin);
-        int rs = (int)(k / a.cin);
-        sx = rs % (int)a.kw;
-        r = rs / (int)a.kw;
-      }
-      const uint32_t bstage = su32(sB + s * B_BYTES);
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const uint32_t n = t / 8 + 16 * j;
-        const int ih = ohs[j] * (int)a.sh - (int)a.ph + r;
-        const int iw = ows[j] * (int)a.sw - (int)a.pw + sx;
-        const bool ok = kv && pv[j] && ih >= 0 && ih < (int)a.h && iw >= 0 && iw < (int)a.w_;
-        const __nv_bfloat16* src = ok ? X + ((size_t)ih * a.w_ + iw) * a.in_cs + a.in_co + ci : X;
-        const uint32_t dst = bstage + n * 128 + ((chunk ^ (n & 7)) << 4);
-        cp_async16(dst, src, ok ? 16u : 0u);
-      }
-      cp_async_commit();
-      if (it >= LOOK) {
-        cp_async_wait<LOOK>();
-        fence_proxy_async();
-        mbar_arrive(&full[(it - LOOK) % TC_STAGES]);
+      fence_proxy_async();
+      mbar_arrive(&full[it % TC_STAGES]);
+      const uint32_t nxt = it + TC_STAGES;
+      if (nxt < nkl) {
+        const uint32_t s = nxt % TC_STAGES;
+        mbar_wait(&empty[s], ((nxt / TC_STAGES) & 1) ^ 1);   // MMA of stage `it` retired
+        if (t == 0) {
+          mbar_arrive_tx(&full[s], A_BYTES);
+          tma_load_2d(sA + s * A_BYTES, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
+        }
+        issue_B(nxt);
       }
     }
-    cp_async_wait<0>();
-    fence_proxy_async();
-    for (uint32_t it = (nkl > LOOK ? nkl - LOOK : 0); it < nkl; ++it) mbar_arrive(&full[it % TC_STAGES]);
   } else {
     // ------------------------------------------------------------ MMA warp
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(su32(tmem_slot)),
@@ -305,6 +370,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 #pragma unroll
         for (int i = 0; i < 16; ++i) stage[(c * 16 + i) * TC_BM + row] = v[i];
       }
+      if (trace && threadIdx.x == 0) tr[8] = globaltimer();
     } else {
 #pragma unroll 8
       for (int j = 0; j < 64; ++j) stage[j * TC_BM + row] = 0.f;
@@ -313,15 +379,32 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   if (a.ksplit == 1) {
     // 2. coalesced epilogue: item = (pixel, 8-channel group), 16-byte loads/stores
     if (warp < 4) {
+      // every item of this thread has channel group g = t % 16: one bias load; all
+      // residual loads are issued before the tile is read (latency overlap)
+      const uint32_t g = threadIdx.x % (TC_BM / 8), co = m0 + g * 8;
+      constexpr uint32_t NIT = TC_BN * (TC_BM / 8) / NPROD;   // 8 items per thread
+      float bias[8];
+      load_bias8(a, co, bias);
+      uint4 res[NIT];
+      const bool has_res = (a.flags & LF_RESIDUAL) != 0;
+#pragma unroll
+      for (uint32_t i = 0; i < NIT; ++i) {
+        const uint32_t px = (threadIdx.x + i * NPROD) / (TC_BM / 8);
+        const uint32_t p = n0 + px;
+        if (has_res && p < P && co < a.cout) res[i] = load_res8(a, p, co);
+      }
+      if (trace && threadIdx.x == 0) tr[9] = globaltimer();
       asm volatile("bar.sync 1, 128;" ::: "memory");   // the 4 epilogue warps only
-      for (uint32_t item = threadIdx.x; item < TC_BN * (TC_BM / 8); item += NPROD) {
-        const uint32_t px = item / (TC_BM / 8), g = item % (TC_BM / 8);
-        const uint32_t p = n0 + px, co = m0 + g * 8;
+      if (trace && threadIdx.x == 0) tr[10] = globaltimer();
+#pragma unroll
+      for (uint32_t i = 0; i < NIT; ++i) {
+        const uint32_t px = (threadIdx.x + i * NPROD) / (TC_BM / 8);
+        const uint32_t p = n0 + px;
         if (p < P && co < a.cout) {
           const float4* q = reinterpret_cast<const float4*>(stage + px * TC_BM + g * 8);
           float4 u0 = q[0], u1 = q[1];
           float v[8] = {u0.x, u0.y, u0.z, u0.w, u1.x, u1.y, u1.z, u1.w};
-          epi_store8(a, p, co, v);
+          epi_store8(a, p, co, v, bias, res[i]);
         }
       }
     }
@@ -330,36 +413,53 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     // 1/ksplit slice of the tile's pixel rows over DSMEM (16-byte loads) and runs the
     // epilogue for it -- no global workspace, no atomics.
     __syncwarp();
+    if (trace && threadIdx.x == 0) tr[9] = globaltimer();
     asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    if (trace && threadIdx.x == 0) tr[10] = globaltimer();
     if (warp < 4) {
       const uint32_t ks = a.ksplit;
       const uint32_t rows = TC_BN / ks;
       const uint32_t px0 = split * rows;
       const uint32_t base = su32(stage);
+      // items of this thread share channel group g = t % 16 (one bias load)
+      const uint32_t g = threadIdx.x % (TC_BM / 8), co = m0 + g * 8;
+      float bias[8];
+      load_bias8(a, co, bias);
       for (uint32_t item = threadIdx.x; item < rows * (TC_BM / 8); item += NPROD) {
-        const uint32_t px = px0 + item / (TC_BM / 8), g = item % (TC_BM / 8);
-        const uint32_t p = n0 + px, co = m0 + g * 8;
+        const uint32_t px = px0 + item / (TC_BM / 8);
+        const uint32_t p = n0 + px;
         if (p < P && co < a.cout) {
-          float v[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+          uint4 res = make_uint4(0, 0, 0, 0);
+          if (a.flags & LF_RESIDUAL) res = load_res8(a, p, co);
           const uint32_t off = (px * TC_BM + g * 8) * 4;
-          for (uint32_t r = 0; r < ks; ++r) {
-            uint32_t peer;
-            asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(peer) : "r"(base + off), "r"(r));
-            float x0, x1, x2, x3, x4, x5, x6, x7;
-            asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
-                         : "=f"(x0), "=f"(x1), "=f"(x2), "=f"(x3)
-                         : "r"(peer));
-            asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
-                         : "=f"(x4), "=f"(x5), "=f"(x6), "=f"(x7)
-                         : "r"(peer + 16));
-            v[0] += x0; v[1] += x1; v[2] += x2; v[3] += x3;
-            v[4] += x4; v[5] += x5; v[6] += x6; v[7] += x7;
+          float4 part[16][2];
+#pragma unroll
+          for (uint32_t r = 0; r < 16; ++r) {   // every peer's slice in flight at once
+            if (r < ks) {
+              uint32_t peer;
+              asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(peer) : "r"(base + off), "r"(r));
+              asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
+                           : "=f"(part[r][0].x), "=f"(part[r][0].y), "=f"(part[r][0].z), "=f"(part[r][0].w)
+                           : "r"(peer));
+              asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
+                           : "=f"(part[r][1].x), "=f"(part[r][1].y), "=f"(part[r][1].z), "=f"(part[r][1].w)
+                           : "r"(peer + 16));
+            }
           }
-          epi_store8(a, p, co, v);
+          float v[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+#pragma unroll
+          for (uint32_t r = 0; r < 16; ++r) {
+            if (r < ks) {
+              v[0] += part[r][0].x; v[1] += part[r][0].y; v[2] += part[r][0].z; v[3] += part[r][0].w;
+              v[4] += part[r][1].x; v[5] += part[r][1].y; v[6] += part[r][1].z; v[7] += part[r][1].w;
+            }
+          }
+          epi_store8(a, p, co, v, bias, res);
         }
       }
     }
     // no CTA may leave while a peer still reads its shared memory
+    if (trace && threadIdx.x == 0) tr[14] = globaltimer();
     __syncwarp();
     asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
   }
@@ -378,8 +478,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 uint32_t tc_smem_bytes() { return 1024 + TC_STAGES * (A_BYTES + B_BYTES) + 128; }
 
 void tc_kernel_table(KernelFn* instr, KernelFn* plain) {
-  instr[0] = (KernelFn)k_conv_tc<true>;
-  plain[0] = (KernelFn)k_conv_tc<false>;
+  instr[0] = (KernelFn)k_conv_tc<true, false>;
+  plain[0] = (KernelFn)k_conv_tc<false, false>;
+  instr[1] = (KernelFn)k_conv_tc<true, true>;     // with the DenseNet prologue
+  plain[1] = (KernelFn)k_conv_tc<false, true>;
 }
 
 // Host: tensor map for the packed weights [rows][kpad] bf16, box 64 x 128, SW128.

@@ -224,7 +224,7 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
           const uint32_t K = nd.kh * nd.kw * cin;
           const uint32_t kpad = (uint32_t)align_up(K, 64);
           a.kpad = kpad;
-          const bool use_tc_here = tc && (a.flags & LF_PROLOGUE) == 0;
+          const bool use_tc_here = tc;
           const uint32_t rows = use_tc_here ? (uint32_t)align_up(nd.c, TC_BM) : nd.c;
           // pack [rows][kpad], k = (r, s, ci)
           std::vector<float> wp((size_t)rows * kpad, 0.f);
@@ -244,17 +244,20 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
             k.w_bytes = wp.size() * 4;
           }
           if (use_tc_here) {
-            k.kind = KIND_CONV_TC;
+            k.kind = (a.flags & LF_PROLOGUE) ? KIND_CONV_TC_PRO : KIND_CONV_TC;
             a.tiles_m = rows / TC_BM;
             a.tiles_n = (P_out + TC_BN - 1) / TC_BN;
             uint32_t nk = kpad / TC_BK;
             uint32_t tiles = a.tiles_m * a.tiles_n;
             // split K so the grid approaches one wave of SMs, >= 2 k-blocks per split;
-            // the splits of a tile form one thread-block cluster (<= 8, portable)
+            // the splits of a tile form one thread-block cluster
             uint32_t split = 1;
             const char* e = std::getenv("PAELLA_NOSPLIT");
             if (!e) {
-              while (split < 8 && tiles * split * 2 <= P->sms && nk / (split * 2) >= 2) split *= 2;
+              // splitting pays only for deep K: a cluster barrier + DSMEM reduction cost ~1 us;
+              // clusters of up to 16 CTAs (non-portable size, allowed on sm_100)
+              if (nk >= 12)
+                while (split < 16 && tiles * split * 2 <= P->sms && nk / (split * 2) >= 4) split *= 2;
             }
             a.ksplit = split;
             k.grid[0] = a.tiles_n;

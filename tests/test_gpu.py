@@ -118,17 +118,19 @@ def _serve_and_check(e, specs, n, n_clients, seed, rate_us=30.0):
                 done += 1
 
 
-@pytest.mark.parametrize("policy,group,streams,ring", [
-    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536),
-    (L.POLICY_FIFO, 16, 32, 65536),
-    (L.POLICY_SRPT_DEFICIT, 1, 8, 256),      # G = 1 debug mode, ring wraps many laps
-    (L.POLICY_SRPT_DEFICIT, 16, 1, 1024),    # a single stream
+@pytest.mark.parametrize("policy,group,streams,ring,look,lt", [
+    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 0, 0),
+    (L.POLICY_FIFO, 16, 32, 65536, 0, 0),
+    (L.POLICY_SRPT_DEFICIT, 1, 8, 1024, 0, 0),     # G = 1 debug mode, ring wraps many laps
+    (L.POLICY_SRPT_DEFICIT, 16, 1, 1024, 0, 0),    # a single stream
+    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 1, 2),  # launch-ahead + launcher threads (bench arm)
+    (L.POLICY_SRPT_DEFICIT, 4, 16, 4096, 2, 3),
 ])
-def test_serving_parity_and_replay(tmp_path, policy, group, streams, ring):
+def test_serving_parity_and_replay(tmp_path, policy, group, streams, ring, look, lt):
     log = str(tmp_path / "gpu_%u.log")
     names = ["toy", "resnet18", "mobilenet_v2", "squeezenet1_1"]
     with L.Engine(num_clients=3, policy=policy, group=group, streams=streams, ring_capacity=ring,
-                  event_log=log, max_jobs_per_model=32) as e:
+                  event_log=log, max_jobs_per_model=32, lookahead=look, launch_threads=lt) as e:
         specs = []
         for nm in names:
             g = archs.build(nm)
@@ -144,9 +146,10 @@ def test_serving_parity_and_replay(tmp_path, policy, group, streams, ring):
     assert sim.check_exactly_once(ex["records"], grids, cfg.group) == []
 
 
-def test_naive_baseline_outputs():
+@pytest.mark.parametrize("lt", [0, 2])
+def test_naive_baseline_outputs(lt):
     names = ["toy", "squeezenet1_1"]
-    with L.Engine(num_clients=2, naive=True, instrument=False) as e:
+    with L.Engine(num_clients=2, naive=True, instrument=False, launch_threads=lt) as e:
         specs = []
         for nm in names:
             g = archs.build(nm)
