@@ -237,6 +237,9 @@ def run_gpu(args, dist):
     # --- the Paella arm -------------------------------------------------------------
     e, mids = engine(instrument=True, lookahead=args.lookahead)
     x_sat_paella = saturation(e, mids, len(names), stride, slots)
+    jp, _ = e.loadgen(t1, m1, m1, i1, stride, slots)
+    unloaded = {"naive": {nm: float(np.median(jct_unloaded[m1 == m])) / 1e3 for m, nm in enumerate(names)},
+                "paella": {nm: float(np.median(jp[m1 == m])) / 1e3 for m, nm in enumerate(names)}}
     # device-only roofline: summed isolated kernel time per model (uninstrumented twin)
     dev_roof = {}
     kinfo = {}
@@ -310,7 +313,7 @@ def run_gpu(args, dist):
             eb.shutdown()
             base[label] = jct_stats(np.concatenate([a for a, _ in jl]), np.concatenate([b for _, b in jl]), names)
 
-    return dict(names=names, lam=lam, x_sat_naive=x_sat_naive, x_sat_paella=x_sat_paella, slo=slo,
+    return dict(unloaded=unloaded, names=names, lam=lam, x_sat_naive=x_sat_naive, x_sat_paella=x_sat_paella, slo=slo,
                 elapsed=elapsed, completed=completed, jct=jct_stats(jct, models, names), clocks=clk,
                 ev=ev, stats=stats, dev_roof=dev_roof, base=base, e2e_rate=e2e_rate,
                 e2e=jct_stats(e2e_jct, mm, names), h2d=h2d, d2h=d2h, calib_s=calib_s, kinfo=kinfo)
@@ -437,6 +440,7 @@ def main():
                           "theta": 100, "group": 16, "streams": 32},
         "slo_met": bool(all(res["jct"].get(n, {}).get("p99_us", 1e18) <= res["slo"][n] for n in res["names"])),
         "x_sat_req_s": {"naive": round(res["x_sat_naive"], 1), "paella": round(res["x_sat_paella"], 1)},
+        "jct_unloaded_p50_us": {k: {m: round(v, 1) for m, v in d.items()} for k, d in res["unloaded"].items()},
         "device_roofline_us": {k: round(v, 2) for k, v in res["dev_roof"].items()},
         "jct_fraction_of_device_roofline": {n: round(res["dev_roof"][n] / res["jct"][n]["mean_us"], 4)
                                             for n in res["names"] if n in res["jct"]},

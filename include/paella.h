@@ -110,6 +110,11 @@ typedef struct {
                                     n helper threads per GPU perform the launches (stream s is
                                     owned by helper s % n, so per-stream order is kept); the
                                     decisions stay on the one dispatcher core */
+  uint32_t no_proxy;             /* 0 (default): kernels write notification records to a
+                                    device-memory ring and one persistent proxy warp forwards
+                                    them to the pinned host ring (keeps the PCIe write off every
+                                    kernel's exit path); 1: kernels write the host ring directly,
+                                    as in the paper (P1104-1106) */
 } paella_config_t;
 
 /* ---- model description (input to paella_register_model) ---------------- */

@@ -11,6 +11,7 @@
 // where lap = ring index >> log2(capacity).  type 0 = INVALID (P1110-1113).
 #pragma once
 #include <stdint.h>
+#include <stddef.h>
 
 #ifndef __CUDACC__
 #define PAELLA_HD

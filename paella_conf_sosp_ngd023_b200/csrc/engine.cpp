@@ -185,13 +185,45 @@ struct CudaBackend : Backend {
   int dev;
   uint32_t cap, nstreams;
   Rec* ring_h = nullptr;
-  Rec* ring_d = nullptr;
+  Rec* ring_d = nullptr;      // device view of the pinned host ring
+  // notification proxy: kernels write to dev_ring (device memory); one persistent warp
+  // forwards to the host ring, so no kernel pays the PCIe write on its exit path
+  bool proxy = false;
+  Rec* dev_ring = nullptr;
+  uint32_t* proxy_ctl = nullptr;     // pinned mapped: [0] stop flag, [16] heartbeat
+  cudaStream_t proxy_stream = nullptr;
   uint32_t* tail = nullptr;   // device
   uint32_t* ctr = nullptr;    // device, 2*NCTR
   std::vector<cudaStream_t> streams;
   KernelFn tab[2][2][KIND_COUNT];   // [dtype][instr][kind]
   int err_ = 0;
-  CudaBackend(int d, uint32_t c, uint32_t P) : dev(d), cap(c), nstreams(P) {}
+  CudaBackend(int d, uint32_t c, uint32_t P, bool px) : dev(d), cap(c), nstreams(P), proxy(px) {}
+  int start_proxy() {
+    if (cudaMalloc(&dev_ring, (size_t)cap * sizeof(Rec)) != cudaSuccess) return -ENOMEM;
+    cudaMemset(dev_ring, 0, (size_t)cap * sizeof(Rec));
+    if (cudaHostAlloc((void**)&proxy_ctl, 256, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
+      return -ENOMEM;
+    std::memset(proxy_ctl, 0, 256);
+    uint32_t* ctl_d = nullptr;
+    cudaHostGetDevicePointer((void**)&ctl_d, proxy_ctl, 0);
+    if (cudaStreamCreateWithFlags(&proxy_stream, cudaStreamNonBlocking) != cudaSuccess) return -EIO;
+    if (cudaDeviceSynchronize() != cudaSuccess) return -EIO;
+    const Rec* src = dev_ring;
+    Rec* dst = ring_d;
+    uint32_t mask = cap - 1, l2 = 0;
+    while ((1u << l2) < cap) ++l2;
+    const volatile uint32_t* stop = ctl_d;
+    volatile uint32_t* hb = ctl_d + 16;
+    void* args[6] = {(void*)&src, (void*)&dst, (void*)&mask, (void*)&l2, (void*)&stop, (void*)&hb};
+    if (cudaLaunchKernel((const void*)proxy_kernel(), dim3(1), dim3(32), args, 0, proxy_stream) != cudaSuccess)
+      return -EIO;
+    return 0;
+  }
+  void stop_proxy() {
+    if (!proxy_ctl) return;
+    __atomic_store_n(&proxy_ctl[0], 1u, __ATOMIC_SEQ_CST);
+    cudaStreamSynchronize(proxy_stream);
+  }
   int init() override {
     if (cudaSetDevice(dev) != cudaSuccess) return -ENODEV;
     if (cudaHostAlloc((void**)&ring_h, (size_t)cap * sizeof(Rec), cudaHostAllocMapped | cudaHostAllocPortable) !=
@@ -214,10 +246,17 @@ struct CudaBackend : Backend {
     tab[0][1][KIND_CONV_TC_PRO] = tc_i[1];
     tab[0][0][KIND_CONV_TC_PRO] = tc_p[1];
     for (int i = 0; i < 2; ++i) tab[1][i][KIND_CONV_TC] = tab[1][i][KIND_CONV_TC_PRO] = nullptr;
-    return cudaDeviceSynchronize() == cudaSuccess ? 0 : -EIO;
+    if (cudaDeviceSynchronize() != cudaSuccess) return -EIO;
+    // from here on no device-wide synchronisation (cudaDeviceSynchronize / cudaFree)
+    // may run while the proxy kernel is resident: every sync is per stream
+    return proxy ? start_proxy() : 0;
   }
   ~CudaBackend() override {
     cudaSetDevice(dev);
+    stop_proxy();
+    if (proxy_stream) cudaStreamDestroy(proxy_stream);
+    if (dev_ring) cudaFree(dev_ring);
+    if (proxy_ctl) cudaFreeHost(proxy_ctl);
     for (auto& s : streams) cudaStreamDestroy(s);
     if (ring_h) cudaFreeHost(ring_h);
     if (tail) cudaFree(tail);
@@ -226,7 +265,7 @@ struct CudaBackend : Backend {
   Rec* ring() override { return ring_h; }
   uint32_t* tail_dev() override { return tail; }
   uint32_t* ctr_dev() override { return ctr; }
-  void* ring_dev() override { return ring_d; }
+  void* ring_dev() override { return proxy ? (void*)dev_ring : (void*)ring_d; }
   KernelFn fn(uint32_t kind, uint32_t dtype, bool instr) { return tab[dtype][instr ? 1 : 0][kind]; }
   void launch(const KernelInst& k, const LayerArgs& a, const InstrArgs& ia, uint32_t stream, uint32_t dtype,
               bool instr) override {
@@ -252,7 +291,9 @@ struct CudaBackend : Backend {
   }
   bool event_done(void* ev) override { return cudaEventQuery((cudaEvent_t)ev) == cudaSuccess; }
   void release_event(void* ev) override { cudaEventDestroy((cudaEvent_t)ev); }
-  void sync() override { cudaDeviceSynchronize(); }
+  void sync() override {
+    for (auto& s : streams) cudaStreamSynchronize(s);
+  }
 };
 
 // per-(model, gpu) tensor maps for tcgen05 weights (defined in kernels_tc.cu)
@@ -508,8 +549,18 @@ static void dispatcher_main(Gpu* g) {
       g->ev_free.push_back(Gpu::EvPair{a, b, 0, 0});
     }
   }
+  const bool dbg = std::getenv("PAELLA_DEBUG") != nullptr;
   for (;;) {
     g->stats.loop_iters++;
+    if (dbg && (g->stats.loop_iters % 50000000) == 0) {
+      fprintf(stderr, "[dbg gpu%u] iters=%lu admitted=%lu", g->index, (unsigned long)g->stats.loop_iters,
+              (unsigned long)g->stats.admitted);
+      for (uint32_t c = 0; c < N; ++c) fprintf(stderr, " sub[%u]=%lu", c, (unsigned long)g->sub[c]->size());
+      uint32_t nm = P->nmodels.load();
+      for (uint32_t m = 0; m < nm; ++m)
+        fprintf(stderr, " free[%u]=%zu", m, P->models[m]->gpu[g->index].free_slots.size());
+      fprintf(stderr, " live=%lu\n", (unsigned long)g->policy->live_jobs());
+    }
     if (!g->ev_pending.empty() && (g->stats.loop_iters & 63) == 0) harvest_events(g);
     g->be->advance();
     uint32_t nev = 0;
@@ -523,9 +574,11 @@ static void dispatcher_main(Gpu* g) {
         const SubmitSlot* s;
         bool served = false;
         while ((s = q->peek()) != nullptr) {
-          if (s->model_id >= nm) {   // cannot happen through the API; drop defensively
-            q->pop();
-            continue;
+          if (s->model_id >= nm) {
+            // submit validated the id against nmodels, so the model is published: this
+            // iteration loaded nmodels before the submission was pushed; reload it
+            nm = P->nmodels.load(std::memory_order_acquire);
+            if (s->model_id >= nm) break;
           }
           if (!admit(g, c, *s)) break;
           q->pop();
@@ -671,7 +724,8 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     // never reallocated: launcher threads hold pointers into job records
     g->jobs.reserve(65536);
     if (cfg.device == PAELLA_DEVICE_CUDA)
-      g->be.reset(new CudaBackend(g->device, g->cap, cfg.stream_pool));
+      g->be.reset(new CudaBackend(g->device, g->cap, cfg.stream_pool,
+                                  cfg.no_proxy == 0 && !std::getenv("PAELLA_NO_PROXY")));
     else
       g->be.reset(new FakeBackend(P->sms, g->cap, g->log2cap, cfg.group_size, cfg.stream_pool,
                                   cfg.fake_time_scale_ns));
@@ -881,6 +935,7 @@ int paella_shutdown(paella_t* p) {
       if (L->th.joinable()) L->th.join();
     if (P->cfg.device == PAELLA_DEVICE_CUDA) {
       cudaSetDevice(g->device);
+      static_cast<CudaBackend*>(g->be.get())->stop_proxy();
       cudaDeviceSynchronize();
     }
   }
@@ -993,22 +1048,34 @@ static int ensure_iso(Gpu* g) {
   std::memset(g->prof_ring_h, 0, cap * sizeof(Rec));
   cudaHostGetDevicePointer(&g->prof_ring_d, g->prof_ring_h, 0);
   if (cudaMalloc(&g->prof_tail, 256) || cudaMalloc(&g->prof_ctr, 2 * NCTR * sizeof(uint32_t))) return -ENOMEM;
-  cudaMemset(g->prof_tail, 0, 256);
-  cudaMemset(g->prof_ctr, 0, 2 * NCTR * sizeof(uint32_t));
   g->prof_base.assign(NCTR, 0);
   cudaStream_t s;
   cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
   g->prof_stream = s;
+  cudaMemsetAsync(g->prof_tail, 0, 256, s);
+  cudaMemsetAsync(g->prof_ctr, 0, 2 * NCTR * sizeof(uint32_t), s);
+  // isolated runs write their records to device memory (as served kernels do through
+  // the proxy); nobody consumes them except the round-trip benchmark's direct ring
+  if (cudaMalloc(&g->prof_devring, cap * sizeof(Rec))) return -ENOMEM;
+  cudaMemsetAsync(g->prof_devring, 0, cap * sizeof(Rec), s);
+  if (cudaMalloc(&g->trace_buf, 16 * 8 * 8192)) return -ENOMEM;
   g->stage_bytes = 16u << 20;
   if (cudaHostAlloc(&g->stage_in, g->stage_bytes, cudaHostAllocMapped | cudaHostAllocPortable)) return -ENOMEM;
-  return cudaDeviceSynchronize() == cudaSuccess ? 0 : -EIO;
+  return cudaStreamSynchronize(s) == cudaSuccess ? 0 : -EIO;
+}
+
+// the ring isolated runs write to: device memory when served kernels go through the
+// notification proxy (same cost as in serving), else the pinned host ring
+static Rec* iso_ring(Gpu* g) {
+  auto* cb = static_cast<CudaBackend*>(g->be.get());
+  return cb->proxy ? g->prof_devring : (Rec*)g->prof_ring_d;
 }
 
 // launch kernel `l` of model m from the isolated slot on the profiling stream
 static void iso_launch(Gpu* g, Model* m, uint32_t l, bool instr) {
   const KernelInst& k = m->kernels[l];
   InstrArgs ia;
-  ia.ring = (Rec*)g->prof_ring_d;
+  ia.ring = iso_ring(g);
   ia.tail = g->prof_tail;
   uint32_t uid = g->prof_uid++;
   uint32_t slot = uid % NCTR;
@@ -1060,8 +1127,8 @@ static int iso_run(Gpu* g, Model* m, const void* input, void* output, int64_t* k
   uint64_t* trbuf = nullptr;
   LayerArgs saved{};
   if (trace_k >= 0 && trace_k < (int)m->kernels.size() && is_tc(m->kernels[trace_k].kind)) {
-    cudaMalloc(&trbuf, 16 * 8 * m->kernels[trace_k].grid_total());
-    cudaMemset(trbuf, 0, 16 * 8 * m->kernels[trace_k].grid_total());
+    trbuf = (uint64_t*)g->trace_buf;
+    cudaMemsetAsync(trbuf, 0, 16 * 8 * m->kernels[trace_k].grid_total(), s);
     saved = args[trace_k];
     args[trace_k].flags |= LF_TRACE;
     args[trace_k].ws = (float*)trbuf;
@@ -1085,8 +1152,8 @@ static int iso_run(Gpu* g, Model* m, const void* input, void* output, int64_t* k
     cudaStreamSynchronize(s);
     uint32_t nb = m->kernels[trace_k].grid_total();
     std::vector<uint64_t> h(16 * nb);
-    cudaMemcpy(h.data(), trbuf, h.size() * 8, cudaMemcpyDeviceToHost);
-    cudaFree(trbuf);
+    cudaMemcpyAsync(h.data(), trbuf, h.size() * 8, cudaMemcpyDeviceToHost, s);
+    cudaStreamSynchronize(s);
     args[trace_k] = saved;
     uint64_t t0 = UINT64_MAX;
     for (uint32_t b = 0; b < nb; ++b) t0 = std::min(t0, h[16 * b]);
@@ -1130,10 +1197,12 @@ static int setup_model_gpu(Paella* P, Model* m, Gpu* g) {
     cudaMemcpy(wdev, m->blob.data(), m->blob.size(), cudaMemcpyHostToDevice);
     if (cudaMalloc((void**)&wsp, nslot * m->slot_bytes)) return -ENOMEM;
     cudaMemset(wsp, 0, nslot * m->slot_bytes);
+    cudaStreamSynchronize(0);   // legacy-stream memset vs. our non-blocking streams
     if (m->splitk_floats) {
       if (cudaMalloc((void**)&mg.splitk_ws, nslot * m->splitk_floats * 4)) return -ENOMEM;
       if (cudaMalloc((void**)&mg.splitk_ctr, nslot * m->splitk_ctrs * 4)) return -ENOMEM;
       cudaMemset(mg.splitk_ctr, 0, nslot * m->splitk_ctrs * 4);
+      cudaStreamSynchronize(0);
     }
   } else {
     wdev = (uint8_t*)malloc(m->blob.size() + 256);
@@ -1295,7 +1364,7 @@ static void launch_gate(Gpu* g, const volatile uint32_t* gd) {
 
 static InstrArgs iso_instr(Gpu* g, uint32_t grid, uint32_t group, bool last) {
   InstrArgs ia;
-  ia.ring = (Rec*)g->prof_ring_d;
+  ia.ring = iso_ring(g);
   ia.tail = g->prof_tail;
   uint32_t uid = g->prof_uid++;
   uint32_t slot = uid % NCTR;
@@ -1371,6 +1440,9 @@ int paella_bench_empty(paella_t* p, uint32_t gpu, uint32_t grid, uint32_t block,
   auto* cb = static_cast<CudaBackend*>(g->be.get());
   KernelFn f = cb->fn(KIND_EMPTY, 0, instrumented != 0);
   LayerArgs la{};
+  // experiment: PAELLA_BENCH_DEVRING=1 writes the records to device memory instead of
+  // the pinned host ring (isolates the cost of the PCIe write + kernel-end flush)
+  Rec* devring = std::getenv("PAELLA_BENCH_DIRECT") ? (Rec*)g->prof_ring_d : g->prof_devring;
   const volatile uint32_t* gd;
   volatile uint32_t* gate = gate_ptr(g, &gd);
   cudaEvent_t e0, e1;
@@ -1387,6 +1459,7 @@ int paella_bench_empty(paella_t* p, uint32_t gpu, uint32_t grid, uint32_t block,
     cudaEventRecord(e0, s);
     for (uint32_t i = 0; i < nb; ++i) {
       InstrArgs ia = iso_instr(g, grid, group, false);
+      if (devring) ia.ring = devring;
       void* args[2] = {(void*)&la, (void*)&ia};
       cudaLaunchKernel((const void*)f, dim3(grid), dim3(block), args, 0, s);
     }
@@ -1426,6 +1499,7 @@ int paella_bench_roundtrip(paella_t* p, uint32_t gpu, uint32_t n, int64_t* place
   const uint32_t mask = (1u << 16) - 1;
   for (uint32_t i = 0; i < n; ++i) {
     InstrArgs ia = iso_instr(g, 1, 1, false);
+    ia.ring = (Rec*)g->prof_ring_d;   // direct write to the pinned host ring
     void* args[2] = {(void*)&la, (void*)&ia};
     int64_t t0 = now_ns();
     cudaLaunchKernel((const void*)f, dim3(1), dim3(32), args, 0, s);

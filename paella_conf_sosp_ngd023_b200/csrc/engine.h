@@ -178,6 +178,8 @@ struct Gpu {
   Rec* prof_ring_h = nullptr;
   void* prof_ring_d = nullptr;
   uint32_t* prof_tail = nullptr;
+  Rec* prof_devring = nullptr;     // device-memory ring of isolated runs
+  void* trace_buf = nullptr;       // debug phase timestamps
   uint32_t* prof_ctr = nullptr;
   std::vector<uint32_t> prof_base;
   uint32_t prof_uid = 0;

@@ -442,6 +442,49 @@ __global__ void k_gate(const volatile uint32_t* flag) {
 KernelFn gate_kernel() { return (KernelFn)k_gate; }
 
 // ---------------------------------------------------------------------------
+// Notification proxy: one persistent warp forwards records from the device-memory
+// ring (where the instrumented kernels write them: an L2 store, no PCIe write on the
+// kernels' exit path) to the pinned host ring the dispatcher polls.  Lane i checks
+// slot head+i; the valid prefix of the window is copied with one 16-byte store per
+// lane and the device slots are cleared.  Order and lap tags are preserved, so the
+// host sees exactly the records it would see with direct writes.
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(32, 1) k_notify_proxy(const Rec* dev_ring, Rec* host_ring, uint32_t mask,
+                                                        uint32_t log2cap, const volatile uint32_t* stop,
+                                                        volatile uint32_t* heartbeat) {
+  const uint32_t lane = threadIdx.x;
+  uint32_t head = 0;
+  uint32_t idle = 0;
+  for (;;) {
+    const uint32_t idx = head + lane;
+    const Rec* src = dev_ring + (idx & mask);
+    uint64_t w0, w1;
+    asm volatile("ld.volatile.global.v2.u64 {%0, %1}, [%2];" : "=l"(w0), "=l"(w1) : "l"(src));
+    const uint32_t tag = rec_tag(idx >> log2cap);
+    const bool valid = (w0 & 0xff) != REC_INVALID && ((w0 >> 24) & 0xff) == tag && (w1 >> 56) == tag;
+    const uint32_t bal = __ballot_sync(0xffffffffu, valid);
+    const uint32_t n = (bal == 0xffffffffu) ? 32u : (uint32_t)(__ffs(~bal) - 1);   // valid prefix
+    if (lane < n) {
+      Rec* dst = host_ring + (idx & mask);
+      asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(dst), "l"(w0), "l"(w1) : "memory");
+      asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(src), "l"(0ull), "l"(0ull) : "memory");
+    }
+    head += n;
+    if (n == 0) {
+      if ((++idle & 1023) == 0) {
+        if (*stop) break;
+        if (lane == 0) *heartbeat = head;
+      }
+      __nanosleep(64);
+    } else {
+      idle = 0;
+    }
+  }
+}
+
+KernelFn proxy_kernel() { return (KernelFn)k_notify_proxy; }
+
+// ---------------------------------------------------------------------------
 // kernel table
 // ---------------------------------------------------------------------------
 template <typename T, bool I>
