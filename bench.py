@@ -52,6 +52,7 @@ def parse():
     ap.add_argument("--no-baselines", action="store_true")
     ap.add_argument("--lookahead", type=int, default=1, help="NEXT-1 launch-ahead depth of the Paella arm")
     ap.add_argument("--launch-threads", type=int, default=2, help="launcher helper threads per GPU")
+    ap.add_argument("--sat-reqs", type=int, default=1500, help="requests of the saturation calibration")
     ap.add_argument("--fake", action="store_true",
                     help="CPU fake device (tests of the multi-rank plumbing; not a measurement)")
     return ap.parse_args()
@@ -193,7 +194,7 @@ def make_trace(n, rate, cfg, n_models, seed):
     return t, models, inputs
 
 
-def saturation(e, mids, n_models, stride, slots, n=1500, seed=99):
+def saturation(e, mids, n_models, stride, slots, n, seed=99):
     """Closed burst: all requests due at t=0; completions / elapsed."""
     t = np.zeros(n, dtype=np.int64)
     models = np.arange(n) % n_models
@@ -227,7 +228,7 @@ def run_gpu(args, dist):
     # --- calibration (untimed): naive saturation, unloaded JCT -> SLO ---------------
     t_cal = time.time()
     en, mids = engine(naive=True, instrument=False)
-    x_sat_naive = saturation(en, mids, len(names), stride, slots)
+    x_sat_naive = saturation(en, mids, len(names), stride, slots, args.sat_reqs)
     t1, m1, i1 = make_trace(300, 200.0, cfg, len(names), seed=7)
     jct_unloaded, _ = en.loadgen(t1, m1, m1, i1, stride, slots)
     slo = {nm: 5.0 * float(np.median(jct_unloaded[m1 == m])) / 1e3 for m, nm in enumerate(names)}
@@ -236,7 +237,7 @@ def run_gpu(args, dist):
 
     # --- the Paella arm -------------------------------------------------------------
     e, mids = engine(instrument=True, lookahead=args.lookahead)
-    x_sat_paella = saturation(e, mids, len(names), stride, slots)
+    x_sat_paella = saturation(e, mids, len(names), stride, slots, args.sat_reqs)
     jp, _ = e.loadgen(t1, m1, m1, i1, stride, slots)
     unloaded = {"naive": {nm: float(np.median(jct_unloaded[m1 == m])) / 1e3 for m, nm in enumerate(names)},
                 "paella": {nm: float(np.median(jp[m1 == m])) / 1e3 for m, nm in enumerate(names)}}

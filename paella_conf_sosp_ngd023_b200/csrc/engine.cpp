@@ -198,31 +198,42 @@ struct CudaBackend : Backend {
   KernelFn tab[2][2][KIND_COUNT];   // [dtype][instr][kind]
   int err_ = 0;
   CudaBackend(int d, uint32_t c, uint32_t P, bool px) : dev(d), cap(c), nstreams(P), proxy(px) {}
-  int start_proxy() {
+  bool proxy_running = false;
+  uint32_t* ctl_d = nullptr;
+  int setup_proxy(cudaStream_t s) {
     if (cudaMalloc(&dev_ring, (size_t)cap * sizeof(Rec)) != cudaSuccess) return -ENOMEM;
-    cudaMemset(dev_ring, 0, (size_t)cap * sizeof(Rec));
+    cudaMemsetAsync(dev_ring, 0, (size_t)cap * sizeof(Rec), s);
     if (cudaHostAlloc((void**)&proxy_ctl, 256, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
       return -ENOMEM;
     std::memset(proxy_ctl, 0, 256);
-    uint32_t* ctl_d = nullptr;
     cudaHostGetDevicePointer((void**)&ctl_d, proxy_ctl, 0);
     if (cudaStreamCreateWithFlags(&proxy_stream, cudaStreamNonBlocking) != cudaSuccess) return -EIO;
-    if (cudaDeviceSynchronize() != cudaSuccess) return -EIO;
+    return 0;
+  }
+  // dispatcher thread: (re)start the forwarding warp when records may be outstanding
+  void ensure_proxy() {
+    if (!proxy) return;
+    if (proxy_running) {
+      if (__atomic_load_n(&proxy_ctl[32], __ATOMIC_ACQUIRE) == 0) return;
+      proxy_running = false;   // it left after an idle spell
+    }
+    __atomic_store_n(&proxy_ctl[32], 0u, __ATOMIC_RELEASE);
     const Rec* src = dev_ring;
     Rec* dst = ring_d;
     uint32_t mask = cap - 1, l2 = 0;
     while ((1u << l2) < cap) ++l2;
-    const volatile uint32_t* stop = ctl_d;
-    volatile uint32_t* hb = ctl_d + 16;
-    void* args[6] = {(void*)&src, (void*)&dst, (void*)&mask, (void*)&l2, (void*)&stop, (void*)&hb};
-    if (cudaLaunchKernel((const void*)proxy_kernel(), dim3(1), dim3(32), args, 0, proxy_stream) != cudaSuccess)
-      return -EIO;
-    return 0;
+    volatile uint32_t* st = ctl_d;
+    void* args[5] = {(void*)&src, (void*)&dst, (void*)&mask, (void*)&l2, (void*)&st};
+    if (cudaLaunchKernel((const void*)proxy_kernel(), dim3(1), dim3(32), args, 0, proxy_stream) == cudaSuccess)
+      proxy_running = true;
+    else if (!err_)
+      err_ = (int)cudaErrorLaunchFailure;
   }
   void stop_proxy() {
     if (!proxy_ctl) return;
     __atomic_store_n(&proxy_ctl[0], 1u, __ATOMIC_SEQ_CST);
-    cudaStreamSynchronize(proxy_stream);
+    if (proxy_stream) cudaStreamSynchronize(proxy_stream);
+    proxy_running = false;
   }
   int init() override {
     if (cudaSetDevice(dev) != cudaSuccess) return -ENODEV;
@@ -233,11 +244,11 @@ struct CudaBackend : Backend {
     if (cudaHostGetDevicePointer((void**)&ring_d, ring_h, 0) != cudaSuccess) return -EIO;
     if (cudaMalloc(&tail, 256) != cudaSuccess) return -ENOMEM;
     if (cudaMalloc(&ctr, 2 * NCTR * sizeof(uint32_t)) != cudaSuccess) return -ENOMEM;
-    cudaMemset(tail, 0, 256);
-    cudaMemset(ctr, 0, 2 * NCTR * sizeof(uint32_t));
     streams.resize(nstreams);
     for (auto& s : streams)
       if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess) return -EIO;
+    cudaMemsetAsync(tail, 0, 256, streams[0]);
+    cudaMemsetAsync(ctr, 0, 2 * NCTR * sizeof(uint32_t), streams[0]);
     KernelFn tc_i[2], tc_p[2];
     simt_kernel_table(tab[0][1], tab[0][0], tab[1][1], tab[1][0]);
     tc_kernel_table(tc_i, tc_p);
@@ -246,10 +257,12 @@ struct CudaBackend : Backend {
     tab[0][1][KIND_CONV_TC_PRO] = tc_i[1];
     tab[0][0][KIND_CONV_TC_PRO] = tc_p[1];
     for (int i = 0; i < 2; ++i) tab[1][i][KIND_CONV_TC] = tab[1][i][KIND_CONV_TC_PRO] = nullptr;
-    if (cudaDeviceSynchronize() != cudaSuccess) return -EIO;
-    // from here on no device-wide synchronisation (cudaDeviceSynchronize / cudaFree)
-    // may run while the proxy kernel is resident: every sync is per stream
-    return proxy ? start_proxy() : 0;
+    if (proxy) {
+      int rc = setup_proxy(streams[0]);
+      if (rc) return rc;
+    }
+    // stream-scoped: another engine's forwarding warp may be resident on this device
+    return cudaStreamSynchronize(streams[0]) == cudaSuccess ? 0 : -EIO;
   }
   ~CudaBackend() override {
     cudaSetDevice(dev);
@@ -521,6 +534,8 @@ static uint32_t drain_ring(Gpu* g) {
 static void decide_and_launch(Gpu* g) {
   g->issues.clear();
   g->policy->decide(&g->issues);
+  if (!g->issues.empty() && g->P->cfg.device == PAELLA_DEVICE_CUDA)
+    static_cast<CudaBackend*>(g->be.get())->ensure_proxy();
   g->stats.decide_calls++;
   for (const Issue& is : g->issues) {
     JobRec& j = g->jobs[is.job];
@@ -604,7 +619,9 @@ static void dispatcher_main(Gpu* g) {
       if (stopping && g->naive_inflight.empty()) break;
       continue;
     }
-    // 2. notification ring
+    // 2. notification ring (keep the forwarding warp alive while records are due)
+    if (P->cfg.device == PAELLA_DEVICE_CUDA && g->policy->O() > 0 && (g->stats.loop_iters & 1023) == 0)
+      static_cast<CudaBackend*>(g->be.get())->ensure_proxy();
     nev += drain_ring(g);
     // 3. decide (the batch boundary is logged for replay, C2-Q17)
     if (nev) {
@@ -741,6 +758,11 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     pc.streams = cfg.stream_pool;
     pc.lookahead = cfg.lookahead;
     for (int r = 0; r < NRES; ++r) pc.capacity[r] = P->capacity[r];
+    if (cfg.device == PAELLA_DEVICE_CUDA && static_cast<CudaBackend*>(g->be.get())->proxy) {
+      // the resident proxy warp: 1 block, 1 warp, <= 64 regs/thread, the 1 KB reservation
+      const int64_t proxy[NRES] = {1, 1, 64 * 32, 1024, 0};
+      for (int r = 0; r < NRES; ++r) pc.capacity[r] -= proxy[r];
+    }
     g->policy.reset(new Policy(pc));
     for (uint32_t c = 0; c < cfg.num_clients; ++c) {
       auto* s = (SpscRing<SubmitSlot>*)shm_alloc(P.get(), SpscRing<SubmitSlot>::bytes(cfg.submit_slots));
@@ -760,7 +782,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
       logev(g.get(), EV_CONFIG, cfg.num_clients, cfg.policy, (uint64_t)cfg.fairness_threshold,
             ((uint64_t)P->cfg.slack_blocks << 32) | cfg.group_size);
       logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFFu, cfg.ring_capacity, cfg.stream_pool, cfg.lookahead);
-      for (int r = 0; r < NRES; ++r) logev(g.get(), EV_CAPACITY, (uint32_t)r, (uint64_t)P->capacity[r], 0, 0);
+      for (int r = 0; r < NRES; ++r) logev(g.get(), EV_CAPACITY, (uint32_t)r, (uint64_t)pc.capacity[r], 0, 0);
     }
     P->gpus.push_back(std::move(g));
   }
@@ -936,7 +958,8 @@ int paella_shutdown(paella_t* p) {
     if (P->cfg.device == PAELLA_DEVICE_CUDA) {
       cudaSetDevice(g->device);
       static_cast<CudaBackend*>(g->be.get())->stop_proxy();
-      cudaDeviceSynchronize();
+      g->be->sync();
+      if (g->prof_stream) cudaStreamSynchronize((cudaStream_t)g->prof_stream);
     }
   }
   // requests never admitted complete with -ECANCELED
@@ -1020,7 +1043,7 @@ int paella_kernel_info(paella_t* p, uint32_t model_id, uint32_t k, paella_kernel
 
 const char* paella_kernel_name(uint32_t kind) {
   static const char* names[] = {"ingest", "conv_simt", "conv_tcgen05", "dwconv", "maxpool",
-                                "avgpool", "gap", "fc_gemv", "empty", "conv_tcgen05_pro"};
+                                "avgpool", "gap", "fc_gemv", "empty", "conv_tcgen05_pro", "gap_fc"};
   return kind < KIND_COUNT ? names[kind] : "?";
 }
 

@@ -15,7 +15,8 @@ enum KernelKind : uint32_t {
   KIND_FC = 7,
   KIND_EMPTY = 8,
   KIND_CONV_TC_PRO = 9, // tcgen05 conv with the per-channel affine+ReLU input prologue
-  KIND_COUNT = 10,
+  KIND_GAPFC = 10,      // fused global average pool + FC classifier head
+  KIND_COUNT = 11,
 };
 
 typedef void (*KernelFn)();
@@ -24,7 +25,7 @@ void simt_kernel_table(KernelFn (&bf16_instr)[KIND_COUNT], KernelFn (&bf16_plain
                        KernelFn (&f32_instr)[KIND_COUNT], KernelFn (&f32_plain)[KIND_COUNT]);
 
 KernelFn gate_kernel();   // k_gate(const volatile uint32_t* flag)
-KernelFn proxy_kernel();  // k_notify_proxy(dev_ring, host_ring, mask, log2cap, stop, heartbeat)
+KernelFn proxy_kernel();  // k_notify_proxy(dev_ring, host_ring, mask, log2cap, state)
 
 // tcgen05 conv: instrumented / plain instantiations [0] plain input, [1] prologue
 void tc_kernel_table(KernelFn* instr, KernelFn* plain);

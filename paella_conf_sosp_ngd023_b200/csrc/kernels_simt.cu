@@ -423,6 +423,76 @@ __global__ void __launch_bounds__(256) k_fc(const __grid_constant__ LayerArgs a,
 }
 
 // ---------------------------------------------------------------------------
+// Fused global-average-pool + FC (the classifier head of ResNet / MobileNetV2 /
+// DenseNet / Inception): one launch instead of two.  Every block (32 output rows)
+// first averages the C x HW input into shared memory (+ DenseNet's norm5 prologue),
+// then each warp streams 4 weight rows against it.  Same arithmetic and rounding
+// points as GAP -> FC except that the pooled vector stays fp32 (no bf16 rounding
+// between the two, reading C1-Q7: one rounding per fused layer).
+// ---------------------------------------------------------------------------
+template <typename T, bool INSTR>
+__global__ void __launch_bounds__(256) k_gapfc(const __grid_constant__ LayerArgs a,
+                                               const __grid_constant__ InstrArgs ia) {
+  instr_enter<INSTR>(ia);
+  extern __shared__ float pooled[];   // [C]
+  const T* X = static_cast<const T*>(a.in);
+  const T* W = static_cast<const T*>(a.w);
+  const uint32_t C = a.cin, HW = a.h * a.w_;
+  const float inv = 1.f / (float)HW;
+  for (uint32_t g = threadIdx.x; g < C / 8; g += blockDim.x) {
+    const int c = g * 8;
+    float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    float sc[8], sh[8];
+    if (a.flags & LF_PROLOGUE) {
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        sc[i] = a.pro_scale[c + i];
+        sh[i] = a.pro_shift[c + i];
+      }
+    }
+#pragma unroll 4
+    for (uint32_t p = 0; p < HW; ++p) {
+      float xv[8];
+      load8(X + (size_t)p * a.in_cs + a.in_co + c, xv);
+      if (a.flags & LF_PROLOGUE) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) xv[i] = fmaxf(fmaf(sc[i], xv[i], sh[i]), 0.f);
+      }
+#pragma unroll
+      for (int i = 0; i < 8; ++i) acc[i] += xv[i];
+    }
+#pragma unroll
+    for (int i = 0; i < 8; ++i) pooled[c + i] = acc[i] * inv;
+  }
+  __syncthreads();
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+#pragma unroll
+  for (int rr = 0; rr < 4; ++rr) {
+    const int row = blockIdx.x * 32 + warp * 4 + rr;
+    if (row < (int)a.cout) {
+      const T* wr = W + (size_t)row * a.kpad;
+      float acc = 0.f;
+      for (uint32_t k = lane * 8; k < C; k += 32 * 8) {
+        float wv[8];
+        load8(wr + k, wv);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) acc = fmaf(wv[i], pooled[k + i], acc);
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+      if (lane == 0) {
+        float v = act_f(acc + a.bias[row], a.act);
+        if (a.flags & LF_FINAL)
+          static_cast<float*>(a.out)[row] = v;
+        else
+          static_cast<T*>(a.out)[a.out_co + row] = (T)v;
+      }
+    }
+  }
+  instr_exit<INSTR>(ia);
+}
+
+// ---------------------------------------------------------------------------
 // Empty instrumented kernel for the notification microbenchmark (K5, Fig. 15).
 // ---------------------------------------------------------------------------
 template <bool INSTR>
@@ -450,10 +520,13 @@ KernelFn gate_kernel() { return (KernelFn)k_gate; }
 // host sees exactly the records it would see with direct writes.
 // ---------------------------------------------------------------------------
 __global__ void __launch_bounds__(32, 1) k_notify_proxy(const Rec* dev_ring, Rec* host_ring, uint32_t mask,
-                                                        uint32_t log2cap, const volatile uint32_t* stop,
-                                                        volatile uint32_t* heartbeat) {
+                                                        uint32_t log2cap, volatile uint32_t* state) {
+  // state (pinned, mapped): [0] stop request, [16] heartbeat, [32] exited flag,
+  // [48] ring index to resume from.  The warp leaves on its own after ~20 ms without
+  // records (so device-wide synchronisation elsewhere in the process can never wait
+  // on it forever); the dispatcher relaunches it when it has records outstanding.
   const uint32_t lane = threadIdx.x;
-  uint32_t head = 0;
+  uint32_t head = state[48];
   uint32_t idle = 0;
   for (;;) {
     const uint32_t idx = head + lane;
@@ -471,14 +544,20 @@ __global__ void __launch_bounds__(32, 1) k_notify_proxy(const Rec* dev_ring, Rec
     }
     head += n;
     if (n == 0) {
-      if ((++idle & 1023) == 0) {
-        if (*stop) break;
-        if (lane == 0) *heartbeat = head;
+      ++idle;
+      if ((idle & 255) == 0) {
+        if (state[0] || idle > (1u << 16)) break;
+        if (lane == 0) state[16] = head;
       }
       __nanosleep(64);
     } else {
       idle = 0;
     }
+  }
+  if (lane == 0) {
+    state[48] = head;
+    __threadfence_system();
+    state[32] = 1;
   }
 }
 
@@ -497,6 +576,7 @@ static void fill(KernelFn (&t)[KIND_COUNT]) {
   t[KIND_GAP] = (KernelFn)k_gap<T, I>;
   t[KIND_FC] = (KernelFn)k_fc<T, I>;
   t[KIND_EMPTY] = (KernelFn)k_empty<I>;
+  t[KIND_GAPFC] = (KernelFn)k_gapfc<T, I>;
 }
 
 void simt_kernel_table(KernelFn (&bf16_instr)[KIND_COUNT], KernelFn (&bf16_plain)[KIND_COUNT],

@@ -225,7 +225,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   const uint32_t K = a.kh * a.kw * a.cin;
   // (r, s, ci) of k = kbase + 8*chunk, advanced incrementally by TC_BK per stage
   int kr = 0, ks_ = 0, kci = 0;
-  auto issue_B = [&](uint32_t it) {
+  auto issue_B = [&](uint32_t it, bool arrive) {
     const uint32_t s = it % TC_STAGES;
     const uint32_t k = (kb0 + it) * TC_BK + chunk * 8;
     const bool kv = k < K;
@@ -265,7 +265,12 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
                      : "memory");
       }
     }
-    if constexpr (!PRO) cp_async_commit();
+    if constexpr (!PRO) {
+      // the stage's full barrier is arrived on by the hardware once this thread's
+      // copies have landed: the gather warps never wait for their own loads
+      if (arrive)
+        asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(su32(&full[s])) : "memory");
+    }
     // advance (r, s, ci) by TC_BK channels for the next stage
     kci += TC_BK;
     while (kci >= (int)a.cin) {
@@ -292,7 +297,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       kr = rs / (int)a.kw;
     }
     // ... and the first activation gathers, before the CTA-wide barrier
-    for (uint32_t it = 0; it < pre; ++it) issue_B(it);
+    for (uint32_t it = 0; it < pre; ++it) issue_B(it, false);   // barriers not initialised yet
     if (trace && t == 0) tr[13] = globaltimer();
   }
   __syncthreads();
@@ -300,25 +305,33 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 
   if (warp < 4) {
     // ------------------------------------------------------------ producers
-    for (uint32_t it = 0; it < nkl; ++it) {
-      // stage `it` has landed for this thread: make it visible to the tensor core
-      if constexpr (!PRO) {
-        if (it + TC_STAGES <= nkl)
-          cp_async_wait<TC_STAGES - 1>();
-        else
-          cp_async_wait<0>();
-      }
-      fence_proxy_async();
-      mbar_arrive(&full[it % TC_STAGES]);
-      const uint32_t nxt = it + TC_STAGES;
-      if (nxt < nkl) {
+    if constexpr (!PRO) {
+      for (uint32_t it = 0; it < pre; ++it)
+        asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(su32(&full[it])) : "memory");
+      for (uint32_t nxt = TC_STAGES; nxt < nkl; ++nxt) {
         const uint32_t s = nxt % TC_STAGES;
-        mbar_wait(&empty[s], ((nxt / TC_STAGES) & 1) ^ 1);   // MMA of stage `it` retired
+        mbar_wait(&empty[s], ((nxt / TC_STAGES) & 1) ^ 1);   // MMA of stage nxt - STAGES retired
         if (t == 0) {
           mbar_arrive_tx(&full[s], A_BYTES);
           tma_load_2d(sA + s * A_BYTES, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
         }
-        issue_B(nxt);
+        issue_B(nxt, true);
+      }
+    } else {
+      // prologue path: register-staged stores, then a proxy fence and an arrive
+      for (uint32_t it = 0; it < nkl; ++it) {
+        fence_proxy_async();
+        mbar_arrive(&full[it % TC_STAGES]);
+        const uint32_t nxt = it + TC_STAGES;
+        if (nxt < nkl) {
+          const uint32_t s = nxt % TC_STAGES;
+          mbar_wait(&empty[s], ((nxt / TC_STAGES) & 1) ^ 1);
+          if (t == 0) {
+            mbar_arrive_tx(&full[s], A_BYTES);
+            tma_load_2d(sA + s * A_BYTES, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
+          }
+          issue_B(nxt, true);
+        }
       }
     }
   } else {
@@ -337,6 +350,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         const uint32_t s = it % TC_STAGES;
         mbar_wait(&full[s], (it / TC_STAGES) & 1);
         if (trace && it == 0) tr[2] = globaltimer();
+        fence_proxy_async();   // the gathered B tile was written through the generic proxy
         tc_fence_after();
         const uint32_t abase = su32(sA + s * A_BYTES), bbase = su32(sB + s * B_BYTES);
 #pragma unroll

@@ -163,9 +163,25 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
   }
 
   size_t max_splitk = 0, max_tiles = 0;
+  // GAP whose only consumer is an FC: fused into one gap_fc kernel
+  std::vector<uint32_t> consumers(n, 0);
+  for (uint32_t i = 0; i < n; ++i) {
+    for (int32_t s : m->node_inputs[i]) consumers[s]++;
+    if (d->nodes[i].residual >= 0) consumers[d->nodes[i].residual]++;
+  }
+  std::vector<bool> fused_gap(n, false);
+  const bool fuse = !std::getenv("PAELLA_NO_FUSE");
   for (uint32_t i = 1; i < n; ++i) {
     const paella_node_t& nd = d->nodes[i];
-    if (nd.op == PAELLA_OP_CONCAT) continue;
+    if (fuse && nd.op == PAELLA_OP_FC) {
+      int32_t src = m->node_inputs[i][0];
+      const paella_node_t& sn = d->nodes[src];
+      if (sn.op == PAELLA_OP_GAP && consumers[src] == 1 && sn.c % 8 == 0 && sn.c <= 8192) fused_gap[src] = true;
+    }
+  }
+  for (uint32_t i = 1; i < n; ++i) {
+    const paella_node_t& nd = d->nodes[i];
+    if (nd.op == PAELLA_OP_CONCAT || fused_gap[i]) continue;
     int32_t src = m->node_inputs[i][0];
     const paella_node_t& sn = d->nodes[src];
     const bool is_first = sn.op == PAELLA_OP_INPUT;
@@ -320,6 +336,45 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
         break;
       }
       case PAELLA_OP_FC: {
+        if (fused_gap[src]) {
+          // read the GAP's input (C x H x W) directly, with the GAP's prologue
+          const paella_node_t& gn = sn;
+          int32_t gsrc = m->node_inputs[src][0];
+          const paella_node_t& gin = d->nodes[gsrc];
+          k.kind = KIND_GAPFC;
+          k.in_buf = m->buf_of[gsrc];
+          a.in_cs = cs_of(gsrc);
+          a.in_co = m->coff[gsrc];
+          a.cin = gn.c;
+          a.h = gin.h;
+          a.w_ = gin.w;
+          a.kpad = gn.c;
+          if (gn.flags & PAELLA_NODE_PROLOGUE) {
+            if (!gn.pro_scale || !gn.pro_shift) return -EINVAL;
+            a.flags |= LF_PROLOGUE;
+            k.has_pro = true;
+            k.ps_off = blob.put(gn.pro_scale, gn.c * 4);
+            k.pz_off = blob.put(gn.pro_shift, gn.c * 4);
+          }
+          std::vector<float> wp(nd.weight, nd.weight + (size_t)nd.c * gn.c);
+          if (es == 2) {
+            std::vector<uint16_t> wb(wp.size());
+            for (size_t q = 0; q < wp.size(); ++q) wb[q] = f32_to_bf16_exact(wp[q], &exact);
+            k.w_off = blob.put(wb.data(), wb.size() * 2);
+          } else {
+            k.w_off = blob.put(wp.data(), wp.size() * 4);
+          }
+          std::vector<float> bias(nd.c, 0.f);
+          if (nd.bias) std::memcpy(bias.data(), nd.bias, nd.c * 4);
+          k.b_off = blob.put(bias.data(), nd.c * 4);
+          k.grid[0] = (nd.c + 31) / 32;
+          k.block = 256;
+          k.smem = gn.c * 4;
+          k.flops = 2ull * nd.c * gn.c + (uint64_t)gn.c * gin.h * gin.w;
+          k.bytes = (uint64_t)nd.c * gn.c * es + (uint64_t)gin.h * gin.w * gn.c * es +
+                    (uint64_t)nd.c * ((a.flags & LF_FINAL) ? 4 : es);
+          break;
+        }
         k.kind = KIND_FC;
         const uint32_t K = sn.c * sn.h * sn.w;
         if (K % 8 || (sn.h * sn.w > 1 && a.in_cs != sn.c)) return -EINVAL;
