@@ -38,6 +38,7 @@ sys.path.insert(0, ROOT)
 from workload import archs, rng, traces  # noqa: E402
 
 PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
+METRIC = "requests/s at rho*X_sat(naive) with mean/p50/p99 JCT (open-loop, batch-1 mix)"
 
 
 def parse():
@@ -406,11 +407,13 @@ def main():
             cb = cpu_baseline(cfg, seconds=max(2.0, 30.0 / max(1, args.steps)))
             vals.append(cb["value"])
         v = float(np.mean(vals))
-        line = {"impl": "reference", "metric": "requests/s (open-loop mix, JCT at load)", "value": round(v, 3),
+        line = {"impl": "reference", "metric": METRIC, "value": round(v, 3),
                 "unit": "req/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
                 "ms_per_step": round((time.time() - t0) * 1e3 / args.steps, 1), "higher_is_better": True,
                 "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-                "config": {"workload": workload, "clients": cfg["clients"], "batch": 1},
+                "config": {"workload": workload, "models": cfg["models"], "clients": cfg["clients"], "batch": 1,
+                           "arrivals": cfg["arrival"], "rho": args.rho, "requests_per_step": args.reqs,
+                           "parallelism": "oracle on host cores"},
                 "cpu_baseline": {**cb, "value": round(v, 3)},
                 "e2e": {"value": round(v, 3), "unit": "req/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
         print(json.dumps(line))
@@ -427,7 +430,7 @@ def main():
     jm = res["jct"]["mix"]
     launches = res["stats"]["launches"]
     line = {
-        "metric": "requests/s at rho*X_sat(naive) with mean/p50/p99 JCT (open-loop, batch-1 mix)",
+        "metric": METRIC,
         "value": round(value, 2), "unit": "req/s", "n_gpus": args.gpus, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(max_el * 1e3 / args.steps, 2), "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
