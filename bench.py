@@ -233,6 +233,9 @@ def run_gpu(args, dist):
     t1, m1, i1 = make_trace(300, 200.0, cfg, len(names), seed=7)
     jct_unloaded, _ = en.loadgen(t1, m1, m1, i1, stride, slots)
     slo = {nm: 5.0 * float(np.median(jct_unloaded[m1 == m])) / 1e3 for m, nm in enumerate(names)}
+    if cfg["weights"] is None:
+        # Fig. 12 convention (P1482-1483): request mix inversely proportional to job size
+        cfg = dict(cfg, weights=[1.0 / max(1e-9, float(np.median(jct_unloaded[m1 == m]))) for m in range(len(names))])
     en.shutdown()
     lam = args.rho * x_sat_naive
 

@@ -439,30 +439,41 @@ __global__ void __launch_bounds__(256) k_gapfc(const __grid_constant__ LayerArgs
   const T* W = static_cast<const T*>(a.w);
   const uint32_t C = a.cin, HW = a.h * a.w_;
   const float inv = 1.f / (float)HW;
-  for (uint32_t g = threadIdx.x; g < C / 8; g += blockDim.x) {
-    const int c = g * 8;
+  // 8 threads per 8-channel granule split the pixels; shuffle-reduce within the 8
+  const uint32_t l8 = threadIdx.x % 8;
+  for (uint32_t g0 = 0; g0 < C / 8; g0 += blockDim.x / 8) {
+    const uint32_t g = g0 + threadIdx.x / 8;
     float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-    float sc[8], sh[8];
-    if (a.flags & LF_PROLOGUE) {
-#pragma unroll
-      for (int i = 0; i < 8; ++i) {
-        sc[i] = a.pro_scale[c + i];
-        sh[i] = a.pro_shift[c + i];
-      }
-    }
-#pragma unroll 4
-    for (uint32_t p = 0; p < HW; ++p) {
-      float xv[8];
-      load8(X + (size_t)p * a.in_cs + a.in_co + c, xv);
+    if (g < C / 8) {
+      const int c = g * 8;
+      float sc[8], sh[8];
       if (a.flags & LF_PROLOGUE) {
 #pragma unroll
-        for (int i = 0; i < 8; ++i) xv[i] = fmaxf(fmaf(sc[i], xv[i], sh[i]), 0.f);
+        for (int i = 0; i < 8; ++i) {
+          sc[i] = a.pro_scale[c + i];
+          sh[i] = a.pro_shift[c + i];
+        }
       }
+#pragma unroll 4
+      for (uint32_t p = l8; p < HW; p += 8) {
+        float xv[8];
+        load8(X + (size_t)p * a.in_cs + a.in_co + c, xv);
+        if (a.flags & LF_PROLOGUE) {
 #pragma unroll
-      for (int i = 0; i < 8; ++i) acc[i] += xv[i];
+          for (int i = 0; i < 8; ++i) xv[i] = fmaxf(fmaf(sc[i], xv[i], sh[i]), 0.f);
+        }
+#pragma unroll
+        for (int i = 0; i < 8; ++i) acc[i] += xv[i];
+      }
     }
 #pragma unroll
-    for (int i = 0; i < 8; ++i) pooled[c + i] = acc[i] * inv;
+    for (int o = 4; o > 0; o >>= 1)
+#pragma unroll
+      for (int i = 0; i < 8; ++i) acc[i] += __shfl_xor_sync(0xffffffffu, acc[i], o);
+    if (g < C / 8 && l8 == 0) {
+#pragma unroll
+      for (int i = 0; i < 8; ++i) pooled[g * 8 + i] = acc[i] * inv;
+    }
   }
   __syncthreads();
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;

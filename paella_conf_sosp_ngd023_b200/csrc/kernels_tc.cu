@@ -166,8 +166,10 @@ __device__ __forceinline__ uint4 load_res8(const LayerArgs& a, uint32_t p, uint3
                                               a.res_co + co));
 }
 
+// 2 CTAs per SM (two jobs' convs can share an SM): <= 168 registers, since a
+// 160-thread CTA puts 2 of its 5 warps on one sub-partition (16K registers each)
 template <bool INSTR, bool PRO>
-__global__ void __launch_bounds__(TC_THREADS, 1)
+__global__ void __launch_bounds__(TC_THREADS, 2)
     k_conv_tc(const __grid_constant__ LayerArgs a, const __grid_constant__ InstrArgs ia,
               const __grid_constant__ CUtensorMap wmap) {
   const bool trace = (a.flags & LF_TRACE) != 0;
@@ -370,6 +372,22 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   // 1. TMEM -> registers (warp w owns lanes = output channels 32w..32w+31) -> fp32
   //    tile in shared memory [pixel][channel] (conflict-free: a warp writes 32
   //    consecutive words of one pixel row)
+  // epilogue operands that do not depend on the accumulator (bias, residual) are
+  // fetched while the tensor core is still working
+  const uint32_t eg = threadIdx.x % (TC_BM / 8), eco = m0 + eg * 8;
+  constexpr uint32_t NIT = TC_BN * (TC_BM / 8) / NPROD;   // 8 items per thread
+  float ebias[8];
+  uint4 eres[NIT];
+  if (warp < 4 && a.ksplit == 1) {
+    load_bias8(a, eco, ebias);
+    if (a.flags & LF_RESIDUAL) {
+#pragma unroll
+      for (uint32_t i = 0; i < NIT; ++i) {
+        const uint32_t p = n0 + (threadIdx.x + i * NPROD) / (TC_BM / 8);
+        if (p < P && eco < a.cout) eres[i] = load_res8(a, p, eco);
+      }
+    }
+  }
   if (warp < 4) {
     const uint32_t row = warp * 32 + lane;
     if (nkl > 0) {
@@ -393,20 +411,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   if (a.ksplit == 1) {
     // 2. coalesced epilogue: item = (pixel, 8-channel group), 16-byte loads/stores
     if (warp < 4) {
-      // every item of this thread has channel group g = t % 16: one bias load; all
-      // residual loads are issued before the tile is read (latency overlap)
-      const uint32_t g = threadIdx.x % (TC_BM / 8), co = m0 + g * 8;
-      constexpr uint32_t NIT = TC_BN * (TC_BM / 8) / NPROD;   // 8 items per thread
-      float bias[8];
-      load_bias8(a, co, bias);
-      uint4 res[NIT];
-      const bool has_res = (a.flags & LF_RESIDUAL) != 0;
-#pragma unroll
-      for (uint32_t i = 0; i < NIT; ++i) {
-        const uint32_t px = (threadIdx.x + i * NPROD) / (TC_BM / 8);
-        const uint32_t p = n0 + px;
-        if (has_res && p < P && co < a.cout) res[i] = load_res8(a, p, co);
-      }
+      const uint32_t g = eg, co = eco;
       if (trace && threadIdx.x == 0) tr[9] = globaltimer();
       asm volatile("bar.sync 1, 128;" ::: "memory");   // the 4 epilogue warps only
       if (trace && threadIdx.x == 0) tr[10] = globaltimer();
@@ -418,7 +423,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           const float4* q = reinterpret_cast<const float4*>(stage + px * TC_BM + g * 8);
           float4 u0 = q[0], u1 = q[1];
           float v[8] = {u0.x, u0.y, u0.z, u0.w, u1.x, u1.y, u1.z, u1.w};
-          epi_store8(a, p, co, v, bias, res[i]);
+          epi_store8(a, p, co, v, ebias, eres[i]);
         }
       }
     }
@@ -446,26 +451,28 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           uint4 res = make_uint4(0, 0, 0, 0);
           if (a.flags & LF_RESIDUAL) res = load_res8(a, p, co);
           const uint32_t off = (px * TC_BM + g * 8) * 4;
-          float4 part[16][2];
-#pragma unroll
-          for (uint32_t r = 0; r < 16; ++r) {   // every peer's slice in flight at once
-            if (r < ks) {
-              uint32_t peer;
-              asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(peer) : "r"(base + off), "r"(r));
-              asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
-                           : "=f"(part[r][0].x), "=f"(part[r][0].y), "=f"(part[r][0].z), "=f"(part[r][0].w)
-                           : "r"(peer));
-              asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
-                           : "=f"(part[r][1].x), "=f"(part[r][1].y), "=f"(part[r][1].z), "=f"(part[r][1].w)
-                           : "r"(peer + 16));
-            }
-          }
           float v[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+          for (uint32_t r0 = 0; r0 < ks; r0 += 4) {   // 4 peers' slices in flight at once
+            float4 part[4][2];
 #pragma unroll
-          for (uint32_t r = 0; r < 16; ++r) {
-            if (r < ks) {
-              v[0] += part[r][0].x; v[1] += part[r][0].y; v[2] += part[r][0].z; v[3] += part[r][0].w;
-              v[4] += part[r][1].x; v[5] += part[r][1].y; v[6] += part[r][1].z; v[7] += part[r][1].w;
+            for (uint32_t q = 0; q < 4; ++q) {
+              if (r0 + q < ks) {
+                uint32_t peer;
+                asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(peer) : "r"(base + off), "r"(r0 + q));
+                asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
+                             : "=f"(part[q][0].x), "=f"(part[q][0].y), "=f"(part[q][0].z), "=f"(part[q][0].w)
+                             : "r"(peer));
+                asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
+                             : "=f"(part[q][1].x), "=f"(part[q][1].y), "=f"(part[q][1].z), "=f"(part[q][1].w)
+                             : "r"(peer + 16));
+              }
+            }
+#pragma unroll
+            for (uint32_t q = 0; q < 4; ++q) {
+              if (r0 + q < ks) {
+                v[0] += part[q][0].x; v[1] += part[q][0].y; v[2] += part[q][0].z; v[3] += part[q][0].w;
+                v[4] += part[q][1].x; v[5] += part[q][1].y; v[6] += part[q][1].z; v[7] += part[q][1].w;
+              }
             }
           }
           epi_store8(a, p, co, v, bias, res);

@@ -118,19 +118,20 @@ def _serve_and_check(e, specs, n, n_clients, seed, rate_us=30.0):
                 done += 1
 
 
-@pytest.mark.parametrize("policy,group,streams,ring,look,lt", [
-    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 0, 0),
-    (L.POLICY_FIFO, 16, 32, 65536, 0, 0),
-    (L.POLICY_SRPT_DEFICIT, 1, 8, 1024, 0, 0),     # G = 1 debug mode, ring wraps many laps
-    (L.POLICY_SRPT_DEFICIT, 16, 1, 1024, 0, 0),    # a single stream
-    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 1, 2),  # launch-ahead + launcher threads (bench arm)
-    (L.POLICY_SRPT_DEFICIT, 4, 16, 4096, 2, 3),
+@pytest.mark.parametrize("policy,group,streams,ring,look,lt,proxy", [
+    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 0, 0, True),
+    (L.POLICY_FIFO, 16, 32, 65536, 0, 0, True),
+    (L.POLICY_SRPT_DEFICIT, 1, 8, 1024, 0, 0, True),     # G = 1 debug mode, ring wraps many laps
+    (L.POLICY_SRPT_DEFICIT, 16, 1, 1024, 0, 0, True),    # a single stream
+    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 1, 2, True),  # launch-ahead + launcher threads (bench arm)
+    (L.POLICY_SRPT_DEFICIT, 4, 16, 4096, 2, 3, True),
+    (L.POLICY_SRPT_DEFICIT, 16, 32, 2048, 1, 2, False),  # direct record writes (the paper's path)
 ])
-def test_serving_parity_and_replay(tmp_path, policy, group, streams, ring, look, lt):
+def test_serving_parity_and_replay(tmp_path, policy, group, streams, ring, look, lt, proxy):
     log = str(tmp_path / "gpu_%u.log")
     names = ["toy", "resnet18", "mobilenet_v2", "squeezenet1_1"]
     with L.Engine(num_clients=3, policy=policy, group=group, streams=streams, ring_capacity=ring,
-                  event_log=log, max_jobs_per_model=32, lookahead=look, launch_threads=lt) as e:
+                  event_log=log, max_jobs_per_model=32, lookahead=look, launch_threads=lt, proxy=proxy) as e:
         specs = []
         for nm in names:
             g = archs.build(nm)
@@ -176,3 +177,41 @@ def test_ring_records_carry_sm_and_time(tmp_path):
     for (t, typ, uid, n, grp, sm) in recs:
         if typ == sim.COMPLETION:
             assert (t - first_place[uid]) % (1 << 40) < (1 << 39)
+
+
+def test_per_sm_capacity_from_g1_records(tmp_path):
+    """S5 (a) on the GPU: with G = 1 every block reports (SM id, globaltimer) at entry
+    and exit; the blocks resident on any SM at any time never need more than one SM's
+    Table-1 resources (+TMEM) according to the demands the dispatcher accounts."""
+    log = str(tmp_path / "cap_%u.log")
+    names = ["resnet18", "mobilenet_v2", "squeezenet1_1"]
+    with L.Engine(num_clients=3, group=1, event_log=log, ring_capacity=4096, lookahead=1, launch_threads=2) as e:
+        specs = []
+        for nm in names:
+            g = archs.build(nm)
+            specs.append((e.register_model(g, rng.model_params(g)), nm, g))
+        _serve_and_check(e, specs, 60, 3, seed=11, rate_us=5.0)
+    cfg, ms, events, ex = eventlog.read(log % 0)
+    demand = {uid: ms[model][layer].demand for (uid, job, layer, stream, model) in ex["issues"]}
+    opened = {}
+    evs = []
+    for (t, typ, uid, n, grp, sm) in ex["records"]:
+        evs.append((t, 0 if typ == sim.COMPLETION else 1, uid, sm))   # exits before entries at equal t
+    evs.sort()
+    per_sm = (32, 64, 65536, 233472, 512)
+    use = {}
+    worst = [0] * 5
+    for (t, kind, uid, sm) in evs:
+        u = use.setdefault(sm, [0] * 5)
+        d = demand[uid]
+        if kind == 1:
+            for r in range(5):
+                u[r] += d[r]
+                worst[r] = max(worst[r], u[r])
+            opened[(uid, sm)] = opened.get((uid, sm), 0) + 1
+        elif opened.get((uid, sm), 0) > 0:
+            opened[(uid, sm)] -= 1
+            for r in range(5):
+                u[r] -= d[r]
+    for r in range(5):
+        assert worst[r] <= per_sm[r], (r, worst)
