@@ -204,7 +204,7 @@ def saturation(e, mids, n_models, stride, slots, n, seed=99):
 
 
 def run_gpu(args, dist):
-    from paella_conf_sosp_ngd023_b200 import _lib as L
+    from paper_conf_sosp_ngd023_b200 import _lib as L
     L.load()
     cfgname = args.config
     cfg = traces.CONFIGS[cfgname]

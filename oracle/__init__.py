@@ -12,6 +12,6 @@ computes, written from the paper and SURVEY.md §8(c):
 
 Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline`` /
 ``--impl reference`` legs may import anything in this package.  It shares no code
-with ``paella_conf_sosp_ngd023_b200/`` (the CUDA path); both read their inputs from
+with ``paper_conf_sosp_ngd023_b200/`` (the CUDA path); both read their inputs from
 the neutral ``workload`` package.
 """

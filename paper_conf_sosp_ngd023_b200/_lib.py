@@ -95,7 +95,7 @@ def load():
     if _lib is not None:
         return _lib
     if not os.path.exists(LIB_PATH):
-        raise RuntimeError(f"{LIB_PATH} missing: run `python -m paella_conf_sosp_ngd023_b200.build` "
+        raise RuntimeError(f"{LIB_PATH} missing: run `python -m paper_conf_sosp_ngd023_b200.build` "
                            "(there is no CPU fallback of the CUDA path)")
     lib = C.CDLL(LIB_PATH)
     P = C.c_void_p

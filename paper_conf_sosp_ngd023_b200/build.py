@@ -1,6 +1,6 @@
 """Build the in-tree C-ABI library ``libpaella.so`` for sm_100a.
 
-    python -m paella_conf_sosp_ngd023_b200.build
+    python -m paper_conf_sosp_ngd023_b200.build
 
 Host C++ (runtime, dispatcher, planner, policy) is compiled with g++; kernels with
 nvcc ``-gencode arch=compute_100a,code=sm_100a -lineinfo``; everything is linked by

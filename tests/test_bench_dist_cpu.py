@@ -22,7 +22,7 @@ def _free_port():
 
 @pytest.mark.timeout(600)
 def test_bench_two_ranks_gloo_fake_device():
-    from paella_conf_sosp_ngd023_b200 import build
+    from paper_conf_sosp_ngd023_b200 import build
     build.build()
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
            "--master-addr", "127.0.0.1", "--master-port", str(_free_port()), "bench.py", "--gpus", "2",

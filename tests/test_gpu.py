@@ -20,7 +20,7 @@ from workload import archs, rng
 
 pytestmark = pytest.mark.gpu
 
-L = pytest.importorskip("paella_conf_sosp_ngd023_b200._lib")
+L = pytest.importorskip("paper_conf_sosp_ngd023_b200._lib")
 
 BF16_TOL = (2e-2, 1e-2)
 FP32_TOL = (1e-4, 1e-4)
@@ -42,7 +42,7 @@ def within(out, ref, tol):
 
 @pytest.fixture(scope="module")
 def engine():
-    from paella_conf_sosp_ngd023_b200 import build
+    from paper_conf_sosp_ngd023_b200 import build
     build.build()
     e = L.Engine(num_clients=1)
     yield e

@@ -17,13 +17,13 @@ import pytest
 from oracle import eventlog, sim
 from workload import archs, rng
 
-L = pytest.importorskip("paella_conf_sosp_ngd023_b200._lib")
+L = pytest.importorskip("paper_conf_sosp_ngd023_b200._lib")
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
 @pytest.fixture(scope="module", autouse=True)
 def built():
-    from paella_conf_sosp_ngd023_b200 import build
+    from paper_conf_sosp_ngd023_b200 import build
     build.build()
     L.load()
 

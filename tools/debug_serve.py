@@ -1,7 +1,7 @@
 import os, sys, time, json
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np
-from paella_conf_sosp_ngd023_b200 import _lib as L
+from paper_conf_sosp_ngd023_b200 import _lib as L
 from workload import archs, rng, traces
 os.environ["PAELLA_DEBUG"] = "1"
 v = json.loads(sys.argv[1])

@@ -3,7 +3,7 @@ oracle (uses oracle/: test tooling, not product)."""
 import sys, os, time
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np
-from paella_conf_sosp_ngd023_b200 import _lib as L
+from paper_conf_sosp_ngd023_b200 import _lib as L
 from workload import archs, rng
 from oracle import infer
 

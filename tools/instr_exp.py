@@ -1,6 +1,6 @@
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
-from paella_conf_sosp_ngd023_b200 import _lib as L
+from paper_conf_sosp_ngd023_b200 import _lib as L
 e = L.Engine(num_clients=1)
 for dev in (0, 1):
     if not dev: os.environ["PAELLA_BENCH_DIRECT"] = "1"

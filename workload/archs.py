@@ -1,7 +1,7 @@
 """Model architectures of the paper's evaluation mix, as plain layer lists.
 
 NEUTRAL MODULE: this file is *input description* shared by the oracle (``oracle/``)
-and the CUDA path (``paella_conf_sosp_ngd023_b200/``).  It holds no arithmetic of the
+and the CUDA path (``paper_conf_sosp_ngd023_b200/``).  It holds no arithmetic of the
 method (no convolution, no pooling, no scheduling) -- only the graph of layers and
 their static shapes, the same way a model file handed to ``paella_register_model``
 would.  Its correctness is pinned independently by ``tests/test_oracle_infer.py``,
