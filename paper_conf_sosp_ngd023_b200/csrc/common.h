@@ -82,11 +82,6 @@ struct InstrArgs {
 };
 
 constexpr uint32_t NCTR = 4096;   // counter slots; > max in-flight launches (<= P)
-// a slot = CTR_WORDS u32: start counters [0, CTR_SUB), end counters [CTR_SUB, 2 CTR_SUB).
-// Counter mode spreads a launch's blocks over CTR_SUB words (less same-address
-// contention in L2); the proxy sums them.  Block-record mode uses words 0 and CTR_SUB.
-constexpr uint32_t CTR_SUB = 8;
-constexpr uint32_t CTR_WORDS = 2 * CTR_SUB;
 
 // Kernel-side arguments of one layer.  Activations are NHWC with an explicit
 // channel stride/offset so that a concat is just producers writing into disjoint

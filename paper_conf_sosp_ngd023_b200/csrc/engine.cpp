@@ -89,7 +89,7 @@ struct FakeBackend : Backend {
     for (auto& f : freeres)
       for (int r = 0; r < NRES; ++r) f[r] = per_sm[r];
     ringmem.assign(cap, Rec{0, 0});
-    ctr.assign(CTR_WORDS * NCTR, 0);
+    ctr.assign(2 * NCTR, 0);
     streams.resize(nstreams + 1);
     return 0;
   }
@@ -267,12 +267,12 @@ struct CudaBackend : Backend {
     std::memset(ring_h, 0, (size_t)cap * sizeof(Rec));
     if (cudaHostGetDevicePointer((void**)&ring_d, ring_h, 0) != cudaSuccess) return -EIO;
     if (cudaMalloc(&tail, 256) != cudaSuccess) return -ENOMEM;
-    if (cudaMalloc(&ctr, CTR_WORDS * NCTR * sizeof(uint32_t)) != cudaSuccess) return -ENOMEM;
+    if (cudaMalloc(&ctr, 2 * NCTR * sizeof(uint32_t)) != cudaSuccess) return -ENOMEM;
     streams.resize(nstreams);
     for (auto& s : streams)
       if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess) return -EIO;
     cudaMemsetAsync(tail, 0, 256, streams[0]);
-    cudaMemsetAsync(ctr, 0, CTR_WORDS * NCTR * sizeof(uint32_t), streams[0]);
+    cudaMemsetAsync(ctr, 0, 2 * NCTR * sizeof(uint32_t), streams[0]);
     KernelFn tc_i[2], tc_p[2];
     simt_kernel_table(tab[0][1], tab[0][0], tab[1][1], tab[1][0]);
     tc_kernel_table(tc_i, tc_p);
@@ -345,7 +345,7 @@ static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last, bool
   ia.ring = (Rec*)g->be->ring_dev();
   ia.tail = g->be->tail_dev();
   uint32_t slot = uid % NCTR;
-  ia.ctr = g->be->ctr_dev() + CTR_WORDS * slot;
+  ia.ctr = g->be->ctr_dev() + 2 * slot;
   ia.mask = g->cap - 1;
   ia.log2cap = g->log2cap;
   ia.base = g->ctr_base[slot];
@@ -598,25 +598,14 @@ static void dispatcher_main(Gpu* g) {
   const bool dbg = std::getenv("PAELLA_DEBUG") != nullptr;
   for (;;) {
     g->stats.loop_iters++;
-    if (dbg && (g->stats.loop_iters & 0xFFFFF) == 0) {
-      static thread_local int64_t last = 0;
-      int64_t tnow = now_ns();
-      if (tnow - last > 1000000000ll) {
-        last = tnow;
-        fprintf(stderr, "[dbg gpu%u] admitted=%lu completed=%lu launches=%lu records=%lu head=%lu O=%ld Q=%ld live=%lu",
-                g->index, (unsigned long)g->stats.admitted, (unsigned long)g->stats.completed,
-                (unsigned long)g->stats.launches, (unsigned long)g->stats.records, (unsigned long)g->head,
-                (long)g->policy->O(), (long)g->policy->Q(), (unsigned long)g->policy->live_jobs());
-        for (uint32_t c = 0; c < N; ++c) fprintf(stderr, " sub[%u]=%lu", c, (unsigned long)g->sub[c]->size());
-        if (P->cfg.device == PAELLA_DEVICE_CUDA) {
-          auto* cb = static_cast<CudaBackend*>(g->be.get());
-          if (cb->proxy_ctl)
-            fprintf(stderr, " proxy{run=%d exited=%u hb=%u rec=%u ihead=%u itail=%lu}", (int)cb->proxy_running,
-                    cb->proxy_ctl[32], cb->proxy_ctl[16], cb->proxy_ctl[48], cb->proxy_ctl[64],
-                    (unsigned long)cb->issue_tail);
-        }
-        fprintf(stderr, "\n");
-      }
+    if (dbg && (g->stats.loop_iters % 50000000) == 0) {
+      fprintf(stderr, "[dbg gpu%u] iters=%lu admitted=%lu", g->index, (unsigned long)g->stats.loop_iters,
+              (unsigned long)g->stats.admitted);
+      for (uint32_t c = 0; c < N; ++c) fprintf(stderr, " sub[%u]=%lu", c, (unsigned long)g->sub[c]->size());
+      uint32_t nm = P->nmodels.load();
+      for (uint32_t m = 0; m < nm; ++m)
+        fprintf(stderr, " free[%u]=%zu", m, P->models[m]->gpu[g->index].free_slots.size());
+      fprintf(stderr, " live=%lu\n", (unsigned long)g->policy->live_jobs());
     }
     if (!g->ev_pending.empty() && (g->stats.loop_iters & 63) == 0) harvest_events(g);
     g->be->advance();
@@ -1113,13 +1102,13 @@ static int ensure_iso(Gpu* g) {
     return -ENOMEM;
   std::memset(g->prof_ring_h, 0, cap * sizeof(Rec));
   cudaHostGetDevicePointer(&g->prof_ring_d, g->prof_ring_h, 0);
-  if (cudaMalloc(&g->prof_tail, 256) || cudaMalloc(&g->prof_ctr, CTR_WORDS * NCTR * sizeof(uint32_t))) return -ENOMEM;
+  if (cudaMalloc(&g->prof_tail, 256) || cudaMalloc(&g->prof_ctr, 2 * NCTR * sizeof(uint32_t))) return -ENOMEM;
   g->prof_base.assign(NCTR, 0);
   cudaStream_t s;
   cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
   g->prof_stream = s;
   cudaMemsetAsync(g->prof_tail, 0, 256, s);
-  cudaMemsetAsync(g->prof_ctr, 0, CTR_WORDS * NCTR * sizeof(uint32_t), s);
+  cudaMemsetAsync(g->prof_ctr, 0, 2 * NCTR * sizeof(uint32_t), s);
   // isolated runs write their records to device memory (as served kernels do through
   // the proxy); nobody consumes them except the round-trip benchmark's direct ring
   if (cudaMalloc(&g->prof_devring, cap * sizeof(Rec))) return -ENOMEM;
@@ -1146,7 +1135,7 @@ static void iso_launch(Gpu* g, Model* m, uint32_t l, bool instr) {
   ia.tail = g->prof_tail;
   uint32_t uid = g->prof_uid++;
   uint32_t slot = uid % NCTR;
-  ia.ctr = g->prof_ctr + CTR_WORDS * slot;
+  ia.ctr = g->prof_ctr + 2 * slot;
   ia.mask = (1u << 16) - 1;
   ia.log2cap = 16;
   ia.base = g->prof_base[slot];
@@ -1435,7 +1424,7 @@ static InstrArgs iso_instr(Gpu* g, uint32_t grid, uint32_t group, bool last) {
   ia.tail = g->prof_tail;
   uint32_t uid = g->prof_uid++;
   uint32_t slot = uid % NCTR;
-  ia.ctr = g->prof_ctr + CTR_WORDS * slot;
+  ia.ctr = g->prof_ctr + 2 * slot;
   ia.mask = (1u << 16) - 1;
   ia.log2cap = 16;
   ia.base = g->prof_base[slot];

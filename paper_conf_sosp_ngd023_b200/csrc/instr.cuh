@@ -54,10 +54,6 @@ __device__ __forceinline__ void maybe_record(const InstrArgs& ia, uint32_t type,
   }
 }
 
-__device__ __forceinline__ uint32_t lin_block() {
-  return (blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x;
-}
-
 // T = the (1-D) thread that does the bookkeeping; kernels pick an otherwise idle
 // thread so that compute never waits on the counter atomics
 template <bool INSTR, uint32_t T = 0>
@@ -65,8 +61,7 @@ __device__ __forceinline__ void instr_enter(const InstrArgs& ia) {
   if constexpr (INSTR) {
     if (threadIdx.x == T && threadIdx.y == 0 && threadIdx.z == 0) {
       if (ia.flags & INSTR_COUNTERS) {
-        const uint32_t sub = lin_block() % CTR_SUB;
-        asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[sub]) : "memory");
+        asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[0]) : "memory");
       } else {
         uint32_t total = gridDim.x * gridDim.y * gridDim.z;
         uint32_t c = atomicAdd(&ia.ctr[0], 1u) + 1u - ia.base;
@@ -83,20 +78,19 @@ __device__ __forceinline__ void instr_exit(const InstrArgs& ia) {
     if (threadIdx.x == T && threadIdx.y == 0 && threadIdx.z == 0 && (ia.flags & INSTR_COUNTERS)) {
       // release reduction: the block's outputs (ordered before by the barrier) are
       // visible before the proxy can observe the count; nothing to wait for
-      const uint32_t sub = CTR_SUB + lin_block() % CTR_SUB;
       if (ia.flags & INSTR_LAST)
-        asm volatile("red.release.sys.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[sub]) : "memory");
+        asm volatile("red.release.sys.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
       else
-        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[sub]) : "memory");
+        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
     } else if (threadIdx.x == T && threadIdx.y == 0 && threadIdx.z == 0) {
       // acq_rel atomic: releases this block's outputs (ordered before by the barrier,
       // release is cumulative) and acquires the earlier blocks' before the record is
       // written; system scope for a job's last kernel, whose output is in host memory
       uint32_t old;
       if (ia.flags & INSTR_LAST)
-        asm volatile("atom.acq_rel.sys.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(&ia.ctr[CTR_SUB]) : "memory");
+        asm volatile("atom.acq_rel.sys.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(&ia.ctr[1]) : "memory");
       else
-        asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(&ia.ctr[CTR_SUB]) : "memory");
+        asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(&ia.ctr[1]) : "memory");
       uint32_t total = gridDim.x * gridDim.y * gridDim.z;
       maybe_record(ia, REC_COMPLETION, old + 1u - ia.base, total);
     }

@@ -594,20 +594,9 @@ __global__ void __launch_bounds__(128, 1)
     for (uint32_t a = tid; a < na; a += blockDim.x) {
       const uint32_t uid = a_uid[a], grid = a_grid[a], base = a_base[a];
       const uint32_t slot = uid % NCTR;
-      // sum the CTR_SUB start and end sub-counters (4 x 16-byte loads)
-      uint32_t v[16];
-      const uint32_t* cp_ = ctrs + CTR_WORDS * slot;
-#pragma unroll
-      for (int q = 0; q < 4; ++q)
-        asm volatile("ld.volatile.global.v4.u32 {%0,%1,%2,%3}, [%4];"
-                     : "=r"(v[4 * q]), "=r"(v[4 * q + 1]), "=r"(v[4 * q + 2]), "=r"(v[4 * q + 3])
-                     : "l"(cp_ + 4 * q));
-      uint32_t s0 = 0, s1 = 0;
-#pragma unroll
-      for (int q = 0; q < 8; ++q) {
-        s0 += v[q];
-        s1 += v[8 + q];
-      }
+      uint32_t s0, s1;
+      asm volatile("ld.volatile.global.u32 %0, [%1];" : "=r"(s0) : "l"(ctrs + 2 * slot));
+      asm volatile("ld.volatile.global.u32 %0, [%1];" : "=r"(s1) : "l"(ctrs + 2 * slot + 1));
       uint32_t cp = s0 - base, cc = s1 - base;
       if (cp > grid) cp = grid;
       if (cc > grid) cc = grid;
