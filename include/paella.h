@@ -103,10 +103,9 @@ typedef struct {
                                     the durations (paella_stats ev_*): the live roofline */
   uint32_t lookahead;            /* NEXT-1 launch-ahead depth: 0 = the paper's semantics (a
                                     job's next kernel is dispatched after the previous one's
-                                    final COMPLETION); D in 1..6 = once the job's oldest
-                                    in-flight kernel is fully placed (running) and <= D are in
-                                    flight, the next kernel is queued behind it on the same
-                                    stream */
+                                    final COMPLETION); D > 0 = once the previous kernel is
+                                    fully placed and <= D are in flight, the next kernel is
+                                    queued behind it on the same stream */
   uint32_t launch_threads;       /* 0 = each dispatcher calls cudaLaunchKernel itself; n > 0 =
                                     n helper threads per GPU perform the launches (stream s is
                                     owned by helper s % n, so per-stream order is kept); the

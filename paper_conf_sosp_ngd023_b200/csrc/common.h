@@ -59,15 +59,7 @@ PAELLA_HD inline RecFields rec_decode(uint64_t w0, uint64_t w1) {
 
 // Per-launch instrumentation arguments (Fig. 6's extra parameters notifQ, kernId,
 // P887-895, plus the per-launch counter slot -- reading C2-Q1).
-// INSTR_COUNTERS: the block only bumps its launch's {start, end} counters with
-// fire-and-forget reductions; the notification proxy turns counter progress into the
-// same ring records (see kernels_simt.cu::k_notify_counters)
-enum : uint32_t { INSTR_ON = 1u, INSTR_LAST = 2u, INSTR_COUNTERS = 4u };
-
-// launch announcement, dispatcher -> notification proxy (pinned, mapped host memory)
-struct alignas(16) IssueEnt {
-  uint32_t uid, grid, base, seq;   // seq = ring index + 1, written last
-};
+enum : uint32_t { INSTR_ON = 1u, INSTR_LAST = 2u };
 
 struct InstrArgs {
   Rec* ring;          // device-visible pointer to the pinned, mapped ring

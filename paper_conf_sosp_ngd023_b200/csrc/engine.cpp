@@ -186,31 +186,23 @@ struct CudaBackend : Backend {
   uint32_t cap, nstreams;
   Rec* ring_h = nullptr;
   Rec* ring_d = nullptr;      // device view of the pinned host ring
-  // notification proxy (counter mode): instrumented blocks only bump counters; a
-  // resident proxy block turns counter progress into ring records (k_notify_counters)
+  // notification proxy: kernels write to dev_ring (device memory); one persistent warp
+  // forwards to the host ring, so no kernel pays the PCIe write on its exit path
   bool proxy = false;
-  uint32_t group = 16;
-  IssueEnt* issue_h = nullptr;       // pinned mapped launch announcements
-  IssueEnt* issue_d = nullptr;
-  uint64_t issue_tail = 0;
-  static constexpr uint32_t kIssueCap = 8192;
-  uint32_t* proxy_ctl = nullptr;     // pinned mapped: [0] stop [16] heartbeat [32] exited [48] rec [64] issue
+  Rec* dev_ring = nullptr;
+  uint32_t* proxy_ctl = nullptr;     // pinned mapped: [0] stop flag, [16] heartbeat
   cudaStream_t proxy_stream = nullptr;
   uint32_t* tail = nullptr;   // device
   uint32_t* ctr = nullptr;    // device, 2*NCTR
   std::vector<cudaStream_t> streams;
   KernelFn tab[2][2][KIND_COUNT];   // [dtype][instr][kind]
   int err_ = 0;
-  CudaBackend(int d, uint32_t c, uint32_t P, bool px, uint32_t G)
-      : dev(d), cap(c), nstreams(P), proxy(px), group(G) {}
+  CudaBackend(int d, uint32_t c, uint32_t P, bool px) : dev(d), cap(c), nstreams(P), proxy(px) {}
   bool proxy_running = false;
   uint32_t* ctl_d = nullptr;
-  int setup_proxy() {
-    if (cudaHostAlloc((void**)&issue_h, kIssueCap * sizeof(IssueEnt), cudaHostAllocMapped | cudaHostAllocPortable) !=
-        cudaSuccess)
-      return -ENOMEM;
-    std::memset(issue_h, 0, kIssueCap * sizeof(IssueEnt));
-    cudaHostGetDevicePointer((void**)&issue_d, issue_h, 0);
+  int setup_proxy(cudaStream_t s) {
+    if (cudaMalloc(&dev_ring, (size_t)cap * sizeof(Rec)) != cudaSuccess) return -ENOMEM;
+    cudaMemsetAsync(dev_ring, 0, (size_t)cap * sizeof(Rec), s);
     if (cudaHostAlloc((void**)&proxy_ctl, 256, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
       return -ENOMEM;
     std::memset(proxy_ctl, 0, 256);
@@ -218,20 +210,7 @@ struct CudaBackend : Backend {
     if (cudaStreamCreateWithFlags(&proxy_stream, cudaStreamNonBlocking) != cudaSuccess) return -EIO;
     return 0;
   }
-  // dispatcher thread: announce a counted launch to the proxy (before launching it)
-  void announce(uint32_t uid, uint32_t grid, uint32_t base) {
-    // never lap the proxy (bounded by the in-flight launches; practically never waits)
-    while (issue_tail - __atomic_load_n(&proxy_ctl[64], __ATOMIC_ACQUIRE) >= kIssueCap - 64) {
-      ensure_proxy();
-    }
-    IssueEnt* e = &issue_h[issue_tail & (kIssueCap - 1)];
-    e->uid = uid;
-    e->grid = grid;
-    e->base = base;
-    __atomic_store_n(&e->seq, (uint32_t)(issue_tail + 1), __ATOMIC_RELEASE);
-    ++issue_tail;
-  }
-  // dispatcher thread: (re)start the proxy block when records may be outstanding
+  // dispatcher thread: (re)start the forwarding warp when records may be outstanding
   void ensure_proxy() {
     if (!proxy) return;
     if (proxy_running) {
@@ -239,16 +218,13 @@ struct CudaBackend : Backend {
       proxy_running = false;   // it left after an idle spell
     }
     __atomic_store_n(&proxy_ctl[32], 0u, __ATOMIC_RELEASE);
-    const IssueEnt* is = issue_d;
-    uint32_t imask = kIssueCap - 1;
-    const uint32_t* cs = ctr;
+    const Rec* src = dev_ring;
     Rec* dst = ring_d;
-    uint32_t rmask = cap - 1, l2 = 0, G = group;
+    uint32_t mask = cap - 1, l2 = 0;
     while ((1u << l2) < cap) ++l2;
     volatile uint32_t* st = ctl_d;
-    void* args[8] = {(void*)&is, (void*)&imask, (void*)&cs, (void*)&dst, (void*)&rmask, (void*)&l2, (void*)&G,
-                     (void*)&st};
-    if (cudaLaunchKernel((const void*)proxy_kernel(), dim3(1), dim3(128), args, 0, proxy_stream) == cudaSuccess)
+    void* args[5] = {(void*)&src, (void*)&dst, (void*)&mask, (void*)&l2, (void*)&st};
+    if (cudaLaunchKernel((const void*)proxy_kernel(), dim3(1), dim3(32), args, 0, proxy_stream) == cudaSuccess)
       proxy_running = true;
     else if (!err_)
       err_ = (int)cudaErrorLaunchFailure;
@@ -282,7 +258,7 @@ struct CudaBackend : Backend {
     tab[0][0][KIND_CONV_TC_PRO] = tc_p[1];
     for (int i = 0; i < 2; ++i) tab[1][i][KIND_CONV_TC] = tab[1][i][KIND_CONV_TC_PRO] = nullptr;
     if (proxy) {
-      int rc = setup_proxy();
+      int rc = setup_proxy(streams[0]);
       if (rc) return rc;
     }
     // stream-scoped: another engine's forwarding warp may be resident on this device
@@ -292,7 +268,7 @@ struct CudaBackend : Backend {
     cudaSetDevice(dev);
     stop_proxy();
     if (proxy_stream) cudaStreamDestroy(proxy_stream);
-    if (issue_h) cudaFreeHost(issue_h);
+    if (dev_ring) cudaFree(dev_ring);
     if (proxy_ctl) cudaFreeHost(proxy_ctl);
     for (auto& s : streams) cudaStreamDestroy(s);
     if (ring_h) cudaFreeHost(ring_h);
@@ -302,7 +278,7 @@ struct CudaBackend : Backend {
   Rec* ring() override { return ring_h; }
   uint32_t* tail_dev() override { return tail; }
   uint32_t* ctr_dev() override { return ctr; }
-  void* ring_dev() override { return ring_d; }
+  void* ring_dev() override { return proxy ? (void*)dev_ring : (void*)ring_d; }
   KernelFn fn(uint32_t kind, uint32_t dtype, bool instr) { return tab[dtype][instr ? 1 : 0][kind]; }
   void launch(const KernelInst& k, const LayerArgs& a, const InstrArgs& ia, uint32_t stream, uint32_t dtype,
               bool instr) override {
@@ -340,7 +316,7 @@ int make_weight_tmap(void* weights, uint32_t rows, uint32_t kpad, void* out128);
 // ---------------------------------------------------------------------------
 // helpers
 // ---------------------------------------------------------------------------
-static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last, bool instr) {
+static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last) {
   InstrArgs ia;
   ia.ring = (Rec*)g->be->ring_dev();
   ia.tail = g->be->tail_dev();
@@ -353,13 +329,6 @@ static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last, bool
   ia.uid = uid;
   ia.group = g->P->cfg.group_size;
   ia.flags = INSTR_ON | (last ? INSTR_LAST : 0);
-  if (g->P->cfg.device == PAELLA_DEVICE_CUDA) {
-    auto* cb = static_cast<CudaBackend*>(g->be.get());
-    if (cb->proxy) {
-      ia.flags |= INSTR_COUNTERS;
-      if (instr) cb->announce(uid, grid, ia.base);   // uninstrumented twins never count
-    }
-  }
   return ia;
 }
 
@@ -393,7 +362,7 @@ static void launcher_main(Gpu* g, Launcher* L) {
 
 static void do_launch(Gpu* g, Model* m, uint32_t slot, uint32_t layer, uint32_t uid, uint32_t stream, bool instr) {
   const KernelInst& k = m->kernels[layer];
-  InstrArgs ia = make_instr(g, uid, k.grid_total(), layer + 1 == m->kernels.size(), instr);
+  InstrArgs ia = make_instr(g, uid, k.grid_total(), layer + 1 == m->kernels.size());
   const paella_config_t& cfg = g->P->cfg;
   if (!g->launchers.empty()) {
     LaunchDesc d;
@@ -719,9 +688,8 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
   if (cfg.client_region_bytes == 0) cfg.client_region_bytes = 64ull << 20;
   if (cfg.fake_time_scale_ns == 0) cfg.fake_time_scale_ns = 500;
   if (cfg.fairness_threshold < 0) return -EINVAL;
-  if (cfg.lookahead > 6) return -EINVAL;   // uid_of[] tracks up to 8 in flight
+  if (cfg.lookahead > 4) return -EINVAL;
   if (cfg.launch_threads > 16) return -EINVAL;
-  if (!cfg.naive && !cfg.instrument) return -EINVAL;   // the dispatcher needs the notifications
 
   auto P = std::make_unique<Paella>();
   P->cfg = cfg;
@@ -774,7 +742,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     g->jobs.reserve(65536);
     if (cfg.device == PAELLA_DEVICE_CUDA)
       g->be.reset(new CudaBackend(g->device, g->cap, cfg.stream_pool,
-                                  cfg.no_proxy == 0 && !std::getenv("PAELLA_NO_PROXY"), cfg.group_size));
+                                  cfg.no_proxy == 0 && !std::getenv("PAELLA_NO_PROXY")));
     else
       g->be.reset(new FakeBackend(P->sms, g->cap, g->log2cap, cfg.group_size, cfg.stream_pool,
                                   cfg.fake_time_scale_ns));
@@ -1121,10 +1089,9 @@ static int ensure_iso(Gpu* g) {
 
 // the ring isolated runs write to: device memory when served kernels go through the
 // notification proxy (same cost as in serving), else the pinned host ring
-static Rec* iso_ring(Gpu* g) { return (Rec*)g->prof_ring_d; }
-static uint32_t iso_mode(Gpu* g) {
+static Rec* iso_ring(Gpu* g) {
   auto* cb = static_cast<CudaBackend*>(g->be.get());
-  return cb->proxy ? INSTR_COUNTERS : 0u;   // same kernel-side cost as in serving
+  return cb->proxy ? g->prof_devring : (Rec*)g->prof_ring_d;
 }
 
 // launch kernel `l` of model m from the isolated slot on the profiling stream
@@ -1142,7 +1109,7 @@ static void iso_launch(Gpu* g, Model* m, uint32_t l, bool instr) {
   g->prof_base[slot] += k.grid_total();
   ia.uid = uid;
   ia.group = g->P->cfg.group_size;
-  ia.flags = INSTR_ON | (l + 1 == m->kernels.size() ? INSTR_LAST : 0) | iso_mode(g);
+  ia.flags = INSTR_ON | (l + 1 == m->kernels.size() ? INSTR_LAST : 0);
   uint32_t iso_slot = (uint32_t)m->gpu[g->index].args.size() - 1;
   auto* cb = static_cast<CudaBackend*>(g->be.get());
   const void* tm = is_tc(k.kind) ? m->gpu[g->index].tmaps[l].b : nullptr;
@@ -1431,7 +1398,7 @@ static InstrArgs iso_instr(Gpu* g, uint32_t grid, uint32_t group, bool last) {
   g->prof_base[slot] += grid;
   ia.uid = uid;
   ia.group = group;
-  ia.flags = INSTR_ON | (last ? INSTR_LAST : 0) | iso_mode(g);
+  ia.flags = INSTR_ON | (last ? INSTR_LAST : 0);
   return ia;
 }
 
@@ -1498,7 +1465,7 @@ int paella_bench_empty(paella_t* p, uint32_t gpu, uint32_t grid, uint32_t block,
   LayerArgs la{};
   // experiment: PAELLA_BENCH_DEVRING=1 writes the records to device memory instead of
   // the pinned host ring (isolates the cost of the PCIe write + kernel-end flush)
-  const bool direct = std::getenv("PAELLA_BENCH_DIRECT") != nullptr;   // block-written records
+  Rec* devring = std::getenv("PAELLA_BENCH_DIRECT") ? (Rec*)g->prof_ring_d : g->prof_devring;
   const volatile uint32_t* gd;
   volatile uint32_t* gate = gate_ptr(g, &gd);
   cudaEvent_t e0, e1;
@@ -1515,7 +1482,7 @@ int paella_bench_empty(paella_t* p, uint32_t gpu, uint32_t grid, uint32_t block,
     cudaEventRecord(e0, s);
     for (uint32_t i = 0; i < nb; ++i) {
       InstrArgs ia = iso_instr(g, grid, group, false);
-      if (direct) ia.flags &= ~INSTR_COUNTERS;
+      if (devring) ia.ring = devring;
       void* args[2] = {(void*)&la, (void*)&ia};
       cudaLaunchKernel((const void*)f, dim3(grid), dim3(block), args, 0, s);
     }
@@ -1556,7 +1523,6 @@ int paella_bench_roundtrip(paella_t* p, uint32_t gpu, uint32_t n, int64_t* place
   for (uint32_t i = 0; i < n; ++i) {
     InstrArgs ia = iso_instr(g, 1, 1, false);
     ia.ring = (Rec*)g->prof_ring_d;   // direct write to the pinned host ring
-    ia.flags &= ~INSTR_COUNTERS;
     void* args[2] = {(void*)&la, (void*)&ia};
     int64_t t0 = now_ns();
     cudaLaunchKernel((const void*)f, dim3(1), dim3(32), args, 0, s);

@@ -523,145 +523,56 @@ __global__ void k_gate(const volatile uint32_t* flag) {
 KernelFn gate_kernel() { return (KernelFn)k_gate; }
 
 // ---------------------------------------------------------------------------
-// Notification proxy (counter mode).  Instrumented blocks only bump their launch's
-// {start, end} counters with fire-and-forget reductions (instr.cuh, INSTR_COUNTERS);
-// this resident 128-thread block learns of every launch from the dispatcher's issue
-// ring (pinned host memory), polls the counters of the launches in flight, and for
-// every group of G blocks that has started / finished writes exactly the record the
-// block reaching count % G == 0 (or the grid total) would have written (Fig. 6),
-// into the pinned host ring the dispatcher drains.  Records carry smid 0xFF (not
-// known here) and the proxy's %globaltimer.  It leaves after ~35 ms with nothing in
-// flight (resumable: ring and issue indices are saved in `state`), so device-wide
-// synchronisation elsewhere can be delayed by it but never deadlocks.
-// state: [0] stop, [16] heartbeat, [32] exited, [48] record index, [64] issue index.
+// Notification proxy: one persistent warp forwards records from the device-memory
+// ring (where the instrumented kernels write them: an L2 store, no PCIe write on the
+// kernels' exit path) to the pinned host ring the dispatcher polls.  Lane i checks
+// slot head+i; the valid prefix of the window is copied with one 16-byte store per
+// lane and the device slots are cleared.  Order and lap tags are preserved, so the
+// host sees exactly the records it would see with direct writes.
 // ---------------------------------------------------------------------------
-constexpr uint32_t PROXY_MAX_ACTIVE = 1024;
-
-__device__ __forceinline__ uint32_t groups_done(uint32_t c, uint32_t grid, uint32_t G) {
-  return c >= grid ? (grid + G - 1) / G : c / G;
-}
-
-__global__ void __launch_bounds__(128, 1)
-    k_notify_counters(const IssueEnt* issue, uint32_t imask, const uint32_t* ctrs, Rec* host_ring, uint32_t rmask,
-                      uint32_t log2cap, uint32_t G, volatile uint32_t* state) {
-  __shared__ uint32_t a_uid[PROXY_MAX_ACTIVE], a_grid[PROXY_MAX_ACTIVE], a_base[PROXY_MAX_ACTIVE];
-  __shared__ uint32_t a_rp[PROXY_MAX_ACTIVE], a_rc[PROXY_MAX_ACTIVE];
-  __shared__ uint8_t a_alive[PROXY_MAX_ACTIVE];
-  __shared__ uint32_t n_act, rec_tail, ihead, quit;
-  const uint32_t tid = threadIdx.x, lane = tid % 32, warp = tid / 32;
-  if (tid == 0) {
-    n_act = 0;
-    rec_tail = state[48];
-    ihead = state[64];
-    quit = 0;
-  }
-  __syncthreads();
+__global__ void __launch_bounds__(32, 1) k_notify_proxy(const Rec* dev_ring, Rec* host_ring, uint32_t mask,
+                                                        uint32_t log2cap, volatile uint32_t* state) {
+  // state (pinned, mapped): [0] stop request, [16] heartbeat, [32] exited flag,
+  // [48] ring index to resume from.  The warp leaves on its own after ~20 ms without
+  // records (so device-wide synchronisation elsewhere in the process can never wait
+  // on it forever); the dispatcher relaunches it when it has records outstanding.
+  const uint32_t lane = threadIdx.x;
+  uint32_t head = state[48];
   uint32_t idle = 0;
   for (;;) {
-    // (a) warp 0 takes new launch announcements (a 16-byte read per lane)
-    if (warp == 0) {
-      const uint32_t h = ihead;
-      const uint32_t idx = h + lane;
-      uint32_t e0, e1, e2, e3;
-      asm volatile("ld.volatile.global.v4.u32 {%0,%1,%2,%3}, [%4];"
-                   : "=r"(e0), "=r"(e1), "=r"(e2), "=r"(e3)
-                   : "l"(issue + (idx & imask)));
-      const bool valid = e3 == idx + 1;
-      const uint32_t bal = __ballot_sync(0xffffffffu, valid);
-      uint32_t k = (bal == 0xffffffffu) ? 32u : (uint32_t)(__ffs(~bal) - 1);
-      const uint32_t room = PROXY_MAX_ACTIVE - n_act;
-      if (k > room) k = room;
-      if (lane < k) {
-        const uint32_t a = n_act + lane;
-        a_uid[a] = e0;
-        a_grid[a] = e1;
-        a_base[a] = e2;
-        a_rp[a] = 0;
-        a_rc[a] = 0;
-        a_alive[a] = 1;
-      }
-      __syncwarp();
-      if (lane == 0 && k) {
-        n_act += k;
-        ihead = h + k;
-        state[64] = h + k;
-      }
+    const uint32_t idx = head + lane;
+    const Rec* src = dev_ring + (idx & mask);
+    uint64_t w0, w1;
+    asm volatile("ld.volatile.global.v2.u64 {%0, %1}, [%2];" : "=l"(w0), "=l"(w1) : "l"(src));
+    const uint32_t tag = rec_tag(idx >> log2cap);
+    const bool valid = (w0 & 0xff) != REC_INVALID && ((w0 >> 24) & 0xff) == tag && (w1 >> 56) == tag;
+    const uint32_t bal = __ballot_sync(0xffffffffu, valid);
+    const uint32_t n = (bal == 0xffffffffu) ? 32u : (uint32_t)(__ffs(~bal) - 1);   // valid prefix
+    if (lane < n) {
+      Rec* dst = host_ring + (idx & mask);
+      asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(dst), "l"(w0), "l"(w1) : "memory");
+      asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(src), "l"(0ull), "l"(0ull) : "memory");
     }
-    __syncthreads();
-    // (b) every thread polls some launches and emits the records they owe
-    const uint32_t na = n_act;
-    bool any = false;
-    for (uint32_t a = tid; a < na; a += blockDim.x) {
-      const uint32_t uid = a_uid[a], grid = a_grid[a], base = a_base[a];
-      const uint32_t slot = uid % NCTR;
-      uint32_t s0, s1;
-      asm volatile("ld.volatile.global.u32 %0, [%1];" : "=r"(s0) : "l"(ctrs + 2 * slot));
-      asm volatile("ld.volatile.global.u32 %0, [%1];" : "=r"(s1) : "l"(ctrs + 2 * slot + 1));
-      uint32_t cp = s0 - base, cc = s1 - base;
-      if (cp > grid) cp = grid;
-      if (cc > grid) cc = grid;
-      const uint32_t gp0 = groups_done(a_rp[a], grid, G), gp1 = groups_done(cp, grid, G);
-      const uint32_t gc0 = groups_done(a_rc[a], grid, G), gc1 = groups_done(cc, grid, G);
-      const uint32_t nrec = (gp1 - gp0) + (gc1 - gc0);
-      if (nrec) {
-        any = true;
-        uint32_t idx = atomicAdd(&rec_tail, nrec);
-        const uint64_t now = globaltimer();
-        const uint32_t last_n = grid % G ? grid % G : G;
-        for (uint32_t gI = gp0; gI < gp1; ++gI, ++idx) {
-          const uint32_t n = (gI + 1) * G >= grid ? last_n : G;
-          Rec r = rec_encode(REC_PLACEMENT, n, 0xff, idx >> log2cap, uid, now, gI);
-          asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(host_ring + (idx & rmask)), "l"(r.w0), "l"(r.w1)
-                       : "memory");
-        }
-        for (uint32_t gI = gc0; gI < gc1; ++gI, ++idx) {
-          const uint32_t n = (gI + 1) * G >= grid ? last_n : G;
-          Rec r = rec_encode(REC_COMPLETION, n, 0xff, idx >> log2cap, uid, now, gI);
-          asm volatile("st.global.v2.u64 [%0], {%1, %2};" ::"l"(host_ring + (idx & rmask)), "l"(r.w0), "l"(r.w1)
-                       : "memory");
-        }
-        a_rp[a] = cp;
-        a_rc[a] = cc;
-        if (cc == grid) a_alive[a] = 0;
+    head += n;
+    if (n == 0) {
+      ++idle;
+      if ((idle & 255) == 0) {
+        if (state[0] || idle > (1u << 16)) break;
+        if (lane == 0) state[16] = head;
       }
+      __nanosleep(64);
+    } else {
+      idle = 0;
     }
-    const bool busy = __syncthreads_or(any);
-    // (c) thread 0 compacts the table and decides whether to stay
-    if (tid == 0) {
-      uint32_t w = 0;
-      for (uint32_t a = 0; a < n_act; ++a) {
-        if (!a_alive[a]) continue;
-        if (w != a) {
-          a_uid[w] = a_uid[a];
-          a_grid[w] = a_grid[a];
-          a_base[w] = a_base[a];
-          a_rp[w] = a_rp[a];
-          a_rc[w] = a_rc[a];
-          a_alive[w] = 1;
-        }
-        ++w;
-      }
-      n_act = w;
-      if (busy) {
-        idle = 0;
-      } else if ((++idle & 255) == 0) {
-        if (state[0] || (n_act == 0 && idle > (1u << 16))) quit = 1;
-        state[16] = rec_tail;
-      }
-    }
-    __syncthreads();
-    if (quit) break;
-    if (!busy) __nanosleep(32);
   }
-  if (tid == 0) {
-    state[48] = rec_tail;
-    state[64] = ihead;
+  if (lane == 0) {
+    state[48] = head;
     __threadfence_system();
     state[32] = 1;
   }
 }
 
-KernelFn proxy_kernel() { return (KernelFn)k_notify_counters; }
+KernelFn proxy_kernel() { return (KernelFn)k_notify_proxy; }
 
 // ---------------------------------------------------------------------------
 // kernel table

@@ -163,9 +163,7 @@ def test_ring_records_carry_sm_and_time(tmp_path):
     of a block's group never before the first placement of its launch."""
     log = str(tmp_path / "g1_%u.log")
     g = archs.toy()
-    # direct mode: blocks write their own records (with SM id); the proxy's records
-    # carry smid 0xFF
-    with L.Engine(num_clients=1, group=1, event_log=log, proxy=False) as e:
+    with L.Engine(num_clients=1, group=1, event_log=log) as e:
         mid = e.register_model(g, rng.model_params(g))
         _serve_and_check(e, [(mid, "toy", g)], 10, 1, seed=1)
     cfg, ms, events, ex = eventlog.read(log % 0)
@@ -187,8 +185,7 @@ def test_per_sm_capacity_from_g1_records(tmp_path):
     Table-1 resources (+TMEM) according to the demands the dispatcher accounts."""
     log = str(tmp_path / "cap_%u.log")
     names = ["resnet18", "mobilenet_v2", "squeezenet1_1"]
-    with L.Engine(num_clients=3, group=1, event_log=log, ring_capacity=4096, lookahead=1, launch_threads=2,
-                  proxy=False) as e:
+    with L.Engine(num_clients=3, group=1, event_log=log, ring_capacity=4096, lookahead=1, launch_threads=2) as e:
         specs = []
         for nm in names:
             g = archs.build(nm)
