@@ -278,7 +278,8 @@ def run_gpu(args, dist):
     dist.barrier()
     clk = clocks.stop()
     st1 = e.stats()
-    stats = {k: st1[k] - st0[k] for k in st1}
+    stats = {k: ([a - b for a, b in zip(st1[k], st0[k])] if isinstance(st1[k], list) else st1[k] - st0[k])
+             for k in st1}
     # dominant kernel (tcgen05 conv): algorithmic bytes / CUDA-event duration of the
     # served (instrumented) kernels, launched back to back on their stream
     ev = {"launches": 0, "ns": 0, "bytes": 0, "flops": 0, "all_ns": 0}
@@ -458,7 +459,7 @@ def main():
                 "d2h_bytes_per_step": round(res["d2h"] * args.reqs), "jct_us": res["e2e"]["mix"]},
         "gpu_launches": int(launches),
         "clocks": res["clocks"],
-        "dispatcher": {k: int(v) for k, v in res["stats"].items()},
+        "dispatcher": {k: (v if isinstance(v, list) else int(v)) for k, v in res["stats"].items()},
     }
     if args.gpus == 1 and not args.fake:
         line["cpu_baseline"] = cpu_baseline(cfg, seconds=12.0)

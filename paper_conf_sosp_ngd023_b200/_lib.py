@@ -83,7 +83,9 @@ class Stats(C.Structure):
     _fields_ = [("admitted", C.c_uint64), ("completed", C.c_uint64), ("launches", C.c_uint64),
                 ("records", C.c_uint64), ("torn_retries", C.c_uint64), ("decide_calls", C.c_uint64),
                 ("loop_iters", C.c_uint64), ("outstanding_work_ns", C.c_int64), ("ev_launches", C.c_uint64),
-                ("ev_ns", C.c_uint64), ("ev_bytes", C.c_uint64), ("ev_flops", C.c_uint64)]
+                ("ev_ns", C.c_uint64), ("ev_bytes", C.c_uint64), ("ev_flops", C.c_uint64),
+                ("stop_reason", C.c_uint64 * 4), ("sum_ready", C.c_uint64), ("sum_live_jobs", C.c_uint64),
+                ("sum_Q", C.c_uint64)]
 
 
 _lib = None
@@ -343,7 +345,9 @@ class Engine:
     def stats(self, gpu=0):
         st = Stats()
         _check(self.lib.paella_stats(self.h, gpu, C.byref(st)), "paella_stats")
-        return {f: getattr(st, f) for f, _ in Stats._fields_}
+        d = {f: getattr(st, f) for f, _ in Stats._fields_}
+        d["stop_reason"] = list(st.stop_reason)
+        return d
 
     def flush_log(self):
         self.lib.paella_flush_log(self.h)

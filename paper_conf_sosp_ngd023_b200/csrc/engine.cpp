@@ -537,6 +537,10 @@ static void decide_and_launch(Gpu* g) {
   if (!g->issues.empty() && g->P->cfg.device == PAELLA_DEVICE_CUDA)
     static_cast<CudaBackend*>(g->be.get())->ensure_proxy();
   g->stats.decide_calls++;
+  g->stats.stop_reason[g->policy->last_stop()]++;
+  g->stats.sum_ready += g->policy->ready_count();
+  g->stats.sum_live_jobs += g->policy->live_jobs();
+  g->stats.sum_Q += (uint64_t)(g->policy->Q() > 0 ? g->policy->Q() : 0);
   for (const Issue& is : g->issues) {
     JobRec& j = g->jobs[is.job];
     Model* m = g->P->models[j.model].get();

@@ -164,12 +164,22 @@ bool Policy::predicate(uint32_t grid) const {
 void Policy::decide(std::vector<Issue>* out) {
   for (;;) {
     uint32_t jid;
-    if (!pick(&jid)) break;
+    if (!pick(&jid)) {
+      last_stop_ = 0;
+      break;
+    }
     PolicyJob& j = jobs_[jid];
     int s0 = lowest_free();
-    if (j.inflight() == 0 && s0 < 0) break;
+    if (j.inflight() == 0 && s0 < 0) {
+      last_stop_ = 1;
+      break;
+    }
     const PolicyLayer& lay = models_[j.model][j.cursor];
-    if (!predicate(lay.grid)) break;
+    if (!predicate(lay.grid)) {
+      int64_t recs = 2 * (int64_t)((lay.grid + cfg_.group - 1) / cfg_.group);
+      last_stop_ = O_ + recs <= cfg_.ring_capacity ? 2 : 3;
+      break;
+    }
     uint32_t uid = next_uid_++;
     uint32_t stream;
     if (j.inflight() > 0) {

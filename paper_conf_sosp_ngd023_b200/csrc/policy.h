@@ -90,6 +90,9 @@ class Policy {
   const PolicyLaunch& launch(uint32_t uid) const { return launches_[uid % kLaunchSlots]; }
   int64_t deficit(uint32_t c) const { return Dt_[c] + Omega_; }
   int64_t Q() const { return Q_; }
+  // why the last decide() stopped: 0 nothing ready, 1 no free stream, 2 fits, 3 ring
+  int last_stop() const { return last_stop_; }
+  size_t ready_count() const { return srpt_.size(); }
   int64_t O() const { return O_; }
 
  private:
@@ -109,6 +112,7 @@ class Policy {
   std::vector<PolicyLaunch> launches_;
   int64_t U_[NRES] = {0, 0, 0, 0, 0};
   int64_t Q_ = 0, O_ = 0;
+  int last_stop_ = 0;
   std::vector<uint64_t> free_;   // bitmap of free streams
   std::vector<int64_t> Dt_;
   int64_t Omega_ = 0;
