@@ -52,7 +52,7 @@ def parse():
     ap.add_argument("--reqs", type=int, default=2000, help="requests per step")
     ap.add_argument("--no-baselines", action="store_true")
     ap.add_argument("--lookahead", type=int, default=1, help="NEXT-1 launch-ahead depth of the Paella arm")
-    ap.add_argument("--launch-threads", type=int, default=2, help="launcher helper threads per GPU")
+    ap.add_argument("--launch-threads", type=int, default=4, help="launcher helper threads per GPU")
     ap.add_argument("--sat-reqs", type=int, default=1500, help="requests of the saturation calibration")
     ap.add_argument("--fake", action="store_true",
                     help="CPU fake device (tests of the multi-rank plumbing; not a measurement)")

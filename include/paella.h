@@ -115,6 +115,11 @@ typedef struct {
                                     them to the pinned host ring (keeps the PCIe write off every
                                     kernel's exit path); 1: kernels write the host ring directly,
                                     as in the paper (P1104-1106) */
+  uint32_t no_pdl;               /* 0 (default): kernels are launched with programmatic
+                                    dependent launch (a kernel queued behind another on its
+                                    stream starts ~0.6 us after it instead of on the next
+                                    ~2 us front-end quantum); 1: plain launches.
+                                    The naive baseline always uses plain launches. */
 } paella_config_t;
 
 /* ---- model description (input to paella_register_model) ---------------- */

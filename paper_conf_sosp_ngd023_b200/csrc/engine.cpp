@@ -162,23 +162,37 @@ struct FakeBackend : Backend {
 // one launch of kernel k: split-K tcgen05 convs are thread-block clusters
 static bool is_tc(uint32_t kind) { return kind == KIND_CONV_TC || kind == KIND_CONV_TC_PRO; }
 
-static cudaError_t cuda_launch(KernelFn fn, const KernelInst& k, void** args, cudaStream_t s) {
+// pdl: programmatic dependent launch (programmatic stream serialization).  Measured on
+// B200 (tools/launch_quantum.cu, profiles/launch_quantum_r1.txt): a kernel queued
+// behind another on the same stream starts on a ~2.05 us quantum with a plain launch
+// (a 1 us kernel costs 4.1 us back to back) but 0.6 us after its predecessor with
+// PDL.  Every kernel executes griddepcontrol.wait before touching its inputs
+// (instr.cuh), and none triggers early, so the dependency semantics are unchanged:
+// the successor's blocks are placed only once the predecessor has completed.
+static cudaError_t cuda_launch(KernelFn fn, const KernelInst& k, void** args, cudaStream_t s, bool pdl) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(k.grid[0], k.grid[1], k.grid[2]);
+  cfg.blockDim = dim3(k.block);
+  cfg.dynamicSmemBytes = k.smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[2];
+  uint32_t n = 0;
   if (is_tc(k.kind) && k.proto.ksplit > 1) {
-    cudaLaunchConfig_t cfg{};
-    cfg.gridDim = dim3(k.grid[0], k.grid[1], k.grid[2]);
-    cfg.blockDim = dim3(k.block);
-    cfg.dynamicSmemBytes = k.smem;
-    cfg.stream = s;
-    cudaLaunchAttribute at[1];
-    at[0].id = cudaLaunchAttributeClusterDimension;
-    at[0].val.clusterDim.x = 1;
-    at[0].val.clusterDim.y = 1;
-    at[0].val.clusterDim.z = k.proto.ksplit;
-    cfg.attrs = at;
-    cfg.numAttrs = 1;
-    return cudaLaunchKernelExC(&cfg, (const void*)fn, args);
+    at[n].id = cudaLaunchAttributeClusterDimension;
+    at[n].val.clusterDim.x = 1;
+    at[n].val.clusterDim.y = 1;
+    at[n].val.clusterDim.z = k.proto.ksplit;
+    ++n;
   }
-  return cudaLaunchKernel((const void*)fn, dim3(k.grid[0], k.grid[1], k.grid[2]), dim3(k.block), args, k.smem, s);
+  if (pdl) {
+    at[n].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[n].val.programmaticStreamSerializationAllowed = 1;
+    ++n;
+  }
+  if (n == 0) return cudaLaunchKernel((const void*)fn, cfg.gridDim, cfg.blockDim, args, k.smem, s);
+  cfg.attrs = at;
+  cfg.numAttrs = n;
+  return cudaLaunchKernelExC(&cfg, (const void*)fn, args);
 }
 
 struct CudaBackend : Backend {
@@ -189,6 +203,7 @@ struct CudaBackend : Backend {
   // notification proxy: kernels write to dev_ring (device memory); one persistent warp
   // forwards to the host ring, so no kernel pays the PCIe write on its exit path
   bool proxy = false;
+  bool pdl = true;             // programmatic dependent launches (off for the naive baseline)
   Rec* dev_ring = nullptr;
   uint32_t* proxy_ctl = nullptr;     // pinned mapped: [0] stop flag, [16] heartbeat
   cudaStream_t proxy_stream = nullptr;
@@ -283,7 +298,7 @@ struct CudaBackend : Backend {
   void launch(const KernelInst& k, const LayerArgs& a, const InstrArgs& ia, uint32_t stream, uint32_t dtype,
               bool instr) override {
     void* args[3] = {(void*)&a, (void*)&ia, (void*)k_tmap(k)};
-    cudaError_t e = cuda_launch(fn(k.kind, dtype, instr), k, args, streams[stream]);
+    cudaError_t e = cuda_launch(fn(k.kind, dtype, instr), k, args, streams[stream], pdl);
     if (e != cudaSuccess && !err_) err_ = (int)e;
   }
   // the tensor map of a tcgen05 conv is stored right after its KernelInst's proto
@@ -350,7 +365,7 @@ static void launcher_main(Gpu* g, Launcher* L) {
     }
     if (d->kind == 0) {
       void* args[3] = {(void*)&d->a, (void*)&d->ia, (void*)d->tmap};
-      cudaError_t e = cuda_launch(cb->fn(d->k->kind, d->dtype, d->instr != 0), *d->k, args, cb->streams[d->stream]);
+      cudaError_t e = cuda_launch(cb->fn(d->k->kind, d->dtype, d->instr != 0), *d->k, args, cb->streams[d->stream], cb->pdl);
       if (e != cudaSuccess) g->launch_err.store((int)e);
     } else {
       cudaEventRecord((cudaEvent_t)d->event, cb->streams[d->stream]);
@@ -747,6 +762,8 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     if (cfg.device == PAELLA_DEVICE_CUDA)
       g->be.reset(new CudaBackend(g->device, g->cap, cfg.stream_pool,
                                   cfg.no_proxy == 0 && !std::getenv("PAELLA_NO_PROXY")));
+    if (cfg.device == PAELLA_DEVICE_CUDA)
+      static_cast<CudaBackend*>(g->be.get())->pdl = !cfg.naive && !cfg.no_pdl && !std::getenv("PAELLA_NO_PDL");
     else
       g->be.reset(new FakeBackend(P->sms, g->cap, g->log2cap, cfg.group_size, cfg.stream_pool,
                                   cfg.fake_time_scale_ns));
@@ -1118,7 +1135,7 @@ static void iso_launch(Gpu* g, Model* m, uint32_t l, bool instr) {
   auto* cb = static_cast<CudaBackend*>(g->be.get());
   const void* tm = is_tc(k.kind) ? m->gpu[g->index].tmaps[l].b : nullptr;
   void* args[3] = {(void*)&m->gpu[g->index].args[iso_slot][l], (void*)&ia, (void*)tm};
-  cuda_launch(cb->fn(k.kind, m->dtype, instr), k, args, (cudaStream_t)g->prof_stream);
+  cuda_launch(cb->fn(k.kind, m->dtype, instr), k, args, (cudaStream_t)g->prof_stream, cb->pdl);
 }
 
 static int iso_run(Gpu* g, Model* m, const void* input, void* output, int64_t* kernel_ns, bool instr) {
@@ -1438,7 +1455,7 @@ int paella_time_kernels(paella_t* p, uint32_t gpu, uint32_t model_id, uint32_t i
     for (uint32_t r = 0; r < std::min(reps, 256u); ++r) {
       InstrArgs ia = iso_instr(g, k.grid_total(), P->cfg.group_size, l + 1 == m->kernels.size());
       void* args[3] = {(void*)&m->gpu[gpu].args[iso_slot][l], (void*)&ia, (void*)tm};
-      cuda_launch(cb->fn(k.kind, m->dtype, instrumented != 0), k, args, s);
+      cuda_launch(cb->fn(k.kind, m->dtype, instrumented != 0), k, args, s, cb->pdl);
     }
     cudaEventRecord(e1, s);
     std::atomic_thread_fence(std::memory_order_seq_cst);

@@ -65,6 +65,11 @@ __device__ __forceinline__ void instr_enter(const InstrArgs& ia) {
       maybe_record(ia, REC_PLACEMENT, c, total);
     }
   }
+  // programmatic dependent launch: wait until the kernel this one was queued behind
+  // has completed and its memory is visible (a no-op for plain launches).  No kernel
+  // triggers its dependents early, so blocks are placed (and report PLACEMENT) only
+  // once the predecessor has finished, as without PDL.
+  asm volatile("griddepcontrol.wait;" ::: "memory");
 }
 
 template <bool INSTR, uint32_t T = 0>
