@@ -120,6 +120,14 @@ typedef struct {
                                     stream starts ~0.6 us after it instead of on the next
                                     ~2 us front-end quantum); 1: plain launches.
                                     The naive baseline always uses plain launches. */
+  uint32_t prio_classes;         /* 0/1 = one class (the paper).  K > 1: the stream pool is split
+                                    into K classes of consecutive indices created with
+                                    descending hardware stream priority; a job takes a stream
+                                    of the class of its remaining work R_j (number of
+                                    registered models whose whole-job T-bar sum is below R_j,
+                                    clamped to K-1; deficit-override picks take class 0), so the
+                                    blocks the +B slack keeps queued in hardware are also served
+                                    shortest-remaining first (B200-Q2).  K <= P. */
 } paella_config_t;
 
 /* ---- model description (input to paella_register_model) ---------------- */

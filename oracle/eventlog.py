@@ -5,7 +5,7 @@ Format (DESIGN.md §"Event log"): a sequence of 32-byte little-endian records
 ``{u32 type, u32 a, u64 b, u64 c, u64 d}``:
 
   100 CONFIG    a=N clients, b=policy, c=theta, d=(B << 32) | G
-  100 CONFIG    a=0xFFFFFFFF, b=ring capacity, c=stream pool P, d=launch-ahead depth
+  100 CONFIG    a=0xFFFFFFFF, b=ring capacity, c=stream pool P, d=(priority classes << 32) | launch-ahead depth
   101 CAPACITY  a=resource r, b=C_r
   110 MODEL     a=model, b=#kernels
   111 LAYER     a=model, b=layer, c=grid, d=T-bar ns
@@ -43,7 +43,8 @@ def read(path):
             if a == 0xFFFFFFFF:
                 cfg_kw["ring_capacity"] = b
                 cfg_kw["streams"] = c
-                cfg_kw["lookahead"] = d
+                cfg_kw["lookahead"] = d & 0xFFFFFFFF
+                cfg_kw["prio_classes"] = max(1, d >> 32)
             else:
                 cfg_kw["num_clients"] = a
                 cfg_kw["policy"] = b

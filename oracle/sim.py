@@ -54,6 +54,7 @@ class Config:
     streams: int = 32                 # P
     capacity: tuple = (148 * 32, 148 * 64, 148 * 65536, 148 * 233472, 148 * 512)
     lookahead: int = 0                # NEXT-1 launch-ahead depth (0 = the paper's semantics)
+    prio_classes: int = 1             # stream-priority classes (1 = the paper: one class)
 
 
 def groups(g, G):
@@ -114,6 +115,7 @@ class Policy:
         self.next_seq = 0
         self.completed: list[int] = []
         self.issues: list[tuple] = []
+        self.over = False                    # the last pick was a deficit override
         self.checks = True                   # assert invariants (c),(d),(g) as we go
         self.log: list[tuple] | None = None  # consumed-event log in replay format
 
@@ -189,13 +191,31 @@ class Policy:
 
     def pick(self, rdy):
         cfg = self.cfg
+        self.over = False
         if cfg.policy == FIFO:
             return min(rdy, key=lambda j: j.seq)
         clients = sorted({j.client for j in rdy})
         cstar = max(clients, key=lambda c: (self.D(c), -c))
-        if cfg.theta != INF_THETA and self.D(cstar) > cfg.theta * cfg.num_clients:
+        self.over = cfg.theta != INF_THETA and self.D(cstar) > cfg.theta * cfg.num_clients
+        if self.over:
             return min((j for j in rdy if j.client == cstar), key=lambda j: j.seq)
         return min(rdy, key=lambda j: (j.R, j.seq, j.id))
+
+    # Stream-priority classes (B200 adaptation, reading B200-Q2).  The pool's
+    # P streams are split into K classes of consecutive indices (class 0 = highest
+    # hardware priority), so the blocks the +B slack leaves queued in hardware
+    # (P1300-1304) are served in SRPT order too.  A job takes a stream of the class
+    # of its remaining work: the number of registered models whose whole-job T-bar sum
+    # is strictly below R_j (clamped to K-1); a deficit-override pick takes class 0.
+    def stream_class(self, s):
+        return s * self.cfg.prio_classes // self.cfg.streams
+
+    def job_class(self, j):
+        K = self.cfg.prio_classes
+        if K <= 1 or self.over:
+            return 0
+        totals = sorted({sum(layer.tbar for layer in m) for m in self.models if m})
+        return min(K - 1, sum(1 for t in totals if t < j.R))
 
     def predicate(self, grid):
         cfg = self.cfg
@@ -224,7 +244,12 @@ class Policy:
             if j.inflight > 0:
                 stream = j.stream            # launch-ahead: behind its predecessor
             else:
-                stream = j.last_stream if j.last_stream in self.free else min(self.free)
+                c = self.job_class(j)
+                if j.last_stream in self.free and self.stream_class(j.last_stream) == c:
+                    stream = j.last_stream
+                else:
+                    cand = [s for s in self.free if self.stream_class(s) == c]
+                    stream = min(cand) if cand else min(self.free)
                 self.free.remove(stream)
                 j.stream = stream
             self.launches[uid] = Launch(uid, j.id, j.cursor, layer.grid, layer.demand, stream)

@@ -45,7 +45,8 @@ class Config(C.Structure):
                 ("dispatcher_cpus", C.POINTER(C.c_int32)), ("event_log_path", C.c_char_p),
                 ("fake_sms", C.c_uint32), ("fake_time_scale_ns", C.c_uint32), ("event_time_kind", C.c_uint32),
                 ("lookahead", C.c_uint32), ("launch_threads", C.c_uint32),
-                ("no_proxy", C.c_uint32), ("no_pdl", C.c_uint32)]
+                ("no_proxy", C.c_uint32), ("no_pdl", C.c_uint32),
+                ("prio_classes", C.c_uint32)]
 
 
 class Node(C.Structure):
@@ -148,7 +149,7 @@ class Engine:
                  streams=32, route=ROUTE_LEAST_WORK, submit_slots=1024, max_jobs_per_model=128,
                  instrument=True, naive=False, region_bytes=64 << 20, dispatcher_cpus=None,
                  event_log=None, fake_sms=0, fake_time_scale_ns=0, event_time_kind=None, lookahead=0,
-                 launch_threads=0, proxy=True, pdl=True):
+                 launch_threads=0, proxy=True, pdl=True, prio_classes=1):
         self.lib = load()
         cfg = Config()
         cfg.abi_version = ABI_VERSION
@@ -181,6 +182,7 @@ class Engine:
         cfg.launch_threads = launch_threads
         cfg.no_proxy = 0 if proxy else 1
         cfg.no_pdl = 0 if pdl else 1
+        cfg.prio_classes = prio_classes
         self.cfg = cfg
         h = C.c_void_p()
         _check(self.lib.paella_init(C.byref(cfg), C.byref(h)), "paella_init")

@@ -204,6 +204,7 @@ struct CudaBackend : Backend {
   // forwards to the host ring, so no kernel pays the PCIe write on its exit path
   bool proxy = false;
   bool pdl = true;             // programmatic dependent launches (off for the naive baseline)
+  uint32_t prio_classes = 1;   // stream-priority classes (set before init)
   Rec* dev_ring = nullptr;
   uint32_t* proxy_ctl = nullptr;     // pinned mapped: [0] stop flag, [16] heartbeat
   cudaStream_t proxy_stream = nullptr;
@@ -260,8 +261,18 @@ struct CudaBackend : Backend {
     if (cudaMalloc(&tail, 256) != cudaSuccess) return -ENOMEM;
     if (cudaMalloc(&ctr, 2 * NCTR * sizeof(uint32_t)) != cudaSuccess) return -ENOMEM;
     streams.resize(nstreams);
-    for (auto& s : streams)
-      if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess) return -EIO;
+    // stream-priority classes: class c of Policy::stream_class -> hardware priority
+    // greatest + c (clamped to the device's range; class 0 = highest)
+    int least = 0, greatest = 0;
+    cudaDeviceGetStreamPriorityRange(&least, &greatest);
+    for (uint32_t i = 0; i < nstreams; ++i) {
+      int prio = 0;
+      if (prio_classes > 1) {
+        prio = greatest + (int)Policy::stream_class(i, prio_classes, nstreams);
+        if (prio > least) prio = least;
+      }
+      if (cudaStreamCreateWithPriority(&streams[i], cudaStreamNonBlocking, prio) != cudaSuccess) return -EIO;
+    }
     cudaMemsetAsync(tail, 0, 256, streams[0]);
     cudaMemsetAsync(ctr, 0, 2 * NCTR * sizeof(uint32_t), streams[0]);
     KernelFn tc_i[2], tc_p[2];
@@ -708,6 +719,8 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
   if (cfg.fake_time_scale_ns == 0) cfg.fake_time_scale_ns = 500;
   if (cfg.fairness_threshold < 0) return -EINVAL;
   if (cfg.lookahead > 4) return -EINVAL;
+  if (cfg.prio_classes == 0) cfg.prio_classes = 1;
+  if (cfg.prio_classes > cfg.stream_pool && cfg.stream_pool != 0) return -EINVAL;
   if (cfg.launch_threads > 16) return -EINVAL;
 
   auto P = std::make_unique<Paella>();
@@ -762,8 +775,11 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     if (cfg.device == PAELLA_DEVICE_CUDA)
       g->be.reset(new CudaBackend(g->device, g->cap, cfg.stream_pool,
                                   cfg.no_proxy == 0 && !std::getenv("PAELLA_NO_PROXY")));
-    if (cfg.device == PAELLA_DEVICE_CUDA)
-      static_cast<CudaBackend*>(g->be.get())->pdl = !cfg.naive && !cfg.no_pdl && !std::getenv("PAELLA_NO_PDL");
+    if (cfg.device == PAELLA_DEVICE_CUDA) {
+      auto* cb = static_cast<CudaBackend*>(g->be.get());
+      cb->pdl = !cfg.naive && !cfg.no_pdl && !std::getenv("PAELLA_NO_PDL");
+      cb->prio_classes = cfg.naive ? 1 : cfg.prio_classes;
+    }
     else
       g->be.reset(new FakeBackend(P->sms, g->cap, g->log2cap, cfg.group_size, cfg.stream_pool,
                                   cfg.fake_time_scale_ns));
@@ -778,6 +794,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     pc.ring_capacity = cfg.ring_capacity;
     pc.streams = cfg.stream_pool;
     pc.lookahead = cfg.lookahead;
+    pc.prio_classes = cfg.naive ? 1 : cfg.prio_classes;
     for (int r = 0; r < NRES; ++r) pc.capacity[r] = P->capacity[r];
     if (cfg.device == PAELLA_DEVICE_CUDA && static_cast<CudaBackend*>(g->be.get())->proxy) {
       // the resident proxy warp: 1 block, 1 warp, <= 64 regs/thread, the 1 KB reservation
@@ -802,7 +819,8 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
       setvbuf(g->log, nullptr, _IOFBF, 1 << 20);
       logev(g.get(), EV_CONFIG, cfg.num_clients, cfg.policy, (uint64_t)cfg.fairness_threshold,
             ((uint64_t)P->cfg.slack_blocks << 32) | cfg.group_size);
-      logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFFu, cfg.ring_capacity, cfg.stream_pool, cfg.lookahead);
+      logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFFu, cfg.ring_capacity, cfg.stream_pool,
+            ((uint64_t)pc.prio_classes << 32) | cfg.lookahead);
       for (int r = 0; r < NRES; ++r) logev(g.get(), EV_CAPACITY, (uint32_t)r, (uint64_t)pc.capacity[r], 0, 0);
     }
     P->gpus.push_back(std::move(g));

@@ -1,6 +1,7 @@
 // See policy.h.  Rule-for-rule the state machine of SURVEY.md §8(c) C2.
 #include "policy.h"
 
+#include <algorithm>
 #include <cassert>
 #include <climits>
 #include <stdexcept>
@@ -20,6 +21,28 @@ Policy::Policy(const Cfg& c) : cfg_(c) {
 void Policy::add_model(uint32_t mid, const std::vector<PolicyLayer>& layers) {
   if (mid >= kMaxModels) throw std::runtime_error("too many models");
   models_[mid] = layers;
+  int64_t t = 0;
+  for (const auto& l : layers) t += l.tbar;
+  if (!layers.empty()) {
+    auto it = std::lower_bound(totals_.begin(), totals_.end(), t);
+    if (it == totals_.end() || *it != t) totals_.insert(it, t);
+  }
+}
+
+// Stream-priority classes (B200 adaptation, reading B200-Q2; identical to
+// oracle/sim.py Policy.job_class): the number of registered models whose whole-job
+// T-bar sum is strictly below R_j, clamped to K-1; a deficit-override pick -> 0.
+uint32_t Policy::job_class(const PolicyJob& j) const {
+  const uint32_t K = cfg_.prio_classes;
+  if (K <= 1 || over_) return 0;
+  uint32_t c = (uint32_t)(std::lower_bound(totals_.begin(), totals_.end(), j.R) - totals_.begin());
+  return c < K - 1 ? c : K - 1;
+}
+
+int Policy::lowest_free_in_class(uint32_t c) const {
+  for (uint32_t s = 0; s < cfg_.streams; ++s)
+    if ((free_[s / 64] >> (s % 64) & 1) && stream_class(s, cfg_.prio_classes, cfg_.streams) == c) return (int)s;
+  return -1;
 }
 
 bool Policy::is_ready(const PolicyJob& j) const {
@@ -121,6 +144,7 @@ int Policy::lowest_free() const {
 }
 
 bool Policy::pick(uint32_t* job_id) {
+  over_ = false;
   if (srpt_.empty()) return false;
   if (cfg_.policy == POL_FIFO) {
     *job_id = fifo_.begin()->second;
@@ -143,6 +167,7 @@ bool Policy::pick(uint32_t* job_id) {
     if (cfg_.theta <= INT64_MAX / (int64_t)cfg_.num_clients)
       over = best > cfg_.theta * (int64_t)cfg_.num_clients;
   }
+  over_ = over;
   if (over) {
     *job_id = per_client_[cstar].begin()->second;   // oldest ready job of c*
   } else {
@@ -185,9 +210,15 @@ void Policy::decide(std::vector<Issue>* out) {
     if (j.inflight() > 0) {
       stream = (uint32_t)j.stream;   // launch-ahead: queued behind its predecessor
     } else {
-      stream = (uint32_t)s0;
-      if (j.last_stream >= 0 && (free_[j.last_stream / 64] >> (j.last_stream % 64) & 1))
+      const uint32_t c = job_class(j);
+      const uint32_t K = cfg_.prio_classes, P = cfg_.streams;
+      if (j.last_stream >= 0 && (free_[j.last_stream / 64] >> (j.last_stream % 64) & 1) &&
+          stream_class((uint32_t)j.last_stream, K, P) == c) {
         stream = (uint32_t)j.last_stream;
+      } else {
+        int sc = lowest_free_in_class(c);
+        stream = sc >= 0 ? (uint32_t)sc : (uint32_t)s0;
+      }
       free_[stream / 64] &= ~(1ull << (stream % 64));
       j.stream = (int32_t)stream;
     }

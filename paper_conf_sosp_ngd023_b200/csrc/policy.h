@@ -70,7 +70,10 @@ class Policy {
     uint32_t streams = 32;
     int64_t capacity[NRES] = {148 * 32, 148 * 64, 148 * 65536, 148 * 233472, 148 * 512};
     uint32_t lookahead = 0;   // NEXT-1 launch-ahead depth (0 = the paper's semantics)
+    uint32_t prio_classes = 1;   // stream-priority classes (1 = the paper: one class)
   };
+  // class of stream s: consecutive index ranges, class 0 = highest hardware priority
+  static uint32_t stream_class(uint32_t s, uint32_t K, uint32_t P) { return (uint32_t)((uint64_t)s * K / P); }
 
   explicit Policy(const Cfg& c);
 
@@ -99,6 +102,8 @@ class Policy {
   static constexpr uint32_t kLaunchSlots = 8192;
   static constexpr uint32_t kMaxModels = 256;
   bool pick(uint32_t* job_id);
+  uint32_t job_class(const PolicyJob& j) const;
+  int lowest_free_in_class(uint32_t c) const;
   bool predicate(uint32_t grid) const;
   void make_ready(PolicyJob& j);
   void make_unready(PolicyJob& j);
@@ -113,6 +118,8 @@ class Policy {
   int64_t U_[NRES] = {0, 0, 0, 0, 0};
   int64_t Q_ = 0, O_ = 0;
   int last_stop_ = 0;
+  bool over_ = false;                  // the last pick was a deficit override
+  std::vector<int64_t> totals_;        // sorted distinct whole-job T-bar sums of the models
   std::vector<uint64_t> free_;   // bitmap of free streams
   std::vector<int64_t> Dt_;
   int64_t Omega_ = 0;

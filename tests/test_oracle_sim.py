@@ -352,3 +352,32 @@ def test_S5_deficit_rule_and_bound(N, theta):
             series[c].append(pol.D(c))
     assert sim.deficit_bound_holds(series, N, theta) == []
     assert max(max(s) for s in series.values()) <= max(0, theta * N) + N
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_prio_classes_stream_rule(seed):
+    """Stream-priority classes (reading B200-Q2): with enough streams and no
+    deficit override, every fresh stream acquisition lands in the class given by the
+    rank of R_j (remaining T-bar before the kernel) among the models' whole-job sums;
+    K = 1 reproduces the one-class issue sequence exactly."""
+    r = random.Random(300 + seed)
+    models = random_models(r)
+    gpu = GPUModel(sms=8, per_sm=(32, 64, 65536, 233472, 512), launch_delay=500, notif_delay=700)
+    base = dict(num_clients=3, theta=sim.INF_THETA, slack=8, group=4, ring_capacity=4096, streams=32,
+                capacity=tuple(8 * x for x in (32, 64, 65536, 233472, 512)), lookahead=0)
+    trace = random_trace(r, 60, 3, len(models), rate_ns=20000)
+    one = sim.simulate(Config(**base), models, trace, gpu)
+    one_k1 = sim.simulate(Config(**base, prio_classes=1), models, trace, gpu)
+    assert one.issues == one_k1.issues
+    K = 3
+    res = sim.simulate(Config(**base, prio_classes=K), models, trace, gpu)
+    assert len(res.finish) == len(trace)
+    totals = sorted({sum(l.tbar for l in m) for m in models})
+    checked = 0
+    for (t, uid, jid, layer, stream) in res.issues:
+        ls = models[trace[jid][2]]
+        R = sum(l.tbar for l in ls[layer:])
+        want = min(K - 1, sum(1 for x in totals if x < R))
+        assert stream * K // 32 == want, (jid, layer, stream, R, totals)
+        checked += 1
+    assert checked == len(res.issues) > 0
