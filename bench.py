@@ -52,6 +52,10 @@ def parse():
     ap.add_argument("--reqs", type=int, default=2000, help="requests per step")
     ap.add_argument("--no-baselines", action="store_true")
     ap.add_argument("--lookahead", type=int, default=1, help="NEXT-1 launch-ahead depth of the Paella arm")
+    ap.add_argument("--slack", type=int, default=1184,
+                    help="B, blocks issued beyond full utilisation (P1300-1304); 8 x 148 SMs covers the "
+                         "measured dispatch loop delay (DESIGN.md B200-Q1)")
+    ap.add_argument("--prio-classes", type=int, default=4, help="stream-priority classes (DESIGN.md B200-Q2)")
     ap.add_argument("--launch-threads", type=int, default=4, help="launcher helper threads per GPU")
     ap.add_argument("--sat-reqs", type=int, default=1500, help="requests of the saturation calibration")
     ap.add_argument("--fake", action="store_true",
@@ -222,6 +226,9 @@ def run_gpu(args, dist):
 
     def engine(**kw):
         kw.setdefault("launch_threads", 0 if args.fake else args.launch_threads)
+        if not kw.get("naive"):
+            kw.setdefault("slack", args.slack)
+            kw.setdefault("prio_classes", args.prio_classes)
         e, mids = build_engine(L, specs, gpu, fake=args.fake, region_bytes=region, max_jobs_per_model=128, **kw)
         stage_inputs(e, specs, mids, slots, stride, pool)
         return e, mids
@@ -308,7 +315,7 @@ def run_gpu(args, dist):
     base = {}
     if not args.no_baselines:
         for label, kw in (("naive_cuda_ms", dict(naive=True, instrument=False)),
-                          ("paella_paper_lookahead0", dict(lookahead=0)),
+                          ("paella_paper_lookahead0", dict(lookahead=0, slack=0, prio_classes=1, pdl=False)),
                           ("paella_fifo", dict(policy=L.POLICY_FIFO, lookahead=args.lookahead))):
             eb, mb = engine(**kw)
             jl = []
@@ -445,6 +452,7 @@ def main():
                          "as in serving; inputs stream from pinned host memory"},
         "jct_us": res["jct"], "slo_us": res["slo"],
         "paella_config": {"lookahead": args.lookahead, "launch_threads": args.launch_threads, "policy": "srpt+deficit",
+                          "slack_blocks": args.slack, "prio_classes": args.prio_classes, "pdl": True,
                           "theta": 100, "group": 16, "streams": 32},
         "slo_met": bool(all(res["jct"].get(n, {}).get("p99_us", 1e18) <= res["slo"][n] for n in res["names"])),
         "x_sat_req_s": {"naive": round(res["x_sat_naive"], 1), "paella": round(res["x_sat_paella"], 1)},
