@@ -65,11 +65,25 @@ __device__ __forceinline__ void instr_enter(const InstrArgs& ia) {
       maybe_record(ia, REC_PLACEMENT, c, total);
     }
   }
-  // programmatic dependent launch: wait until the kernel this one was queued behind
-  // has completed and its memory is visible (a no-op for plain launches).  No kernel
-  // triggers its dependents early, so blocks are placed (and report PLACEMENT) only
-  // once the predecessor has finished, as without PDL.
-  asm volatile("griddepcontrol.wait;" ::: "memory");
+}
+
+// Programmatic dependent launch.  pdl_wait: block until the kernel this
+// one was queued behind on its stream has completed and its memory is visible (a no-op
+// for plain launches); every read of a predecessor's output and every output store
+// comes after it.  pdl_trigger: this block no longer needs anything that a dependent's
+// early start could disturb, so the dependent grid may be placed (its blocks run
+// their independent prologue -- barrier init, TMEM allocation, weight prefetch -- and
+// then pdl_wait).  Placement is still reported when blocks really start.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
+// SIMT kernels: bookkeeping, wait for the predecessor, then let the successor be
+// placed right away (these kernels are short; the successor's prologue overlaps them)
+template <bool INSTR>
+__device__ __forceinline__ void kernel_begin(const InstrArgs& ia) {
+  instr_enter<INSTR>(ia);
+  pdl_wait();
+  pdl_trigger();
 }
 
 template <bool INSTR, uint32_t T = 0>

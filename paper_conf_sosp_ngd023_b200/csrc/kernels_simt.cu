@@ -58,7 +58,7 @@ __device__ __forceinline__ float act_f(float x, uint32_t act) {
 template <typename T, bool INSTR>
 __global__ void __launch_bounds__(256) k_ingest(const __grid_constant__ LayerArgs a,
                                                 const __grid_constant__ InstrArgs ia) {
-  instr_enter<INSTR>(ia);
+  kernel_begin<INSTR>(ia);
   const float* in = static_cast<const float*>(a.in);
   T* out = static_cast<T*>(a.out);
   uint32_t hw = a.h * a.w_;
@@ -84,7 +84,7 @@ __global__ void __launch_bounds__(256) k_ingest(const __grid_constant__ LayerArg
 template <typename T, bool INSTR>
 __global__ void __launch_bounds__(256) k_conv_simt(const __grid_constant__ LayerArgs a,
                                                    const __grid_constant__ InstrArgs ia) {
-  instr_enter<INSTR>(ia);
+  kernel_begin<INSTR>(ia);
   constexpr int BM = 64, BN = 64, BK = 32;
   __shared__ float As[BK][BM + 4];
   __shared__ float Bs[BK][BN + 4];
@@ -216,7 +216,7 @@ __device__ __forceinline__ void dw_taps(const LayerArgs& a, const T* X, const T*
 template <typename T, bool INSTR>
 __global__ void __launch_bounds__(256) k_dwconv(const __grid_constant__ LayerArgs a,
                                                 const __grid_constant__ InstrArgs ia) {
-  instr_enter<INSTR>(ia);
+  kernel_begin<INSTR>(ia);
   const T* X = static_cast<const T*>(a.in);
   const T* W = static_cast<const T*>(a.w);
   T* Y = static_cast<T*>(a.out);
@@ -288,7 +288,7 @@ __device__ __forceinline__ void pool_taps(const LayerArgs& a, const T* X, int oh
 template <typename T, bool INSTR, bool MAX>
 __global__ void __launch_bounds__(256) k_pool(const __grid_constant__ LayerArgs a,
                                               const __grid_constant__ InstrArgs ia) {
-  instr_enter<INSTR>(ia);
+  kernel_begin<INSTR>(ia);
   const T* X = static_cast<const T*>(a.in);
   T* Y = static_cast<T*>(a.out);
   uint32_t ng = a.cout / 8;
@@ -337,7 +337,7 @@ __global__ void __launch_bounds__(256) k_pool(const __grid_constant__ LayerArgs 
 template <typename T, bool INSTR>
 __global__ void __launch_bounds__(256) k_gap(const __grid_constant__ LayerArgs a,
                                              const __grid_constant__ InstrArgs ia) {
-  instr_enter<INSTR>(ia);
+  kernel_begin<INSTR>(ia);
   const T* X = static_cast<const T*>(a.in);
   uint32_t ng = a.cout / 8;
   uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
@@ -393,7 +393,7 @@ __global__ void __launch_bounds__(256) k_gap(const __grid_constant__ LayerArgs a
 template <typename T, bool INSTR>
 __global__ void __launch_bounds__(256) k_fc(const __grid_constant__ LayerArgs a,
                                             const __grid_constant__ InstrArgs ia) {
-  instr_enter<INSTR>(ia);
+  kernel_begin<INSTR>(ia);
   const T* X = static_cast<const T*>(a.in);
   const T* W = static_cast<const T*>(a.w);
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
@@ -433,7 +433,7 @@ __global__ void __launch_bounds__(256) k_fc(const __grid_constant__ LayerArgs a,
 template <typename T, bool INSTR>
 __global__ void __launch_bounds__(256) k_gapfc(const __grid_constant__ LayerArgs a,
                                                const __grid_constant__ InstrArgs ia) {
-  instr_enter<INSTR>(ia);
+  kernel_begin<INSTR>(ia);
   extern __shared__ float pooled[];   // [C]
   const T* X = static_cast<const T*>(a.in);
   const T* W = static_cast<const T*>(a.w);
@@ -508,7 +508,7 @@ __global__ void __launch_bounds__(256) k_gapfc(const __grid_constant__ LayerArgs
 // ---------------------------------------------------------------------------
 template <bool INSTR>
 __global__ void k_empty(const __grid_constant__ LayerArgs a, const __grid_constant__ InstrArgs ia) {
-  instr_enter<INSTR>(ia);
+  kernel_begin<INSTR>(ia);
   instr_exit<INSTR>(ia);
 }
 

@@ -166,8 +166,10 @@ __device__ __forceinline__ uint4 load_res8(const LayerArgs& a, uint32_t p, uint3
                                               a.res_co + co));
 }
 
-// 2 CTAs per SM (two jobs' convs can share an SM): <= 168 registers, since a
-// 160-thread CTA puts 2 of its 5 warps on one sub-partition (16K registers each)
+// 2 CTAs per SM (two jobs' convs can share an SM): <= 168 registers.  Warp 5 does
+// only the block bookkeeping (instrumentation), so no compute warp waits on its
+// atomics at entry.
+constexpr uint32_t TBOOK = NPROD + 32;   // warp 5, lane 0
 template <bool INSTR, bool PRO>
 __global__ void __launch_bounds__(TC_THREADS, 2)
     k_conv_tc(const __grid_constant__ LayerArgs a, const __grid_constant__ InstrArgs ia,
@@ -177,9 +179,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
                              16 * ((blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x)
                        : nullptr;
   if (trace && threadIdx.x == 0) tr[0] = globaltimer();
-  // the instrumentation runs on an otherwise idle lane of the MMA warp, so neither
-  // the TMA issuer nor the gather warps wait on its atomics (instr.cuh)
-  instr_enter<INSTR, NPROD + 1>(ia);
+  instr_enter<INSTR, TBOOK>(ia);
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   uint8_t* sA = smem;                                  // STAGES x 16 KiB
@@ -298,7 +298,9 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       ks_ = rs % (int)a.kw;
       kr = rs / (int)a.kw;
     }
-    // ... and the first activation gathers, before the CTA-wide barrier
+    // ... and the first activation gathers, before the CTA-wide barrier, once the
+    // predecessor kernel's output is complete (PDL; the weight TMA above needs no wait)
+    pdl_wait();
     for (uint32_t it = 0; it < pre; ++it) issue_B(it, false);   // barriers not initialised yet
     if (trace && t == 0) tr[13] = globaltimer();
   }
@@ -336,7 +338,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
         }
       }
     }
-  } else {
+  } else if (warp == 4) {
     // ------------------------------------------------------------ MMA warp
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(su32(tmem_slot)),
                  "r"(64u)
@@ -388,6 +390,10 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       }
     }
   }
+  // every input of this block has been consumed: let the dependent kernel be placed
+  // (its prologue overlaps this epilogue); warp 5 follows the accumulator too
+  if (warp == 5 && nkl > 0) mbar_wait(accb, 0);
+  pdl_trigger();
   if (warp < 4) {
     const uint32_t row = warp * 32 + lane;
     if (nkl > 0) {
@@ -492,8 +498,8 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tmem_slot), "r"(64u) : "memory");
   }
   if (trace && threadIdx.x == 0) tr[6] = globaltimer();
-  instr_exit<INSTR, NPROD + 1>(ia);
-  if (trace && threadIdx.x == NPROD + 1) tr[7] = globaltimer();
+  instr_exit<INSTR, TBOOK>(ia);
+  if (trace && threadIdx.x == TBOOK) tr[7] = globaltimer();
 }
 
 uint32_t tc_smem_bytes() { return 1024 + TC_STAGES * (A_BYTES + B_BYTES) + 128; }
