@@ -46,6 +46,8 @@ extern "C" {
 #endif
 
 #define PAELLA_ABI_VERSION 1u
+#define PAELLA_NOTIFY_COUNTERS 0u
+#define PAELLA_NOTIFY_RING     1u
 
 /* policies (P1222-1323 §6; FIFO = the Paella-SS-like ablation of Table 3, P1349) */
 #define PAELLA_POLICY_SRPT_DEFICIT 0u
@@ -103,9 +105,10 @@ typedef struct {
                                     the durations (paella_stats ev_*): the live roofline */
   uint32_t lookahead;            /* NEXT-1 launch-ahead depth: 0 = the paper's semantics (a
                                     job's next kernel is dispatched after the previous one's
-                                    final COMPLETION); D > 0 = once the previous kernel is
-                                    fully placed and <= D are in flight, the next kernel is
-                                    queued behind it on the same stream */
+                                    final COMPLETION); D in 1..4 = once the job's OLDEST
+                                    in-flight kernel is fully placed (running) and <= D are in
+                                    flight, the next kernel is queued behind it on the same
+                                    stream (with PDL it starts ~0.6 us after its predecessor) */
   uint32_t launch_threads;       /* 0 = each dispatcher calls cudaLaunchKernel itself; n > 0 =
                                     n helper threads per GPU perform the launches (stream s is
                                     owned by helper s % n, so per-stream order is kept); the
@@ -120,6 +123,17 @@ typedef struct {
                                     stream starts ~0.6 us after it instead of on the next
                                     ~2 us front-end quantum); 1: plain launches.
                                     The naive baseline always uses plain launches. */
+  uint32_t notify_mode;          /* PAELLA_NOTIFY_COUNTERS (0, default): blocks only bump their
+                                    launch's {start, end} counters with fire-and-forget
+                                    reductions; one resident warp mirrors the counter table to
+                                    pinned host memory and the dispatcher turns counter
+                                    progress into the same group-of-G records (no atomic
+                                    round trip and no record write on any block's exit path,
+                                    DESIGN.md §7).  PAELLA_NOTIFY_RING (1): blocks write 16 B
+                                    records into a device ring that a resident warp forwards
+                                    to the pinned host ring (records carry SM id and
+                                    globaltimer; G = 1 debug mode).  no_proxy = 1 overrides
+                                    both with the paper's direct ring writes. */
   uint32_t prio_classes;         /* 0/1 = one class (the paper).  K > 1: the stream pool is split
                                     into K classes of consecutive indices created with
                                     descending hardware stream priority; a job takes a stream

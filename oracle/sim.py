@@ -73,6 +73,7 @@ class Job:
     stream: int = -1         # stream held while kernels are in flight
     last_stream: int = -1
     last_uid: int = -1
+    uids: dict = field(default_factory=dict)   # layer -> launch uid (while in flight)
 
     @property
     def inflight(self):
@@ -95,9 +96,9 @@ class Policy:
     """The dispatcher state machine of SURVEY.md §8(c) C2, integer-exact.
 
     Launch-ahead (NEXT-1; off by default): with lookahead = D > 0 a
-    job whose most recent kernel is fully placed (p_eff = grid) and that has at most
-    D kernels in flight may issue its next kernel onto the SAME stream (stream order
-    carries the dependency, P947-951); the paper's semantics is D = 0."""
+    job whose OLDEST in-flight kernel is fully placed (p_eff = grid, i.e. running) and
+    that has at most D kernels in flight may issue its next kernel onto the SAME stream
+    (stream order carries the dependency, P947-951); the paper's semantics is D = 0."""
 
     def __init__(self, cfg: Config, models: list[list[Layer]]):
         self.cfg = cfg
@@ -183,7 +184,7 @@ class Policy:
             return True
         if self.cfg.lookahead <= 0 or j.inflight > self.cfg.lookahead:
             return False
-        L = self.launches.get(j.last_uid)
+        L = self.launches.get(j.uids.get(j.done))     # the oldest kernel still in flight
         return L is not None and max(L.p, L.f) >= L.grid
 
     def ready(self):
@@ -259,6 +260,7 @@ class Policy:
             self.O += 2 * groups(layer.grid, cfg.group)
             j.R -= layer.tbar
             rec = (uid, j.id, j.cursor, stream)
+            j.uids[j.cursor] = uid
             j.cursor += 1
             j.last_uid = uid
             if self.checks:

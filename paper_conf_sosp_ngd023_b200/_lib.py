@@ -17,6 +17,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "libpaella.so")
 
 ABI_VERSION = 1
+NOTIFY_COUNTERS, NOTIFY_RING = 0, 1
 POLICY_SRPT_DEFICIT, POLICY_FIFO = 0, 1
 ROUTE_LEAST_WORK, ROUTE_ROUND_ROBIN = 0, 1
 DEVICE_CUDA, DEVICE_FAKE = 0, 1
@@ -46,7 +47,7 @@ class Config(C.Structure):
                 ("fake_sms", C.c_uint32), ("fake_time_scale_ns", C.c_uint32), ("event_time_kind", C.c_uint32),
                 ("lookahead", C.c_uint32), ("launch_threads", C.c_uint32),
                 ("no_proxy", C.c_uint32), ("no_pdl", C.c_uint32),
-                ("prio_classes", C.c_uint32)]
+                ("notify_mode", C.c_uint32), ("prio_classes", C.c_uint32)]
 
 
 class Node(C.Structure):
@@ -149,7 +150,8 @@ class Engine:
                  streams=32, route=ROUTE_LEAST_WORK, submit_slots=1024, max_jobs_per_model=128,
                  instrument=True, naive=False, region_bytes=64 << 20, dispatcher_cpus=None,
                  event_log=None, fake_sms=0, fake_time_scale_ns=0, event_time_kind=None, lookahead=0,
-                 launch_threads=0, proxy=True, pdl=True, prio_classes=1):
+                 launch_threads=0, proxy=True, pdl=True, prio_classes=1,
+                 notify="counters"):
         self.lib = load()
         cfg = Config()
         cfg.abi_version = ABI_VERSION
@@ -183,6 +185,13 @@ class Engine:
         cfg.no_proxy = 0 if proxy else 1
         cfg.no_pdl = 0 if pdl else 1
         cfg.prio_classes = prio_classes
+        # notification path: "counters" (default), "ring" (device ring + forwarding warp),
+        # "direct" (the paper's direct ring writes; same as proxy=False)
+        if notify not in ("counters", "ring", "direct"):
+            raise ValueError(notify)
+        cfg.notify_mode = NOTIFY_RING if notify == "ring" else NOTIFY_COUNTERS
+        if notify == "direct":
+            cfg.no_proxy = 1
         self.cfg = cfg
         h = C.c_void_p()
         _check(self.lib.paella_init(C.byref(cfg), C.byref(h)), "paella_init")

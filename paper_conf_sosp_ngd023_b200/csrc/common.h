@@ -59,7 +59,11 @@ PAELLA_HD inline RecFields rec_decode(uint64_t w0, uint64_t w1) {
 
 // Per-launch instrumentation arguments (Fig. 6's extra parameters notifQ, kernId,
 // P887-895, plus the per-launch counter slot -- reading C2-Q1).
-enum : uint32_t { INSTR_ON = 1u, INSTR_LAST = 2u };
+// INSTR_CTR (counter mode): the block only bumps its launch's {start,
+// end} counters with fire-and-forget reductions and writes no record; the mirror warp
+// (k_notify_mirror) copies the counters to pinned host memory and the dispatcher turns
+// counter progress into the same group-of-G records (engine.cpp::drain_counters)
+enum : uint32_t { INSTR_ON = 1u, INSTR_LAST = 2u, INSTR_CTR = 4u };
 
 struct InstrArgs {
   Rec* ring;          // device-visible pointer to the pinned, mapped ring
@@ -74,6 +78,7 @@ struct InstrArgs {
 };
 
 constexpr uint32_t NCTR = 4096;   // counter slots; > max in-flight launches (<= P)
+constexpr uint32_t NCTR_M = 256;  // counter-mode slots (free list; > P x (lookahead + 1))
 
 // Kernel-side arguments of one layer.  Activations are NHWC with an explicit
 // channel stride/offset so that a concat is just producers writing into disjoint

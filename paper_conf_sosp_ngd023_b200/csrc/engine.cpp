@@ -203,6 +203,10 @@ struct CudaBackend : Backend {
   // notification proxy: kernels write to dev_ring (device memory); one persistent warp
   // forwards to the host ring, so no kernel pays the PCIe write on its exit path
   bool proxy = false;
+  bool mirror = false;         // counter mode: kernels only count, k_notify_mirror copies
+  uint32_t* ctr_m = nullptr;   // device: NCTR_M x {start, end}
+  uint32_t* mirror_h = nullptr;   // pinned, mapped host copy
+  uint32_t* mirror_d = nullptr;
   bool pdl = true;             // programmatic dependent launches (off for the naive baseline)
   uint32_t prio_classes = 1;   // stream-priority classes (set before init)
   Rec* dev_ring = nullptr;
@@ -213,22 +217,35 @@ struct CudaBackend : Backend {
   std::vector<cudaStream_t> streams;
   KernelFn tab[2][2][KIND_COUNT];   // [dtype][instr][kind]
   int err_ = 0;
-  CudaBackend(int d, uint32_t c, uint32_t P, bool px) : dev(d), cap(c), nstreams(P), proxy(px) {}
+  CudaBackend(int d, uint32_t c, uint32_t P, bool px, bool mir)
+      : dev(d), cap(c), nstreams(P), proxy(px && !mir), mirror(mir) {}
   bool proxy_running = false;
   uint32_t* ctl_d = nullptr;
   int setup_proxy(cudaStream_t s) {
-    if (cudaMalloc(&dev_ring, (size_t)cap * sizeof(Rec)) != cudaSuccess) return -ENOMEM;
-    cudaMemsetAsync(dev_ring, 0, (size_t)cap * sizeof(Rec), s);
+    if (mirror) {
+      if (cudaMalloc(&ctr_m, 2 * NCTR_M * sizeof(uint32_t)) != cudaSuccess) return -ENOMEM;
+      cudaMemsetAsync(ctr_m, 0, 2 * NCTR_M * sizeof(uint32_t), s);
+      if (cudaHostAlloc((void**)&mirror_h, 2 * NCTR_M * sizeof(uint32_t), cudaHostAllocMapped | cudaHostAllocPortable) !=
+          cudaSuccess)
+        return -ENOMEM;
+      std::memset(mirror_h, 0, 2 * NCTR_M * sizeof(uint32_t));
+      cudaHostGetDevicePointer((void**)&mirror_d, mirror_h, 0);
+    } else {
+      if (cudaMalloc(&dev_ring, (size_t)cap * sizeof(Rec)) != cudaSuccess) return -ENOMEM;
+      cudaMemsetAsync(dev_ring, 0, (size_t)cap * sizeof(Rec), s);
+    }
     if (cudaHostAlloc((void**)&proxy_ctl, 256, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
       return -ENOMEM;
     std::memset(proxy_ctl, 0, 256);
     cudaHostGetDevicePointer((void**)&ctl_d, proxy_ctl, 0);
-    if (cudaStreamCreateWithFlags(&proxy_stream, cudaStreamNonBlocking) != cudaSuccess) return -EIO;
+    int least = 0, greatest = 0;   // the forwarding warp outranks every pool stream
+    cudaDeviceGetStreamPriorityRange(&least, &greatest);
+    if (cudaStreamCreateWithPriority(&proxy_stream, cudaStreamNonBlocking, greatest) != cudaSuccess) return -EIO;
     return 0;
   }
   // dispatcher thread: (re)start the forwarding warp when records may be outstanding
   void ensure_proxy() {
-    if (!proxy) return;
+    if (!proxy && !mirror) return;
     if (proxy_running) {
       if (__atomic_load_n(&proxy_ctl[32], __ATOMIC_ACQUIRE) == 0) return;
       proxy_running = false;   // it left after an idle spell
@@ -240,7 +257,11 @@ struct CudaBackend : Backend {
     while ((1u << l2) < cap) ++l2;
     volatile uint32_t* st = ctl_d;
     void* args[5] = {(void*)&src, (void*)&dst, (void*)&mask, (void*)&l2, (void*)&st};
-    if (cudaLaunchKernel((const void*)proxy_kernel(), dim3(1), dim3(32), args, 0, proxy_stream) == cudaSuccess)
+    const uint4* mc = (const uint4*)ctr_m;
+    uint4* mh = (uint4*)mirror_d;
+    void* margs[3] = {(void*)&mc, (void*)&mh, (void*)&st};
+    if (cudaLaunchKernel(mirror ? (const void*)mirror_kernel() : (const void*)proxy_kernel(), dim3(1), dim3(32),
+                         mirror ? margs : args, 0, proxy_stream) == cudaSuccess)
       proxy_running = true;
     else if (!err_)
       err_ = (int)cudaErrorLaunchFailure;
@@ -283,7 +304,7 @@ struct CudaBackend : Backend {
     tab[0][1][KIND_CONV_TC_PRO] = tc_i[1];
     tab[0][0][KIND_CONV_TC_PRO] = tc_p[1];
     for (int i = 0; i < 2; ++i) tab[1][i][KIND_CONV_TC] = tab[1][i][KIND_CONV_TC_PRO] = nullptr;
-    if (proxy) {
+    if (proxy || mirror) {
       int rc = setup_proxy(streams[0]);
       if (rc) return rc;
     }
@@ -295,6 +316,8 @@ struct CudaBackend : Backend {
     stop_proxy();
     if (proxy_stream) cudaStreamDestroy(proxy_stream);
     if (dev_ring) cudaFree(dev_ring);
+    if (ctr_m) cudaFree(ctr_m);
+    if (mirror_h) cudaFreeHost(mirror_h);
     if (proxy_ctl) cudaFreeHost(proxy_ctl);
     for (auto& s : streams) cudaStreamDestroy(s);
     if (ring_h) cudaFreeHost(ring_h);
@@ -342,19 +365,31 @@ int make_weight_tmap(void* weights, uint32_t rows, uint32_t kpad, void* out128);
 // ---------------------------------------------------------------------------
 // helpers
 // ---------------------------------------------------------------------------
-static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last) {
+static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last, bool instr) {
   InstrArgs ia;
   ia.ring = (Rec*)g->be->ring_dev();
   ia.tail = g->be->tail_dev();
-  uint32_t slot = uid % NCTR;
-  ia.ctr = g->be->ctr_dev() + 2 * slot;
   ia.mask = g->cap - 1;
   ia.log2cap = g->log2cap;
-  ia.base = g->ctr_base[slot];
-  g->ctr_base[slot] += grid;
   ia.uid = uid;
   ia.group = g->P->cfg.group_size;
   ia.flags = INSTR_ON | (last ? INSTR_LAST : 0);
+  if (g->ctr_mode && instr) {
+    // counter mode: a free slot of the mirrored counter table (> P x (lookahead + 1)
+    // slots, so one is always free); the slot returns when its last block has exited
+    uint32_t slot = g->ctr_free.back();
+    g->ctr_free.pop_back();
+    ia.ctr = static_cast<CudaBackend*>(g->be.get())->ctr_m + 2 * slot;
+    ia.base = g->ctr_mbase[slot];
+    g->ctr_mbase[slot] += grid;
+    ia.flags |= INSTR_CTR;
+    g->ctr_live.push_back(Gpu::CtrLive{uid, slot, ia.base, grid, 0, 0});
+    return ia;
+  }
+  uint32_t slot = uid % NCTR;
+  ia.ctr = g->be->ctr_dev() + 2 * slot;
+  ia.base = g->ctr_base[slot];
+  g->ctr_base[slot] += grid;
   return ia;
 }
 
@@ -388,7 +423,7 @@ static void launcher_main(Gpu* g, Launcher* L) {
 
 static void do_launch(Gpu* g, Model* m, uint32_t slot, uint32_t layer, uint32_t uid, uint32_t stream, bool instr) {
   const KernelInst& k = m->kernels[layer];
-  InstrArgs ia = make_instr(g, uid, k.grid_total(), layer + 1 == m->kernels.size());
+  InstrArgs ia = make_instr(g, uid, k.grid_total(), layer + 1 == m->kernels.size(), instr);
   const paella_config_t& cfg = g->P->cfg;
   if (!g->launchers.empty()) {
     LaunchDesc d;
@@ -557,6 +592,50 @@ static uint32_t drain_ring(Gpu* g) {
   return n;
 }
 
+// Counter mode: turn the progress of every in-flight launch's mirrored {start, end}
+// counters into the group-of-G records the ring would carry (group g of a launch
+// covers counts (gG, min((g+1)G, grid)] and is reported once all of them are in;
+// Fig. 6's aggregation, reading C2-Q2), in launch order, PLACEMENT before COMPLETION.
+static uint32_t drain_counters(Gpu* g) {
+  auto* cb = static_cast<CudaBackend*>(g->be.get());
+  const uint32_t G = g->P->cfg.group_size;
+  uint32_t n = 0;
+  for (size_t i = 0; i < g->ctr_live.size();) {
+    Gpu::CtrLive& L = g->ctr_live[i];
+    const uint64_t v = *reinterpret_cast<volatile uint64_t*>(cb->mirror_h + 2 * L.slot);
+    uint32_t cnt[2] = {(uint32_t)v - L.base, (uint32_t)(v >> 32) - L.base};
+    uint32_t* seen[2] = {&L.p, &L.f};
+    bool finished = false;
+    for (int t = 0; t < 2; ++t) {
+      const uint32_t now = cnt[t];
+      if (now > L.grid) continue;   // not yet published for this use of the slot
+      while (*seen[t] < now) {
+        const uint32_t grp = *seen[t] / G;
+        const uint32_t end = std::min((grp + 1) * G, L.grid);
+        if (now < end) break;       // group incomplete
+        const uint32_t cnt_g = end - grp * G;
+        const uint32_t type = t == 0 ? REC_PLACEMENT : REC_COMPLETION;
+        *seen[t] = end;
+        n++;
+        g->stats.records++;
+        logev(g, EV_RECORD, type, L.uid, cnt_g, ((uint64_t)grp << 40) | (0xFFull << 56));
+        int64_t done = -1;
+        g->policy->record(type, L.uid, cnt_g, &done);
+        if (done >= 0) finish_job(g, (uint32_t)done, 0);
+      }
+      if (t == 1 && L.f == L.grid) finished = true;
+    }
+    if (finished) {
+      g->ctr_free.push_back(L.slot);
+      g->ctr_live[i] = g->ctr_live.back();
+      g->ctr_live.pop_back();
+    } else {
+      ++i;
+    }
+  }
+  return n;
+}
+
 static void decide_and_launch(Gpu* g) {
   g->issues.clear();
   g->policy->decide(&g->issues);
@@ -652,7 +731,7 @@ static void dispatcher_main(Gpu* g) {
     // 2. notification ring (keep the forwarding warp alive while records are due)
     if (P->cfg.device == PAELLA_DEVICE_CUDA && g->policy->O() > 0 && (g->stats.loop_iters & 1023) == 0)
       static_cast<CudaBackend*>(g->be.get())->ensure_proxy();
-    nev += drain_ring(g);
+    nev += g->ctr_mode ? drain_counters(g) : drain_ring(g);
     // 3. decide (the batch boundary is logged for replay, C2-Q17)
     if (nev) {
       logev(g, EV_BATCH_END, 0, 0, 0, 0);
@@ -720,6 +799,11 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
   if (cfg.fairness_threshold < 0) return -EINVAL;
   if (cfg.lookahead > 4) return -EINVAL;
   if (cfg.prio_classes == 0) cfg.prio_classes = 1;
+  if (cfg.notify_mode > PAELLA_NOTIFY_RING) return -EINVAL;
+  // counter mode: in-flight launches (<= P x (lookahead + 1)) must fit the slot table
+  if (cfg.notify_mode == PAELLA_NOTIFY_COUNTERS &&
+      (uint64_t)(cfg.stream_pool ? cfg.stream_pool : 32) * (cfg.lookahead + 1) >= NCTR_M)
+    return -EINVAL;
   if (cfg.prio_classes > cfg.stream_pool && cfg.stream_pool != 0) return -EINVAL;
   if (cfg.launch_threads > 16) return -EINVAL;
 
@@ -774,11 +858,18 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     g->jobs.reserve(65536);
     if (cfg.device == PAELLA_DEVICE_CUDA)
       g->be.reset(new CudaBackend(g->device, g->cap, cfg.stream_pool,
-                                  cfg.no_proxy == 0 && !std::getenv("PAELLA_NO_PROXY")));
+                                  cfg.no_proxy == 0 && !std::getenv("PAELLA_NO_PROXY"),
+                                  cfg.no_proxy == 0 && cfg.notify_mode == PAELLA_NOTIFY_COUNTERS &&
+                                      !cfg.naive && !std::getenv("PAELLA_NO_PROXY")));
     if (cfg.device == PAELLA_DEVICE_CUDA) {
       auto* cb = static_cast<CudaBackend*>(g->be.get());
       cb->pdl = !cfg.naive && !cfg.no_pdl && !std::getenv("PAELLA_NO_PDL");
       cb->prio_classes = cfg.naive ? 1 : cfg.prio_classes;
+      if (cb->mirror) {
+        g->ctr_mode = true;
+        g->ctr_mbase.assign(NCTR_M, 0);
+        for (uint32_t sl = NCTR_M; sl-- > 0;) g->ctr_free.push_back(sl);
+      }
     }
     else
       g->be.reset(new FakeBackend(P->sms, g->cap, g->log2cap, cfg.group_size, cfg.stream_pool,
@@ -796,7 +887,8 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     pc.lookahead = cfg.lookahead;
     pc.prio_classes = cfg.naive ? 1 : cfg.prio_classes;
     for (int r = 0; r < NRES; ++r) pc.capacity[r] = P->capacity[r];
-    if (cfg.device == PAELLA_DEVICE_CUDA && static_cast<CudaBackend*>(g->be.get())->proxy) {
+    if (cfg.device == PAELLA_DEVICE_CUDA &&
+        (static_cast<CudaBackend*>(g->be.get())->proxy || static_cast<CudaBackend*>(g->be.get())->mirror)) {
       // the resident proxy warp: 1 block, 1 warp, <= 64 regs/thread, the 1 KB reservation
       const int64_t proxy[NRES] = {1, 1, 64 * 32, 1024, 0};
       for (int r = 0; r < NRES; ++r) pc.capacity[r] -= proxy[r];
@@ -1438,6 +1530,7 @@ static InstrArgs iso_instr(Gpu* g, uint32_t grid, uint32_t group, bool last) {
   ia.uid = uid;
   ia.group = group;
   ia.flags = INSTR_ON | (last ? INSTR_LAST : 0);
+  if (static_cast<CudaBackend*>(g->be.get())->mirror) ia.flags |= INSTR_CTR;   // as in serving
   return ia;
 }
 

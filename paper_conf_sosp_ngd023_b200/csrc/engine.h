@@ -158,6 +158,14 @@ struct Gpu {
   uint64_t head = 0;        // notification ring consumer index
   uint32_t cap = 0, log2cap = 0;
   std::vector<uint32_t> ctr_base;   // running base per counter slot
+  // counter-mode notification: launches in flight and their slots
+  struct CtrLive {
+    uint32_t uid, slot, base, grid, p, f;   // p, f: counts already turned into records
+  };
+  bool ctr_mode = false;
+  std::vector<CtrLive> ctr_live;
+  std::vector<uint32_t> ctr_free;           // free counter-mode slots
+  std::vector<uint32_t> ctr_mbase;          // running base per counter-mode slot
   std::vector<JobRec> jobs;         // indexed by job id (dense)
   std::vector<uint32_t> free_job_ids;
   uint32_t next_job = 0;

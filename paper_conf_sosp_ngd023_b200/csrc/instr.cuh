@@ -60,9 +60,13 @@ template <bool INSTR, uint32_t T = 0>
 __device__ __forceinline__ void instr_enter(const InstrArgs& ia) {
   if constexpr (INSTR) {
     if (threadIdx.x == T && threadIdx.y == 0 && threadIdx.z == 0) {
-      uint32_t total = gridDim.x * gridDim.y * gridDim.z;
-      uint32_t c = atomicAdd(&ia.ctr[0], 1u) + 1u - ia.base;
-      maybe_record(ia, REC_PLACEMENT, c, total);
+      if (ia.flags & INSTR_CTR) {
+        asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[0]) : "memory");
+      } else {
+        uint32_t total = gridDim.x * gridDim.y * gridDim.z;
+        uint32_t c = atomicAdd(&ia.ctr[0], 1u) + 1u - ia.base;
+        maybe_record(ia, REC_PLACEMENT, c, total);
+      }
     }
   }
 }
@@ -90,7 +94,15 @@ template <bool INSTR, uint32_t T = 0>
 __device__ __forceinline__ void instr_exit(const InstrArgs& ia) {
   if constexpr (INSTR) {
     __syncthreads();
-    if (threadIdx.x == T && threadIdx.y == 0 && threadIdx.z == 0) {
+    if (threadIdx.x == T && threadIdx.y == 0 && threadIdx.z == 0 && (ia.flags & INSTR_CTR)) {
+      // counter mode: a release reduction (the block's outputs, ordered before it by the
+      // barrier, are visible before the count is); nothing is waited for, the block
+      // retires at once.  System scope for a job's last kernel (output in host memory).
+      if (ia.flags & INSTR_LAST)
+        asm volatile("red.release.sys.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+      else
+        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+    } else if (threadIdx.x == T && threadIdx.y == 0 && threadIdx.z == 0) {
       // acq_rel atomic: releases this block's outputs (ordered before by the barrier,
       // release is cumulative) and acquires the earlier blocks' before the record is
       // written; system scope for a job's last kernel, whose output is in host memory

@@ -575,6 +575,63 @@ __global__ void __launch_bounds__(32, 1) k_notify_proxy(const Rec* dev_ring, Rec
 KernelFn proxy_kernel() { return (KernelFn)k_notify_proxy; }
 
 // ---------------------------------------------------------------------------
+// Counter mirror (counter-mode notification): one resident warp copies
+// the NCTR_M {start, end} launch counters (2 KiB of device memory) to pinned host
+// memory whenever they change.  Lane i owns 16-byte chunks i, i+32, i+64, i+96 (two
+// slots each).  A changed chunk is copied as loaded (acquire loads), so the host sees
+// a block's outputs no later than the count that covers the block.  The warp leaves
+// after ~35 ms without changes; the dispatcher relaunches it while launches are in
+// flight (the counters are the state, so nothing is lost across a relaunch).
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(32, 1) k_notify_mirror(const uint4* ctrs, uint4* host, volatile uint32_t* state) {
+  const uint32_t lane = threadIdx.x;
+  constexpr uint32_t NQ = NCTR_M * 2 / 4 / 32;   // 16-byte chunks per lane
+  uint4 prev[NQ];
+#pragma unroll
+  for (uint32_t i = 0; i < NQ; ++i) prev[i] = make_uint4(~0u, ~0u, ~0u, ~0u);   // publish everything once
+  uint32_t idle = 0;
+  for (;;) {
+    uint4 cur[NQ];
+    bool ch = false;
+#pragma unroll
+    for (uint32_t i = 0; i < NQ; ++i) {
+      asm volatile("ld.acquire.gpu.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+                   : "=r"(cur[i].x), "=r"(cur[i].y), "=r"(cur[i].z), "=r"(cur[i].w)
+                   : "l"(ctrs + lane + 32 * i));
+      ch |= cur[i].x != prev[i].x || cur[i].y != prev[i].y || cur[i].z != prev[i].z || cur[i].w != prev[i].w;
+    }
+    if (__any_sync(0xffffffffu, ch)) {
+      // no fence needed: each published word IS the loaded count (the store depends on
+      // the load), and a block's release reduction made its outputs visible -- at
+      // system scope for a job's last kernel -- before that count could be loaded
+#pragma unroll
+      for (uint32_t i = 0; i < NQ; ++i) {
+        if (cur[i].x != prev[i].x || cur[i].y != prev[i].y || cur[i].z != prev[i].z || cur[i].w != prev[i].w) {
+          asm volatile("st.relaxed.sys.global.v4.u32 [%0], {%1, %2, %3, %4};" ::"l"(host + lane + 32 * i),
+                       "r"(cur[i].x), "r"(cur[i].y), "r"(cur[i].z), "r"(cur[i].w)
+                       : "memory");
+          prev[i] = cur[i];
+        }
+      }
+      idle = 0;
+    } else {
+      ++idle;
+      if ((idle & 255) == 0) {
+        if (state[0] || idle > (1u << 16)) break;
+        if (lane == 0) state[16] = idle;
+      }
+      __nanosleep(64);
+    }
+  }
+  if (lane == 0) {
+    __threadfence_system();
+    state[32] = 1;
+  }
+}
+
+KernelFn mirror_kernel() { return (KernelFn)k_notify_mirror; }
+
+// ---------------------------------------------------------------------------
 // kernel table
 // ---------------------------------------------------------------------------
 template <typename T, bool I>

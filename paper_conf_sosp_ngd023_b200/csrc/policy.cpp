@@ -50,9 +50,12 @@ bool Policy::is_ready(const PolicyJob& j) const {
   uint32_t infl = j.inflight();
   if (infl == 0) return true;
   if (cfg_.lookahead == 0 || infl > cfg_.lookahead) return false;
-  const PolicyLaunch& L = launches_[j.last_uid % kLaunchSlots];
-  if (!L.live || L.uid != j.last_uid) return false;
-  return (L.p > L.f ? L.p : L.f) >= L.grid;   // most recent kernel fully placed
+  // kernels of a job complete in order (one stream), so layer `done` is the oldest
+  // kernel still in flight; launch-ahead once it is fully placed (running)
+  const uint32_t oldest = j.uid_of[j.done % 8];
+  const PolicyLaunch& L = launches_[oldest % kLaunchSlots];
+  if (!L.live || L.uid != oldest) return false;
+  return (L.p > L.f ? L.p : L.f) >= L.grid;
 }
 
 // bring the ready structures in line with is_ready(j)
@@ -237,6 +240,7 @@ void Policy::decide(std::vector<Issue>* out) {
     make_unready(j);
     j.R -= lay.tbar;
     work_ -= lay.tbar;
+    j.uid_of[j.cursor % 8] = uid;
     j.cursor += 1;
     j.last_uid = uid;
     Dt_[j.client] -= (int64_t)cfg_.num_clients;

@@ -42,6 +42,7 @@ struct PolicyJob {
   int32_t stream = -1;       // stream held while kernels are in flight
   int32_t last_stream = -1;
   uint32_t last_uid = 0;
+  uint32_t uid_of[8] = {0};  // launch uid of layer l (l mod 8) while in flight
   bool live = false;
   bool in_ready = false;
   uint32_t inflight() const { return cursor - done; }

@@ -118,20 +118,22 @@ def _serve_and_check(e, specs, n, n_clients, seed, rate_us=30.0):
                 done += 1
 
 
-@pytest.mark.parametrize("policy,group,streams,ring,look,lt,proxy", [
-    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 0, 0, True),
-    (L.POLICY_FIFO, 16, 32, 65536, 0, 0, True),
-    (L.POLICY_SRPT_DEFICIT, 1, 8, 1024, 0, 0, True),     # G = 1 debug mode, ring wraps many laps
-    (L.POLICY_SRPT_DEFICIT, 16, 1, 1024, 0, 0, True),    # a single stream
-    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 1, 2, True),  # launch-ahead + launcher threads (bench arm)
-    (L.POLICY_SRPT_DEFICIT, 4, 16, 4096, 2, 3, True),
-    (L.POLICY_SRPT_DEFICIT, 16, 32, 2048, 1, 2, False),  # direct record writes (the paper's path)
+@pytest.mark.parametrize("policy,group,streams,ring,look,lt,notify,prio", [
+    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 0, 0, "counters", 1),
+    (L.POLICY_FIFO, 16, 32, 65536, 0, 0, "counters", 1),
+    (L.POLICY_SRPT_DEFICIT, 1, 8, 1024, 0, 0, "ring", 1),     # G = 1 debug mode, ring wraps many laps
+    (L.POLICY_SRPT_DEFICIT, 1, 8, 1024, 0, 0, "counters", 2),
+    (L.POLICY_SRPT_DEFICIT, 16, 1, 1024, 0, 0, "counters", 1),    # a single stream
+    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 1, 4, "counters", 4),  # the bench arm
+    (L.POLICY_SRPT_DEFICIT, 4, 16, 4096, 2, 3, "ring", 4),
+    (L.POLICY_SRPT_DEFICIT, 16, 32, 2048, 1, 2, "direct", 1),  # direct record writes (the paper's path)
 ])
-def test_serving_parity_and_replay(tmp_path, policy, group, streams, ring, look, lt, proxy):
+def test_serving_parity_and_replay(tmp_path, policy, group, streams, ring, look, lt, notify, prio):
     log = str(tmp_path / "gpu_%u.log")
     names = ["toy", "resnet18", "mobilenet_v2", "squeezenet1_1"]
     with L.Engine(num_clients=3, policy=policy, group=group, streams=streams, ring_capacity=ring,
-                  event_log=log, max_jobs_per_model=32, lookahead=look, launch_threads=lt, proxy=proxy) as e:
+                  event_log=log, max_jobs_per_model=32, lookahead=look, launch_threads=lt, notify=notify,
+                  prio_classes=prio, slack=1184 if prio > 1 else 0) as e:
         specs = []
         for nm in names:
             g = archs.build(nm)
@@ -163,7 +165,7 @@ def test_ring_records_carry_sm_and_time(tmp_path):
     of a block's group never before the first placement of its launch."""
     log = str(tmp_path / "g1_%u.log")
     g = archs.toy()
-    with L.Engine(num_clients=1, group=1, event_log=log) as e:
+    with L.Engine(num_clients=1, group=1, event_log=log, notify="ring") as e:
         mid = e.register_model(g, rng.model_params(g))
         _serve_and_check(e, [(mid, "toy", g)], 10, 1, seed=1)
     cfg, ms, events, ex = eventlog.read(log % 0)
@@ -185,7 +187,8 @@ def test_per_sm_capacity_from_g1_records(tmp_path):
     Table-1 resources (+TMEM) according to the demands the dispatcher accounts."""
     log = str(tmp_path / "cap_%u.log")
     names = ["resnet18", "mobilenet_v2", "squeezenet1_1"]
-    with L.Engine(num_clients=3, group=1, event_log=log, ring_capacity=4096, lookahead=1, launch_threads=2) as e:
+    with L.Engine(num_clients=3, group=1, event_log=log, ring_capacity=4096, lookahead=1, launch_threads=2,
+                  notify="ring") as e:
         specs = []
         for nm in names:
             g = archs.build(nm)
