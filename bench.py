@@ -51,7 +51,7 @@ def parse():
     ap.add_argument("--rho", type=float, default=0.7)
     ap.add_argument("--reqs", type=int, default=2000, help="requests per step")
     ap.add_argument("--no-baselines", action="store_true")
-    ap.add_argument("--lookahead", type=int, default=1, help="NEXT-1 launch-ahead depth of the Paella arm")
+    ap.add_argument("--lookahead", type=int, default=3, help="NEXT-1 launch-ahead depth of the Paella arm")
     ap.add_argument("--slack", type=int, default=1184,
                     help="B, blocks issued beyond full utilisation (P1300-1304); 8 x 148 SMs covers the "
                          "measured dispatch loop delay (DESIGN.md B200-Q1)")

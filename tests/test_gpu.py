@@ -124,7 +124,7 @@ def _serve_and_check(e, specs, n, n_clients, seed, rate_us=30.0):
     (L.POLICY_SRPT_DEFICIT, 1, 8, 1024, 0, 0, "ring", 1),     # G = 1 debug mode, ring wraps many laps
     (L.POLICY_SRPT_DEFICIT, 1, 8, 1024, 0, 0, "counters", 2),
     (L.POLICY_SRPT_DEFICIT, 16, 1, 1024, 0, 0, "counters", 1),    # a single stream
-    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 1, 4, "counters", 4),  # the bench arm
+    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 3, 4, "counters", 4),  # the bench arm
     (L.POLICY_SRPT_DEFICIT, 4, 16, 4096, 2, 3, "ring", 4),
     (L.POLICY_SRPT_DEFICIT, 16, 32, 2048, 1, 2, "direct", 1),  # direct record writes (the paper's path)
 ])
