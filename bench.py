@@ -55,7 +55,7 @@ def parse():
     ap.add_argument("--slack", type=int, default=1184,
                     help="B, blocks issued beyond full utilisation (P1300-1304); 8 x 148 SMs covers the "
                          "measured dispatch loop delay (DESIGN.md B200-Q1)")
-    ap.add_argument("--prio-classes", type=int, default=4, help="stream-priority classes (DESIGN.md B200-Q2)")
+    ap.add_argument("--prio-classes", type=int, default=1, help="stream-priority classes (DESIGN.md B200-Q2)")
     ap.add_argument("--launch-threads", type=int, default=4, help="launcher helper threads per GPU")
     ap.add_argument("--sat-reqs", type=int, default=1500, help="requests of the saturation calibration")
     ap.add_argument("--fake", action="store_true",
