@@ -58,6 +58,9 @@ def parse():
     ap.add_argument("--prio-classes", type=int, default=1, help="stream-priority classes (DESIGN.md B200-Q2)")
     ap.add_argument("--launch-threads", type=int, default=4, help="launcher helper threads per GPU")
     ap.add_argument("--sat-reqs", type=int, default=1500, help="requests of the saturation calibration")
+    ap.add_argument("--slo-rhos", default="0.5,0.7,0.9,1.0,1.1,1.2,1.35,1.5",
+                    help="offered loads (x X_sat(naive)) of the req/s-at-p99-SLO ladder ('' = skip)")
+    ap.add_argument("--slo-reqs", type=int, default=1500, help="requests per point of the SLO ladder")
     ap.add_argument("--fake", action="store_true",
                     help="CPU fake device (tests of the multi-rank plumbing; not a measurement)")
     return ap.parse_args()
@@ -207,6 +210,27 @@ def saturation(e, mids, n_models, stride, slots, n, seed=99):
     return n / (el / 1e9)
 
 
+def slo_ladder(e, args, cfg, names, x_sat_naive, slo, stride, slots, seed):
+    """req/s at p99 SLO: the largest offered lambda of the ladder
+    rho * X_sat(naive) at which every model's p99 JCT is within its SLO (an
+    overloaded point fails it: the backlog grows through the point's window)."""
+    rhos = [float(r) for r in args.slo_rhos.split(",") if r.strip()]
+    pts, best = [], 0.0
+    for i, r in enumerate(rhos):
+        lam = r * x_sat_naive
+        t, mm, ii = make_trace(args.slo_reqs, lam, cfg, len(names), seed=seed + i)
+        jct, el = e.loadgen(t, mm, mm, ii, stride, slots)
+        st = jct_stats(jct, mm, names)
+        ok = all(st.get(n, {}).get("p99_us", 1e18) <= slo[n] for n in names)
+        served = (jct >= 0).sum() / (el / 1e9)
+        pts.append({"rho": r, "offered_req_s": round(lam, 1), "served_req_s": round(float(served), 1),
+                    "p99_us": {n: round(st[n]["p99_us"], 1) for n in names if n in st},
+                    "mean_us": round(st["mix"]["mean_us"], 1), "slo_met": bool(ok)})
+        if ok:
+            best = max(best, lam)
+    return {"req_s": round(best, 1), "ladder": pts}
+
+
 def run_gpu(args, dist):
     from paper_conf_sosp_ngd023_b200 import _lib as L
     L.load()
@@ -307,6 +331,9 @@ def run_gpu(args, dist):
     t, mm, ii = make_trace(args.reqs, lam, cfg, len(names), seed=seed0 + 500)
     e2e_jct, e2e_el = e.loadgen(t, mm, mm, ii, stride, slots, copy_inputs=copy_in)
     e2e_rate = (e2e_jct >= 0).sum() / (e2e_el / 1e9)
+    slo_at = {}
+    if args.slo_rhos and not args.no_baselines:
+        slo_at["paella"] = slo_ladder(e, args, cfg, names, x_sat_naive, slo, stride, slots, seed0 + 700)
     h2d = float(np.mean([sizes[m] - specs[m][0].num_classes * 4 for m in mm]))
     d2h = float(np.mean([specs[m][0].num_classes * 4 for m in mm]))
     e.shutdown()
@@ -323,13 +350,16 @@ def run_gpu(args, dist):
                 t, mm, ii = make_trace(args.reqs, lam, cfg, len(names), seed=seed0 + 100 + s)
                 j, _ = eb.loadgen(t, mm, mm, ii, stride, slots)
                 jl.append((j, mm))
+            if label == "naive_cuda_ms" and args.slo_rhos:
+                slo_at["naive"] = slo_ladder(eb, args, cfg, names, x_sat_naive, slo, stride, slots, seed0 + 700)
             eb.shutdown()
             base[label] = jct_stats(np.concatenate([a for a, _ in jl]), np.concatenate([b for _, b in jl]), names)
 
     return dict(unloaded=unloaded, names=names, lam=lam, x_sat_naive=x_sat_naive, x_sat_paella=x_sat_paella, slo=slo,
                 elapsed=elapsed, completed=completed, jct=jct_stats(jct, models, names), clocks=clk,
                 ev=ev, stats=stats, dev_roof=dev_roof, base=base, e2e_rate=e2e_rate,
-                e2e=jct_stats(e2e_jct, mm, names), h2d=h2d, d2h=d2h, calib_s=calib_s, kinfo=kinfo)
+                e2e=jct_stats(e2e_jct, mm, names), h2d=h2d, d2h=d2h, calib_s=calib_s, kinfo=kinfo,
+                slo_at=slo_at)
 
 
 def cpu_baseline(cfg, seconds=12.0):
@@ -455,6 +485,8 @@ def main():
                           "slack_blocks": args.slack, "prio_classes": args.prio_classes, "pdl": True,
                           "theta": 100, "group": 16, "streams": 32},
         "slo_met": bool(all(res["jct"].get(n, {}).get("p99_us", 1e18) <= res["slo"][n] for n in res["names"])),
+        "req_s_at_p99_slo": {k: v["req_s"] for k, v in res["slo_at"].items()},
+        "slo_ladder": res["slo_at"],
         "x_sat_req_s": {"naive": round(res["x_sat_naive"], 1), "paella": round(res["x_sat_paella"], 1)},
         "jct_unloaded_p50_us": {k: {m: round(v, 1) for m, v in d.items()} for k, d in res["unloaded"].items()},
         "device_roofline_us": {k: round(v, 2) for k, v in res["dev_roof"].items()},
