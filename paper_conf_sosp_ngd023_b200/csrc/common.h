@@ -109,6 +109,7 @@ struct LayerArgs {
   uint32_t kpad;            // packed K (conv) / row pitch (fc), in elements
   uint32_t tiles_m, tiles_n;// tcgen05 conv: tile grid
   uint32_t ksplit;          // split-K factor (1 = none)
+  uint32_t a_rows;          // tcgen05 conv: weight rows fetched per stage (TMA box), <= 128
   float* ws;                // fp32 split-K workspace
   uint32_t* ws_ctr;         // split-K arrival counters (one per output tile)
 };

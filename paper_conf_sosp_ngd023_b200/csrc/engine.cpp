@@ -359,7 +359,7 @@ struct CudaBackend : Backend {
 };
 
 // per-(model, gpu) tensor maps for tcgen05 weights (defined in kernels_tc.cu)
-int make_weight_tmap(void* weights, uint32_t rows, uint32_t kpad, void* out128);
+int make_weight_tmap(void* weights, uint32_t rows, uint32_t kpad, uint32_t box_rows, void* out128);
 
 
 // ---------------------------------------------------------------------------
@@ -1312,10 +1312,10 @@ static int iso_run(Gpu* g, Model* m, const void* input, void* output, int64_t* k
     uint64_t t0 = UINT64_MAX;
     for (uint32_t b = 0; b < nb; ++b) t0 = std::min(t0, h[16 * b]);
     const char* names[16] = {"entry", "setup", "full0", "mma_done", "accb", "epi_done", "pre_exit", "exit",
-                             "tmem2smem", "pre_bar", "post_bar", "inited", "tma_issued", "b_issued", "reduced", "-"};
+                             "tmem2smem", "pre_bar", "post_bar", "inited", "tma_issued", "b_issued", "reduced", "peers01"};
     fprintf(stderr, "trace kernel %d grid %u (ns from first CTA entry): phase min/med/max\n", trace_k, nb);
-    const int order[15] = {0, 11, 12, 13, 1, 2, 3, 4, 8, 9, 10, 14, 5, 6, 7};
-    for (int oi = 0; oi < 15; ++oi) {
+    const int order[16] = {0, 11, 12, 13, 1, 2, 3, 4, 8, 9, 10, 15, 14, 5, 6, 7};
+    for (int oi = 0; oi < 16; ++oi) {
       int ph = order[oi];
       std::vector<int64_t> v;
       for (uint32_t b = 0; b < nb; ++b)
@@ -1392,7 +1392,7 @@ static int setup_model_gpu(Paella* P, Model* m, Gpu* g) {
       k.regs = (uint32_t)fa.numRegs;
       k.static_smem = (uint32_t)fa.sharedSizeBytes;
       if (is_tc(k.kind)) {
-        if (make_weight_tmap(wdev + k.w_off, k.proto.tiles_m * TC_BM, k.proto.kpad, tmaps[l].b)) return -EIO;
+        if (make_weight_tmap(wdev + k.w_off, k.proto.tiles_m * TC_BM, k.proto.kpad, k.proto.a_rows, tmaps[l].b)) return -EIO;
       }
     } else {
       k.regs = 64;

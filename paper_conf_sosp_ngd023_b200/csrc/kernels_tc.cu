@@ -166,6 +166,49 @@ __device__ __forceinline__ uint4 load_res8(const LayerArgs& a, uint32_t p, uint3
                                               a.res_co + co));
 }
 
+// ksplit == 1 epilogue of one thread: 8 items (pixel px0 + 8 i, channel group g),
+// activation and residual fixed at compile time so the unrolled items carry no
+// branches and interleave (a single warp per SM sub-partition runs this: its speed
+// is instruction latency, not bandwidth); one output pointer advanced by 8 pixels.
+template <uint32_t ACT, bool RES, uint32_t NIT>
+__device__ __forceinline__ void epi_tile(const LayerArgs& a, const float* stage, uint32_t n0, uint32_t P,
+                                         uint32_t g, uint32_t co, const float (&bias)[8],
+                                         const uint4 (&res)[NIT]) {
+  const uint32_t px0 = threadIdx.x / (TC_BM / 8);
+  __nv_bfloat16* out = static_cast<__nv_bfloat16*>(a.out) + (size_t)(n0 + px0) * a.out_cs + a.out_co + co;
+  const size_t ostep = (size_t)(NPROD / (TC_BM / 8)) * a.out_cs;
+  // all items are computed (the staged tile has 64 pixel rows), only the stores are
+  // predicated: no branches around the item bodies, so the compiler interleaves them
+#pragma unroll
+  for (uint32_t i = 0; i < NIT; ++i) {
+    const uint32_t px = px0 + i * (NPROD / (TC_BM / 8));
+    const float4* q = reinterpret_cast<const float4*>(stage + px * TC_BM + g * 8);
+    const float4 u0 = q[0], u1 = q[1];
+    float x[8] = {u0.x + bias[0], u0.y + bias[1], u0.z + bias[2], u0.w + bias[3],
+                  u1.x + bias[4], u1.y + bias[5], u1.z + bias[6], u1.w + bias[7]};
+    if constexpr (RES) {
+      const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&res[i]);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const float2 f = __bfloat1622float2(h[j]);
+        x[2 * j] += f.x;
+        x[2 * j + 1] += f.y;
+      }
+    }
+    uint4 o;
+    __nv_bfloat162* oh = reinterpret_cast<__nv_bfloat162*>(&o);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      float y0 = x[2 * j], y1 = x[2 * j + 1];
+      if constexpr (ACT >= 1) { y0 = fmaxf(y0, 0.f); y1 = fmaxf(y1, 0.f); }
+      if constexpr (ACT == 2) { y0 = fminf(y0, 6.f); y1 = fminf(y1, 6.f); }
+      oh[j] = __floats2bfloat162_rn(y0, y1);
+    }
+    if (n0 + px < P) *reinterpret_cast<uint4*>(out) = o;
+    out += ostep;
+  }
+}
+
 // 2 CTAs per SM (two jobs' convs can share an SM): <= 168 registers.  Warp 5 does
 // only the block bookkeeping (instrumentation), so no compute warp waits on its
 // atomics at entry.
@@ -181,7 +224,10 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   if (trace && threadIdx.x == 0) tr[0] = globaltimer();
   instr_enter<INSTR, TBOOK>(ia);
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  // 1024-byte aligned (SW128 atoms); pointer arithmetic on smem_raw (not an integer
+  // cast) keeps the shared address space visible to the compiler: LDS/STS, no
+  // aliasing with global stores
+  uint8_t* smem = smem_raw + ((1024u - (su32(smem_raw) & 1023u)) & 1023u);
   uint8_t* sA = smem;                                  // STAGES x 16 KiB
   uint8_t* sB = smem + TC_STAGES * A_BYTES;            // STAGES x 8 KiB
   uint64_t* full = (uint64_t*)(sB + TC_STAGES * B_BYTES);
@@ -201,6 +247,9 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   const uint32_t nkl = kb1 > kb0 ? kb1 - kb0 : 0;
 
   const uint32_t pre = nkl < TC_STAGES ? nkl : TC_STAGES;
+  // narrow layers (Cout < 128) fetch only a_rows weight rows per stage; rows a_rows..127
+  // of every A stage are zeroed once below (the UMMA still runs M = 128)
+  const uint32_t abytes = a.a_rows * 128;
   if (warp == 4 && lane == 0) {
     // the MMA warp's leader sets up the barriers and starts the weight stream while
     // the gather warps compute their addresses
@@ -212,34 +261,43 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     if (trace) tr[11] = globaltimer();
     for (uint32_t it = 0; it < pre; ++it) {   // the first stages need no empty-wait
-      mbar_arrive_tx(&full[it], A_BYTES);
+      mbar_arrive_tx(&full[it], abytes);
       tma_load_2d(sA + it * A_BYTES, &wmap, &full[it], (int)((kb0 + it) * TC_BK), (int)m0);
     }
     if (trace) tr[12] = globaltimer();
   }
+  // epilogue operands that do not depend on the accumulator: the bias (a weight) is
+  // fetched before the PDL wait, the residual right after it, both hidden behind the
+  // main loop.  Thread t owns channel group eg = t % 16 and pixels t / 16 + 8 i.
+  const uint32_t eg = threadIdx.x % (TC_BM / 8), eco = m0 + eg * 8;
+  constexpr uint32_t NIT = TC_BN * (TC_BM / 8) / NPROD;   // 8 items per thread
+  float ebias[8];
+  uint4 eres[NIT];
+  if (warp < 4 && a.ksplit == 1) load_bias8(a, eco, ebias);
   // ---- producer state (warps 0-3): this thread gathers 16-byte chunk `chunk` of
   // pixel rows n = t/8 + 16 j (j < 4) of every B stage
   const __nv_bfloat16* X = static_cast<const __nv_bfloat16*>(a.in);
   const uint32_t t = threadIdx.x;
   const uint32_t chunk = t % 8;
-  int ohs[4], ows[4];
-  bool pv[4];
+  // per pixel row j: top-left input coordinate of its window (invalid pixels get a
+  // coordinate that fails every bounds check) and its element offset; per stage only
+  // the (r, s, ci) offset `dk`, common to the 4 rows, changes
+  int ih0[4], iw0[4], off0[4];
   const uint32_t K = a.kh * a.kw * a.cin;
+  const uint32_t dst0 = (t / 8) * 128 + ((chunk ^ ((t / 8) & 7)) << 4);   // row t/8 of the SW128 atom
   // (r, s, ci) of k = kbase + 8*chunk, advanced incrementally by TC_BK per stage
   int kr = 0, ks_ = 0, kci = 0;
+  uint32_t kcur = 0;
   auto issue_B = [&](uint32_t it, bool arrive) {
     const uint32_t s = it % TC_STAGES;
-    const uint32_t k = (kb0 + it) * TC_BK + chunk * 8;
-    const bool kv = k < K;
-    const uint32_t bstage = su32(sB + s * B_BYTES);
+    const bool kv = kcur < K;
+    const int dk = (kr * (int)a.w_ + ks_) * (int)a.in_cs + kci;
+    const uint32_t bstage = su32(sB + s * B_BYTES) + dst0;
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
-      const uint32_t n = t / 8 + 16 * j;
-      const int ih = ohs[j] * (int)a.sh - (int)a.ph + kr;
-      const int iw = ows[j] * (int)a.sw - (int)a.pw + ks_;
-      const bool ok = kv && pv[j] && ih >= 0 && ih < (int)a.h && iw >= 0 && iw < (int)a.w_;
-      const __nv_bfloat16* src = ok ? X + ((size_t)ih * a.w_ + iw) * a.in_cs + a.in_co + kci : X;
-      const uint32_t dst = bstage + n * 128 + ((chunk ^ (n & 7)) << 4);
+      const bool ok = kv && (uint32_t)(ih0[j] + kr) < a.h && (uint32_t)(iw0[j] + ks_) < a.w_;
+      const __nv_bfloat16* src = ok ? X + (off0[j] + dk) : X;
+      const uint32_t dst = bstage + j * 2048;   // pixel row n = t/8 + 16 j
       if constexpr (!PRO) {
         cp_async16(dst, src, ok ? 16u : 0u);
       } else {
@@ -274,6 +332,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
         asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(su32(&full[s])) : "memory");
     }
     // advance (r, s, ci) by TC_BK channels for the next stage
+    kcur += TC_BK;
     kci += TC_BK;
     while (kci >= (int)a.cin) {
       kci -= (int)a.cin;
@@ -286,22 +345,42 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   if (warp < 4) {
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
-      uint32_t p = n0 + t / 8 + 16 * j;
-      pv[j] = p < P;
-      ohs[j] = pv[j] ? (int)(p / a.ow) : 0;
-      ows[j] = pv[j] ? (int)(p % a.ow) : 0;
+      const uint32_t p = n0 + t / 8 + 16 * j;
+      const bool pv = p < P;
+      const int oh = (int)(p / a.ow), ow = (int)(p - (uint32_t)oh * a.ow);
+      ih0[j] = pv ? oh * (int)a.sh - (int)a.ph : -(1 << 20);
+      iw0[j] = pv ? ow * (int)a.sw - (int)a.pw : -(1 << 20);
+      off0[j] = pv ? (ih0[j] * (int)a.w_ + iw0[j]) * (int)a.in_cs + (int)a.in_co : 0;
     }
     {
       const uint32_t k0 = kb0 * TC_BK + chunk * 8;
+      kcur = k0;
       kci = (int)(k0 % a.cin);
       const int rs = (int)(k0 / a.cin);
       ks_ = rs % (int)a.kw;
       kr = rs / (int)a.kw;
     }
+    if (a.a_rows < TC_BM) {
+      const uint32_t zb = A_BYTES - abytes;   // bytes per stage, multiple of 1024
+      for (uint32_t o = t * 16; o < TC_STAGES * zb; o += NPROD * 16) {
+        const uint32_t st = o / zb;
+        asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(su32(sA + st * A_BYTES + abytes + (o - st * zb))),
+                     "r"(0u)
+                     : "memory");
+      }
+      fence_proxy_async();   // visible to the tensor core (async proxy) after the CTA barrier
+    }
     // ... and the first activation gathers, before the CTA-wide barrier, once the
     // predecessor kernel's output is complete (PDL; the weight TMA above needs no wait)
     pdl_wait();
     for (uint32_t it = 0; it < pre; ++it) issue_B(it, false);   // barriers not initialised yet
+    if (a.ksplit == 1 && (a.flags & LF_RESIDUAL) && eco < a.cout) {
+#pragma unroll
+      for (uint32_t i = 0; i < NIT; ++i) {
+        const uint32_t p = n0 + t / (TC_BM / 8) + i * (NPROD / (TC_BM / 8));
+        if (p < P) eres[i] = load_res8(a, p, eco);
+      }
+    }
     if (trace && t == 0) tr[13] = globaltimer();
   }
   __syncthreads();
@@ -316,7 +395,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
         const uint32_t s = nxt % TC_STAGES;
         mbar_wait(&empty[s], ((nxt / TC_STAGES) & 1) ^ 1);   // MMA of stage nxt - STAGES retired
         if (t == 0) {
-          mbar_arrive_tx(&full[s], A_BYTES);
+          mbar_arrive_tx(&full[s], abytes);
           tma_load_2d(sA + s * A_BYTES, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
         }
         issue_B(nxt, true);
@@ -331,7 +410,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
           const uint32_t s = nxt % TC_STAGES;
           mbar_wait(&empty[s], ((nxt / TC_STAGES) & 1) ^ 1);
           if (t == 0) {
-            mbar_arrive_tx(&full[s], A_BYTES);
+            mbar_arrive_tx(&full[s], abytes);
             tma_load_2d(sA + s * A_BYTES, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
           }
           issue_B(nxt, true);
@@ -374,22 +453,6 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   // 1. TMEM -> registers (warp w owns lanes = output channels 32w..32w+31) -> fp32
   //    tile in shared memory [pixel][channel] (conflict-free: a warp writes 32
   //    consecutive words of one pixel row)
-  // epilogue operands that do not depend on the accumulator (bias, residual) are
-  // fetched while the tensor core is still working
-  const uint32_t eg = threadIdx.x % (TC_BM / 8), eco = m0 + eg * 8;
-  constexpr uint32_t NIT = TC_BN * (TC_BM / 8) / NPROD;   // 8 items per thread
-  float ebias[8];
-  uint4 eres[NIT];
-  if (warp < 4 && a.ksplit == 1) {
-    load_bias8(a, eco, ebias);
-    if (a.flags & LF_RESIDUAL) {
-#pragma unroll
-      for (uint32_t i = 0; i < NIT; ++i) {
-        const uint32_t p = n0 + (threadIdx.x + i * NPROD) / (TC_BM / 8);
-        if (p < P && eco < a.cout) eres[i] = load_res8(a, p, eco);
-      }
-    }
-  }
   // every input of this block has been consumed: let the dependent kernel be placed
   // (its prologue overlaps this epilogue); warp 5 follows the accumulator too
   if (warp == 5 && nkl > 0) mbar_wait(accb, 0);
@@ -421,15 +484,17 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       if (trace && threadIdx.x == 0) tr[9] = globaltimer();
       asm volatile("bar.sync 1, 128;" ::: "memory");   // the 4 epilogue warps only
       if (trace && threadIdx.x == 0) tr[10] = globaltimer();
-#pragma unroll
-      for (uint32_t i = 0; i < NIT; ++i) {
-        const uint32_t px = (threadIdx.x + i * NPROD) / (TC_BM / 8);
-        const uint32_t p = n0 + px;
-        if (p < P && co < a.cout) {
-          const float4* q = reinterpret_cast<const float4*>(stage + px * TC_BM + g * 8);
-          float4 u0 = q[0], u1 = q[1];
-          float v[8] = {u0.x, u0.y, u0.z, u0.w, u1.x, u1.y, u1.z, u1.w};
-          epi_store8(a, p, co, v, ebias, eres[i]);
+      if (co < a.cout) {
+        const bool rf = (a.flags & LF_RESIDUAL) != 0;
+        if (a.act == 1) {
+          if (rf) epi_tile<1, true>(a, stage, n0, P, g, co, ebias, eres);
+          else epi_tile<1, false>(a, stage, n0, P, g, co, ebias, eres);
+        } else if (a.act == 2) {
+          if (rf) epi_tile<2, true>(a, stage, n0, P, g, co, ebias, eres);
+          else epi_tile<2, false>(a, stage, n0, P, g, co, ebias, eres);
+        } else {
+          if (rf) epi_tile<0, true>(a, stage, n0, P, g, co, ebias, eres);
+          else epi_tile<0, false>(a, stage, n0, P, g, co, ebias, eres);
         }
       }
     }
@@ -437,58 +502,100 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     // split-K across the CTAs of a cluster (1 x 1 x ksplit): each CTA reduces a
     // 1/ksplit slice of the tile's pixel rows over DSMEM (16-byte loads) and runs the
     // epilogue for it -- no global workspace, no atomics.
+    // Items of thread t: pixel rows px0 + (t + 128 i) / 16 (i < 4, ksplit >= 2), one
+    // channel group g = t % 16.  Bias and residual are fetched before the cluster
+    // barrier; after it each peer's slices of all items are loaded back to back.
+    constexpr uint32_t MAXI = TC_BN * (TC_BM / 8) / (2 * NPROD);   // 4 items at ksplit 2
+    const uint32_t ks = a.ksplit;
+    const uint32_t rows = TC_BN / ks;
+    const uint32_t px0 = split * rows;
+    const uint32_t g = threadIdx.x % (TC_BM / 8), co = m0 + g * 8;
+    const uint32_t nitems = rows * (TC_BM / 8);
+    float bias[8];
+    uint4 rres[MAXI];
+    if (warp < 4 && co < a.cout) {
+      load_bias8(a, co, bias);
+      if (a.flags & LF_RESIDUAL) {
+#pragma unroll
+        for (uint32_t i = 0; i < MAXI; ++i) {
+          const uint32_t item = threadIdx.x + i * NPROD;
+          const uint32_t p = n0 + px0 + item / (TC_BM / 8);
+          if (item < nitems && p < P) rres[i] = load_res8(a, p, co);
+        }
+      }
+    }
     __syncwarp();
     if (trace && threadIdx.x == 0) tr[9] = globaltimer();
-    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    // the staged partial tile (shared::cta writes) is released to the cluster with the
+    // restricted fence (MEMBAR.CTA; a plain arrive.release would be MEMBAR.GPU, which
+    // also drains every outstanding global access), then a relaxed arrive
+    asm volatile(
+        "fence.release.sync_restrict::shared::cta.cluster;\n\t"
+        "barrier.cluster.arrive.relaxed.aligned;\n\tbarrier.cluster.wait.aligned;" ::: "memory");
     if (trace && threadIdx.x == 0) tr[10] = globaltimer();
-    if (warp < 4) {
-      const uint32_t ks = a.ksplit;
-      const uint32_t rows = TC_BN / ks;
-      const uint32_t px0 = split * rows;
+    if (warp < 4 && co < a.cout) {
+      float4 acc[MAXI][2];
+#pragma unroll
+      for (uint32_t i = 0; i < MAXI; ++i) acc[i][0] = acc[i][1] = make_float4(0.f, 0.f, 0.f, 0.f);
+      // two peers at a time (ksplit is a power of two): their 4 x MAXI 16-byte loads
+      // are issued back to back (ld.shared::cluster), then accumulated.  CTA r starts with its
+      // own slice, then r + 1, ... (staggered): every round each CTA's shared memory serves one reader
+      // (DSMEM bandwidth is paid by the serving SM's port)
       const uint32_t base = su32(stage);
-      // items of this thread share channel group g = t % 16 (one bias load)
-      const uint32_t g = threadIdx.x % (TC_BM / 8), co = m0 + g * 8;
-      float bias[8];
-      load_bias8(a, co, bias);
-      for (uint32_t item = threadIdx.x; item < rows * (TC_BM / 8); item += NPROD) {
-        const uint32_t px = px0 + item / (TC_BM / 8);
-        const uint32_t p = n0 + px;
-        if (p < P && co < a.cout) {
-          uint4 res = make_uint4(0, 0, 0, 0);
-          if (a.flags & LF_RESIDUAL) res = load_res8(a, p, co);
-          const uint32_t off = (px * TC_BM + g * 8) * 4;
-          float v[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-          for (uint32_t r0 = 0; r0 < ks; r0 += 4) {   // 4 peers' slices in flight at once
-            float4 part[4][2];
+      for (uint32_t q = 0; q < ks; q += 2) {
+        float4 part[2][MAXI][2];
 #pragma unroll
-            for (uint32_t q = 0; q < 4; ++q) {
-              if (r0 + q < ks) {
-                uint32_t peer;
-                asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(peer) : "r"(base + off), "r"(r0 + q));
-                asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
-                             : "=f"(part[q][0].x), "=f"(part[q][0].y), "=f"(part[q][0].z), "=f"(part[q][0].w)
-                             : "r"(peer));
-                asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
-                             : "=f"(part[q][1].x), "=f"(part[q][1].y), "=f"(part[q][1].z), "=f"(part[q][1].w)
-                             : "r"(peer + 16));
-              }
-            }
+        for (uint32_t h = 0; h < 2; ++h) {
 #pragma unroll
-            for (uint32_t q = 0; q < 4; ++q) {
-              if (r0 + q < ks) {
-                v[0] += part[q][0].x; v[1] += part[q][0].y; v[2] += part[q][0].z; v[3] += part[q][0].w;
-                v[4] += part[q][1].x; v[5] += part[q][1].y; v[6] += part[q][1].z; v[7] += part[q][1].w;
-              }
+          for (uint32_t i = 0; i < MAXI; ++i) {
+            const uint32_t item = threadIdx.x + i * NPROD;
+            if (item < nitems && n0 + px0 + item / (TC_BM / 8) < P) {   // no traffic for the tail's empty rows
+              uint32_t peer;
+              asm volatile("mapa.shared::cluster.u32 %0, %1, %2;"
+                           : "=r"(peer)
+                           : "r"(base + ((px0 + item / (TC_BM / 8)) * TC_BM + g * 8) * 4),
+                             "r"((split + q + h) & (ks - 1)));
+              asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
+                           : "=f"(part[h][i][0].x), "=f"(part[h][i][0].y), "=f"(part[h][i][0].z),
+                             "=f"(part[h][i][0].w)
+                           : "r"(peer));
+              asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
+                           : "=f"(part[h][i][1].x), "=f"(part[h][i][1].y), "=f"(part[h][i][1].z),
+                             "=f"(part[h][i][1].w)
+                           : "r"(peer + 16));
             }
           }
-          epi_store8(a, p, co, v, bias, res);
+        }
+#pragma unroll
+        for (uint32_t h = 0; h < 2; ++h) {
+#pragma unroll
+          for (uint32_t i = 0; i < MAXI; ++i) {
+            const uint32_t item = threadIdx.x + i * NPROD;
+            if (item < nitems && n0 + px0 + item / (TC_BM / 8) < P) {
+              acc[i][0].x += part[h][i][0].x; acc[i][0].y += part[h][i][0].y;
+              acc[i][0].z += part[h][i][0].z; acc[i][0].w += part[h][i][0].w;
+              acc[i][1].x += part[h][i][1].x; acc[i][1].y += part[h][i][1].y;
+              acc[i][1].z += part[h][i][1].z; acc[i][1].w += part[h][i][1].w;
+            }
+          }
+        }
+        if (trace && q == 0 && threadIdx.x == 0) tr[15] = globaltimer();
+      }
+#pragma unroll
+      for (uint32_t i = 0; i < MAXI; ++i) {
+        const uint32_t item = threadIdx.x + i * NPROD;
+        const uint32_t p = n0 + px0 + item / (TC_BM / 8);
+        if (item < nitems && p < P) {
+          const float v[8] = {acc[i][0].x, acc[i][0].y, acc[i][0].z, acc[i][0].w,
+                              acc[i][1].x, acc[i][1].y, acc[i][1].z, acc[i][1].w};
+          epi_store8(a, p, co, v, bias, rres[i]);
         }
       }
     }
     // no CTA may leave while a peer still reads its shared memory
     if (trace && threadIdx.x == 0) tr[14] = globaltimer();
     __syncwarp();
-    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    asm volatile("barrier.cluster.arrive.relaxed.aligned;\n\tbarrier.cluster.wait.aligned;" ::: "memory");
   }
   if (trace && threadIdx.x == 0) tr[5] = globaltimer();
   tc_fence_before();
@@ -511,12 +618,13 @@ void tc_kernel_table(KernelFn* instr, KernelFn* plain) {
   plain[1] = (KernelFn)k_conv_tc<false, true>;
 }
 
-// Host: tensor map for the packed weights [rows][kpad] bf16, box 64 x 128, SW128.
+// Host: tensor map for the packed weights [rows][kpad] bf16, box 64 x box_rows
+// (128, or Cout rounded up to 8 for narrow layers), SW128.
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
 
-int make_weight_tmap(void* weights, uint32_t rows, uint32_t kpad, void* out128) {
+int make_weight_tmap(void* weights, uint32_t rows, uint32_t kpad, uint32_t box_rows, void* out128) {
   static EncodeTiledFn enc = nullptr;
   if (!enc) {
     cudaDriverEntryPointQueryResult q;
@@ -528,7 +636,7 @@ int make_weight_tmap(void* weights, uint32_t rows, uint32_t kpad, void* out128) 
   }
   cuuint64_t dims[2] = {kpad, rows};
   cuuint64_t strides[1] = {(cuuint64_t)kpad * 2};
-  cuuint32_t box[2] = {TC_BK, TC_BM};
+  cuuint32_t box[2] = {TC_BK, box_rows};
   cuuint32_t estr[2] = {1, 1};
   CUresult r = enc((CUtensorMap*)out128, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, weights, dims, strides, box, estr,
                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,

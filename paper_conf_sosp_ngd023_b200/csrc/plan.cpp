@@ -212,6 +212,7 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
     a.groups = nd.groups ? nd.groups : 1;
     a.act = nd.act;
     a.ksplit = 1;
+    a.a_rows = TC_BM;
     if (i == n - 1) a.flags |= LF_FINAL;
     if (nd.flags & PAELLA_NODE_PROLOGUE) {
       if (!nd.pro_scale || !nd.pro_shift) return -EINVAL;
@@ -276,6 +277,8 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
                 while (split < 16 && tiles * split * 2 <= P->sms && nk / (split * 2) >= 4) split *= 2;
             }
             a.ksplit = split;
+            // narrow layers: fetch only the live weight rows (SW128 atoms are 8 rows)
+            a.a_rows = nd.c < TC_BM ? (uint32_t)align_up(nd.c, 8) : TC_BM;
             k.grid[0] = a.tiles_n;
             k.grid[1] = a.tiles_m;
             k.grid[2] = split;
