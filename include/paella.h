@@ -257,6 +257,9 @@ typedef struct {
                                   [0] none (all ready work issued), [1] no free stream,
                                   [2] occupancy predicate (fits), [3] ring flow control */
   uint64_t sum_ready, sum_live_jobs, sum_Q;   /* summed over decide() passes (averages) */
+  uint64_t rel_events;         /* counter mode: stream-release events recorded (a job left idle) */
+  uint64_t xstream_waits;      /* ... of which the job's next kernel went to another stream
+                                  and waited for the event (relaxed exits) */
 } paella_stats_t;
 
 int paella_stats(paella_t* p, uint32_t gpu, paella_stats_t* st);

@@ -87,7 +87,7 @@ class Stats(C.Structure):
                 ("loop_iters", C.c_uint64), ("outstanding_work_ns", C.c_int64), ("ev_launches", C.c_uint64),
                 ("ev_ns", C.c_uint64), ("ev_bytes", C.c_uint64), ("ev_flops", C.c_uint64),
                 ("stop_reason", C.c_uint64 * 4), ("sum_ready", C.c_uint64), ("sum_live_jobs", C.c_uint64),
-                ("sum_Q", C.c_uint64)]
+                ("sum_Q", C.c_uint64), ("rel_events", C.c_uint64), ("xstream_waits", C.c_uint64)]
 
 
 _lib = None

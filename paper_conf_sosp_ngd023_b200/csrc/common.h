@@ -63,7 +63,7 @@ PAELLA_HD inline RecFields rec_decode(uint64_t w0, uint64_t w1) {
 // end} counters with fire-and-forget reductions and writes no record; the mirror warp
 // (k_notify_mirror) copies the counters to pinned host memory and the dispatcher turns
 // counter progress into the same group-of-G records (engine.cpp::drain_counters)
-enum : uint32_t { INSTR_ON = 1u, INSTR_LAST = 2u, INSTR_CTR = 4u };
+enum : uint32_t { INSTR_ON = 1u, INSTR_LAST = 2u, INSTR_CTR = 4u, INSTR_RELAXED = 8u };
 
 struct InstrArgs {
   Rec* ring;          // device-visible pointer to the pinned, mapped ring

@@ -152,6 +152,8 @@ struct FakeBackend : Backend {
   }
   // naive mode is a CUDA-only baseline; on the fake device jobs finish at once
   void record_event(uint32_t, void** ev) override { *ev = nullptr; }
+  void record_existing(uint32_t, void*) override {}
+  void wait_event(uint32_t, void*) override {}
   bool event_done(void*) override { return true; }
   void release_event(void*) override {}
 };
@@ -351,6 +353,8 @@ struct CudaBackend : Backend {
     cudaEventRecord(e, streams[stream]);
     *ev = e;
   }
+  void record_existing(uint32_t stream, void* ev) override { cudaEventRecord((cudaEvent_t)ev, streams[stream]); }
+  void wait_event(uint32_t stream, void* ev) override { cudaStreamWaitEvent(streams[stream], (cudaEvent_t)ev, 0); }
   bool event_done(void* ev) override { return cudaEventQuery((cudaEvent_t)ev) == cudaSuccess; }
   void release_event(void* ev) override { cudaEventDestroy((cudaEvent_t)ev); }
   void sync() override {
@@ -383,6 +387,7 @@ static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last, bool
     ia.base = g->ctr_mbase[slot];
     g->ctr_mbase[slot] += grid;
     ia.flags |= INSTR_CTR;
+    if (!last) ia.flags |= INSTR_RELAXED;   // the job's data dependency is carried by streams
     g->ctr_live.push_back(Gpu::CtrLive{uid, slot, ia.base, grid, 0, 0});
     return ia;
   }
@@ -413,9 +418,14 @@ static void launcher_main(Gpu* g, Launcher* L) {
       void* args[3] = {(void*)&d->a, (void*)&d->ia, (void*)d->tmap};
       cudaError_t e = cuda_launch(cb->fn(d->k->kind, d->dtype, d->instr != 0), *d->k, args, cb->streams[d->stream], cb->pdl);
       if (e != cudaSuccess) g->launch_err.store((int)e);
-    } else {
+    } else if (d->kind == 1) {
       cudaEventRecord((cudaEvent_t)d->event, cb->streams[d->stream]);
       __atomic_store_n(d->recorded, (uint8_t)1, __ATOMIC_RELEASE);
+    } else {
+      // the record is on another launcher's stream: it must have been issued first
+      while (!__atomic_load_n(d->recorded, __ATOMIC_ACQUIRE)) {
+      }
+      cudaStreamWaitEvent(cb->streams[d->stream], (cudaEvent_t)d->event, 0);
     }
     L->q.pop();
   }
@@ -592,6 +602,33 @@ static uint32_t drain_ring(Gpu* g) {
   return n;
 }
 
+// Counter mode, relaxed exits: a launch of a live job completed; if that left the job
+// with nothing in flight, the policy released its stream -> record the release event
+// there (in stream order right after the job's kernels)
+static void maybe_release(Gpu* g, uint32_t uid) {
+  const PolicyLaunch& pl = g->policy->launch(uid);
+  const PolicyJob& pj = g->policy->job(pl.job);
+  if (pj.stream >= 0) return;   // still in flight (launch-ahead): stream order holds
+  JobRec& j = g->jobs[pl.job];
+  const uint32_t s = pl.stream;
+  j.rel_stream = (int32_t)s;
+  g->stats.rel_events++;
+  if (!g->launchers.empty()) {
+    if (!j.rel_ev) cudaEventCreateWithFlags((cudaEvent_t*)&j.rel_ev, cudaEventDisableTiming);
+    __atomic_store_n(&j.rel_recorded, (uint8_t)0, __ATOMIC_RELAXED);
+    LaunchDesc d{};
+    d.event = j.rel_ev;
+    d.recorded = &j.rel_recorded;
+    d.stream = s;
+    d.kind = 1;
+    launcher_push(g, d);
+  } else {
+    if (!j.rel_ev) g->be->record_event(s, &j.rel_ev);
+    else g->be->record_existing(s, j.rel_ev);
+    j.rel_recorded = 1;
+  }
+}
+
 // Counter mode: turn the progress of every in-flight launch's mirrored {start, end}
 // counters into the group-of-G records the ring would carry (group g of a launch
 // covers counts (gG, min((g+1)G, grid)] and is reported once all of them are in;
@@ -620,8 +657,11 @@ static uint32_t drain_counters(Gpu* g) {
         g->stats.records++;
         logev(g, EV_RECORD, type, L.uid, cnt_g, ((uint64_t)grp << 40) | (0xFFull << 56));
         int64_t done = -1;
-        g->policy->record(type, L.uid, cnt_g, &done);
-        if (done >= 0) finish_job(g, (uint32_t)done, 0);
+        const bool complete = g->policy->record(type, L.uid, cnt_g, &done);
+        if (done >= 0)
+          finish_job(g, (uint32_t)done, 0);
+        else if (complete)
+          maybe_release(g, L.uid);
       }
       if (t == 1 && L.f == L.grid) finished = true;
     }
@@ -650,6 +690,22 @@ static void decide_and_launch(Gpu* g) {
     JobRec& j = g->jobs[is.job];
     Model* m = g->P->models[j.model].get();
     logev(g, EV_ISSUE, is.stream, is.uid, is.job, is.layer);
+    if (j.rel_stream >= 0) {
+      if ((uint32_t)j.rel_stream != is.stream) {   // moved: wait for the previous stream's release
+        g->stats.xstream_waits++;
+        if (!g->launchers.empty()) {
+          LaunchDesc d{};
+          d.event = j.rel_ev;
+          d.recorded = &j.rel_recorded;
+          d.stream = is.stream;
+          d.kind = 2;
+          launcher_push(g, d);
+        } else {
+          g->be->wait_event(is.stream, j.rel_ev);
+        }
+      }
+      j.rel_stream = -1;
+    }
     do_launch(g, m, j.slot, is.layer, is.uid, is.stream, g->P->cfg.instrument != 0);
     g->stats.launches++;
   }
@@ -1241,6 +1297,8 @@ static void iso_launch(Gpu* g, Model* m, uint32_t l, bool instr) {
   ia.uid = uid;
   ia.group = g->P->cfg.group_size;
   ia.flags = INSTR_ON | (l + 1 == m->kernels.size() ? INSTR_LAST : 0);
+  if (static_cast<CudaBackend*>(g->be.get())->mirror)   // as in serving
+    ia.flags |= INSTR_CTR | (l + 1 == m->kernels.size() ? 0u : INSTR_RELAXED);
   uint32_t iso_slot = (uint32_t)m->gpu[g->index].args.size() - 1;
   auto* cb = static_cast<CudaBackend*>(g->be.get());
   const void* tm = is_tc(k.kind) ? m->gpu[g->index].tmaps[l].b : nullptr;
@@ -1530,7 +1588,8 @@ static InstrArgs iso_instr(Gpu* g, uint32_t grid, uint32_t group, bool last) {
   ia.uid = uid;
   ia.group = group;
   ia.flags = INSTR_ON | (last ? INSTR_LAST : 0);
-  if (static_cast<CudaBackend*>(g->be.get())->mirror) ia.flags |= INSTR_CTR;   // as in serving
+  if (static_cast<CudaBackend*>(g->be.get())->mirror)   // as in serving
+    ia.flags |= INSTR_CTR | (last ? 0u : INSTR_RELAXED);
   return ia;
 }
 

@@ -83,6 +83,13 @@ struct JobRec {
   uint32_t stream = 0;
   void* event = nullptr;
   uint8_t event_recorded = 0;  // set by the launcher thread (__atomic builtins)
+  // counter mode, relaxed exits: when the job's in-flight kernels have
+  // all completed and the policy released its stream, an event is recorded on that
+  // stream; if the job's next kernel is issued on another stream, that stream waits
+  // for the event (stream order carries the data dependency, reading C2-Q19)
+  void* rel_ev = nullptr;
+  uint8_t rel_recorded = 0;
+  int32_t rel_stream = -1;
 };
 
 struct Paella;
@@ -96,7 +103,7 @@ struct LaunchDesc {
   void* event;                 // kind 1: record this event on the stream
   uint8_t* recorded;
   uint32_t stream, dtype;
-  uint8_t instr, kind;         // kind 0 = kernel, 1 = event record
+  uint8_t instr, kind;         // kind 0 = kernel, 1 = event record, 2 = wait for a recorded event
 };
 
 // plain (in-process) single-producer / single-consumer queue
@@ -144,6 +151,8 @@ struct Backend {
   virtual void* ring_dev() = 0;
   // naive mode completion detection
   virtual void record_event(uint32_t stream, void** ev) = 0;
+  virtual void record_existing(uint32_t stream, void* ev) = 0;   // re-record a created event
+  virtual void wait_event(uint32_t stream, void* ev) = 0;
   virtual bool event_done(void* ev) = 0;
   virtual void release_event(void* ev) = 0;
   virtual void sync() {}

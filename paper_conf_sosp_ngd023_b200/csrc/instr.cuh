@@ -100,6 +100,8 @@ __device__ __forceinline__ void instr_exit(const InstrArgs& ia) {
       // retires at once.  System scope for a job's last kernel (output in host memory).
       if (ia.flags & INSTR_LAST)
         asm volatile("red.release.sys.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+      else if (ia.flags & INSTR_RELAXED)   // data dependencies ride on stream order
+        asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
       else
         asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
     } else if (threadIdx.x == T && threadIdx.y == 0 && threadIdx.z == 0) {
