@@ -185,6 +185,12 @@ static cudaError_t cuda_launch(KernelFn fn, const KernelInst& k, void** args, cu
     at[n].val.clusterDim.y = 1;
     at[n].val.clusterDim.z = k.proto.ksplit;
     ++n;
+  } else if (k.kind == KIND_GAPFC) {
+    at[n].id = cudaLaunchAttributeClusterDimension;
+    at[n].val.clusterDim.x = GAPFC_CLUSTER;
+    at[n].val.clusterDim.y = 1;
+    at[n].val.clusterDim.z = 1;
+    ++n;
   }
   if (pdl) {
     at[n].id = cudaLaunchAttributeProgrammaticStreamSerialization;

@@ -34,6 +34,7 @@ constexpr uint32_t TC_BM = 128;       // Cout rows per CTA (UMMA M, TMEM lanes)
 constexpr uint32_t TC_BN = 64;        // output pixels per CTA (UMMA N)
 constexpr uint32_t TC_BK = 64;        // K per pipeline stage (128 B of bf16 = one swizzle row)
 constexpr uint32_t TC_STAGES = 4;
+constexpr uint32_t GAPFC_CLUSTER = 8;   // fused GAP+FC head: CTAs per cluster (pooling split)
 constexpr uint32_t TC_THREADS = 192;    // 4 producer/epilogue warps + 1 MMA warp + 1 bookkeeping warp
 uint32_t tc_smem_bytes();
 

@@ -62,12 +62,35 @@ __global__ void __launch_bounds__(256) k_ingest(const __grid_constant__ LayerArg
   const float* in = static_cast<const float*>(a.in);
   T* out = static_cast<T*>(a.out);
   uint32_t hw = a.h * a.w_;
-  uint32_t p = blockIdx.x * blockDim.x + threadIdx.x;
-  if (p < hw) {
-    float v[8];
+  if ((hw & 3) == 0 && (reinterpret_cast<uintptr_t>(in) & 15) == 0) {
+    // 4 consecutive pixels per thread: one 16-byte read per channel plane (fewer,
+    // larger PCIe read requests), four 16-byte NHWC stores
+    const uint32_t p = 4 * (blockIdx.x * blockDim.x + threadIdx.x);
+    if (p < hw) {
+      float4 q[8];
 #pragma unroll
-    for (int c = 0; c < 8; ++c) v[c] = (c < (int)a.cin) ? __ldcs(in + (size_t)c * hw + p) : 0.f;
-    store8(out + (size_t)p * a.out_cs + a.out_co, v);
+      for (int c = 0; c < 8; ++c)
+        q[c] = (c < (int)a.cin) ? __ldcs(reinterpret_cast<const float4*>(in + (size_t)c * hw + p))
+                                : make_float4(0.f, 0.f, 0.f, 0.f);
+      float v[4][8];
+#pragma unroll
+      for (int c = 0; c < 8; ++c) {
+        v[0][c] = q[c].x;
+        v[1][c] = q[c].y;
+        v[2][c] = q[c].z;
+        v[3][c] = q[c].w;
+      }
+#pragma unroll
+      for (int i = 0; i < 4; ++i) store8(out + (size_t)(p + i) * a.out_cs + a.out_co, v[i]);
+    }
+  } else {
+    uint32_t p = blockIdx.x * blockDim.x + threadIdx.x;
+    for (; p < hw; p += gridDim.x * blockDim.x) {
+      float v[8];
+#pragma unroll
+      for (int c = 0; c < 8; ++c) v[c] = (c < (int)a.cin) ? __ldcs(in + (size_t)c * hw + p) : 0.f;
+      store8(out + (size_t)p * a.out_cs + a.out_co, v);
+    }
   }
   instr_exit<INSTR>(ia);
 }
@@ -341,7 +364,7 @@ __global__ void __launch_bounds__(256) k_gap(const __grid_constant__ LayerArgs a
   const T* X = static_cast<const T*>(a.in);
   uint32_t ng = a.cout / 8;
   uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
-  uint32_t g = tid / 8, l = tid % 8;
+  uint32_t g = tid / 32, l = tid % 32;   // a warp per 8-channel granule
   float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   const uint32_t HW = a.h * a.w_;
   if (g < ng) {
@@ -355,7 +378,7 @@ __global__ void __launch_bounds__(256) k_gap(const __grid_constant__ LayerArgs a
       }
     }
 #pragma unroll 4
-    for (uint32_t p = l; p < HW; p += 8) {
+    for (uint32_t p = l; p < HW; p += 32) {
       float xv[8];
       load8(X + (size_t)p * a.in_cs + a.in_co + c, xv);
       if (a.flags & LF_PROLOGUE) {
@@ -367,7 +390,7 @@ __global__ void __launch_bounds__(256) k_gap(const __grid_constant__ LayerArgs a
     }
   }
 #pragma unroll
-  for (int o = 4; o > 0; o >>= 1)
+  for (int o = 16; o > 0; o >>= 1)
 #pragma unroll
     for (int i = 0; i < 8; ++i) acc[i] += __shfl_xor_sync(0xffffffffu, acc[i], o);
   if (g < ng && l == 0) {
@@ -433,19 +456,28 @@ __global__ void __launch_bounds__(256) k_fc(const __grid_constant__ LayerArgs a,
 template <typename T, bool INSTR>
 __global__ void __launch_bounds__(256) k_gapfc(const __grid_constant__ LayerArgs a,
                                                const __grid_constant__ InstrArgs ia) {
+  // Batch-1 latency layout: clusters of GAPFC_CLUSTER CTAs; the CTAs of a cluster
+  // pool 1/GAPFC_CLUSTER of the channels each, exchange the pooled slices over DSMEM,
+  // then every warp computes one FC row (8 rows per CTA, ~128 CTAs for 1000 classes:
+  // the weight stream is spread over many SMs).
   kernel_begin<INSTR>(ia);
-  extern __shared__ float pooled[];   // [C]
+  extern __shared__ float pooled[];   // [C], every CTA ends up with all of it
   const T* X = static_cast<const T*>(a.in);
   const T* W = static_cast<const T*>(a.w);
-  const uint32_t C = a.cin, HW = a.h * a.w_;
+  const uint32_t C = a.cin, HW = a.h * a.w_, NG = C / 8;
   const float inv = 1.f / (float)HW;
-  // 8 threads per 8-channel granule split the pixels; shuffle-reduce within the 8
-  const uint32_t l8 = threadIdx.x % 8;
-  for (uint32_t g0 = 0; g0 < C / 8; g0 += blockDim.x / 8) {
-    const uint32_t g = g0 + threadIdx.x / 8;
+  uint32_t rank;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
+  const uint32_t per = (NG + GAPFC_CLUSTER - 1) / GAPFC_CLUSTER;   // granules per CTA
+  const uint32_t g0 = rank * per, g1 = min(NG, g0 + per);
+  uint32_t tpg = 32;
+  while (tpg > 1 && per * tpg > blockDim.x) tpg >>= 1;
+  const uint32_t sub = threadIdx.x % tpg, gpb = blockDim.x / tpg;
+  for (uint32_t gi = threadIdx.x / tpg; gi < (per + gpb - 1) / gpb * gpb; gi += gpb) {
+    const uint32_t g = g0 + gi;
     float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-    if (g < C / 8) {
-      const int c = g * 8;
+    if (g < g1) {
+      const uint32_t c = g * 8;
       float sc[8], sh[8];
       if (a.flags & LF_PROLOGUE) {
 #pragma unroll
@@ -454,10 +486,11 @@ __global__ void __launch_bounds__(256) k_gapfc(const __grid_constant__ LayerArgs
           sh[i] = a.pro_shift[c + i];
         }
       }
+      const T* xp = X + a.in_co + c;
 #pragma unroll 4
-      for (uint32_t p = l8; p < HW; p += 8) {
+      for (uint32_t p = sub; p < HW; p += tpg) {
         float xv[8];
-        load8(X + (size_t)p * a.in_cs + a.in_co + c, xv);
+        load8(xp + (size_t)p * a.in_cs, xv);
         if (a.flags & LF_PROLOGUE) {
 #pragma unroll
           for (int i = 0; i < 8; ++i) xv[i] = fmaxf(fmaf(sc[i], xv[i], sh[i]), 0.f);
@@ -466,40 +499,57 @@ __global__ void __launch_bounds__(256) k_gapfc(const __grid_constant__ LayerArgs
         for (int i = 0; i < 8; ++i) acc[i] += xv[i];
       }
     }
-#pragma unroll
-    for (int o = 4; o > 0; o >>= 1)
+    for (uint32_t o = tpg / 2; o > 0; o >>= 1)
 #pragma unroll
       for (int i = 0; i < 8; ++i) acc[i] += __shfl_xor_sync(0xffffffffu, acc[i], o);
-    if (g < C / 8 && l8 == 0) {
+    if (g < g1 && sub == 0) {
 #pragma unroll
       for (int i = 0; i < 8; ++i) pooled[g * 8 + i] = acc[i] * inv;
     }
   }
+  // publish the slice to the cluster (restricted release: MEMBAR.CTA), then gather the
+  // peers' slices (16-byte DSMEM loads) into the local copy
+  asm volatile(
+      "fence.release.sync_restrict::shared::cta.cluster;\n\t"
+      "barrier.cluster.arrive.relaxed.aligned;\n\tbarrier.cluster.wait.aligned;" ::: "memory");
+  const uint32_t base = (uint32_t)__cvta_generic_to_shared(pooled);
+  for (uint32_t q = threadIdx.x; q < C / 4; q += blockDim.x) {
+    const uint32_t owner = (q * 4 / 8) / per;
+    if (owner == rank) continue;
+    uint32_t peer;
+    float4 v;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(peer) : "r"(base + q * 16), "r"(owner));
+    asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
+                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+                 : "r"(peer));
+    reinterpret_cast<float4*>(pooled)[q] = v;
+  }
+  // done reading the peers; the matching wait (peers stay resident) is at the end
+  asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
   __syncthreads();
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int row = blockIdx.x * (blockDim.x / 32) + warp;
+  if (row < (int)a.cout) {
+    const T* wr = W + (size_t)row * a.kpad;
+    float acc = 0.f;
+#pragma unroll 8
+    for (uint32_t k = lane * 8; k < C; k += 32 * 8) {
+      float wv[8];
+      load8(wr + k, wv);
 #pragma unroll
-  for (int rr = 0; rr < 4; ++rr) {
-    const int row = blockIdx.x * 32 + warp * 4 + rr;
-    if (row < (int)a.cout) {
-      const T* wr = W + (size_t)row * a.kpad;
-      float acc = 0.f;
-      for (uint32_t k = lane * 8; k < C; k += 32 * 8) {
-        float wv[8];
-        load8(wr + k, wv);
+      for (int i = 0; i < 8; ++i) acc = fmaf(wv[i], pooled[k + i], acc);
+    }
 #pragma unroll
-        for (int i = 0; i < 8; ++i) acc = fmaf(wv[i], pooled[k + i], acc);
-      }
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-      if (lane == 0) {
-        float v = act_f(acc + a.bias[row], a.act);
-        if (a.flags & LF_FINAL)
-          static_cast<float*>(a.out)[row] = v;
-        else
-          static_cast<T*>(a.out)[a.out_co + row] = (T)v;
-      }
+    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (lane == 0) {
+      float v = act_f(acc + a.bias[row], a.act);
+      if (a.flags & LF_FINAL)
+        static_cast<float*>(a.out)[row] = v;
+      else
+        static_cast<T*>(a.out)[a.out_co + row] = (T)v;
     }
   }
+  asm volatile("barrier.cluster.wait.aligned;" ::: "memory");
   instr_exit<INSTR>(ia);
 }
 

@@ -156,7 +156,7 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
     a.ow = in.w;
     a.out_cs = 8;
     a.out_co = 0;
-    k.grid[0] = (in.h * in.w + 255) / 256;
+    k.grid[0] = (in.h * in.w % 4 == 0) ? (in.h * in.w / 4 + 255) / 256 : (in.h * in.w + 255) / 256;
     k.block = 256;
     k.bytes = (uint64_t)in.c * in.h * in.w * 4 + (uint64_t)8 * in.h * in.w * es;
     m->kernels.push_back(k);
@@ -333,7 +333,7 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
       case PAELLA_OP_GAP: {
         k.kind = KIND_GAP;
         if (nd.c != sn.c || sn.c % 8) return -EINVAL;
-        k.grid[0] = (nd.c + 255) / 256;   // 8 threads per 8-channel granule
+        k.grid[0] = (nd.c / 8 * 32 + 255) / 256;   // a warp per 8-channel granule
         k.block = 256;
         k.bytes = (uint64_t)sn.h * sn.w * sn.c * es + (uint64_t)nd.c * ((a.flags & LF_FINAL) ? 4 : es);
         break;
@@ -370,7 +370,8 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
           std::vector<float> bias(nd.c, 0.f);
           if (nd.bias) std::memcpy(bias.data(), nd.bias, nd.c * 4);
           k.b_off = blob.put(bias.data(), nd.c * 4);
-          k.grid[0] = (nd.c + 31) / 32;
+          // one FC row per warp, 8 warps per CTA, whole clusters of GAPFC_CLUSTER CTAs
+          k.grid[0] = ((nd.c + 7) / 8 + GAPFC_CLUSTER - 1) / GAPFC_CLUSTER * GAPFC_CLUSTER;
           k.block = 256;
           k.smem = gn.c * 4;
           k.flops = 2ull * nd.c * gn.c + (uint64_t)gn.c * gin.h * gin.w;
