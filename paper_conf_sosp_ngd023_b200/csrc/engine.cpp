@@ -1402,6 +1402,85 @@ static int iso_run(Gpu* g, Model* m, const void* input, void* output, int64_t* k
   return 0;
 }
 
+static volatile uint32_t* gate_ptr(Gpu* g, const volatile uint32_t** dev);
+static void launch_gate(Gpu* g, const volatile uint32_t* gd);
+static InstrArgs iso_instr(Gpu* g, uint32_t grid, uint32_t group, bool last);
+
+// Device time of kernel l: `reps` back-to-back launches of it (PDL, as served) behind a
+// gate on the profiling stream, timed with CUDA events; ns per launch, -1 on error.
+static int64_t time_layer(Gpu* g, Model* m, uint32_t l, bool instr, uint32_t reps) {
+  cudaSetDevice(g->device);
+  cudaStream_t s = (cudaStream_t)g->prof_stream;
+  auto* cb = static_cast<CudaBackend*>(g->be.get());
+  const uint32_t iso_slot = (uint32_t)m->gpu[g->index].args.size() - 1;
+  const KernelInst& k = m->kernels[l];
+  reps = std::min(reps, 256u);
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  const volatile uint32_t* gd;
+  volatile uint32_t* gate = gate_ptr(g, &gd);
+  *gate = 0;
+  launch_gate(g, gd);
+  cudaEventRecord(e0, s);
+  const void* tm = is_tc(k.kind) ? m->gpu[g->index].tmaps[l].b : nullptr;
+  for (uint32_t r = 0; r < reps; ++r) {
+    InstrArgs ia = iso_instr(g, k.grid_total(), g->P->cfg.group_size, l + 1 == m->kernels.size());
+    void* args[3] = {(void*)&m->gpu[g->index].args[iso_slot][l], (void*)&ia, (void*)tm};
+    cuda_launch(cb->fn(k.kind, m->dtype, instr), k, args, s, cb->pdl);
+  }
+  cudaEventRecord(e1, s);
+  std::atomic_thread_fence(std::memory_order_seq_cst);
+  *gate = 1;
+  int64_t ns = -1;
+  if (cudaStreamSynchronize(s) == cudaSuccess) {
+    float ms = 0;
+    cudaEventElapsedTime(&ms, e0, e1);
+    ns = (int64_t)((double)ms * 1e6 / reps);
+  }
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  return ns;
+}
+
+// Split-K autotuning of the tcgen05 convs (GPU 0, at registration, before T-bar is
+// profiled): every admissible split (power of two, <= 16 = the cluster limit, >= 1
+// k-block per split, <= one wave at 2 CTAs/SM) is timed as served (instrumented, PDL
+// chain); a larger split must win by >= 5 % (it occupies more SMs under load).
+static int autotune_splits(Gpu* g, Model* m) {
+  if (std::getenv("PAELLA_NO_AUTOTUNE") || std::getenv("PAELLA_NOSPLIT")) return 0;
+  if (iso_run(g, m, nullptr, nullptr, nullptr, true)) return -EIO;
+  auto& mg = m->gpu[g->index];
+  for (uint32_t l = 0; l < m->kernels.size(); ++l) {
+    KernelInst& k = m->kernels[l];
+    if (!is_tc(k.kind)) continue;
+    const uint32_t nk = k.proto.kpad / TC_BK, tiles = k.proto.tiles_m * k.proto.tiles_n;
+    auto set = [&](uint32_t sp) {
+      k.proto.ksplit = sp;
+      k.grid[2] = sp;
+      for (auto& A : mg.args) A[l].ksplit = sp;
+    };
+    const uint32_t orig = k.proto.ksplit;
+    uint32_t best = orig;
+    int64_t best_t = INT64_MAX;
+    for (uint32_t sp = 1; sp <= 16 && sp <= nk && tiles * sp <= 2 * g->P->sms; sp *= 2) {
+      set(sp);
+      time_layer(g, m, l, true, 8);   // warm
+      const int64_t t = time_layer(g, m, l, true, 40);
+      if (t < 0) return -EIO;
+      if (best_t == INT64_MAX || t * 100 < best_t * 95) {
+        best_t = t;
+        best = sp;
+      }
+    }
+    set(best);
+    if (std::getenv("PAELLA_AUTOTUNE_LOG"))
+      fprintf(stderr, "autotune %s layer %u: nk %u tiles %u split %u -> %u (%lld ns)\n", m->name.c_str(), l, nk,
+              tiles, orig, best, (long long)best_t);
+  }
+  return 0;
+}
+
 static int setup_model_gpu(Paella* P, Model* m, Gpu* g) {
   ModelGpu& mg = m->gpu[g->index];
   const uint32_t slots = P->cfg.max_jobs_per_model;
@@ -1499,6 +1578,7 @@ static int setup_model_gpu(Paella* P, Model* m, Gpu* g) {
   // profile T-bar (P1249-1254; reading C2-Q15): GPU 0 measures, others copy
   if (g->index == 0) {
     uint32_t runs = 20;
+    if (cuda && autotune_splits(g, m)) return -EIO;
     if (cuda) {
       std::vector<int64_t> t(m->kernels.size()), acc(m->kernels.size(), 0);
       for (int w = 0; w < 5; ++w)
@@ -1613,36 +1693,10 @@ int paella_time_kernels(paella_t* p, uint32_t gpu, uint32_t model_id, uint32_t i
   Model* m = P->models[model_id].get();
   int rc = iso_run(g, m, nullptr, nullptr, nullptr, true);   // materialise valid activations
   if (rc) return rc;
-  cudaSetDevice(g->device);
-  cudaStream_t s = (cudaStream_t)g->prof_stream;
-  auto* cb = static_cast<CudaBackend*>(g->be.get());
-  uint32_t iso_slot = (uint32_t)m->gpu[gpu].args.size() - 1;
-  cudaEvent_t e0, e1;
-  cudaEventCreate(&e0);
-  cudaEventCreate(&e1);
   for (uint32_t l = 0; l < m->kernels.size(); ++l) {
-    const KernelInst& k = m->kernels[l];
-    const volatile uint32_t* gd;
-    volatile uint32_t* gate = gate_ptr(g, &gd);
-    *gate = 0;
-    launch_gate(g, gd);
-    cudaEventRecord(e0, s);
-    const void* tm = is_tc(k.kind) ? m->gpu[gpu].tmaps[l].b : nullptr;
-    for (uint32_t r = 0; r < std::min(reps, 256u); ++r) {
-      InstrArgs ia = iso_instr(g, k.grid_total(), P->cfg.group_size, l + 1 == m->kernels.size());
-      void* args[3] = {(void*)&m->gpu[gpu].args[iso_slot][l], (void*)&ia, (void*)tm};
-      cuda_launch(cb->fn(k.kind, m->dtype, instrumented != 0), k, args, s, cb->pdl);
-    }
-    cudaEventRecord(e1, s);
-    std::atomic_thread_fence(std::memory_order_seq_cst);
-    *gate = 1;
-    if (cudaStreamSynchronize(s) != cudaSuccess) return -EIO;
-    float ms = 0;
-    cudaEventElapsedTime(&ms, e0, e1);
-    kernel_ns[l] = (int64_t)((double)ms * 1e6 / std::min(reps, 256u));
+    kernel_ns[l] = time_layer(g, m, l, instrumented != 0, reps);
+    if (kernel_ns[l] < 0) return -EIO;
   }
-  cudaEventDestroy(e0);
-  cudaEventDestroy(e1);
   return 0;
 }
 

@@ -298,31 +298,15 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       const bool ok = kv && (uint32_t)(ih0[j] + kr) < a.h && (uint32_t)(iw0[j] + ks_) < a.w_;
       const __nv_bfloat16* src = ok ? X + (off0[j] + dk) : X;
       const uint32_t dst = bstage + j * 2048;   // pixel row n = t/8 + 16 j
-      if constexpr (!PRO) {
-        cp_async16(dst, src, ok ? 16u : 0u);
-      } else {
-        // DenseNet pre-activation: relu(scale[c] * x + shift[c]) through registers;
-        // padding stays zero (it pads the activated tensor)
-        uint4 u = make_uint4(0, 0, 0, 0);
-        if (ok) {
-          u = __ldg(reinterpret_cast<const uint4*>(src));
-          const float4 s0 = __ldg(reinterpret_cast<const float4*>(a.pro_scale + kci));
-          const float4 s1 = __ldg(reinterpret_cast<const float4*>(a.pro_scale + kci + 4));
-          const float4 z0 = __ldg(reinterpret_cast<const float4*>(a.pro_shift + kci));
-          const float4 z1 = __ldg(reinterpret_cast<const float4*>(a.pro_shift + kci + 4));
-          const float sc[8] = {s0.x, s0.y, s0.z, s0.w, s1.x, s1.y, s1.z, s1.w};
-          const float sh[8] = {z0.x, z0.y, z0.z, z0.w, z1.x, z1.y, z1.z, z1.w};
-          __nv_bfloat162* h = reinterpret_cast<__nv_bfloat162*>(&u);
-#pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            float2 f = __bfloat1622float2(h[i]);
-            h[i] = __floats2bfloat162_rn(fmaxf(fmaf(sc[2 * i], f.x, sh[2 * i]), 0.f),
-                                         fmaxf(fmaf(sc[2 * i + 1], f.y, sh[2 * i + 1]), 0.f));
-          }
-        }
-        asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(dst), "r"(u.x), "r"(u.y), "r"(u.z),
-                     "r"(u.w)
-                     : "memory");
+      cp_async16(dst, src, ok ? 16u : 0u);
+    }
+    if constexpr (PRO) {
+      // DenseNet pre-activation: the raw tile lands by cp.async like the plain path;
+      // transform_B applies relu(scale * x + shift) in place once it has landed.  Warm
+      // L1 with this chunk's prologue vectors meanwhile.
+      if (kv) {
+        asm volatile("prefetch.global.L1 [%0];" ::"l"(a.pro_scale + kci));
+        asm volatile("prefetch.global.L1 [%0];" ::"l"(a.pro_shift + kci));
       }
     }
     if constexpr (!PRO) {
@@ -339,6 +323,50 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       if (++ks_ == (int)a.kw) {
         ks_ = 0;
         ++kr;
+      }
+    }
+  };
+  // PRO: the transform cursor (r, s, ci, k) trails the issue cursor by the stages in flight
+  int tr_r = 0, tr_s = 0, tr_ci = 0;
+  uint32_t tr_k = 0;
+  auto transform_B = [&](uint32_t it) {
+    const uint32_t bstage = su32(sB + (it % TC_STAGES) * B_BYTES) + dst0;
+    if (tr_k < K) {
+      const float4 s0 = __ldg(reinterpret_cast<const float4*>(a.pro_scale + tr_ci));
+      const float4 s1 = __ldg(reinterpret_cast<const float4*>(a.pro_scale + tr_ci + 4));
+      const float4 z0 = __ldg(reinterpret_cast<const float4*>(a.pro_shift + tr_ci));
+      const float4 z1 = __ldg(reinterpret_cast<const float4*>(a.pro_shift + tr_ci + 4));
+      const float sc[8] = {s0.x, s0.y, s0.z, s0.w, s1.x, s1.y, s1.z, s1.w};
+      const float sh[8] = {z0.x, z0.y, z0.z, z0.w, z1.x, z1.y, z1.z, z1.w};
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        // padding and empty pixels stay zero (padding pads the activated tensor)
+        if ((uint32_t)(ih0[j] + tr_r) < a.h && (uint32_t)(iw0[j] + tr_s) < a.w_) {
+          const uint32_t adr = bstage + j * 2048;
+          uint4 u;
+          asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
+                       : "=r"(u.x), "=r"(u.y), "=r"(u.z), "=r"(u.w)
+                       : "r"(adr));
+          __nv_bfloat162* h = reinterpret_cast<__nv_bfloat162*>(&u);
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const float2 f = __bfloat1622float2(h[i]);
+            h[i] = __floats2bfloat162_rn(fmaxf(fmaf(sc[2 * i], f.x, sh[2 * i]), 0.f),
+                                         fmaxf(fmaf(sc[2 * i + 1], f.y, sh[2 * i + 1]), 0.f));
+          }
+          asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(adr), "r"(u.x), "r"(u.y), "r"(u.z),
+                       "r"(u.w)
+                       : "memory");
+        }
+      }
+    }
+    tr_k += TC_BK;
+    tr_ci += TC_BK;
+    while (tr_ci >= (int)a.cin) {
+      tr_ci -= (int)a.cin;
+      if (++tr_s == (int)a.kw) {
+        tr_s = 0;
+        ++tr_r;
       }
     }
   };
@@ -359,6 +387,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       const int rs = (int)(k0 / a.cin);
       ks_ = rs % (int)a.kw;
       kr = rs / (int)a.kw;
+      tr_k = kcur, tr_ci = kci, tr_s = ks_, tr_r = kr;
     }
     if (a.a_rows < TC_BM) {
       const uint32_t zb = A_BYTES - abytes;   // bytes per stage, multiple of 1024
@@ -373,7 +402,10 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     // ... and the first activation gathers, before the CTA-wide barrier, once the
     // predecessor kernel's output is complete (PDL; the weight TMA above needs no wait)
     pdl_wait();
-    for (uint32_t it = 0; it < pre; ++it) issue_B(it, false);   // barriers not initialised yet
+    for (uint32_t it = 0; it < pre; ++it) {   // barriers not initialised yet
+      issue_B(it, false);
+      if constexpr (PRO) cp_async_commit();   // one group per stage
+    }
     if (a.ksplit == 1 && (a.flags & LF_RESIDUAL) && eco < a.cout) {
 #pragma unroll
       for (uint32_t i = 0; i < NIT; ++i) {
@@ -401,8 +433,17 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
         issue_B(nxt, true);
       }
     } else {
-      // prologue path: register-staged stores, then a proxy fence and an arrive
+      // prologue path: wait for this thread's own copies of stage it (cp.async groups,
+      // STAGES in flight), transform them in place, publish to the async proxy, arrive
       for (uint32_t it = 0; it < nkl; ++it) {
+        const uint32_t issued = min(nkl, it + TC_STAGES);
+        switch (issued - it - 1) {
+          case 0: cp_async_wait<0>(); break;
+          case 1: cp_async_wait<1>(); break;
+          case 2: cp_async_wait<2>(); break;
+          default: cp_async_wait<3>(); break;
+        }
+        transform_B(it);
         fence_proxy_async();
         mbar_arrive(&full[it % TC_STAGES]);
         const uint32_t nxt = it + TC_STAGES;
@@ -413,7 +454,8 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
             mbar_arrive_tx(&full[s], abytes);
             tma_load_2d(sA + s * A_BYTES, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
           }
-          issue_B(nxt, true);
+          issue_B(nxt, false);
+          cp_async_commit();
         }
       }
     }

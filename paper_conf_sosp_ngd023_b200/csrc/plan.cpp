@@ -273,8 +273,12 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
             if (!e) {
               // splitting pays only for deep K: a cluster barrier + DSMEM reduction cost ~1 us;
               // clusters of up to 16 CTAs (non-portable size, allowed on sm_100)
-              if (nk >= 12)
-                while (split < 16 && tiles * split * 2 <= P->sms && nk / (split * 2) >= 4) split *= 2;
+              // measured (kernel_times): with the restricted-fence cluster barrier and the
+              // staggered DSMEM reduction, splits down to 2 k-blocks each pay from nk >= 6
+              static const uint32_t min_nk = std::getenv("PAELLA_SPLIT_MIN_NK") ? atoi(std::getenv("PAELLA_SPLIT_MIN_NK")) : 6;
+              static const uint32_t min_st = std::getenv("PAELLA_SPLIT_MIN_STAGES") ? atoi(std::getenv("PAELLA_SPLIT_MIN_STAGES")) : 2;
+              if (nk >= min_nk)
+                while (split < 16 && tiles * split * 2 <= P->sms && nk / (split * 2) >= min_st) split *= 2;
             }
             a.ksplit = split;
             // narrow layers: fetch only the live weight rows (SW128 atoms are 8 rows)

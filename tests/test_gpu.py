@@ -141,9 +141,10 @@ def test_serving_parity_and_replay(tmp_path, policy, group, streams, ring, look,
         _serve_and_check(e, specs, 120, 3, seed=policy * 7 + group)
         st = e.stats()
         assert st["completed"] == 120
-        if notify == "counters":
+        if notify == "counters" and look == 0:
             # relaxed exits: jobs that went idle recorded a release event; moves to another
-            # stream waited for it (the outputs above are checked either way)
+            # stream waited for it (the outputs above are checked either way; with
+            # launch-ahead a job rarely goes idle between its kernels)
             assert st["rel_events"] > 0
             print("release events", st["rel_events"], "cross-stream waits", st["xstream_waits"])
     cfg, ms, events, ex = eventlog.read(log % 0)
