@@ -55,6 +55,7 @@ def parse():
     ap.add_argument("--slack", type=int, default=1184,
                     help="B, blocks issued beyond full utilisation (P1300-1304); 8 x 148 SMs covers the "
                          "measured dispatch loop delay (DESIGN.md B200-Q1)")
+    ap.add_argument("--theta", type=int, default=100, help="fairness threshold (kernel dispatches, P1296-1297)")
     ap.add_argument("--prio-classes", type=int, default=1, help="stream-priority classes (DESIGN.md B200-Q2)")
     ap.add_argument("--launch-threads", type=int, default=4, help="launcher helper threads per GPU")
     ap.add_argument("--sat-reqs", type=int, default=1500, help="requests of the saturation calibration")
@@ -251,6 +252,7 @@ def run_gpu(args, dist):
     def engine(**kw):
         kw.setdefault("launch_threads", 0 if args.fake else args.launch_threads)
         if not kw.get("naive"):
+            kw.setdefault("theta", args.theta)
             kw.setdefault("slack", args.slack)
             kw.setdefault("prio_classes", args.prio_classes)
         e, mids = build_engine(L, specs, gpu, fake=args.fake, region_bytes=region, max_jobs_per_model=128, **kw)
@@ -359,7 +361,7 @@ def run_gpu(args, dist):
                 elapsed=elapsed, completed=completed, jct=jct_stats(jct, models, names), clocks=clk,
                 ev=ev, stats=stats, dev_roof=dev_roof, base=base, e2e_rate=e2e_rate,
                 e2e=jct_stats(e2e_jct, mm, names), h2d=h2d, d2h=d2h, calib_s=calib_s, kinfo=kinfo,
-                slo_at=slo_at)
+                slo_at=slo_at, config=cfgname)
 
 
 def cpu_baseline(cfg, seconds=12.0):
@@ -421,8 +423,16 @@ def roofline_entry(res, peaks):
     flops_per = ev["flops"] / ev["launches"]
     gbs = bytes_per / dur
     peak = peaks.get("hbm_gbs", 6650.0)
+    # DRAM traffic per launch from the committed ncu --set full capture of the same
+    # launches (tools/profile_round.sh -> tools/ncu_traffic.py), if present
+    traffic, tsrc = None, None
+    tp = os.path.join(ROOT, "profiles", f"conv_traffic_{res['config']}.json")
+    if os.path.exists(tp):
+        tj = json.load(open(tp))
+        traffic, tsrc = tj.get("conv_tcgen05_dram_bytes_per_launch"), tj.get("source")
     return {"kernel": "conv_tcgen05", "bound": "hbm", "achieved": round(gbs, 2), "peak": peak, "unit": "GB/s",
-            "frac": round(gbs / peak, 4), "traffic": None, "launches_per_mix": ev["launches"],
+            "frac": round(gbs / peak, 4), "traffic": traffic, "traffic_source": tsrc,
+            "algorithmic_bytes_per_launch": round(bytes_per), "launches_per_mix": ev["launches"],
             "mean_launch_us": round(dur / 1e3, 3), "tflops": round(flops_per / dur / 1e3, 3),
             "share_of_device_time": round(ev["ns"] / max(1, ev["all_ns"]), 3),
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (burst copy)"}
@@ -483,7 +493,7 @@ def main():
         "jct_us": res["jct"], "slo_us": res["slo"],
         "paella_config": {"lookahead": args.lookahead, "launch_threads": args.launch_threads, "policy": "srpt+deficit",
                           "slack_blocks": args.slack, "prio_classes": args.prio_classes, "pdl": True,
-                          "theta": 100, "group": 16, "streams": 32},
+                          "theta": args.theta, "group": 16, "streams": 32},
         "slo_met": bool(all(res["jct"].get(n, {}).get("p99_us", 1e18) <= res["slo"][n] for n in res["names"])),
         "req_s_at_p99_slo": {k: v["req_s"] for k, v in res["slo_at"].items()},
         "slo_ladder": res["slo_at"],

@@ -1447,10 +1447,31 @@ static int64_t time_layer(Gpu* g, Model* m, uint32_t l, bool instr, uint32_t rep
 // profiled): every admissible split (power of two, <= 16 = the cluster limit, >= 1
 // k-block per split, <= one wave at 2 CTAs/SM) is timed as served (instrumented, PDL
 // chain); a larger split must win by >= 5 % (it occupies more SMs under load).
+// PAELLA_SPLITS_FILE: a cache of the choices ("model layer split" lines): read if it
+// exists (profiling runs reuse the served configuration without re-timing), appended to
+// otherwise.
 static int autotune_splits(Gpu* g, Model* m) {
   if (std::getenv("PAELLA_NO_AUTOTUNE") || std::getenv("PAELLA_NOSPLIT")) return 0;
-  if (iso_run(g, m, nullptr, nullptr, nullptr, true)) return -EIO;
   auto& mg = m->gpu[g->index];
+  const char* cache = std::getenv("PAELLA_SPLITS_FILE");
+  if (cache) {
+    if (FILE* f = std::fopen(cache, "r")) {
+      char name[256];
+      unsigned l, sp;
+      bool any = false;
+      while (std::fscanf(f, "%255s %u %u", name, &l, &sp) == 3) {
+        if (m->name != name || l >= m->kernels.size() || !is_tc(m->kernels[l].kind)) continue;
+        KernelInst& k = m->kernels[l];
+        k.proto.ksplit = sp;
+        k.grid[2] = sp;
+        for (auto& A : mg.args) A[l].ksplit = sp;
+        any = true;
+      }
+      std::fclose(f);
+      if (any) return 0;
+    }
+  }
+  if (iso_run(g, m, nullptr, nullptr, nullptr, true)) return -EIO;
   for (uint32_t l = 0; l < m->kernels.size(); ++l) {
     KernelInst& k = m->kernels[l];
     if (!is_tc(k.kind)) continue;
@@ -1474,6 +1495,11 @@ static int autotune_splits(Gpu* g, Model* m) {
       }
     }
     set(best);
+    if (cache)
+      if (FILE* f = std::fopen(cache, "a")) {
+        std::fprintf(f, "%s %u %u\n", m->name.c_str(), l, best);
+        std::fclose(f);
+      }
     if (std::getenv("PAELLA_AUTOTUNE_LOG"))
       fprintf(stderr, "autotune %s layer %u: nk %u tiles %u split %u -> %u (%lld ns)\n", m->name.c_str(), l, nk,
               tiles, orig, best, (long long)best_t);

@@ -44,5 +44,10 @@ with L.Engine(num_clients=1) as e:
         for r in top:
             print(f"     #{r['i']:3d} {r['name']:10s} g={r['grid']:4d} {r['t_plain_ns']/1e3:6.2f} us "
                   f"{r['bytes']/1e6:6.2f} MB {r['flops']/1e9:6.3f} GF")
+# config 5 (BASELINE): per-kernel instrumentation slowdown over every distinct layer
+# kernel of the models above (instrumented as served vs the uninstrumented twin)
+sl = np.array([r["t_instr_ns"] / max(1, r["t_plain_ns"]) - 1.0 for rows in out.values() for r in rows])
+print(f"per-kernel instrumentation slowdown over {len(sl)} kernels: median {np.median(sl)*100:.1f} %, "
+      f"p90 {np.percentile(sl, 90)*100:.1f} %, max {sl.max()*100:.1f} %")
 os.makedirs("gpurun_out", exist_ok=True)
 json.dump({"empty_ns": empty, "models": out}, open("gpurun_out/kernel_times.json", "w"))
