@@ -90,6 +90,30 @@ __device__ __forceinline__ void kernel_begin(const InstrArgs& ia) {
   pdl_trigger();
 }
 
+// exit count of a block whose every other thread is already past a CTA barrier (the
+// caller is the block's last active thread): no second barrier
+template <bool INSTR>
+__device__ __forceinline__ void instr_exit_last_thread(const InstrArgs& ia) {
+  if constexpr (INSTR) {
+    if (ia.flags & INSTR_CTR) {
+      if (ia.flags & INSTR_LAST)
+        asm volatile("red.release.sys.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+      else if (ia.flags & INSTR_RELAXED)
+        asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+      else
+        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+    } else {
+      uint32_t old;
+      if (ia.flags & INSTR_LAST)
+        asm volatile("atom.acq_rel.sys.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(&ia.ctr[1]) : "memory");
+      else
+        asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(&ia.ctr[1]) : "memory");
+      const uint32_t total = gridDim.x * gridDim.y * gridDim.z;
+      maybe_record(ia, REC_COMPLETION, old + 1u - ia.base, total);
+    }
+  }
+}
+
 template <bool INSTR, uint32_t T = 0>
 __device__ __forceinline__ void instr_exit(const InstrArgs& ia) {
   if constexpr (INSTR) {

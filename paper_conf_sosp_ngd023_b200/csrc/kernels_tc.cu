@@ -645,10 +645,12 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   if (warp == 4) {
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tmem_slot), "r"(64u) : "memory");
+    // every other thread is past the barrier above: the MMA warp, last to finish, counts
+    // the block's exit itself (no second block barrier)
+    if (trace && lane == 0) tr[6] = globaltimer();
+    if (lane == 0) instr_exit_last_thread<INSTR>(ia);
+    if (trace && lane == 0) tr[7] = globaltimer();
   }
-  if (trace && threadIdx.x == 0) tr[6] = globaltimer();
-  instr_exit<INSTR, TBOOK>(ia);
-  if (trace && threadIdx.x == TBOOK) tr[7] = globaltimer();
 }
 
 uint32_t tc_smem_bytes() { return 1024 + TC_STAGES * (A_BYTES + B_BYTES) + 128; }
