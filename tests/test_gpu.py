@@ -72,6 +72,28 @@ def test_isolated_fp32_parity(engine, name):
     assert within(out, ref, FP32_TOL).all(), np.abs(out - ref).max()
 
 
+@pytest.mark.parametrize("name", ["resnet18", "densenet121"])
+def test_forced_split_k_parity(engine, name, tmp_path, monkeypatch):
+    """Every cluster split-K factor the autotuner may pick (1..16, DSMEM reduction,
+    including splits with empty k-ranges), forced on every tcgen05 layer through the
+    split cache (PAELLA_SPLITS_FILE), stays within the bf16 tolerance."""
+    g = archs.build(name)
+    P = rng.model_params(g)
+    ref = oracle_out(name, 0, "bf16")
+    for sp in (1, 2, 4, 8, 16):
+        mname = f"{name}-split{sp}"
+        f = tmp_path / f"splits{sp}.txt"
+        f.write_text("".join(f"{mname} {l} {sp}\n" for l in range(len(g.nodes) + 2)))
+        monkeypatch.setenv("PAELLA_SPLITS_FILE", str(f))
+        mid = engine.register_model(g, P, dtype=L.DTYPE_BF16, name=mname)
+        monkeypatch.delenv("PAELLA_SPLITS_FILE")
+        ks = engine.kernels(mid)
+        assert any(k["name"].startswith("conv_tcgen05") and k["grid"] % sp == 0 for k in ks)
+        out = engine.run_isolated(mid, rng.image(g, 0))
+        ok = within(out, ref, BF16_TOL)
+        assert ok.all(), f"{name} split {sp}: max err {np.abs(out - ref).max()}"
+
+
 def _serve_and_check(e, specs, n, n_clients, seed, rate_us=30.0):
     """specs: list of (model id, model name, graph).  Submits n requests with Poisson
     gaps, distinct pooled inputs, checks all outputs against the oracle."""
