@@ -68,6 +68,10 @@ extern "C" {
 
 /* flags */
 #define PAELLA_NONBLOCK 1u      /* submit: -EAGAIN if the ring is full; poll: -EAGAIN if none */
+#define PAELLA_HYBRID   2u      /* poll: hybrid interrupt/poll wait (P1157-1171): spin ~20 us,
+                                   then sleep on a futex until the dispatcher issues the
+                                   LAST kernel of one of this client's jobs (the "almost
+                                   finished" hint) or pushes a completion, then spin again */
 
 /* maximum sizes */
 #define PAELLA_MAX_GPUS    8u
@@ -217,6 +221,7 @@ int64_t paella_submit_at(paella_t* p, uint32_t client_id, uint32_t model_id,
 int64_t paella_poll_completion(paella_t* p, uint32_t client_id, uint32_t flags, int32_t* status);
 /* Returns the req_id of the FIRST available completion of this client (completion
    order, not submission order, P1149).  PAELLA_NONBLOCK: -EAGAIN if none (P1155);
+   PAELLA_HYBRID: spin, then futex sleep between the dispatcher's hints (above);
    otherwise spins until one is available.  *status (if non-NULL): 0 ok, -EIO CUDA
    error on that GPU, -ECANCELED shutdown. */
 

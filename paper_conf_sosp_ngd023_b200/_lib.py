@@ -23,6 +23,7 @@ ROUTE_LEAST_WORK, ROUTE_ROUND_ROBIN = 0, 1
 DEVICE_CUDA, DEVICE_FAKE = 0, 1
 DTYPE_BF16, DTYPE_FP32 = 0, 1
 NONBLOCK = 1
+HYBRID = 2
 OP = {"input": 0, "conv": 1, "maxpool": 2, "avgpool": 3, "gap": 4, "fc": 5, "concat": 6}
 ACT = {"none": 0, "relu": 1, "relu6": 2}
 NODE_PROLOGUE, NODE_CEIL = 1, 2

@@ -26,6 +26,11 @@
 
 #include <cuda_runtime.h>
 
+#include <linux/futex.h>
+#include <sys/syscall.h>
+#include <unistd.h>
+#include <climits>
+
 #include "engine.h"
 
 namespace paella {
@@ -496,6 +501,14 @@ static void harvest_events(Gpu* g) {
   }
 }
 
+// hybrid completion path: bump the client's futex word; a syscall only if it sleeps
+static void wake_client(Paella* P, uint32_t client) {
+  P->wake_seq[client]->fetch_add(1, std::memory_order_release);
+  if (P->sleepers[client]->load(std::memory_order_acquire) != 0)
+    syscall(SYS_futex, reinterpret_cast<uint32_t*>(P->wake_seq[client]), FUTEX_WAKE_PRIVATE, INT32_MAX, nullptr,
+            nullptr, 0);
+}
+
 static void push_completion(Gpu* g, const JobRec& j, int32_t status) {
   CompleteSlot cs{};
   cs.req_id = j.req_id;
@@ -506,6 +519,7 @@ static void push_completion(Gpu* g, const JobRec& j, int32_t status) {
     // completion ring full: the client is not polling; spin (bounded by client)
     if (g->stop.load(std::memory_order_relaxed)) break;
   }
+  wake_client(g->P, j.client);
 }
 
 static void finish_job(Gpu* g, uint32_t jid, int32_t status) {
@@ -714,6 +728,7 @@ static void decide_and_launch(Gpu* g) {
     }
     do_launch(g, m, j.slot, is.layer, is.uid, is.stream, g->P->cfg.instrument != 0);
     g->stats.launches++;
+    if (is.layer + 1 == m->kernels.size()) wake_client(g->P, j.client);   // "almost finished" hint
   }
 }
 
@@ -904,6 +919,8 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     }
     P->region.push_back((uint8_t*)r);
     P->client_seq.push_back(new std::atomic<uint64_t>(0));
+    P->wake_seq.push_back(new std::atomic<uint32_t>(0));
+    P->sleepers.push_back(new std::atomic<uint32_t>(0));
   }
   P->rr_next.assign(cfg.num_clients, 0);
   P->poll_rr.assign(cfg.num_clients, 0);
@@ -1117,6 +1134,7 @@ int64_t paella_poll_completion(paella_t* p, uint32_t client_id, uint32_t flags, 
   Paella* P = (Paella*)p;
   if (!P || client_id >= P->cfg.num_clients) return -EINVAL;
   uint32_t ng = (uint32_t)P->gpus.size();
+  int64_t spin_start = 0;
   for (;;) {
     for (uint32_t k = 0; k < ng; ++k) {
       uint32_t g = (P->poll_rr[client_id] + k) % ng;
@@ -1134,6 +1152,22 @@ int64_t paella_poll_completion(paella_t* p, uint32_t client_id, uint32_t flags, 
     bool alive = false;
     for (auto& g : P->gpus) alive |= g->thread.joinable() && !g->stop.load();
     if (!alive) return -ESHUTDOWN;
+    if (flags & PAELLA_HYBRID) {
+      // spin ~20 us after the last wake-up, then sleep until the next hint/completion
+      const uint32_t seen = P->wake_seq[client_id]->load(std::memory_order_acquire);
+      if (spin_start == 0) spin_start = now_ns();
+      if (now_ns() - spin_start < 20000) continue;
+      P->sleepers[client_id]->fetch_add(1, std::memory_order_acq_rel);
+      bool empty = true;   // re-check after announcing the sleep (no lost wake-up)
+      for (uint32_t k = 0; k < ng && empty; ++k) empty = P->gpus[k]->done[client_id]->peek() == nullptr;
+      if (empty && P->wake_seq[client_id]->load(std::memory_order_acquire) == seen) {
+        timespec ts{0, 2000000};   // 2 ms cap: shutdown and error paths need no wake-up
+        syscall(SYS_futex, reinterpret_cast<uint32_t*>(P->wake_seq[client_id]), FUTEX_WAIT_PRIVATE, seen, &ts,
+                nullptr, 0);
+      }
+      P->sleepers[client_id]->fetch_sub(1, std::memory_order_acq_rel);
+      spin_start = now_ns();
+    }
   }
 }
 
@@ -1192,6 +1226,8 @@ int paella_shutdown(paella_t* p) {
   P->gpus.clear();
   for (size_t i = 0; i < P->shm_maps.size(); ++i) munmap(P->shm_maps[i], P->shm_sizes[i]);
   for (auto* a : P->client_seq) delete a;
+  for (auto* a : P->wake_seq) delete a;
+  for (auto* a : P->sleepers) delete a;
   delete P;
   return 0;
 }

@@ -234,6 +234,11 @@ struct Paella {
   std::vector<std::atomic<uint64_t>*> client_seq;
   std::vector<uint32_t> rr_next;                // per-client round-robin router state
   std::vector<uint32_t> poll_rr;                // per-client completion ring scan start
+  // hybrid completion wait (PAELLA_HYBRID, P1157-1171): per-client futex word bumped by
+  // the dispatchers on the "almost finished" hint and on every completion, and the
+  // number of client threads sleeping on it (no syscall on the dispatcher otherwise)
+  std::vector<std::atomic<uint32_t>*> wake_seq;
+  std::vector<std::atomic<uint32_t>*> sleepers;
   std::atomic<bool> shutting{false};
   int64_t capacity[NRES];
 };

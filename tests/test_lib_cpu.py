@@ -174,3 +174,39 @@ def test_shutdown_cancels_unadmitted():
     for i in range(50):
         assert e.submit(0, mid, i * 16384, need) >= 0
     e.shutdown()
+
+
+def test_hybrid_poll_sleeps_between_hints():
+    """PAELLA_HYBRID (NEXT-3, P1157-1171): a client waiting for sparse completions
+    spins briefly, then sleeps on the futex the dispatcher bumps on the "almost
+    finished" hint and on completion -- every request completes, and the waiting thread
+    uses a small fraction of one core (a spinning poll would use all of it)."""
+    import threading
+    e = _toy_engine(num_clients=1)
+    mid = e.register_model(archs.toy(), rng.model_params(archs.toy()))
+    info = e.model_info(mid)
+    need = info["input_bytes"] + info["output_bytes"]
+    n, gap = 20, 0.01
+    got = []
+
+    def waiter():
+        t0 = time.thread_time()
+        while len(got) < n:
+            rid, st = e.poll(0, L.HYBRID)
+            assert rid >= 0 and st == 0, (rid, st)
+            got.append(rid)
+        got.append(time.thread_time() - t0)
+
+    th = threading.Thread(target=waiter)
+    th.start()
+    w0 = time.time()
+    sent = []
+    for i in range(n):
+        sent.append(e.submit(0, mid, (i % 8) * 16384, need))
+        time.sleep(gap)
+    th.join(timeout=30)
+    assert not th.is_alive()
+    cpu, wall = got.pop(), time.time() - w0
+    assert sorted(got) == sorted(sent)
+    assert cpu < 0.5 * wall, (cpu, wall)
+    e.shutdown()
