@@ -318,6 +318,16 @@ int64_t paella_loadgen(paella_t* p, const paella_req_t* reqs, uint32_t n, size_t
                        uint32_t slots_per_client, const void* const* const* copy_inputs,
                        int64_t t0_ns, int64_t* jct_ns, int64_t* elapsed_ns);
 
+int paella_bench_wait(paella_t* p, uint32_t client_id, uint32_t model_id, uint32_t n, int64_t gap_ns,
+                      uint32_t poll_flags, size_t stride, uint32_t slots, int64_t* jct_ns,
+                      double* waiter_cpu_frac);
+/* NEXT-3 measurement (P1157-1171, Fig. 14): the calling thread submits n requests of
+   one model at a fixed gap (open loop, slots of `stride` bytes in the client's region,
+   inputs pre-staged); a second thread waits for the completions with
+   paella_poll_completion(poll_flags: 0 = spin, PAELLA_HYBRID).  jct_ns[n]: submit ->
+   completion seen; *waiter_cpu_frac: the waiting thread's CPU time / wall time.
+   Returns 0 or -errno. */
+
 /* Debug: copy node `node`'s activation of the last isolated run to host as fp32
    NCHW (C*H*W floats).  Returns 0 or -errno. */
 int paella_debug_node(paella_t* p, uint32_t gpu, uint32_t model_id, uint32_t node, float* out);

@@ -34,7 +34,7 @@ SYMBOLS = ["paella_init", "paella_register_model", "paella_submit", "paella_subm
            "paella_poll_completion", "paella_shutdown", "paella_client_region", "paella_model_info",
            "paella_kernel_info", "paella_kernel_name", "paella_stats", "paella_flush_log",
            "paella_run_isolated", "paella_debug_node", "paella_time_kernels", "paella_bench_empty",
-           "paella_bench_roundtrip", "paella_loadgen"]
+           "paella_bench_roundtrip", "paella_loadgen", "paella_bench_wait"]
 
 
 class Config(C.Structure):
@@ -129,6 +129,9 @@ def load():
     lib.paella_loadgen.argtypes = [P, C.POINTER(Req), C.c_uint32, C.c_size_t, C.c_uint32, P, C.c_int64,
                                    C.POINTER(C.c_int64), C.POINTER(C.c_int64)]
     lib.paella_loadgen.restype = C.c_int64
+    lib.paella_bench_wait.argtypes = [P, C.c_uint32, C.c_uint32, C.c_uint32, C.c_int64, C.c_uint32, C.c_size_t,
+                                      C.c_uint32, C.POINTER(C.c_int64), C.POINTER(C.c_double)]
+    lib.paella_bench_wait.restype = C.c_int
     _lib = lib
     return lib
 
@@ -325,6 +328,14 @@ class Engine:
         _check(self.lib.paella_bench_roundtrip(self.h, gpu, n, a.ctypes.data_as(C.POINTER(C.c_int64)),
                                                b.ctypes.data_as(C.POINTER(C.c_int64))), "paella_bench_roundtrip")
         return a, b
+
+    def bench_wait(self, client, model, n, gap_ns, poll_flags, stride, slots):
+        """NEXT-3 measurement: (jct_ns array, waiter CPU fraction); see paella_bench_wait."""
+        j = np.zeros(n, dtype=np.int64)
+        f = C.c_double()
+        _check(self.lib.paella_bench_wait(self.h, client, model, n, int(gap_ns), poll_flags, stride, slots,
+                                          j.ctypes.data_as(C.POINTER(C.c_int64)), C.byref(f)), "paella_bench_wait")
+        return j, f.value
 
     def loadgen(self, t_ns, clients, models, inputs, stride, slots, copy_inputs=None, t0_ns=0):
         """Open-loop replay of a trace from the calling thread (GIL released).

@@ -3,7 +3,10 @@
 // shared region (P1039-1061) and readResult(NONBLOCK) polling (P1147-1155).
 #include <errno.h>
 
+#include <atomic>
 #include <cstring>
+#include <thread>
+#include <time.h>
 #include <vector>
 
 #include "engine.h"
@@ -84,4 +87,66 @@ extern "C" int64_t paella_loadgen(paella_t* p, const paella_req_t* reqs, uint32_
   }
   if (elapsed_ns) *elapsed_ns = now_ns() - t0;
   return done;
+}
+
+extern "C" int paella_bench_wait(paella_t* p, uint32_t client_id, uint32_t model_id, uint32_t n, int64_t gap_ns,
+                                 uint32_t poll_flags, size_t stride, uint32_t slots, int64_t* jct_ns,
+                                 double* waiter_cpu_frac) {
+  Paella* P = (Paella*)p;
+  if (!P || !jct_ns || !waiter_cpu_frac || client_id >= P->cfg.num_clients || model_id >= P->nmodels.load() ||
+      slots == 0 || (size_t)slots * stride > P->region_bytes)
+    return -EINVAL;
+  Model* m = P->models[model_id].get();
+  std::vector<std::atomic<int64_t>> t_sub(n);
+  std::vector<std::atomic<uint32_t>> slot_free(slots);
+  for (auto& f : slot_free) f.store(1);
+  std::vector<uint32_t> slot_of(n, 0);
+  std::atomic<uint32_t> done{0};
+  std::atomic<int64_t> seq0{-1};   // req_id sequence number of request 0 (ids are per-client seqs)
+  double cpu_frac = 0;
+  std::thread waiter([&] {
+    timespec c0, c1;
+    clock_gettime(CLOCK_THREAD_CPUTIME_ID, &c0);
+    const int64_t w0 = now_ns();
+    while (done.load() < n) {
+      int32_t st = 0;
+      int64_t rid = paella_poll_completion(p, client_id, poll_flags, &st);
+      if (rid < 0) {
+        if (rid == -EAGAIN) continue;
+        break;
+      }
+      const int64_t t = now_ns();
+      while (seq0.load(std::memory_order_acquire) < 0) {
+      }
+      const uint32_t i = (uint32_t)(((uint64_t)rid & 0xFFFFFFFFFFFFull) - (uint64_t)seq0.load());
+      if (i >= n) continue;
+      jct_ns[i] = st == 0 ? t - t_sub[i].load(std::memory_order_acquire) : -1;
+      slot_free[slot_of[i]].store(1, std::memory_order_release);
+      done.fetch_add(1);
+    }
+    clock_gettime(CLOCK_THREAD_CPUTIME_ID, &c1);
+    const double cpu = (c1.tv_sec - c0.tv_sec) + (c1.tv_nsec - c0.tv_nsec) * 1e-9;
+    cpu_frac = cpu / ((now_ns() - w0) * 1e-9);
+  });
+  int64_t due = now_ns();
+  int rc = 0;
+  for (uint32_t i = 0; i < n && rc == 0; ++i) {
+    due += gap_ns;
+    while (now_ns() < due) {
+    }
+    uint32_t s = i % slots;
+    while (!slot_free[s].load(std::memory_order_acquire)) {
+    }
+    slot_free[s].store(0);
+    slot_of[i] = s;
+    t_sub[i].store(now_ns(), std::memory_order_release);
+    uint8_t* io = P->region[client_id] + (size_t)s * stride;
+    int64_t rid = paella_submit(p, client_id, model_id, io, m->input_bytes + m->output_bytes, 0);
+    if (rid < 0) rc = (int)rid;
+    else if (i == 0) seq0.store((int64_t)((uint64_t)rid & 0xFFFFFFFFFFFFull), std::memory_order_release);
+  }
+  if (rc) done.store(n);
+  waiter.join();
+  *waiter_cpu_frac = cpu_frac;
+  return rc;
 }

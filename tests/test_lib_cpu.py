@@ -210,3 +210,17 @@ def test_hybrid_poll_sleeps_between_hints():
     assert sorted(got) == sorted(sent)
     assert cpu < 0.5 * wall, (cpu, wall)
     e.shutdown()
+
+
+def test_bench_wait_spin_vs_hybrid_fake():
+    """paella_bench_wait (the NEXT-3 measurement): every request completes under both
+    waiting modes; the hybrid waiter uses less CPU than the spinning one."""
+    e = _toy_engine(num_clients=1)
+    mid = e.register_model(archs.toy(), rng.model_params(archs.toy()))
+    info = e.model_info(mid)
+    stride = (info["input_bytes"] + info["output_bytes"] + 4095) // 4096 * 4096
+    j0, spin = e.bench_wait(0, mid, 200, 500_000, 0, stride, 16)
+    j1, hyb = e.bench_wait(0, mid, 200, 500_000, L.HYBRID, stride, 16)
+    assert (j0 > 0).all() and (j1 > 0).all()
+    assert hyb < 0.5 * spin, (hyb, spin)
+    e.shutdown()
