@@ -438,6 +438,27 @@ def roofline_entry(res, peaks):
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (burst copy)"}
 
 
+def saturating_conv(args):
+    """The dominant kernel where its roofline is reachable: the tcgen05
+    conv on 3x3 256->256 layers over 56x56 and 448x448 pixels (tools/conv_saturating.py),
+    timed like the batch-1 kernels (PDL chain, CUDA events), against the measured bf16
+    tensor peak."""
+    import importlib.util
+    spec = importlib.util.spec_from_file_location("conv_saturating", os.path.join(ROOT, "tools", "conv_saturating.py"))
+    cs = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(cs)
+    from paper_conf_sosp_ngd023_b200 import _lib as L
+    peaks = json.load(open(PEAKS_PATH)) if os.path.exists(PEAKS_PATH) else {}
+    peak = peaks.get("bf16_tflops", 2250.0)
+    with L.Engine(num_clients=1, max_jobs_per_model=1, first_gpu=int(os.environ.get("LOCAL_RANK", "0"))) as e:
+        rows = [cs.measure(e, hw) for hw in (56, 448)]
+    best = max(rows, key=lambda r: r["tflops_instr"])
+    return {"kernel": "conv_tcgen05", "bound": "tensor", "achieved": best["tflops_instr"], "peak": peak,
+            "unit": "TFLOP/s", "frac": round(best["tflops_instr"] / peak, 4),
+            "peak_source": "MEASURED_PEAKS.json bf16_tflops (cuBLAS burst)" if peaks else "nominal 2250",
+            "shapes": rows}
+
+
 def main():
     args = parse()
     dist = Dist(args.gpus)
@@ -512,6 +533,10 @@ def main():
         "dispatcher": {k: (v if isinstance(v, list) else int(v)) for k, v in res["stats"].items()},
     }
     if args.gpus == 1 and not args.fake:
+        try:
+            line["roofline_saturating"] = saturating_conv(args)
+        except Exception as ex:   # diagnostic only: never fail the bench line for it
+            line["roofline_saturating"] = {"error": str(ex)[:200]}
         line["cpu_baseline"] = cpu_baseline(cfg, seconds=12.0)
     if args.fake:
         line["data"] = "synthetic, FAKE CPU device (plumbing test, not a measurement)"
