@@ -55,6 +55,8 @@ def parse():
     ap.add_argument("--slack", type=int, default=1184,
                     help="B, blocks issued beyond full utilisation (P1300-1304); 8 x 148 SMs covers the "
                          "measured dispatch loop delay (DESIGN.md B200-Q1)")
+    ap.add_argument("--policy", default="srpt", choices=["srpt", "fifo", "sjf", "rr"],
+                    help="policy of the Paella arm (sjf/rr: Table 3 ablations, NEXT-2)")
     ap.add_argument("--theta", type=int, default=100, help="fairness threshold (kernel dispatches, P1296-1297)")
     ap.add_argument("--prio-classes", type=int, default=1, help="stream-priority classes (DESIGN.md B200-Q2)")
     ap.add_argument("--launch-threads", type=int, default=4, help="launcher helper threads per GPU")
@@ -252,6 +254,8 @@ def run_gpu(args, dist):
     def engine(**kw):
         kw.setdefault("launch_threads", 0 if args.fake else args.launch_threads)
         if not kw.get("naive"):
+            kw.setdefault("policy", {"srpt": L.POLICY_SRPT_DEFICIT, "fifo": L.POLICY_FIFO, "sjf": L.POLICY_SJF,
+                                     "rr": L.POLICY_RR}[args.policy])
             kw.setdefault("theta", args.theta)
             kw.setdefault("slack", args.slack)
             kw.setdefault("prio_classes", args.prio_classes)
@@ -344,7 +348,8 @@ def run_gpu(args, dist):
     base = {}
     if not args.no_baselines:
         for label, kw in (("naive_cuda_ms", dict(naive=True, instrument=False)),
-                          ("paella_paper_lookahead0", dict(lookahead=0, slack=0, prio_classes=1, pdl=False)),
+                          ("paella_paper_lookahead0", dict(policy=L.POLICY_SRPT_DEFICIT, lookahead=0, slack=0, prio_classes=1,
+                                                           pdl=False)),
                           ("paella_fifo", dict(policy=L.POLICY_FIFO, lookahead=args.lookahead))):
             eb, mb = engine(**kw)
             jl = []
@@ -512,7 +517,7 @@ def main():
                    "l2": "not flushed: steps are open-loop traces whose weights (~33 MB bf16) stay L2-resident "
                          "as in serving; inputs stream from pinned host memory"},
         "jct_us": res["jct"], "slo_us": res["slo"],
-        "paella_config": {"lookahead": args.lookahead, "launch_threads": args.launch_threads, "policy": "srpt+deficit",
+        "paella_config": {"lookahead": args.lookahead, "launch_threads": args.launch_threads, "policy": {"srpt": "srpt+deficit"}.get(args.policy, args.policy),
                           "slack_blocks": args.slack, "prio_classes": args.prio_classes, "pdl": True,
                           "theta": args.theta, "group": 16, "streams": 32},
         "slo_met": bool(all(res["jct"].get(n, {}).get("p99_us", 1e18) <= res["slo"][n] for n in res["names"])),

@@ -52,6 +52,8 @@ extern "C" {
 /* policies (P1222-1323 §6; FIFO = the Paella-SS-like ablation of Table 3, P1349) */
 #define PAELLA_POLICY_SRPT_DEFICIT 0u
 #define PAELLA_POLICY_FIFO         1u
+#define PAELLA_POLICY_SJF          2u   /* ablation (NEXT-2, Table 3): shortest whole job first */
+#define PAELLA_POLICY_RR           3u   /* ablation: kernel-granular round robin over ready jobs */
 
 /* routing across GPUs */
 #define PAELLA_ROUTE_LEAST_WORK    0u

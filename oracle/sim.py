@@ -30,7 +30,7 @@ import itertools
 from dataclasses import dataclass, field
 
 PLACEMENT, COMPLETION = 1, 2
-SRPT_DEFICIT, FIFO = 0, 1
+SRPT_DEFICIT, FIFO, SJF, RR = 0, 1, 2, 3   # SJF / RR: Table 3 ablations (NEXT-2, P1341-1359)
 RESOURCES = ("blocks", "warps", "regs", "smem", "tmem")
 INF_THETA = (1 << 63) - 1
 
@@ -74,6 +74,7 @@ class Job:
     last_stream: int = -1
     last_uid: int = -1
     uids: dict = field(default_factory=dict)   # layer -> launch uid (while in flight)
+    rr: int = -1             # RR ablation: uid of the job's last issued kernel (-1 = never)
 
     @property
     def inflight(self):
@@ -195,6 +196,10 @@ class Policy:
         self.over = False
         if cfg.policy == FIFO:
             return min(rdy, key=lambda j: j.seq)
+        if cfg.policy == SJF:      # shortest (whole) job first: T-bar sum of the model
+            return min(rdy, key=lambda j: (self.remaining(j.model, 0), j.seq, j.id))
+        if cfg.policy == RR:       # kernel-granular round robin: least recently issued job
+            return min(rdy, key=lambda j: (j.rr, j.seq, j.id))
         clients = sorted({j.client for j in rdy})
         cstar = max(clients, key=lambda c: (self.D(c), -c))
         self.over = cfg.theta != INF_THETA and self.D(cstar) > cfg.theta * cfg.num_clients
@@ -263,6 +268,7 @@ class Policy:
             j.uids[j.cursor] = uid
             j.cursor += 1
             j.last_uid = uid
+            j.rr = uid
             if self.checks:
                 assert j.R >= 0
             self.Dt[j.client] -= cfg.num_clients

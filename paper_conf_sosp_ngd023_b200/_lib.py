@@ -18,7 +18,7 @@ LIB_PATH = os.path.join(HERE, "libpaella.so")
 
 ABI_VERSION = 1
 NOTIFY_COUNTERS, NOTIFY_RING = 0, 1
-POLICY_SRPT_DEFICIT, POLICY_FIFO = 0, 1
+POLICY_SRPT_DEFICIT, POLICY_FIFO, POLICY_SJF, POLICY_RR = 0, 1, 2, 3
 ROUTE_LEAST_WORK, ROUTE_ROUND_ROBIN = 0, 1
 DEVICE_CUDA, DEVICE_FAKE = 0, 1
 DTYPE_BF16, DTYPE_FP32 = 0, 1

@@ -861,7 +861,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
   paella_config_t cfg = *cfg_in;
   if (cfg.num_gpus < 1 || cfg.num_gpus > PAELLA_MAX_GPUS) return -EINVAL;
   if (cfg.num_clients < 1 || cfg.num_clients > PAELLA_MAX_CLIENTS) return -EINVAL;
-  if (cfg.policy > PAELLA_POLICY_FIFO || cfg.device > PAELLA_DEVICE_FAKE) return -EINVAL;
+  if (cfg.policy > PAELLA_POLICY_RR || cfg.device > PAELLA_DEVICE_FAKE) return -EINVAL;
   if (cfg.group_size == 0) cfg.group_size = 16;
   if (cfg.group_size > 16) return -EINVAL;
   if (cfg.ring_capacity == 0) cfg.ring_capacity = 65536;

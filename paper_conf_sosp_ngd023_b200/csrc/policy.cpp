@@ -16,6 +16,7 @@ Policy::Policy(const Cfg& c) : cfg_(c) {
   unfinished_.assign(c.num_clients, 0);
   per_client_.resize(c.num_clients);
   models_.resize(kMaxModels);   // never reallocated: models are added while dispatching
+  model_total_.assign(kMaxModels, 0);
 }
 
 void Policy::add_model(uint32_t mid, const std::vector<PolicyLayer>& layers) {
@@ -23,6 +24,7 @@ void Policy::add_model(uint32_t mid, const std::vector<PolicyLayer>& layers) {
   models_[mid] = layers;
   int64_t t = 0;
   for (const auto& l : layers) t += l.tbar;
+  model_total_[mid] = t;
   if (!layers.empty()) {
     auto it = std::lower_bound(totals_.begin(), totals_.end(), t);
     if (it == totals_.end() || *it != t) totals_.insert(it, t);
@@ -65,16 +67,24 @@ void Policy::refresh(PolicyJob& j) {
   else if (!r && j.in_ready) make_unready(j);
 }
 
+// ready-set order key: SRPT (R_j), SJF (the model's whole-job T-bar sum), RR (uid of the
+// job's last issued kernel, -1 = never); ties (seq, id).  Identical to oracle Policy.pick.
+int64_t Policy::order_key(const PolicyJob& j) const {
+  if (cfg_.policy == POL_SJF) return model_total_[j.model];
+  if (cfg_.policy == POL_RR) return j.rr;
+  return j.R;
+}
+
 void Policy::make_ready(PolicyJob& j) {
   j.in_ready = true;
-  srpt_.emplace(j.R, j.seq, j.id);
+  srpt_.emplace(order_key(j), j.seq, j.id);
   fifo_.emplace(j.seq, j.id);
   per_client_[j.client].emplace(j.seq, j.id);
 }
 
 void Policy::make_unready(PolicyJob& j) {
   j.in_ready = false;
-  srpt_.erase(std::make_tuple(j.R, j.seq, j.id));
+  srpt_.erase(std::make_tuple(order_key(j), j.seq, j.id));
   fifo_.erase(std::make_pair(j.seq, j.id));
   per_client_[j.client].erase(std::make_pair(j.seq, j.id));
 }
@@ -151,6 +161,10 @@ bool Policy::pick(uint32_t* job_id) {
   if (srpt_.empty()) return false;
   if (cfg_.policy == POL_FIFO) {
     *job_id = fifo_.begin()->second;
+    return true;
+  }
+  if (cfg_.policy == POL_SJF || cfg_.policy == POL_RR) {   // pure orders, no deficit rule
+    *job_id = std::get<2>(*srpt_.begin());
     return true;
   }
   // c* = argmax (D_c, -c) over clients with a ready job
@@ -243,6 +257,7 @@ void Policy::decide(std::vector<Issue>* out) {
     j.uid_of[j.cursor % 8] = uid;
     j.cursor += 1;
     j.last_uid = uid;
+    j.rr = uid;   // after make_unready above: the ready-set key changes only out of the set
     Dt_[j.client] -= (int64_t)cfg_.num_clients;
     Omega_ += 1;
     out->push_back(Issue{uid, jid, L.layer, stream});

@@ -42,6 +42,7 @@ struct PolicyJob {
   int32_t stream = -1;       // stream held while kernels are in flight
   int32_t last_stream = -1;
   uint32_t last_uid = 0;
+  int64_t rr = -1;           // RR ablation: uid of the last issued kernel (-1 = never)
   uint32_t uid_of[8] = {0};  // launch uid of layer l (l mod 8) while in flight
   bool live = false;
   bool in_ready = false;
@@ -58,7 +59,7 @@ struct Issue {
   uint32_t uid, job, layer, stream;
 };
 
-enum : uint32_t { POL_SRPT_DEFICIT = 0, POL_FIFO = 1 };
+enum : uint32_t { POL_SRPT_DEFICIT = 0, POL_FIFO = 1, POL_SJF = 2, POL_RR = 3 };   // SJF/RR: Table 3 ablations
 
 class Policy {
  public:
@@ -106,6 +107,7 @@ class Policy {
   uint32_t job_class(const PolicyJob& j) const;
   int lowest_free_in_class(uint32_t c) const;
   bool predicate(uint32_t grid) const;
+  int64_t order_key(const PolicyJob& j) const;
   void make_ready(PolicyJob& j);
   void make_unready(PolicyJob& j);
   bool is_ready(const PolicyJob& j) const;
@@ -121,6 +123,7 @@ class Policy {
   int last_stop_ = 0;
   bool over_ = false;                  // the last pick was a deficit override
   std::vector<int64_t> totals_;        // sorted distinct whole-job T-bar sums of the models
+  std::vector<int64_t> model_total_;   // whole-job T-bar sum per model (SJF key)
   std::vector<uint64_t> free_;   // bitmap of free streams
   std::vector<int64_t> Dt_;
   int64_t Omega_ = 0;

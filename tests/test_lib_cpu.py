@@ -113,7 +113,9 @@ def _serve(e, mids, n, n_clients, seed, stride=16384, timeout=60):
     (L.POLICY_SRPT_DEFICIT, 3, 16, 2, 0, 1), (L.POLICY_SRPT_DEFICIT, 100, 16, 8, 1, 1),
     (L.POLICY_FIFO, 100, 4, 4, 1, 1), (L.POLICY_SRPT_DEFICIT, 0, 1, 16, 2, 1),
     (L.POLICY_SRPT_DEFICIT, 100, 16, 8, 1, 4), (L.POLICY_SRPT_DEFICIT, 3, 4, 12, 2, 3),
-    (L.POLICY_SRPT_DEFICIT, None, 16, 32, 0, 2), (L.POLICY_FIFO, 100, 16, 8, 1, 2)])
+    (L.POLICY_SRPT_DEFICIT, None, 16, 32, 0, 2), (L.POLICY_FIFO, 100, 16, 8, 1, 2),
+    (L.POLICY_SJF, 100, 16, 8, 0, 1), (L.POLICY_SJF, 100, 4, 4, 2, 2),
+    (L.POLICY_RR, 100, 16, 8, 0, 1), (L.POLICY_RR, 100, 4, 12, 1, 3)])
 def test_fake_device_replay_parity(tmp_path, policy, theta, group, streams, look, prio):
     log = str(tmp_path / "ev_%u.log")
     models = [archs.toy(), archs.squeezenet1_1()]

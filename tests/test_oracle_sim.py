@@ -381,3 +381,35 @@ def test_prio_classes_stream_rule(seed):
         assert stream * K // 32 == want, (jid, layer, stream, R, totals)
         checked += 1
     assert checked == len(res.issues) > 0
+
+
+# --- NEXT-2 ablations (Table 3, P1341-1359): SJF and RR orders ----------------------
+
+@pytest.mark.parametrize("seed", range(40))
+def test_sjf_optimal_all_released_at_zero(seed):
+    """Single server, all jobs at t = 0: shortest-whole-job-first serves jobs one after
+    another in SPT order, which is optimal (the same brute force as S1a)."""
+    r = random.Random(500 + seed)
+    jobs = [[r.randint(1, 9) for _ in range(r.randint(1, 3))] for _ in range(r.randint(2, 4))]
+    models = whole_sm_models(jobs)
+    trace = [(0, 0, m) for m in range(len(jobs))]
+    cfg = single_server_cfg()
+    cfg.policy = sim.SJF
+    res = sim.simulate(cfg, models, trace, ONE_SM)
+    assert sum(res.jct().values()) == brute_min_total_completion(jobs) * UNIT
+
+
+@pytest.mark.parametrize("n,k", [(2, 3), (3, 2), (4, 4), (5, 1)])
+def test_rr_closed_form(n, k):
+    """n identical jobs of k unit kernels, single server, all at t = 0: kernel-granular
+    round robin finishes job i (arrival order) at (k - 1) n + i + 1 units, so the total
+    JCT is n^2 (k - 1) + n (n + 1) / 2 (SRPT would give k n (n + 1) / 2)."""
+    models = whole_sm_models([[1] * k for _ in range(n)])
+    trace = [(0, 0, m) for m in range(n)]
+    cfg = single_server_cfg()
+    cfg.policy = sim.RR
+    res = sim.simulate(cfg, models, trace, ONE_SM)
+    assert sum(res.jct().values()) == (n * n * (k - 1) + n * (n + 1) // 2) * UNIT
+    cfg2 = single_server_cfg()
+    res2 = sim.simulate(cfg2, models, trace, ONE_SM)
+    assert sum(res2.jct().values()) == (k * n * (n + 1) // 2) * UNIT
