@@ -57,6 +57,8 @@ def parse():
                          "measured dispatch loop delay (DESIGN.md B200-Q1)")
     ap.add_argument("--policy", default="srpt", choices=["srpt", "fifo", "sjf", "rr"],
                     help="policy of the Paella arm (sjf/rr: Table 3 ablations, NEXT-2)")
+    ap.add_argument("--decide-delay-ns", type=int, default=0,
+                    help="injected scheduler delay before every decide pass (Fig. 9 sensitivity)")
     ap.add_argument("--theta", type=int, default=100, help="fairness threshold (kernel dispatches, P1296-1297)")
     ap.add_argument("--prio-classes", type=int, default=1, help="stream-priority classes (DESIGN.md B200-Q2)")
     ap.add_argument("--launch-threads", type=int, default=4, help="launcher helper threads per GPU")
@@ -257,6 +259,7 @@ def run_gpu(args, dist):
             kw.setdefault("policy", {"srpt": L.POLICY_SRPT_DEFICIT, "fifo": L.POLICY_FIFO, "sjf": L.POLICY_SJF,
                                      "rr": L.POLICY_RR}[args.policy])
             kw.setdefault("theta", args.theta)
+            kw.setdefault("decide_delay_ns", args.decide_delay_ns)
             kw.setdefault("slack", args.slack)
             kw.setdefault("prio_classes", args.prio_classes)
         e, mids = build_engine(L, specs, gpu, fake=args.fake, region_bytes=region, max_jobs_per_model=128, **kw)
@@ -519,7 +522,7 @@ def main():
         "jct_us": res["jct"], "slo_us": res["slo"],
         "paella_config": {"lookahead": args.lookahead, "launch_threads": args.launch_threads, "policy": {"srpt": "srpt+deficit"}.get(args.policy, args.policy),
                           "slack_blocks": args.slack, "prio_classes": args.prio_classes, "pdl": True,
-                          "theta": args.theta, "group": 16, "streams": 32},
+                          "theta": args.theta, "group": 16, "streams": 32, "decide_delay_ns": args.decide_delay_ns},
         "slo_met": bool(all(res["jct"].get(n, {}).get("p99_us", 1e18) <= res["slo"][n] for n in res["names"])),
         "req_s_at_p99_slo": {k: v["req_s"] for k, v in res["slo_at"].items()},
         "slo_ladder": res["slo_at"],

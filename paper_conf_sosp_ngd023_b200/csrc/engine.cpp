@@ -697,6 +697,11 @@ static uint32_t drain_counters(Gpu* g) {
 }
 
 static void decide_and_launch(Gpu* g) {
+  if (const uint32_t d = g->P->cfg.decide_delay_ns) {   // injected scheduler delay (Fig. 9)
+    const int64_t until = now_ns() + d;
+    while (now_ns() < until) {
+    }
+  }
   g->issues.clear();
   g->policy->decide(&g->issues);
   if (!g->issues.empty() && g->P->cfg.device == PAELLA_DEVICE_CUDA)
