@@ -57,6 +57,7 @@ def parse():
                          "measured dispatch loop delay (DESIGN.md B200-Q1)")
     ap.add_argument("--policy", default="srpt", choices=["srpt", "fifo", "sjf", "rr"],
                     help="policy of the Paella arm (sjf/rr: Table 3 ablations, NEXT-2)")
+    ap.add_argument("--online-tbar", action="store_true", help="NEXT-4 online T-bar refinement in the Paella arm")
     ap.add_argument("--decide-delay-ns", type=int, default=0,
                     help="injected scheduler delay before every decide pass (Fig. 9 sensitivity)")
     ap.add_argument("--theta", type=int, default=100, help="fairness threshold (kernel dispatches, P1296-1297)")
@@ -260,6 +261,7 @@ def run_gpu(args, dist):
                                      "rr": L.POLICY_RR}[args.policy])
             kw.setdefault("theta", args.theta)
             kw.setdefault("decide_delay_ns", args.decide_delay_ns)
+            kw.setdefault("online_tbar", args.online_tbar)
             kw.setdefault("slack", args.slack)
             kw.setdefault("prio_classes", args.prio_classes)
         e, mids = build_engine(L, specs, gpu, fake=args.fake, region_bytes=region, max_jobs_per_model=128, **kw)
@@ -522,7 +524,8 @@ def main():
         "jct_us": res["jct"], "slo_us": res["slo"],
         "paella_config": {"lookahead": args.lookahead, "launch_threads": args.launch_threads, "policy": {"srpt": "srpt+deficit"}.get(args.policy, args.policy),
                           "slack_blocks": args.slack, "prio_classes": args.prio_classes, "pdl": True,
-                          "theta": args.theta, "group": 16, "streams": 32, "decide_delay_ns": args.decide_delay_ns},
+                          "theta": args.theta, "group": 16, "streams": 32, "decide_delay_ns": args.decide_delay_ns,
+                          "online_tbar": bool(args.online_tbar)},
         "slo_met": bool(all(res["jct"].get(n, {}).get("p99_us", 1e18) <= res["slo"][n] for n in res["names"])),
         "req_s_at_p99_slo": {k: v["req_s"] for k, v in res["slo_at"].items()},
         "slo_ladder": res["slo_at"],

@@ -148,6 +148,10 @@ typedef struct {
                                     clamped to K-1; deficit-override picks take class 0), so the
                                     blocks the +B slack keeps queued in hardware are also served
                                     shortest-remaining first (B200-Q2).  K <= P. */
+  uint32_t online_tbar;           /* NEXT-4: 1 = refine T-bar online, as the running average of
+                                    the profiling runs and every observed duration of that
+                                    kernel (first placement -> final completion seen by the
+                                    dispatcher, P1249-1266); 0 (default) = frozen profile */
   uint32_t decide_delay_ns;       /* NEXT-2 sensitivity (Fig. 9, P1215-1241): the dispatcher
                                     busy-waits this long before every decide() pass, an
                                     injected scheduler delay; 0 (default) = none */

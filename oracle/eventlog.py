@@ -6,6 +6,7 @@ Format (DESIGN.md §"Event log"): a sequence of 32-byte little-endian records
 
   100 CONFIG    a=N clients, b=policy, c=theta, d=(B << 32) | G
   100 CONFIG    a=0xFFFFFFFF, b=ring capacity, c=stream pool P, d=(priority classes << 32) | launch-ahead depth
+  100 CONFIG    a=0xFFFFFFFE, b=online T-bar refinement (NEXT-4)
   101 CAPACITY  a=resource r, b=C_r
   110 MODEL     a=model, b=#kernels
   111 LAYER     a=model, b=layer, c=grid, d=T-bar ns
@@ -15,6 +16,7 @@ Format (DESIGN.md §"Event log"): a sequence of 32-byte little-endian records
     3 BATCH_END
     4 ISSUE     a=stream, b=uid, c=job, d=layer
     5 COMPLETE  b=job, c=t ns
+    6 OBSERVE   b=uid, c=observed duration ns (NEXT-4; precedes the final COMPLETION)
 """
 import numpy as np
 
@@ -40,7 +42,9 @@ def read(path):
     for r in raw:
         t, a, b, c, d = int(r["type"]), int(r["a"]), int(r["b"]), int(r["c"]), int(r["d"])
         if t == 100:
-            if a == 0xFFFFFFFF:
+            if a == 0xFFFFFFFE:
+                cfg_kw["online_tbar"] = b
+            elif a == 0xFFFFFFFF:
                 cfg_kw["ring_capacity"] = b
                 cfg_kw["streams"] = c
                 cfg_kw["lookahead"] = d & 0xFFFFFFFF
@@ -72,6 +76,8 @@ def read(path):
         elif t == 4:
             events.append((sim.EV_ISSUE, b, c, d, a))
             issues.append((b, c, d, a, arrivals[c][1]))   # (uid, job, layer, stream, model)
+        elif t == 6:
+            events.append((sim.EV_OBSERVE, b, c))
         elif t == 5:
             events.append((sim.EV_COMPLETE, b))
             completes.append((b, c))

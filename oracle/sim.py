@@ -55,6 +55,17 @@ class Config:
     capacity: tuple = (148 * 32, 148 * 64, 148 * 65536, 148 * 233472, 148 * 512)
     lookahead: int = 0                # NEXT-1 launch-ahead depth (0 = the paper's semantics)
     prio_classes: int = 1             # stream-priority classes (1 = the paper: one class)
+    online_tbar: int = 0              # NEXT-4: refine T-bar online (running average, P1252-1254)
+
+
+# NEXT-4 (P1249-1266: "x-bar is the average of all previous observations of x"; "these
+# profiles can be further refined online"): with online_tbar, T-bar of (model, layer)
+# is the integer running average of the PROFILE_RUNS profiling observations plus every
+# observed duration of that kernel (first PLACEMENT seen -> final COMPLETION seen by the
+# dispatcher, logged as an OBSERVE event).  It is updated when the launch completes;
+# every live job whose remaining kernels include that layer has R_j adjusted by the
+# change.  SJF keys and stream-priority classes keep the frozen profile.
+PROFILE_RUNS = 20
 
 
 def groups(g, G):
@@ -120,6 +131,11 @@ class Policy:
         self.over = False                    # the last pick was a deficit override
         self.checks = True                   # assert invariants (c),(d),(g) as we go
         self.log: list[tuple] | None = None  # consumed-event log in replay format
+        # current T-bar per (model, layer) and the running-average state (NEXT-4)
+        self.tb = [[l.tbar for l in m] for m in models]
+        self.tb_sum = [[l.tbar * PROFILE_RUNS for l in m] for m in models]
+        self.tb_cnt = [[PROFILE_RUNS for _ in m] for m in models]
+        self.obs: dict[int, int] = {}        # launch uid -> observed duration (pending)
 
     # effective deficit, units of 1/N
     def D(self, c):
@@ -127,7 +143,28 @@ class Policy:
 
     def remaining(self, model, cursor):
         """R_j = sum of T-bar over kernels not yet dispatched (C2-Q8, C2-Q9)."""
-        return sum(l.tbar for l in self.models[model][cursor:])
+        return sum(self.tb[model][cursor:])
+
+    def observe(self, uid, d):
+        """NEXT-4: the duration of launch uid, consumed before its final COMPLETION."""
+        if self.log is not None:
+            self.log.append((EV_OBSERVE, uid, d))
+        self.obs[uid] = d
+
+    def _refine(self, L):
+        d = self.obs.pop(L.uid, None)
+        if not self.cfg.online_tbar or d is None:
+            return
+        m, lay = self.jobs[L.job].model, L.layer
+        self.tb_sum[m][lay] += d
+        self.tb_cnt[m][lay] += 1
+        new = self.tb_sum[m][lay] // self.tb_cnt[m][lay]
+        delta = new - self.tb[m][lay]
+        self.tb[m][lay] = new
+        if delta:
+            for j in self.jobs.values():
+                if j.model == m and j.cursor <= lay:
+                    j.R += delta
 
     # --- events -------------------------------------------------------------
     def arrival(self, job_id, client, model):
@@ -161,6 +198,7 @@ class Policy:
         done = None
         if L.f == L.grid:
             del self.launches[uid]
+            self._refine(L)
             j = self.jobs[L.job]
             j.done += 1
             if j.inflight == 0:
@@ -196,8 +234,8 @@ class Policy:
         self.over = False
         if cfg.policy == FIFO:
             return min(rdy, key=lambda j: j.seq)
-        if cfg.policy == SJF:      # shortest (whole) job first: T-bar sum of the model
-            return min(rdy, key=lambda j: (self.remaining(j.model, 0), j.seq, j.id))
+        if cfg.policy == SJF:      # shortest (whole) job first: profiled T-bar sum of the model
+            return min(rdy, key=lambda j: (sum(l.tbar for l in self.models[j.model]), j.seq, j.id))
         if cfg.policy == RR:       # kernel-granular round robin: least recently issued job
             return min(rdy, key=lambda j: (j.rr, j.seq, j.id))
         clients = sorted({j.client for j in rdy})
@@ -263,7 +301,7 @@ class Policy:
                 self.U[r] += layer.grid * layer.demand[r]
             self.Q += layer.grid
             self.O += 2 * groups(layer.grid, cfg.group)
-            j.R -= layer.tbar
+            j.R -= self.tb[j.model][j.cursor]
             rec = (uid, j.id, j.cursor, stream)
             j.uids[j.cursor] = uid
             j.cursor += 1
@@ -284,7 +322,7 @@ class Policy:
 # Replay mode (pin S6)
 # ---------------------------------------------------------------------------
 
-EV_ARRIVAL, EV_RECORD, EV_BATCH_END, EV_ISSUE, EV_COMPLETE = 1, 2, 3, 4, 5
+EV_ARRIVAL, EV_RECORD, EV_BATCH_END, EV_ISSUE, EV_COMPLETE, EV_OBSERVE = 1, 2, 3, 4, 5, 6
 
 
 def replay(cfg: Config, models, events):
@@ -305,6 +343,8 @@ def replay(cfg: Config, models, events):
         k = ev[0]
         if k == EV_ARRIVAL:
             pol.arrival(ev[1], ev[2], ev[3])
+        elif k == EV_OBSERVE:
+            pol.observe(ev[1], ev[2])
         elif k == EV_RECORD:
             d = pol.record(ev[1], ev[2], ev[3])
             if d is not None:

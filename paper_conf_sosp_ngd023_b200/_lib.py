@@ -48,7 +48,8 @@ class Config(C.Structure):
                 ("fake_sms", C.c_uint32), ("fake_time_scale_ns", C.c_uint32), ("event_time_kind", C.c_uint32),
                 ("lookahead", C.c_uint32), ("launch_threads", C.c_uint32),
                 ("no_proxy", C.c_uint32), ("no_pdl", C.c_uint32),
-                ("notify_mode", C.c_uint32), ("prio_classes", C.c_uint32), ("decide_delay_ns", C.c_uint32)]
+                ("notify_mode", C.c_uint32), ("prio_classes", C.c_uint32), ("online_tbar", C.c_uint32),
+                ("decide_delay_ns", C.c_uint32)]
 
 
 class Node(C.Structure):
@@ -155,7 +156,7 @@ class Engine:
                  instrument=True, naive=False, region_bytes=64 << 20, dispatcher_cpus=None,
                  event_log=None, fake_sms=0, fake_time_scale_ns=0, event_time_kind=None, lookahead=0,
                  launch_threads=0, proxy=True, pdl=True, prio_classes=1,
-                 notify="counters", decide_delay_ns=0):
+                 notify="counters", decide_delay_ns=0, online_tbar=False):
         self.lib = load()
         cfg = Config()
         cfg.abi_version = ABI_VERSION
@@ -190,6 +191,7 @@ class Engine:
         cfg.no_pdl = 0 if pdl else 1
         cfg.prio_classes = prio_classes
         cfg.decide_delay_ns = decide_delay_ns
+        cfg.online_tbar = 1 if online_tbar else 0
         # notification path: "counters" (default), "ring" (device ring + forwarding warp),
         # "direct" (the paper's direct ring writes; same as proxy=False)
         if notify not in ("counters", "ring", "direct"):

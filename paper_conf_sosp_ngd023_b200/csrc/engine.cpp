@@ -44,7 +44,7 @@ int64_t now_ns() {
 // ---------------------------------------------------------------------------
 // event log (replay input for oracle/sim.py::replay; format in DESIGN.md)
 // ---------------------------------------------------------------------------
-enum : uint32_t { EV_ARRIVAL = 1, EV_RECORD = 2, EV_BATCH_END = 3, EV_ISSUE = 4, EV_COMPLETE = 5,
+enum : uint32_t { EV_ARRIVAL = 1, EV_RECORD = 2, EV_BATCH_END = 3, EV_ISSUE = 4, EV_COMPLETE = 5, EV_OBSERVE = 6,
                   EV_CONFIG = 100, EV_CAPACITY = 101, EV_MODEL = 110, EV_LAYER = 111, EV_DEMAND = 112 };
 
 struct LogEv {
@@ -593,6 +593,8 @@ static bool admit(Gpu* g, uint32_t client, const SubmitSlot& s) {
   return true;
 }
 
+static void observe_before_record(Gpu* g, uint32_t type, uint32_t uid, uint32_t n);
+
 static uint32_t drain_ring(Gpu* g) {
   Rec* ring = g->be->ring();
   uint32_t n = 0;
@@ -614,12 +616,30 @@ static uint32_t drain_ring(Gpu* g) {
     g->head++;
     n++;
     g->stats.records++;
+    observe_before_record(g, f.type, f.uid, f.count);   // OBSERVE precedes its RECORD in the log
     logev(g, EV_RECORD, f.type, f.uid, f.count, f.gtimer | ((uint64_t)f.group << 40) | ((uint64_t)f.smid << 56));
     int64_t done = -1;
     g->policy->record(f.type, f.uid, f.count, &done);
     if (done >= 0) finish_job(g, (uint32_t)done, 0);
   }
   return n;
+}
+
+// NEXT-4 (online T-bar): before the policy consumes a record, note when a launch's
+// first PLACEMENT was seen; right before its final COMPLETION, hand the policy (and the
+// event log) the observed duration.
+static void observe_before_record(Gpu* g, uint32_t type, uint32_t uid, uint32_t n) {
+  if (!g->P->cfg.online_tbar) return;
+  const PolicyLaunch& L = g->policy->launch(uid);
+  if (!L.live || L.uid != uid) return;
+  int64_t& t0 = g->first_place_ns[uid % Gpu::kObsSlots];
+  if (type == REC_PLACEMENT && L.p == 0 && L.f == 0) t0 = now_ns();
+  if (type == REC_COMPLETION && L.f + n == L.grid) {
+    if (L.p == 0 && L.f == 0) t0 = now_ns();   // completion seen before any placement
+    const int64_t d = std::max<int64_t>(1, now_ns() - t0);
+    logev(g, EV_OBSERVE, 0, uid, (uint64_t)d, 0);
+    g->policy->observe(uid, d);
+  }
 }
 
 // Counter mode, relaxed exits: a launch of a live job completed; if that left the job
@@ -675,6 +695,7 @@ static uint32_t drain_counters(Gpu* g) {
         *seen[t] = end;
         n++;
         g->stats.records++;
+        observe_before_record(g, type, L.uid, cnt_g);   // OBSERVE precedes its RECORD in the log
         logev(g, EV_RECORD, type, L.uid, cnt_g, ((uint64_t)grp << 40) | (0xFFull << 56));
         int64_t done = -1;
         const bool complete = g->policy->record(type, L.uid, cnt_g, &done);
@@ -970,6 +991,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     pc.streams = cfg.stream_pool;
     pc.lookahead = cfg.lookahead;
     pc.prio_classes = cfg.naive ? 1 : cfg.prio_classes;
+    pc.online_tbar = cfg.online_tbar;
     for (int r = 0; r < NRES; ++r) pc.capacity[r] = P->capacity[r];
     if (cfg.device == PAELLA_DEVICE_CUDA &&
         (static_cast<CudaBackend*>(g->be.get())->proxy || static_cast<CudaBackend*>(g->be.get())->mirror)) {
@@ -997,6 +1019,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
             ((uint64_t)P->cfg.slack_blocks << 32) | cfg.group_size);
       logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFFu, cfg.ring_capacity, cfg.stream_pool,
             ((uint64_t)pc.prio_classes << 32) | cfg.lookahead);
+      logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFEu, cfg.online_tbar, 0, 0);
       for (int r = 0; r < NRES; ++r) logev(g.get(), EV_CAPACITY, (uint32_t)r, (uint64_t)pc.capacity[r], 0, 0);
     }
     P->gpus.push_back(std::move(g));

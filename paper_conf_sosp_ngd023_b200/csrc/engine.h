@@ -159,6 +159,8 @@ struct Backend {
 };
 
 struct Gpu {
+  static constexpr uint32_t kObsSlots = 8192;   // = Policy::kLaunchSlots
+  std::vector<int64_t> first_place_ns = std::vector<int64_t>(kObsSlots, 0);   // NEXT-4
   Paella* P = nullptr;
   uint32_t index = 0;       // instance-local index
   int device = 0;           // CUDA ordinal

@@ -17,6 +17,9 @@ Policy::Policy(const Cfg& c) : cfg_(c) {
   per_client_.resize(c.num_clients);
   models_.resize(kMaxModels);   // never reallocated: models are added while dispatching
   model_total_.assign(kMaxModels, 0);
+  tb_sum_.resize(kMaxModels);
+  tb_cnt_.resize(kMaxModels);
+  live_by_model_.resize(kMaxModels);
 }
 
 void Policy::add_model(uint32_t mid, const std::vector<PolicyLayer>& layers) {
@@ -25,6 +28,9 @@ void Policy::add_model(uint32_t mid, const std::vector<PolicyLayer>& layers) {
   int64_t t = 0;
   for (const auto& l : layers) t += l.tbar;
   model_total_[mid] = t;
+  tb_sum_[mid].assign(layers.size(), 0);
+  tb_cnt_[mid].assign(layers.size(), kProfileRuns);
+  for (size_t l = 0; l < layers.size(); ++l) tb_sum_[mid][l] = layers[l].tbar * kProfileRuns;
   if (!layers.empty()) {
     auto it = std::lower_bound(totals_.begin(), totals_.end(), t);
     if (it == totals_.end() || *it != t) totals_.insert(it, t);
@@ -67,6 +73,36 @@ void Policy::refresh(PolicyJob& j) {
   else if (!r && j.in_ready) make_unready(j);
 }
 
+void Policy::observe(uint32_t uid, int64_t d) {
+  PolicyLaunch& L = launches_[uid % kLaunchSlots];
+  if (!L.live || L.uid != uid) throw std::runtime_error("observation for unknown launch");
+  L.obs = d;
+  L.has_obs = true;
+}
+
+// NEXT-4 (identical to oracle Policy._refine): fold the launch's observed duration into
+// the running average of its (model, layer) T-bar and shift R_j of every live job that
+// has not dispatched that layer yet by the change.
+void Policy::refine(const PolicyLaunch& L) {
+  if (!cfg_.online_tbar || !L.has_obs) return;
+  const uint32_t m = jobs_[L.job].model, lay = L.layer;
+  tb_sum_[m][lay] += L.obs;
+  tb_cnt_[m][lay] += 1;
+  const int64_t nv = tb_sum_[m][lay] / tb_cnt_[m][lay];
+  const int64_t delta = nv - models_[m][lay].tbar;
+  models_[m][lay].tbar = nv;
+  if (delta == 0) return;
+  for (uint32_t id : live_by_model_[m]) {
+    PolicyJob& j = jobs_[id];
+    if (j.cursor > lay) continue;
+    const bool rdy = j.in_ready;
+    if (rdy) make_unready(j);
+    j.R += delta;
+    work_ += delta;
+    if (rdy) make_ready(j);
+  }
+}
+
 // ready-set order key: SRPT (R_j), SJF (the model's whole-job T-bar sum), RR (uid of the
 // job's last issued kernel, -1 = never); ties (seq, id).  Identical to oracle Policy.pick.
 int64_t Policy::order_key(const PolicyJob& j) const {
@@ -103,6 +139,8 @@ void Policy::arrival(uint32_t job_id, uint32_t client, uint32_t model) {
   for (const auto& l : models_[model]) R += l.tbar;
   j.R = R;
   j.live = true;
+  j.model_pos = (uint32_t)live_by_model_[model].size();
+  live_by_model_[model].push_back(job_id);
   work_ += R;
   live_jobs_ += 1;
   refresh(j);
@@ -132,6 +170,7 @@ bool Policy::record(uint32_t type, uint32_t uid, uint32_t n, int64_t* job_done) 
     return false;
   }
   L.live = false;
+  refine(L);
   j.done += 1;
   if (j.inflight() == 0) {
     free_[L.stream / 64] |= 1ull << (L.stream % 64);
@@ -141,6 +180,10 @@ bool Policy::record(uint32_t type, uint32_t uid, uint32_t n, int64_t* job_done) 
   if (j.done == models_[j.model].size()) {
     if (j.in_ready) make_unready(j);
     j.live = false;
+    auto& lm = live_by_model_[j.model];   // swap-remove from the model's live list
+    jobs_[lm.back()].model_pos = j.model_pos;
+    lm[j.model_pos] = lm.back();
+    lm.pop_back();
     unfinished_[j.client] -= 1;
     live_jobs_ -= 1;
     *job_done = j.id;
@@ -247,6 +290,7 @@ void Policy::decide(std::vector<Issue>* out) {
     L.grid = lay.grid;
     L.stream = stream;
     L.p = L.f = 0;
+    L.has_obs = false;
     L.live = true;
     for (int r = 0; r < NRES; ++r) U_[r] += (int64_t)lay.grid * lay.demand[r];
     Q_ += lay.grid;

@@ -43,6 +43,7 @@ struct PolicyJob {
   int32_t last_stream = -1;
   uint32_t last_uid = 0;
   int64_t rr = -1;           // RR ablation: uid of the last issued kernel (-1 = never)
+  uint32_t model_pos = 0;    // index in live_by_model_[model] (NEXT-4)
   uint32_t uid_of[8] = {0};  // launch uid of layer l (l mod 8) while in flight
   bool live = false;
   bool in_ready = false;
@@ -53,6 +54,8 @@ struct PolicyLaunch {
   uint32_t uid = 0, job = 0, layer = 0, grid = 0, stream = 0;
   uint32_t p = 0, f = 0;
   bool live = false;
+  bool has_obs = false;      // NEXT-4: an observed duration is pending for this launch
+  int64_t obs = 0;
 };
 
 struct Issue {
@@ -73,7 +76,9 @@ class Policy {
     int64_t capacity[NRES] = {148 * 32, 148 * 64, 148 * 65536, 148 * 233472, 148 * 512};
     uint32_t lookahead = 0;   // NEXT-1 launch-ahead depth (0 = the paper's semantics)
     uint32_t prio_classes = 1;   // stream-priority classes (1 = the paper: one class)
+    uint32_t online_tbar = 0;    // NEXT-4: refine T-bar online (running average, P1252-1254)
   };
+  static constexpr int64_t kProfileRuns = 20;   // observations behind the profiled T-bar
   // class of stream s: consecutive index ranges, class 0 = highest hardware priority
   static uint32_t stream_class(uint32_t s, uint32_t K, uint32_t P) { return (uint32_t)((uint64_t)s * K / P); }
 
@@ -86,6 +91,9 @@ class Policy {
   void arrival(uint32_t job_id, uint32_t client, uint32_t model);
   // returns true if the launch finished; *job_done set if its job completed
   bool record(uint32_t type, uint32_t uid, uint32_t n, int64_t* job_done);
+  // NEXT-4: duration of launch uid (first PLACEMENT seen -> final COMPLETION seen),
+  // consumed right before its final COMPLETION record (logged as an OBSERVE event)
+  void observe(uint32_t uid, int64_t d);
   // dispatch loop; appends issues
   void decide(std::vector<Issue>* out);
 
@@ -108,6 +116,7 @@ class Policy {
   int lowest_free_in_class(uint32_t c) const;
   bool predicate(uint32_t grid) const;
   int64_t order_key(const PolicyJob& j) const;
+  void refine(const PolicyLaunch& L);
   void make_ready(PolicyJob& j);
   void make_unready(PolicyJob& j);
   bool is_ready(const PolicyJob& j) const;
@@ -124,6 +133,8 @@ class Policy {
   bool over_ = false;                  // the last pick was a deficit override
   std::vector<int64_t> totals_;        // sorted distinct whole-job T-bar sums of the models
   std::vector<int64_t> model_total_;   // whole-job T-bar sum per model (SJF key)
+  std::vector<std::vector<int64_t>> tb_sum_, tb_cnt_;   // NEXT-4 running averages
+  std::vector<std::vector<uint32_t>> live_by_model_;    // live job ids per model (NEXT-4)
   std::vector<uint64_t> free_;   // bitmap of free streams
   std::vector<int64_t> Dt_;
   int64_t Omega_ = 0;

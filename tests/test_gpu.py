@@ -149,13 +149,17 @@ def _serve_and_check(e, specs, n, n_clients, seed, rate_us=30.0):
     (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 3, 4, "counters", 4),  # the bench arm
     (L.POLICY_SRPT_DEFICIT, 4, 16, 4096, 2, 3, "ring", 4),
     (L.POLICY_SRPT_DEFICIT, 16, 32, 2048, 1, 2, "direct", 1),  # direct record writes (the paper's path)
+    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 3, 4, "counters", -4),  # bench arm + online T-bar (NEXT-4)
+    (L.POLICY_SJF, 16, 32, 65536, 3, 4, "counters", 1),
+    (L.POLICY_RR, 16, 8, 4096, 0, 0, "counters", 1),
 ])
 def test_serving_parity_and_replay(tmp_path, policy, group, streams, ring, look, lt, notify, prio):
     log = str(tmp_path / "gpu_%u.log")
     names = ["toy", "resnet18", "mobilenet_v2", "squeezenet1_1"]
+    online, prio = prio < 0, abs(prio)
     with L.Engine(num_clients=3, policy=policy, group=group, streams=streams, ring_capacity=ring,
                   event_log=log, max_jobs_per_model=32, lookahead=look, launch_threads=lt, notify=notify,
-                  prio_classes=prio, slack=1184 if prio > 1 else 0) as e:
+                  prio_classes=prio, slack=1184 if prio > 1 else 0, online_tbar=online) as e:
         specs = []
         for nm in names:
             g = archs.build(nm)

@@ -115,17 +115,23 @@ def _serve(e, mids, n, n_clients, seed, stride=16384, timeout=60):
     (L.POLICY_SRPT_DEFICIT, 100, 16, 8, 1, 4), (L.POLICY_SRPT_DEFICIT, 3, 4, 12, 2, 3),
     (L.POLICY_SRPT_DEFICIT, None, 16, 32, 0, 2), (L.POLICY_FIFO, 100, 16, 8, 1, 2),
     (L.POLICY_SJF, 100, 16, 8, 0, 1), (L.POLICY_SJF, 100, 4, 4, 2, 2),
-    (L.POLICY_RR, 100, 16, 8, 0, 1), (L.POLICY_RR, 100, 4, 12, 1, 3)])
+    (L.POLICY_RR, 100, 16, 8, 0, 1), (L.POLICY_RR, 100, 4, 12, 1, 3),
+    (L.POLICY_SRPT_DEFICIT, 100, 16, 8, 0, -1), (L.POLICY_SRPT_DEFICIT, None, 4, 12, 2, -3),
+    (L.POLICY_SJF, 3, 16, 8, 1, -1)])
 def test_fake_device_replay_parity(tmp_path, policy, theta, group, streams, look, prio):
+    """prio < 0: |prio| classes with NEXT-4 online T-bar refinement (OBSERVE events)."""
     log = str(tmp_path / "ev_%u.log")
     models = [archs.toy(), archs.squeezenet1_1()]
+    online, prio = prio < 0, abs(prio)
     with _toy_engine(num_clients=3, policy=policy, theta=theta, group=group, streams=streams,
-                     event_log=log, ring_capacity=1024, slack=8, lookahead=look, prio_classes=prio) as e:
+                     event_log=log, ring_capacity=1024, slack=8, lookahead=look, prio_classes=prio,
+                     online_tbar=online) as e:
         mids = [e.register_model(g, rng.model_params(g)) for g in models]
         _serve(e, mids, 300, 3, seed=policy * 10 + group)
     cfg, ms, events, ex = eventlog.read(log % 0)
     assert cfg.num_clients == 3 and cfg.policy == policy and cfg.group == group and cfg.lookahead == look
-    assert cfg.prio_classes == prio
+    assert cfg.prio_classes == prio and cfg.online_tbar == int(online)
+    assert any(ev[0] == sim.EV_OBSERVE for ev in events) == online
     ok, msg, n = sim.replay(cfg, ms, events)
     assert ok, msg
     assert n == len(ex["issues"]) > 0 and ex["n_arrivals"] == 300 == len(ex["completes"])

@@ -413,3 +413,47 @@ def test_rr_closed_form(n, k):
     cfg2 = single_server_cfg()
     res2 = sim.simulate(cfg2, models, trace, ONE_SM)
     assert sum(res2.jct().values()) == (k * n * (n + 1) // 2) * UNIT
+
+
+# --- NEXT-4: online T-bar refinement (running average, P1249-1266) -------------------
+
+def test_online_tbar_running_average_and_remaining_invariant():
+    """T-bar of a layer = integer mean of the PROFILE_RUNS profiled observations and
+    every observed duration; R_j of every live job stays the sum of the current T-bar
+    over its undispatched kernels (so it reaches exactly 0 at its last issue)."""
+    layers = [Layer(1, (1, 1, 1, 1, 0), t) for t in (1000, 3000, 5000)]
+    cfg = Config(num_clients=1, theta=sim.INF_THETA, slack=0, streams=8, online_tbar=1)
+    pol = sim.Policy(cfg, [layers])
+    for jid in range(3):
+        pol.arrival(jid, 0, 0)
+    obs = {}
+    for step in range(40):
+        for (uid, job, layer, stream) in pol.decide():
+            obs[uid] = (job, layer)
+        if not pol.launches:
+            break
+        uid = min(pol.launches)
+        job, layer = obs[uid]
+        d = 2000 + 700 * layer + 13 * uid
+        before_sum = pol.tb_sum[0][layer]
+        pol.observe(uid, d)
+        pol.record(sim.PLACEMENT, uid, 1)
+        pol.record(sim.COMPLETION, uid, 1)
+        assert pol.tb_sum[0][layer] == before_sum + d
+        assert pol.tb[0][layer] == pol.tb_sum[0][layer] // pol.tb_cnt[0][layer]
+        for j in pol.jobs.values():
+            assert j.R == pol.remaining(0, j.cursor)
+    assert pol.completed == [0, 1, 2] or sorted(pol.completed) == [0, 1, 2]
+    # closed form for the first layer: 3 observations on top of 20 profiled runs
+    ds = [2000 + 13 * u for u, (jb, ly) in obs.items() if ly == 0]
+    assert pol.tb[0][0] == (1000 * sim.PROFILE_RUNS + sum(ds)) // (sim.PROFILE_RUNS + len(ds))
+
+
+def test_online_tbar_off_keeps_profile():
+    layers = [Layer(1, (1, 1, 1, 1, 0), 1000)]
+    pol = sim.Policy(Config(num_clients=1, slack=0), [layers])
+    pol.arrival(0, 0, 0)
+    (uid, _, _, _), = pol.decide()
+    pol.observe(uid, 99999)
+    pol.record(sim.COMPLETION, uid, 1)
+    assert pol.tb[0][0] == 1000
