@@ -58,6 +58,8 @@ extern "C" {
 /* routing across GPUs */
 #define PAELLA_ROUTE_LEAST_WORK    0u
 #define PAELLA_ROUTE_ROUND_ROBIN   1u
+#define PAELLA_ROUTE_POWER_OF_TWO  2u   /* power-of-two choices: the lower W_g of two GPUs
+                                          drawn from the request id (paella_route_pair) */
 
 /* device backends */
 #define PAELLA_DEVICE_CUDA 0u   /* real sm_100a GPUs */
@@ -233,6 +235,16 @@ int64_t paella_poll_completion(paella_t* p, uint32_t client_id, uint32_t flags, 
    PAELLA_HYBRID: spin, then futex sleep between the dispatcher's hints (above);
    otherwise spins until one is available.  *status (if non-NULL): 0 ok, -EIO CUDA
    error on that GPU, -ECANCELED shutdown. */
+
+int paella_route_pair(uint64_t req_id, uint32_t num_gpus, uint32_t* g0, uint32_t* g1);
+/* The two candidate GPUs of PAELLA_ROUTE_POWER_OF_TWO (SURVEY.md §8(e) "Variants:
+   round-robin, power-of-two-choices"; the paper routes nothing, it serves one GPU,
+   P1024-1033).  Pure and deterministic: h = splitmix64(req_id) (one output of the
+   generator seeded with req_id), *g0 = h mod num_gpus, *g1 = (*g0 + 1 + (h >> 32)
+   mod (num_gpus - 1)) mod num_gpus, so *g0 != *g1 when num_gpus > 1 (both 0 when
+   num_gpus == 1).  paella_submit sends the request to the candidate with the lower
+   published outstanding work W_g (+ unadmitted estimate), ties to the lower index.
+   -EINVAL num_gpus == 0 or > PAELLA_MAX_GPUS or a NULL output. */
 
 int paella_shutdown(paella_t* p);
 /* Stop admitting; drain in-flight kernels; requests not yet admitted complete with

@@ -584,3 +584,35 @@ def deficit_bound_holds(trace_of_D, N, theta):
             if d > max(d0, theta * N) + N:
                 bad.append((c, d0, d))
     return bad
+
+
+# --- multi-GPU routing variant ---------------------------------
+
+M64 = (1 << 64) - 1
+
+
+def splitmix64(state):
+    """One output of Vigna's SplitMix64 generator from ``state`` (the state is
+    advanced by the golden gamma, then mixed)."""
+    z = (state + 0x9E3779B97F4A7C15) & M64
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & M64
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & M64
+    return z ^ (z >> 31)
+
+
+def route_pair(req_id, num_gpus):
+    """Power-of-two-choices candidates of request ``req_id`` (SURVEY.md §8(e),
+    ``include/paella.h`` paella_route_pair): two distinct GPUs drawn from one
+    SplitMix64 output of the request id."""
+    if num_gpus == 1:
+        return 0, 0
+    h = splitmix64(req_id)
+    g0 = h % num_gpus
+    g1 = (g0 + 1 + (h >> 32) % (num_gpus - 1)) % num_gpus
+    return g0, g1
+
+
+def route_pick(pair, W):
+    """The candidate with the lower outstanding work W[g]; ties to the lower index."""
+    lo, hi = min(pair), max(pair)
+    return hi if W[hi] < W[lo] else lo

@@ -19,7 +19,7 @@ LIB_PATH = os.path.join(HERE, "libpaella.so")
 ABI_VERSION = 1
 NOTIFY_COUNTERS, NOTIFY_RING = 0, 1
 POLICY_SRPT_DEFICIT, POLICY_FIFO, POLICY_SJF, POLICY_RR = 0, 1, 2, 3
-ROUTE_LEAST_WORK, ROUTE_ROUND_ROBIN = 0, 1
+ROUTE_LEAST_WORK, ROUTE_ROUND_ROBIN, ROUTE_POWER_OF_TWO = 0, 1, 2
 DEVICE_CUDA, DEVICE_FAKE = 0, 1
 DTYPE_BF16, DTYPE_FP32 = 0, 1
 NONBLOCK = 1
@@ -34,7 +34,7 @@ SYMBOLS = ["paella_init", "paella_register_model", "paella_submit", "paella_subm
            "paella_poll_completion", "paella_shutdown", "paella_client_region", "paella_model_info",
            "paella_kernel_info", "paella_kernel_name", "paella_stats", "paella_flush_log",
            "paella_run_isolated", "paella_debug_node", "paella_time_kernels", "paella_bench_empty",
-           "paella_bench_roundtrip", "paella_loadgen", "paella_bench_wait"]
+           "paella_bench_roundtrip", "paella_loadgen", "paella_bench_wait", "paella_route_pair"]
 
 
 class Config(C.Structure):
@@ -114,6 +114,7 @@ def load():
     lib.paella_poll_completion.argtypes = [P, C.c_uint32, C.c_uint32, C.POINTER(C.c_int32)]
     lib.paella_poll_completion.restype = C.c_int64
     lib.paella_shutdown.argtypes = [P]
+    lib.paella_route_pair.argtypes = [C.c_uint64, C.c_uint32, C.POINTER(C.c_uint32), C.POINTER(C.c_uint32)]
     lib.paella_client_region.argtypes = [P, C.c_uint32, C.POINTER(P), C.POINTER(C.c_size_t)]
     lib.paella_model_info.argtypes = [P, C.c_uint32, C.POINTER(ModelInfo)]
     lib.paella_kernel_info.argtypes = [P, C.c_uint32, C.c_uint32, C.POINTER(KernelInfo)]
@@ -145,6 +146,13 @@ def _check(rc, what):
 
 def _fptr(a):
     return a.ctypes.data_as(C.POINTER(C.c_float)) if a is not None else None
+
+
+def route_pair(req_id, num_gpus):
+    """``paella_route_pair``: the two candidate GPUs of ROUTE_POWER_OF_TWO."""
+    g0, g1 = C.c_uint32(), C.c_uint32()
+    _check(load().paella_route_pair(req_id, num_gpus, C.byref(g0), C.byref(g1)), "paella_route_pair")
+    return g0.value, g1.value
 
 
 class Engine:

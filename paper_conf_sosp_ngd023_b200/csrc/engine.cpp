@@ -1099,6 +1099,21 @@ int paella_register_model(paella_t* p, const paella_model_desc_t* desc, uint32_t
   return 0;
 }
 
+int paella_route_pair(uint64_t req_id, uint32_t num_gpus, uint32_t* g0, uint32_t* g1) {
+  if (num_gpus == 0 || num_gpus > PAELLA_MAX_GPUS || !g0 || !g1) return -EINVAL;
+  uint64_t z = req_id + 0x9E3779B97F4A7C15ull;   // splitmix64, one step from state req_id
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  z ^= z >> 31;
+  if (num_gpus == 1) {
+    *g0 = *g1 = 0;
+    return 0;
+  }
+  *g0 = (uint32_t)(z % num_gpus);
+  *g1 = (uint32_t)((*g0 + 1 + (z >> 32) % (num_gpus - 1)) % num_gpus);
+  return 0;
+}
+
 static int64_t submit_impl(Paella* P, uint32_t client_id, uint32_t model_id, void* io, size_t len, uint32_t flags,
                            int64_t t_sched) {
   if (!P) return -EINVAL;
@@ -1111,19 +1126,29 @@ static int64_t submit_impl(Paella* P, uint32_t client_id, uint32_t model_id, voi
   if (b < base || b + len > base + P->region_bytes || b + len < b) return -EFAULT;
   if (len < m->input_bytes + m->output_bytes) return -EINVAL;
   if (((uintptr_t)io & 15) != 0) return -EINVAL;
+  uint64_t seq = P->client_seq[client_id]->fetch_add(1);
+  uint64_t req_id = ((uint64_t)client_id << 48) | (seq & ((1ull << 48) - 1));
   // route: least outstanding work, ties to the lowest index
   uint32_t gsel = 0;
   uint32_t ng = (uint32_t)P->gpus.size();
+  auto work_of = [&](uint32_t g) {
+    Gpu* Gg = P->gpus[g].get();
+    int64_t pending = (int64_t)(Gg->submitted.load(std::memory_order_relaxed) -
+                                Gg->admitted_pub.load(std::memory_order_acquire));
+    return Gg->work_published.load(std::memory_order_acquire) + pending * m->total_tbar;
+  };
   if (ng > 1) {
     if (P->cfg.route == PAELLA_ROUTE_ROUND_ROBIN) {
       gsel = P->rr_next[client_id]++ % ng;
+    } else if (P->cfg.route == PAELLA_ROUTE_POWER_OF_TWO) {
+      uint32_t g0, g1;
+      paella_route_pair(req_id, ng, &g0, &g1);
+      uint32_t lo = g0 < g1 ? g0 : g1, hi = g0 < g1 ? g1 : g0;
+      gsel = work_of(hi) < work_of(lo) ? hi : lo;
     } else {
       int64_t best = INT64_MAX;
       for (uint32_t g = 0; g < ng; ++g) {
-        Gpu* G = P->gpus[g].get();
-        int64_t pending = (int64_t)(G->submitted.load(std::memory_order_relaxed) -
-                                    G->admitted_pub.load(std::memory_order_acquire));
-        int64_t w = G->work_published.load(std::memory_order_acquire) + pending * m->total_tbar;
+        int64_t w = work_of(g);
         if (w < best) {
           best = w;
           gsel = g;
@@ -1133,8 +1158,7 @@ static int64_t submit_impl(Paella* P, uint32_t client_id, uint32_t model_id, voi
   }
   Gpu* G = P->gpus[gsel].get();
   SubmitSlot s{};
-  uint64_t seq = P->client_seq[client_id]->fetch_add(1);
-  s.req_id = ((uint64_t)client_id << 48) | (seq & ((1ull << 48) - 1));
+  s.req_id = req_id;
   s.model_id = model_id;
   s.flags = flags;
   s.io_off = (uint64_t)(b - base);

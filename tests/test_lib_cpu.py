@@ -154,7 +154,7 @@ def test_fake_replay_with_job_id_reuse(tmp_path):
     assert ok and n == 3000, msg
 
 
-@pytest.mark.parametrize("route", [L.ROUTE_LEAST_WORK, L.ROUTE_ROUND_ROBIN])
+@pytest.mark.parametrize("route", [L.ROUTE_LEAST_WORK, L.ROUTE_ROUND_ROBIN, L.ROUTE_POWER_OF_TWO])
 def test_router_multi_gpu_fake(tmp_path, route):
     log = str(tmp_path / "ev_%u.log")
     g = archs.toy()
@@ -165,7 +165,7 @@ def test_router_multi_gpu_fake(tmp_path, route):
     assert sum(per) == 400
     if route == L.ROUTE_ROUND_ROBIN:
         assert max(per) - min(per) <= 2 and min(per) > 0
-    else:   # least outstanding work, ties to the lowest index: a burst spreads out
+    else:   # least outstanding work (of all GPUs or of two candidates): a burst spreads out
         assert sum(1 for x in per if x > 0) >= 2
     for gi in range(4):   # every per-GPU dispatcher replays exactly
         cfg, ms, events, ex = eventlog.read(log % gi)
@@ -232,3 +232,18 @@ def test_bench_wait_spin_vs_hybrid_fake():
     assert (j0 > 0).all() and (j1 > 0).all()
     assert hyb < 0.5 * spin, (hyb, spin)
     e.shutdown()
+
+
+def test_route_pair_matches_oracle():
+    """paella_route_pair (power-of-two choices) is bit-exact with the
+    oracle's independent SplitMix64 derivation on every GPU count, and rejects bad
+    arguments."""
+    from oracle import sim
+    r = np.random.default_rng(5)
+    ids = [0, 1, (1 << 48) - 1, (63 << 48) | 12345] + [int(x) for x in r.integers(0, 1 << 62, 2000)]
+    for ng in range(1, 9):
+        for rid in ids:
+            assert L.route_pair(rid, ng) == sim.route_pair(rid, ng), (rid, ng)
+    for ng in (0, 9):
+        with pytest.raises(OSError):
+            L.route_pair(1, ng)

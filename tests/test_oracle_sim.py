@@ -457,3 +457,30 @@ def test_online_tbar_off_keeps_profile():
     pol.observe(uid, 99999)
     pol.record(sim.COMPLETION, uid, 1)
     assert pol.tb[0][0] == 1000
+
+
+def test_splitmix64_published_outputs():
+    """Pin of sim.splitmix64: the first outputs of Vigna's reference splitmix64.c
+    seeded with 0 are 0xE220A8397B1DCDAF, 0x6E789E6AA1B965F4, 0x06C45D188009454F
+    (state advances by the gamma 0x9E3779B97F4A7C15 per output)."""
+    g = 0x9E3779B97F4A7C15
+    want = [0xE220A8397B1DCDAF, 0x6E789E6AA1B965F4, 0x06C45D188009454F]
+    assert [sim.splitmix64((k * g) & sim.M64) for k in range(3)] == want
+
+
+def test_route_pair_candidates_valid_and_spread():
+    """Power-of-two choices: two distinct in-range candidates; over
+    many request ids every unordered pair of 8 GPUs is drawn about equally often;
+    the pick is the lower-W candidate with ties to the lower index."""
+    from collections import Counter
+    for ng in range(2, 9):
+        for rid in range(500):
+            a, b = sim.route_pair(rid, ng)
+            assert 0 <= a < ng and 0 <= b < ng and a != b
+    assert sim.route_pair(123, 1) == (0, 0)
+    cnt = Counter(frozenset(sim.route_pair(rid, 8)) for rid in range(28000))
+    assert len(cnt) == 28
+    assert all(700 <= v <= 1300 for v in cnt.values()), cnt
+    assert sim.route_pick((5, 2), [0, 0, 7, 0, 0, 3, 0, 0]) == 5
+    assert sim.route_pick((5, 2), [0, 0, 3, 0, 0, 3, 0, 0]) == 2
+    assert sim.route_pick((2, 5), [0, 0, 1, 0, 0, 3, 0, 0]) == 2
