@@ -17,6 +17,8 @@ Format (DESIGN.md §"Event log"): a sequence of 32-byte little-endian records
     4 ISSUE     a=stream, b=uid, c=job, d=layer
     5 COMPLETE  b=job, c=t ns
     6 OBSERVE   b=uid, c=observed duration ns (NEXT-4; precedes the final COMPLETION)
+    7 ROUTE     a=g0 | g1 << 8 | route << 16, b=req_id, c=W_g0, d=W_g1 (multi-GPU only;
+                the router's decision inputs, logged by the GPU it chose, before ARRIVAL)
 """
 import numpy as np
 
@@ -38,6 +40,7 @@ def read(path):
     records = []
     issues = []
     completes = []
+    routes = []
     narrivals = 0
     for r in raw:
         t, a, b, c, d = int(r["type"]), int(r["a"]), int(r["b"]), int(r["c"]), int(r["d"])
@@ -76,6 +79,9 @@ def read(path):
         elif t == 4:
             events.append((sim.EV_ISSUE, b, c, d, a))
             issues.append((b, c, d, a, arrivals[c][1]))   # (uid, job, layer, stream, model)
+        elif t == 7:
+            routes.append((a & 0xFF, (a >> 8) & 0xFF, a >> 16, b,
+                           c if c < (1 << 63) else c - (1 << 64), d if d < (1 << 63) else d - (1 << 64)))
         elif t == 6:
             events.append((sim.EV_OBSERVE, b, c))
         elif t == 5:
@@ -91,5 +97,5 @@ def read(path):
             ms.append(sim.Layer(grid, (1, w, rg, sm, tm), tbar))
         models.append(ms)
     extras = dict(records=records, issues=issues, completes=completes, arrivals=arrivals,
-                  n_arrivals=narrivals)
+                  n_arrivals=narrivals, routes=routes)
     return cfg, models, events, extras

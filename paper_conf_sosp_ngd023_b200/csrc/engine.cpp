@@ -44,7 +44,7 @@ int64_t now_ns() {
 // ---------------------------------------------------------------------------
 // event log (replay input for oracle/sim.py::replay; format in DESIGN.md)
 // ---------------------------------------------------------------------------
-enum : uint32_t { EV_ARRIVAL = 1, EV_RECORD = 2, EV_BATCH_END = 3, EV_ISSUE = 4, EV_COMPLETE = 5, EV_OBSERVE = 6,
+enum : uint32_t { EV_ARRIVAL = 1, EV_RECORD = 2, EV_BATCH_END = 3, EV_ISSUE = 4, EV_COMPLETE = 5, EV_OBSERVE = 6, EV_ROUTE = 7,
                   EV_CONFIG = 100, EV_CAPACITY = 101, EV_MODEL = 110, EV_LAYER = 111, EV_DEMAND = 112 };
 
 struct LogEv {
@@ -564,6 +564,7 @@ static bool admit(Gpu* g, uint32_t client, const SubmitSlot& s) {
   args.front().in = j.io;                           // ingest reads client memory
   args.back().out = j.io + m->input_bytes;           // last kernel writes the logits in place
   g->stats.admitted++;
+  if (P->gpus.size() > 1) logev(g, EV_ROUTE, s.route_meta, s.req_id, (uint64_t)s.route_w[0], (uint64_t)s.route_w[1]);
   logev(g, EV_ARRIVAL, client, jid, s.model_id, (uint64_t)s.t_sched_ns);
   if (P->cfg.naive) {
     // CUDA-MS baseline: every kernel of the job enters stream jid % P now
@@ -1137,14 +1138,22 @@ static int64_t submit_impl(Paella* P, uint32_t client_id, uint32_t model_id, voi
                                 Gg->admitted_pub.load(std::memory_order_acquire));
     return Gg->work_published.load(std::memory_order_acquire) + pending * m->total_tbar;
   };
+  SubmitSlot s{};
   if (ng > 1) {
+    // the decision and its W snapshot travel in the slot and are logged at admission
+    // (ROUTE event) so the routing replays: (g0, g1, W_g0, W_g1) for power-of-two,
+    // (chosen, runner-up or chosen, W of both) otherwise
+    uint32_t g0 = 0, g1 = 0;
     if (P->cfg.route == PAELLA_ROUTE_ROUND_ROBIN) {
-      gsel = P->rr_next[client_id]++ % ng;
+      gsel = g0 = g1 = P->rr_next[client_id]++ % ng;
+      s.route_w[0] = s.route_w[1] = work_of(gsel);
     } else if (P->cfg.route == PAELLA_ROUTE_POWER_OF_TWO) {
-      uint32_t g0, g1;
       paella_route_pair(req_id, ng, &g0, &g1);
+      s.route_w[0] = work_of(g0);
+      s.route_w[1] = work_of(g1);
       uint32_t lo = g0 < g1 ? g0 : g1, hi = g0 < g1 ? g1 : g0;
-      gsel = work_of(hi) < work_of(lo) ? hi : lo;
+      int64_t wlo = lo == g0 ? s.route_w[0] : s.route_w[1], whi = hi == g0 ? s.route_w[0] : s.route_w[1];
+      gsel = whi < wlo ? hi : lo;
     } else {
       int64_t best = INT64_MAX;
       for (uint32_t g = 0; g < ng; ++g) {
@@ -1154,10 +1163,12 @@ static int64_t submit_impl(Paella* P, uint32_t client_id, uint32_t model_id, voi
           gsel = g;
         }
       }
+      g0 = g1 = gsel;
+      s.route_w[0] = s.route_w[1] = best;
     }
+    s.route_meta = g0 | (g1 << 8) | (P->cfg.route << 16);
   }
   Gpu* G = P->gpus[gsel].get();
-  SubmitSlot s{};
   s.req_id = req_id;
   s.model_id = model_id;
   s.flags = flags;

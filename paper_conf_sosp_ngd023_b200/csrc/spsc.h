@@ -21,7 +21,9 @@ struct alignas(64) SubmitSlot {     // 64 B, SURVEY.md §8(a) a1
   uint64_t io_off;                  // offset of io inside the client's region
   uint64_t len;
   int64_t t_sched_ns;               // scheduled arrival (CLOCK_MONOTONIC)
-  uint64_t pad[3];
+  int64_t route_w[2];               // router's W snapshot of the two candidates (ng > 1)
+  uint32_t route_meta;              // g0 | g1 << 8 | route << 16 (ng > 1), logged as ROUTE
+  uint32_t pad;
 };
 static_assert(sizeof(SubmitSlot) == 64, "slot size");
 

@@ -167,10 +167,20 @@ def test_router_multi_gpu_fake(tmp_path, route):
         assert max(per) - min(per) <= 2 and min(per) > 0
     else:   # least outstanding work (of all GPUs or of two candidates): a burst spreads out
         assert sum(1 for x in per if x > 0) >= 2
+    nroutes = 0
     for gi in range(4):   # every per-GPU dispatcher replays exactly
         cfg, ms, events, ex = eventlog.read(log % gi)
         ok, msg, n = sim.replay(cfg, ms, events)
         assert ok, (gi, msg)
+        for g0, g1, r, rid, w0, w1 in ex["routes"]:   # the routing decisions replay too
+            assert r == route
+            if route == L.ROUTE_POWER_OF_TWO:
+                assert (g0, g1) == sim.route_pair(rid, 4)
+                assert sim.route_pick((g0, g1), {g0: w0, g1: w1}) == gi
+            else:
+                assert g0 == g1 == gi
+        nroutes += len(ex["routes"])
+    assert nroutes == 400
 
 
 def test_shutdown_cancels_unadmitted():
