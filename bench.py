@@ -62,6 +62,10 @@ def parse():
                     help="injected scheduler delay before every decide pass (Fig. 9 sensitivity)")
     ap.add_argument("--theta", type=int, default=100, help="fairness threshold (kernel dispatches, P1296-1297)")
     ap.add_argument("--prio-classes", type=int, default=1, help="stream-priority classes (DESIGN.md B200-Q2)")
+    ap.add_argument("--dispatcher-cpu", type=int, default=-1,
+                    help="pin each rank's dispatcher to core (this + LOCAL_RANK); -1 = unpinned")
+    ap.add_argument("--dispatcher-fifo", type=int, default=0,
+                    help="SCHED_FIFO priority of the pinned dispatcher (0 = SCHED_OTHER)")
     ap.add_argument("--launch-threads", type=int, default=4, help="launcher helper threads per GPU")
     ap.add_argument("--sat-reqs", type=int, default=1500, help="requests of the saturation calibration")
     ap.add_argument("--slo-rhos", default="0.5,0.7,0.9,1.0,1.1,1.2,1.35,1.5",
@@ -256,6 +260,8 @@ def run_gpu(args, dist):
 
     def engine(**kw):
         kw.setdefault("launch_threads", 0 if args.fake else args.launch_threads)
+        if args.dispatcher_cpu >= 0:
+            kw.setdefault("dispatcher_cpus", [args.dispatcher_cpu + gpu])
         if not kw.get("naive"):
             kw.setdefault("policy", {"srpt": L.POLICY_SRPT_DEFICIT, "fifo": L.POLICY_FIFO, "sjf": L.POLICY_SJF,
                                      "rr": L.POLICY_RR}[args.policy])
@@ -471,6 +477,8 @@ def saturating_conv(args):
 
 def main():
     args = parse()
+    if args.dispatcher_fifo > 0:
+        os.environ["PAELLA_DISPATCHER_FIFO"] = str(args.dispatcher_fifo)
     dist = Dist(args.gpus)
     cfg = traces.CONFIGS[args.config]
     workload = {"c2_mix": "BASELINE configs[1]: 1 GPU, mixed ResNet-18/MobileNetV2/SqueezeNet1.1 batch-1, "
@@ -522,7 +530,8 @@ def main():
                    "l2": "not flushed: steps are open-loop traces whose weights (~33 MB bf16) stay L2-resident "
                          "as in serving; inputs stream from pinned host memory"},
         "jct_us": res["jct"], "slo_us": res["slo"],
-        "paella_config": {"lookahead": args.lookahead, "launch_threads": args.launch_threads, "policy": {"srpt": "srpt+deficit"}.get(args.policy, args.policy),
+        "paella_config": {"lookahead": args.lookahead, "launch_threads": args.launch_threads,
+                          "dispatcher_cpu": args.dispatcher_cpu, "dispatcher_fifo": args.dispatcher_fifo, "policy": {"srpt": "srpt+deficit"}.get(args.policy, args.policy),
                           "slack_blocks": args.slack, "prio_classes": args.prio_classes, "pdl": True,
                           "theta": args.theta, "group": 16, "streams": 32, "decide_delay_ns": args.decide_delay_ns,
                           "online_tbar": bool(args.online_tbar)},

@@ -767,6 +767,15 @@ static void dispatcher_main(Gpu* g) {
     CPU_ZERO(&cs);
     CPU_SET(P->cfg.dispatcher_cpus[g->index], &cs);
     pthread_setaffinity_np(pthread_self(), sizeof cs, &cs);
+    // a dedicated core with SCHED_FIFO (PAELLA_DISPATCHER_FIFO=<prio>);
+    // only with a pinned core, so the spinning dispatcher cannot starve migrating threads
+    if (const char* fifo = std::getenv("PAELLA_DISPATCHER_FIFO")) {
+      sched_param sp{};
+      sp.sched_priority = atoi(fifo);
+      int rc = pthread_setschedparam(pthread_self(), SCHED_FIFO, &sp);
+      if (rc) fprintf(stderr, "[paella] dispatcher %u: SCHED_FIFO %d refused (%s)\n", g->index, sp.sched_priority,
+                      strerror(rc));
+    }
   }
   const uint32_t N = P->cfg.num_clients;
   if (P->cfg.device == PAELLA_DEVICE_CUDA && P->cfg.event_time_kind) {
