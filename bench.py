@@ -479,6 +479,11 @@ def main():
     args = parse()
     if args.dispatcher_fifo > 0:
         os.environ["PAELLA_DISPATCHER_FIFO"] = str(args.dispatcher_fifo)
+    if args.dispatcher_cpu >= 0:
+        # a DEDICATED core: every thread created from here on (launchers, load
+        # generator, completion pollers) inherits a mask without the dispatcher's core
+        core = args.dispatcher_cpu + int(os.environ.get("LOCAL_RANK", "0"))
+        os.sched_setaffinity(0, os.sched_getaffinity(0) - {core})
     dist = Dist(args.gpus)
     cfg = traces.CONFIGS[args.config]
     workload = {"c2_mix": "BASELINE configs[1]: 1 GPU, mixed ResNet-18/MobileNetV2/SqueezeNet1.1 batch-1, "
