@@ -62,8 +62,9 @@ def parse():
                     help="injected scheduler delay before every decide pass (Fig. 9 sensitivity)")
     ap.add_argument("--theta", type=int, default=100, help="fairness threshold (kernel dispatches, P1296-1297)")
     ap.add_argument("--prio-classes", type=int, default=1, help="stream-priority classes (DESIGN.md B200-Q2)")
-    ap.add_argument("--dispatcher-cpu", type=int, default=-1,
-                    help="pin each rank's dispatcher to core (this + LOCAL_RANK); -1 = unpinned")
+    ap.add_argument("--dispatcher-cpu", type=int, default=-2,
+                    help="pin each rank's dispatcher to core (this + LOCAL_RANK), exclusive; -1 = unpinned; "
+                         "default: 2 when the host has >= 2 + 2N cores")
     ap.add_argument("--dispatcher-fifo", type=int, default=0,
                     help="SCHED_FIFO priority of the pinned dispatcher (0 = SCHED_OTHER)")
     ap.add_argument("--launch-threads", type=int, default=4, help="launcher helper threads per GPU")
@@ -479,11 +480,17 @@ def main():
     args = parse()
     if args.dispatcher_fifo > 0:
         os.environ["PAELLA_DISPATCHER_FIFO"] = str(args.dispatcher_fifo)
+    if args.dispatcher_cpu == -2:   # default: core 2 + LOCAL_RANK if the host has room
+        avail = os.sched_getaffinity(0)
+        first = 2
+        args.dispatcher_cpu = first if (set(range(first, first + args.gpus)) <= avail
+                                         and len(avail) >= first + 2 * args.gpus) else -1
     if args.dispatcher_cpu >= 0:
-        # a DEDICATED core: every thread created from here on (launchers, load
-        # generator, completion pollers) inherits a mask without the dispatcher's core
-        core = args.dispatcher_cpu + int(os.environ.get("LOCAL_RANK", "0"))
-        os.sched_setaffinity(0, os.sched_getaffinity(0) - {core})
+        # DEDICATED cores: every thread created from here on
+        # (launchers, load generator, completion pollers) inherits a mask without any
+        # rank's dispatcher core; measured on B200 in profiles/pin_r1c
+        cores = set(range(args.dispatcher_cpu, args.dispatcher_cpu + args.gpus))
+        os.sched_setaffinity(0, os.sched_getaffinity(0) - cores)
     dist = Dist(args.gpus)
     cfg = traces.CONFIGS[args.config]
     workload = {"c2_mix": "BASELINE configs[1]: 1 GPU, mixed ResNet-18/MobileNetV2/SqueezeNet1.1 batch-1, "
