@@ -10,6 +10,7 @@
 * the naive baseline path produces the same outputs;
 * ring wrap-around (small ring, many laps), G = 1, a single stream.
 """
+import os
 import time
 
 import numpy as np
@@ -250,3 +251,30 @@ def test_per_sm_capacity_from_g1_records(tmp_path):
                 u[r] -= d[r]
     for r in range(5):
         assert worst[r] <= per_sm[r], (r, worst)
+
+
+@pytest.mark.gpu
+def test_serving_parity_c3_models_bench_arm(tmp_path):
+    """C-3's models (ResNet-50, DenseNet-121, Inception-v3, MobileNetV2) served
+    concurrently in the launch configuration bench.py times (launch-ahead 3, 4 launcher
+    threads, counter notification, B = 8x148, dispatcher on its own core): every output
+    within the bf16 tolerance of the float64 oracle and the issue order replayed."""
+    log = str(tmp_path / "gpu_%u.log")
+    names = ["resnet50", "densenet121", "inception_v3", "mobilenet_v2"]
+    for nm in names:   # the float64 references first: the serving loop has a 120 s bound
+        for i in range(4):
+            oracle_out(nm, i, "bf16")
+    cpus = sorted(os.sched_getaffinity(0))
+    with L.Engine(num_clients=4, event_log=log, max_jobs_per_model=32, lookahead=3, launch_threads=4,
+                  slack=1184, dispatcher_cpus=[cpus[min(2, len(cpus) - 1)]]) as e:
+        specs = []
+        for nm in names:
+            g = archs.build(nm)
+            specs.append((e.register_model(g, rng.model_params(g)), nm, g))
+        _serve_and_check(e, specs, 80, 4, seed=21)
+        st = e.stats()
+        assert st["completed"] == 80
+    cfg, ms, events, ex = eventlog.read(log % 0)
+    ok, msg, n = sim.replay(cfg, ms, events)
+    assert ok, msg
+    assert n == len(ex["issues"]) == st["launches"]
