@@ -266,7 +266,8 @@ def test_serving_parity_c3_models_bench_arm(tmp_path):
             oracle_out(nm, i, "bf16")
     cpus = sorted(os.sched_getaffinity(0))
     with L.Engine(num_clients=4, event_log=log, max_jobs_per_model=32, lookahead=3, launch_threads=4,
-                  slack=1184, dispatcher_cpus=[cpus[min(2, len(cpus) - 1)]]) as e:
+                  slack=1184, region_bytes=96 << 20,   # 64 slots of Inception-v3's 1.08 MB io buffer
+                  dispatcher_cpus=[cpus[min(2, len(cpus) - 1)]]) as e:
         specs = []
         for nm in names:
             g = archs.build(nm)
