@@ -480,6 +480,8 @@ def main():
     args = parse()
     if args.dispatcher_fifo > 0:
         os.environ["PAELLA_DISPATCHER_FIFO"] = str(args.dispatcher_fifo)
+    if args.impl == "reference":   # no dispatcher: the oracle keeps every host core
+        args.dispatcher_cpu = -1
     if args.dispatcher_cpu == -2:   # default: core 2 + LOCAL_RANK if the host has room
         avail = os.sched_getaffinity(0)
         first = 2
