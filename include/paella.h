@@ -157,7 +157,57 @@ typedef struct {
   uint32_t decide_delay_ns;       /* NEXT-2 sensitivity (Fig. 9, P1215-1241): the dispatcher
                                     busy-waits this long before every decide() pass, an
                                     injected scheduler delay; 0 (default) = none */
+  uint32_t naive_pdl;             /* naive baseline only: 1 = launch its kernels with programmatic
+                                    dependent launch too (CUDA-MS + PDL: the same launch mechanics
+                                    as the Paella path, so a comparison isolates the scheduler);
+                                    0 (default) = plain launches */
+  uint32_t watchdog_ms;           /* 0 = off.  A GPU whose in-flight launches report no record
+                                    progress for this long is declared hung: its live jobs complete
+                                    with -ETIMEDOUT, later requests are routed to the remaining GPUs
+                                    (or complete with -EIO when none is left) */
+  uint32_t fake_fault;            /* FAKE device fault injection (tests): PAELLA_FAULT_*, on GPU 0
+                                    of the instance only */
+  uint32_t fake_fault_arg;        /* ... the ordinal of the record / launch it applies to */
+  const char* route_log_path;     /* multi-GPU routing log (printf pattern, "%u" = client id), or
+                                    NULL: every routing decision of that client with the W_g
+                                    snapshot of ALL GPUs it was taken on (paella_route_rec_t
+                                    records, written at shutdown / paella_flush_log), so the
+                                    router replays against oracle/sim.py */
+  uint32_t max_active_jobs;       /* K (reading B200-Q6): 0 = no cap (the paper).  K > 0:
+                                    a ready job may issue only if it is among the K first jobs,
+                                    in the policy's order (SRPT: remaining time R_j; FIFO: arrival),
+                                    of the live jobs that still have kernels to issue (a deficit
+                                    override is exempt).  Preemption stays kernel-granular: a
+                                    job pushed out of the K first stops issuing, its in-flight
+                                    kernels drain */
 } paella_config_t;
+
+/* One routing decision.  W_g = work[g] + pending[g] * tbar_model:
+   work[g] = the outstanding work (sum of R_j, ns) GPU g's dispatcher last published,
+   pending[g] = submissions routed to g that its dispatcher has not admitted yet, each
+   estimated at the whole-job T-bar sum of the request's model.  alive = bit g set if
+   GPU g had not failed. */
+typedef struct {
+  uint64_t req_id;
+  uint32_t route;              /* PAELLA_ROUTE_* */
+  uint32_t chosen;             /* GPU the request went to */
+  uint32_t g0, g1;             /* power-of-two candidates (route 2), else = chosen */
+  uint32_t num_gpus, model;
+  uint32_t alive, pad;
+  int64_t  tbar_model;
+  int64_t  work[8];
+  int64_t  pending[8];
+} paella_route_rec_t;
+
+/* fault injection of the FAKE device (paella_config_t.fake_fault); n = fake_fault_arg */
+#define PAELLA_FAULT_NONE    0u
+#define PAELLA_FAULT_DROP    1u   /* the n-th COMPLETION record is lost on its way to the ring */
+#define PAELLA_FAULT_DUP     2u   /* the n-th record is written twice (two ring slots) */
+#define PAELLA_FAULT_TORN    3u   /* every record's second half lands one poll iteration after
+                                     its first half (n ignored): the reader must re-read, never
+                                     consume a torn slot (P1107-1113) */
+#define PAELLA_FAULT_HANG    4u   /* blocks of the n-th launch never complete (a hung kernel) */
+#define PAELLA_FAULT_CORRUPT 5u   /* the n-th record carries an invalid record type */
 
 /* ---- model description (input to paella_register_model) ---------------- */
 #define PAELLA_OP_INPUT   0u

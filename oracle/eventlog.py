@@ -6,7 +6,7 @@ Format (DESIGN.md §"Event log"): a sequence of 32-byte little-endian records
 
   100 CONFIG    a=N clients, b=policy, c=theta, d=(B << 32) | G
   100 CONFIG    a=0xFFFFFFFF, b=ring capacity, c=stream pool P, d=(priority classes << 32) | launch-ahead depth
-  100 CONFIG    a=0xFFFFFFFE, b=online T-bar refinement (NEXT-4)
+  100 CONFIG    a=0xFFFFFFFE, b=online T-bar refinement (NEXT-4), c=max_active K (B200-Q6)
   101 CAPACITY  a=resource r, b=C_r
   110 MODEL     a=model, b=#kernels
   111 LAYER     a=model, b=layer, c=grid, d=T-bar ns
@@ -47,6 +47,7 @@ def read(path):
         if t == 100:
             if a == 0xFFFFFFFE:
                 cfg_kw["online_tbar"] = b
+                cfg_kw["max_active"] = c
             elif a == 0xFFFFFFFF:
                 cfg_kw["ring_capacity"] = b
                 cfg_kw["streams"] = c
@@ -62,6 +63,7 @@ def read(path):
             cap[a] = b
         elif t == 110:
             nlayers[a] = b
+            events.append((sim.EV_MODEL, a))
         elif t == 111:
             layers[(a, b)] = (c, d)
         elif t == 112:
@@ -99,3 +101,22 @@ def read(path):
     extras = dict(records=records, issues=issues, completes=completes, arrivals=arrivals,
                   n_arrivals=narrivals, routes=routes)
     return cfg, models, events, extras
+
+
+# routing log (paella_config_t.route_log_path): paella_route_rec_t, include/paella.h
+ROUTE_DT = np.dtype([("req_id", "<u8"), ("route", "<u4"), ("chosen", "<u4"), ("g0", "<u4"), ("g1", "<u4"),
+                     ("num_gpus", "<u4"), ("model", "<u4"), ("alive", "<u4"), ("pad", "<u4"),
+                     ("tbar_model", "<i8"), ("work", "<i8", (8,)), ("pending", "<i8", (8,))])
+
+
+def read_routes(path):
+    """Every routing decision of one client, in submission order (dicts)."""
+    raw = np.fromfile(path, dtype=ROUTE_DT)
+    out = []
+    for r in raw:
+        ng = int(r["num_gpus"])
+        out.append(dict(req_id=int(r["req_id"]), route=int(r["route"]), chosen=int(r["chosen"]),
+                        g0=int(r["g0"]), g1=int(r["g1"]), num_gpus=ng, model=int(r["model"]),
+                        alive=int(r["alive"]), tbar_model=int(r["tbar_model"]),
+                        work=[int(x) for x in r["work"][:ng]], pending=[int(x) for x in r["pending"][:ng]]))
+    return out

@@ -56,6 +56,8 @@ class Config:
     lookahead: int = 0                # NEXT-1 launch-ahead depth (0 = the paper's semantics)
     prio_classes: int = 1             # stream-priority classes (1 = the paper: one class)
     online_tbar: int = 0              # NEXT-4: refine T-bar online (running average, P1252-1254)
+    max_active: int = 0               # K: only the K first jobs in the policy's order that still
+                                      # have kernels to issue may issue (0 = no cap); B200-Q6
 
 
 # NEXT-4 (P1249-1266: "x-bar is the average of all previous observations of x"; "these
@@ -136,6 +138,10 @@ class Policy:
         self.tb_sum = [[l.tbar * PROFILE_RUNS for l in m] for m in models]
         self.tb_cnt = [[PROFILE_RUNS for _ in m] for m in models]
         self.obs: dict[int, int] = {}        # launch uid -> observed duration (pending)
+        # models known to the dispatcher so far (a model registered while serving enters
+        # the stream-priority class boundaries at its MODEL event; replay feeds them in
+        # log order, a fresh Policy knows every model)
+        self.registered = set(range(len(models)))
 
     # effective deficit, units of 1/N
     def D(self, c):
@@ -229,21 +235,39 @@ class Policy:
     def ready(self):
         return [j for j in self.jobs.values() if self.is_ready(j)]
 
+    def order(self, j):
+        """The policy's total order on jobs (ties: arrival seq, then job id)."""
+        p = self.cfg.policy
+        if p == FIFO:
+            return (j.seq, j.id)
+        if p == SJF:               # shortest (whole) job first: profiled T-bar sum of the model
+            return (sum(l.tbar for l in self.models[j.model]), j.seq, j.id)
+        if p == RR:                # kernel-granular round robin: least recently issued job
+            return (j.rr, j.seq, j.id)
+        return (j.R, j.seq, j.id)  # SRPT
+
+    def eligible(self):
+        """B200-Q6: with max_active = K > 0, the ids of the K first jobs, in the
+        policy's order, among the live jobs that still have kernels to issue; None = no cap."""
+        K = self.cfg.max_active
+        if K <= 0:
+            return None
+        left = [j for j in self.jobs.values() if j.cursor < len(self.models[j.model])]
+        return {j.id for j in sorted(left, key=self.order)[:K]}
+
     def pick(self, rdy):
         cfg = self.cfg
         self.over = False
-        if cfg.policy == FIFO:
-            return min(rdy, key=lambda j: j.seq)
-        if cfg.policy == SJF:      # shortest (whole) job first: profiled T-bar sum of the model
-            return min(rdy, key=lambda j: (sum(l.tbar for l in self.models[j.model]), j.seq, j.id))
-        if cfg.policy == RR:       # kernel-granular round robin: least recently issued job
-            return min(rdy, key=lambda j: (j.rr, j.seq, j.id))
+        top = self.eligible()
+        ok = rdy if top is None else [j for j in rdy if j.id in top]
+        if cfg.policy != SRPT_DEFICIT:
+            return min(ok, key=self.order) if ok else None
         clients = sorted({j.client for j in rdy})
         cstar = max(clients, key=lambda c: (self.D(c), -c))
         self.over = cfg.theta != INF_THETA and self.D(cstar) > cfg.theta * cfg.num_clients
-        if self.over:
+        if self.over:            # the deficit rule overrides the cap as it overrides SRPT
             return min((j for j in rdy if j.client == cstar), key=lambda j: j.seq)
-        return min(rdy, key=lambda j: (j.R, j.seq, j.id))
+        return min(ok, key=self.order) if ok else None
 
     # Stream-priority classes (B200 adaptation, DESIGN.md reading B200-Q2).  The pool's
     # P streams are split into K classes of consecutive indices (class 0 = highest
@@ -258,7 +282,8 @@ class Policy:
         K = self.cfg.prio_classes
         if K <= 1 or self.over:
             return 0
-        totals = sorted({sum(layer.tbar for layer in m) for m in self.models if m})
+        totals = sorted({sum(layer.tbar for layer in m) for i, m in enumerate(self.models)
+                         if m and i in self.registered})
         return min(K - 1, sum(1 for t in totals if t < j.R))
 
     def predicate(self, grid):
@@ -278,6 +303,8 @@ class Policy:
             if not rdy:
                 break
             j = self.pick(rdy)
+            if j is None:
+                break
             if j.inflight == 0 and not self.free:
                 break
             layer = self.models[j.model][j.cursor]
@@ -323,9 +350,10 @@ class Policy:
 # ---------------------------------------------------------------------------
 
 EV_ARRIVAL, EV_RECORD, EV_BATCH_END, EV_ISSUE, EV_COMPLETE, EV_OBSERVE = 1, 2, 3, 4, 5, 6
+EV_MODEL = 110
 
 
-def replay(cfg: Config, models, events):
+def replay(cfg: Config, models, events, published=None):
     """Drive ``Policy`` with a recorded event sequence.
 
     events: iterable of tuples
@@ -334,14 +362,24 @@ def replay(cfg: Config, models, events):
     Inputs (arrivals, records, batch ends) are applied in order; the policy's own
     issues / completions are compared with the logged ones.  Returns
     (ok, first_divergence_message, n_issues_checked).
+
+    published: optional list; receives the dispatcher's outstanding work W_g = sum of
+    R_j over live jobs after every decide pass (the value it publishes to the router,
+    SURVEY.md §8(e)), starting with 0.
     """
     pol = Policy(cfg, models)
+    if published is not None:
+        published.append(0)
+    if any(ev[0] == EV_MODEL for ev in events):
+        pol.registered = set()     # models enter at their MODEL events
     expect = []            # issues the policy produced, awaiting the logged ones
     expect_done = []
     n = 0
     for ev in events:
         k = ev[0]
-        if k == EV_ARRIVAL:
+        if k == EV_MODEL:
+            pol.registered.add(ev[1])
+        elif k == EV_ARRIVAL:
             pol.arrival(ev[1], ev[2], ev[3])
         elif k == EV_OBSERVE:
             pol.observe(ev[1], ev[2])
@@ -353,6 +391,8 @@ def replay(cfg: Config, models, events):
             if expect:
                 return False, f"dispatcher issued fewer kernels than the reference: missing {expect[0]}", n
             expect = list(pol.decide())
+            if published is not None:
+                published.append(sum(j.R for j in pol.jobs.values()))
         elif k == EV_ISSUE:
             got = tuple(ev[1:5])
             if not expect:
@@ -616,3 +656,51 @@ def route_pick(pair, W):
     """The candidate with the lower outstanding work W[g]; ties to the lower index."""
     lo, hi = min(pair), max(pair)
     return hi if W[hi] < W[lo] else lo
+
+
+# --- least-outstanding-work routing (SURVEY.md §8(e)) -------------------------------
+
+def route_least_work(work, pending, tbar_model, alive):
+    """The GPU a request goes to under least outstanding work: W_g = work[g] (the sum of
+    R_j its dispatcher last published) + pending[g] (submissions routed to g and not yet
+    admitted) x the request model's whole-job T-bar sum; argmin over the GPUs that have
+    not failed (bit g of ``alive``), ties to the lowest index."""
+    best = None
+    for g in range(len(work)):
+        if not (alive >> g) & 1:
+            continue
+        w = work[g] + pending[g] * tbar_model
+        if best is None or w < best[0]:
+            best = (w, g)
+    return None if best is None else best[1]
+
+
+def check_inflight_bound(events, models, lookahead):
+    """NEXT-1 invariant on a consumed-event log: a job never has more than lookahead + 1
+    kernels issued whose final COMPLETION has not been consumed (launch-ahead depth D),
+    and its kernels are issued in layer order.  Returns the violations."""
+    model_of, grid_of, done_of, infl, nxt = {}, {}, {}, {}, {}
+    bad = []
+    for ev in events:
+        k = ev[0]
+        if k == EV_ARRIVAL:
+            model_of[ev[1]] = ev[3]
+            infl[ev[1]] = 0
+            nxt[ev[1]] = 0
+        elif k == EV_ISSUE:
+            uid, job, layer = ev[1], ev[2], ev[3]
+            if layer != nxt[job]:
+                bad.append(("order", uid, job, layer))
+            nxt[job] = layer + 1
+            grid_of[uid] = (job, models[model_of[job]][layer].grid)
+            done_of[uid] = 0
+            infl[job] += 1
+            if infl[job] > lookahead + 1:
+                bad.append(("depth", uid, job, infl[job]))
+        elif k == EV_RECORD and ev[1] == COMPLETION and ev[2] in grid_of:
+            uid = ev[2]
+            done_of[uid] += ev[3]
+            job, g = grid_of[uid]
+            if done_of[uid] == g:
+                infl[job] -= 1
+    return bad

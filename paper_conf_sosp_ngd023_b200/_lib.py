@@ -23,6 +23,7 @@ ROUTE_LEAST_WORK, ROUTE_ROUND_ROBIN, ROUTE_POWER_OF_TWO = 0, 1, 2
 DEVICE_CUDA, DEVICE_FAKE = 0, 1
 DTYPE_BF16, DTYPE_FP32 = 0, 1
 NONBLOCK = 1
+FAULT_NONE, FAULT_DROP, FAULT_DUP, FAULT_TORN, FAULT_HANG, FAULT_CORRUPT = 0, 1, 2, 3, 4, 5
 HYBRID = 2
 OP = {"input": 0, "conv": 1, "maxpool": 2, "avgpool": 3, "gap": 4, "fc": 5, "concat": 6}
 ACT = {"none": 0, "relu": 1, "relu6": 2}
@@ -49,7 +50,9 @@ class Config(C.Structure):
                 ("lookahead", C.c_uint32), ("launch_threads", C.c_uint32),
                 ("no_proxy", C.c_uint32), ("no_pdl", C.c_uint32),
                 ("notify_mode", C.c_uint32), ("prio_classes", C.c_uint32), ("online_tbar", C.c_uint32),
-                ("decide_delay_ns", C.c_uint32)]
+                ("decide_delay_ns", C.c_uint32), ("naive_pdl", C.c_uint32), ("watchdog_ms", C.c_uint32),
+                ("fake_fault", C.c_uint32), ("fake_fault_arg", C.c_uint32), ("route_log_path", C.c_char_p),
+                ("max_active_jobs", C.c_uint32)]
 
 
 class Node(C.Structure):
@@ -164,7 +167,8 @@ class Engine:
                  instrument=True, naive=False, region_bytes=64 << 20, dispatcher_cpus=None,
                  event_log=None, fake_sms=0, fake_time_scale_ns=0, event_time_kind=None, lookahead=0,
                  launch_threads=0, proxy=True, pdl=True, prio_classes=1,
-                 notify="counters", decide_delay_ns=0, online_tbar=False):
+                 notify="counters", decide_delay_ns=0, online_tbar=False, naive_pdl=False, watchdog_ms=0,
+                 fake_fault=0, fake_fault_arg=0, route_log=None, max_active=0):
         self.lib = load()
         cfg = Config()
         cfg.abi_version = ABI_VERSION
@@ -200,6 +204,13 @@ class Engine:
         cfg.prio_classes = prio_classes
         cfg.decide_delay_ns = decide_delay_ns
         cfg.online_tbar = 1 if online_tbar else 0
+        cfg.naive_pdl = 1 if naive_pdl else 0
+        cfg.watchdog_ms = watchdog_ms
+        cfg.fake_fault = fake_fault
+        cfg.fake_fault_arg = fake_fault_arg
+        self._rlog = route_log.encode() if route_log else None
+        cfg.route_log_path = self._rlog
+        cfg.max_active_jobs = max_active
         # notification path: "counters" (default), "ring" (device ring + forwarding warp),
         # "direct" (the paper's direct ring writes; same as proxy=False)
         if notify not in ("counters", "ring", "direct"):

@@ -87,8 +87,13 @@ struct FakeBackend : Backend {
   int64_t now = 0, dt;
   std::vector<void*> evs;
 
-  FakeBackend(uint32_t s, uint32_t c, uint32_t l2, uint32_t g, uint32_t P, int64_t d)
-      : sms(s), cap(c), log2cap(l2), G(g), nstreams(P), dt(d) {}
+  // fault injection (paella_config_t.fake_fault): record / launch ordinals, 1-based
+  uint32_t fault = PAELLA_FAULT_NONE, fault_arg = 0;
+  uint64_t rec_seq = 0, launch_seq = 0;
+  std::vector<std::pair<uint32_t, uint64_t>> torn_pending;   // (slot, w1) landing next advance()
+
+  FakeBackend(uint32_t s, uint32_t c, uint32_t l2, uint32_t g, uint32_t P, int64_t d, uint32_t f, uint32_t fa)
+      : sms(s), cap(c), log2cap(l2), G(g), nstreams(P), dt(d), fault(f), fault_arg(fa) {}
   int init() override {
     freeres.assign(sms, {});
     for (auto& f : freeres)
@@ -102,12 +107,28 @@ struct FakeBackend : Backend {
   uint32_t* tail_dev() override { return &tail; }
   uint32_t* ctr_dev() override { return ctr.data(); }
   void* ring_dev() override { return ringmem.data(); }
+  void put(uint32_t type, uint32_t n, uint32_t uid, uint32_t group) {
+    uint32_t idx = tail++;
+    Rec r = rec_encode(type, n, 0, idx >> log2cap, uid, (uint64_t)now, group);
+    Rec& slot = ringmem[idx & (cap - 1)];
+    if (fault == PAELLA_FAULT_TORN) {   // first half now, second half next iteration
+      reinterpret_cast<volatile uint64_t*>(&slot)[0] = r.w0;
+      torn_pending.emplace_back(idx & (cap - 1), r.w1);
+    } else {
+      slot = r;
+    }
+  }
   void emit(FK* k, uint32_t type, uint32_t count) {
     uint32_t r = count % G;
     if (r == 0 || count == k->grid) {
-      uint32_t idx = tail++;
-      ringmem[idx & (cap - 1)] = rec_encode(type, r == 0 ? G : r, 0, idx >> log2cap, k->uid,
-                                            (uint64_t)now, (count - 1) / G);
+      // DROP counts COMPLETION records only (a lost PLACEMENT is absorbed by p_eff =
+      // max(p, f)); the other faults count every record
+      const bool counted = fault != PAELLA_FAULT_DROP || type == REC_COMPLETION;
+      const bool hit = counted && ++rec_seq == fault_arg;
+      if (hit && fault == PAELLA_FAULT_DROP) return;   // lost on the way to the ring
+      const uint32_t n = r == 0 ? G : r, grp = (count - 1) / G;
+      put(hit && fault == PAELLA_FAULT_CORRUPT ? 7u : type, n, k->uid, grp);
+      if (hit && fault == PAELLA_FAULT_DUP) put(type, n, k->uid, grp);
     }
   }
   void launch(const KernelInst& k, const LayerArgs&, const InstrArgs& ia, uint32_t stream, uint32_t,
@@ -118,6 +139,7 @@ struct FakeBackend : Backend {
     f->stream = stream;
     for (int r = 0; r < NRES; ++r) f->demand[r] = k.demand[r];
     f->dur = k.tbar > 0 ? k.tbar : 1000;
+    if (fault == PAELLA_FAULT_HANG && ++launch_seq == fault_arg) f->dur = INT64_MAX / 4;   // never ends
     streams[stream].push_back(f);
   }
   void place() {
@@ -141,6 +163,8 @@ struct FakeBackend : Backend {
     }
   }
   void advance() override {
+    for (auto& tp : torn_pending) reinterpret_cast<volatile uint64_t*>(&ringmem[tp.first])[1] = tp.second;
+    torn_pending.clear();
     now += dt;
     while (!ends.empty() && ends.top().t <= now) {
       End e = ends.top();
@@ -509,23 +533,36 @@ static void wake_client(Paella* P, uint32_t client) {
             nullptr, 0);
 }
 
-static void push_completion(Gpu* g, const JobRec& j, int32_t status) {
+// Completion to the client's ring; if the ring is full (the client is not polling) the
+// completion waits in a per-client overflow queue, in order, and the dispatcher moves
+// on (it never blocks on a client).
+static void push_completion(Gpu* g, uint32_t client, uint64_t req_id, int32_t status) {
   CompleteSlot cs{};
-  cs.req_id = j.req_id;
+  cs.req_id = req_id;
   cs.status = status;
   cs.gpu = g->index;
   cs.t_done_ns = now_ns();
-  while (!g->done[j.client]->push(cs)) {
-    // completion ring full: the client is not polling; spin (bounded by client)
-    if (g->stop.load(std::memory_order_relaxed)) break;
+  auto& ov = g->overflow[client];
+  if (!ov.empty() || !g->done[client]->push(cs)) ov.push_back(cs);
+  wake_client(g->P, client);
+}
+
+static void flush_overflow(Gpu* g) {
+  for (uint32_t c = 0; c < g->overflow.size(); ++c) {
+    auto& ov = g->overflow[c];
+    bool moved = false;
+    while (!ov.empty() && g->done[c]->push(ov.front())) {
+      ov.pop_front();
+      moved = true;
+    }
+    if (moved) wake_client(g->P, c);
   }
-  wake_client(g->P, j.client);
 }
 
 static void finish_job(Gpu* g, uint32_t jid, int32_t status) {
   JobRec& j = g->jobs[jid];
   Model* m = g->P->models[j.model].get();
-  push_completion(g, j, status);
+  push_completion(g, j.client, j.req_id, status);
   m->gpu[g->index].free_slots.push_back(j.slot);
   j.live = false;
   g->free_job_ids.push_back(jid);
@@ -539,6 +576,8 @@ static bool admit(Gpu* g, uint32_t client, const SubmitSlot& s) {
   Model* m = P->models[s.model_id].get();
   ModelGpu& mg = m->gpu[g->index];
   if (mg.free_slots.empty()) return false;
+  // a job id first (ids come back when jobs finish), then the workspace slot
+  if (g->free_job_ids.empty() && g->next_job >= g->jobs.capacity()) return false;
   uint32_t slot = mg.free_slots.back();
   mg.free_slots.pop_back();
   uint32_t jid;
@@ -546,7 +585,6 @@ static bool admit(Gpu* g, uint32_t client, const SubmitSlot& s) {
     jid = g->free_job_ids.back();
     g->free_job_ids.pop_back();
   } else {
-    if (g->next_job >= g->jobs.capacity()) return false;
     jid = g->next_job++;
     g->jobs.resize(g->next_job);
   }
@@ -759,34 +797,69 @@ static void decide_and_launch(Gpu* g) {
   }
 }
 
-static void dispatcher_main(Gpu* g) {
+// Models posted by paella_register_model: added to this GPU's policy and logged by the
+// dispatcher thread itself, between two loop iterations.
+static void apply_inbox(Gpu* g) {
+  const uint32_t posted = g->inbox_n.load(std::memory_order_acquire);
+  if (g->models_applied.load(std::memory_order_relaxed) == posted) return;
+  std::vector<std::pair<uint32_t, std::vector<PolicyLayer>>> todo;
+  {
+    std::lock_guard<std::mutex> lk(g->inbox_mu);
+    todo.swap(g->inbox);
+  }
+  for (auto& mt : todo) {
+    const uint32_t nm = mt.first;
+    const auto& layers = mt.second;
+    g->policy->add_model(nm, layers);
+    logev(g, EV_MODEL, nm, layers.size(), 0, 0);
+    for (uint32_t l = 0; l < layers.size(); ++l) {
+      logev(g, EV_LAYER, nm, l, layers[l].grid, (uint64_t)layers[l].tbar);
+      logev(g, EV_DEMAND, nm, l, ((uint64_t)layers[l].demand[1] << 32) | (uint64_t)layers[l].demand[2],
+            ((uint64_t)layers[l].demand[3] << 32) | (uint64_t)layers[l].demand[4]);
+    }
+    if (g->log) fflush(g->log);
+    g->models_applied.fetch_add(1, std::memory_order_release);
+  }
+}
+
+// Fail this GPU: every live job completes with `status` (-EIO: a CUDA error or an
+// inconsistent notification stream; -ETIMEDOUT: the watchdog).  The router stops
+// sending work here (submit_impl checks err).
+static void fail_gpu(Gpu* g, int status, const char* why) {
+  fprintf(stderr, "[paella] GPU %u failed (%s): live jobs complete with %d\n", g->index, why, status);
+  g->err.store(status, std::memory_order_release);
+  for (uint32_t jid = 0; jid < g->jobs.size(); ++jid)
+    if (g->jobs[jid].live) finish_job(g, jid, status);
+  g->naive_inflight.clear();
+  if (g->log) fflush(g->log);
+}
+
+// Dead mode: the GPU is not used any more, but submissions that were routed here before
+// the router noticed still get an answer (-EIO), and models keep being acknowledged.
+static void dead_loop(Gpu* g) {
+  const uint32_t N = g->P->cfg.num_clients;
+  while (!g->stop.load(std::memory_order_acquire)) {
+    apply_inbox(g);
+    for (uint32_t c = 0; c < N; ++c) {
+      const SubmitSlot* s;
+      while ((s = g->sub[c]->peek()) != nullptr) {
+        push_completion(g, c, s->req_id, -EIO);
+        g->sub[c]->pop();
+        g->popped.fetch_add(1, std::memory_order_release);
+      }
+    }
+    flush_overflow(g);
+    struct timespec ts{0, 20000};
+    nanosleep(&ts, nullptr);
+  }
+}
+
+static void dispatch_loop(Gpu* g) {
   Paella* P = g->P;
-  if (P->cfg.device == PAELLA_DEVICE_CUDA) cudaSetDevice(g->device);
-  if (P->cfg.dispatcher_cpus) {
-    cpu_set_t cs;
-    CPU_ZERO(&cs);
-    CPU_SET(P->cfg.dispatcher_cpus[g->index], &cs);
-    pthread_setaffinity_np(pthread_self(), sizeof cs, &cs);
-    // SURVEY.md §8(e): a dedicated core with SCHED_FIFO (PAELLA_DISPATCHER_FIFO=<prio>);
-    // only with a pinned core, so the spinning dispatcher cannot starve migrating threads
-    if (const char* fifo = std::getenv("PAELLA_DISPATCHER_FIFO")) {
-      sched_param sp{};
-      sp.sched_priority = atoi(fifo);
-      int rc = pthread_setschedparam(pthread_self(), SCHED_FIFO, &sp);
-      if (rc) fprintf(stderr, "[paella] dispatcher %u: SCHED_FIFO %d refused (%s)\n", g->index, sp.sched_priority,
-                      strerror(rc));
-    }
-  }
   const uint32_t N = P->cfg.num_clients;
-  if (P->cfg.device == PAELLA_DEVICE_CUDA && P->cfg.event_time_kind) {
-    for (int i = 0; i < 512; ++i) {
-      cudaEvent_t a, b;
-      cudaEventCreate(&a);
-      cudaEventCreate(&b);
-      g->ev_free.push_back(Gpu::EvPair{a, b, 0, 0});
-    }
-  }
   const bool dbg = std::getenv("PAELLA_DEBUG") != nullptr;
+  const int64_t watchdog_ns = (int64_t)P->cfg.watchdog_ms * 1000000;
+  g->last_progress_ns = now_ns();
   for (;;) {
     g->stats.loop_iters++;
     if (dbg && (g->stats.loop_iters % 50000000) == 0) {
@@ -798,7 +871,11 @@ static void dispatcher_main(Gpu* g) {
         fprintf(stderr, " free[%u]=%zu", m, P->models[m]->gpu[g->index].free_slots.size());
       fprintf(stderr, " live=%lu\n", (unsigned long)g->policy->live_jobs());
     }
-    if (!g->ev_pending.empty() && (g->stats.loop_iters & 63) == 0) harvest_events(g);
+    if ((g->stats.loop_iters & 63) == 0) {
+      apply_inbox(g);
+      flush_overflow(g);
+      if (!g->ev_pending.empty()) harvest_events(g);
+    }
     g->be->advance();
     uint32_t nev = 0;
     // 1. client rings, round-robin, starting after the last client served (C2-Q16)
@@ -819,6 +896,7 @@ static void dispatcher_main(Gpu* g) {
           }
           if (!admit(g, c, *s)) break;
           q->pop();
+          g->popped.fetch_add(1, std::memory_order_release);
           nev++;
           served = true;
         }
@@ -827,6 +905,7 @@ static void dispatcher_main(Gpu* g) {
       g->admitted_pub.store(g->stats.admitted, std::memory_order_release);
     }
     if (P->cfg.naive) {
+      bool progressed = false;
       for (size_t i = 0; i < g->naive_inflight.size();) {
         uint32_t jid = g->naive_inflight[i];
         if (__atomic_load_n(&g->jobs[jid].event_recorded, __ATOMIC_ACQUIRE) && g->be->event_done(g->jobs[jid].event)) {
@@ -834,17 +913,36 @@ static void dispatcher_main(Gpu* g) {
           finish_job(g, jid, 0);
           g->naive_inflight[i] = g->naive_inflight.back();
           g->naive_inflight.pop_back();
+          progressed = true;
         } else {
           ++i;
         }
       }
-      if (stopping && g->naive_inflight.empty()) break;
+      if (progressed || g->naive_inflight.empty()) {
+        if (watchdog_ns) g->last_progress_ns = now_ns();
+      } else if (watchdog_ns && (g->stats.loop_iters & 1023) == 0 && now_ns() - g->last_progress_ns > watchdog_ns) {
+        fail_gpu(g, -ETIMEDOUT, "watchdog: no job completed");
+        return;
+      }
+      if (g->be->error() || g->launch_err.load(std::memory_order_relaxed)) {
+        fail_gpu(g, -EIO, "CUDA error");
+        return;
+      }
+      if (stopping && g->naive_inflight.empty()) return;
       continue;
     }
     // 2. notification ring (keep the forwarding warp alive while records are due)
     if (P->cfg.device == PAELLA_DEVICE_CUDA && g->policy->O() > 0 && (g->stats.loop_iters & 1023) == 0)
       static_cast<CudaBackend*>(g->be.get())->ensure_proxy();
-    nev += g->ctr_mode ? drain_counters(g) : drain_ring(g);
+    const uint32_t nrec = g->ctr_mode ? drain_counters(g) : drain_ring(g);
+    nev += nrec;
+    // watchdog: records are due (launches in flight) but none arrived for too long
+    if (nrec || g->policy->O() == 0) {
+      if (watchdog_ns) g->last_progress_ns = now_ns();
+    } else if (watchdog_ns && (g->stats.loop_iters & 1023) == 0 && now_ns() - g->last_progress_ns > watchdog_ns) {
+      fail_gpu(g, -ETIMEDOUT, "watchdog: in-flight launches report no progress");
+      return;
+    }
     // 3. decide (the batch boundary is logged for replay, C2-Q17)
     if (nev) {
       logev(g, EV_BATCH_END, 0, 0, 0, 0);
@@ -854,14 +952,48 @@ static void dispatcher_main(Gpu* g) {
     int e = g->be->error();
     if (!e) e = g->launch_err.load(std::memory_order_relaxed);
     if (e) {
-      g->err.store(-EIO);
-      // fail every live job of this GPU with -EIO
-      for (uint32_t jid = 0; jid < g->jobs.size(); ++jid)
-        if (g->jobs[jid].live) finish_job(g, jid, -EIO);
-      break;
+      fail_gpu(g, -EIO, "CUDA error");
+      return;
     }
-    if (stopping && g->policy->live_jobs() == 0) break;
+    if (stopping && g->policy->live_jobs() == 0) return;
   }
+}
+
+static void dispatcher_main(Gpu* g) {
+  Paella* P = g->P;
+  if (P->cfg.device == PAELLA_DEVICE_CUDA) cudaSetDevice(g->device);
+  if (P->cfg.dispatcher_cpus) {
+    cpu_set_t cs;
+    CPU_ZERO(&cs);
+    CPU_SET(P->cfg.dispatcher_cpus[g->index], &cs);
+    pthread_setaffinity_np(pthread_self(), sizeof cs, &cs);
+    // SURVEY.md §8(e): a dedicated core with SCHED_FIFO (PAELLA_DISPATCHER_FIFO=<prio>);
+    // only with a pinned core, so the spinning dispatcher cannot starve migrating threads
+    if (const char* fifo = std::getenv("PAELLA_DISPATCHER_FIFO")) {
+      sched_param sp{};
+      sp.sched_priority = atoi(fifo);
+      int rc = pthread_setschedparam(pthread_self(), SCHED_FIFO, &sp);
+      if (rc) fprintf(stderr, "[paella] dispatcher %u: SCHED_FIFO %d refused (%s)\n", g->index, sp.sched_priority,
+                      strerror(rc));
+    }
+  }
+  if (P->cfg.device == PAELLA_DEVICE_CUDA && P->cfg.event_time_kind) {
+    for (int i = 0; i < 512; ++i) {
+      cudaEvent_t a, b;
+      cudaEventCreate(&a);
+      cudaEventCreate(&b);
+      g->ev_free.push_back(Gpu::EvPair{a, b, 0, 0});
+    }
+  }
+  // An inconsistent notification stream (a record for an unknown launch, a count beyond
+  // the grid, an invalid type: a device or transport fault) makes the policy throw; that
+  // fails this GPU's jobs with -EIO instead of terminating the process.
+  try {
+    dispatch_loop(g);
+  } catch (const std::exception& ex) {
+    fail_gpu(g, -EIO, ex.what());
+  }
+  if (g->err.load(std::memory_order_acquire)) dead_loop(g);
 }
 
 // ---------------------------------------------------------------------------
@@ -919,6 +1051,8 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     return -EINVAL;
   if (cfg.prio_classes > cfg.stream_pool && cfg.stream_pool != 0) return -EINVAL;
   if (cfg.launch_threads > 16) return -EINVAL;
+  if (cfg.max_jobs_per_model > 4096) return -EINVAL;   // job ids: 65,536 per GPU
+  if (cfg.fake_fault > PAELLA_FAULT_CORRUPT) return -EINVAL;
 
   auto P = std::make_unique<Paella>();
   P->cfg = cfg;
@@ -959,6 +1093,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     P->sleepers.push_back(new std::atomic<uint32_t>(0));
   }
   P->rr_next.assign(cfg.num_clients, 0);
+  P->route_log.resize(cfg.num_clients);
   P->poll_rr.assign(cfg.num_clients, 0);
 
   for (uint32_t gi = 0; gi < cfg.num_gpus; ++gi) {
@@ -969,6 +1104,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     g->cap = cfg.ring_capacity;
     g->log2cap = ilog2(cfg.ring_capacity);
     g->ctr_base.assign(NCTR, 0);
+    g->overflow.resize(cfg.num_clients);
     // never reallocated: launcher threads hold pointers into job records
     g->jobs.reserve(65536);
     if (cfg.device == PAELLA_DEVICE_CUDA)
@@ -978,7 +1114,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
                                       !cfg.naive && !std::getenv("PAELLA_NO_PROXY")));
     if (cfg.device == PAELLA_DEVICE_CUDA) {
       auto* cb = static_cast<CudaBackend*>(g->be.get());
-      cb->pdl = !cfg.naive && !cfg.no_pdl && !std::getenv("PAELLA_NO_PDL");
+      cb->pdl = (!cfg.naive || cfg.naive_pdl) && !cfg.no_pdl && !std::getenv("PAELLA_NO_PDL");
       cb->prio_classes = cfg.naive ? 1 : cfg.prio_classes;
       if (cb->mirror) {
         g->ctr_mode = true;
@@ -988,7 +1124,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     }
     else
       g->be.reset(new FakeBackend(P->sms, g->cap, g->log2cap, cfg.group_size, cfg.stream_pool,
-                                  cfg.fake_time_scale_ns));
+                                  cfg.fake_time_scale_ns, gi == 0 ? cfg.fake_fault : 0u, cfg.fake_fault_arg));
     int rc = g->be->init();
     if (rc) return rc;
     Policy::Cfg pc;
@@ -1002,6 +1138,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     pc.lookahead = cfg.lookahead;
     pc.prio_classes = cfg.naive ? 1 : cfg.prio_classes;
     pc.online_tbar = cfg.online_tbar;
+    pc.max_active = cfg.max_active_jobs;
     for (int r = 0; r < NRES; ++r) pc.capacity[r] = P->capacity[r];
     if (cfg.device == PAELLA_DEVICE_CUDA &&
         (static_cast<CudaBackend*>(g->be.get())->proxy || static_cast<CudaBackend*>(g->be.get())->mirror)) {
@@ -1029,7 +1166,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
             ((uint64_t)P->cfg.slack_blocks << 32) | cfg.group_size);
       logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFFu, cfg.ring_capacity, cfg.stream_pool,
             ((uint64_t)pc.prio_classes << 32) | cfg.lookahead);
-      logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFEu, cfg.online_tbar, 0, 0);
+      logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFEu, cfg.online_tbar, cfg.max_active_jobs, 0);
       for (int r = 0; r < NRES; ++r) logev(g.get(), EV_CAPACITY, (uint32_t)r, (uint64_t)pc.capacity[r], 0, 0);
     }
     P->gpus.push_back(std::move(g));
@@ -1091,18 +1228,18 @@ int paella_register_model(paella_t* p, const paella_model_desc_t* desc, uint32_t
   }
   Model* mp = m.get();
   P->models[nm] = std::move(m);
+  // each dispatcher adds the model to its own policy on its own thread (apply_inbox);
+  // the model is published (nmodels) once every dispatcher has it
   for (auto& g : P->gpus) {
-    // the dispatcher thread only reads a model once nmodels covers it; the policy
-    // table is written before publication
-    g->policy->add_model(nm, layers);
-    logev(g.get(), EV_MODEL, nm, layers.size(), 0, 0);
-    for (uint32_t l = 0; l < layers.size(); ++l) {
-      logev(g.get(), EV_LAYER, nm, l, layers[l].grid, (uint64_t)layers[l].tbar);
-      logev(g.get(), EV_DEMAND, nm, l, ((uint64_t)layers[l].demand[1] << 32) | (uint64_t)layers[l].demand[2],
-            ((uint64_t)layers[l].demand[3] << 32) | (uint64_t)layers[l].demand[4]);
-    }
-    if (g->log) fflush(g->log);
+    std::lock_guard<std::mutex> lk2(g->inbox_mu);
+    g->inbox.emplace_back(nm, layers);
+    g->inbox_n.fetch_add(1, std::memory_order_release);
   }
+  for (auto& g : P->gpus)
+    while (g->models_applied.load(std::memory_order_acquire) < nm + 1) {
+      if (g->stop.load(std::memory_order_acquire)) return -ESHUTDOWN;
+      std::this_thread::yield();
+    }
   (void)mp;
   P->nmodels.store(nm + 1, std::memory_order_release);
   if (model_id) *model_id = nm;
@@ -1138,44 +1275,70 @@ static int64_t submit_impl(Paella* P, uint32_t client_id, uint32_t model_id, voi
   if (((uintptr_t)io & 15) != 0) return -EINVAL;
   uint64_t seq = P->client_seq[client_id]->fetch_add(1);
   uint64_t req_id = ((uint64_t)client_id << 48) | (seq & ((1ull << 48) - 1));
-  // route: least outstanding work, ties to the lowest index
+  // route: least outstanding work W_g, ties to the lowest index;
+  // W_g = published sum of R_j + unadmitted submissions x the model's whole-job T-bar.
+  // A failed GPU (err != 0) is never chosen; -EIO once none is left.
   uint32_t gsel = 0;
   uint32_t ng = (uint32_t)P->gpus.size();
-  auto work_of = [&](uint32_t g) {
-    Gpu* Gg = P->gpus[g].get();
-    int64_t pending = (int64_t)(Gg->submitted.load(std::memory_order_relaxed) -
-                                Gg->admitted_pub.load(std::memory_order_acquire));
-    return Gg->work_published.load(std::memory_order_acquire) + pending * m->total_tbar;
-  };
   SubmitSlot s{};
   if (ng > 1) {
-    // the decision and its W snapshot travel in the slot and are logged at admission
-    // (ROUTE event) so the routing replays: (g0, g1, W_g0, W_g1) for power-of-two,
-    // (chosen, runner-up or chosen, W of both) otherwise
+    int64_t work[PAELLA_MAX_GPUS] = {0}, pend[PAELLA_MAX_GPUS] = {0}, W[PAELLA_MAX_GPUS] = {0};
+    uint32_t alive = 0;
+    for (uint32_t g = 0; g < ng; ++g) {
+      Gpu* Gg = P->gpus[g].get();
+      if (Gg->err.load(std::memory_order_acquire) == 0) alive |= 1u << g;
+      // pending before work: an admission moves a job from the first to the second
+      pend[g] = (int64_t)(Gg->submitted.load(std::memory_order_relaxed) - Gg->admitted_pub.load(std::memory_order_acquire));
+      work[g] = Gg->work_published.load(std::memory_order_acquire);
+      W[g] = work[g] + pend[g] * m->total_tbar;
+    }
+    if (!alive) return -EIO;
+    auto least = [&]() {
+      uint32_t best = ng;
+      for (uint32_t g = 0; g < ng; ++g)
+        if ((alive >> g & 1) && (best == ng || W[g] < W[best])) best = g;
+      return best;
+    };
     uint32_t g0 = 0, g1 = 0;
     if (P->cfg.route == PAELLA_ROUTE_ROUND_ROBIN) {
-      gsel = g0 = g1 = P->rr_next[client_id]++ % ng;
-      s.route_w[0] = s.route_w[1] = work_of(gsel);
+      // the client's next GPU in cyclic order, skipping failed ones
+      uint32_t k = 0;
+      do {
+        gsel = P->rr_next[client_id]++ % ng;
+      } while (!(alive >> gsel & 1) && ++k < ng);
+      g0 = g1 = gsel;
     } else if (P->cfg.route == PAELLA_ROUTE_POWER_OF_TWO) {
       paella_route_pair(req_id, ng, &g0, &g1);
-      s.route_w[0] = work_of(g0);
-      s.route_w[1] = work_of(g1);
-      uint32_t lo = g0 < g1 ? g0 : g1, hi = g0 < g1 ? g1 : g0;
-      int64_t wlo = lo == g0 ? s.route_w[0] : s.route_w[1], whi = hi == g0 ? s.route_w[0] : s.route_w[1];
-      gsel = whi < wlo ? hi : lo;
+      const uint32_t lo = g0 < g1 ? g0 : g1, hi = g0 < g1 ? g1 : g0;
+      if ((alive >> lo & 1) && (alive >> hi & 1)) gsel = W[hi] < W[lo] ? hi : lo;
+      else if (alive >> lo & 1) gsel = lo;
+      else if (alive >> hi & 1) gsel = hi;
+      else gsel = least();
     } else {
-      int64_t best = INT64_MAX;
-      for (uint32_t g = 0; g < ng; ++g) {
-        int64_t w = work_of(g);
-        if (w < best) {
-          best = w;
-          gsel = g;
-        }
-      }
-      g0 = g1 = gsel;
-      s.route_w[0] = s.route_w[1] = best;
+      gsel = g0 = g1 = least();
     }
+    s.route_w[0] = W[g0];
+    s.route_w[1] = W[g1];
     s.route_meta = g0 | (g1 << 8) | (P->cfg.route << 16);
+    if (P->cfg.route_log_path) {
+      paella_route_rec_t rr{};
+      rr.req_id = req_id;
+      rr.route = P->cfg.route;
+      rr.chosen = gsel;
+      rr.g0 = g0;
+      rr.g1 = g1;
+      rr.num_gpus = ng;
+      rr.model = model_id;
+      rr.alive = alive;
+      rr.tbar_model = m->total_tbar;
+      for (uint32_t g = 0; g < ng; ++g) {
+        rr.work[g] = work[g];
+        rr.pending[g] = pend[g];
+      }
+      P->route_log[client_id].push_back(rr);
+    }
+  } else if (P->gpus[0]->err.load(std::memory_order_acquire)) {
+    return -EIO;
   }
   Gpu* G = P->gpus[gsel].get();
   s.req_id = req_id;
@@ -1220,6 +1383,17 @@ int64_t paella_poll_completion(paella_t* p, uint32_t client_id, uint32_t flags, 
         return id;
       }
     }
+    // every GPU failed and every submission has been answered: nothing will come
+    bool all_dead = true;
+    for (auto& g : P->gpus)
+      all_dead &= g->err.load(std::memory_order_acquire) != 0 &&
+                  g->popped.load(std::memory_order_acquire) >= g->submitted.load(std::memory_order_acquire);
+    if (all_dead) {
+      bool empty = true;   // re-check: a completion may have landed since the scan
+      for (uint32_t k = 0; k < ng && empty; ++k) empty = P->gpus[k]->done[client_id]->peek() == nullptr;
+      if (empty) return -EIO;
+      continue;
+    }
     if (flags & PAELLA_NONBLOCK) return -EAGAIN;
     bool alive = false;
     for (auto& g : P->gpus) alive |= g->thread.joinable() && !g->stop.load();
@@ -1243,6 +1417,21 @@ int64_t paella_poll_completion(paella_t* p, uint32_t client_id, uint32_t flags, 
   }
 }
 
+// routing log of every client (cfg.route_log_path), rewritten in full
+static int write_route_logs(Paella* P) {
+  if (!P->cfg.route_log_path) return 0;
+  for (uint32_t c = 0; c < P->route_log.size(); ++c) {
+    char path[4096];
+    snprintf(path, sizeof path, P->cfg.route_log_path, c);
+    FILE* f = fopen(path, "wb");
+    if (!f) return -EINVAL;
+    const auto& v = P->route_log[c];
+    if (!v.empty()) fwrite(v.data(), sizeof(paella_route_rec_t), v.size(), f);
+    fclose(f);
+  }
+  return 0;
+}
+
 int paella_shutdown(paella_t* p) {
   Paella* P = (Paella*)p;
   if (!P) return -EINVAL;
@@ -1261,8 +1450,10 @@ int paella_shutdown(paella_t* p) {
       if (g->prof_stream) cudaStreamSynchronize((cudaStream_t)g->prof_stream);
     }
   }
+  write_route_logs(P);
   // requests never admitted complete with -ECANCELED
   for (auto& g : P->gpus) {
+    flush_overflow(g.get());
     for (uint32_t c = 0; c < P->cfg.num_clients; ++c) {
       const SubmitSlot* s;
       while ((s = g->sub[c]->peek()) != nullptr) {
@@ -1309,7 +1500,7 @@ int paella_flush_log(paella_t* p) {
   if (!P) return -EINVAL;
   for (auto& g : P->gpus)
     if (g->log) fflush(g->log);
-  return 0;
+  return write_route_logs(P);
 }
 
 int paella_model_info(paella_t* p, uint32_t model_id, paella_model_info_t* info) {

@@ -3,6 +3,7 @@
 #include <atomic>
 #include <cstdint>
 #include <cstdio>
+#include <deque>
 #include <memory>
 #include <mutex>
 #include <string>
@@ -187,7 +188,18 @@ struct Gpu {
   std::atomic<int64_t> work_published{0};
   std::atomic<uint64_t> admitted_pub{0};
   std::atomic<uint64_t> submitted{0};
-  std::atomic<int> err{0};
+  std::atomic<int> err{0};          // != 0: this GPU failed (-EIO) or hung (-ETIMEDOUT); it only
+                                    // completes submissions with -EIO from then on (dead mode)
+  std::atomic<uint64_t> popped{0};  // submissions taken out of this GPU's rings (any outcome)
+  // completions the client's ring could not take yet (never blocks the dispatcher)
+  std::vector<std::deque<CompleteSlot>> overflow;
+  int64_t last_progress_ns = 0;     // watchdog: last time a record was consumed (or nothing was due)
+  // model registration is applied by the dispatcher thread itself (no data race with
+  // decide(); the MODEL events are ordered with the rest of the log)
+  std::mutex inbox_mu;
+  std::vector<std::pair<uint32_t, std::vector<PolicyLayer>>> inbox;
+  std::atomic<uint32_t> inbox_n{0};          // models posted
+  std::atomic<uint32_t> models_applied{0};   // models the dispatcher has added to its policy
   uint32_t rr_start = 0;
   FILE* log = nullptr;
   std::mutex log_mu;
@@ -243,6 +255,9 @@ struct Paella {
   std::vector<std::atomic<uint32_t>*> sleepers;
   std::atomic<bool> shutting{false};
   int64_t capacity[NRES];
+  // routing log (multi-GPU, cfg.route_log_path): every decision with the full W_g
+  // snapshot it was taken on, one vector per client (written by that client's thread)
+  std::vector<std::vector<paella_route_rec_t>> route_log;
 };
 
 // planner (plan.cpp)

@@ -651,9 +651,12 @@ __global__ void __launch_bounds__(32, 1) k_notify_mirror(const uint4* ctrs, uint
       ch |= cur[i].x != prev[i].x || cur[i].y != prev[i].y || cur[i].z != prev[i].z || cur[i].w != prev[i].w;
     }
     if (__any_sync(0xffffffffu, ch)) {
-      // no fence needed: each published word IS the loaded count (the store depends on
-      // the load), and a block's release reduction made its outputs visible -- at
-      // system scope for a job's last kernel -- before that count could be loaded
+      // A block's release reduction made its outputs visible (at system scope for a
+      // job's last kernel) before its count could be loaded with acquire; PTX gives no
+      // ordering from the load->store data dependency, so one system-scope fence per
+      // batch of changed chunks orders those outputs before the relaxed stores that
+      // publish the counts to the host (cumulativity of fence.acq_rel.sys)
+      asm volatile("fence.acq_rel.sys;" ::: "memory");
 #pragma unroll
       for (uint32_t i = 0; i < NQ; ++i) {
         if (cur[i].x != prev[i].x || cur[i].y != prev[i].y || cur[i].z != prev[i].z || cur[i].w != prev[i].w) {

@@ -97,8 +97,10 @@ void Policy::refine(const PolicyLaunch& L) {
     if (j.cursor > lay) continue;
     const bool rdy = j.in_ready;
     if (rdy) make_unready(j);
+    active_erase(j);
     j.R += delta;
     work_ += delta;
+    active_insert(j);
     if (rdy) make_ready(j);
   }
 }
@@ -109,6 +111,18 @@ int64_t Policy::order_key(const PolicyJob& j) const {
   if (cfg_.policy == POL_SJF) return model_total_[j.model];
   if (cfg_.policy == POL_RR) return j.rr;
   return j.R;
+}
+
+// the policy's total order (oracle Policy.order): SRPT R_j, SJF model T-bar sum, RR last
+// issued uid, FIFO arrival only; ties (seq, id)
+int64_t Policy::active_key(const PolicyJob& j) const {
+  return cfg_.policy == POL_FIFO ? 0 : order_key(j);
+}
+void Policy::active_erase(const PolicyJob& j) {
+  if (cfg_.max_active) active_.erase(std::make_tuple(active_key(j), j.seq, j.id));
+}
+void Policy::active_insert(const PolicyJob& j) {
+  if (cfg_.max_active && j.cursor < models_[j.model].size()) active_.emplace(active_key(j), j.seq, j.id);
 }
 
 void Policy::make_ready(PolicyJob& j) {
@@ -143,6 +157,7 @@ void Policy::arrival(uint32_t job_id, uint32_t client, uint32_t model) {
   live_by_model_[model].push_back(job_id);
   work_ += R;
   live_jobs_ += 1;
+  active_insert(j);
   refresh(j);
 }
 
@@ -199,9 +214,24 @@ int Policy::lowest_free() const {
   return -1;
 }
 
+// B200-Q6 (max_active = K): the first ready job among the K first jobs of active_ (the
+// policy's order over live jobs with kernels left to issue); false if none is ready
+bool Policy::pick_capped(uint32_t* job_id) const {
+  uint32_t k = 0;
+  for (auto it = active_.begin(); it != active_.end() && k < cfg_.max_active; ++it, ++k) {
+    const uint32_t id = std::get<2>(*it);
+    if (jobs_[id].in_ready) {
+      *job_id = id;
+      return true;
+    }
+  }
+  return false;
+}
+
 bool Policy::pick(uint32_t* job_id) {
   over_ = false;
   if (srpt_.empty()) return false;
+  if (cfg_.policy != POL_SRPT_DEFICIT && cfg_.max_active) return pick_capped(job_id);
   if (cfg_.policy == POL_FIFO) {
     *job_id = fifo_.begin()->second;
     return true;
@@ -229,7 +259,9 @@ bool Policy::pick(uint32_t* job_id) {
   }
   over_ = over;
   if (over) {
-    *job_id = per_client_[cstar].begin()->second;   // oldest ready job of c*
+    *job_id = per_client_[cstar].begin()->second;   // oldest ready job of c* (overrides the cap too)
+  } else if (cfg_.max_active) {
+    return pick_capped(job_id);
   } else {
     *job_id = std::get<2>(*srpt_.begin());           // SRPT: (R, seq, id)
   }
@@ -296,12 +328,14 @@ void Policy::decide(std::vector<Issue>* out) {
     Q_ += lay.grid;
     O_ += 2 * (int64_t)((lay.grid + cfg_.group - 1) / cfg_.group);
     make_unready(j);
+    active_erase(j);
     j.R -= lay.tbar;
     work_ -= lay.tbar;
     j.uid_of[j.cursor % 8] = uid;
     j.cursor += 1;
     j.last_uid = uid;
     j.rr = uid;   // after make_unready above: the ready-set key changes only out of the set
+    active_insert(j);
     Dt_[j.client] -= (int64_t)cfg_.num_clients;
     Omega_ += 1;
     out->push_back(Issue{uid, jid, L.layer, stream});

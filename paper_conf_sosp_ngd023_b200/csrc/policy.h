@@ -77,6 +77,8 @@ class Policy {
     uint32_t lookahead = 0;   // NEXT-1 launch-ahead depth (0 = the paper's semantics)
     uint32_t prio_classes = 1;   // stream-priority classes (1 = the paper: one class)
     uint32_t online_tbar = 0;    // NEXT-4: refine T-bar online (running average, P1252-1254)
+    uint32_t max_active = 0;     // K: only the K first jobs in the policy's order that still
+                                 // have kernels to issue may issue (0 = no cap); B200-Q6
   };
   static constexpr int64_t kProfileRuns = 20;   // observations behind the profiled T-bar
   // class of stream s: consecutive index ranges, class 0 = highest hardware priority
@@ -112,10 +114,14 @@ class Policy {
   static constexpr uint32_t kLaunchSlots = 8192;
   static constexpr uint32_t kMaxModels = 256;
   bool pick(uint32_t* job_id);
+  bool pick_capped(uint32_t* job_id) const;
   uint32_t job_class(const PolicyJob& j) const;
   int lowest_free_in_class(uint32_t c) const;
   bool predicate(uint32_t grid) const;
   int64_t order_key(const PolicyJob& j) const;
+  int64_t active_key(const PolicyJob& j) const;
+  void active_erase(const PolicyJob& j);
+  void active_insert(const PolicyJob& j);
   void refine(const PolicyLaunch& L);
   void make_ready(PolicyJob& j);
   void make_unready(PolicyJob& j);
@@ -147,6 +153,8 @@ class Policy {
   std::set<std::tuple<int64_t, uint64_t, uint32_t>> srpt_;     // (R, seq, id)
   std::set<std::pair<uint64_t, uint32_t>> fifo_;               // (seq, id)
   std::vector<std::set<std::pair<uint64_t, uint32_t>>> per_client_;  // (seq, id)
+  // B200-Q6: live jobs with kernels left to issue, in the policy's order (max_active > 0)
+  std::set<std::tuple<int64_t, uint64_t, uint32_t>> active_;
 };
 
 }  // namespace paella

@@ -484,3 +484,181 @@ def test_route_pair_candidates_valid_and_spread():
     assert sim.route_pick((5, 2), [0, 0, 7, 0, 0, 3, 0, 0]) == 5
     assert sim.route_pick((5, 2), [0, 0, 3, 0, 0, 3, 0, 0]) == 2
     assert sim.route_pick((2, 5), [0, 0, 1, 0, 0, 3, 0, 0]) == 2
+
+
+# --- NEXT-1 launch-ahead: closed forms derived by hand (not the rule re-typed) -------
+
+def _chain(L, d):
+    return [[Layer(1, (1, 1, 1, 1, 0), d, d) for _ in range(L)]]
+
+
+@pytest.mark.parametrize("D", [0, 1, 2, 3])
+def test_launch_ahead_closed_form_zero_delay(D):
+    """One job of L single-block kernels of duration d, zero launch/notification delay:
+    at t = 0 kernels 0..D are issued (each new one is queued behind a fully placed
+    predecessor); every time kernel m completes, kernel m+1 is placed and kernel m+D+1
+    is issued.  So kernel k is issued at max(0, (k - D) d), and JCT = L d for every D.
+    A rule that looked at the NEWEST in-flight kernel instead of the oldest would issue
+    only one kernel ahead; one that ignored D would issue all L at t = 0."""
+    Lk, d = 6, 1000
+    cfg = Config(num_clients=1, theta=sim.INF_THETA, slack=10**6, lookahead=D,
+                 capacity=(10**6, 10**9, 10**12, 10**12, 10**9))
+    res = sim.simulate(cfg, _chain(Lk, d), [(0, 0, 0)], GPUModel(sms=1, per_sm=(1, 64, 65536, 233472, 512)))
+    issue_t = [t for (t, uid, jid, layer, stream) in sorted(res.issues, key=lambda x: x[3])]
+    assert issue_t == [max(0, (k - D) * d) for k in range(Lk)]
+    assert res.jct()[0] == Lk * d
+    assert len({s for (_, _, _, _, s) in res.issues}) == (1 if D > 0 else 1)
+
+
+def test_launch_ahead_closed_form_with_delays():
+    """d = 10, launch delay 2, notification delay 3, L = 4 (times in units of 1 us),
+    derived step by step in the test docstring's notation:
+    D = 0: each kernel waits for its predecessor's completion record:
+           issue at 0, 15, 30, 45; the last completion is seen at 60.
+    D = 1: k0 issued 0, placed 2, PLACEMENT seen 5 -> k1 issued 5 (launched 7, queued);
+           k0 ends 12, k1 placed 12, both records seen 15 -> k2 issued 15;
+           k1 ends 22, k2 placed 22, seen 25 -> k3 issued 25; k3 runs 32..42, seen 45."""
+    u = 1000
+    gpu = GPUModel(sms=1, per_sm=(1, 64, 65536, 233472, 512), launch_delay=2 * u, notif_delay=3 * u)
+    for D, want_issue, want_jct in ((0, [0, 15, 30, 45], 60), (1, [0, 5, 15, 25], 45)):
+        cfg = Config(num_clients=1, theta=sim.INF_THETA, slack=10**6, lookahead=D,
+                     capacity=(10**6, 10**9, 10**12, 10**12, 10**9))
+        res = sim.simulate(cfg, _chain(4, 10 * u), [(0, 0, 0)], gpu)
+        assert [t for (t, *_r) in sorted(res.issues, key=lambda x: x[3])] == [x * u for x in want_issue]
+        assert res.jct()[0] == want_jct * u
+
+
+@pytest.mark.parametrize("D", [0, 1, 3])
+def test_inflight_bound_checker(D):
+    """check_inflight_bound accepts every simulator log at its own depth; on the chain of
+    test_launch_ahead_closed_form_zero_delay (depth D + 1 reached at t = 0) it rejects
+    the log when checked against depth D - 1."""
+    r = random.Random(900 + D)
+    models = random_models(r)
+    gpu = GPUModel(sms=4, per_sm=(32, 64, 65536, 233472, 512), launch_delay=300, notif_delay=400)
+    cfg = Config(num_clients=2, slack=64, group=4, streams=8, lookahead=D,
+                 capacity=tuple(4 * x for x in (32, 64, 65536, 233472, 512)))
+    trace = random_trace(r, 30, 2, len(models), rate_ns=3000)
+    res = _run_policy_with_log(cfg, models, trace, gpu)
+    assert sim.check_inflight_bound(res.policy.log, models, D) == []
+    chain = _chain(6, 1000)
+    cfg1 = Config(num_clients=1, theta=sim.INF_THETA, slack=10**6, lookahead=D,
+                  capacity=(10**6, 10**9, 10**12, 10**12, 10**9))
+    res1 = _run_policy_with_log(cfg1, chain, [(0, 0, 0)], GPUModel(sms=1, per_sm=(1, 64, 65536, 233472, 512)))
+    assert sim.check_inflight_bound(res1.policy.log, chain, D) == []
+    if D > 0:
+        assert sim.check_inflight_bound(res1.policy.log, chain, D - 1) != []
+
+
+# --- stream-priority classes: worked example (B200-Q2) -------------------------------
+
+def _one_layer_models(tbars):
+    return [[Layer(1, (1, 1, 1, 1, 0), t, t)] for t in tbars]
+
+
+def test_prio_classes_worked_example():
+    """Models with whole-job T-bar 10, 20, 40; K = 3 classes over P = 6 streams
+    (class of stream s = floor(3 s / 6): {0,1}, {2,3}, {4,5}); one client, theta = inf.
+    Jobs A (40), B (10), C (20), D (40), E (40) arrive at once.  SRPT issues B, C, A, D, E.
+    Class of a job = number of models whose sum is strictly below R_j:
+    B -> 0 -> stream 0;  C -> 1 -> stream 2;  A -> 2 -> stream 4;  D -> 2 -> stream 5;
+    E -> 2, class 2 full -> the lowest free stream overall, 1."""
+    models = _one_layer_models([10, 20, 40])
+    cfg = Config(num_clients=1, theta=sim.INF_THETA, slack=10**6, streams=6, prio_classes=3,
+                 capacity=(10**6, 10**9, 10**12, 10**12, 10**9))
+    pol = sim.Policy(cfg, models)
+    for jid, m in enumerate([2, 0, 1, 2, 2]):     # A B C D E
+        pol.arrival(jid, 0, m)
+    got = [(job, stream) for (uid, job, layer, stream) in pol.decide()]
+    assert got == [(1, 0), (2, 2), (0, 4), (3, 5), (4, 1)]
+
+
+def test_prio_classes_deficit_override_takes_class0():
+    """theta = 0, two clients.  Y (client 1, R = 10) is picked first by SRPT (both
+    deficits 0, not > 0) -> class 0, stream 0; deficits become D0 = +1, D1 = -1 (units
+    1/N).  X (client 0, R = 40) is then picked by the deficit override (1 > 0) and takes
+    class 0 -> stream 1 (without the override it would be class 2, stream 4)."""
+    models = _one_layer_models([10, 20, 40])
+    cfg = Config(num_clients=2, theta=0, slack=10**6, streams=6, prio_classes=3,
+                 capacity=(10**6, 10**9, 10**12, 10**12, 10**9))
+    pol = sim.Policy(cfg, models)
+    pol.arrival(0, 0, 2)    # X
+    pol.arrival(1, 1, 0)    # Y
+    got = [(job, stream) for (uid, job, layer, stream) in pol.decide()]
+    assert got == [(1, 0), (0, 1)]
+    assert (pol.D(0), pol.D(1)) == (0, 0)
+
+
+# --- B200-Q6: the job cap K (max_active) ---------------------------------------------
+
+def test_max_active_worked_example():
+    """K = 2, SRPT, one client, theta = inf, single-kernel jobs with T-bar 30, 10, 20
+    arriving together: only the two shortest (10, 20) may issue; the 30 waits until one
+    of them has issued its last kernel (then it has no kernel left and leaves the set)."""
+    models = _one_layer_models([30, 10, 20])
+    cfg = Config(num_clients=1, theta=sim.INF_THETA, slack=10**6, streams=8, max_active=2,
+                 capacity=(10**6, 10**9, 10**12, 10**12, 10**9))
+    pol = sim.Policy(cfg, models)
+    for jid, m in enumerate([0, 1, 2]):
+        pol.arrival(jid, 0, m)
+    first = [job for (uid, job, layer, stream) in pol.decide()]
+    # both capped jobs issued their only kernel, so the set {1, 2} is exhausted and job 0
+    # becomes one of the K first with kernels left: same pass
+    assert first == [1, 2, 0]
+    # two-kernel jobs: the set keeps them while they have kernels left
+    models2 = [[Layer(1, (1, 1, 1, 1, 0), 15, 15)] * 2, _one_layer_models([10])[0], _one_layer_models([20])[0]]
+    pol2 = sim.Policy(Config(num_clients=1, theta=sim.INF_THETA, slack=10**6, streams=8, max_active=2,
+                             capacity=(10**6, 10**9, 10**12, 10**12, 10**9)), models2)
+    for jid, m in enumerate([0, 1, 2]):      # R = 30, 10, 20
+        pol2.arrival(jid, 0, m)
+    iss = pol2.decide()
+    # SRPT top-2 = {1 (10), 2 (20)}: both issue; then {0 (30)} is top -> issues layer 0;
+    # job 0 is in flight (no launch-ahead) so the pass ends
+    assert [job for (_, job, _, _) in iss] == [1, 2, 0]
+    uid0 = iss[2][0]
+    pol2.record(sim.PLACEMENT, uid0, 1)
+    pol2.record(sim.COMPLETION, uid0, 1)
+    pol2.arrival(3, 0, 1)                    # a short job arrives (R = 10) with job 0 at R = 15
+    assert [job for (_, job, _, _) in pol2.decide()] == [3, 0]
+
+
+def test_max_active_fifo_order_and_override():
+    """FIFO, K = 1, launch-ahead 1, two 2-kernel jobs: job 1 may start only once job 0
+    has issued its LAST kernel (it then has nothing left to issue and leaves the set).
+    SRPT, K = 1, theta = 0, two clients: P (client 0, 2 x 5 ns) is the SRPT head and
+    issues; Q (client 1, 40 ns) is outside the cap, but after P's dispatch client 1's
+    deficit is +1 > theta N = 0, so the override issues Q in the same pass."""
+    big = (10**6, 10**9, 10**12, 10**12, 10**9)
+    models = [[Layer(1, (1, 1, 1, 1, 0), 10, 10)] * 2] * 2
+    pol = sim.Policy(Config(num_clients=1, policy=sim.FIFO, slack=10**6, streams=8, max_active=1,
+                            lookahead=1, capacity=big), models)
+    pol.arrival(0, 0, 0)
+    pol.arrival(1, 0, 1)
+    iss = pol.decide()
+    assert [(j, l) for (_, j, l, _) in iss] == [(0, 0)]
+    pol.record(sim.PLACEMENT, iss[0][0], 1)
+    assert [(j, l) for (_, j, l, _) in pol.decide()] == [(0, 1), (1, 0)]
+    m2 = [[Layer(1, (1, 1, 1, 1, 0), 5, 5)] * 2, [Layer(1, (1, 1, 1, 1, 0), 40, 40)]]
+    pol2 = sim.Policy(Config(num_clients=2, theta=0, slack=10**6, streams=8, max_active=1, capacity=big), m2)
+    pol2.arrival(0, 0, 0)    # P
+    pol2.arrival(1, 1, 1)    # Q
+    assert [(j, l) for (_, j, l, _) in pol2.decide()] == [(0, 0), (1, 0)]
+    assert pol2.over
+
+
+# --- S5 (b) exactly-once checker on bad logs ------------------------------------------
+
+def test_exactly_once_checker_rejects_bad_logs():
+    """grid 40, G 16 -> groups (0:16), (1:16), (2:8) per type.  Each corruption a device
+    or a consumer could produce must be flagged."""
+    good = []
+    for typ in (sim.PLACEMENT, sim.COMPLETION):
+        good += [(0, typ, 7, 16, 0), (0, typ, 7, 16, 1), (0, typ, 7, 8, 2)]
+    assert sim.check_exactly_once(good, {7: 40}, 16) == []
+    dropped = good[:-1]
+    dup = good + [good[0]]
+    wrong_count = good[:2] + [(0, sim.PLACEMENT, 7, 7, 2)] + good[3:]
+    wrong_group = good[:2] + [(0, sim.PLACEMENT, 7, 8, 1)] + good[3:]
+    other_uid = good[:5] + [(0, sim.COMPLETION, 8, 8, 2)]
+    for bad in (dropped, dup, wrong_count, wrong_group, other_uid):
+        assert sim.check_exactly_once(bad, {7: 40}, 16) != []
