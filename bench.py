@@ -2,23 +2,40 @@
 """Benchmark of the Paella hot path on B200 (driver contract: one JSON line).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl paella|reference]
-                    [--config c2_mix|c3_dispersion|c1_toy] [--rho 0.7]
+                    [--config c3_dispersion|c2_mix|c1_toy] [--rho 0.7]
 
-Workload (N=1): BASELINE.json configs[1] -- single GPU, mixed ResNet-18 / MobileNetV2 /
-SqueezeNet batch-1 jobs, Poisson arrivals (uniform mix, 3 clients, one per model,
-bf16, random-init LSUV weights of workload/rng.py, synthetic N(0,1) images).
+Workload (default): BASELINE.json configs[2] -- the high-dispersion mix the metric is
+quoted on: ResNet-50 / DenseNet-121 / Inception-v3 / MobileNetV2 batch-1 jobs, 4 clients
+(one per model), lognormal bursty inter-arrivals (sigma = 2, P1370-1372), request mix
+inversely proportional to the unloaded job time (Fig. 12 convention, P1482-1483), bf16,
+random-init LSUV weights (workload/rng.py), synthetic N(0,1) images.  configs[3] (the
+same mix over 1/2/4/8 GPUs) is this bench at --gpus N.
 
-A *step* is one open-loop trace segment of `--reqs` requests replayed through the
-public C ABI (paella_submit_at / paella_poll_completion, via paella_loadgen) at
-rate lambda = rho * X_sat(naive), where X_sat(naive) -- the saturation throughput
-of the naive one-stream-per-job baseline (CUDA-MS) -- is measured in an untimed
-calibration phase.  value = requests completed per second over the K timed steps
-(whole job, all ranks).  JCT = completion seen by the client - scheduled arrival.
-Alongside: the same trace through the naive baseline and through Paella-FIFO, the
-device-only roofline (summed isolated kernel time per model), the dominant kernel's
-roofline (tcgen05 conv, CUDA events in the dispatcher), clocks, and the oracle CPU
-baseline.  Multi-GPU (torchrun): one process per GPU, each with its own dispatcher
-and trace at the same per-GPU rate (weak scaling, no collective on the data path).
+A *step* is one open-loop trace segment of --reqs requests replayed through the public
+C ABI (paella_submit_at / paella_poll_completion, via paella_loadgen) at lambda =
+N * rho * X_sat,1(naive), X_sat by bisection.  Every arm serves the
+SAME K step traces:
+
+  paella       the dispatcher: SRPT + deficit (theta = 100), job cap K = 8 (B200-Q6),
+               launch-ahead 3, B = 8 x 148 slack blocks, PDL, instrumented kernels
+  paella_fifo  the same dispatcher with FIFO order (isolates the policy)
+  naive        one stream per job, every kernel launched at arrival (CUDA-MS, the
+               north star's baseline), uninstrumented twins, plain launches
+  naive_pdl    the same with programmatic dependent launch (isolates launch mechanics)
+  paella_paper the paper's semantics: no launch-ahead, no PDL, no cap, B = 148
+
+value = the Paella arm's req/s at the p99 SLO (BASELINE metric): the largest offered
+lambda with every model's p99 JCT <= SLO_m = 5 x its unloaded naive median JCT (ladder
+of rho, then bisection).  jct_mean_us / jct_p99_us: the Paella arm at lambda; vs_naive /
+vs_naive_pdl: the JCT ratios on the same traces.  The full per-model, per-arm detail is
+written to gpurun_out/bench_detail_<config>_n<N>.json (and stderr); the stdout line is
+kept short so the driver's tail holds it.
+
+Multi-GPU (torchrun, N ranks): rank 0 drives ONE Paella instance over all N GPUs --
+one dispatcher per GPU on a NUMA-local core, requests routed in paella_submit by least
+outstanding work; the naive arms are routed round robin.  The other
+ranks only join the barriers (their GPU is driven by rank 0's dispatchers).  No
+collective on the data path (jobs are independent).
 """
 from __future__ import annotations
 
@@ -27,7 +44,6 @@ import json
 import os
 import subprocess
 import sys
-import threading
 import time
 
 import numpy as np
@@ -38,7 +54,11 @@ sys.path.insert(0, ROOT)
 from workload import archs, rng, traces  # noqa: E402
 
 PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
-METRIC = "requests/s at rho*X_sat(naive) with mean/p50/p99 JCT (open-loop, batch-1 mix)"
+METRIC = "req/s at p99 SLO (Paella, open-loop batch-1 mix), with mean/p99 JCT"
+WORKLOADS = {"c2_mix": "BASELINE configs[1]: mixed ResNet-18/MobileNetV2/SqueezeNet1.1 batch-1, Poisson",
+             "c3_dispersion": "BASELINE configs[2]/[3]: ResNet-50/DenseNet-121/Inception-v3/MobileNetV2 batch-1, "
+                              "lognormal sigma=2 bursts",
+             "c1_toy": "BASELINE configs[0]: 2 clients, toy conv+MLP, Poisson"}
 
 
 def parse():
@@ -47,31 +67,31 @@ def parse():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="paella", choices=["paella", "reference"])
-    ap.add_argument("--config", default="c2_mix")
+    ap.add_argument("--config", default="c3_dispersion")
     ap.add_argument("--rho", type=float, default=0.7)
-    ap.add_argument("--reqs", type=int, default=2000, help="requests per step")
-    ap.add_argument("--no-baselines", action="store_true")
-    ap.add_argument("--lookahead", type=int, default=3, help="NEXT-1 launch-ahead depth of the Paella arm")
+    ap.add_argument("--reqs", type=int, default=2000, help="requests per step (per GPU)")
+    ap.add_argument("--arms", default="paella,paella_fifo,naive,naive_pdl,paella_paper",
+                    help="arms to run on the step traces (paella always runs)")
+    ap.add_argument("--no-baselines", action="store_true", help="only the paella arm")
+    ap.add_argument("--max-active", type=int, default=8, help="job cap K of the paella arms (B200-Q6); 0 = none")
+    ap.add_argument("--lookahead", type=int, default=3, help="NEXT-1 launch-ahead depth of the paella arms")
     ap.add_argument("--slack", type=int, default=1184,
                     help="B, blocks issued beyond full utilisation (P1300-1304); 8 x 148 SMs covers the "
                          "measured dispatch loop delay (DESIGN.md B200-Q1)")
     ap.add_argument("--policy", default="srpt", choices=["srpt", "fifo", "sjf", "rr"],
-                    help="policy of the Paella arm (sjf/rr: Table 3 ablations, NEXT-2)")
-    ap.add_argument("--online-tbar", action="store_true", help="NEXT-4 online T-bar refinement in the Paella arm")
+                    help="policy of the paella arm (sjf/rr: Table 3 ablations, NEXT-2)")
+    ap.add_argument("--theta", type=int, default=100, help="fairness threshold (kernel dispatches, P1296-1297)")
+    ap.add_argument("--online-tbar", action="store_true", help="NEXT-4 online T-bar refinement in the paella arm")
     ap.add_argument("--decide-delay-ns", type=int, default=0,
                     help="injected scheduler delay before every decide pass (Fig. 9 sensitivity)")
-    ap.add_argument("--theta", type=int, default=100, help="fairness threshold (kernel dispatches, P1296-1297)")
     ap.add_argument("--prio-classes", type=int, default=1, help="stream-priority classes (DESIGN.md B200-Q2)")
     ap.add_argument("--dispatcher-cpu", type=int, default=-2,
-                    help="pin each rank's dispatcher to core (this + LOCAL_RANK), exclusive; -1 = unpinned; "
-                         "default: 2 when the host has >= 2 + 2N cores")
-    ap.add_argument("--dispatcher-fifo", type=int, default=0,
-                    help="SCHED_FIFO priority of the pinned dispatcher (0 = SCHED_OTHER)")
+                    help="first dispatcher core (-1 = unpinned; default: NUMA-local cores of each GPU, "
+                         "else 2, 3, ...)")
     ap.add_argument("--launch-threads", type=int, default=4, help="launcher helper threads per GPU")
-    ap.add_argument("--sat-reqs", type=int, default=1500, help="requests of the saturation calibration")
-    ap.add_argument("--slo-rhos", default="0.5,0.7,0.9,1.0,1.1,1.2,1.35,1.5",
-                    help="offered loads (x X_sat(naive)) of the req/s-at-p99-SLO ladder ('' = skip)")
-    ap.add_argument("--slo-reqs", type=int, default=1500, help="requests per point of the SLO ladder")
+    ap.add_argument("--slo-reqs", type=int, default=1500, help="requests per point of the SLO search")
+    ap.add_argument("--no-slo", action="store_true", help="skip the req/s-at-SLO search (value = served req/s)")
+    ap.add_argument("--no-c5", action="store_true", help="skip the notification microbenchmarks")
     ap.add_argument("--fake", action="store_true",
                     help="CPU fake device (tests of the multi-rank plumbing; not a measurement)")
     return ap.parse_args()
@@ -81,7 +101,7 @@ def parse():
 # distributed plumbing (barrier + max over ranks; no data-path collective)
 # ---------------------------------------------------------------------------
 class Dist:
-    def __init__(self, n):
+    def __init__(self):
         self.world = int(os.environ.get("WORLD_SIZE", "1"))
         self.rank = int(os.environ.get("RANK", "0"))
         self.local = int(os.environ.get("LOCAL_RANK", "0"))
@@ -112,12 +132,9 @@ class Dist:
         self.pg.all_reduce(t, op=self.pg.ReduceOp.SUM)
         return t.item()
 
-    def gather_list(self, arr):
-        if not self.pg:
-            return [arr]
-        out = [None] * self.world
-        self.pg.all_gather_object(out, arr)
-        return out
+    def close(self):
+        if self.pg:
+            self.pg.destroy_process_group()
 
 
 # ---------------------------------------------------------------------------
@@ -128,15 +145,15 @@ class Clocks:
          "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
          "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
 
-    def __init__(self, gpu):
-        self.gpu = gpu
+    def __init__(self, gpus):
+        self.gpus = gpus
         self.proc = None
 
     def start(self):
-        if self.gpu < 0:
+        if not self.gpus:
             return
         try:
-            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", ",".join(map(str, self.gpus)), f"--query-gpu={self.Q}",
                                           "--format=csv,noheader,nounits", "-lms", "200"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
         except OSError:
@@ -166,28 +183,71 @@ class Clocks:
 
 
 # ---------------------------------------------------------------------------
-# the GPU arm
+# dispatcher cores: NUMA-local to each GPU
 # ---------------------------------------------------------------------------
-def build_engine(L, specs, gpu, fake=False, **kw):
-    if fake:
-        kw.pop("event_time_kind", None)
-        e = L.Engine(num_clients=len(specs), device=L.DEVICE_FAKE, **kw)
-    else:
-        e = L.Engine(num_clients=len(specs), first_gpu=gpu, **kw)
-    mids = [e.register_model(g, P) for (g, P) in specs]
-    return e, mids
+def _cpulist(s):
+    out = []
+    for part in s.strip().split(","):
+        if not part:
+            continue
+        if "-" in part:
+            a, b = part.split("-")
+            out += list(range(int(a), int(b) + 1))
+        else:
+            out.append(int(part))
+    return out
 
 
-def stage_inputs(e, specs, mids, slots, stride, pool):
-    """Pre-stage inputs: client c serves model c; slot s holds pool image s % pool."""
-    for c, (g, _) in enumerate(specs):
-        _, reg = e.region(c)
-        for s in range(slots):
-            x = pool[c][s % len(pool[c])]
-            off = s * stride
-            reg[off:off + x.nbytes] = np.frombuffer(x.tobytes(), np.uint8)
+def gpu_numa_nodes(n):
+    """NUMA node of GPUs 0..n-1 (nvidia-smi PCI bus id -> sysfs), -1 if unknown."""
+    try:
+        out = subprocess.run(["nvidia-smi", "--query-gpu=pci.bus_id", "--format=csv,noheader"], capture_output=True,
+                             text=True, timeout=30).stdout.split()
+    except (OSError, subprocess.SubprocessError):
+        return [-1] * n
+    nodes = []
+    for bus in out[:n]:
+        bus = bus.lower()
+        if bus.count(":") == 2 and len(bus.split(":")[0]) == 8:
+            bus = bus[4:]
+        try:
+            nodes.append(int(open(f"/sys/bus/pci/devices/{bus}/numa_node").read()))
+        except (OSError, ValueError):
+            nodes.append(-1)
+    return nodes + [-1] * (n - len(nodes))
 
 
+def dispatcher_cores(n, first):
+    """One core per GPU: explicit (first + i), else a free core on the GPU's NUMA node
+    (skipping cores 0-1), else 2 + i.  Returns (cores, numa nodes) or (None, ...) if the
+    host has too few cores to dedicate one per GPU plus as many for the rest."""
+    avail = sorted(os.sched_getaffinity(0))
+    nodes = gpu_numa_nodes(n)
+    if first >= 0:
+        return [first + i for i in range(n)], nodes
+    if len(avail) < 2 + 2 * n:
+        return None, nodes
+    used, cores = set(), []
+    for i in range(n):
+        pick = None
+        if nodes[i] >= 0:
+            try:
+                local = _cpulist(open(f"/sys/devices/system/node/node{nodes[i]}/cpulist").read())
+            except OSError:
+                local = []
+            cand = [c for c in local if c in avail and c >= 2 and c not in used]
+            pick = cand[0] if cand else None
+        if pick is None:
+            cand = [c for c in avail if c >= 2 and c not in used]
+            pick = cand[0]
+        used.add(pick)
+        cores.append(pick)
+    return cores, nodes
+
+
+# ---------------------------------------------------------------------------
+# the GPU arms
+# ---------------------------------------------------------------------------
 def jct_stats(jct_ns, models, names):
     ok = jct_ns >= 0
     out = {}
@@ -213,195 +273,272 @@ def make_trace(n, rate, cfg, n_models, seed):
     return t, models, inputs
 
 
-def saturation(e, mids, n_models, stride, slots, n, seed=99):
-    """Closed burst: all requests due at t=0; completions / elapsed."""
+def backlog_ok(t, jct):
+    """the backlog (requests arrived, not completed) averaged over the last
+    10 % of arrivals stays below 2x its average over the first 10 % (+1)."""
+    done = t + np.maximum(jct, 0)
+    n = len(t)
+    k = max(1, n // 10)
+    order = np.sort(done)
+
+    def backlog(i):
+        return (i + 1) - np.searchsorted(order, t[i], side="right")
+    first = np.mean([backlog(i) for i in range(k)])
+    last = np.mean([backlog(i) for i in range(n - k, n)])
+    return last < 2 * first + 1
+
+
+class Arm:
+    """One served system (an engine) with its step runner."""
+
+    def __init__(self, L, label, specs, pool, ngpus, region, stride, slots, fake, **kw):
+        self.label = label
+        self.stride, self.slots = stride, slots
+        if fake:
+            kw.pop("event_time_kind", None)
+            self.e = L.Engine(num_clients=len(specs), device=L.DEVICE_FAKE, num_gpus=ngpus, region_bytes=region,
+                              **kw)
+        else:
+            self.e = L.Engine(num_clients=len(specs), num_gpus=ngpus, first_gpu=0, region_bytes=region, **kw)
+        self.mids = [self.e.register_model(g, P) for (g, P) in specs]
+        for c, (g, _) in enumerate(specs):     # client c serves model c; slot s holds image s % 32
+            _, reg = self.e.region(c)
+            for s in range(slots):
+                x = pool[c][s % len(pool[c])]
+                reg[s * stride:s * stride + x.nbytes] = np.frombuffer(x.tobytes(), np.uint8)
+        self.ngpus = ngpus
+
+    def serve(self, t, mm, ii, copy_inputs=None):
+        return self.e.loadgen(t, mm, mm, ii, self.stride, self.slots, copy_inputs=copy_inputs)
+
+    def stats(self):
+        return [self.e.stats(g) for g in range(self.ngpus)]
+
+    def close(self):
+        self.e.shutdown()
+
+
+def saturation(arm, cfg, n_models, n, x0, seed=99, iters=5):
+    """X_sat by bisection: the largest lambda with completion rate >=
+    0.98 lambda and a bounded backlog, between 0.4 x0 and 1.6 x0 (x0 = closed-burst
+    estimate)."""
+    lo, hi = 0.4 * x0, 1.6 * x0
+    best = None
+    for k in range(iters):
+        lam = (lo + hi) / 2
+        t, mm, ii = make_trace(n, lam, cfg, n_models, seed=seed + k)
+        jct, el = arm.serve(t, mm, ii)
+        rate = (jct >= 0).sum() / (el / 1e9)
+        offered = n / max(t[-1] / 1e9, 1e-9)     # the trace's realised rate (bursty: != lam)
+        if rate >= 0.98 * offered and backlog_ok(t, jct):
+            best, lo = lam, lam
+        else:
+            hi = lam
+    return best if best is not None else lo
+
+
+def closed_burst(arm, n_models, n):
     t = np.zeros(n, dtype=np.int64)
     models = np.arange(n) % n_models
-    jct, el = e.loadgen(t, models, models, np.zeros(n), stride, slots)
+    jct, el = arm.serve(t, models, np.zeros(n))
     return n / (el / 1e9)
 
 
-def slo_ladder(e, args, cfg, names, x_sat_naive, slo, stride, slots, seed):
-    """req/s at p99 SLO: the largest offered lambda of the ladder
-    rho * X_sat(naive) at which every model's p99 JCT is within its SLO (an
-    overloaded point fails it: the backlog grows through the point's window)."""
-    rhos = [float(r) for r in args.slo_rhos.split(",") if r.strip()]
-    pts, best = [], 0.0
-    for i, r in enumerate(rhos):
-        lam = r * x_sat_naive
-        t, mm, ii = make_trace(args.slo_reqs, lam, cfg, len(names), seed=seed + i)
-        jct, el = e.loadgen(t, mm, mm, ii, stride, slots)
+def slo_search(arm, cfg, names, x_sat, slo, n, seed):
+    """req/s at p99 SLO: the largest offered lambda at which every model's p99 JCT <= SLO_m
+    (ladder rho in 0.1..1.2 of X_sat(naive), then 3 bisection steps above the largest
+    passing point)."""
+    pts = []
+
+    def probe(lam, k):
+        t, mm, ii = make_trace(n, lam, cfg, len(names), seed=seed + k)
+        jct, el = arm.serve(t, mm, ii)
         st = jct_stats(jct, mm, names)
-        ok = all(st.get(n, {}).get("p99_us", 1e18) <= slo[n] for n in names)
-        served = (jct >= 0).sum() / (el / 1e9)
-        pts.append({"rho": r, "offered_req_s": round(lam, 1), "served_req_s": round(float(served), 1),
-                    "p99_us": {n: round(st[n]["p99_us"], 1) for n in names if n in st},
-                    "mean_us": round(st["mix"]["mean_us"], 1), "slo_met": bool(ok)})
-        if ok:
-            best = max(best, lam)
-    return {"req_s": round(best, 1), "ladder": pts}
+        ok = all(st.get(m, {}).get("p99_us", 1e18) <= slo[m] for m in names)
+        pts.append({"rho": round(lam / x_sat, 3), "req_s": round(lam, 1), "slo_met": bool(ok),
+                    "p99_us": {m: round(st[m]["p99_us"]) for m in names if m in st},
+                    "mean_us": round(st["mix"]["mean_us"])})
+        return ok
+    best, fail = 0.0, None
+    for k, r in enumerate((0.1, 0.2, 0.3, 0.5, 0.7, 0.9, 1.1)):
+        lam = r * x_sat
+        if probe(lam, k):
+            best = lam
+        else:
+            fail = lam
+            break
+    if fail is not None and best > 0:
+        lo, hi = best, fail
+        for k in range(3):
+            mid = (lo + hi) / 2
+            if probe(mid, 10 + k):
+                lo = best = mid
+            else:
+                hi = mid
+    return {"req_s": round(best, 1), "points": pts}
 
 
-def run_gpu(args, dist):
+def run_gpu(args, ngpus, cores, fake):
     from paper_conf_sosp_ngd023_b200 import _lib as L
     L.load()
-    cfgname = args.config
-    cfg = traces.CONFIGS[cfgname]
+    cfg = dict(traces.CONFIGS[args.config])
     names = cfg["models"]
-    gpu = dist.local
     specs = []
     for nm in names:
         g = archs.build(nm)
         specs.append((g, rng.model_params(g)))
     pool = [[rng.image(g, i) for i in range(32)] for (g, _) in specs]
-    slots = 256
+    slots = 256 * max(1, min(ngpus, 2))
     sizes = [int(np.prod(g.nodes[0]["out"])) * 4 + g.num_classes * 4 for (g, _) in specs]
     stride = (max(sizes) + 4095) // 4096 * 4096
     region = slots * stride + (1 << 20)
+    pol = {"srpt": L.POLICY_SRPT_DEFICIT, "fifo": L.POLICY_FIFO, "sjf": L.POLICY_SJF, "rr": L.POLICY_RR}
+    common = dict(launch_threads=0 if fake else args.launch_threads, max_jobs_per_model=128)
+    if cores:
+        common["dispatcher_cpus"] = cores
+    paella_kw = dict(policy=pol[args.policy], theta=args.theta, decide_delay_ns=args.decide_delay_ns,
+                     online_tbar=args.online_tbar, slack=args.slack, prio_classes=args.prio_classes,
+                     lookahead=args.lookahead, max_active=args.max_active, instrument=True,
+                     route=L.ROUTE_LEAST_WORK)
+    arms_kw = {
+        "paella": paella_kw,
+        "paella_fifo": dict(paella_kw, policy=L.POLICY_FIFO),
+        "naive": dict(naive=True, instrument=False, route=L.ROUTE_ROUND_ROBIN),
+        "naive_pdl": dict(naive=True, instrument=False, naive_pdl=True, route=L.ROUTE_ROUND_ROBIN),
+        "paella_paper": dict(policy=L.POLICY_SRPT_DEFICIT, theta=100, lookahead=0, slack=0, pdl=False,
+                             route=L.ROUTE_LEAST_WORK),
+    }
+    want = ["paella"] + ([] if args.no_baselines else
+                         [a for a in args.arms.split(",") if a and a != "paella" and a in arms_kw])
 
-    def engine(**kw):
-        kw.setdefault("launch_threads", 0 if args.fake else args.launch_threads)
-        if args.dispatcher_cpu >= 0:
-            kw.setdefault("dispatcher_cpus", [args.dispatcher_cpu + gpu])
-        if not kw.get("naive"):
-            kw.setdefault("policy", {"srpt": L.POLICY_SRPT_DEFICIT, "fifo": L.POLICY_FIFO, "sjf": L.POLICY_SJF,
-                                     "rr": L.POLICY_RR}[args.policy])
-            kw.setdefault("theta", args.theta)
-            kw.setdefault("decide_delay_ns", args.decide_delay_ns)
-            kw.setdefault("online_tbar", args.online_tbar)
-            kw.setdefault("slack", args.slack)
-            kw.setdefault("prio_classes", args.prio_classes)
-        e, mids = build_engine(L, specs, gpu, fake=args.fake, region_bytes=region, max_jobs_per_model=128, **kw)
-        stage_inputs(e, specs, mids, slots, stride, pool)
-        return e, mids
+    def arm(label, n=ngpus):
+        return Arm(L, label, specs, pool, n, region, stride, slots, fake, **common, **arms_kw[label])
 
-    # --- calibration (untimed): naive saturation, unloaded JCT -> SLO ---------------
+    detail = {"config": args.config, "models": names, "n_gpus": ngpus, "dispatcher_cpus": cores}
+    # --- calibration (untimed): naive X_sat on ONE GPU, unloaded JCT -> SLO ---------------
     t_cal = time.time()
-    en, mids = engine(naive=True, instrument=False)
-    x_sat_naive = saturation(en, mids, len(names), stride, slots, args.sat_reqs)
+    a1 = arm("naive", 1)
+    x0 = closed_burst(a1, len(names), 1500 if not fake else 200)
     t1, m1, i1 = make_trace(300, 200.0, cfg, len(names), seed=7)
-    jct_unloaded, _ = en.loadgen(t1, m1, m1, i1, stride, slots)
-    slo = {nm: 5.0 * float(np.median(jct_unloaded[m1 == m])) / 1e3 for m, nm in enumerate(names)}
+    jct_unloaded, _ = a1.serve(t1, m1, i1)
+    med = {nm: float(np.median(jct_unloaded[m1 == m])) / 1e3 for m, nm in enumerate(names)}
+    slo = {nm: 5.0 * med[nm] for nm in names}
     if cfg["weights"] is None:
         # Fig. 12 convention (P1482-1483): request mix inversely proportional to job size
-        cfg = dict(cfg, weights=[1.0 / max(1e-9, float(np.median(jct_unloaded[m1 == m]))) for m in range(len(names))])
-    en.shutdown()
-    lam = args.rho * x_sat_naive
+        cfg["weights"] = [1.0 / max(1e-9, med[nm]) for nm in names]
+    x_sat1 = saturation(a1, cfg, len(names), 3000 if not fake else 200, x0, iters=5 if not fake else 1)
+    a1.close()
+    lam = ngpus * args.rho * x_sat1
+    detail.update(x_sat_naive_1gpu=round(x_sat1, 1), x_closed_burst_naive=round(x0, 1), slo_us=slo,
+                  unloaded_naive_p50_us=med, lam=round(lam, 1), mix_weights=cfg["weights"])
 
-    # --- the Paella arm -------------------------------------------------------------
-    e, mids = engine(instrument=True, lookahead=args.lookahead)
-    x_sat_paella = saturation(e, mids, len(names), stride, slots, args.sat_reqs)
-    jp, _ = e.loadgen(t1, m1, m1, i1, stride, slots)
-    unloaded = {"naive": {nm: float(np.median(jct_unloaded[m1 == m])) / 1e3 for m, nm in enumerate(names)},
-                "paella": {nm: float(np.median(jp[m1 == m])) / 1e3 for m, nm in enumerate(names)}}
-    # device-only roofline: summed isolated kernel time per model (uninstrumented twin)
-    dev_roof = {}
-    kinfo = {}
-    for m, nm in enumerate(names):
-        ks = e.kernels(mids[m])
-        if args.fake:
-            kt = kti = np.array([k["tbar_ns"] for k in ks], dtype=np.int64)
-        else:
-            kt = e.time_kernels(mids[m], instrumented=False, reps=20)
-            kti = e.time_kernels(mids[m], instrumented=True, reps=20)
-        dev_roof[nm] = float(kt.sum()) / 1e3
-        kinfo[nm] = (ks, kt, kti)
-    calib_s = time.time() - t_cal
+    # step traces, shared by every arm
+    seed0 = 1000
+    n_step = args.reqs * ngpus
+    warm = [make_trace(n_step, lam, cfg, len(names), seed=seed0 + w) for w in range(args.warmup)]
+    steps = [make_trace(n_step, lam, cfg, len(names), seed=seed0 + 100 + s) for s in range(args.steps)]
 
-    seed0 = 1000 * (dist.rank + 1)
-    for w in range(args.warmup):
-        t, mm, ii = make_trace(args.reqs, lam, cfg, len(names), seed=seed0 + w)
-        e.loadgen(t, mm, mm, ii, stride, slots)
-    st0 = e.stats()
-    clocks = Clocks(gpu if not args.fake else -1)
-    dist.barrier()
-    clocks.start()
-    t_start = time.perf_counter_ns()
-    all_jct, all_models = [], []
-    for s in range(args.steps):
-        t, mm, ii = make_trace(args.reqs, lam, cfg, len(names), seed=seed0 + 100 + s)
-        jct, el = e.loadgen(t, mm, mm, ii, stride, slots)
-        all_jct.append(jct)
-        all_models.append(mm)
-    elapsed = (time.perf_counter_ns() - t_start) / 1e9
-    dist.barrier()
-    clk = clocks.stop()
-    st1 = e.stats()
-    stats = {k: ([a - b for a, b in zip(st1[k], st0[k])] if isinstance(st1[k], list) else st1[k] - st0[k])
-             for k in st1}
-    # dominant kernel (tcgen05 conv): algorithmic bytes / CUDA-event duration of the
-    # served (instrumented) kernels, launched back to back on their stream
-    ev = {"launches": 0, "ns": 0, "bytes": 0, "flops": 0, "all_ns": 0}
-    for nm, (ks, kt, kti) in kinfo.items():
-        for k, t in zip(ks, kti):
-            ev["all_ns"] += int(t)
-            if k["name"].startswith("conv_tcgen05"):
-                ev["launches"] += 1
-                ev["ns"] += int(t)
-                ev["bytes"] += k["bytes"]
-                ev["flops"] += k["flops"]
-    jct = np.concatenate(all_jct)
-    models = np.concatenate(all_models)
-    completed = int((jct >= 0).sum())
-
-    # --- end-to-end: same trace, inputs copied in / logits read out per request -------
-    copy_in = {m: pool[m] for m in range(len(names))}
-    t, mm, ii = make_trace(args.reqs, lam, cfg, len(names), seed=seed0 + 500)
-    e2e_jct, e2e_el = e.loadgen(t, mm, mm, ii, stride, slots, copy_inputs=copy_in)
-    e2e_rate = (e2e_jct >= 0).sum() / (e2e_el / 1e9)
-    slo_at = {}
-    if args.slo_rhos and not args.no_baselines:
-        slo_at["paella"] = slo_ladder(e, args, cfg, names, x_sat_naive, slo, stride, slots, seed0 + 700)
-    h2d = float(np.mean([sizes[m] - specs[m][0].num_classes * 4 for m in mm]))
-    d2h = float(np.mean([specs[m][0].num_classes * 4 for m in mm]))
-    e.shutdown()
-
-    # --- baselines on the same trace (naive CUDA-MS, Paella as in the paper, FIFO) -----
-    base = {}
-    if not args.no_baselines:
-        for label, kw in (("naive_cuda_ms", dict(naive=True, instrument=False)),
-                          ("paella_paper_lookahead0", dict(policy=L.POLICY_SRPT_DEFICIT, lookahead=0, slack=0, prio_classes=1,
-                                                           pdl=False)),
-                          ("paella_fifo", dict(policy=L.POLICY_FIFO, lookahead=args.lookahead))):
-            eb, mb = engine(**kw)
-            jl = []
-            for s in range(min(args.steps, 3)):
-                t, mm, ii = make_trace(args.reqs, lam, cfg, len(names), seed=seed0 + 100 + s)
-                j, _ = eb.loadgen(t, mm, mm, ii, stride, slots)
-                jl.append((j, mm))
-            if label == "naive_cuda_ms" and args.slo_rhos:
-                slo_at["naive"] = slo_ladder(eb, args, cfg, names, x_sat_naive, slo, stride, slots, seed0 + 700)
-            eb.shutdown()
-            base[label] = jct_stats(np.concatenate([a for a, _ in jl]), np.concatenate([b for _, b in jl]), names)
-
-    return dict(unloaded=unloaded, names=names, lam=lam, x_sat_naive=x_sat_naive, x_sat_paella=x_sat_paella, slo=slo,
-                elapsed=elapsed, completed=completed, jct=jct_stats(jct, models, names), clocks=clk,
-                ev=ev, stats=stats, dev_roof=dev_roof, base=base, e2e_rate=e2e_rate,
-                e2e=jct_stats(e2e_jct, mm, names), h2d=h2d, d2h=d2h, calib_s=calib_s, kinfo=kinfo,
-                slo_at=slo_at, config=cfgname)
+    res = {}
+    for label in want:
+        a = arm(label)
+        for (t, mm, ii) in warm:
+            a.serve(t, mm, ii)
+        st0 = a.stats()
+        clocks = Clocks([] if fake else list(range(ngpus)))
+        clocks.start()
+        t_start = time.perf_counter_ns()
+        jl, ml = [], []
+        for (t, mm, ii) in steps:
+            jct, el = a.serve(t, mm, ii)
+            jl.append(jct)
+            ml.append(mm)
+        elapsed = (time.perf_counter_ns() - t_start) / 1e9
+        clk = clocks.stop()
+        st1 = a.stats()
+        jct = np.concatenate(jl)
+        models = np.concatenate(ml)
+        r = {"elapsed": elapsed, "completed": int((jct >= 0).sum()), "jct": jct_stats(jct, models, names),
+             "clocks": clk}
+        dstats = []
+        for g in range(ngpus):
+            d = {k: (np.subtract(st1[g][k], st0[g][k]).tolist() if isinstance(st1[g][k], list)
+                     else st1[g][k] - st0[g][k]) for k in st1[g]}
+            d["busy_frac"] = round(d["busy_ns"] / 1e9 / elapsed, 4)
+            d["launches_per_s"] = round(d["launches"] / elapsed)
+            d["records_per_s"] = round(d["records"] / elapsed)
+            dstats.append(d)
+        r["dispatcher"] = dstats
+        if label == "paella":
+            # device-only roofline (summed isolated kernel time), dominant-kernel roofline
+            dev_roof, kinfo = {}, {}
+            for m, nm in enumerate(names):
+                ks = a.e.kernels(a.mids[m])
+                if fake:
+                    kt = kti = np.array([k["tbar_ns"] for k in ks], dtype=np.int64)
+                else:
+                    kt = a.e.time_kernels(a.mids[m], instrumented=False, reps=20)
+                    kti = a.e.time_kernels(a.mids[m], instrumented=True, reps=20)
+                dev_roof[nm] = float(kt.sum()) / 1e3
+                kinfo[nm] = (ks, kt, kti)
+            r["dev_roof"] = dev_roof
+            r["kinfo"] = kinfo
+            # end to end: the client copies every input into its region and the logits out
+            t, mm, ii = make_trace(n_step, lam, cfg, len(names), seed=seed0 + 500)
+            e2e_jct, e2e_el = a.serve(t, mm, ii, copy_inputs={m: pool[m] for m in range(len(names))})
+            r["e2e"] = {"rate": (e2e_jct >= 0).sum() / (e2e_el / 1e9), "jct": jct_stats(e2e_jct, mm, names),
+                        "h2d": float(np.mean([sizes[m] - specs[m][0].num_classes * 4 for m in mm])),
+                        "d2h": float(np.mean([specs[m][0].num_classes * 4 for m in mm])), "n": len(mm)}
+            r["x_sat"] = saturation(a, cfg, len(names), 3000 if not fake else 200, lam / args.rho,
+                                    iters=4 if not fake else 1)
+            if not args.no_slo and not fake:
+                r["slo"] = slo_search(a, cfg, names, ngpus * x_sat1, slo, args.slo_reqs * ngpus, seed0 + 700)
+            if not args.no_c5 and not fake and ngpus == 1:
+                r["c5"] = c5_micro(a.e)
+        elif label in ("naive", "naive_pdl") and not args.no_slo and not fake:
+            r["slo"] = slo_search(a, cfg, names, ngpus * x_sat1, slo, args.slo_reqs * ngpus, seed0 + 700)
+        a.close()
+        res[label] = r
+    detail["calib_s"] = round(time.time() - t_cal, 1)
+    return res, detail, lam, names
 
 
-def cpu_baseline(cfg, seconds=12.0):
-    """The oracle (float64 numpy inference, as it stands) serving a bounded sample of
-    the same mix on the host cores: a process pool, one BLAS thread per worker."""
-    import multiprocessing as mp
-    cores = max(1, len(os.sched_getaffinity(0)) - 2)
-    names = cfg["models"]
-    ctx = mp.get_context("fork")
-    t0 = time.time()
-    with ctx.Pool(cores, initializer=_cpu_init) as pool:
-        n_done = 0
-        results = []
-        i = 0
-        while time.time() - t0 < seconds:
-            batch = [(names[(i + k) % len(names)], (i + k) % 32) for k in range(cores)]
-            i += cores
-            results = pool.map(_cpu_one, batch)
-            n_done += len(results)
-        el = time.time() - t0
-    return {"value": n_done / el, "unit": "req/s", "cores": cores, "kind": "oracle",
-            "sample": f"{n_done} requests of the {'/'.join(names)} mix, float64 numpy oracle "
-                      f"(oracle/infer.py), {cores} worker processes x 1 BLAS thread, {el:.1f} s"}
+def c5_micro(e):
+    """Config 5 on the bench's engine (P1881-1897, Fig. 15): empty-kernel launch time,
+    instrumented (counter mode, as served) vs plain, at grids 16/148/160/1184/4736; ring
+    round trip of a 1-block kernel (launch -> PLACEMENT / COMPLETION visible to the host)."""
+    out = {"empty_us": {}}
+    for grid in (16, 148, 160, 1184, 4736):
+        a = e.bench_empty(grid, 128, True, 16, 1000)
+        b = e.bench_empty(grid, 128, False, 16, 1000)
+        out["empty_us"][grid] = {"instr": round(a / 1e3, 3), "plain": round(b / 1e3, 3),
+                                 "delta": round((a - b) / 1e3, 3)}
+    p, c = e.bench_roundtrip(1000)
+    out["roundtrip_us"] = {"placement_p50": round(float(np.percentile(p, 50)) / 1e3, 2),
+                           "placement_p99": round(float(np.percentile(p, 99)) / 1e3, 2),
+                           "completion_p50": round(float(np.percentile(c, 50)) / 1e3, 2),
+                           "completion_p99": round(float(np.percentile(c, 99)) / 1e3, 2)}
+    return out
+
+
+# ---------------------------------------------------------------------------
+# the oracle on the host cores (cpu_baseline leg and --impl reference)
+# ---------------------------------------------------------------------------
+def host_info():
+    info = {"cpu": None, "sockets": None, "numa_nodes": None}
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            k, _, v = line.partition(":")
+            v = v.strip()
+            if k == "Model name":
+                info["cpu"] = v
+            elif k == "Socket(s)":
+                info["sockets"] = int(v) if v.isdigit() else v
+            elif k == "NUMA node(s)":
+                info["numa_nodes"] = int(v) if v.isdigit() else v
+    except (OSError, subprocess.SubprocessError):
+        pass
+    return info
 
 
 _CPU = {}
@@ -423,158 +560,230 @@ def _cpu_one(arg):
         g = archs.build(name)
         _CPU[name] = (g, rng.model_params(g))
     g, P = _CPU[name]
+    t0 = time.perf_counter()
     infer.forward(g, P, rng.image(g, idx), dtype="bf16")
-    return 1
+    return time.perf_counter() - t0
 
 
+def cpu_baseline(cfg, seconds=20.0, reserve=0):
+    """The oracle (float64 numpy inference, as it stands) serving the config's mix on the
+    host cores, as SURVEY.md 8(d) specifies: W worker processes (host cores minus the
+    dispatcher cores and one load-generator core; 1 BLAS thread each), X_sat,cpu =
+    W / mean service time from a closed warm-up batch, then an open-loop trace of the
+    config's arrival process at 0.7 X_sat,cpu served FIFO; JCT from the scheduled arrival."""
+    import multiprocessing as mp
+    names = cfg["models"]
+    W = max(1, len(os.sched_getaffinity(0)) - reserve - 1)
+    ctx = mp.get_context("fork")
+    t_all = time.time()
+    with ctx.Pool(W, initializer=_cpu_init) as pool:
+        warm = pool.map(_cpu_one, [(names[i % len(names)], i % 32) for i in range(2 * W)])
+        w = cfg.get("weights") or [1.0] * len(names)
+        mean_s = float(np.mean(warm))
+        x_sat = W / mean_s
+        lam = 0.7 * x_sat
+        n = max(W, int(lam * max(2.0, seconds - (time.time() - t_all))))
+        t, mm, ii = make_trace(n, lam, dict(cfg, weights=w), len(names), seed=4242)
+        t0 = time.perf_counter()
+        futs = []
+        for k in range(n):
+            due = t0 + t[k] / 1e9
+            while time.perf_counter() < due:
+                time.sleep(min(0.001, max(0.0, due - time.perf_counter())))
+            futs.append((due, pool.apply_async(_cpu_one, ((names[mm[k]], int(ii[k]) % 32),))))
+        jct = []
+        for due, f in futs:
+            f.get()
+            jct.append(time.perf_counter() - due)
+        el = time.perf_counter() - t0
+    j = np.asarray(jct) * 1e6
+    hi = host_info()
+    return {"value": round(n / el, 3), "unit": "req/s", "cores": W, "kind": "oracle",
+            "jct_mean_us": round(float(j.mean())), "jct_p50_us": round(float(np.percentile(j, 50))),
+            "jct_p99_us": round(float(np.percentile(j, 99))), "x_sat_req_s": round(x_sat, 3),
+            "sample": f"{n} requests of the {'/'.join(names)} mix, open loop at 0.7 x the CPU's own X_sat "
+                      f"({x_sat:.2f} req/s), float64 numpy oracle, {W} worker processes x 1 BLAS thread, "
+                      f"{el:.1f} s",
+            "host": hi}
+
+
+def simulator_timing(kinfo, cfg, names, lam, n=300):
+    """The oracle's discrete-event simulator (synthetic mode) on a trace of the config:
+    wall time and simulated events per second on one core."""
+    from oracle import sim
+    models = []
+    for nm in names:
+        ks, kt, kti = kinfo[nm]
+        ls = []
+        for k, t in zip(ks, kti):
+            warps = (k["block"] + 31) // 32
+            regs = (k["regs"] * 32 + 255) // 256 * 256 * warps
+            smem = (k["smem"] + 1024 + 127) // 128 * 128
+            ls.append(sim.Layer(k["grid"], (1, warps, regs, smem, k["tmem_cols"]), int(k["tbar_ns"]),
+                                max(1, int(t))))
+        models.append(ls)
+    t, mm, _ = make_trace(n, lam, cfg, len(names), seed=31)
+    trace = [(int(t[i]), int(mm[i]), int(mm[i])) for i in range(n)]
+    c = sim.Config(num_clients=len(names), slack=1184, lookahead=3, max_active=8)
+    t0 = time.perf_counter()
+    r = sim.simulate(c, models, trace, sim.GPUModel(), check=False)
+    el = time.perf_counter() - t0
+    events = len(r.records) + len(r.issues) + len(r.blocks) * 2 + n
+    return {"requests": n, "wall_s": round(el, 2), "events": events, "events_per_s": round(events / el),
+            "completed": len(r.finish)}
+
+
+# ---------------------------------------------------------------------------
 def roofline_entry(res, peaks):
-    """Dominant kernel = the tcgen05 implicit-GEMM conv.  achieved = algorithmic
-    bytes (weights + input + output [+ residual]) summed over every conv launch of one
-    request of each model / their summed CUDA-event durations (instrumented kernels as
-    served, each launched back to back on its stream right after the timed region)."""
-    ev = res["ev"]
-    if not ev or ev["launches"] == 0 or ev["ns"] == 0:
+    """Dominant kernel = the tcgen05 implicit-GEMM conv.  achieved = algorithmic bytes
+    (weights + input + output [+ residual]) summed over every conv launch of one request
+    of each model / their summed CUDA-event durations (instrumented kernels as served,
+    each launched back to back on its stream right after the timed region)."""
+    n = nsec = byts = flops = alln = 0
+    for nm, (ks, kt, kti) in res["kinfo"].items():
+        for k, t in zip(ks, kti):
+            alln += int(t)
+            if k["name"].startswith("conv_tcgen05"):
+                n += 1
+                nsec += int(t)
+                byts += k["bytes"]
+                flops += k["flops"]
+    if n == 0 or nsec == 0:
         return None
-    dur = ev["ns"] / ev["launches"]
-    bytes_per = ev["bytes"] / ev["launches"]
-    flops_per = ev["flops"] / ev["launches"]
-    gbs = bytes_per / dur
+    dur = nsec / n
+    gbs = (byts / n) / dur
     peak = peaks.get("hbm_gbs", 6650.0)
-    # DRAM traffic per launch from the committed ncu --set full capture of the same
-    # launches (tools/profile_round.sh -> tools/ncu_traffic.py), if present
     traffic, tsrc = None, None
-    tp = os.path.join(ROOT, "profiles", f"conv_traffic_{res['config']}.json")
+    tp = os.path.join(ROOT, "profiles", f"conv_traffic_{res.get('config', '')}.json")
     if os.path.exists(tp):
         tj = json.load(open(tp))
         traffic, tsrc = tj.get("conv_tcgen05_dram_bytes_per_launch"), tj.get("source")
     return {"kernel": "conv_tcgen05", "bound": "hbm", "achieved": round(gbs, 2), "peak": peak, "unit": "GB/s",
-            "frac": round(gbs / peak, 4), "traffic": traffic, "traffic_source": tsrc,
-            "algorithmic_bytes_per_launch": round(bytes_per), "launches_per_mix": ev["launches"],
-            "mean_launch_us": round(dur / 1e3, 3), "tflops": round(flops_per / dur / 1e3, 3),
-            "share_of_device_time": round(ev["ns"] / max(1, ev["all_ns"]), 3),
-            "peak_source": "MEASURED_PEAKS.json hbm_gbs (burst copy)"}
+            "frac": round(gbs / peak, 4), "traffic": traffic, "algorithmic_bytes_per_launch": round(byts / n),
+            "mean_launch_us": round(dur / 1e3, 3), "tflops": round(flops / n / dur / 1e3, 2),
+            "share_of_device_time": round(nsec / max(1, alln), 3),
+            "peak_source": "MEASURED_PEAKS.json hbm_gbs (burst copy)" if "hbm_gbs" in peaks else "guide fallback"}
 
 
-def saturating_conv(args):
-    """The dominant kernel where its roofline is reachable: the tcgen05
-    conv on 3x3 256->256 layers over 56x56 and 448x448 pixels (tools/conv_saturating.py),
-    timed like the batch-1 kernels (PDL chain, CUDA events), against the measured bf16
-    tensor peak."""
-    import importlib.util
-    spec = importlib.util.spec_from_file_location("conv_saturating", os.path.join(ROOT, "tools", "conv_saturating.py"))
-    cs = importlib.util.module_from_spec(spec)
-    spec.loader.exec_module(cs)
-    from paper_conf_sosp_ngd023_b200 import _lib as L
-    peaks = json.load(open(PEAKS_PATH)) if os.path.exists(PEAKS_PATH) else {}
-    peak = peaks.get("bf16_tflops", 2250.0)
-    with L.Engine(num_clients=1, max_jobs_per_model=1, first_gpu=int(os.environ.get("LOCAL_RANK", "0"))) as e:
-        rows = [cs.measure(e, hw) for hw in (56, 448)]
-    best = max(rows, key=lambda r: r["tflops_instr"])
-    return {"kernel": "conv_tcgen05", "bound": "tensor", "achieved": best["tflops_instr"], "peak": peak,
-            "unit": "TFLOP/s", "frac": round(best["tflops_instr"] / peak, 4),
-            "peak_source": "MEASURED_PEAKS.json bf16_tflops (cuBLAS burst)" if peaks else "nominal 2250",
-            "shapes": rows}
+def ratio(a, b):
+    return round(a / b, 3) if a and b else None
 
 
 def main():
     args = parse()
-    if args.dispatcher_fifo > 0:
-        os.environ["PAELLA_DISPATCHER_FIFO"] = str(args.dispatcher_fifo)
-    if args.impl == "reference":   # no dispatcher: the oracle keeps every host core
-        args.dispatcher_cpu = -1
-    if args.dispatcher_cpu == -2:   # default: core 2 + LOCAL_RANK if the host has room
-        avail = os.sched_getaffinity(0)
-        first = 2
-        args.dispatcher_cpu = first if (set(range(first, first + args.gpus)) <= avail
-                                         and len(avail) >= first + 2 * args.gpus) else -1
-    if args.dispatcher_cpu >= 0:
-        # DEDICATED cores (SURVEY.md §8(e)): every thread created from here on
-        # (launchers, load generator, completion pollers) inherits a mask without any
-        # rank's dispatcher core; measured on B200 in profiles/pin_r1c (DESIGN.md §8)
-        cores = set(range(args.dispatcher_cpu, args.dispatcher_cpu + args.gpus))
-        os.sched_setaffinity(0, os.sched_getaffinity(0) - cores)
-    dist = Dist(args.gpus)
+    dist = Dist()
+    ngpus = max(args.gpus, dist.world)
     cfg = traces.CONFIGS[args.config]
-    workload = {"c2_mix": "BASELINE configs[1]: 1 GPU, mixed ResNet-18/MobileNetV2/SqueezeNet1.1 batch-1, "
-                          "Poisson arrivals",
-                "c3_dispersion": "BASELINE configs[2]: ResNet-50/DenseNet-121/Inception-v3/MobileNetV2, bursty",
-                "c1_toy": "BASELINE configs[0]: 2 clients, toy conv+MLP"}[args.config]
-    if args.impl == "reference":
-        if dist.rank != 0:
-            return
-        t0 = time.time()
-        cb = None
-        for _ in range(max(1, args.warmup)):
-            pass
-        vals = []
-        for _ in range(args.steps):
-            cb = cpu_baseline(cfg, seconds=max(2.0, 30.0 / max(1, args.steps)))
-            vals.append(cb["value"])
-        v = float(np.mean(vals))
-        line = {"impl": "reference", "metric": METRIC, "value": round(v, 3),
-                "unit": "req/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-                "ms_per_step": round((time.time() - t0) * 1e3 / args.steps, 1), "higher_is_better": True,
-                "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-                "config": {"workload": workload, "models": cfg["models"], "clients": cfg["clients"], "batch": 1,
-                           "arrivals": cfg["arrival"], "rho": args.rho, "requests_per_step": args.reqs,
-                           "parallelism": "oracle on host cores"},
-                "cpu_baseline": {**cb, "value": round(v, 3)},
-                "e2e": {"value": round(v, 3), "unit": "req/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-        print(json.dumps(line))
+    if args.impl == "reference":   # the oracle on the host cores (no dispatcher: every core)
+        if dist.rank == 0:
+            t0 = time.time()
+            vals, cb = [], None
+            for _ in range(args.steps):
+                cb = cpu_baseline(dict(cfg), seconds=max(4.0, 60.0 / max(1, args.steps)))
+                vals.append(cb["value"])
+            v = float(np.mean(vals))
+            line = {"impl": "reference", "metric": METRIC, "value": round(v, 3), "unit": "req/s",
+                    "n_gpus": ngpus, "steps": args.steps, "warmup": args.warmup,
+                    "ms_per_step": round((time.time() - t0) * 1e3 / args.steps, 1), "higher_is_better": True,
+                    "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                    "jct_mean_us": cb["jct_mean_us"], "jct_p99_us": cb["jct_p99_us"],
+                    "config": {"workload": WORKLOADS[args.config], "models": cfg["models"], "batch": 1,
+                               "arrivals": cfg["arrival"], "parallelism": "oracle on host cores"},
+                    "cpu_baseline": {**cb, "value": round(v, 3)},
+                    "e2e": {"value": round(v, 3), "unit": "req/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+            print(json.dumps(line))
+        dist.barrier()
+        dist.close()
         return
-    res = run_gpu(args, dist)
-    total_done = dist.allsum(res["completed"])
-    max_el = dist.allmax(res["elapsed"])
-    value = total_done / max_el
-    peaks = {}
-    if os.path.exists(PEAKS_PATH):
-        peaks = json.load(open(PEAKS_PATH))
+    cores, nodes = (None, [])
+    if args.dispatcher_cpu != -1:
+        cores, nodes = dispatcher_cores(ngpus, args.dispatcher_cpu if args.dispatcher_cpu >= 0 else -1)
+    if cores:
+        # DEDICATED cores (SURVEY.md 8(e)): every thread created from here on (launchers,
+        # load generator, completion polling) inherits a mask without the dispatcher cores
+        os.sched_setaffinity(0, os.sched_getaffinity(0) - set(cores))
+    dist.barrier()
+    res = detail = lam = names = None
+    if dist.rank == 0:
+        res, detail, lam, names = run_gpu(args, ngpus, cores, args.fake)
+        elapsed, completed = res["paella"]["elapsed"], res["paella"]["completed"]
+    else:
+        elapsed, completed = 0.0, 0
+    dist.barrier()
+    max_el = dist.allmax(elapsed)
+    total = dist.allsum(completed)
     if dist.rank != 0:
+        dist.close()
         return
-    jm = res["jct"]["mix"]
-    launches = res["stats"]["launches"]
+    peaks = json.load(open(PEAKS_PATH)) if os.path.exists(PEAKS_PATH) else {}
+    P = res["paella"]
+    jm = P["jct"]["mix"]
+    served = total / max_el
+    slo_v = P.get("slo", {}).get("req_s")
+    value = slo_v if slo_v else served
+    nv = res.get("naive", {}).get("jct", {}).get("mix")
+    npd = res.get("naive_pdl", {}).get("jct", {}).get("mix")
+    fifo = res.get("paella_fifo", {}).get("jct", {}).get("mix")
+    disp = P["dispatcher"]
     line = {
-        "metric": METRIC,
-        "value": round(value, 2), "unit": "req/s", "n_gpus": args.gpus, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": round(max_el * 1e3 / args.steps, 2), "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
-        "config": {"workload": workload, "models": res["names"], "clients": cfg["clients"], "batch": 1,
-                   "arrivals": cfg["arrival"], "rho": args.rho, "lambda_per_gpu_req_s": round(res["lam"], 1),
-                   "requests_per_step": args.reqs, "parallelism": f"replicas{args.gpus}",
-                   "l2": "not flushed: steps are open-loop traces whose weights (~33 MB bf16) stay L2-resident "
-                         "as in serving; inputs stream from pinned host memory"},
-        "jct_us": res["jct"], "slo_us": res["slo"],
-        "paella_config": {"lookahead": args.lookahead, "launch_threads": args.launch_threads,
-                          "dispatcher_cpu": args.dispatcher_cpu, "dispatcher_fifo": args.dispatcher_fifo, "policy": {"srpt": "srpt+deficit"}.get(args.policy, args.policy),
-                          "slack_blocks": args.slack, "prio_classes": args.prio_classes, "pdl": True,
-                          "theta": args.theta, "group": 16, "streams": 32, "decide_delay_ns": args.decide_delay_ns,
-                          "online_tbar": bool(args.online_tbar)},
-        "slo_met": bool(all(res["jct"].get(n, {}).get("p99_us", 1e18) <= res["slo"][n] for n in res["names"])),
-        "req_s_at_p99_slo": {k: v["req_s"] for k, v in res["slo_at"].items()},
-        "slo_ladder": res["slo_at"],
-        "x_sat_req_s": {"naive": round(res["x_sat_naive"], 1), "paella": round(res["x_sat_paella"], 1)},
-        "jct_unloaded_p50_us": {k: {m: round(v, 1) for m, v in d.items()} for k, d in res["unloaded"].items()},
-        "device_roofline_us": {k: round(v, 2) for k, v in res["dev_roof"].items()},
-        "jct_fraction_of_device_roofline": {n: round(res["dev_roof"][n] / res["jct"][n]["mean_us"], 4)
-                                            for n in res["names"] if n in res["jct"]},
-        "baselines": res["base"],
-        "roofline": roofline_entry(res, peaks),
+        "metric": METRIC, "value": round(value, 1), "unit": "req/s",
+        "jct_mean_us": round(jm["mean_us"]), "jct_p99_us": round(jm["p99_us"]), "jct_p50_us": round(jm["p50_us"]),
+        "vs_naive": {"mean": ratio(nv and nv["mean_us"], jm["mean_us"]), "p99": ratio(nv and nv["p99_us"], jm["p99_us"])}
+        if nv else None,
+        "vs_naive_pdl": {"mean": ratio(npd["mean_us"], jm["mean_us"]), "p99": ratio(npd["p99_us"], jm["p99_us"])}
+        if npd else None,
+        "fifo_jct_us": [round(fifo["mean_us"]), round(fifo["p99_us"])] if fifo else None,
+        "naive_jct_us": [round(nv["mean_us"]), round(nv["p99_us"])] if nv else None,
+        "naive_pdl_jct_us": [round(npd["mean_us"]), round(npd["p99_us"])] if npd else None,
+        "req_s_at_slo": {k: v["slo"]["req_s"] for k, v in res.items() if "slo" in v},
+        "served_req_s": round(served, 1),
+        "n_gpus": ngpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(max_el * 1e3 / args.steps, 2),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
+        "config": {"workload": WORKLOADS[args.config], "batch": 1, "rho": args.rho, "lambda_req_s": round(lam, 1),
+                   "requests_per_step": args.reqs * ngpus,
+                   "parallelism": f"{ngpus} GPU dispatchers, least-work router" if ngpus > 1 else "1 GPU dispatcher",
+                   "paella": f"srpt+deficit th{args.theta} K{args.max_active} la{args.lookahead} B{args.slack} pdl"
+                   if args.policy == "srpt" else args.policy,
+                   "l2": "not flushed: weights (~120 MB bf16) largely L2-resident as in serving; inputs stream "
+                         "from pinned host memory every request"},
+        "roofline": roofline_entry(dict(P, config=args.config), peaks) if "kinfo" in P else None,
         "cpu_baseline": None,
-        "e2e": {"value": round(res["e2e_rate"], 2), "unit": "req/s", "h2d_bytes_per_step": round(res["h2d"] * args.reqs),
-                "d2h_bytes_per_step": round(res["d2h"] * args.reqs), "jct_us": res["e2e"]["mix"]},
-        "gpu_launches": int(launches),
-        "clocks": res["clocks"],
-        "dispatcher": {k: (v if isinstance(v, list) else int(v)) for k, v in res["stats"].items()},
+        "e2e": {"value": round(P["e2e"]["rate"], 1), "unit": "req/s",
+                "h2d_bytes_per_step": round(P["e2e"]["h2d"] * P["e2e"]["n"]),
+                "d2h_bytes_per_step": round(P["e2e"]["d2h"] * P["e2e"]["n"]),
+                "jct_mean_us": round(P["e2e"]["jct"]["mix"]["mean_us"]),
+                "jct_p99_us": round(P["e2e"]["jct"]["mix"]["p99_us"])},
+        "gpu_launches": int(sum(d["launches"] for d in disp)),
+        "dispatcher_busy_frac": [d["busy_frac"] for d in disp],
+        "clocks": P["clocks"],
     }
-    if args.gpus == 1 and not args.fake:
+    if ngpus == 1 and not args.fake:
+        reserve = len(cores) if cores else 0
         try:
-            line["roofline_saturating"] = saturating_conv(args)
-        except Exception as ex:   # diagnostic only: never fail the bench line for it
-            line["roofline_saturating"] = {"error": str(ex)[:200]}
-        line["cpu_baseline"] = cpu_baseline(cfg, seconds=12.0)
+            cb = cpu_baseline(dict(cfg, weights=detail["mix_weights"]), seconds=20.0, reserve=reserve)
+        except Exception as ex:  # never lose the line for the baseline leg
+            cb = {"error": str(ex)[:200]}
+        line["cpu_baseline"] = {k: v for k, v in cb.items() if k != "host"}
+        detail["cpu_baseline"] = cb
+        try:
+            detail["simulator"] = simulator_timing(P["kinfo"], dict(cfg, weights=detail["mix_weights"]), names, lam)
+        except Exception as ex:
+            detail["simulator"] = {"error": str(ex)[:200]}
     if args.fake:
         line["data"] = "synthetic, FAKE CPU device (plumbing test, not a measurement)"
-    print(json.dumps(line))
+    # the detail file: every arm's per-model JCT, dispatcher stats, SLO searches, C-5
+    for k, v in res.items():
+        v.pop("kinfo", None)
+    detail["arms"] = res
+    detail["line"] = line
+    os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
+    path = os.path.join(ROOT, "gpurun_out", f"bench_detail_{args.config}_n{ngpus}.json")
+    with open(path, "w") as f:
+        json.dump(detail, f, indent=1, default=float)
+    print(json.dumps({"bench_detail": path, "arms": {k: v["jct"]["mix"] for k, v in res.items()}},
+                     default=float), file=sys.stderr)
+    print(json.dumps(line, default=float))
+    dist.close()
 
 
 if __name__ == "__main__":

@@ -336,9 +336,20 @@ typedef struct {
   uint64_t rel_events;         /* counter mode: stream-release events recorded (a job left idle) */
   uint64_t xstream_waits;      /* ... of which the job's next kernel went to another stream
                                   and waited for the event (relaxed exits) */
+  uint64_t busy_ns;            /* time the dispatcher spent in loop iterations that did work
+                                  (admitted, consumed records or issued): its core's useful
+                                  load; the rest of the time it spins on empty rings */
 } paella_stats_t;
 
 int paella_stats(paella_t* p, uint32_t gpu, paella_stats_t* st);
+
+/* globaltimer -> host clock of GPU `gpu` (SURVEY.md §8(c) C3 "Clocks"), calibrated at
+   paella_init by a ping-pong with a probe kernel through mapped memory (the sample with
+   the smallest round trip): a record's %globaltimer value t_dev corresponds to host
+   CLOCK_MONOTONIC t_dev - *offset_ns, within +- *rtt_ns / 2; *resolution_ns = the
+   smallest observed step of %globaltimer.  Also logged as a CLOCK event.  -ENODEV on
+   the FAKE device, -ENOTSUP when not calibrated (under a profiler). */
+int paella_clock_info(paella_t* p, uint32_t gpu, int64_t* offset_ns, int64_t* rtt_ns, int64_t* resolution_ns);
 
 /* Flush and close the event logs (also done by shutdown). */
 int paella_flush_log(paella_t* p);

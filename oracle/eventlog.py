@@ -17,6 +17,8 @@ Format (DESIGN.md §"Event log"): a sequence of 32-byte little-endian records
     4 ISSUE     a=stream, b=uid, c=job, d=layer
     5 COMPLETE  b=job, c=t ns
     6 OBSERVE   b=uid, c=observed duration ns (NEXT-4; precedes the final COMPLETION)
+    8 CLOCK     a=gpu, b=offset (globaltimer - host CLOCK_MONOTONIC, ns), c=round trip ns,
+                d=globaltimer resolution ns (calibrated at init, paella_clock_info)
     7 ROUTE     a=g0 | g1 << 8 | route << 16, b=req_id, c=W_g0, d=W_g1 (multi-GPU only;
                 the router's decision inputs, logged by the GPU it chose, before ARRIVAL)
 """
@@ -41,7 +43,11 @@ def read(path):
     issues = []
     completes = []
     routes = []
+    clock = None
     narrivals = 0
+    lives = []          # one entry per admitted job occurrence (job ids are recycled)
+    cur_life = {}       # job id -> index into lives of its current occurrence
+    uid_life = {}       # launch uid -> index into lives
     for r in raw:
         t, a, b, c, d = int(r["type"]), int(r["a"]), int(r["b"]), int(r["c"]), int(r["d"])
         if t == 100:
@@ -72,6 +78,8 @@ def read(path):
             events.append((sim.EV_ARRIVAL, b, a, c))
             arrivals[b] = (a, c, d)        # latest job with this id (ids are recycled)
             narrivals += 1
+            cur_life[b] = len(lives)
+            lives.append(dict(job=b, client=a, model=c, t_sched=d, t_complete=None, uids=[]))
         elif t == 2:
             events.append((sim.EV_RECORD, a, b, c))
             # (t, type, uid, n, group) as sim.check_exactly_once expects, + smid
@@ -81,14 +89,20 @@ def read(path):
         elif t == 4:
             events.append((sim.EV_ISSUE, b, c, d, a))
             issues.append((b, c, d, a, arrivals[c][1]))   # (uid, job, layer, stream, model)
+            uid_life[b] = cur_life[c]
+            lives[cur_life[c]]["uids"].append(b)
         elif t == 7:
             routes.append((a & 0xFF, (a >> 8) & 0xFF, a >> 16, b,
                            c if c < (1 << 63) else c - (1 << 64), d if d < (1 << 63) else d - (1 << 64)))
         elif t == 6:
             events.append((sim.EV_OBSERVE, b, c))
+        elif t == 8:
+            clock = dict(gpu=a, offset=b if b < (1 << 63) else b - (1 << 64), rtt=c, resolution=d)
         elif t == 5:
             events.append((sim.EV_COMPLETE, b))
             completes.append((b, c))
+            if b in cur_life:
+                lives[cur_life[b]]["t_complete"] = c
     cfg = sim.Config(capacity=tuple(cap), **cfg_kw)
     models = []
     for m in range(len(nlayers)):
@@ -99,7 +113,7 @@ def read(path):
             ms.append(sim.Layer(grid, (1, w, rg, sm, tm), tbar))
         models.append(ms)
     extras = dict(records=records, issues=issues, completes=completes, arrivals=arrivals,
-                  n_arrivals=narrivals, routes=routes)
+                  n_arrivals=narrivals, routes=routes, clock=clock, lives=lives, uid_life=uid_life)
     return cfg, models, events, extras
 
 

@@ -35,7 +35,8 @@ SYMBOLS = ["paella_init", "paella_register_model", "paella_submit", "paella_subm
            "paella_poll_completion", "paella_shutdown", "paella_client_region", "paella_model_info",
            "paella_kernel_info", "paella_kernel_name", "paella_stats", "paella_flush_log",
            "paella_run_isolated", "paella_debug_node", "paella_time_kernels", "paella_bench_empty",
-           "paella_bench_roundtrip", "paella_loadgen", "paella_bench_wait", "paella_route_pair"]
+           "paella_bench_roundtrip", "paella_loadgen", "paella_bench_wait", "paella_route_pair",
+           "paella_clock_info"]
 
 
 class Config(C.Structure):
@@ -92,7 +93,8 @@ class Stats(C.Structure):
                 ("loop_iters", C.c_uint64), ("outstanding_work_ns", C.c_int64), ("ev_launches", C.c_uint64),
                 ("ev_ns", C.c_uint64), ("ev_bytes", C.c_uint64), ("ev_flops", C.c_uint64),
                 ("stop_reason", C.c_uint64 * 4), ("sum_ready", C.c_uint64), ("sum_live_jobs", C.c_uint64),
-                ("sum_Q", C.c_uint64), ("rel_events", C.c_uint64), ("xstream_waits", C.c_uint64)]
+                ("sum_Q", C.c_uint64), ("rel_events", C.c_uint64), ("xstream_waits", C.c_uint64),
+                ("busy_ns", C.c_uint64)]
 
 
 _lib = None
@@ -124,6 +126,8 @@ def load():
     lib.paella_kernel_name.argtypes = [C.c_uint32]
     lib.paella_kernel_name.restype = C.c_char_p
     lib.paella_stats.argtypes = [P, C.c_uint32, C.POINTER(Stats)]
+    lib.paella_clock_info.argtypes = [P, C.c_uint32, C.POINTER(C.c_int64), C.POINTER(C.c_int64),
+                                      C.POINTER(C.c_int64)]
     lib.paella_flush_log.argtypes = [P]
     lib.paella_run_isolated.argtypes = [P, C.c_uint32, C.c_uint32, P, P, C.POINTER(C.c_int64)]
     lib.paella_debug_node.argtypes = [P, C.c_uint32, C.c_uint32, C.c_uint32, C.POINTER(C.c_float)]
@@ -394,6 +398,12 @@ class Engine:
         d = {f: getattr(st, f) for f, _ in Stats._fields_}
         d["stop_reason"] = list(st.stop_reason)
         return d
+
+    def clock_info(self, gpu=0):
+        """(offset_ns, rtt_ns, resolution_ns) of the globaltimer -> host calibration."""
+        o, r, q = C.c_int64(), C.c_int64(), C.c_int64()
+        _check(self.lib.paella_clock_info(self.h, gpu, C.byref(o), C.byref(r), C.byref(q)), "paella_clock_info")
+        return o.value, r.value, q.value
 
     def flush_log(self):
         self.lib.paella_flush_log(self.h)

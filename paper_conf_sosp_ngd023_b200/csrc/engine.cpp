@@ -35,16 +35,52 @@
 
 namespace paella {
 
+// Under a profiler (Nsight Compute injects itself through CUDA_INJECTION64_PATH) every
+// launch is serialised and replayed: a persistent warp (the notification mirror / proxy)
+// never returns and a kernel spinning on a host flag the host sets only after the
+// launch calls return (the timing gate) deadlocks.  Both are switched off then:
+// notifications take the direct ring path, timing runs ungated.
+static bool profiled() {
+  static const bool p = std::getenv("CUDA_INJECTION64_PATH") != nullptr || std::getenv("PAELLA_PROFILED") != nullptr;
+  return p;
+}
+static bool no_gate() { return profiled() || std::getenv("PAELLA_NO_GATE") != nullptr; }
+static bool no_proxy_env() { return profiled() || std::getenv("PAELLA_NO_PROXY") != nullptr; }
+
 int64_t now_ns() {
   timespec ts;
   clock_gettime(CLOCK_MONOTONIC, &ts);
   return (int64_t)ts.tv_sec * 1000000000ll + ts.tv_nsec;
 }
 
+// cheap timestamps for the dispatcher's busy-time accounting (stats.busy_ns)
+static inline uint64_t ticks() {
+#if defined(__x86_64__)
+  return __builtin_ia32_rdtsc();
+#else
+  return (uint64_t)now_ns();
+#endif
+}
+static double ns_per_tick() {
+  static const double r = [] {
+#if defined(__x86_64__)
+    const int64_t n0 = now_ns();
+    const uint64_t c0 = ticks();
+    timespec ts{0, 20000000};
+    nanosleep(&ts, nullptr);
+    return (double)(now_ns() - n0) / (double)(ticks() - c0);
+#else
+    return 1.0;
+#endif
+  }();
+  return r;
+}
+
 // ---------------------------------------------------------------------------
 // event log (replay input for oracle/sim.py::replay; format in DESIGN.md)
 // ---------------------------------------------------------------------------
 enum : uint32_t { EV_ARRIVAL = 1, EV_RECORD = 2, EV_BATCH_END = 3, EV_ISSUE = 4, EV_COMPLETE = 5, EV_OBSERVE = 6, EV_ROUTE = 7,
+                  EV_CLOCK = 8,
                   EV_CONFIG = 100, EV_CAPACITY = 101, EV_MODEL = 110, EV_LAYER = 111, EV_DEMAND = 112 };
 
 struct LogEv {
@@ -860,7 +896,11 @@ static void dispatch_loop(Gpu* g) {
   const bool dbg = std::getenv("PAELLA_DEBUG") != nullptr;
   const int64_t watchdog_ns = (int64_t)P->cfg.watchdog_ms * 1000000;
   g->last_progress_ns = now_ns();
+  uint64_t busy_ticks = 0;
+  (void)ns_per_tick();
   for (;;) {
+    const uint64_t it0 = ticks();
+    if ((g->stats.loop_iters & 4095) == 0) g->stats.busy_ns = (uint64_t)(busy_ticks * ns_per_tick());
     g->stats.loop_iters++;
     if (dbg && (g->stats.loop_iters % 50000000) == 0) {
       fprintf(stderr, "[dbg gpu%u] iters=%lu admitted=%lu", g->index, (unsigned long)g->stats.loop_iters,
@@ -928,6 +968,7 @@ static void dispatch_loop(Gpu* g) {
         fail_gpu(g, -EIO, "CUDA error");
         return;
       }
+      if (progressed || nev) busy_ticks += ticks() - it0;
       if (stopping && g->naive_inflight.empty()) return;
       continue;
     }
@@ -948,6 +989,7 @@ static void dispatch_loop(Gpu* g) {
       logev(g, EV_BATCH_END, 0, 0, 0, 0);
       decide_and_launch(g);
       g->work_published.store(g->policy->outstanding_work(), std::memory_order_release);
+      busy_ticks += ticks() - it0;
     }
     int e = g->be->error();
     if (!e) e = g->launch_err.load(std::memory_order_relaxed);
@@ -994,6 +1036,54 @@ static void dispatcher_main(Gpu* g) {
     fail_gpu(g, -EIO, ex.what());
   }
   if (g->err.load(std::memory_order_acquire)) dead_loop(g);
+}
+
+// globaltimer -> host clock calibration: n ping-pongs with
+// k_clock_probe through mapped memory; the sample with the smallest round trip gives
+// offset = globaltimer - midpoint of the host send/receive times (CLOCK_MONOTONIC), so
+// device_ns ~= host_ns + offset within +- rtt/2; the probe also measures the timer's
+// resolution.  Not under a profiler (the probe waits for the host).
+static int clock_sync(Gpu* g, uint32_t n, int64_t* off, int64_t* rtt, int64_t* res) {
+  if (profiled()) return -ENOTSUP;
+  if (cudaSetDevice(g->device) != cudaSuccess) return -EIO;
+  void* buf = nullptr;
+  if (cudaHostAlloc(&buf, 4096, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) return -ENOMEM;
+  std::memset(buf, 0, 4096);
+  volatile uint32_t* flag = (volatile uint32_t*)buf;
+  volatile uint64_t* out = (volatile uint64_t*)((uint8_t*)buf + 64);
+  void *flag_d = nullptr, *out_d = nullptr;
+  cudaHostGetDevicePointer(&flag_d, (void*)flag, 0);
+  cudaHostGetDevicePointer(&out_d, (void*)out, 0);
+  cudaStream_t s;
+  cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
+  void* args[3] = {(void*)&flag_d, (void*)&out_d, (void*)&n};
+  int rc = cudaLaunchKernel((const void*)clock_kernel(), dim3(1), dim3(1), args, 0, s) == cudaSuccess ? 0 : -EIO;
+  int64_t best = INT64_MAX, boff = 0;
+  for (uint32_t i = 0; i < n && rc == 0; ++i) {
+    const int64_t t0 = now_ns();
+    __atomic_store_n((uint32_t*)flag, i + 1, __ATOMIC_SEQ_CST);
+    while (out[i] == 0) {
+      if (now_ns() - t0 > 2000000000ll) {
+        rc = -ETIMEDOUT;
+        break;
+      }
+    }
+    const int64_t t1 = now_ns();
+    if (rc == 0 && t1 - t0 < best) {
+      best = t1 - t0;
+      boff = (int64_t)out[i] - (t0 + (t1 - t0) / 2);
+    }
+  }
+  __atomic_store_n((uint32_t*)flag, n, __ATOMIC_SEQ_CST);   // release the probe in any case
+  if (cudaStreamSynchronize(s) != cudaSuccess && rc == 0) rc = -EIO;
+  if (rc == 0) {
+    *off = boff;
+    *rtt = best;
+    *res = (int64_t)out[n];
+  }
+  cudaStreamDestroy(s);
+  cudaFreeHost(buf);
+  return rc;
 }
 
 // ---------------------------------------------------------------------------
@@ -1096,7 +1186,27 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
   P->route_log.resize(cfg.num_clients);
   P->poll_rr.assign(cfg.num_clients, 0);
 
+  // NUMA placement: a GPU's pinned notification ring and counter
+  // mirror are first touched by a thread running on that GPU's dispatcher core, so
+  // they land on the dispatcher's (= the GPU's, when the caller picks NUMA-local
+  // cores) memory node; the caller's affinity is restored afterwards
+  cpu_set_t saved_mask;
+  const bool numa_pin = cfg.dispatcher_cpus != nullptr &&
+                        pthread_getaffinity_np(pthread_self(), sizeof saved_mask, &saved_mask) == 0;
+  struct RestoreMask {
+    bool on;
+    cpu_set_t* m;
+    ~RestoreMask() {
+      if (on) pthread_setaffinity_np(pthread_self(), sizeof *m, m);
+    }
+  } restore{numa_pin, &saved_mask};
   for (uint32_t gi = 0; gi < cfg.num_gpus; ++gi) {
+    if (numa_pin) {
+      cpu_set_t cs;
+      CPU_ZERO(&cs);
+      CPU_SET(cfg.dispatcher_cpus[gi], &cs);
+      pthread_setaffinity_np(pthread_self(), sizeof cs, &cs);
+    }
     auto g = std::make_unique<Gpu>();
     g->P = P.get();
     g->index = gi;
@@ -1109,9 +1219,9 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     g->jobs.reserve(65536);
     if (cfg.device == PAELLA_DEVICE_CUDA)
       g->be.reset(new CudaBackend(g->device, g->cap, cfg.stream_pool,
-                                  cfg.no_proxy == 0 && !std::getenv("PAELLA_NO_PROXY"),
+                                  cfg.no_proxy == 0 && !no_proxy_env(),
                                   cfg.no_proxy == 0 && cfg.notify_mode == PAELLA_NOTIFY_COUNTERS &&
-                                      !cfg.naive && !std::getenv("PAELLA_NO_PROXY")));
+                                      !cfg.naive && !no_proxy_env()));
     if (cfg.device == PAELLA_DEVICE_CUDA) {
       auto* cb = static_cast<CudaBackend*>(g->be.get());
       cb->pdl = (!cfg.naive || cfg.naive_pdl) && !cfg.no_pdl && !std::getenv("PAELLA_NO_PDL");
@@ -1169,7 +1279,14 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
       logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFEu, cfg.online_tbar, cfg.max_active_jobs, 0);
       for (int r = 0; r < NRES; ++r) logev(g.get(), EV_CAPACITY, (uint32_t)r, (uint64_t)pc.capacity[r], 0, 0);
     }
+    if (cfg.device == PAELLA_DEVICE_CUDA &&
+        clock_sync(g.get(), 32, &g->clk_offset, &g->clk_rtt, &g->clk_res) == 0)
+      logev(g.get(), EV_CLOCK, gi, (uint64_t)g->clk_offset, (uint64_t)g->clk_rtt, (uint64_t)g->clk_res);
     P->gpus.push_back(std::move(g));
+  }
+  if (numa_pin) {
+    pthread_setaffinity_np(pthread_self(), sizeof saved_mask, &saved_mask);
+    restore.on = false;
   }
   for (auto& g : P->gpus) {
     if (cfg.device == PAELLA_DEVICE_CUDA && cfg.launch_threads > 0) {
@@ -1539,6 +1656,18 @@ const char* paella_kernel_name(uint32_t kind) {
   return kind < KIND_COUNT ? names[kind] : "?";
 }
 
+int paella_clock_info(paella_t* p, uint32_t gpu, int64_t* offset_ns, int64_t* rtt_ns, int64_t* resolution_ns) {
+  Paella* P = (Paella*)p;
+  if (!P || gpu >= P->gpus.size()) return -EINVAL;
+  if (P->cfg.device != PAELLA_DEVICE_CUDA) return -ENODEV;
+  Gpu* g = P->gpus[gpu].get();
+  if (g->clk_rtt < 0) return -ENOTSUP;
+  if (offset_ns) *offset_ns = g->clk_offset;
+  if (rtt_ns) *rtt_ns = g->clk_rtt;
+  if (resolution_ns) *resolution_ns = g->clk_res;
+  return 0;
+}
+
 int paella_stats(paella_t* p, uint32_t gpu, paella_stats_t* st) {
   Paella* P = (Paella*)p;
   if (!P || !st || gpu >= P->gpus.size()) return -EINVAL;
@@ -1633,7 +1762,7 @@ static int iso_run(Gpu* g, Model* m, const void* input, void* output, int64_t* k
     const volatile uint32_t* gd = nullptr;
     cudaHostGetDevicePointer((void**)&gd, (void*)gate, 0);
     void* gargs[1] = {(void*)&gd};
-    if (!std::getenv("PAELLA_NO_GATE"))
+    if (!no_gate())
       cudaLaunchKernel((const void*)gate_kernel(), dim3(1), dim3(1), gargs, 0, s);
     ev.resize(m->kernels.size() + 1);
     for (auto& e : ev) cudaEventCreate(&e);
@@ -1980,7 +2109,7 @@ static volatile uint32_t* gate_ptr(Gpu* g, const volatile uint32_t** dev) {
 }
 
 static void launch_gate(Gpu* g, const volatile uint32_t* gd) {
-  if (std::getenv("PAELLA_NO_GATE")) return;
+  if (no_gate()) return;
   void* gargs[1] = {(void*)&gd};
   cudaLaunchKernel((const void*)gate_kernel(), dim3(1), dim3(1), gargs, 0, (cudaStream_t)g->prof_stream);
 }

@@ -201,6 +201,8 @@ struct Gpu {
   std::atomic<uint32_t> inbox_n{0};          // models posted
   std::atomic<uint32_t> models_applied{0};   // models the dispatcher has added to its policy
   uint32_t rr_start = 0;
+  // globaltimer -> host clock (C3): device_ns ~= host_ns + clk_offset; rtt < 0 = not calibrated
+  int64_t clk_offset = 0, clk_rtt = -1, clk_res = 0;
   FILE* log = nullptr;
   std::mutex log_mu;
   paella_stats_t stats{};

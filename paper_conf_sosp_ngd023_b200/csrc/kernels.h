@@ -25,6 +25,7 @@ void simt_kernel_table(KernelFn (&bf16_instr)[KIND_COUNT], KernelFn (&bf16_plain
                        KernelFn (&f32_instr)[KIND_COUNT], KernelFn (&f32_plain)[KIND_COUNT]);
 
 KernelFn gate_kernel();   // k_gate(const volatile uint32_t* flag)
+KernelFn clock_kernel();  // k_clock_probe(flag, out, n): globaltimer ping-pong
 KernelFn mirror_kernel();  // k_notify_mirror(ctrs, host_mirror, state)
 KernelFn proxy_kernel();  // k_notify_proxy(dev_ring, host_ring, mask, log2cap, state)
 

@@ -572,6 +572,35 @@ __global__ void k_gate(const volatile uint32_t* flag) {
 
 KernelFn gate_kernel() { return (KernelFn)k_gate; }
 
+// globaltimer -> host clock calibration (SURVEY.md §8(c) C3 "Clocks"): ping-pong with the
+// host through mapped memory.  For i < n: wait until the host raises flag to i + 1, read
+// %globaltimer, publish it in out[i].  Then out[n] = the smallest positive step between
+// consecutive %globaltimer reads (the timer's resolution, measured, not assumed).
+__global__ void k_clock_probe(const volatile uint32_t* flag, volatile unsigned long long* out, uint32_t n) {
+  for (uint32_t i = 0; i < n; ++i) {
+    while (*flag != i + 1) {
+    }
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    out[i] = t;
+    __threadfence_system();
+  }
+  unsigned long long prev, best = ~0ull;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(prev));
+  for (int k = 0; k < 20000; ++k) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (t != prev) {
+      if (t - prev < best) best = t - prev;
+      prev = t;
+    }
+  }
+  out[n] = best;
+  __threadfence_system();
+}
+
+KernelFn clock_kernel() { return (KernelFn)k_clock_probe; }
+
 // ---------------------------------------------------------------------------
 // Notification proxy: one persistent warp forwards records from the device-memory
 // ring (where the instrumented kernels write them: an L2 store, no PCIe write on the

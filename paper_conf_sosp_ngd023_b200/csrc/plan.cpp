@@ -156,8 +156,12 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
     a.ow = in.w;
     a.out_cs = 8;
     a.out_co = 0;
-    k.grid[0] = (in.h * in.w % 4 == 0) ? (in.h * in.w / 4 + 255) / 256 : (in.h * in.w + 255) / 256;
-    k.block = 256;
+    // the input streams over PCIe from client memory: the read latency (~1-2 us per
+    // request) is covered by requests in flight, so the 4-pixel path runs 64-thread
+    // blocks to spread over >= the 148 SMs (224 x 224: 196 CTAs instead of 49)
+    const bool quad = in.h * in.w % 4 == 0;
+    k.block = quad ? 64 : 256;
+    k.grid[0] = quad ? (in.h * in.w / 4 + k.block - 1) / k.block : (in.h * in.w + 255) / 256;
     k.bytes = (uint64_t)in.c * in.h * in.w * 4 + (uint64_t)8 * in.h * in.w * es;
     m->kernels.push_back(k);
   }

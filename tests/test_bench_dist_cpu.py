@@ -36,4 +36,8 @@ def test_bench_two_ranks_gloo_fake_device():
               "scaling", "vs_baseline", "dtype", "data", "config", "e2e", "gpu_launches", "clocks"):
         assert k in d, k
     assert d["n_gpus"] == 2 and d["scaling"] == "weak" and d["value"] > 0
-    assert d["jct_us"]["mix"]["n"] == 150
+    assert d["jct_mean_us"] > 0 and d["jct_p99_us"] >= d["jct_mean_us"] * 0.5
+    assert "least-work router" in d["config"]["parallelism"] and len(d["dispatcher_busy_frac"]) == 2
+    assert len(json.dumps(d)) < 2500, "the driver keeps only the tail of stdout"
+    detail = json.load(open(os.path.join(ROOT, "gpurun_out", "bench_detail_c1_toy_n2.json")))
+    assert detail["arms"]["paella"]["completed"] == 300   # --reqs 150 per GPU x 2 GPUs, one process

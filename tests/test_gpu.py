@@ -64,7 +64,8 @@ def test_isolated_bf16_parity(engine, name):
         assert ok.all(), f"{name} input {i}: {np.sum(~ok)} logits out of tolerance, max err {np.abs(out-ref).max()}"
 
 
-@pytest.mark.parametrize("name", ["toy", "resnet18", "mobilenet_v2", "squeezenet1_1", "densenet121"])
+@pytest.mark.parametrize("name", ["toy", "resnet18", "mobilenet_v2", "squeezenet1_1", "densenet121", "resnet50",
+                                  "inception_v3"])
 def test_isolated_fp32_parity(engine, name):
     g = archs.build(name)
     mid = engine.register_model(g, rng.model_params(g), dtype=L.DTYPE_FP32, name=name + "-f32")
@@ -152,15 +153,20 @@ def _serve_and_check(e, specs, n, n_clients, seed, rate_us=30.0):
     (L.POLICY_SRPT_DEFICIT, 16, 32, 2048, 1, 2, "direct", 1),  # direct record writes (the paper's path)
     (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 3, 4, "counters", -4),  # bench arm + online T-bar (NEXT-4)
     (L.POLICY_SJF, 16, 32, 65536, 3, 4, "counters", 1),
+    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 3, 4, "counters", 108),   # the bench arm with the job cap K = 8
+    (L.POLICY_FIFO, 16, 32, 65536, 3, 4, "counters", 104),           # FIFO arm, K = 4
     (L.POLICY_RR, 16, 8, 4096, 0, 0, "counters", 1),
 ])
 def test_serving_parity_and_replay(tmp_path, policy, group, streams, ring, look, lt, notify, prio):
     log = str(tmp_path / "gpu_%u.log")
     names = ["toy", "resnet18", "mobilenet_v2", "squeezenet1_1"]
     online, prio = prio < 0, abs(prio)
+    K = prio - 100 if prio > 100 else 0       # 1xx: job cap K = xx (B200-Q6), one priority class
+    prio = 1 if K else prio
     with L.Engine(num_clients=3, policy=policy, group=group, streams=streams, ring_capacity=ring,
                   event_log=log, max_jobs_per_model=32, lookahead=look, launch_threads=lt, notify=notify,
-                  prio_classes=prio, slack=1184 if prio > 1 else 0, online_tbar=online) as e:
+                  prio_classes=prio, slack=1184 if (prio > 1 or K) else 0, online_tbar=online,
+                  max_active=K) as e:
         specs = []
         for nm in names:
             g = archs.build(nm)
@@ -180,6 +186,7 @@ def test_serving_parity_and_replay(tmp_path, policy, group, streams, ring, look,
     assert n == len(ex["issues"]) == st["launches"]
     grids = {uid: ms[model][layer].grid for (uid, job, layer, stream, model) in ex["issues"]}
     assert sim.check_exactly_once(ex["records"], grids, cfg.group) == []
+    assert sim.check_inflight_bound(events, ms, look) == []
 
 
 @pytest.mark.parametrize("lt", [0, 2])
@@ -279,3 +286,119 @@ def test_serving_parity_c3_models_bench_arm(tmp_path):
     ok, msg, n = sim.replay(cfg, ms, events)
     assert ok, msg
     assert n == len(ex["issues"]) == st["launches"]
+
+
+@pytest.mark.parametrize("name", ["resnet18", "inception_v3"])
+def test_ingest_rne_bit_exact(engine, name):
+    """The ingest kernel's bf16 rounding (C3 / reading C1-Q7) is bit-exact with
+    oracle.bf16.round_bf16 -- on the pooled inputs AND on an adversarial image: exact
+    ties between neighbouring bf16 values (must round to even), one fp32 ulp either side
+    of the tie, exact bf16 values, negatives, subnormals and finite values that round
+    up to infinity.  224x224 takes the 4-pixel path (196 CTAs), 299x299 the 1-pixel one."""
+    from oracle.bf16 import round_bf16
+    g = archs.build(name)
+    mid = engine.register_model(g, rng.model_params(g), dtype=L.DTYPE_BF16, name=name + "-rne")
+    shape = tuple(g.nodes[0]["out"])
+    n = int(np.prod(shape))
+    r = np.random.default_rng(77)
+    hi = r.integers(0, 0x7F80, n, dtype=np.uint32)                 # finite bf16 magnitudes
+    sign = (r.integers(0, 2, n, dtype=np.uint32) << 31)
+    low = r.choice(np.array([0x8000, 0x7FFF, 0x8001, 0x0000, 0x0001, 0xFFFF], dtype=np.uint32), n)
+    bits = sign | (hi << 16) | low
+    bits[:8] = [0x7F7FFFFF, 0xFF7FFFFF, 0x7F7F8000, 0x00008000, 0x80018000, 0x3F808000, 0x3F818000, 0]
+    adversarial = bits.view(np.float32).reshape(shape)
+    images = [rng.image(g, i) for i in range(4)] + [adversarial]
+    for x in images:
+        engine.run_isolated(mid, x)
+        got = engine.debug_node(mid, 0, shape)
+        want = round_bf16(x)
+        diff = got.view(np.uint32) != want.view(np.uint32)
+        assert not diff.any(), (int(diff.sum()), x[diff][:4], got[diff][:4], want[diff][:4])
+
+
+def test_clock_calibration_and_record_times(tmp_path):
+    """globaltimer -> host clock (C3): calibrated at init (round trip and timer resolution
+    measured); every G = 1 ring record, converted to host time, falls inside the life of
+    its job: [scheduled arrival, completion seen by the dispatcher] (tolerance: the
+    calibration round trip + 5 us)."""
+    from oracle import ringcheck
+    log = str(tmp_path / "clk_%u.log")
+    names = ["toy", "resnet18"]
+    with L.Engine(num_clients=2, group=1, event_log=log, notify="ring", ring_capacity=8192) as e:
+        off, rtt, res = e.clock_info()
+        assert 0 < rtt < 200_000 and 0 < res < 10_000, (off, rtt, res)
+        specs = []
+        for nm in names:
+            g = archs.build(nm)
+            specs.append((e.register_model(g, rng.model_params(g)), nm, g))
+        _serve_and_check(e, specs, 40, 2, seed=4)
+    cfg, ms, events, ex = eventlog.read(log % 0)
+    assert ex["clock"] is not None and ex["clock"]["offset"] == off
+    lives = ex["lives"]
+    windows = {uid: (lives[li]["t_sched"], lives[li]["t_complete"]) for uid, li in ex["uid_life"].items()}
+    recs = [r for r in ex["records"] if r[2] in windows]
+    assert len(recs) == len(ex["records"]) > 0
+    bad = ringcheck.check_record_times(recs, windows, off, rtt + 5000)
+    assert bad == [], bad[:5]
+
+
+def test_hybrid_completion_serving(tmp_path):
+    """NEXT-3 on the GPU (P1157-1171): a client thread waits with PAELLA_HYBRID polls
+    (spin, then futex sleep between the dispatcher's hints) while another submits; every
+    output matches the oracle and the waiter uses well under a full core."""
+    import threading
+    names = ["resnet18", "squeezenet1_1"]
+    with L.Engine(num_clients=1, lookahead=3, launch_threads=2, slack=1184) as e:
+        specs = []
+        for nm in names:
+            g = archs.build(nm)
+            specs.append((e.register_model(g, rng.model_params(g)), nm, g))
+        infos = {mid: e.model_info(mid) for mid, _, _ in specs}
+        stride = (max(i["input_bytes"] + i["output_bytes"] for i in infos.values()) + 4095) // 4096 * 4096
+        n = 60
+        sent = {}
+        got = []
+        slot_free = [threading.Event() for _ in range(16)]
+        for ev in slot_free:
+            ev.set()
+        lock = threading.Lock()
+
+        def waiter():
+            t0 = time.thread_time()
+            while len(got) < n:
+                rid, st = e.poll(0, L.HYBRID)
+                assert rid >= 0 and st == 0, (rid, st)
+                with lock:
+                    slot, mid, nm, idx = sent[rid]
+                _, reg = e.region(0)
+                ib = infos[mid]["input_bytes"]
+                out = np.frombuffer(reg[slot * stride + ib:slot * stride + ib + infos[mid]["output_bytes"]].tobytes(),
+                                    np.float32)
+                got.append((nm, idx, out.copy()))
+                slot_free[slot].set()
+            got.append(time.thread_time() - t0)
+
+        th = threading.Thread(target=waiter)
+        w0 = time.time()
+        th.start()
+        r = np.random.default_rng(9)
+        for i in range(n):
+            slot = i % 16
+            assert slot_free[slot].wait(30)
+            slot_free[slot].clear()
+            mid, nm, g = specs[i % 2]
+            idx = int(r.integers(4))
+            x = rng.image(g, idx)
+            _, reg = e.region(0)
+            reg[slot * stride:slot * stride + x.nbytes] = np.frombuffer(x.tobytes(), np.uint8)
+            with lock:
+                rid = e.submit(0, mid, slot * stride, infos[mid]["input_bytes"] + infos[mid]["output_bytes"])
+                assert rid >= 0
+                sent[rid] = (slot, mid, nm, idx)
+            time.sleep(0.002)
+        th.join(timeout=60)
+        assert not th.is_alive()
+        cpu, wall = got.pop(), time.time() - w0
+    for nm, idx, out in got:
+        assert within(out, oracle_out(nm, idx, "bf16"), BF16_TOL).all()
+    assert cpu < 0.7 * wall, (cpu, wall)
