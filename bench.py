@@ -407,6 +407,13 @@ def run_gpu(args, ngpus, cores, fake):
         "naive_pdl": dict(naive=True, instrument=False, naive_pdl=True, route=L.ROUTE_ROUND_ROBIN),
         "paella_paper": dict(policy=L.POLICY_SRPT_DEFICIT, theta=100, lookahead=0, slack=0, pdl=False,
                              route=L.ROUTE_LEAST_WORK),
+        # Table 3 variants (P1341-1359, NEXT-2): Paella-SS = job dispatch through the memory
+        # channels onto ONE stream (FIFO); Paella-MS-jbj = job dispatch onto many streams
+        # (= the naive arm, which already uses the memory channels); Paella-MS-kbk = kernel
+        # by kernel dispatch, CUDA decides (no occupancy predicate, arrival order)
+        "paella_ss": dict(naive=True, instrument=False, streams=1, route=L.ROUTE_ROUND_ROBIN),
+        "paella_ms_kbk": dict(policy=L.POLICY_FIFO, lookahead=0, slack=1 << 30, pdl=False,
+                              route=L.ROUTE_LEAST_WORK),
     }
     want = ["paella"] + ([] if args.no_baselines else
                          [a for a in args.arms.split(",") if a and a != "paella" and a in arms_kw])
@@ -482,6 +489,11 @@ def run_gpu(args, ngpus, cores, fake):
                 kinfo[nm] = (ks, kt, kti)
             r["dev_roof"] = dev_roof
             r["kinfo"] = kinfo
+            # the served kernel table (simulator inputs, tools/sim_delay_sweep.py)
+            detail["kernels"] = {nm: [dict(name=k["name"], grid=k["grid"], block=k["block"], regs=k["regs"],
+                                           smem=k["smem"], tmem=k["tmem_cols"], tbar_ns=k["tbar_ns"],
+                                           plain_ns=int(p), instr_ns=int(q), bytes=k["bytes"], flops=k["flops"])
+                                      for k, p, q in zip(*kinfo[nm])] for nm in names}
             # end to end: the client copies every input into its region and the logits out
             t, mm, ii = make_trace(n_step, lam, cfg, len(names), seed=seed0 + 500)
             e2e_jct, e2e_el = a.serve(t, mm, ii, copy_inputs={m: pool[m] for m in range(len(names))})

@@ -351,6 +351,12 @@ int paella_stats(paella_t* p, uint32_t gpu, paella_stats_t* st);
    the FAKE device, -ENOTSUP when not calibrated (under a profiler). */
 int paella_clock_info(paella_t* p, uint32_t gpu, int64_t* offset_ns, int64_t* rtt_ns, int64_t* resolution_ns);
 
+/* Re-calibrate GPU `gpu`'s clock now (the two clocks drift apart by ppm): a new CLOCK
+   event is written to its event log at the dispatcher's current position, so records
+   can be converted by interpolating between calibrations.  Blocks for ~100 us; do not
+   call it with a profiler attached.  0, -ENODEV (FAKE device), -ENOTSUP, -EIO. */
+int paella_clock_sync(paella_t* p, uint32_t gpu);
+
 /* Flush and close the event logs (also done by shutdown). */
 int paella_flush_log(paella_t* p);
 

@@ -17,8 +17,9 @@ Format (DESIGN.md §"Event log"): a sequence of 32-byte little-endian records
     4 ISSUE     a=stream, b=uid, c=job, d=layer
     5 COMPLETE  b=job, c=t ns
     6 OBSERVE   b=uid, c=observed duration ns (NEXT-4; precedes the final COMPLETION)
-    8 CLOCK     a=gpu, b=offset (globaltimer - host CLOCK_MONOTONIC, ns), c=round trip ns,
-                d=globaltimer resolution ns (calibrated at init, paella_clock_info)
+    8 CLOCK     a=gpu | resolution ns << 8, b=offset (globaltimer - host CLOCK_MONOTONIC, ns),
+                c=round trip ns, d=host time of the calibration sample (at init and at every
+                paella_clock_sync)
     7 ROUTE     a=g0 | g1 << 8 | route << 16, b=req_id, c=W_g0, d=W_g1 (multi-GPU only;
                 the router's decision inputs, logged by the GPU it chose, before ARRIVAL)
 """
@@ -43,7 +44,7 @@ def read(path):
     issues = []
     completes = []
     routes = []
-    clock = None
+    clocks = []
     narrivals = 0
     lives = []          # one entry per admitted job occurrence (job ids are recycled)
     cur_life = {}       # job id -> index into lives of its current occurrence
@@ -97,7 +98,8 @@ def read(path):
         elif t == 6:
             events.append((sim.EV_OBSERVE, b, c))
         elif t == 8:
-            clock = dict(gpu=a, offset=b if b < (1 << 63) else b - (1 << 64), rtt=c, resolution=d)
+            clocks.append(dict(gpu=a & 0xFF, resolution=a >> 8, offset=b if b < (1 << 63) else b - (1 << 64),
+                               rtt=c, at=d))
         elif t == 5:
             events.append((sim.EV_COMPLETE, b))
             completes.append((b, c))
@@ -113,7 +115,7 @@ def read(path):
             ms.append(sim.Layer(grid, (1, w, rg, sm, tm), tbar))
         models.append(ms)
     extras = dict(records=records, issues=issues, completes=completes, arrivals=arrivals,
-                  n_arrivals=narrivals, routes=routes, clock=clock, lives=lives, uid_life=uid_life)
+                  n_arrivals=narrivals, routes=routes, clocks=clocks, lives=lives, uid_life=uid_life)
     return cfg, models, events, extras
 
 

@@ -68,19 +68,36 @@ def device_to_host_ns(gtimer40, offset_ns, ref_host_ns):
     return gtimer40 + k * span - offset_ns
 
 
-def check_record_times(records, windows, offset_ns, tol_ns):
+def offset_at(clocks, host_ns):
+    """globaltimer - host offset at host time host_ns: linear interpolation between the
+    calibrations (dicts with 'at' = host time of the sample, 'offset'), extrapolated with
+    the nearest segment; one calibration = a constant offset (the clocks drift by ppm)."""
+    cs = sorted(clocks, key=lambda c: c["at"])
+    if len(cs) == 1:
+        return cs[0]["offset"]
+    i = 0
+    while i + 2 < len(cs) and host_ns > cs[i + 1]["at"]:
+        i += 1
+    a, b = cs[i], cs[i + 1]
+    return a["offset"] + (b["offset"] - a["offset"]) * (host_ns - a["at"]) / max(1, b["at"] - a["at"])
+
+
+def check_record_times(records, windows, clocks, tol_ns):
     """Every record of a launch, converted to host time, must fall inside the life of
     the job that issued it: [scheduled arrival - tol, completion seen by the dispatcher
     + tol].
 
     records: (gtimer40, type, uid, count, group[, smid]) as eventlog extras["records"];
-    windows: uid -> (t_sched, t_complete) in host CLOCK_MONOTONIC ns.  Returns the
-    violations (uid, ns after arrival, ns before completion)."""
+    windows: uid -> (t_sched, t_complete) in host CLOCK_MONOTONIC ns; clocks: the
+    calibrations (offset_at), or one offset.  Returns the violations (uid, ns after
+    arrival, ns before completion)."""
+    if not isinstance(clocks, (list, tuple)):
+        clocks = [{"at": 0, "offset": clocks}]
     bad = []
     for r in records:
         t40, uid = r[0], r[2]
         t_arr, t_done = windows[uid]
-        t = device_to_host_ns(t40, offset_ns, t_done)
+        t = device_to_host_ns(t40, round(offset_at(clocks, t_done)), t_done)
         if not t_arr - tol_ns <= t <= t_done + tol_ns:
             bad.append((uid, t - t_arr, t_done - t))
     return bad

@@ -421,6 +421,9 @@ class GPUModel:
     hw_queues: int = 32                            # H
     launch_delay: int = 0                          # delta_l, ns
     notif_delay: int = 0                           # delta_n, ns
+    decide_delay: int = 0                          # scheduler delay per decide pass, ns (Fig. 9):
+                                                   # the dispatcher is busy that long after each
+                                                   # pass; its issues launch after it
 
 
 @dataclass
@@ -525,15 +528,25 @@ def simulate(cfg: Config, models, trace, gpu: GPUModel, system="paella", naive_s
             if pol is not None:
                 push(t + gpu.notif_delay, "record", typ, k.uid, n)
 
+    busy = [0, False]       # dispatcher busy until busy[0]; a deferred pass is pending
+
     def dispatch(t):
+        if gpu.decide_delay:
+            if t < busy[0]:                 # still deciding: one more pass once it is free
+                if not busy[1]:
+                    busy[1] = True
+                    push(busy[0], "decide")
+                return
+            busy[0] = t + gpu.decide_delay
         for (uid, jid, layer, stream) in pol.decide():
             m = pol.jobs[jid].model
             L = models[m][layer]
             res.issues.append((t, uid, jid, layer, stream))
-            push(t + gpu.launch_delay, "launch",
+            push(t + gpu.decide_delay + gpu.launch_delay, "launch",
                  _Kernel(uid, jid, layer, L.grid, L.demand, L.dur, stream))
 
     kernels_left = {}
+    seen = False
     while evq:
         t, _, kind, a = heapq.heappop(evq)
         if horizon is not None and t > horizon:
@@ -581,8 +594,15 @@ def simulate(cfg: Config, models, trace, gpu: GPUModel, system="paella", naive_s
             done = pol.record(typ, uid, n)
             if done is not None:
                 res.finish[done] = t
-        # the dispatcher decides once every event of this instant is consumed
-        if pol is not None and (not evq or evq[0][0] > t):
+        elif kind == "decide":
+            busy[1] = False
+        # the dispatcher decides once every event of this instant is consumed -- after the
+        # events it observes (arrivals, records, its own deferred pass); launches and block
+        # starts/ends inside the GPU change nothing the policy can see
+        if kind in ("arrival", "record", "decide"):
+            seen = True
+        if pol is not None and seen and (not evq or evq[0][0] > t):
+            seen = False
             dispatch(t)
         if check:
             for i in range(S):

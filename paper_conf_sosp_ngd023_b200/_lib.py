@@ -36,7 +36,7 @@ SYMBOLS = ["paella_init", "paella_register_model", "paella_submit", "paella_subm
            "paella_kernel_info", "paella_kernel_name", "paella_stats", "paella_flush_log",
            "paella_run_isolated", "paella_debug_node", "paella_time_kernels", "paella_bench_empty",
            "paella_bench_roundtrip", "paella_loadgen", "paella_bench_wait", "paella_route_pair",
-           "paella_clock_info"]
+           "paella_clock_info", "paella_clock_sync"]
 
 
 class Config(C.Structure):
@@ -128,6 +128,7 @@ def load():
     lib.paella_stats.argtypes = [P, C.c_uint32, C.POINTER(Stats)]
     lib.paella_clock_info.argtypes = [P, C.c_uint32, C.POINTER(C.c_int64), C.POINTER(C.c_int64),
                                       C.POINTER(C.c_int64)]
+    lib.paella_clock_sync.argtypes = [P, C.c_uint32]
     lib.paella_flush_log.argtypes = [P]
     lib.paella_run_isolated.argtypes = [P, C.c_uint32, C.c_uint32, P, P, C.POINTER(C.c_int64)]
     lib.paella_debug_node.argtypes = [P, C.c_uint32, C.c_uint32, C.c_uint32, C.POINTER(C.c_float)]
@@ -404,6 +405,9 @@ class Engine:
         o, r, q = C.c_int64(), C.c_int64(), C.c_int64()
         _check(self.lib.paella_clock_info(self.h, gpu, C.byref(o), C.byref(r), C.byref(q)), "paella_clock_info")
         return o.value, r.value, q.value
+
+    def clock_sync(self, gpu=0):
+        _check(self.lib.paella_clock_sync(self.h, gpu), "paella_clock_sync")
 
     def flush_log(self):
         self.lib.paella_flush_log(self.h)

@@ -75,6 +75,11 @@ struct InstrArgs {
   uint32_t uid;       // unique launch id (kernel id of the paper)
   uint32_t group;     // G
   uint32_t flags;     // INSTR_*
+  // counter mode, a job's last kernel: per-slot ticket counter (device memory, never
+  // reset, running base tbase) that elects the block that exits last; only that block
+  // pays the system-scope fence and publishes the whole grid's exit count
+  uint32_t* ticket;
+  uint32_t tbase;
 };
 
 constexpr uint32_t NCTR = 4096;   // counter slots; > max in-flight launches (<= P)

@@ -41,7 +41,8 @@ namespace paella {
 // launch calls return (the timing gate) deadlocks.  Both are switched off then:
 // notifications take the direct ring path, timing runs ungated.
 static bool profiled() {
-  static const bool p = std::getenv("CUDA_INJECTION64_PATH") != nullptr || std::getenv("PAELLA_PROFILED") != nullptr;
+  static const bool p = std::getenv("CUDA_INJECTION64_PATH") != nullptr || std::getenv("NV_NSIGHT_INJECTION_TRANSPORT_TYPE") != nullptr ||
+                        std::getenv("NV_TPS_LAUNCH_TOKEN") != nullptr || std::getenv("PAELLA_PROFILED") != nullptr;
   return p;
 }
 static bool no_gate() { return profiled() || std::getenv("PAELLA_NO_GATE") != nullptr; }
@@ -278,6 +279,7 @@ struct CudaBackend : Backend {
   bool proxy = false;
   bool mirror = false;         // counter mode: kernels only count, k_notify_mirror copies
   uint32_t* ctr_m = nullptr;   // device: NCTR_M x {start, end}
+  uint32_t* ticket_m = nullptr;   // device: NCTR_M last-block tickets (a job's last kernel)
   uint32_t* mirror_h = nullptr;   // pinned, mapped host copy
   uint32_t* mirror_d = nullptr;
   bool pdl = true;             // programmatic dependent launches (off for the naive baseline)
@@ -298,6 +300,8 @@ struct CudaBackend : Backend {
     if (mirror) {
       if (cudaMalloc(&ctr_m, 2 * NCTR_M * sizeof(uint32_t)) != cudaSuccess) return -ENOMEM;
       cudaMemsetAsync(ctr_m, 0, 2 * NCTR_M * sizeof(uint32_t), s);
+      if (cudaMalloc(&ticket_m, NCTR_M * sizeof(uint32_t)) != cudaSuccess) return -ENOMEM;
+      cudaMemsetAsync(ticket_m, 0, NCTR_M * sizeof(uint32_t), s);
       if (cudaHostAlloc((void**)&mirror_h, 2 * NCTR_M * sizeof(uint32_t), cudaHostAllocMapped | cudaHostAllocPortable) !=
           cudaSuccess)
         return -ENOMEM;
@@ -390,6 +394,7 @@ struct CudaBackend : Backend {
     if (proxy_stream) cudaStreamDestroy(proxy_stream);
     if (dev_ring) cudaFree(dev_ring);
     if (ctr_m) cudaFree(ctr_m);
+    if (ticket_m) cudaFree(ticket_m);
     if (mirror_h) cudaFreeHost(mirror_h);
     if (proxy_ctl) cudaFreeHost(proxy_ctl);
     for (auto& s : streams) cudaStreamDestroy(s);
@@ -441,7 +446,7 @@ int make_weight_tmap(void* weights, uint32_t rows, uint32_t kpad, uint32_t box_r
 // helpers
 // ---------------------------------------------------------------------------
 static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last, bool instr) {
-  InstrArgs ia;
+  InstrArgs ia{};
   ia.ring = (Rec*)g->be->ring_dev();
   ia.tail = g->be->tail_dev();
   ia.mask = g->cap - 1;
@@ -457,6 +462,9 @@ static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last, bool
     ia.ctr = static_cast<CudaBackend*>(g->be.get())->ctr_m + 2 * slot;
     ia.base = g->ctr_mbase[slot];
     g->ctr_mbase[slot] += grid;
+    ia.ticket = static_cast<CudaBackend*>(g->be.get())->ticket_m + slot;
+    ia.tbase = g->ctr_tbase[slot];
+    if (last) g->ctr_tbase[slot] += grid;
     ia.flags |= INSTR_CTR;
     if (!last) ia.flags |= INSTR_RELAXED;   // the job's data dependency is carried by streams
     g->ctr_live.push_back(Gpu::CtrLive{uid, slot, ia.base, grid, 0, 0});
@@ -836,6 +844,19 @@ static void decide_and_launch(Gpu* g) {
 // Models posted by paella_register_model: added to this GPU's policy and logged by the
 // dispatcher thread itself, between two loop iterations.
 static void apply_inbox(Gpu* g) {
+  if (g->clk_req.load(std::memory_order_acquire) != g->clk_applied.load(std::memory_order_relaxed)) {
+    std::lock_guard<std::mutex> lk(g->inbox_mu);
+    if (g->clk_pending) {
+      g->clk_offset = g->clk_new[0];
+      g->clk_rtt = g->clk_new[1];
+      g->clk_res = g->clk_new[2];
+      g->clk_at = g->clk_new[3];
+      logev(g, EV_CLOCK, g->index | ((uint32_t)std::min<int64_t>(g->clk_res, 0xFFFFFF) << 8), (uint64_t)g->clk_offset,
+            (uint64_t)g->clk_rtt, (uint64_t)g->clk_at);
+      g->clk_pending = false;
+    }
+    g->clk_applied.store(g->clk_req.load(std::memory_order_acquire), std::memory_order_release);
+  }
   const uint32_t posted = g->inbox_n.load(std::memory_order_acquire);
   if (g->models_applied.load(std::memory_order_relaxed) == posted) return;
   std::vector<std::pair<uint32_t, std::vector<PolicyLayer>>> todo;
@@ -1043,7 +1064,7 @@ static void dispatcher_main(Gpu* g) {
 // offset = globaltimer - midpoint of the host send/receive times (CLOCK_MONOTONIC), so
 // device_ns ~= host_ns + offset within +- rtt/2; the probe also measures the timer's
 // resolution.  Not under a profiler (the probe waits for the host).
-static int clock_sync(Gpu* g, uint32_t n, int64_t* off, int64_t* rtt, int64_t* res) {
+static int clock_sync(Gpu* g, uint32_t n, int64_t* off, int64_t* rtt, int64_t* res, int64_t* at) {
   if (profiled()) return -ENOTSUP;
   if (cudaSetDevice(g->device) != cudaSuccess) return -EIO;
   void* buf = nullptr;
@@ -1072,6 +1093,7 @@ static int clock_sync(Gpu* g, uint32_t n, int64_t* off, int64_t* rtt, int64_t* r
     if (rc == 0 && t1 - t0 < best) {
       best = t1 - t0;
       boff = (int64_t)out[i] - (t0 + (t1 - t0) / 2);
+      *at = t0 + (t1 - t0) / 2;
     }
   }
   __atomic_store_n((uint32_t*)flag, n, __ATOMIC_SEQ_CST);   // release the probe in any case
@@ -1229,6 +1251,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
       if (cb->mirror) {
         g->ctr_mode = true;
         g->ctr_mbase.assign(NCTR_M, 0);
+        g->ctr_tbase.assign(NCTR_M, 0);
         for (uint32_t sl = NCTR_M; sl-- > 0;) g->ctr_free.push_back(sl);
       }
     }
@@ -1280,8 +1303,9 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
       for (int r = 0; r < NRES; ++r) logev(g.get(), EV_CAPACITY, (uint32_t)r, (uint64_t)pc.capacity[r], 0, 0);
     }
     if (cfg.device == PAELLA_DEVICE_CUDA &&
-        clock_sync(g.get(), 32, &g->clk_offset, &g->clk_rtt, &g->clk_res) == 0)
-      logev(g.get(), EV_CLOCK, gi, (uint64_t)g->clk_offset, (uint64_t)g->clk_rtt, (uint64_t)g->clk_res);
+        clock_sync(g.get(), 32, &g->clk_offset, &g->clk_rtt, &g->clk_res, &g->clk_at) == 0)
+      logev(g.get(), EV_CLOCK, gi | ((uint32_t)std::min<int64_t>(g->clk_res, 0xFFFFFF) << 8), (uint64_t)g->clk_offset,
+            (uint64_t)g->clk_rtt, (uint64_t)g->clk_at);
     P->gpus.push_back(std::move(g));
   }
   if (numa_pin) {
@@ -1656,6 +1680,31 @@ const char* paella_kernel_name(uint32_t kind) {
   return kind < KIND_COUNT ? names[kind] : "?";
 }
 
+int paella_clock_sync(paella_t* p, uint32_t gpu) {
+  Paella* P = (Paella*)p;
+  if (!P || gpu >= P->gpus.size()) return -EINVAL;
+  if (P->cfg.device != PAELLA_DEVICE_CUDA) return -ENODEV;
+  Gpu* g = P->gpus[gpu].get();
+  int64_t off, rtt, res, at;
+  int rc = clock_sync(g, 32, &off, &rtt, &res, &at);
+  if (rc) return rc;
+  {
+    std::lock_guard<std::mutex> lk(g->inbox_mu);   // applied by the dispatcher thread (log order)
+    g->clk_pending = true;
+    g->clk_new[0] = off;
+    g->clk_new[1] = rtt;
+    g->clk_new[2] = res;
+    g->clk_new[3] = at;
+  }
+  const uint64_t seen = g->clk_applied.load(std::memory_order_acquire);
+  g->clk_req.fetch_add(1, std::memory_order_release);
+  while (g->clk_applied.load(std::memory_order_acquire) == seen) {
+    if (g->stop.load(std::memory_order_acquire)) return -ESHUTDOWN;
+    std::this_thread::yield();
+  }
+  return 0;
+}
+
 int paella_clock_info(paella_t* p, uint32_t gpu, int64_t* offset_ns, int64_t* rtt_ns, int64_t* resolution_ns) {
   Paella* P = (Paella*)p;
   if (!P || gpu >= P->gpus.size()) return -EINVAL;
@@ -1691,13 +1740,17 @@ static int ensure_iso(Gpu* g) {
     return -ENOMEM;
   std::memset(g->prof_ring_h, 0, cap * sizeof(Rec));
   cudaHostGetDevicePointer(&g->prof_ring_d, g->prof_ring_h, 0);
-  if (cudaMalloc(&g->prof_tail, 256) || cudaMalloc(&g->prof_ctr, 2 * NCTR * sizeof(uint32_t))) return -ENOMEM;
+  if (cudaMalloc(&g->prof_tail, 256) || cudaMalloc(&g->prof_ctr, 2 * NCTR * sizeof(uint32_t)) ||
+      cudaMalloc(&g->prof_ticket, NCTR * sizeof(uint32_t)))
+    return -ENOMEM;
   g->prof_base.assign(NCTR, 0);
+  g->prof_tbase.assign(NCTR, 0);
   cudaStream_t s;
   cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
   g->prof_stream = s;
   cudaMemsetAsync(g->prof_tail, 0, 256, s);
   cudaMemsetAsync(g->prof_ctr, 0, 2 * NCTR * sizeof(uint32_t), s);
+  cudaMemsetAsync(g->prof_ticket, 0, NCTR * sizeof(uint32_t), s);
   // isolated runs write their records to device memory (as served kernels do through
   // the proxy); nobody consumes them except the round-trip benchmark's direct ring
   if (cudaMalloc(&g->prof_devring, cap * sizeof(Rec))) return -ENOMEM;
@@ -1716,23 +1769,11 @@ static Rec* iso_ring(Gpu* g) {
 }
 
 // launch kernel `l` of model m from the isolated slot on the profiling stream
+static InstrArgs iso_instr(Gpu* g, uint32_t grid, uint32_t group, bool last);
+
 static void iso_launch(Gpu* g, Model* m, uint32_t l, bool instr) {
   const KernelInst& k = m->kernels[l];
-  InstrArgs ia;
-  ia.ring = iso_ring(g);
-  ia.tail = g->prof_tail;
-  uint32_t uid = g->prof_uid++;
-  uint32_t slot = uid % NCTR;
-  ia.ctr = g->prof_ctr + 2 * slot;
-  ia.mask = (1u << 16) - 1;
-  ia.log2cap = 16;
-  ia.base = g->prof_base[slot];
-  g->prof_base[slot] += k.grid_total();
-  ia.uid = uid;
-  ia.group = g->P->cfg.group_size;
-  ia.flags = INSTR_ON | (l + 1 == m->kernels.size() ? INSTR_LAST : 0);
-  if (static_cast<CudaBackend*>(g->be.get())->mirror)   // as in serving
-    ia.flags |= INSTR_CTR | (l + 1 == m->kernels.size() ? 0u : INSTR_RELAXED);
+  InstrArgs ia = iso_instr(g, k.grid_total(), g->P->cfg.group_size, l + 1 == m->kernels.size());
   uint32_t iso_slot = (uint32_t)m->gpu[g->index].args.size() - 1;
   auto* cb = static_cast<CudaBackend*>(g->be.get());
   const void* tm = is_tc(k.kind) ? m->gpu[g->index].tmaps[l].b : nullptr;
@@ -2115,7 +2156,7 @@ static void launch_gate(Gpu* g, const volatile uint32_t* gd) {
 }
 
 static InstrArgs iso_instr(Gpu* g, uint32_t grid, uint32_t group, bool last) {
-  InstrArgs ia;
+  InstrArgs ia{};
   ia.ring = iso_ring(g);
   ia.tail = g->prof_tail;
   uint32_t uid = g->prof_uid++;
@@ -2128,6 +2169,9 @@ static InstrArgs iso_instr(Gpu* g, uint32_t grid, uint32_t group, bool last) {
   ia.uid = uid;
   ia.group = group;
   ia.flags = INSTR_ON | (last ? INSTR_LAST : 0);
+  ia.ticket = g->prof_ticket + slot;
+  ia.tbase = g->prof_tbase[slot];
+  if (last) g->prof_tbase[slot] += grid;
   if (static_cast<CudaBackend*>(g->be.get())->mirror)   // as in serving
     ia.flags |= INSTR_CTR | (last ? 0u : INSTR_RELAXED);
   return ia;
@@ -2228,6 +2272,7 @@ int paella_bench_roundtrip(paella_t* p, uint32_t gpu, uint32_t n, int64_t* place
   for (uint32_t i = 0; i < n; ++i) {
     InstrArgs ia = iso_instr(g, 1, 1, false);
     ia.ring = (Rec*)g->prof_ring_d;   // direct write to the pinned host ring
+    ia.flags &= ~(INSTR_CTR | INSTR_RELAXED);   // records, also when serving uses counter mode
     void* args[2] = {(void*)&la, (void*)&ia};
     int64_t t0 = now_ns();
     cudaLaunchKernel((const void*)f, dim3(1), dim3(32), args, 0, s);

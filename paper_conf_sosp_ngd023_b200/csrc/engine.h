@@ -178,6 +178,7 @@ struct Gpu {
   std::vector<CtrLive> ctr_live;
   std::vector<uint32_t> ctr_free;           // free counter-mode slots
   std::vector<uint32_t> ctr_mbase;          // running base per counter-mode slot
+  std::vector<uint32_t> ctr_tbase;          // running base of each slot's last-block ticket
   std::vector<JobRec> jobs;         // indexed by job id (dense)
   std::vector<uint32_t> free_job_ids;
   uint32_t next_job = 0;
@@ -202,7 +203,10 @@ struct Gpu {
   std::atomic<uint32_t> models_applied{0};   // models the dispatcher has added to its policy
   uint32_t rr_start = 0;
   // globaltimer -> host clock (C3): device_ns ~= host_ns + clk_offset; rtt < 0 = not calibrated
-  int64_t clk_offset = 0, clk_rtt = -1, clk_res = 0;
+  int64_t clk_offset = 0, clk_rtt = -1, clk_res = 0, clk_at = 0;   // clk_at: host time of the sample
+  bool clk_pending = false;           // paella_clock_sync -> the dispatcher logs it (inbox_mu)
+  int64_t clk_new[4] = {0, 0, 0, 0};
+  std::atomic<uint64_t> clk_req{0}, clk_applied{0};
   FILE* log = nullptr;
   std::mutex log_mu;
   paella_stats_t stats{};
@@ -214,7 +218,8 @@ struct Gpu {
   Rec* prof_devring = nullptr;     // device-memory ring of isolated runs
   void* trace_buf = nullptr;       // debug phase timestamps
   uint32_t* prof_ctr = nullptr;
-  std::vector<uint32_t> prof_base;
+  uint32_t* prof_ticket = nullptr;
+  std::vector<uint32_t> prof_base, prof_tbase;
   uint32_t prof_uid = 0;
   void* prof_stream = nullptr;
   void* stage_in = nullptr;    // pinned mapped staging for isolated-run io

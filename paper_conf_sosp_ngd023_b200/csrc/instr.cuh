@@ -90,6 +90,24 @@ __device__ __forceinline__ void kernel_begin(const InstrArgs& ia) {
   pdl_trigger();
 }
 
+// Counter mode, a job's LAST kernel (its output is the logits in client host memory):
+// the system-scope flush is paid once per kernel, not once per block.  Every block
+// releases its outputs at gpu scope with an acq_rel ticket atomic; the block that draws
+// the last ticket has acquired all of them, issues one fence.sc.sys (cumulative: the
+// other blocks' host-memory writes are ordered before what follows at system scope) and
+// only then publishes the exit count of the WHOLE grid with a release reduction.  The
+// host therefore never sees the launch complete before every logit is visible.  The
+// caller is one thread of a block whose other threads are past a CTA barrier.
+__device__ __forceinline__ void last_kernel_exit(const InstrArgs& ia) {
+  const uint32_t total = gridDim.x * gridDim.y * gridDim.z;
+  uint32_t old;
+  asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(ia.ticket) : "memory");
+  if (old + 1u - ia.tbase == total) {
+    asm volatile("fence.sc.sys;" ::: "memory");
+    asm volatile("red.release.sys.global.add.u32 [%0], %1;" ::"l"(&ia.ctr[1]), "r"(total) : "memory");
+  }
+}
+
 // exit count of a block whose every other thread is already past a CTA barrier (the
 // caller is the block's last active thread): no second barrier
 template <bool INSTR>
@@ -97,7 +115,7 @@ __device__ __forceinline__ void instr_exit_last_thread(const InstrArgs& ia) {
   if constexpr (INSTR) {
     if (ia.flags & INSTR_CTR) {
       if (ia.flags & INSTR_LAST)
-        asm volatile("red.release.sys.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+        last_kernel_exit(ia);
       else if (ia.flags & INSTR_RELAXED)
         asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
       else
@@ -117,13 +135,23 @@ __device__ __forceinline__ void instr_exit_last_thread(const InstrArgs& ia) {
 template <bool INSTR, uint32_t T = 0>
 __device__ __forceinline__ void instr_exit(const InstrArgs& ia) {
   if constexpr (INSTR) {
+    if ((ia.flags & (INSTR_CTR | INSTR_RELAXED)) == (INSTR_CTR | INSTR_RELAXED)) {
+      // relaxed exit count (B200-Q4): it orders nothing (the job's data
+      // dependencies ride on stream order), so no block barrier either -- the
+      // bookkeeping thread counts the block when it gets here; the dispatcher may see
+      // the block finished a few hundred ns before its last warp retires, which only
+      // shifts the occupancy estimate
+      if (threadIdx.x == T && threadIdx.y == 0 && threadIdx.z == 0)
+        asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+      return;
+    }
     __syncthreads();
     if (threadIdx.x == T && threadIdx.y == 0 && threadIdx.z == 0 && (ia.flags & INSTR_CTR)) {
       // counter mode: a release reduction (the block's outputs, ordered before it by the
       // barrier, are visible before the count is); nothing is waited for, the block
-      // retires at once.  System scope for a job's last kernel (output in host memory).
+      // retires at once.  A job's last kernel: one system-scope flush per grid.
       if (ia.flags & INSTR_LAST)
-        asm volatile("red.release.sys.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+        last_kernel_exit(ia);
       else if (ia.flags & INSTR_RELAXED)   // data dependencies ride on stream order
         asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
       else

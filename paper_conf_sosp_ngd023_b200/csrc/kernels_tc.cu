@@ -498,6 +498,14 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   // every input of this block has been consumed: let the dependent kernel be placed
   // (its prologue overlaps this epilogue); warp 5 follows the accumulator too
   if (warp == 5 && nkl > 0) mbar_wait(accb, 0);
+  constexpr uint32_t RELAXED_CTR = INSTR_CTR | INSTR_RELAXED;
+  if constexpr (INSTR) {
+    // relaxed exit count (B200-Q7): it orders nothing, so the bookkeeping warp
+    // counts the block as soon as its MMAs are complete -- the count travels while the
+    // epilogue runs instead of trailing the block's last store
+    if (warp == 5 && lane == 0 && (ia.flags & RELAXED_CTR) == RELAXED_CTR)
+      asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+  }
   pdl_trigger();
   if (warp < 4) {
     const uint32_t row = warp * 32 + lane;
@@ -648,7 +656,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     // every other thread is past the barrier above: the MMA warp, last to finish, counts
     // the block's exit itself (no second block barrier)
     if (trace && lane == 0) tr[6] = globaltimer();
-    if (lane == 0) instr_exit_last_thread<INSTR>(ia);
+    if (lane == 0 && (ia.flags & RELAXED_CTR) != RELAXED_CTR) instr_exit_last_thread<INSTR>(ia);
     if (trace && lane == 0) tr[7] = globaltimer();
   }
 }

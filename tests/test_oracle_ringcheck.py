@@ -57,3 +57,13 @@ def test_record_time_windows():
     assert rc.check_record_times(recs, {5: (2000, 3000)}, off, 0) == []
     assert rc.check_record_times(recs, {5: (2600, 3000)}, off, 0) != []       # before arrival
     assert rc.check_record_times(recs, {5: (2000, 2800)}, off, 50) != []      # after completion
+
+
+def test_offset_interpolation():
+    cl = [{"at": 1000, "offset": 100}, {"at": 3000, "offset": 300}]
+    assert rc.offset_at(cl, 2000) == 200
+    assert rc.offset_at(cl, 5000) == 500          # extrapolated on the last segment
+    assert rc.offset_at(cl[:1], 9999) == 100
+    off = lambda h: rc.offset_at(cl, h)   # noqa: E731
+    recs = [(int(2500 + off(2500)), 1, 5, 16, 0)]
+    assert rc.check_record_times(recs, {5: (2400, 2600)}, cl, 0) == []

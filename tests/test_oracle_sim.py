@@ -662,3 +662,36 @@ def test_exactly_once_checker_rejects_bad_logs():
     other_uid = good[:5] + [(0, sim.COMPLETION, 8, 8, 2)]
     for bad in (dropped, dup, wrong_count, wrong_group, other_uid):
         assert sim.check_exactly_once(bad, {7: 40}, 16) != []
+
+
+# --- Fig. 9: scheduler-delay injection in the simulator (NEXT-2) ---------------------
+
+def test_decide_delay_closed_form():
+    """One job of 3 kernels (d = 10), launch delay 2, notification delay 3, decide delay 5
+    (units of 1 us), no launch-ahead: each decision takes 5 before its launch is sent,
+    so decisions happen at 0, 20, 40 (= k (5 + 2 + 10 + 3)) and the job completes at 60."""
+    u = 1000
+    gpu = GPUModel(sms=1, per_sm=(1, 64, 65536, 233472, 512), launch_delay=2 * u, notif_delay=3 * u,
+                   decide_delay=5 * u)
+    cfg = Config(num_clients=1, theta=sim.INF_THETA, slack=10**6, capacity=(10**6, 10**9, 10**12, 10**12, 10**9))
+    res = sim.simulate(cfg, _chain(3, 10 * u), [(0, 0, 0)], gpu)
+    assert [t for (t, *_r) in sorted(res.issues, key=lambda x: x[3])] == [0, 20 * u, 40 * u]
+    assert res.jct()[0] == 60 * u
+
+
+def test_decide_delay_throughput_falls():
+    """Fig. 9 (P1178-1241): a saturated stream of jobs is served at a rate that does not
+    rise as the per-decision delay grows, and falls once the delay is comparable to a
+    kernel (the dispatcher, not the GPU, becomes the bottleneck)."""
+    models = [[Layer(4, (1, 4, 4096, 1024, 0), 2000, 2000)] * 6]
+    trace = [(i * 500, 0, 0) for i in range(120)]
+    cfg = Config(num_clients=1, slack=64, lookahead=0, streams=32,
+                 capacity=tuple(8 * x for x in (32, 64, 65536, 233472, 512)))
+    rates = []
+    for dd in (0, 100, 1000, 10000):
+        gpu = GPUModel(sms=8, launch_delay=500, notif_delay=500, decide_delay=dd)
+        res = sim.simulate(cfg, models, trace, gpu, check=False)
+        assert len(res.finish) == 120
+        rates.append(120 / max(res.finish.values()))
+    assert all(a >= b for a, b in zip(rates, rates[1:])), rates
+    assert rates[-1] < 0.5 * rates[0], rates
