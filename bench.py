@@ -85,6 +85,9 @@ def parse():
     ap.add_argument("--decide-delay-ns", type=int, default=0,
                     help="injected scheduler delay before every decide pass (Fig. 9 sensitivity)")
     ap.add_argument("--prio-classes", type=int, default=1, help="stream-priority classes (DESIGN.md B200-Q2)")
+    ap.add_argument("--branches", type=int, default=0,
+                    help="1 = NEXT-4 intra-job branch concurrency in the paella arms (kernel DAG over virtual "
+                         "streams)")
     ap.add_argument("--dispatcher-cpu", type=int, default=-2,
                     help="first dispatcher core (-1 = unpinned; default: NUMA-local cores of each GPU, "
                          "else 2, 3, ...)")
@@ -399,7 +402,7 @@ def run_gpu(args, ngpus, cores, fake):
     paella_kw = dict(policy=pol[args.policy], theta=args.theta, decide_delay_ns=args.decide_delay_ns,
                      online_tbar=args.online_tbar, slack=args.slack, prio_classes=args.prio_classes,
                      lookahead=args.lookahead, max_active=args.max_active, instrument=True,
-                     route=L.ROUTE_LEAST_WORK)
+                     route=L.ROUTE_LEAST_WORK, branches=bool(args.branches))
     arms_kw = {
         "paella": paella_kw,
         "paella_fifo": dict(paella_kw, policy=L.POLICY_FIFO),
@@ -754,8 +757,8 @@ def main():
         "config": {"workload": WORKLOADS[args.config], "batch": 1, "rho": args.rho, "lambda_req_s": round(lam, 1),
                    "requests_per_step": args.reqs * ngpus,
                    "parallelism": f"{ngpus} GPU dispatchers, least-work router" if ngpus > 1 else "1 GPU dispatcher",
-                   "paella": f"srpt+deficit th{args.theta} K{args.max_active} la{args.lookahead} B{args.slack} pdl"
-                   if args.policy == "srpt" else args.policy,
+                   "paella": (f"srpt+deficit th{args.theta}" if args.policy == "srpt" else args.policy)
+                   + f" K{args.max_active} la{args.lookahead} B{args.slack} pdl" + (" branches" if args.branches else ""),
                    "l2": "not flushed: weights (~120 MB bf16) largely L2-resident as in serving; inputs stream "
                          "from pinned host memory every request"},
         "roofline": roofline_entry(dict(P, config=args.config), peaks) if "kinfo" in P else None,

@@ -168,6 +168,11 @@ typedef struct {
   uint32_t fake_fault;            /* FAKE device fault injection (tests): PAELLA_FAULT_*, on GPU 0
                                     of the instance only */
   uint32_t fake_fault_arg;        /* ... the ordinal of the record / launch it applies to */
+  uint32_t branches;              /* NEXT-4 intra-job concurrency (Fig. 7 waitlists, P906-951): 1 =
+                                    a job's kernels form a DAG over up to 4 virtual streams
+                                    (Inception / SqueezeNet / ResNet branches run concurrently on
+                                    several CUDA streams; a kernel is issued once its cross-
+                                    stream inputs have completed); 0 (default) = one chain per job */
   const char* route_log_path;     /* multi-GPU routing log (printf pattern, "%u" = client id), or
                                     NULL: every routing decision of that client with the W_g
                                     snapshot of ALL GPUs it was taken on (paella_route_rec_t
@@ -319,6 +324,9 @@ typedef struct {
   uint32_t kind;               /* kernel kind id (paella_kernel_name) */
   int64_t  tbar_ns;            /* frozen profile */
   uint64_t flops, bytes;       /* algorithmic work per launch */
+  uint32_t vs;                 /* virtual stream in the job's kernel DAG (NEXT-4) */
+  uint32_t n_deps;             /* kernels whose outputs it reads (through concats / fused GAPs) */
+  uint32_t deps[8];            /* the first 8 of them */
 } paella_kernel_info_t;
 
 int paella_kernel_info(paella_t* p, uint32_t model_id, uint32_t k, paella_kernel_info_t* info);

@@ -11,6 +11,8 @@ Format (DESIGN.md §"Event log"): a sequence of 32-byte little-endian records
   110 MODEL     a=model, b=#kernels
   111 LAYER     a=model, b=layer, c=grid, d=T-bar ns
   112 DEMAND    a=model, b=layer, c=(warps << 32) | regs, d=(smem << 32) | tmem
+  114 VS        a=model, b=layer, c=virtual stream            (NEXT-4 branches only)
+  113 DEP       a=model, b=layer, c=a kernel of ANOTHER virtual stream it consumes
     1 ARRIVAL   a=client, b=job, c=model, d=t_sched ns
     2 RECORD    a=type, b=uid, c=count, d=globaltimer:40 | group:16 | smid:8
     3 BATCH_END
@@ -45,6 +47,7 @@ def read(path):
     completes = []
     routes = []
     clocks = []
+    vss, xdeps = {}, {}   # NEXT-4 DAG: virtual stream and cross-stream dependencies per layer
     narrivals = 0
     lives = []          # one entry per admitted job occurrence (job ids are recycled)
     cur_life = {}       # job id -> index into lives of its current occurrence
@@ -75,6 +78,10 @@ def read(path):
             layers[(a, b)] = (c, d)
         elif t == 112:
             demands[(a, b)] = (c >> 32, c & 0xFFFFFFFF, d >> 32, d & 0xFFFFFFFF)
+        elif t == 114:
+            vss[(a, b)] = c
+        elif t == 113:
+            xdeps.setdefault((a, b), []).append(c)
         elif t == 1:
             events.append((sim.EV_ARRIVAL, b, a, c))
             arrivals[b] = (a, c, d)        # latest job with this id (ids are recycled)
@@ -112,7 +119,11 @@ def read(path):
         for l in range(nlayers[m]):
             grid, tbar = layers[(m, l)]
             w, rg, sm, tm = demands[(m, l)]
-            ms.append(sim.Layer(grid, (1, w, rg, sm, tm), tbar))
+            if (m, l) in vss:
+                ms.append(sim.Layer(grid, (1, w, rg, sm, tm), tbar, deps=tuple(xdeps.get((m, l), ())),
+                                    vs=vss[(m, l)]))
+            else:
+                ms.append(sim.Layer(grid, (1, w, rg, sm, tm), tbar))
         models.append(ms)
     extras = dict(records=records, issues=issues, completes=completes, arrivals=arrivals,
                   n_arrivals=narrivals, routes=routes, clocks=clocks, lives=lives, uid_life=uid_life)

@@ -41,6 +41,27 @@ class Layer:
     demand: tuple          # per-block demand, one int per RESOURCES entry (blocks=1)
     tbar: int              # profiled mean kernel time, ns (frozen)
     dur: int = 0           # synthetic-mode block duration, ns
+    # NEXT-4 intra-job concurrency (Fig. 7 waitlists, P918-951): the kernels this one
+    # consumes (None = the previous kernel: a chain) and its virtual stream
+    deps: tuple | None = None
+    vs: int = 0
+
+
+class Topo:
+    """A model's kernel DAG as the dispatcher sees it (Fig. 7 waitlists, P906-951):
+    per kernel its dependencies and virtual stream; per virtual stream its kernels in
+    order.  A kernel is *active* (CUDA stream semantics, P943-947) when it is the next
+    kernel of its virtual stream and every kernel it depends on in ANOTHER virtual stream
+    has completed; its predecessors in its own virtual stream are ordered by the stream."""
+
+    def __init__(self, layers):
+        n = len(layers)
+        self.deps = [tuple(range(k - 1, k)) if L.deps is None else tuple(L.deps) for k, L in enumerate(layers)]
+        self.vs = [L.vs for L in layers]
+        nv = 1 + max(self.vs, default=0)
+        self.vs_kernels = [[k for k in range(n) if self.vs[k] == v] for v in range(nv)]
+        self.pos = [self.vs_kernels[self.vs[k]].index(k) for k in range(n)]
+        self.cross = [tuple(d for d in self.deps[k] if self.vs[d] != self.vs[k]) for k in range(n)]
 
 
 @dataclass
@@ -81,13 +102,18 @@ class Job:
     model: int
     seq: int
     R: int
-    cursor: int = 0          # next kernel to issue (= kernels dispatched, c_i of P1265)
+    cursor: int = 0          # kernels dispatched (c_i of P1265)
     done: int = 0            # kernels completed
-    stream: int = -1         # stream held while kernels are in flight
-    last_stream: int = -1
     last_uid: int = -1
-    uids: dict = field(default_factory=dict)   # layer -> launch uid (while in flight)
     rr: int = -1             # RR ablation: uid of the job's last issued kernel (-1 = never)
+    # per kernel: 0 = waiting, 1 = in flight, 2 = completed
+    state: list = field(default_factory=list)
+    # per virtual stream: next kernel (position), in-flight uids (issue order), the CUDA
+    # stream held while it has kernels in flight, the last stream it held
+    vs_next: list = field(default_factory=list)
+    vs_uids: list = field(default_factory=list)
+    vs_stream: list = field(default_factory=list)
+    vs_last: list = field(default_factory=list)
 
     @property
     def inflight(self):
@@ -142,6 +168,7 @@ class Policy:
         # the stream-priority class boundaries at its MODEL event; replay feeds them in
         # log order, a fresh Policy knows every model)
         self.registered = set(range(len(models)))
+        self.topo = [Topo(m) for m in models]
 
     # effective deficit, units of 1/N
     def D(self, c):
@@ -169,7 +196,7 @@ class Policy:
         self.tb[m][lay] = new
         if delta:
             for j in self.jobs.values():
-                if j.model == m and j.cursor <= lay:
+                if j.model == m and j.state[lay] == 0:      # not dispatched yet
                     j.R += delta
 
     # --- events -------------------------------------------------------------
@@ -180,6 +207,10 @@ class Policy:
         if self.log is not None:
             self.log.append((EV_ARRIVAL, job_id, client, model))
         j = Job(job_id, client, model, self.next_seq, self.remaining(model, 0))
+        nv = len(self.topo[model].vs_kernels)
+        j.state = [0] * len(self.models[model])
+        j.vs_next, j.vs_uids = [0] * nv, [[] for _ in range(nv)]
+        j.vs_stream, j.vs_last = [-1] * nv, [-1] * nv
         self.next_seq += 1
         self.jobs[job_id] = j
         return j
@@ -207,10 +238,13 @@ class Policy:
             self._refine(L)
             j = self.jobs[L.job]
             j.done += 1
-            if j.inflight == 0:
+            j.state[L.layer] = 2
+            v = self.topo[j.model].vs[L.layer]
+            j.vs_uids[v].remove(uid)
+            if not j.vs_uids[v]:              # the virtual stream drained: its stream is free
                 self.free.add(L.stream)
-                j.stream = -1
-                j.last_stream = L.stream
+                j.vs_stream[v] = -1
+                j.vs_last[v] = L.stream
             if j.done == len(self.models[j.model]):
                 if self.checks:
                     assert j.R == 0
@@ -222,15 +256,32 @@ class Policy:
                 done = j.id
         return done
 
+    def head(self, j):
+        """The job's lowest-index active kernel that may be dispatched now, or None:
+        the next kernel of a virtual stream whose cross-stream dependencies have all
+        completed, and whose stream is idle -- or, with launch-ahead D > 0, whose oldest
+        in-flight kernel is fully placed (running) with at most D in flight."""
+        T = self.topo[j.model]
+        best = None
+        for v, ks in enumerate(T.vs_kernels):
+            if j.vs_next[v] >= len(ks):
+                continue
+            k = ks[j.vs_next[v]]
+            if any(j.state[d] != 2 for d in T.cross[k]):
+                continue
+            infl = len(j.vs_uids[v])
+            if infl > 0:
+                if self.cfg.lookahead <= 0 or infl > self.cfg.lookahead:
+                    continue
+                L = self.launches[j.vs_uids[v][0]]          # the oldest kernel in flight
+                if max(L.p, L.f) < L.grid:
+                    continue
+            if best is None or k < best:
+                best = k
+        return best
+
     def is_ready(self, j):
-        if j.cursor >= len(self.models[j.model]):
-            return False
-        if j.inflight == 0:
-            return True
-        if self.cfg.lookahead <= 0 or j.inflight > self.cfg.lookahead:
-            return False
-        L = self.launches.get(j.uids.get(j.done))     # the oldest kernel still in flight
-        return L is not None and max(L.p, L.f) >= L.grid
+        return self.head(j) is not None
 
     def ready(self):
         return [j for j in self.jobs.values() if self.is_ready(j)]
@@ -305,32 +356,37 @@ class Policy:
             j = self.pick(rdy)
             if j is None:
                 break
-            if j.inflight == 0 and not self.free:
+            k = self.head(j)
+            v = self.topo[j.model].vs[k]
+            if not j.vs_uids[v] and not self.free:
                 break
-            layer = self.models[j.model][j.cursor]
+            layer = self.models[j.model][k]
             if not self.predicate(layer.grid):
                 break
             uid = self.next_uid
             self.next_uid += 1
-            if j.inflight > 0:
-                stream = j.stream            # launch-ahead: behind its predecessor
+            if j.vs_uids[v]:
+                stream = j.vs_stream[v]      # launch-ahead: behind its predecessor
             else:
                 c = self.job_class(j)
-                if j.last_stream in self.free and self.stream_class(j.last_stream) == c:
-                    stream = j.last_stream
+                last = j.vs_last[v]
+                if last in self.free and self.stream_class(last) == c:
+                    stream = last
                 else:
                     cand = [s for s in self.free if self.stream_class(s) == c]
                     stream = min(cand) if cand else min(self.free)
                 self.free.remove(stream)
-                j.stream = stream
-            self.launches[uid] = Launch(uid, j.id, j.cursor, layer.grid, layer.demand, stream)
+                j.vs_stream[v] = stream
+            self.launches[uid] = Launch(uid, j.id, k, layer.grid, layer.demand, stream)
             for r in range(len(RESOURCES)):
                 self.U[r] += layer.grid * layer.demand[r]
             self.Q += layer.grid
             self.O += 2 * groups(layer.grid, cfg.group)
-            j.R -= self.tb[j.model][j.cursor]
-            rec = (uid, j.id, j.cursor, stream)
-            j.uids[j.cursor] = uid
+            j.R -= self.tb[j.model][k]
+            rec = (uid, j.id, k, stream)
+            j.state[k] = 1
+            j.vs_uids[v].append(uid)
+            j.vs_next[v] += 1
             j.cursor += 1
             j.last_uid = uid
             j.rr = uid
@@ -697,30 +753,35 @@ def route_least_work(work, pending, tbar_model, alive):
 
 def check_inflight_bound(events, models, lookahead):
     """NEXT-1 invariant on a consumed-event log: a job never has more than lookahead + 1
-    kernels issued whose final COMPLETION has not been consumed (launch-ahead depth D),
-    and its kernels are issued in layer order.  Returns the violations."""
+    kernels of one virtual stream issued whose final COMPLETION has not been consumed
+    (launch-ahead depth D), and each virtual stream issues its kernels in order (a chain
+    job has one virtual stream: layer order).  Returns the violations."""
+    topo = [Topo(m) for m in models]
     model_of, grid_of, done_of, infl, nxt = {}, {}, {}, {}, {}
     bad = []
     for ev in events:
         k = ev[0]
         if k == EV_ARRIVAL:
             model_of[ev[1]] = ev[3]
-            infl[ev[1]] = 0
-            nxt[ev[1]] = 0
+            nv = len(topo[ev[3]].vs_kernels)
+            infl[ev[1]] = [0] * nv
+            nxt[ev[1]] = [0] * nv
         elif k == EV_ISSUE:
             uid, job, layer = ev[1], ev[2], ev[3]
-            if layer != nxt[job]:
+            T = topo[model_of[job]]
+            v = T.vs[layer]
+            if T.vs_kernels[v][nxt[job][v]] != layer:
                 bad.append(("order", uid, job, layer))
-            nxt[job] = layer + 1
-            grid_of[uid] = (job, models[model_of[job]][layer].grid)
+            nxt[job][v] += 1
+            grid_of[uid] = (job, v, models[model_of[job]][layer].grid)
             done_of[uid] = 0
-            infl[job] += 1
-            if infl[job] > lookahead + 1:
-                bad.append(("depth", uid, job, infl[job]))
+            infl[job][v] += 1
+            if infl[job][v] > lookahead + 1:
+                bad.append(("depth", uid, job, infl[job][v]))
         elif k == EV_RECORD and ev[1] == COMPLETION and ev[2] in grid_of:
             uid = ev[2]
             done_of[uid] += ev[3]
-            job, g = grid_of[uid]
+            job, v, g = grid_of[uid]
             if done_of[uid] == g:
-                infl[job] -= 1
+                infl[job][v] -= 1
     return bad

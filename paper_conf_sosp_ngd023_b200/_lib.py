@@ -52,7 +52,8 @@ class Config(C.Structure):
                 ("no_proxy", C.c_uint32), ("no_pdl", C.c_uint32),
                 ("notify_mode", C.c_uint32), ("prio_classes", C.c_uint32), ("online_tbar", C.c_uint32),
                 ("decide_delay_ns", C.c_uint32), ("naive_pdl", C.c_uint32), ("watchdog_ms", C.c_uint32),
-                ("fake_fault", C.c_uint32), ("fake_fault_arg", C.c_uint32), ("route_log_path", C.c_char_p),
+                ("fake_fault", C.c_uint32), ("fake_fault_arg", C.c_uint32), ("branches", C.c_uint32),
+                ("route_log_path", C.c_char_p),
                 ("max_active_jobs", C.c_uint32)]
 
 
@@ -79,7 +80,8 @@ class ModelInfo(C.Structure):
 class KernelInfo(C.Structure):
     _fields_ = [("grid", C.c_uint32), ("block", C.c_uint32), ("smem", C.c_uint32), ("regs", C.c_uint32),
                 ("tmem_cols", C.c_uint32), ("kind", C.c_uint32), ("tbar_ns", C.c_int64),
-                ("flops", C.c_uint64), ("bytes", C.c_uint64)]
+                ("flops", C.c_uint64), ("bytes", C.c_uint64), ("vs", C.c_uint32), ("n_deps", C.c_uint32),
+                ("deps", C.c_uint32 * 8)]
 
 
 class Req(C.Structure):
@@ -173,7 +175,7 @@ class Engine:
                  event_log=None, fake_sms=0, fake_time_scale_ns=0, event_time_kind=None, lookahead=0,
                  launch_threads=0, proxy=True, pdl=True, prio_classes=1,
                  notify="counters", decide_delay_ns=0, online_tbar=False, naive_pdl=False, watchdog_ms=0,
-                 fake_fault=0, fake_fault_arg=0, route_log=None, max_active=0):
+                 fake_fault=0, fake_fault_arg=0, route_log=None, max_active=0, branches=False):
         self.lib = load()
         cfg = Config()
         cfg.abi_version = ABI_VERSION
@@ -216,6 +218,7 @@ class Engine:
         self._rlog = route_log.encode() if route_log else None
         cfg.route_log_path = self._rlog
         cfg.max_active_jobs = max_active
+        cfg.branches = 1 if branches else 0
         # notification path: "counters" (default), "ring" (device ring + forwarding warp),
         # "direct" (the paper's direct ring writes; same as proxy=False)
         if notify not in ("counters", "ring", "direct"):
@@ -291,6 +294,7 @@ class Engine:
         info = KernelInfo()
         _check(self.lib.paella_kernel_info(self.h, mid, k, C.byref(info)), "paella_kernel_info")
         d = {f: getattr(info, f) for f, _ in KernelInfo._fields_}
+        d["deps"] = list(info.deps)[:min(8, info.n_deps)]
         d["name"] = self.lib.paella_kernel_name(info.kind).decode()
         return d
 

@@ -63,7 +63,7 @@ PAELLA_HD inline RecFields rec_decode(uint64_t w0, uint64_t w1) {
 // end} counters with fire-and-forget reductions and writes no record; the mirror warp
 // (k_notify_mirror) copies the counters to pinned host memory and the dispatcher turns
 // counter progress into the same group-of-G records (engine.cpp::drain_counters)
-enum : uint32_t { INSTR_ON = 1u, INSTR_LAST = 2u, INSTR_CTR = 4u, INSTR_RELAXED = 8u };
+enum : uint32_t { INSTR_ON = 1u, INSTR_LAST = 2u, INSTR_CTR = 4u, INSTR_RELAXED = 8u, INSTR_SYSREL = 16u };
 
 struct InstrArgs {
   Rec* ring;          // device-visible pointer to the pinned, mapped ring
@@ -75,11 +75,6 @@ struct InstrArgs {
   uint32_t uid;       // unique launch id (kernel id of the paper)
   uint32_t group;     // G
   uint32_t flags;     // INSTR_*
-  // counter mode, a job's last kernel: per-slot ticket counter (device memory, never
-  // reset, running base tbase) that elects the block that exits last; only that block
-  // pays the system-scope fence and publishes the whole grid's exit count
-  uint32_t* ticket;
-  uint32_t tbase;
 };
 
 constexpr uint32_t NCTR = 4096;   // counter slots; > max in-flight launches (<= P)

@@ -82,7 +82,8 @@ static double ns_per_tick() {
 // ---------------------------------------------------------------------------
 enum : uint32_t { EV_ARRIVAL = 1, EV_RECORD = 2, EV_BATCH_END = 3, EV_ISSUE = 4, EV_COMPLETE = 5, EV_OBSERVE = 6, EV_ROUTE = 7,
                   EV_CLOCK = 8,
-                  EV_CONFIG = 100, EV_CAPACITY = 101, EV_MODEL = 110, EV_LAYER = 111, EV_DEMAND = 112 };
+                  EV_CONFIG = 100, EV_CAPACITY = 101, EV_MODEL = 110, EV_LAYER = 111, EV_DEMAND = 112, EV_DEP = 113,
+                  EV_VS = 114 };
 
 struct LogEv {
   uint32_t type, a;
@@ -279,7 +280,6 @@ struct CudaBackend : Backend {
   bool proxy = false;
   bool mirror = false;         // counter mode: kernels only count, k_notify_mirror copies
   uint32_t* ctr_m = nullptr;   // device: NCTR_M x {start, end}
-  uint32_t* ticket_m = nullptr;   // device: NCTR_M last-block tickets (a job's last kernel)
   uint32_t* mirror_h = nullptr;   // pinned, mapped host copy
   uint32_t* mirror_d = nullptr;
   bool pdl = true;             // programmatic dependent launches (off for the naive baseline)
@@ -300,8 +300,6 @@ struct CudaBackend : Backend {
     if (mirror) {
       if (cudaMalloc(&ctr_m, 2 * NCTR_M * sizeof(uint32_t)) != cudaSuccess) return -ENOMEM;
       cudaMemsetAsync(ctr_m, 0, 2 * NCTR_M * sizeof(uint32_t), s);
-      if (cudaMalloc(&ticket_m, NCTR_M * sizeof(uint32_t)) != cudaSuccess) return -ENOMEM;
-      cudaMemsetAsync(ticket_m, 0, NCTR_M * sizeof(uint32_t), s);
       if (cudaHostAlloc((void**)&mirror_h, 2 * NCTR_M * sizeof(uint32_t), cudaHostAllocMapped | cudaHostAllocPortable) !=
           cudaSuccess)
         return -ENOMEM;
@@ -394,7 +392,6 @@ struct CudaBackend : Backend {
     if (proxy_stream) cudaStreamDestroy(proxy_stream);
     if (dev_ring) cudaFree(dev_ring);
     if (ctr_m) cudaFree(ctr_m);
-    if (ticket_m) cudaFree(ticket_m);
     if (mirror_h) cudaFreeHost(mirror_h);
     if (proxy_ctl) cudaFreeHost(proxy_ctl);
     for (auto& s : streams) cudaStreamDestroy(s);
@@ -445,7 +442,7 @@ int make_weight_tmap(void* weights, uint32_t rows, uint32_t kpad, uint32_t box_r
 // ---------------------------------------------------------------------------
 // helpers
 // ---------------------------------------------------------------------------
-static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last, bool instr) {
+static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last, bool instr, bool xout) {
   InstrArgs ia{};
   ia.ring = (Rec*)g->be->ring_dev();
   ia.tail = g->be->tail_dev();
@@ -462,11 +459,11 @@ static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last, bool
     ia.ctr = static_cast<CudaBackend*>(g->be.get())->ctr_m + 2 * slot;
     ia.base = g->ctr_mbase[slot];
     g->ctr_mbase[slot] += grid;
-    ia.ticket = static_cast<CudaBackend*>(g->be.get())->ticket_m + slot;
-    ia.tbase = g->ctr_tbase[slot];
-    if (last) g->ctr_tbase[slot] += grid;
+    if (last && std::getenv("PAELLA_LAST_SYS")) ia.flags |= INSTR_SYSREL;
     ia.flags |= INSTR_CTR;
-    if (!last) ia.flags |= INSTR_RELAXED;   // the job's data dependency is carried by streams
+    // the job's data dependencies are carried by streams -- except towards a consumer on
+    // another virtual stream (NEXT-4), launched once this kernel's final count is seen
+    if (!last && !xout) ia.flags |= INSTR_RELAXED;
     g->ctr_live.push_back(Gpu::CtrLive{uid, slot, ia.base, grid, 0, 0});
     return ia;
   }
@@ -512,7 +509,8 @@ static void launcher_main(Gpu* g, Launcher* L) {
 
 static void do_launch(Gpu* g, Model* m, uint32_t slot, uint32_t layer, uint32_t uid, uint32_t stream, bool instr) {
   const KernelInst& k = m->kernels[layer];
-  InstrArgs ia = make_instr(g, uid, k.grid_total(), layer + 1 == m->kernels.size(), instr);
+  InstrArgs ia = make_instr(g, uid, k.grid_total(), layer + 1 == m->kernels.size(), instr,
+                            g->P->cfg.branches && k.xout);
   const paella_config_t& cfg = g->P->cfg;
   if (!g->launchers.empty()) {
     LaunchDesc d;
@@ -642,6 +640,7 @@ static bool admit(Gpu* g, uint32_t client, const SubmitSlot& s) {
   j.io = P->region[client] + s.io_off;
   j.t_sched = s.t_sched_ns;
   j.live = true;
+  for (uint32_t v = 0; v < MAX_VS; ++v) j.rel_stream[v] = -1;
   auto& args = mg.args[slot];
   args.front().in = j.io;                           // ingest reads client memory
   args.back().out = j.io + m->input_bytes;           // last kernel writes the logits in place
@@ -731,24 +730,25 @@ static void observe_before_record(Gpu* g, uint32_t type, uint32_t uid, uint32_t 
 static void maybe_release(Gpu* g, uint32_t uid) {
   const PolicyLaunch& pl = g->policy->launch(uid);
   const PolicyJob& pj = g->policy->job(pl.job);
-  if (pj.stream >= 0) return;   // still in flight (launch-ahead): stream order holds
+  const uint32_t v = g->policy->model(pj.model)[pl.layer].vs;
+  if (pj.vs_stream[v] >= 0) return;   // still in flight (launch-ahead): stream order holds
   JobRec& j = g->jobs[pl.job];
   const uint32_t s = pl.stream;
-  j.rel_stream = (int32_t)s;
+  j.rel_stream[v] = (int32_t)s;
   g->stats.rel_events++;
   if (!g->launchers.empty()) {
-    if (!j.rel_ev) cudaEventCreateWithFlags((cudaEvent_t*)&j.rel_ev, cudaEventDisableTiming);
-    __atomic_store_n(&j.rel_recorded, (uint8_t)0, __ATOMIC_RELAXED);
+    if (!j.rel_ev[v]) cudaEventCreateWithFlags((cudaEvent_t*)&j.rel_ev[v], cudaEventDisableTiming);
+    __atomic_store_n(&j.rel_recorded[v], (uint8_t)0, __ATOMIC_RELAXED);
     LaunchDesc d{};
-    d.event = j.rel_ev;
-    d.recorded = &j.rel_recorded;
+    d.event = j.rel_ev[v];
+    d.recorded = &j.rel_recorded[v];
     d.stream = s;
     d.kind = 1;
     launcher_push(g, d);
   } else {
-    if (!j.rel_ev) g->be->record_event(s, &j.rel_ev);
-    else g->be->record_existing(s, j.rel_ev);
-    j.rel_recorded = 1;
+    if (!j.rel_ev[v]) g->be->record_event(s, &j.rel_ev[v]);
+    else g->be->record_existing(s, j.rel_ev[v]);
+    j.rel_recorded[v] = 1;
   }
 }
 
@@ -819,21 +819,22 @@ static void decide_and_launch(Gpu* g) {
     JobRec& j = g->jobs[is.job];
     Model* m = g->P->models[j.model].get();
     logev(g, EV_ISSUE, is.stream, is.uid, is.job, is.layer);
-    if (j.rel_stream >= 0) {
-      if ((uint32_t)j.rel_stream != is.stream) {   // moved: wait for the previous stream's release
+    const uint32_t v = g->policy->model(j.model)[is.layer].vs;
+    if (j.rel_stream[v] >= 0) {
+      if ((uint32_t)j.rel_stream[v] != is.stream) {   // moved: wait for the previous stream's release
         g->stats.xstream_waits++;
         if (!g->launchers.empty()) {
           LaunchDesc d{};
-          d.event = j.rel_ev;
-          d.recorded = &j.rel_recorded;
+          d.event = j.rel_ev[v];
+          d.recorded = &j.rel_recorded[v];
           d.stream = is.stream;
           d.kind = 2;
           launcher_push(g, d);
         } else {
-          g->be->wait_event(is.stream, j.rel_ev);
+          g->be->wait_event(is.stream, j.rel_ev[v]);
         }
       }
-      j.rel_stream = -1;
+      j.rel_stream[v] = -1;
     }
     do_launch(g, m, j.slot, is.layer, is.uid, is.stream, g->P->cfg.instrument != 0);
     g->stats.launches++;
@@ -873,6 +874,10 @@ static void apply_inbox(Gpu* g) {
       logev(g, EV_LAYER, nm, l, layers[l].grid, (uint64_t)layers[l].tbar);
       logev(g, EV_DEMAND, nm, l, ((uint64_t)layers[l].demand[1] << 32) | (uint64_t)layers[l].demand[2],
             ((uint64_t)layers[l].demand[3] << 32) | (uint64_t)layers[l].demand[4]);
+      if (g->P->cfg.branches) {   // NEXT-4: the DAG (virtual stream + cross-stream dependencies)
+        logev(g, EV_VS, nm, l, layers[l].vs, 0);
+        for (uint32_t d : layers[l].cross) logev(g, EV_DEP, nm, l, d, 0);
+      }
     }
     if (g->log) fflush(g->log);
     g->models_applied.fetch_add(1, std::memory_order_release);
@@ -1164,7 +1169,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
   if (cfg.prio_classes > cfg.stream_pool && cfg.stream_pool != 0) return -EINVAL;
   if (cfg.launch_threads > 16) return -EINVAL;
   if (cfg.max_jobs_per_model > 4096) return -EINVAL;   // job ids: 65,536 per GPU
-  if (cfg.fake_fault > PAELLA_FAULT_CORRUPT) return -EINVAL;
+  if (cfg.fake_fault > PAELLA_FAULT_CORRUPT || cfg.branches > 1) return -EINVAL;
 
   auto P = std::make_unique<Paella>();
   P->cfg = cfg;
@@ -1251,7 +1256,6 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
       if (cb->mirror) {
         g->ctr_mode = true;
         g->ctr_mbase.assign(NCTR_M, 0);
-        g->ctr_tbase.assign(NCTR_M, 0);
         for (uint32_t sl = NCTR_M; sl-- > 0;) g->ctr_free.push_back(sl);
       }
     }
@@ -1299,7 +1303,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
             ((uint64_t)P->cfg.slack_blocks << 32) | cfg.group_size);
       logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFFu, cfg.ring_capacity, cfg.stream_pool,
             ((uint64_t)pc.prio_classes << 32) | cfg.lookahead);
-      logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFEu, cfg.online_tbar, cfg.max_active_jobs, 0);
+      logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFEu, cfg.online_tbar, cfg.max_active_jobs, cfg.branches);
       for (int r = 0; r < NRES; ++r) logev(g.get(), EV_CAPACITY, (uint32_t)r, (uint64_t)pc.capacity[r], 0, 0);
     }
     if (cfg.device == PAELLA_DEVICE_CUDA &&
@@ -1364,6 +1368,11 @@ int paella_register_model(paella_t* p, const paella_model_desc_t* desc, uint32_t
     L.grid = k.grid_total();
     for (int r = 0; r < NRES; ++r) L.demand[r] = k.demand[r];
     L.tbar = k.tbar;
+    if (P->cfg.branches) {   // NEXT-4: virtual streams; else the chain of the paper's jobs
+      L.vs = k.vs;
+      for (uint32_t d : k.deps)
+        if (m->kernels[d].vs != k.vs) L.cross.push_back(d);
+    }
     m->total_tbar += k.tbar;
     layers.push_back(L);
   }
@@ -1671,6 +1680,9 @@ int paella_kernel_info(paella_t* p, uint32_t model_id, uint32_t k, paella_kernel
   info->tbar_ns = ki.tbar;
   info->flops = ki.flops;
   info->bytes = ki.bytes;
+  info->vs = ki.vs;
+  info->n_deps = (uint32_t)ki.deps.size();
+  for (uint32_t i = 0; i < ki.deps.size() && i < 8; ++i) info->deps[i] = ki.deps[i];
   return 0;
 }
 
@@ -1740,17 +1752,13 @@ static int ensure_iso(Gpu* g) {
     return -ENOMEM;
   std::memset(g->prof_ring_h, 0, cap * sizeof(Rec));
   cudaHostGetDevicePointer(&g->prof_ring_d, g->prof_ring_h, 0);
-  if (cudaMalloc(&g->prof_tail, 256) || cudaMalloc(&g->prof_ctr, 2 * NCTR * sizeof(uint32_t)) ||
-      cudaMalloc(&g->prof_ticket, NCTR * sizeof(uint32_t)))
-    return -ENOMEM;
+  if (cudaMalloc(&g->prof_tail, 256) || cudaMalloc(&g->prof_ctr, 2 * NCTR * sizeof(uint32_t))) return -ENOMEM;
   g->prof_base.assign(NCTR, 0);
-  g->prof_tbase.assign(NCTR, 0);
   cudaStream_t s;
   cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
   g->prof_stream = s;
   cudaMemsetAsync(g->prof_tail, 0, 256, s);
   cudaMemsetAsync(g->prof_ctr, 0, 2 * NCTR * sizeof(uint32_t), s);
-  cudaMemsetAsync(g->prof_ticket, 0, NCTR * sizeof(uint32_t), s);
   // isolated runs write their records to device memory (as served kernels do through
   // the proxy); nobody consumes them except the round-trip benchmark's direct ring
   if (cudaMalloc(&g->prof_devring, cap * sizeof(Rec))) return -ENOMEM;
@@ -2169,9 +2177,7 @@ static InstrArgs iso_instr(Gpu* g, uint32_t grid, uint32_t group, bool last) {
   ia.uid = uid;
   ia.group = group;
   ia.flags = INSTR_ON | (last ? INSTR_LAST : 0);
-  ia.ticket = g->prof_ticket + slot;
-  ia.tbase = g->prof_tbase[slot];
-  if (last) g->prof_tbase[slot] += grid;
+  if (last && std::getenv("PAELLA_LAST_SYS")) ia.flags |= INSTR_SYSREL;
   if (static_cast<CudaBackend*>(g->be.get())->mirror)   // as in serving
     ia.flags |= INSTR_CTR | (last ? 0u : INSTR_RELAXED);
   return ia;

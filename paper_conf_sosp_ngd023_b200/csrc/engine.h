@@ -34,6 +34,13 @@ struct KernelInst {
   int64_t tbar = 0;
   uint64_t flops = 0, bytes = 0;
   int64_t demand[NRES] = {1, 0, 0, 0, 0};
+  // NEXT-4 intra-job concurrency (Fig. 7 waitlists, P906-951): the kernels whose
+  // outputs this one reads (through concats and fused GAPs), its virtual stream, and
+  // whether a kernel on another virtual stream consumes its output (then its exit count
+  // is a release: the consumer is launched on another CUDA stream once it is seen)
+  std::vector<uint32_t> deps;
+  uint32_t vs = 0;
+  bool xout = false;
   uint32_t grid_total() const { return grid[0] * grid[1] * grid[2]; }
 };
 
@@ -72,6 +79,7 @@ struct Model {
   uint32_t in_c = 0, in_h = 0, in_w = 0, out_n = 0;
   std::vector<ModelGpu> gpu;
   int64_t total_tbar = 0;
+  uint32_t n_vs = 1;          // virtual streams of the DAG (1 = a chain)
 };
 
 struct JobRec {
@@ -88,9 +96,10 @@ struct JobRec {
   // all completed and the policy released its stream, an event is recorded on that
   // stream; if the job's next kernel is issued on another stream, that stream waits
   // for the event (stream order carries the data dependency, reading C2-Q19)
-  void* rel_ev = nullptr;
-  uint8_t rel_recorded = 0;
-  int32_t rel_stream = -1;
+  // (per virtual stream, NEXT-4: a job may hold several streams)
+  void* rel_ev[MAX_VS] = {nullptr, nullptr, nullptr, nullptr};
+  uint8_t rel_recorded[MAX_VS] = {0, 0, 0, 0};
+  int32_t rel_stream[MAX_VS] = {-1, -1, -1, -1};
 };
 
 struct Paella;
@@ -178,7 +187,6 @@ struct Gpu {
   std::vector<CtrLive> ctr_live;
   std::vector<uint32_t> ctr_free;           // free counter-mode slots
   std::vector<uint32_t> ctr_mbase;          // running base per counter-mode slot
-  std::vector<uint32_t> ctr_tbase;          // running base of each slot's last-block ticket
   std::vector<JobRec> jobs;         // indexed by job id (dense)
   std::vector<uint32_t> free_job_ids;
   uint32_t next_job = 0;
@@ -218,8 +226,7 @@ struct Gpu {
   Rec* prof_devring = nullptr;     // device-memory ring of isolated runs
   void* trace_buf = nullptr;       // debug phase timestamps
   uint32_t* prof_ctr = nullptr;
-  uint32_t* prof_ticket = nullptr;
-  std::vector<uint32_t> prof_base, prof_tbase;
+  std::vector<uint32_t> prof_base;
   uint32_t prof_uid = 0;
   void* prof_stream = nullptr;
   void* stage_in = nullptr;    // pinned mapped staging for isolated-run io

@@ -91,21 +91,18 @@ __device__ __forceinline__ void kernel_begin(const InstrArgs& ia) {
 }
 
 // Counter mode, a job's LAST kernel (its output is the logits in client host memory):
-// the system-scope flush is paid once per kernel, not once per block.  Every block
-// releases its outputs at gpu scope with an acq_rel ticket atomic; the block that draws
-// the last ticket has acquired all of them, issues one fence.sc.sys (cumulative: the
-// other blocks' host-memory writes are ordered before what follows at system scope) and
-// only then publishes the exit count of the WHOLE grid with a release reduction.  The
-// host therefore never sees the launch complete before every logit is visible.  The
-// caller is one thread of a block whose other threads are past a CTA barrier.
+// each block releases its outputs with a GPU-scope release reduction of the exit count.
+// The host learns the count only through the mirror warp, which acquires it and issues a
+// system-scope fence before publishing it (k_notify_mirror): that fence is cumulative
+// over the logits the blocks released to it, so the host never sees the launch complete
+// before every logit is visible -- one system-scope flush per batch of counter changes
+// instead of one per block.  INSTR_SYSREL (experiment) restores the per-block
+// system-scope release.
 __device__ __forceinline__ void last_kernel_exit(const InstrArgs& ia) {
-  const uint32_t total = gridDim.x * gridDim.y * gridDim.z;
-  uint32_t old;
-  asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(ia.ticket) : "memory");
-  if (old + 1u - ia.tbase == total) {
-    asm volatile("fence.sc.sys;" ::: "memory");
-    asm volatile("red.release.sys.global.add.u32 [%0], %1;" ::"l"(&ia.ctr[1]), "r"(total) : "memory");
-  }
+  if (ia.flags & INSTR_SYSREL)
+    asm volatile("red.release.sys.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+  else
+    asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
 }
 
 // exit count of a block whose every other thread is already past a CTA barrier (the

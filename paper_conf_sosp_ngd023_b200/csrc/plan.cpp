@@ -12,6 +12,7 @@
 //  * concat = producers write disjoint channel ranges of one buffer (zero-copy);
 //  * conv: groups==1 -> tcgen05 implicit GEMM (bf16) or SIMT implicit GEMM (fp32);
 //    depthwise -> K2c;  FC -> GEMV;  pools / GAP -> SIMT.
+#include <algorithm>
 #include <cmath>
 #include <cstdlib>
 #include <cstring>
@@ -424,6 +425,60 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
   if (!exact && es == 2) return -EINVAL;   // bf16 path requires bf16-representable weights
   m->splitk_floats = max_splitk;
   m->splitk_ctrs = max_tiles;
+
+  // ---- NEXT-4: the kernel DAG and its virtual streams (Fig. 7 waitlists) ----
+  // producers(node) = the kernels that write node's tensor: its own kernel, or through a
+  // concat (no kernel, zero-copy) the producers of its inputs, or through a GAP fused
+  // into its FC the producers of the GAP's input
+  std::vector<int32_t> kernel_of(n, -1);
+  for (uint32_t k = 0; k < m->kernels.size(); ++k) kernel_of[m->kernels[k].node < 0 ? 0 : m->kernels[k].node] = k;
+  kernel_of[0] = 0;
+  std::vector<std::vector<uint32_t>> prod(n);
+  for (uint32_t i = 0; i < n; ++i) {
+    if (kernel_of[i] >= 0 && !fused_gap[i]) {
+      prod[i] = {(uint32_t)kernel_of[i]};
+    } else {
+      for (int32_t s : m->node_inputs[i]) prod[i].insert(prod[i].end(), prod[s].begin(), prod[s].end());
+    }
+  }
+  const uint32_t nk = (uint32_t)m->kernels.size();
+  std::vector<int32_t> tail_of_vs;   // last kernel of each virtual stream so far
+  for (uint32_t k = 0; k < nk; ++k) {
+    KernelInst& K = m->kernels[k];
+    std::vector<uint32_t> deps;
+    if (k > 0) {
+      const uint32_t node = (uint32_t)K.node;
+      for (int32_t s : m->node_inputs[node]) deps.insert(deps.end(), prod[s].begin(), prod[s].end());
+      if (d->nodes[node].residual >= 0) {
+        const auto& r = prod[d->nodes[node].residual];
+        deps.insert(deps.end(), r.begin(), r.end());
+      }
+    }
+    std::sort(deps.begin(), deps.end());
+    deps.erase(std::unique(deps.begin(), deps.end()), deps.end());
+    for (uint32_t x : deps)
+      if (x >= k) return -EINVAL;
+    K.deps = deps;
+    // virtual stream: continue the stream whose tail is the most recent dependency;
+    // otherwise open a new one (at most MAX_VS), else join the latest dependency's
+    int32_t vs = -1;
+    for (auto it = deps.rbegin(); it != deps.rend() && vs < 0; ++it)
+      if (tail_of_vs[m->kernels[*it].vs] == (int32_t)*it) vs = (int32_t)m->kernels[*it].vs;
+    if (vs < 0) {
+      if (tail_of_vs.size() < MAX_VS || deps.empty()) {
+        vs = deps.empty() && !tail_of_vs.empty() ? 0 : (int32_t)tail_of_vs.size();
+        if (vs == (int32_t)tail_of_vs.size()) tail_of_vs.push_back(-1);
+      } else {
+        vs = (int32_t)m->kernels[deps.back()].vs;
+      }
+    }
+    K.vs = (uint32_t)vs;
+    tail_of_vs[vs] = (int32_t)k;
+  }
+  m->n_vs = (uint32_t)tail_of_vs.size();
+  for (uint32_t k = 0; k < nk; ++k)
+    for (uint32_t x : m->kernels[k].deps)
+      if (m->kernels[x].vs != m->kernels[k].vs) m->kernels[x].xout = true;
   return 0;
 }
 

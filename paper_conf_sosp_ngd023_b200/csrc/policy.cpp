@@ -16,6 +16,7 @@ Policy::Policy(const Cfg& c) : cfg_(c) {
   unfinished_.assign(c.num_clients, 0);
   per_client_.resize(c.num_clients);
   models_.resize(kMaxModels);   // never reallocated: models are added while dispatching
+  vs_kernels_.resize(kMaxModels);
   model_total_.assign(kMaxModels, 0);
   tb_sum_.resize(kMaxModels);
   tb_cnt_.resize(kMaxModels);
@@ -25,6 +26,13 @@ Policy::Policy(const Cfg& c) : cfg_(c) {
 void Policy::add_model(uint32_t mid, const std::vector<PolicyLayer>& layers) {
   if (mid >= kMaxModels) throw std::runtime_error("too many models");
   models_[mid] = layers;
+  uint32_t nv = 1;
+  for (const auto& l : layers) {
+    if (l.vs >= MAX_VS) throw std::runtime_error("too many virtual streams");
+    nv = std::max(nv, l.vs + 1);
+  }
+  vs_kernels_[mid].assign(nv, {});
+  for (uint32_t k = 0; k < layers.size(); ++k) vs_kernels_[mid][layers[k].vs].push_back(k);
   int64_t t = 0;
   for (const auto& l : layers) t += l.tbar;
   model_total_[mid] = t;
@@ -53,17 +61,31 @@ int Policy::lowest_free_in_class(uint32_t c) const {
   return -1;
 }
 
-bool Policy::is_ready(const PolicyJob& j) const {
-  if (!j.live || j.cursor >= models_[j.model].size()) return false;
-  uint32_t infl = j.inflight();
-  if (infl == 0) return true;
-  if (cfg_.lookahead == 0 || infl > cfg_.lookahead) return false;
-  // kernels of a job complete in order (one stream), so layer `done` is the oldest
-  // kernel still in flight; launch-ahead once it is fully placed (running)
-  const uint32_t oldest = j.uid_of[j.done % 8];
-  const PolicyLaunch& L = launches_[oldest % kLaunchSlots];
-  if (!L.live || L.uid != oldest) return false;
-  return (L.p > L.f ? L.p : L.f) >= L.grid;
+// The job's lowest-index active kernel that may be dispatched now, or -1 (identical to
+// oracle Policy.head): the next kernel of a virtual stream whose cross-stream
+// dependencies have completed and whose stream is idle -- or, with launch-ahead D > 0,
+// whose oldest in-flight kernel is fully placed (running) with at most D in flight.
+int64_t Policy::head(const PolicyJob& j) const {
+  if (!j.live || j.cursor >= models_[j.model].size()) return -1;
+  const auto& ml = models_[j.model];
+  const auto& vk = vs_kernels_[j.model];
+  int64_t best = -1;
+  for (uint32_t v = 0; v < j.nvs; ++v) {
+    if (j.vs_next[v] >= vk[v].size()) continue;
+    const uint32_t k = vk[v][j.vs_next[v]];
+    bool deps_done = true;
+    for (uint32_t d : ml[k].cross) deps_done &= j.state[d] == 2;
+    if (!deps_done) continue;
+    const uint32_t infl = j.vs_infl[v];
+    if (infl > 0) {
+      if (cfg_.lookahead == 0 || infl > cfg_.lookahead) continue;
+      const uint32_t oldest = j.vs_uid[v][j.vs_head[v] % 8];
+      const PolicyLaunch& L = launches_[oldest % kLaunchSlots];
+      if (!L.live || L.uid != oldest || (L.p > L.f ? L.p : L.f) < L.grid) continue;
+    }
+    if (best < 0 || (int64_t)k < best) best = k;
+  }
+  return best;
 }
 
 // bring the ready structures in line with is_ready(j)
@@ -94,7 +116,7 @@ void Policy::refine(const PolicyLaunch& L) {
   if (delta == 0) return;
   for (uint32_t id : live_by_model_[m]) {
     PolicyJob& j = jobs_[id];
-    if (j.cursor > lay) continue;
+    if (j.state[lay] != 0) continue;   // already dispatched
     const bool rdy = j.in_ready;
     if (rdy) make_unready(j);
     active_erase(j);
@@ -148,6 +170,8 @@ void Policy::arrival(uint32_t job_id, uint32_t client, uint32_t model) {
   j.id = job_id;
   j.client = client;
   j.model = model;
+  j.state.assign(models_[model].size(), 0);
+  j.nvs = (uint32_t)vs_kernels_[model].size();
   j.seq = next_seq_++;
   int64_t R = 0;
   for (const auto& l : models_[model]) R += l.tbar;
@@ -187,10 +211,14 @@ bool Policy::record(uint32_t type, uint32_t uid, uint32_t n, int64_t* job_done) 
   L.live = false;
   refine(L);
   j.done += 1;
-  if (j.inflight() == 0) {
+  j.state[L.layer] = 2;
+  const uint32_t v = models_[j.model][L.layer].vs;
+  j.vs_head[v] += 1;                 // a virtual stream's kernels complete in order
+  j.vs_infl[v] -= 1;
+  if (j.vs_infl[v] == 0) {           // drained: its CUDA stream is free
     free_[L.stream / 64] |= 1ull << (L.stream % 64);
-    j.stream = -1;
-    j.last_stream = (int32_t)L.stream;
+    j.vs_stream[v] = -1;
+    j.vs_last[v] = (int32_t)L.stream;
   }
   if (j.done == models_[j.model].size()) {
     if (j.in_ready) make_unready(j);
@@ -286,12 +314,14 @@ void Policy::decide(std::vector<Issue>* out) {
       break;
     }
     PolicyJob& j = jobs_[jid];
+    const uint32_t k = (uint32_t)head(j);
+    const uint32_t v = models_[j.model][k].vs;
     int s0 = lowest_free();
-    if (j.inflight() == 0 && s0 < 0) {
+    if (j.vs_infl[v] == 0 && s0 < 0) {
       last_stop_ = 1;
       break;
     }
-    const PolicyLayer& lay = models_[j.model][j.cursor];
+    const PolicyLayer& lay = models_[j.model][k];
     if (!predicate(lay.grid)) {
       int64_t recs = 2 * (int64_t)((lay.grid + cfg_.group - 1) / cfg_.group);
       last_stop_ = O_ + recs <= cfg_.ring_capacity ? 2 : 3;
@@ -299,26 +329,26 @@ void Policy::decide(std::vector<Issue>* out) {
     }
     uint32_t uid = next_uid_++;
     uint32_t stream;
-    if (j.inflight() > 0) {
-      stream = (uint32_t)j.stream;   // launch-ahead: queued behind its predecessor
+    if (j.vs_infl[v] > 0) {
+      stream = (uint32_t)j.vs_stream[v];   // launch-ahead: queued behind its predecessor
     } else {
       const uint32_t c = job_class(j);
       const uint32_t K = cfg_.prio_classes, P = cfg_.streams;
-      if (j.last_stream >= 0 && (free_[j.last_stream / 64] >> (j.last_stream % 64) & 1) &&
-          stream_class((uint32_t)j.last_stream, K, P) == c) {
-        stream = (uint32_t)j.last_stream;
+      const int32_t last = j.vs_last[v];
+      if (last >= 0 && (free_[last / 64] >> (last % 64) & 1) && stream_class((uint32_t)last, K, P) == c) {
+        stream = (uint32_t)last;
       } else {
         int sc = lowest_free_in_class(c);
         stream = sc >= 0 ? (uint32_t)sc : (uint32_t)s0;
       }
       free_[stream / 64] &= ~(1ull << (stream % 64));
-      j.stream = (int32_t)stream;
+      j.vs_stream[v] = (int32_t)stream;
     }
     PolicyLaunch& L = launches_[uid % kLaunchSlots];
     if (L.live) throw std::runtime_error("launch slot table overflow");
     L.uid = uid;
     L.job = jid;
-    L.layer = j.cursor;
+    L.layer = k;
     L.grid = lay.grid;
     L.stream = stream;
     L.p = L.f = 0;
@@ -331,7 +361,10 @@ void Policy::decide(std::vector<Issue>* out) {
     active_erase(j);
     j.R -= lay.tbar;
     work_ -= lay.tbar;
-    j.uid_of[j.cursor % 8] = uid;
+    j.state[k] = 1;
+    j.vs_uid[v][(j.vs_head[v] + j.vs_infl[v]) % 8] = uid;
+    j.vs_infl[v] += 1;
+    j.vs_next[v] += 1;
     j.cursor += 1;
     j.last_uid = uid;
     j.rr = uid;   // after make_unready above: the ready-set key changes only out of the set

@@ -30,23 +30,36 @@ struct PolicyLayer {
   uint32_t grid;
   int64_t demand[NRES];
   int64_t tbar;
+  // NEXT-4 intra-job concurrency (Fig. 7 waitlists, P906-951): virtual stream of the
+  // kernel and the kernels of OTHER virtual streams it consumes (they must have
+  // completed; predecessors on its own virtual stream are ordered by the stream)
+  uint32_t vs = 0;
+  std::vector<uint32_t> cross;
 };
+
+constexpr uint32_t MAX_VS = 4;   // virtual streams per job
 
 struct PolicyJob {
   uint32_t id = 0;
   uint32_t client = 0, model = 0;
   uint64_t seq = 0;
   int64_t R = 0;
-  uint32_t cursor = 0;       // next kernel to issue (kernels dispatched)
+  uint32_t cursor = 0;       // kernels dispatched
   uint32_t done = 0;         // kernels completed
-  int32_t stream = -1;       // stream held while kernels are in flight
-  int32_t last_stream = -1;
   uint32_t last_uid = 0;
   int64_t rr = -1;           // RR ablation: uid of the last issued kernel (-1 = never)
   uint32_t model_pos = 0;    // index in live_by_model_[model] (NEXT-4)
-  uint32_t uid_of[8] = {0};  // launch uid of layer l (l mod 8) while in flight
   bool live = false;
   bool in_ready = false;
+  std::vector<uint8_t> state;   // per kernel: 0 waiting, 1 in flight, 2 completed
+  // per virtual stream: next kernel (position in the stream), in-flight uids (FIFO),
+  // the CUDA stream held while it has kernels in flight, the last one it held
+  uint32_t nvs = 1;
+  uint32_t vs_next[MAX_VS] = {0};
+  uint32_t vs_uid[MAX_VS][8] = {{0}};
+  uint8_t vs_head[MAX_VS] = {0}, vs_infl[MAX_VS] = {0};
+  int32_t vs_stream[MAX_VS] = {-1, -1, -1, -1};
+  int32_t vs_last[MAX_VS] = {-1, -1, -1, -1};
   uint32_t inflight() const { return cursor - done; }
 };
 
@@ -125,12 +138,14 @@ class Policy {
   void refine(const PolicyLaunch& L);
   void make_ready(PolicyJob& j);
   void make_unready(PolicyJob& j);
-  bool is_ready(const PolicyJob& j) const;
+  bool is_ready(const PolicyJob& j) const { return head(j) >= 0; }
+  int64_t head(const PolicyJob& j) const;
   void refresh(PolicyJob& j);
   int lowest_free() const;
 
   Cfg cfg_;
   std::vector<std::vector<PolicyLayer>> models_;
+  std::vector<std::vector<std::vector<uint32_t>>> vs_kernels_;   // per model, per virtual stream
   std::vector<PolicyJob> jobs_;
   std::vector<PolicyLaunch> launches_;
   int64_t U_[NRES] = {0, 0, 0, 0, 0};

@@ -411,3 +411,32 @@ def test_hybrid_completion_serving(tmp_path):
     for nm, idx, out in got:
         assert within(out, oracle_out(nm, idx, "bf16"), BF16_TOL).all()
     assert cpu < 0.7 * wall, (cpu, wall)
+
+
+@pytest.mark.parametrize("look,K", [(3, 8), (0, 0)])
+def test_serving_branches_c3_models(tmp_path, look, K):
+    """NEXT-4 intra-job branch concurrency on the GPU: C-3's models served with their
+    kernel DAGs over virtual streams (Inception / ResNet-50 branches on several CUDA
+    streams at once; a consumer on another stream is issued after its inputs' final
+    COMPLETION, whose exit count is a release): every output within the bf16 tolerance,
+    the issue order replayed bit-exactly, launch-ahead depth respected per stream."""
+    log = str(tmp_path / "br_%u.log")
+    names = ["resnet50", "inception_v3", "mobilenet_v2", "squeezenet1_1"]
+    for nm in names:
+        for i in range(4):
+            oracle_out(nm, i, "bf16")
+    with L.Engine(num_clients=4, event_log=log, max_jobs_per_model=32, lookahead=look, launch_threads=4,
+                  slack=1184, region_bytes=96 << 20, branches=True, max_active=K) as e:
+        specs = []
+        for nm in names:
+            g = archs.build(nm)
+            specs.append((e.register_model(g, rng.model_params(g)), nm, g))
+        _serve_and_check(e, specs, 80, 4, seed=23 + look)
+        st = e.stats()
+        assert st["completed"] == 80
+    cfg, ms, events, ex = eventlog.read(log % 0)
+    assert any(l.vs > 0 for m in ms for l in m)
+    ok, msg, n = sim.replay(cfg, ms, events)
+    assert ok, msg
+    assert n == len(ex["issues"]) == st["launches"]
+    assert sim.check_inflight_bound(events, ms, look) == []

@@ -277,3 +277,102 @@ def test_fake_replay_max_active(tmp_path, policy, theta, K, look):
     ok, msg, n = sim.replay(cfg, ms, events)
     assert ok, msg
     assert n == len(ex["issues"]) > 0 and len(ex["completes"]) == 200
+
+
+# --- NEXT-4 intra-job branch concurrency (Fig. 7 waitlists, P906-951) ---------------
+
+def _graph_kernel_deps(g):
+    """Independent derivation of each kernel's inputs from the graph: kernel nodes are
+    every node except concats and a GAP whose only consumer is an FC (fused); a node's
+    tensor is written by its own kernel, else (concat / fused GAP) by the kernels of its
+    inputs.  Returns {node: sorted producer nodes of the node's inputs + residual}."""
+    nodes = g.nodes
+    users = {}
+    for i, n in enumerate(nodes):
+        for s in n["inputs"]:
+            users.setdefault(s, []).append(i)
+        if n.get("residual") is not None:
+            users.setdefault(n["residual"], []).append(i)
+    fused = {i for i, n in enumerate(nodes) if n["op"] == "gap" and len(users.get(i, [])) == 1
+             and nodes[users[i][0]]["op"] == "fc"}
+
+    def writers(i):
+        if i == 0 or (nodes[i]["op"] != "concat" and i not in fused):
+            return {i}
+        out = set()
+        for s in nodes[i]["inputs"]:
+            out |= writers(s)
+        return out
+    deps = {}
+    for i, n in enumerate(nodes):
+        if i == 0 or n["op"] == "concat" or i in fused:
+            continue
+        ws = set()
+        for s in n["inputs"]:
+            ws |= writers(s)
+        if n.get("residual") is not None:
+            ws |= writers(n["residual"])
+        deps[i] = sorted(ws)
+    return deps
+
+
+@pytest.mark.parametrize("name", ["squeezenet1_1", "inception_v3", "resnet50", "densenet121"])
+def test_planner_dag_matches_graph(name):
+    """The planner's per-kernel dependencies equal an independent derivation from the
+    graph; virtual streams number <= 4; every dependency on the SAME virtual stream is an
+    earlier kernel of that stream (so stream order covers it)."""
+    g = archs.build(name)
+    with _toy_engine(num_clients=1, branches=True) as e:
+        mid = e.register_model(g, rng.model_params(g))
+        ks = e.kernels(mid)
+    node_of = {}
+    kidx = 1
+    want = _graph_kernel_deps(g)
+    kernel_nodes = [0] + sorted(want)
+    assert len(kernel_nodes) == len(ks)
+    node_of = {k: n for k, n in enumerate(kernel_nodes)}
+    kof = {n: k for k, n in node_of.items()}
+    for k, info in enumerate(ks):
+        if k == 0:
+            assert info["n_deps"] == 0
+            continue
+        exp = [kof[n] for n in want[node_of[k]]]
+        assert info["n_deps"] == len(exp), (k, info["n_deps"], exp)
+        assert info["deps"] == exp[:8], (k, info["deps"], exp)
+        assert info["vs"] < 4
+    nvs = len({k["vs"] for k in ks})
+    if name in ("inception_v3", "squeezenet1_1", "resnet50"):
+        assert nvs >= 2                   # branches exist
+    if name == "densenet121":
+        assert nvs == 1                   # every layer reads all earlier ones: one chain
+
+
+@pytest.mark.parametrize("policy,look,K", [(L.POLICY_SRPT_DEFICIT, 0, 0), (L.POLICY_SRPT_DEFICIT, 2, 0),
+                                           (L.POLICY_FIFO, 3, 2), (L.POLICY_SRPT_DEFICIT, 3, 3)])
+def test_fake_replay_branches(tmp_path, policy, look, K):
+    """NEXT-4: jobs whose kernels form a DAG over virtual streams (several CUDA streams
+    per job) replay bit-exactly through the oracle policy (Topo / head)."""
+    log = str(tmp_path / "ev_%u.log")
+    models = [archs.squeezenet1_1(), archs.inception_v3()]
+    with _toy_engine(num_clients=2, policy=policy, streams=12, event_log=log, ring_capacity=4096, slack=8,
+                     lookahead=look, branches=True, max_active=K, fake_sms=8) as e:
+        mids = [e.register_model(g, rng.model_params(g)) for g in models]
+        _serve(e, mids, 60, 2, seed=17 + look)
+    cfg, ms, events, ex = eventlog.read(log % 0)
+    assert any(l.vs > 0 for m in ms for l in m)
+    ok, msg, n = sim.replay(cfg, ms, events)
+    assert ok, msg
+    assert n == len(ex["issues"]) and len(ex["completes"]) == 60
+    # two kernels of one job were in flight on different streams at the same time
+    grid = {uid: ms[model][layer].grid for (uid, job, layer, stream, model) in ex["issues"]}
+    done, live, conc = {}, {}, False
+    for ev in events:
+        if ev[0] == sim.EV_ISSUE:
+            uid, job, layer, stream = ev[1:5]
+            live[uid] = (job, stream)
+            conc |= len({s for (j, s) in live.values() if j == job}) > 1
+        elif ev[0] == sim.EV_RECORD and ev[1] == sim.COMPLETION:
+            done[ev[2]] = done.get(ev[2], 0) + ev[3]
+            if done[ev[2]] == grid[ev[2]]:
+                live.pop(ev[2])
+    assert conc

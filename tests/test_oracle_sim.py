@@ -695,3 +695,54 @@ def test_decide_delay_throughput_falls():
         rates.append(120 / max(res.finish.values()))
     assert all(a >= b for a, b in zip(rates, rates[1:])), rates
     assert rates[-1] < 0.5 * rates[0], rates
+
+
+# --- NEXT-4: intra-job branches (Fig. 7 waitlists, P906-951), hand-derived ----------
+
+def _diamond(d):
+    """k0 (vs 0) -> k1 (vs 0) and k2 (vs 1) -> k3 (vs 0, consumes k2 from vs 1)."""
+    Ld = lambda deps, vs: Layer(1, (1, 1, 1, 1, 0), d, d, deps=deps, vs=vs)   # noqa: E731
+    return [[Ld((), 0), Ld((), 0), Ld((0,), 1), Ld((2,), 0)]]
+
+
+@pytest.mark.parametrize("D", [0, 1])
+def test_branches_diamond_closed_form(D):
+    """Zero delays, 2 SMs, d = 1 unit.  t = 0: k0 issued (with D = 1 also k1, queued
+    behind it on stream 0); k2 waits for its cross-stream input k0.  t = 1: k0 completes;
+    k2 is issued on a second stream (and k1 too when D = 0, lower index first); k1 and
+    k2 run together 1..2.  k3 waits for k2 (another virtual stream) even with
+    launch-ahead: issued at 2, done at 3.  JCT = 3 units (the chain takes 4)."""
+    u = 1000
+    cfg = Config(num_clients=1, theta=sim.INF_THETA, slack=10**6, lookahead=D, streams=4,
+                 capacity=(10**6, 10**9, 10**12, 10**12, 10**9))
+    gpu = GPUModel(sms=2, per_sm=(1, 64, 65536, 233472, 512))
+    res = sim.simulate(cfg, _diamond(u), [(0, 0, 0)], gpu)
+    t_issue = {layer: t for (t, uid, jid, layer, stream) in res.issues}
+    stream = {layer: s for (t, uid, jid, layer, s) in res.issues}
+    assert t_issue == ({0: 0, 1: u, 2: u, 3: 2 * u} if D == 0 else {0: 0, 1: 0, 2: u, 3: 2 * u})
+    assert stream[2] != stream[1] and stream[0] == stream[1] == stream[3]
+    assert res.jct()[0] == 3 * u
+    chain = [[Layer(1, (1, 1, 1, 1, 0), u, u)] * 4]
+    assert sim.simulate(cfg, chain, [(0, 0, 0)], gpu).jct()[0] == 4 * u
+
+
+def test_branches_cross_dependency_blocks_until_completion():
+    """k3 consumes k2 from another virtual stream: it is not active while k2 is merely
+    placed, only once k2's final COMPLETION is consumed (policy-level trace)."""
+    pol = sim.Policy(Config(num_clients=1, theta=sim.INF_THETA, slack=10**6, lookahead=3, streams=4,
+                            capacity=(10**6, 10**9, 10**12, 10**12, 10**9)), _diamond(10))
+    pol.arrival(0, 0, 0)
+    (u0, _, l0, s0), = pol.decide()
+    assert l0 == 0
+    pol.record(sim.PLACEMENT, u0, 1)
+    (u1, _, l1, _), = pol.decide()
+    assert l1 == 1                                              # k1 behind k0; k2 not active
+    pol.record(sim.COMPLETION, u0, 1)
+    iss = pol.decide()
+    assert [l for (_, _, l, _) in iss] == [2]
+    u2 = iss[0][0]
+    pol.record(sim.PLACEMENT, u2, 1)
+    pol.record(sim.PLACEMENT, u1, 1)
+    assert pol.head(pol.jobs[0]) is None      # k1 running (launch-ahead would allow k3) but k2 not done
+    pol.record(sim.COMPLETION, u2, 1)
+    assert pol.head(pol.jobs[0]) == 3

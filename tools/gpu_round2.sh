@@ -13,3 +13,10 @@ if [ -n "$KT" ]; then
 timeout 900 python tools/kernel_times.py > gpurun_out/kernel_times_${TAG}.txt 2>&1; echo "kt rc=$?"; tail -2 gpurun_out/kernel_times_${TAG}.txt
 cp gpurun_out/kernel_times.json gpurun_out/kernel_times_${TAG}.json
 fi
+if [ -n "$KTSYS" ]; then
+PAELLA_LAST_SYS=1 timeout 900 python tools/kernel_times.py > gpurun_out/kernel_times_${TAG}_sys.txt 2>&1; echo "ktsys rc=$?"; tail -1 gpurun_out/kernel_times_${TAG}_sys.txt
+cp gpurun_out/kernel_times.json gpurun_out/kernel_times_${TAG}_sys.json
+fi
+if [ -n "$SWEEP" ]; then
+VAR=$SWEEP TAG=${TAG}_sweep LAM=${LAM:-3600} bash tools/gpu_sweep_r2.sh
+fi

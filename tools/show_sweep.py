@@ -15,6 +15,8 @@ for path in sys.argv[1:]:
                 tag += f" K{v['max_active']}"
             if "theta" in v:
                 tag += f" th{v['theta']}"
+            if v.get("branches"):
+                tag += " br"
             if v.get("prio_classes", 1) > 1:
                 tag += f" pc{v['prio_classes']}"
         pm = " ".join(f"{k[:5]}={x:.0f}" for k, x in d["per_model_mean_us"].items())
