@@ -396,7 +396,10 @@ def run_gpu(args, ngpus, cores, fake):
     stride = (max(sizes) + 4095) // 4096 * 4096
     region = slots * stride + (1 << 20)
     pol = {"srpt": L.POLICY_SRPT_DEFICIT, "fifo": L.POLICY_FIFO, "sjf": L.POLICY_SJF, "rr": L.POLICY_RR}
-    common = dict(launch_threads=0 if fake else args.launch_threads, max_jobs_per_model=128)
+    # launcher helper threads spin on their queues: keep dispatchers + helpers within the host
+    ncores = len(os.sched_getaffinity(0))
+    lt = min(args.launch_threads, max(1, (ncores - 2 - ngpus) // max(1, ngpus)))
+    common = dict(launch_threads=0 if fake else lt, max_jobs_per_model=128)
     if cores:
         common["dispatcher_cpus"] = cores
     paella_kw = dict(policy=pol[args.policy], theta=args.theta, decide_delay_ns=args.decide_delay_ns,
@@ -424,7 +427,8 @@ def run_gpu(args, ngpus, cores, fake):
     def arm(label, n=ngpus):
         return Arm(L, label, specs, pool, n, region, stride, slots, fake, **common, **arms_kw[label])
 
-    detail = {"config": args.config, "models": names, "n_gpus": ngpus, "dispatcher_cpus": cores}
+    detail = {"config": args.config, "models": names, "n_gpus": ngpus, "dispatcher_cpus": cores,
+              "launch_threads_per_gpu": common["launch_threads"], "host_cores": ncores}
     # --- calibration (untimed): naive X_sat on ONE GPU, unloaded JCT -> SLO ---------------
     t_cal = time.time()
     a1 = arm("naive", 1)

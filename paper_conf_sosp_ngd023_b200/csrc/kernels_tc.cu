@@ -499,6 +499,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   // (its prologue overlaps this epilogue); warp 5 follows the accumulator too
   if (warp == 5 && nkl > 0) mbar_wait(accb, 0);
   constexpr uint32_t RELAXED_CTR = INSTR_CTR | INSTR_RELAXED;
+  pdl_trigger();
   if constexpr (INSTR) {
     // relaxed exit count (B200-Q7): it orders nothing, so the bookkeeping warp
     // counts the block as soon as its MMAs are complete -- the count travels while the
@@ -506,7 +507,6 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     if (warp == 5 && lane == 0 && (ia.flags & RELAXED_CTR) == RELAXED_CTR)
       asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
   }
-  pdl_trigger();
   if (warp < 4) {
     const uint32_t row = warp * 32 + lane;
     if (nkl > 0) {

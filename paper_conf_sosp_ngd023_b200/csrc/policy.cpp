@@ -79,7 +79,7 @@ int64_t Policy::head(const PolicyJob& j) const {
     const uint32_t infl = j.vs_infl[v];
     if (infl > 0) {
       if (cfg_.lookahead == 0 || infl > cfg_.lookahead) continue;
-      const uint32_t oldest = j.vs_uid[v][j.vs_head[v] % 8];
+      const uint32_t oldest = j.vs_uid[v][0];
       const PolicyLaunch& L = launches_[oldest % kLaunchSlots];
       if (!L.live || L.uid != oldest || (L.p > L.f ? L.p : L.f) < L.grid) continue;
     }
@@ -213,7 +213,15 @@ bool Policy::record(uint32_t type, uint32_t uid, uint32_t n, int64_t* job_done) 
   j.done += 1;
   j.state[L.layer] = 2;
   const uint32_t v = models_[j.model][L.layer].vs;
-  j.vs_head[v] += 1;                 // a virtual stream's kernels complete in order
+  // drop the uid from the stream's in-flight list (completions of one stream may be
+  // consumed out of issue order: the drain visits launches in any order)
+  {
+    uint32_t* u = j.vs_uid[v];
+    uint32_t n = j.vs_infl[v], i = 0;
+    while (i < n && u[i] != L.uid) ++i;
+    if (i == n) throw std::runtime_error("completion of a launch not in flight on its stream");
+    for (; i + 1 < n; ++i) u[i] = u[i + 1];
+  }
   j.vs_infl[v] -= 1;
   if (j.vs_infl[v] == 0) {           // drained: its CUDA stream is free
     free_[L.stream / 64] |= 1ull << (L.stream % 64);
@@ -362,7 +370,7 @@ void Policy::decide(std::vector<Issue>* out) {
     j.R -= lay.tbar;
     work_ -= lay.tbar;
     j.state[k] = 1;
-    j.vs_uid[v][(j.vs_head[v] + j.vs_infl[v]) % 8] = uid;
+    j.vs_uid[v][j.vs_infl[v]] = uid;
     j.vs_infl[v] += 1;
     j.vs_next[v] += 1;
     j.cursor += 1;

@@ -56,8 +56,8 @@ struct PolicyJob {
   // the CUDA stream held while it has kernels in flight, the last one it held
   uint32_t nvs = 1;
   uint32_t vs_next[MAX_VS] = {0};
-  uint32_t vs_uid[MAX_VS][8] = {{0}};
-  uint8_t vs_head[MAX_VS] = {0}, vs_infl[MAX_VS] = {0};
+  uint32_t vs_uid[MAX_VS][8] = {{0}};   // in-flight uids in issue order (vs_infl of them)
+  uint8_t vs_infl[MAX_VS] = {0};
   int32_t vs_stream[MAX_VS] = {-1, -1, -1, -1};
   int32_t vs_last[MAX_VS] = {-1, -1, -1, -1};
   uint32_t inflight() const { return cursor - done; }

@@ -440,3 +440,71 @@ def test_serving_branches_c3_models(tmp_path, look, K):
     assert ok, msg
     assert n == len(ex["issues"]) == st["launches"]
     assert sim.check_inflight_bound(events, ms, look) == []
+
+
+@pytest.mark.parametrize("dtype", ["bf16", "fp32"])
+def test_c1_toy_config(tmp_path, dtype):
+    """BASELINE configs[0] / SURVEY.md 8(d) C-1 as specified: 2 clients x 100 requests of
+    the toy model, superposed Poisson arrivals at 5,000 req/s, every request with its own
+    input (pool indices 0..199), theta = 100, B = 148, G = 16.  Every output is checked
+    against the float64 oracle (bf16: 2e-2 / 1e-2, fp32: 1e-4), the issue order replays
+    bit-exactly, records tile every launch exactly once, and the oracle simulator runs
+    the same trace (synthetic mode, profiled T-bar) in seconds."""
+    from workload import traces
+    log = str(tmp_path / "c1_%u.log")
+    g = archs.toy()
+    P = rng.model_params(g)
+    n = 200
+    t = traces.arrivals(n, 5000.0, kind="poisson", seed=1)
+    clients = np.arange(n) % 2
+    tol = BF16_TOL if dtype == "bf16" else FP32_TOL
+    with L.Engine(num_clients=2, event_log=log, slack=148) as e:
+        mid = e.register_model(g, P, dtype=L.DTYPE_BF16 if dtype == "bf16" else L.DTYPE_FP32)
+        info = e.model_info(mid)
+        need = info["input_bytes"] + info["output_bytes"]
+        stride = (need + 255) // 256 * 256
+        offs = {}
+        for i in range(n):                       # request i: its own slot and input
+            c = int(clients[i])
+            off = (i // 2) * stride
+            x = rng.image(g, i)
+            _, reg = e.region(c)
+            reg[off:off + x.nbytes] = np.frombuffer(x.tobytes(), np.uint8)
+            offs[i] = (c, off)
+        t0 = time.monotonic_ns() + 2_000_000
+        pending = set()
+        i = 0
+        while i < n or pending:
+            now = time.monotonic_ns()
+            while i < n and t0 + int(t[i]) <= now:
+                c, off = offs[i]
+                rid = e.submit(c, mid, off, need, t_sched_ns=t0 + int(t[i]))
+                assert rid >= 0
+                pending.add(rid)
+                i += 1
+            for c in (0, 1):
+                rid, st = e.poll(c)
+                if rid >= 0:
+                    assert st == 0
+                    pending.discard(rid)
+            assert time.monotonic_ns() - t0 < 30e9
+        ib = info["input_bytes"]
+        for i in range(n):                       # every output, against the float64 oracle
+            c, off = offs[i]
+            _, reg = e.region(c)
+            out = np.frombuffer(reg[off + ib:off + need].tobytes(), np.float32)
+            ref = infer.forward(g, P, rng.image(g, i), dtype=dtype)
+            assert within(out, ref, tol).all(), (i, np.abs(out - ref).max())
+    cfg, ms, events, ex = eventlog.read(log % 0)
+    ok, msg, nchk = sim.replay(cfg, ms, events)
+    assert ok, msg
+    grids = {uid: ms[model][layer].grid for (uid, job, layer, stream, model) in ex["issues"]}
+    assert sim.check_exactly_once(ex["records"], grids, cfg.group) == []
+    assert ex["n_arrivals"] == n == len(ex["completes"])
+    # the simulator on the same trace: synthetic GPU, block durations = profiled T-bar
+    models = [[sim.Layer(l.grid, l.demand, l.tbar, max(1, l.tbar)) for l in m] for m in ms]
+    trace = [(int(t[k]), int(clients[k]), 0) for k in range(n)]
+    ts = time.perf_counter()
+    res = sim.simulate(sim.Config(num_clients=2, slack=148), models, trace, sim.GPUModel(), check=True)
+    assert len(res.finish) == n and not res.violations
+    assert time.perf_counter() - ts < 30

@@ -20,3 +20,6 @@ fi
 if [ -n "$SWEEP" ]; then
 VAR=$SWEEP TAG=${TAG}_sweep LAM=${LAM:-3600} bash tools/gpu_sweep_r2.sh
 fi
+if [ -n "$C5" ]; then
+timeout 600 python tools/c5_table.py ${TAG} > gpurun_out/c5_${TAG}.txt 2>&1; echo "c5 rc=$?"; tail -3 gpurun_out/c5_${TAG}.txt
+fi

@@ -32,9 +32,13 @@ if cfg["weights"] is None:   # Fig. 12 convention: inverse of the unloaded job s
 for v in variants:
     v = dict(v)
     v.setdefault("launch_threads", 2)
-    e, mids = bench.build_engine(L, specs, 0, fake=False, region_bytes=slots * stride + (1 << 20),
-                                 max_jobs_per_model=128, **v)
-    bench.stage_inputs(e, specs, mids, slots, stride, pool)
+    e = L.Engine(num_clients=len(specs), region_bytes=slots * stride + (1 << 20), max_jobs_per_model=128, **v)
+    mids = [e.register_model(g, P) for (g, P) in specs]
+    for c, (g, _) in enumerate(specs):
+        _, reg = e.region(c)
+        for s_ in range(slots):
+            x = pool[c][s_ % len(pool[c])]
+            reg[s_ * stride:s_ * stride + x.nbytes] = np.frombuffer(x.tobytes(), np.uint8)
     t, mm, ii = bench.make_trace(nreq // 3, lam, cfg, len(names), seed=5)
     e.loadgen(t, mm, mm, ii, stride, slots)   # warm-up
     s0 = e.stats()
