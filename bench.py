@@ -58,6 +58,8 @@ METRIC = "req/s at p99 SLO (Paella, open-loop batch-1 mix), with mean/p99 JCT"
 WORKLOADS = {"c2_mix": "BASELINE configs[1]: mixed ResNet-18/MobileNetV2/SqueezeNet1.1 batch-1, Poisson",
              "c3_dispersion": "BASELINE configs[2]/[3]: ResNet-50/DenseNet-121/Inception-v3/MobileNetV2 batch-1, "
                               "lognormal sigma=2 bursts",
+             "c3_sigma15": "BASELINE configs[2] variant: the C-3 mix with lognormal sigma=1.5 arrivals",
+             "c3_uniform": "BASELINE configs[2] variant: the C-3 models in a uniform mix, sigma=2",
              "c1_toy": "BASELINE configs[0]: 2 clients, toy conv+MLP, Poisson"}
 
 

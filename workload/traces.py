@@ -49,4 +49,10 @@ CONFIGS = {
                    arrival="poisson"),
     "c3_dispersion": dict(models=["resnet50", "densenet121", "inception_v3", "mobilenet_v2"], weights=None,
                           clients=4, arrival="lognormal", sigma=2.0),
+    # C-3 variants: the less bursty arrivals (sigma = 1.5, P1370-1372) and
+    # a uniform model mix (Fig. 11 convention, P1463-1464)
+    "c3_sigma15": dict(models=["resnet50", "densenet121", "inception_v3", "mobilenet_v2"], weights=None,
+                       clients=4, arrival="lognormal", sigma=1.5),
+    "c3_uniform": dict(models=["resnet50", "densenet121", "inception_v3", "mobilenet_v2"], weights=[1, 1, 1, 1],
+                       clients=4, arrival="lognormal", sigma=2.0),
 }
