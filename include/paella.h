@@ -222,6 +222,9 @@ typedef struct {
 #define PAELLA_OP_GAP     4u   /* global average pool */
 #define PAELLA_OP_FC      5u
 #define PAELLA_OP_CONCAT  6u   /* channel concat, realised by channel-offset stores */
+#define PAELLA_OP_SPIN    7u   /* synthetic kernel of the HoL microbenchmark (Fig. 2, P431-445):
+                                  one block of 128 threads resident for kh microseconds that
+                                  copies its input (c channels, 1 x 1) to its output */
 
 #define PAELLA_ACT_NONE  0u
 #define PAELLA_ACT_RELU  1u

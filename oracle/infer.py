@@ -146,6 +146,8 @@ def forward(g, params, image, dtype="bf16", return_all=False):
             y = y.reshape(-1, 1, 1)
         elif op == "concat":
             y = np.concatenate(ins, axis=0)
+        elif op == "spin":          # Fig. 2 synthetic kernel: occupies the GPU, computes nothing
+            y = ins[0]
         else:
             raise ValueError(op)
         assert y.shape == n["out"], (n["name"], y.shape, n["out"])

@@ -25,7 +25,7 @@ DTYPE_BF16, DTYPE_FP32 = 0, 1
 NONBLOCK = 1
 FAULT_NONE, FAULT_DROP, FAULT_DUP, FAULT_TORN, FAULT_HANG, FAULT_CORRUPT = 0, 1, 2, 3, 4, 5
 HYBRID = 2
-OP = {"input": 0, "conv": 1, "maxpool": 2, "avgpool": 3, "gap": 4, "fc": 5, "concat": 6}
+OP = {"input": 0, "conv": 1, "maxpool": 2, "avgpool": 3, "gap": 4, "fc": 5, "concat": 6, "spin": 7}
 ACT = {"none": 0, "relu": 1, "relu6": 2}
 NODE_PROLOGUE, NODE_CEIL = 1, 2
 INT64_MAX = (1 << 63) - 1
@@ -265,6 +265,8 @@ class Engine:
                 nd.groups = 1
             elif n["op"] == "fc":
                 nd.cout = n["cout"]
+            elif n["op"] == "spin":
+                nd.kh = n["us"]
             if n["op"] in ("conv", "fc"):
                 w = np.ascontiguousarray(params[n["name"] + ".weight"], dtype=np.float32)
                 b = np.ascontiguousarray(params[n["name"] + ".bias"], dtype=np.float32)

@@ -1174,6 +1174,10 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
   auto P = std::make_unique<Paella>();
   P->cfg = cfg;
   if (cfg.device == PAELLA_DEVICE_CUDA) {
+    // 32 hardware work queues (the default is 8) for every system, so
+    // the stream pool's 32 streams map onto distinct queues.  Effective only if this
+    // process has not initialised CUDA yet (an existing value is kept).
+    setenv("CUDA_DEVICE_MAX_CONNECTIONS", "32", 0);
     int n = 0;
     if (cudaGetDeviceCount(&n) != cudaSuccess || n < (int)(cfg.first_gpu + cfg.num_gpus)) return -ENODEV;
     cudaDeviceProp prop;
@@ -1688,7 +1692,7 @@ int paella_kernel_info(paella_t* p, uint32_t model_id, uint32_t k, paella_kernel
 
 const char* paella_kernel_name(uint32_t kind) {
   static const char* names[] = {"ingest", "conv_simt", "conv_tcgen05", "dwconv", "maxpool",
-                                "avgpool", "gap", "fc_gemv", "empty", "conv_tcgen05_pro", "gap_fc"};
+                                "avgpool", "gap", "fc_gemv", "empty", "conv_tcgen05_pro", "gap_fc", "spin"};
   return kind < KIND_COUNT ? names[kind] : "?";
 }
 

@@ -16,7 +16,8 @@ enum KernelKind : uint32_t {
   KIND_EMPTY = 8,
   KIND_CONV_TC_PRO = 9, // tcgen05 conv with the per-channel affine+ReLU input prologue
   KIND_GAPFC = 10,      // fused global average pool + FC classifier head
-  KIND_COUNT = 11,
+  KIND_SPIN = 11,       // synthetic HoL-microbenchmark kernel (Fig. 2): one resident block
+  KIND_COUNT = 12,
 };
 
 typedef void (*KernelFn)();

@@ -554,6 +554,24 @@ __global__ void __launch_bounds__(256) k_gapfc(const __grid_constant__ LayerArgs
 }
 
 // ---------------------------------------------------------------------------
+// Synthetic kernel of the HoL microbenchmark (Fig. 2, P431-445): one block stays
+// resident a.kh microseconds (globaltimer) and copies its 8-channel 1x1 input.
+// ---------------------------------------------------------------------------
+template <typename T, bool INSTR>
+__global__ void __launch_bounds__(128) k_spin(const __grid_constant__ LayerArgs a,
+                                              const __grid_constant__ InstrArgs ia) {
+  kernel_begin<INSTR>(ia);
+  if (threadIdx.x == 0) {
+    float v[8];
+    load8(static_cast<const T*>(a.in) + a.in_co, v);
+    const uint64_t t0 = globaltimer(), dur = (uint64_t)a.kh * 1000u;
+    while (globaltimer() - t0 < dur) __nanosleep(200);
+    store8(static_cast<T*>(a.out) + a.out_co, v);
+  }
+  instr_exit<INSTR>(ia);
+}
+
+// ---------------------------------------------------------------------------
 // Empty instrumented kernel for the notification microbenchmark (K5, Fig. 15).
 // ---------------------------------------------------------------------------
 template <bool INSTR>
@@ -727,6 +745,7 @@ static void fill(KernelFn (&t)[KIND_COUNT]) {
   t[KIND_FC] = (KernelFn)k_fc<T, I>;
   t[KIND_EMPTY] = (KernelFn)k_empty<I>;
   t[KIND_GAPFC] = (KernelFn)k_gapfc<T, I>;
+  t[KIND_SPIN] = (KernelFn)k_spin<T, I>;
 }
 
 void simt_kernel_table(KernelFn (&bf16_instr)[KIND_COUNT], KernelFn (&bf16_plain)[KIND_COUNT],

@@ -339,6 +339,14 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
         k.bytes = (uint64_t)sn.h * sn.w * sn.c * es + (uint64_t)P_out * nd.c * es;
         break;
       }
+      case PAELLA_OP_SPIN: {   // Fig. 2 synthetic kernel (HoL microbenchmark)
+        k.kind = KIND_SPIN;
+        if (nd.c != cin || nd.h != sn.h || nd.w != sn.w || nd.h * nd.w != 1 || nd.c % 8) return -EINVAL;
+        k.grid[0] = 1;
+        k.block = 128;
+        k.bytes = 2ull * nd.c * es;
+        break;
+      }
       case PAELLA_OP_GAP: {
         k.kind = KIND_GAP;
         if (nd.c != sn.c || sn.c % 8) return -EINVAL;

@@ -508,3 +508,17 @@ def test_c1_toy_config(tmp_path, dtype):
     res = sim.simulate(sim.Config(num_clients=2, slack=148), models, trace, sim.GPUModel(), check=True)
     assert len(res.finish) == n and not res.violations
     assert time.perf_counter() - ts < 30
+
+
+def test_hol_spin_kernels(engine):
+    """The Fig. 2 synthetic job on the GPU: 8 one-block kernels, each resident >= its spin
+    time (device time of the chain >= 8 x 20 us), output = the bf16-rounded input
+    (identity copies; oracle closed form)."""
+    from oracle.bf16 import round_bf16
+    g = archs.hol_synthetic(8, 20)
+    mid = engine.register_model(g, rng.model_params(g), name="hol-test")
+    for i in range(3):
+        x = rng.image(g, i)
+        out, kt = engine.run_isolated(mid, x, timing=True)
+        assert np.array_equal(out, round_bf16(x).reshape(-1)), (out, x)
+        assert all(t >= 20_000 for t in kt[1:9]), kt

@@ -376,3 +376,21 @@ def test_fake_replay_branches(tmp_path, policy, look, K):
             if done[ev[2]] == grid[ev[2]]:
                 live.pop(ev[2])
     assert conc
+
+
+def test_hol_synthetic_model_plans_and_serves():
+    """Fig. 2's synthetic job (8 one-block spin kernels + a 1-pixel GAP): planned as
+    ingest + 8 spin kernels + GAP, each spin kernel 1 block x 128 threads; served on the
+    fake device; the oracle's forward is the identity on the 8-channel input (closed form)."""
+    from oracle import infer
+    g = archs.hol_synthetic(8, 50)
+    P = rng.model_params(g)
+    assert P == {}
+    x = rng.image(g, 3)
+    assert np.array_equal(infer.forward(g, P, x, dtype="fp32"), x.reshape(-1).astype(np.float64))
+    with _toy_engine(num_clients=1, max_jobs_per_model=64) as e:
+        mid = e.register_model(g, P)
+        ks = e.kernels(mid)
+        assert [k["name"] for k in ks] == ["ingest"] + ["spin"] * 8 + ["gap"]
+        assert all(k["grid"] == 1 and k["block"] == 128 for k in ks[1:9])
+        _serve(e, [mid], 40, 1, seed=2, stride=256)

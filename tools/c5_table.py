@@ -13,6 +13,7 @@ notification latency, written to gpurun_out/c5_<tag>.json and printed as a table
 """
 import json
 import os
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
 import sys
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))

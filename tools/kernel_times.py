@@ -4,6 +4,7 @@ each launch, uninstrumented and instrumented.  Writes gpurun_out/kernel_times.js
 and prints a per-model summary.  Diagnosis tool (no oracle)."""
 import json
 import os
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
 import sys
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))

@@ -6,6 +6,7 @@ decision diagnostics (why decide() passes stopped, average ready / live jobs, Q)
 Diagnosis tool (no oracle)."""
 import json
 import os
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
 import sys
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))

@@ -7,6 +7,7 @@ bursty C-3 mix and its variants (sigma = 1.5, uniform mix).  Writes JSONL rows
 """
 import json
 import os
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
 import sys
 import time
 

@@ -103,6 +103,11 @@ class Graph:
         return self._add("gap", name or f"gap{len(self.nodes)}", [x], (c, 1, 1),
                          prologue=prologue)
 
+    def spin(self, x, us, name=None):
+        """Synthetic kernel of the HoL microbenchmark (Fig. 2, P431-445): one block that
+        stays resident `us` microseconds and copies its input (identity)."""
+        return self._add("spin", name or f"spin{len(self.nodes)}", [x], self.shape(x), us=us)
+
     def fc(self, x, cout, act="none", name=None):
         c, h, w = self.shape(x)
         return self._add("fc", name or f"fc{len(self.nodes)}", [x], (cout, 1, 1),
@@ -166,6 +171,18 @@ def toy():
     x = g.maxpool(x, 2, 2, 0, name="pool1")
     x = g.fc(x, 128, act="relu", name="fc1")
     g.fc(x, 10, act="none", name="fc2")
+    return g
+
+
+def hol_synthetic(n_kernels=8, spin_us=300):
+    """Fig. 2's synthetic job (P431-445): a chain of `n_kernels` kernels, each ONE block
+    of 128 threads resident for `spin_us` us, on a 1x1 input of 8 channels (identity
+    copies), closed by a global average pool over the single pixel (8 outputs)."""
+    g = Graph(f"hol{n_kernels}x{spin_us}", (8, 1, 1), 8)
+    x = g.input
+    for i in range(n_kernels):
+        x = g.spin(x, spin_us, name=f"spin{i}")
+    g.gap(x, name="out")
     return g
 
 

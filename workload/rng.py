@@ -43,7 +43,7 @@ def _gen(*key):
 def raw_params(g: archs.Graph, model_seed: int | None = None):
     """Unscaled float64 parameters {name: array} in canonical layouts."""
     if model_seed is None:
-        model_seed = MODEL_SEED + archs.MODEL_INDEX[g.name]
+        model_seed = MODEL_SEED + archs.MODEL_INDEX.get(g.name, len(archs.MODEL_INDEX))
     shapes = g.param_shapes()
     out = {}
     for n in g.nodes:
@@ -83,7 +83,7 @@ def model_params(g: archs.Graph, scales: dict | None = None):
     ``scales`` maps layer name -> LSUV factor (defaults to the stored table).
     """
     if scales is None:
-        scales = load_scales(g.name)
+        scales = load_scales(g.name) if g.weight_nodes() else {}
     raw = raw_params(g)
     out = {}
     for n in g.weight_nodes():
@@ -98,7 +98,7 @@ def model_params(g: archs.Graph, scales: dict | None = None):
 
 def image(g: archs.Graph, i: int):
     """Input i of the model's pool: fp32 NCHW (1, C, H, W), N(0,1)."""
-    rng = _gen(INPUT_SEED_BASE + i, archs.MODEL_INDEX[g.name])
+    rng = _gen(INPUT_SEED_BASE + i, archs.MODEL_INDEX.get(g.name, len(archs.MODEL_INDEX)))
     return rng.standard_normal((1,) + g.nodes[0]["out"]).astype(np.float32)
 
 
