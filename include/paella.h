@@ -311,6 +311,32 @@ int paella_shutdown(paella_t* p);
 int paella_client_region(paella_t* p, uint32_t client_id, void** base, size_t* bytes);
 /* The shared io region of a client (page-locked, device-mapped on every GPU). */
 
+/* ---- client processes (P1030-1033: "each client obtains a shared memory region when
+   setting up the connection") ---------------------------------------------------------
+   All client channels -- the io regions, the submission / completion rings and the
+   routing state the dispatchers publish -- live in one shared mapping created by
+   paella_init.  Another process of the same user attaches to it by path and then
+   submits and polls exactly as paella_submit / paella_poll_completion do (same code,
+   same semantics and error codes, zero copy: its io buffers are in the mapped region).
+   A client id may be held by one process at a time (the rings are single-producer). */
+typedef struct paella_client_s paella_client_t;
+
+int paella_channel_path(paella_t* p, char* buf, size_t n);
+/* Path of the channel mapping ("/proc/<pid>/fd/<n>"), valid while the instance lives. */
+int paella_client_attach(const char* path, uint32_t client_id, paella_client_t** out);
+/* Map the channels and claim client_id.  -EINVAL bad path / layout / id; -EBUSY the id
+   is attached by another process; -errno of open(2). */
+int paella_client_region_of(paella_client_t* c, void** base, size_t* bytes);
+/* The attached client's io region in this process. */
+int paella_client_model_io(paella_client_t* c, uint32_t model_id, size_t* input_bytes, size_t* output_bytes);
+/* io sizes of a registered model (-EINVAL if not registered). */
+int64_t paella_client_submit(paella_client_t* c, uint32_t model_id, void* io, size_t len, uint32_t flags);
+/* = paella_submit for the attached client id. */
+int64_t paella_client_poll(paella_client_t* c, uint32_t flags, int32_t* status);
+/* = paella_poll_completion for the attached client id. */
+int paella_client_detach(paella_client_t* c);
+/* Release the id and unmap. */
+
 /* ---- introspection (tests, bench) ---------------------------------------- */
 
 typedef struct {

@@ -36,7 +36,9 @@ SYMBOLS = ["paella_init", "paella_register_model", "paella_submit", "paella_subm
            "paella_kernel_info", "paella_kernel_name", "paella_stats", "paella_flush_log",
            "paella_run_isolated", "paella_debug_node", "paella_time_kernels", "paella_bench_empty",
            "paella_bench_roundtrip", "paella_loadgen", "paella_bench_wait", "paella_route_pair",
-           "paella_clock_info", "paella_clock_sync"]
+           "paella_clock_info", "paella_clock_sync", "paella_channel_path", "paella_client_attach",
+           "paella_client_region_of", "paella_client_model_io", "paella_client_submit", "paella_client_poll",
+           "paella_client_detach"]
 
 
 class Config(C.Structure):
@@ -131,6 +133,15 @@ def load():
     lib.paella_clock_info.argtypes = [P, C.c_uint32, C.POINTER(C.c_int64), C.POINTER(C.c_int64),
                                       C.POINTER(C.c_int64)]
     lib.paella_clock_sync.argtypes = [P, C.c_uint32]
+    lib.paella_channel_path.argtypes = [P, C.c_char_p, C.c_size_t]
+    lib.paella_client_attach.argtypes = [C.c_char_p, C.c_uint32, C.POINTER(P)]
+    lib.paella_client_region_of.argtypes = [P, C.POINTER(P), C.POINTER(C.c_size_t)]
+    lib.paella_client_model_io.argtypes = [P, C.c_uint32, C.POINTER(C.c_size_t), C.POINTER(C.c_size_t)]
+    lib.paella_client_submit.argtypes = [P, C.c_uint32, P, C.c_size_t, C.c_uint32]
+    lib.paella_client_submit.restype = C.c_int64
+    lib.paella_client_poll.argtypes = [P, C.c_uint32, C.POINTER(C.c_int32)]
+    lib.paella_client_poll.restype = C.c_int64
+    lib.paella_client_detach.argtypes = [P]
     lib.paella_flush_log.argtypes = [P]
     lib.paella_run_isolated.argtypes = [P, C.c_uint32, C.c_uint32, P, P, C.POINTER(C.c_int64)]
     lib.paella_debug_node.argtypes = [P, C.c_uint32, C.c_uint32, C.c_uint32, C.POINTER(C.c_float)]
@@ -412,6 +423,12 @@ class Engine:
         _check(self.lib.paella_clock_info(self.h, gpu, C.byref(o), C.byref(r), C.byref(q)), "paella_clock_info")
         return o.value, r.value, q.value
 
+    def channel_path(self):
+        """Path another process passes to Client() to attach to this instance."""
+        buf = C.create_string_buffer(256)
+        _check(self.lib.paella_channel_path(self.h, buf, 256), "paella_channel_path")
+        return buf.value.decode()
+
     def clock_sync(self, gpu=0):
         _check(self.lib.paella_clock_sync(self.h, gpu), "paella_clock_sync")
 
@@ -431,6 +448,40 @@ class Engine:
 
     def __exit__(self, *exc):
         self.shutdown()
+
+
+class Client:
+    """A client in ANOTHER process (``paella_client_attach``): the same zero-copy
+    predict / readResult channel as Engine.submit / Engine.poll."""
+
+    def __init__(self, path, client_id):
+        self.lib = load()
+        h = C.c_void_p()
+        _check(self.lib.paella_client_attach(path.encode(), client_id, C.byref(h)), "paella_client_attach")
+        self.h = h
+        base, size = C.c_void_p(), C.c_size_t()
+        _check(self.lib.paella_client_region_of(self.h, C.byref(base), C.byref(size)), "paella_client_region_of")
+        self.base = base.value
+        self.region = np.frombuffer((C.c_uint8 * size.value).from_address(base.value), dtype=np.uint8)
+
+    def model_io(self, model):
+        i, o = C.c_size_t(), C.c_size_t()
+        _check(self.lib.paella_client_model_io(self.h, model, C.byref(i), C.byref(o)), "paella_client_model_io")
+        return i.value, o.value
+
+    def submit(self, model, io_off, length, flags=0):
+        return self.lib.paella_client_submit(self.h, model, self.base + io_off, length, flags)
+
+    def poll(self, flags=NONBLOCK):
+        st = C.c_int32()
+        rid = self.lib.paella_client_poll(self.h, flags, C.byref(st))
+        return rid, st.value
+
+    def close(self):
+        if self.h:
+            self.region = None
+            self.lib.paella_client_detach(self.h)
+            self.h = None
 
 
 EAGAIN = errno.EAGAIN

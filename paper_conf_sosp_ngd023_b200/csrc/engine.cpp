@@ -568,12 +568,7 @@ static void harvest_events(Gpu* g) {
 }
 
 // hybrid completion path: bump the client's futex word; a syscall only if it sleeps
-static void wake_client(Paella* P, uint32_t client) {
-  P->wake_seq[client]->fetch_add(1, std::memory_order_release);
-  if (P->sleepers[client]->load(std::memory_order_acquire) != 0)
-    syscall(SYS_futex, reinterpret_cast<uint32_t*>(P->wake_seq[client]), FUTEX_WAKE_PRIVATE, INT32_MAX, nullptr,
-            nullptr, 0);
-}
+static void wake_client(Paella* P, uint32_t client) { channel_wake(P->ch.hdr, client); }
 
 // Completion to the client's ring; if the ring is full (the client is not polling) the
 // completion waits in a per-client overflow queue, in order, and the dispatcher moves
@@ -889,7 +884,7 @@ static void apply_inbox(Gpu* g) {
 // sending work here (submit_impl checks err).
 static void fail_gpu(Gpu* g, int status, const char* why) {
   fprintf(stderr, "[paella] GPU %u failed (%s): live jobs complete with %d\n", g->index, why, status);
-  g->err.store(status, std::memory_order_release);
+  g->pub->err.store(status, std::memory_order_release);
   for (uint32_t jid = 0; jid < g->jobs.size(); ++jid)
     if (g->jobs[jid].live) finish_job(g, jid, status);
   g->naive_inflight.clear();
@@ -907,7 +902,7 @@ static void dead_loop(Gpu* g) {
       while ((s = g->sub[c]->peek()) != nullptr) {
         push_completion(g, c, s->req_id, -EIO);
         g->sub[c]->pop();
-        g->popped.fetch_add(1, std::memory_order_release);
+        g->pub->popped.fetch_add(1, std::memory_order_release);
       }
     }
     flush_overflow(g);
@@ -962,13 +957,13 @@ static void dispatch_loop(Gpu* g) {
           }
           if (!admit(g, c, *s)) break;
           q->pop();
-          g->popped.fetch_add(1, std::memory_order_release);
+          g->pub->popped.fetch_add(1, std::memory_order_release);
           nev++;
           served = true;
         }
         if (served) g->rr_start = (c + 1) % N;
       }
-      g->admitted_pub.store(g->stats.admitted, std::memory_order_release);
+      g->pub->admitted.store(g->stats.admitted, std::memory_order_release);
     }
     if (P->cfg.naive) {
       bool progressed = false;
@@ -1014,7 +1009,7 @@ static void dispatch_loop(Gpu* g) {
     if (nev) {
       logev(g, EV_BATCH_END, 0, 0, 0, 0);
       decide_and_launch(g);
-      g->work_published.store(g->policy->outstanding_work(), std::memory_order_release);
+      g->pub->work.store(g->policy->outstanding_work(), std::memory_order_release);
       busy_ticks += ticks() - it0;
     }
     int e = g->be->error();
@@ -1061,7 +1056,7 @@ static void dispatcher_main(Gpu* g) {
   } catch (const std::exception& ex) {
     fail_gpu(g, -EIO, ex.what());
   }
-  if (g->err.load(std::memory_order_acquire)) dead_loop(g);
+  if (g->pub->err.load(std::memory_order_acquire)) dead_loop(g);
 }
 
 // globaltimer -> host clock calibration: n ping-pongs with
@@ -1116,12 +1111,29 @@ static int clock_sync(Gpu* g, uint32_t n, int64_t* off, int64_t* rtt, int64_t* r
 // ---------------------------------------------------------------------------
 // shared memory helpers
 // ---------------------------------------------------------------------------
-static void* shm_alloc(Paella* P, size_t bytes) {
-  void* p = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_SHARED | MAP_ANONYMOUS, -1, 0);
-  if (p == MAP_FAILED) return nullptr;
-  P->shm_maps.push_back(p);
-  P->shm_sizes.push_back(bytes);
-  return p;
+// The client channels (channel.h) in one memfd mapping: other processes attach to it
+// through /proc/<pid>/fd/<fd> (paella_channel_path / paella_client_attach).
+static int channel_create(Paella* P) {
+  const paella_config_t& cfg = P->cfg;
+  ShmHeader layout{};
+  const size_t total = channel_layout(&layout, cfg.num_clients, cfg.num_gpus, cfg.submit_slots, P->region_bytes);
+  const int fd = (int)syscall(SYS_memfd_create, "paella-channels", 0u);
+  if (fd < 0) return -errno;
+  if (ftruncate(fd, (off_t)total) != 0) {
+    close(fd);
+    return -ENOMEM;
+  }
+  void* p = mmap(nullptr, total, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+  if (p == MAP_FAILED) {
+    close(fd);
+    return -ENOMEM;
+  }
+  P->shm_fd = fd;
+  P->shm_bytes = total;
+  P->ch.hdr = (ShmHeader*)p;
+  P->ch.base = (uint8_t*)p;
+  channel_init(P->ch, layout, cfg.route);
+  return 0;
 }
 
 static uint32_t ilog2(uint32_t x) {
@@ -1198,24 +1210,20 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
   if (cfg.slack_blocks == 0) P->cfg.slack_blocks = P->sms;
   P->models.resize(256);
 
-  // client regions (shared, page-locked and mapped into every GPU)
+  // client channels: regions (page-locked and mapped into every GPU) and rings in one
+  // shared mapping (P1030-1033: each client's shared memory region)
   P->region_bytes = cfg.client_region_bytes;
+  if (int rc = channel_create(P.get())) return rc;
   for (uint32_t c = 0; c < cfg.num_clients; ++c) {
-    void* r = shm_alloc(P.get(), P->region_bytes);
-    if (!r) return -ENOMEM;
+    uint8_t* r = P->ch.region(c);
     if (cfg.device == PAELLA_DEVICE_CUDA) {
       cudaSetDevice(cfg.first_gpu);
       if (cudaHostRegister(r, P->region_bytes, cudaHostRegisterPortable | cudaHostRegisterMapped) != cudaSuccess)
         return -ENOMEM;
     }
-    P->region.push_back((uint8_t*)r);
-    P->client_seq.push_back(new std::atomic<uint64_t>(0));
-    P->wake_seq.push_back(new std::atomic<uint32_t>(0));
-    P->sleepers.push_back(new std::atomic<uint32_t>(0));
+    P->region.push_back(r);
   }
-  P->rr_next.assign(cfg.num_clients, 0);
   P->route_log.resize(cfg.num_clients);
-  P->poll_rr.assign(cfg.num_clients, 0);
 
   // NUMA placement: a GPU's pinned notification ring and counter
   // mirror are first touched by a thread running on that GPU's dispatcher core, so
@@ -1288,14 +1296,10 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
       for (int r = 0; r < NRES; ++r) pc.capacity[r] -= proxy[r];
     }
     g->policy.reset(new Policy(pc));
+    g->pub = &P->ch.hdr->gpu[gi];
     for (uint32_t c = 0; c < cfg.num_clients; ++c) {
-      auto* s = (SpscRing<SubmitSlot>*)shm_alloc(P.get(), SpscRing<SubmitSlot>::bytes(cfg.submit_slots));
-      auto* d = (SpscRing<CompleteSlot>*)shm_alloc(P.get(), SpscRing<CompleteSlot>::bytes(cfg.submit_slots));
-      if (!s || !d) return -ENOMEM;
-      s->init(cfg.submit_slots);
-      d->init(cfg.submit_slots);
-      g->sub.push_back(s);
-      g->done.push_back(d);
+      g->sub.push_back(P->ch.sub(gi, c));
+      g->done.push_back(P->ch.done(gi, c));
     }
     if (cfg.event_log_path) {
       char path[4096];
@@ -1395,7 +1399,13 @@ int paella_register_model(paella_t* p, const paella_model_desc_t* desc, uint32_t
       std::this_thread::yield();
     }
   (void)mp;
+  if (nm >= SHM_MAX_MODELS) return -ENOMEM;
+  ModelPub& pubm = P->ch.hdr->models[nm];   // io sizes and T-bar for every client process
+  pubm.input_bytes = mp->input_bytes;
+  pubm.output_bytes = mp->output_bytes;
+  pubm.total_tbar = mp->total_tbar;
   P->nmodels.store(nm + 1, std::memory_order_release);
+  P->ch.hdr->nmodels.store(nm + 1, std::memory_order_release);
   if (model_id) *model_id = nm;
   return 0;
 }
@@ -1418,96 +1428,9 @@ int paella_route_pair(uint64_t req_id, uint32_t num_gpus, uint32_t* g0, uint32_t
 static int64_t submit_impl(Paella* P, uint32_t client_id, uint32_t model_id, void* io, size_t len, uint32_t flags,
                            int64_t t_sched) {
   if (!P) return -EINVAL;
-  if (P->shutting.load()) return -ESHUTDOWN;
   if (client_id >= P->cfg.num_clients) return -EINVAL;
-  if (model_id >= P->nmodels.load(std::memory_order_acquire)) return -EINVAL;
-  Model* m = P->models[model_id].get();
-  uint8_t* base = P->region[client_id];
-  uint8_t* b = (uint8_t*)io;
-  if (b < base || b + len > base + P->region_bytes || b + len < b) return -EFAULT;
-  if (len < m->input_bytes + m->output_bytes) return -EINVAL;
-  if (((uintptr_t)io & 15) != 0) return -EINVAL;
-  uint64_t seq = P->client_seq[client_id]->fetch_add(1);
-  uint64_t req_id = ((uint64_t)client_id << 48) | (seq & ((1ull << 48) - 1));
-  // route: least outstanding work W_g, ties to the lowest index;
-  // W_g = published sum of R_j + unadmitted submissions x the model's whole-job T-bar.
-  // A failed GPU (err != 0) is never chosen; -EIO once none is left.
-  uint32_t gsel = 0;
-  uint32_t ng = (uint32_t)P->gpus.size();
-  SubmitSlot s{};
-  if (ng > 1) {
-    int64_t work[PAELLA_MAX_GPUS] = {0}, pend[PAELLA_MAX_GPUS] = {0}, W[PAELLA_MAX_GPUS] = {0};
-    uint32_t alive = 0;
-    for (uint32_t g = 0; g < ng; ++g) {
-      Gpu* Gg = P->gpus[g].get();
-      if (Gg->err.load(std::memory_order_acquire) == 0) alive |= 1u << g;
-      // pending before work: an admission moves a job from the first to the second
-      pend[g] = (int64_t)(Gg->submitted.load(std::memory_order_relaxed) - Gg->admitted_pub.load(std::memory_order_acquire));
-      work[g] = Gg->work_published.load(std::memory_order_acquire);
-      W[g] = work[g] + pend[g] * m->total_tbar;
-    }
-    if (!alive) return -EIO;
-    auto least = [&]() {
-      uint32_t best = ng;
-      for (uint32_t g = 0; g < ng; ++g)
-        if ((alive >> g & 1) && (best == ng || W[g] < W[best])) best = g;
-      return best;
-    };
-    uint32_t g0 = 0, g1 = 0;
-    if (P->cfg.route == PAELLA_ROUTE_ROUND_ROBIN) {
-      // the client's next GPU in cyclic order, skipping failed ones
-      uint32_t k = 0;
-      do {
-        gsel = P->rr_next[client_id]++ % ng;
-      } while (!(alive >> gsel & 1) && ++k < ng);
-      g0 = g1 = gsel;
-    } else if (P->cfg.route == PAELLA_ROUTE_POWER_OF_TWO) {
-      paella_route_pair(req_id, ng, &g0, &g1);
-      const uint32_t lo = g0 < g1 ? g0 : g1, hi = g0 < g1 ? g1 : g0;
-      if ((alive >> lo & 1) && (alive >> hi & 1)) gsel = W[hi] < W[lo] ? hi : lo;
-      else if (alive >> lo & 1) gsel = lo;
-      else if (alive >> hi & 1) gsel = hi;
-      else gsel = least();
-    } else {
-      gsel = g0 = g1 = least();
-    }
-    s.route_w[0] = W[g0];
-    s.route_w[1] = W[g1];
-    s.route_meta = g0 | (g1 << 8) | (P->cfg.route << 16);
-    if (P->cfg.route_log_path) {
-      paella_route_rec_t rr{};
-      rr.req_id = req_id;
-      rr.route = P->cfg.route;
-      rr.chosen = gsel;
-      rr.g0 = g0;
-      rr.g1 = g1;
-      rr.num_gpus = ng;
-      rr.model = model_id;
-      rr.alive = alive;
-      rr.tbar_model = m->total_tbar;
-      for (uint32_t g = 0; g < ng; ++g) {
-        rr.work[g] = work[g];
-        rr.pending[g] = pend[g];
-      }
-      P->route_log[client_id].push_back(rr);
-    }
-  } else if (P->gpus[0]->err.load(std::memory_order_acquire)) {
-    return -EIO;
-  }
-  Gpu* G = P->gpus[gsel].get();
-  s.req_id = req_id;
-  s.model_id = model_id;
-  s.flags = flags;
-  s.io_off = (uint64_t)(b - base);
-  s.len = len;
-  s.t_sched_ns = t_sched;
-  for (;;) {
-    if (G->sub[client_id]->push(s)) break;
-    if (flags & PAELLA_NONBLOCK) return -EAGAIN;
-    if (P->shutting.load()) return -ESHUTDOWN;
-  }
-  G->submitted.fetch_add(1, std::memory_order_relaxed);
-  return (int64_t)s.req_id;
+  return channel_submit(P->ch, client_id, model_id, io, len, flags, t_sched,
+                        P->cfg.route_log_path && P->gpus.size() > 1 ? &P->route_log[client_id] : nullptr);
 }
 
 int64_t paella_submit(paella_t* p, uint32_t client_id, uint32_t model_id, void* io, size_t len, uint32_t flags) {
@@ -1522,53 +1445,14 @@ int64_t paella_submit_at(paella_t* p, uint32_t client_id, uint32_t model_id, voi
 int64_t paella_poll_completion(paella_t* p, uint32_t client_id, uint32_t flags, int32_t* status) {
   Paella* P = (Paella*)p;
   if (!P || client_id >= P->cfg.num_clients) return -EINVAL;
-  uint32_t ng = (uint32_t)P->gpus.size();
-  int64_t spin_start = 0;
-  for (;;) {
-    for (uint32_t k = 0; k < ng; ++k) {
-      uint32_t g = (P->poll_rr[client_id] + k) % ng;
-      SpscRing<CompleteSlot>* q = P->gpus[g]->done[client_id];
-      const CompleteSlot* c = q->peek();
-      if (c) {
-        int64_t id = (int64_t)c->req_id;
-        if (status) *status = c->status;
-        q->pop();
-        P->poll_rr[client_id] = (g + 1) % ng;
-        return id;
-      }
-    }
-    // every GPU failed and every submission has been answered: nothing will come
-    bool all_dead = true;
-    for (auto& g : P->gpus)
-      all_dead &= g->err.load(std::memory_order_acquire) != 0 &&
-                  g->popped.load(std::memory_order_acquire) >= g->submitted.load(std::memory_order_acquire);
-    if (all_dead) {
-      bool empty = true;   // re-check: a completion may have landed since the scan
-      for (uint32_t k = 0; k < ng && empty; ++k) empty = P->gpus[k]->done[client_id]->peek() == nullptr;
-      if (empty) return -EIO;
-      continue;
-    }
-    if (flags & PAELLA_NONBLOCK) return -EAGAIN;
-    bool alive = false;
-    for (auto& g : P->gpus) alive |= g->thread.joinable() && !g->stop.load();
-    if (!alive) return -ESHUTDOWN;
-    if (flags & PAELLA_HYBRID) {
-      // spin ~20 us after the last wake-up, then sleep until the next hint/completion
-      const uint32_t seen = P->wake_seq[client_id]->load(std::memory_order_acquire);
-      if (spin_start == 0) spin_start = now_ns();
-      if (now_ns() - spin_start < 20000) continue;
-      P->sleepers[client_id]->fetch_add(1, std::memory_order_acq_rel);
-      bool empty = true;   // re-check after announcing the sleep (no lost wake-up)
-      for (uint32_t k = 0; k < ng && empty; ++k) empty = P->gpus[k]->done[client_id]->peek() == nullptr;
-      if (empty && P->wake_seq[client_id]->load(std::memory_order_acquire) == seen) {
-        timespec ts{0, 2000000};   // 2 ms cap: shutdown and error paths need no wake-up
-        syscall(SYS_futex, reinterpret_cast<uint32_t*>(P->wake_seq[client_id]), FUTEX_WAIT_PRIVATE, seen, &ts,
-                nullptr, 0);
-      }
-      P->sleepers[client_id]->fetch_sub(1, std::memory_order_acq_rel);
-      spin_start = now_ns();
-    }
-  }
+  return channel_poll(P->ch, client_id, flags, status);
+}
+
+int paella_channel_path(paella_t* p, char* buf, size_t n) {
+  Paella* P = (Paella*)p;
+  if (!P || !buf || n == 0 || P->shm_fd < 0) return -EINVAL;
+  const int k = snprintf(buf, n, "/proc/%d/fd/%d", (int)getpid(), P->shm_fd);
+  return k > 0 && (size_t)k < n ? 0 : -ENAMETOOLONG;
 }
 
 // routing log of every client (cfg.route_log_path), rewritten in full
@@ -1589,7 +1473,7 @@ static int write_route_logs(Paella* P) {
 int paella_shutdown(paella_t* p) {
   Paella* P = (Paella*)p;
   if (!P) return -EINVAL;
-  P->shutting.store(true);
+  P->ch.hdr->shutting.store(1, std::memory_order_release);
   for (auto& g : P->gpus) g->stop.store(true, std::memory_order_release);
   for (auto& g : P->gpus)
     if (g->thread.joinable()) g->thread.join();
@@ -1641,10 +1525,8 @@ int paella_shutdown(paella_t* p) {
   if (P->cfg.device == PAELLA_DEVICE_CUDA)
     for (auto* r : P->region) cudaHostUnregister(r);
   P->gpus.clear();
-  for (size_t i = 0; i < P->shm_maps.size(); ++i) munmap(P->shm_maps[i], P->shm_sizes[i]);
-  for (auto* a : P->client_seq) delete a;
-  for (auto* a : P->wake_seq) delete a;
-  for (auto* a : P->sleepers) delete a;
+  munmap(P->ch.base, P->shm_bytes);
+  if (P->shm_fd >= 0) close(P->shm_fd);
   delete P;
   return 0;
 }
@@ -1737,7 +1619,7 @@ int paella_stats(paella_t* p, uint32_t gpu, paella_stats_t* st) {
   Paella* P = (Paella*)p;
   if (!P || !st || gpu >= P->gpus.size()) return -EINVAL;
   *st = P->gpus[gpu]->stats;   // racy snapshot of counters, fine for reporting
-  st->outstanding_work_ns = P->gpus[gpu]->work_published.load();
+  st->outstanding_work_ns = P->gpus[gpu]->pub->work.load();
   return 0;
 }
 

@@ -11,6 +11,7 @@
 #include <vector>
 
 #include "../../include/paella.h"
+#include "channel.h"
 #include "common.h"
 #include "kernels.h"
 #include "policy.h"
@@ -190,16 +191,14 @@ struct Gpu {
   std::vector<JobRec> jobs;         // indexed by job id (dense)
   std::vector<uint32_t> free_job_ids;
   uint32_t next_job = 0;
-  std::vector<SpscRing<SubmitSlot>*> sub;     // per client
+  std::vector<SpscRing<SubmitSlot>*> sub;     // per client (in the shared channel mapping)
   std::vector<SpscRing<CompleteSlot>*> done;  // per client
   std::thread thread;
   std::atomic<bool> stop{false};
-  std::atomic<int64_t> work_published{0};
-  std::atomic<uint64_t> admitted_pub{0};
-  std::atomic<uint64_t> submitted{0};
-  std::atomic<int> err{0};          // != 0: this GPU failed (-EIO) or hung (-ETIMEDOUT); it only
-                                    // completes submissions with -EIO from then on (dead mode)
-  std::atomic<uint64_t> popped{0};  // submissions taken out of this GPU's rings (any outcome)
+  // published in the shared channel header for every client process: W_g, admissions,
+  // submissions, pops, and err (!= 0: this GPU failed (-EIO) or hung (-ETIMEDOUT); it
+  // only completes submissions with -EIO from then on: dead mode)
+  GpuPub* pub = nullptr;
   // completions the client's ring could not take yet (never blocks the dispatcher)
   std::vector<std::deque<CompleteSlot>> overflow;
   int64_t last_progress_ns = 0;     // watchdog: last time a record was consumed (or nothing was due)
@@ -255,19 +254,13 @@ struct Paella {
   std::vector<std::unique_ptr<Model>> models;   // capacity reserved; published via nmodels
   std::atomic<uint32_t> nmodels{0};
   std::mutex reg_mu;
-  std::vector<uint8_t*> region;                 // client io regions
+  // the client channels (channel.h): one shared memfd mapping holding the header
+  // (routing state, model io sizes, per-client words), the io regions and the rings
+  Channel ch;
+  int shm_fd = -1;
+  size_t shm_bytes = 0;
+  std::vector<uint8_t*> region;                 // client io regions (into ch)
   size_t region_bytes = 0;
-  std::vector<void*> shm_maps;
-  std::vector<size_t> shm_sizes;
-  std::vector<std::atomic<uint64_t>*> client_seq;
-  std::vector<uint32_t> rr_next;                // per-client round-robin router state
-  std::vector<uint32_t> poll_rr;                // per-client completion ring scan start
-  // hybrid completion wait (PAELLA_HYBRID, P1157-1171): per-client futex word bumped by
-  // the dispatchers on the "almost finished" hint and on every completion, and the
-  // number of client threads sleeping on it (no syscall on the dispatcher otherwise)
-  std::vector<std::atomic<uint32_t>*> wake_seq;
-  std::vector<std::atomic<uint32_t>*> sleepers;
-  std::atomic<bool> shutting{false};
   int64_t capacity[NRES];
   // routing log (multi-GPU, cfg.route_log_path): every decision with the full W_g
   // snapshot it was taken on, one vector per client (written by that client's thread)
