@@ -513,6 +513,9 @@ def run_gpu(args, ngpus, cores, fake):
                         "d2h": float(np.mean([specs[m][0].num_classes * 4 for m in mm])), "n": len(mm)}
             r["x_sat"] = saturation(a, cfg, len(names), 3000 if not fake else 200, lam / args.rho,
                                     iters=4 if not fake else 1)
+            if not fake and ngpus == 1:
+                # X_dev: the same mix as CUDA graphs on 32 streams at overload, no dispatcher
+                r["x_dev"] = a.e.bench_xdev(a.mids, steps[0][1], streams=32)
             if not args.no_slo and not fake:
                 r["slo"] = slo_search(a, cfg, names, ngpus * x_sat1, slo, args.slo_reqs * ngpus, seed0 + 700)
             if not args.no_c5 and not fake and ngpus == 1:
@@ -759,6 +762,8 @@ def main():
         "naive_jct_us": [round(nv["mean_us"]), round(nv["p99_us"])] if nv else None,
         "naive_pdl_jct_us": [round(npd["mean_us"]), round(npd["p99_us"])] if npd else None,
         "req_s_at_slo": {k: v["slo"]["req_s"] for k, v in res.items() if "slo" in v},
+        "x_sat_req_s": {"paella": round(P.get("x_sat", 0), 1), "naive": detail["x_sat_naive_1gpu"],
+                        "x_dev": round(P.get("x_dev", 0), 1)},
         "served_req_s": round(served, 1),
         "n_gpus": ngpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(max_el * 1e3 / args.steps, 2),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",

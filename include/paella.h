@@ -413,6 +413,14 @@ int paella_run_isolated(paella_t* p, uint32_t gpu, uint32_t model_id, const void
 int paella_time_kernels(paella_t* p, uint32_t gpu, uint32_t model_id, uint32_t instrumented,
                         uint32_t reps, int64_t* kernel_ns);
 
+/* X_dev, the device-only saturation throughput: request i runs model
+   models[seq[i]] as a CUDA graph of its uninstrumented kernel chain on stream i % streams
+   (workspace slot = stream; needs max_jobs_per_model >= streams and no serving in
+   progress); all n requests are enqueued at once and *req_per_s = n / device time.  No
+   dispatcher, no notifications: the bound the served throughput is compared with. */
+int paella_bench_xdev(paella_t* p, uint32_t gpu, const uint32_t* models, uint32_t n_models, const uint32_t* seq,
+                      uint32_t n, uint32_t streams, double* req_per_s);
+
 /* Notification microbenchmarks (config 5, P1881-1897 Fig. 15).
    paella_bench_empty: `iters` launches of an empty kernel with `grid` x `block`
    threads, back to back behind a gate; *ns_per_launch = elapsed / iters.

@@ -38,7 +38,7 @@ SYMBOLS = ["paella_init", "paella_register_model", "paella_submit", "paella_subm
            "paella_bench_roundtrip", "paella_loadgen", "paella_bench_wait", "paella_route_pair",
            "paella_clock_info", "paella_clock_sync", "paella_channel_path", "paella_client_attach",
            "paella_client_region_of", "paella_client_model_io", "paella_client_submit", "paella_client_poll",
-           "paella_client_detach"]
+           "paella_client_detach", "paella_bench_xdev"]
 
 
 class Config(C.Structure):
@@ -134,6 +134,8 @@ def load():
                                       C.POINTER(C.c_int64)]
     lib.paella_clock_sync.argtypes = [P, C.c_uint32]
     lib.paella_channel_path.argtypes = [P, C.c_char_p, C.c_size_t]
+    lib.paella_bench_xdev.argtypes = [P, C.c_uint32, C.POINTER(C.c_uint32), C.c_uint32, C.POINTER(C.c_uint32),
+                                      C.c_uint32, C.c_uint32, C.POINTER(C.c_double)]
     lib.paella_client_attach.argtypes = [C.c_char_p, C.c_uint32, C.POINTER(P)]
     lib.paella_client_region_of.argtypes = [P, C.POINTER(P), C.POINTER(C.c_size_t)]
     lib.paella_client_model_io.argtypes = [P, C.c_uint32, C.POINTER(C.c_size_t), C.POINTER(C.c_size_t)]
@@ -372,6 +374,15 @@ class Engine:
         _check(self.lib.paella_bench_roundtrip(self.h, gpu, n, a.ctypes.data_as(C.POINTER(C.c_int64)),
                                                b.ctypes.data_as(C.POINTER(C.c_int64))), "paella_bench_roundtrip")
         return a, b
+
+    def bench_xdev(self, models, seq, streams=32, gpu=0):
+        """X_dev: device-only saturation req/s of the mix (paella_bench_xdev)."""
+        ms = (C.c_uint32 * len(models))(*models)
+        sq = (C.c_uint32 * len(seq))(*[int(x) for x in seq])
+        v = C.c_double()
+        _check(self.lib.paella_bench_xdev(self.h, gpu, ms, len(models), sq, len(seq), streams, C.byref(v)),
+               "paella_bench_xdev")
+        return v.value
 
     def bench_wait(self, client, model, n, gap_ns, poll_flags, stride, slots):
         """NEXT-3 measurement: (jct_ns array, waiter CPU fraction); see paella_bench_wait."""

@@ -2073,6 +2073,87 @@ static InstrArgs iso_instr(Gpu* g, uint32_t grid, uint32_t group, bool last) {
 
 extern "C" {
 
+// X_dev (SURVEY.md 8(d) "Throughput"): device-only saturation of a request mix, no
+// dispatcher.  One CUDA graph per (model, stream) holds the model's uninstrumented
+// kernel chain (PDL edges, as served) on workspace slot = stream; the requests of `seq`
+// are replayed as graph launches round-robin over `streams` streams, all enqueued at
+// once (overload); rate = requests / elapsed (CUDA events).
+int paella_bench_xdev(paella_t* p, uint32_t gpu, const uint32_t* models, uint32_t n_models, const uint32_t* seq,
+                      uint32_t n, uint32_t streams, double* req_per_s) {
+  Paella* P = (Paella*)p;
+  if (!P || gpu >= P->gpus.size() || !models || !seq || !req_per_s || n == 0 || streams == 0 || streams > 64)
+    return -EINVAL;
+  if (P->cfg.device != PAELLA_DEVICE_CUDA) return -ENODEV;
+  Gpu* g = P->gpus[gpu].get();
+  std::lock_guard<std::mutex> lk(g->iso_mu);
+  int rc = ensure_iso(g);
+  if (rc) return rc;
+  for (uint32_t i = 0; i < n_models; ++i)
+    if (models[i] >= P->nmodels.load() || P->cfg.max_jobs_per_model < streams) return -EINVAL;
+  for (uint32_t i = 0; i < n; ++i)
+    if (seq[i] >= n_models) return -EINVAL;
+  cudaSetDevice(g->device);
+  auto* cb = static_cast<CudaBackend*>(g->be.get());
+  std::vector<cudaStream_t> ss(streams);
+  for (auto& s : ss) cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
+  std::vector<cudaGraphExec_t> ex((size_t)n_models * streams, nullptr);
+  uint8_t* st = (uint8_t*)g->stage_in;   // every request reads the same staged input
+  std::memset(st, 0, 2 << 20);
+  for (uint32_t mi = 0; mi < n_models && rc == 0; ++mi) {
+    Model* m = P->models[models[mi]].get();
+    ModelGpu& mg = m->gpu[gpu];
+    for (uint32_t s = 0; s < streams && rc == 0; ++s) {
+      std::vector<LayerArgs> A = mg.args[s];          // slot s, private copy of the parameters
+      A.front().in = st;
+      A.back().out = st + (8 << 20);   // past the largest input
+      cudaGraph_t graph;
+      if (cudaStreamBeginCapture(ss[s], cudaStreamCaptureModeThreadLocal) != cudaSuccess) rc = -EIO;
+      for (uint32_t l = 0; l < m->kernels.size() && rc == 0; ++l) {
+        const KernelInst& k = m->kernels[l];
+        InstrArgs ia{};
+        const void* tm = is_tc(k.kind) ? mg.tmaps[l].b : nullptr;
+        void* args[3] = {(void*)&A[l], (void*)&ia, (void*)tm};
+        if (cuda_launch(cb->fn(k.kind, m->dtype, false), k, args, ss[s], true) != cudaSuccess) rc = -EIO;
+      }
+      if (cudaStreamEndCapture(ss[s], &graph) != cudaSuccess) rc = -EIO;
+      if (rc == 0 && cudaGraphInstantiate(&ex[(size_t)mi * streams + s], graph, 0) != cudaSuccess) rc = -EIO;
+      if (rc == 0) cudaGraphDestroy(graph);
+    }
+  }
+  if (rc == 0) {
+    // warm every graph once, then the timed overload
+    for (size_t i = 0; i < ex.size(); ++i) cudaGraphLaunch(ex[i], ss[i % streams]);
+    for (auto& s : ss) cudaStreamSynchronize(s);
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    cudaEventRecord(e0, ss[0]);
+    for (uint32_t s = 1; s < streams; ++s) cudaStreamWaitEvent(ss[s], e0, 0);
+    for (uint32_t i = 0; i < n; ++i) {
+      const uint32_t s = i % streams;
+      cudaGraphLaunch(ex[(size_t)seq[i] * streams + s], ss[s]);
+    }
+    std::vector<cudaEvent_t> done(streams);
+    for (uint32_t s = 0; s < streams; ++s) {
+      cudaEventCreateWithFlags(&done[s], cudaEventDisableTiming);
+      cudaEventRecord(done[s], ss[s]);
+      cudaStreamWaitEvent(ss[0], done[s], 0);
+    }
+    cudaEventRecord(e1, ss[0]);
+    if (cudaEventSynchronize(e1) != cudaSuccess) rc = -EIO;
+    float ms = 0;
+    cudaEventElapsedTime(&ms, e0, e1);
+    *req_per_s = n / (ms * 1e-3);
+    for (auto& e : done) cudaEventDestroy(e);
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+  }
+  for (auto& x : ex)
+    if (x) cudaGraphExecDestroy(x);
+  for (auto& s : ss) cudaStreamDestroy(s);
+  return rc;
+}
+
 int paella_time_kernels(paella_t* p, uint32_t gpu, uint32_t model_id, uint32_t instrumented, uint32_t reps,
                         int64_t* kernel_ns) {
   Paella* P = (Paella*)p;

@@ -522,3 +522,18 @@ def test_hol_spin_kernels(engine):
         out, kt = engine.run_isolated(mid, x, timing=True)
         assert np.array_equal(out, round_bf16(x).reshape(-1)), (out, x)
         assert all(t >= 20_000 for t in kt[1:9]), kt
+
+
+def test_bench_xdev_graph_replay():
+    """X_dev: each model's uninstrumented chain captured as a CUDA graph
+    (PDL edges) per stream and replayed at overload; the device-only rate of a 2-model
+    mix exceeds what one stream achieves (concurrency pays) and is finite."""
+    with L.Engine(num_clients=1, max_jobs_per_model=32) as e:
+        mids = []
+        for nm in ("resnet18", "squeezenet1_1"):
+            g = archs.build(nm)
+            mids.append(e.register_model(g, rng.model_params(g)))
+        seq = np.arange(400) % 2
+        r32 = e.bench_xdev(mids, seq, streams=32)
+        r1 = e.bench_xdev(mids, seq, streams=1)
+    assert 0 < r1 < r32 < 1e6, (r1, r32)
