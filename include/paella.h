@@ -366,9 +366,10 @@ typedef struct {
   uint64_t loop_iters;
   int64_t  outstanding_work_ns;   /* W_g published for the router */
   uint64_t ev_launches, ev_ns, ev_bytes, ev_flops;   /* event-timed launches (event_time_kind) */
-  uint64_t stop_reason[4];     /* decide() passes that stopped with ready work left behind:
-                                  [0] none (all ready work issued), [1] no free stream,
-                                  [2] occupancy predicate (fits), [3] ring flow control */
+  uint64_t stop_reason[5];     /* why each decide() pass stopped: [0] no ready work left,
+                                  [1] no free stream, [2] occupancy predicate (fits),
+                                  [3] ring flow control, [4] ready jobs exist but all are
+                                  outside the job cap K (B200-Q6) */
   uint64_t sum_ready, sum_live_jobs, sum_Q;   /* summed over decide() passes (averages) */
   uint64_t rel_events;         /* counter mode: stream-release events recorded (a job left idle) */
   uint64_t xstream_waits;      /* ... of which the job's next kernel went to another stream

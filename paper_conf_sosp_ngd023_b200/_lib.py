@@ -96,7 +96,7 @@ class Stats(C.Structure):
                 ("records", C.c_uint64), ("torn_retries", C.c_uint64), ("decide_calls", C.c_uint64),
                 ("loop_iters", C.c_uint64), ("outstanding_work_ns", C.c_int64), ("ev_launches", C.c_uint64),
                 ("ev_ns", C.c_uint64), ("ev_bytes", C.c_uint64), ("ev_flops", C.c_uint64),
-                ("stop_reason", C.c_uint64 * 4), ("sum_ready", C.c_uint64), ("sum_live_jobs", C.c_uint64),
+                ("stop_reason", C.c_uint64 * 5), ("sum_ready", C.c_uint64), ("sum_live_jobs", C.c_uint64),
                 ("sum_Q", C.c_uint64), ("rel_events", C.c_uint64), ("xstream_waits", C.c_uint64),
                 ("busy_ns", C.c_uint64)]
 

@@ -318,7 +318,7 @@ void Policy::decide(std::vector<Issue>* out) {
   for (;;) {
     uint32_t jid;
     if (!pick(&jid)) {
-      last_stop_ = 0;
+      last_stop_ = srpt_.empty() ? 0 : 4;   // 4: ready jobs, all outside the job cap
       break;
     }
     PolicyJob& j = jobs_[jid];

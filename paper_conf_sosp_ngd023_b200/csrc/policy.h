@@ -118,7 +118,8 @@ class Policy {
   const PolicyLaunch& launch(uint32_t uid) const { return launches_[uid % kLaunchSlots]; }
   int64_t deficit(uint32_t c) const { return Dt_[c] + Omega_; }
   int64_t Q() const { return Q_; }
-  // why the last decide() stopped: 0 nothing ready, 1 no free stream, 2 fits, 3 ring
+  // why the last decide() stopped: 0 nothing ready, 1 no free stream, 2 fits, 3 ring,
+  // 4 ready jobs all outside the job cap
   int last_stop() const { return last_stop_; }
   size_t ready_count() const { return srpt_.size(); }
   int64_t O() const { return O_; }
