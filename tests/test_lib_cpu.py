@@ -394,3 +394,29 @@ def test_hol_synthetic_model_plans_and_serves():
         assert [k["name"] for k in ks] == ["ingest"] + ["spin"] * 8 + ["gap"]
         assert all(k["grid"] == 1 and k["block"] == 128 for k in ks[1:9])
         _serve(e, [mid], 40, 1, seed=2, stride=256)
+
+
+def test_struct_layout_matches_header(tmp_path):
+    """The ctypes mirrors of paella_config_t / paella_stats_t / paella_kernel_info_t /
+    paella_route_rec_t have exactly the C layout of include/paella.h (sizes and every
+    field offset, compiled with gcc here): marshalling cannot silently shift a field."""
+    import ctypes as C
+    checks = [("paella_config_t", L.Config), ("paella_stats_t", L.Stats), ("paella_kernel_info_t", L.KernelInfo),
+              ("paella_model_info_t", L.ModelInfo), ("paella_req_t", L.Req), ("paella_node_t", L.Node),
+              ("paella_model_desc_t", L.ModelDesc)]
+    lines = ['#include <stdio.h>', '#include <stddef.h>', '#include "paella.h"', "int main(void){"]
+    for cname, py in checks:
+        lines.append(f'printf("{cname} %zu\\n", sizeof({cname}));')
+        for f, _ in py._fields_:
+            lines.append(f'printf("{cname}.{f} %zu\\n", offsetof({cname}, {f}));')
+    lines.append("return 0;}")
+    src = tmp_path / "layout.c"
+    src.write_text("\n".join(lines))
+    exe = tmp_path / "layout"
+    subprocess.run(["gcc", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)], check=True)
+    out = dict(l.rsplit(" ", 1) for l in subprocess.run([str(exe)], capture_output=True, text=True,
+                                                         check=True).stdout.splitlines())
+    for cname, py in checks:
+        assert int(out[cname]) == C.sizeof(py), cname
+        for f, _ in py._fields_:
+            assert int(out[f"{cname}.{f}"]) == getattr(py, f).offset, (cname, f)
