@@ -533,6 +533,8 @@ def c5_micro(e):
     instrumented (counter mode, as served) vs plain, at grids 16/148/160/1184/4736; ring
     round trip of a 1-block kernel (launch -> PLACEMENT / COMPLETION visible to the host)."""
     out = {"empty_us": {}}
+    e.bench_empty(16, 128, True, 16, 200)     # warm the isolated-run path
+    e.bench_empty(16, 128, False, 16, 200)
     for grid in (16, 148, 160, 1184, 4736):
         a = e.bench_empty(grid, 128, True, 16, 1000)
         b = e.bench_empty(grid, 128, False, 16, 1000)
@@ -633,7 +635,7 @@ def cpu_baseline(cfg, seconds=20.0, reserve=0):
             "host": hi}
 
 
-def simulator_timing(kinfo, cfg, names, lam, n=300):
+def simulator_timing(kinfo, cfg, names, lam, n=60):
     """The oracle's discrete-event simulator (synthetic mode) on a trace of the config:
     wall time and simulated events per second on one core."""
     from oracle import sim

@@ -18,7 +18,7 @@ from oracle import sim  # noqa: E402
 from workload import traces  # noqa: E402
 
 detail = json.load(open(sys.argv[1]))
-n = int(sys.argv[2]) if len(sys.argv) > 2 else 400
+n = int(sys.argv[2]) if len(sys.argv) > 2 else 60
 names = detail["models"]
 models = []
 for nm in names:
@@ -35,7 +35,7 @@ t = traces.arrivals(n, lam, kind="lognormal", sigma=cfg.get("sigma", 2.0), seed=
 mm = traces.model_choices(n, cfg["weights"], seed=11)
 trace = [(int(t[i]), int(mm[i]), int(mm[i])) for i in range(n)]
 rows = []
-for dd in (0, 100, 1000, 5000, 20000, 100000):
+for dd in (0, 1000, 10000, 50000):
     gpu = sim.GPUModel(launch_delay=3000, notif_delay=5000, decide_delay=dd)
     c = sim.Config(num_clients=len(names), slack=1184, lookahead=3, max_active=8)
     t0 = time.perf_counter()
