@@ -635,7 +635,7 @@ def cpu_baseline(cfg, seconds=20.0, reserve=0):
             "host": hi}
 
 
-def simulator_timing(kinfo, cfg, names, lam, n=60):
+def simulator_timing(kinfo, cfg, names, lam, n=20):
     """The oracle's discrete-event simulator (synthetic mode) on a trace of the config:
     wall time and simulated events per second on one core."""
     from oracle import sim
