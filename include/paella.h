@@ -395,6 +395,14 @@ int paella_clock_info(paella_t* p, uint32_t gpu, int64_t* offset_ns, int64_t* rt
    call it with a profiler attached.  0, -ENODEV (FAKE device), -ENOTSUP, -EIO. */
 int paella_clock_sync(paella_t* p, uint32_t gpu);
 
+/* Counter mode, device side of the exactly-once invariant (S5 b, C3): with no job live,
+   every counter slot's device {start, end} counts and their host mirror equal the sum of
+   the grids of all launches counted on that slot (each block entered and exited once;
+   nothing lost, nothing doubled).  Returns the number of mismatching slots (0 = all
+   good), *slots_checked = slots used so far; -EBUSY jobs live, -ENOTSUP not counter
+   mode, -ENODEV FAKE device. */
+int paella_check_counters(paella_t* p, uint32_t gpu, uint32_t* slots_checked);
+
 /* Flush and close the event logs (also done by shutdown). */
 int paella_flush_log(paella_t* p);
 

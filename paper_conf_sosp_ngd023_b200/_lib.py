@@ -38,7 +38,7 @@ SYMBOLS = ["paella_init", "paella_register_model", "paella_submit", "paella_subm
            "paella_bench_roundtrip", "paella_loadgen", "paella_bench_wait", "paella_route_pair",
            "paella_clock_info", "paella_clock_sync", "paella_channel_path", "paella_client_attach",
            "paella_client_region_of", "paella_client_model_io", "paella_client_submit", "paella_client_poll",
-           "paella_client_detach", "paella_bench_xdev"]
+           "paella_client_detach", "paella_bench_xdev", "paella_check_counters"]
 
 
 class Config(C.Structure):
@@ -133,6 +133,7 @@ def load():
     lib.paella_clock_info.argtypes = [P, C.c_uint32, C.POINTER(C.c_int64), C.POINTER(C.c_int64),
                                       C.POINTER(C.c_int64)]
     lib.paella_clock_sync.argtypes = [P, C.c_uint32]
+    lib.paella_check_counters.argtypes = [P, C.c_uint32, C.POINTER(C.c_uint32)]
     lib.paella_channel_path.argtypes = [P, C.c_char_p, C.c_size_t]
     lib.paella_bench_xdev.argtypes = [P, C.c_uint32, C.POINTER(C.c_uint32), C.c_uint32, C.POINTER(C.c_uint32),
                                       C.c_uint32, C.c_uint32, C.POINTER(C.c_double)]
@@ -439,6 +440,12 @@ class Engine:
         buf = C.create_string_buffer(256)
         _check(self.lib.paella_channel_path(self.h, buf, 256), "paella_channel_path")
         return buf.value.decode()
+
+    def check_counters(self, gpu=0):
+        """(mismatching slots, slots used): paella_check_counters."""
+        n = C.c_uint32()
+        bad = _check(self.lib.paella_check_counters(self.h, gpu, C.byref(n)), "paella_check_counters")
+        return bad, n.value
 
     def clock_sync(self, gpu=0):
         _check(self.lib.paella_clock_sync(self.h, gpu), "paella_clock_sync")

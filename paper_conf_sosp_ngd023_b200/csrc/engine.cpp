@@ -1578,6 +1578,30 @@ const char* paella_kernel_name(uint32_t kind) {
   return kind < KIND_COUNT ? names[kind] : "?";
 }
 
+int paella_check_counters(paella_t* p, uint32_t gpu, uint32_t* slots_checked) {
+  Paella* P = (Paella*)p;
+  if (!P || gpu >= P->gpus.size()) return -EINVAL;
+  if (P->cfg.device != PAELLA_DEVICE_CUDA) return -ENODEV;
+  Gpu* g = P->gpus[gpu].get();
+  if (!g->ctr_mode) return -ENOTSUP;
+  if (g->policy->live_jobs() != 0 || !g->ctr_live.empty()) return -EBUSY;
+  auto* cb = static_cast<CudaBackend*>(g->be.get());
+  std::vector<uint32_t> dev(2 * NCTR_M), mir(2 * NCTR_M);
+  cudaSetDevice(g->device);
+  if (cudaMemcpy(dev.data(), cb->ctr_m, dev.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess) return -EIO;
+  std::memcpy(mir.data(), (const void*)cb->mirror_h, mir.size() * 4);
+  int bad = 0;
+  uint32_t used = 0;
+  for (uint32_t s = 0; s < NCTR_M; ++s) {
+    const uint32_t want = g->ctr_mbase[s];   // sum of the grids of every launch counted on slot s
+    if (want) ++used;
+    // device counters AND their host mirror: every block entered and exited exactly once
+    if (dev[2 * s] != want || dev[2 * s + 1] != want || mir[2 * s] != want || mir[2 * s + 1] != want) ++bad;
+  }
+  if (slots_checked) *slots_checked = used;
+  return bad;
+}
+
 int paella_clock_sync(paella_t* p, uint32_t gpu) {
   Paella* P = (Paella*)p;
   if (!P || gpu >= P->gpus.size()) return -EINVAL;

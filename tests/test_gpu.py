@@ -174,6 +174,12 @@ def test_serving_parity_and_replay(tmp_path, policy, group, streams, ring, look,
         _serve_and_check(e, specs, 120, 3, seed=policy * 7 + group)
         st = e.stats()
         assert st["completed"] == 120
+        if notify == "counters":
+            # S5 (b) on the device: the blocks' own counts, not the records the dispatcher
+            # synthesised from them -- every slot advanced by exactly its launches' grids
+            time.sleep(0.01)
+            bad, used = e.check_counters()
+            assert bad == 0 and used > 0, (bad, used)
         if notify == "counters" and look == 0:
             # relaxed exits: jobs that went idle recorded a release event; moves to another
             # stream waited for it (the outputs above are checked either way; with
