@@ -565,8 +565,13 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     const uint32_t px0 = split * rows;
     const uint32_t g = threadIdx.x % (TC_BM / 8), co = m0 + g * 8;
     const uint32_t nitems = rows * (TC_BM / 8);
-    const uint32_t slice = rows * TC_BM * 4;                // bytes of one slice
+    const uint32_t slice = rows * TC_BM * 4;                // bytes of one slice (slot pitch)
     float* recv = stage + TC_BN * TC_BM;                    // ks - 1 received slices (free A stages)
+    // only the slice rows that hold real pixels travel (the tile tail past P does not)
+    auto valid_rows = [&](uint32_t owner) -> uint32_t {
+      const uint32_t r0 = n0 + owner * rows;
+      return r0 >= P ? 0u : min(rows, P - r0);
+    };
     float bias[8];
     uint4 rres[MAXI];
     if (warp < 4 && co < a.cout) {
@@ -580,7 +585,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
         }
       }
     }
-    if (threadIdx.x == 0) mbar_arrive_tx(rbar, (ks - 1) * slice);   // before any peer can push
+    if (threadIdx.x == 0) mbar_arrive_tx(rbar, (ks - 1) * valid_rows(split) * TC_BM * 4);   // before any push
     if (warp < 4) fence_proxy_async();   // the staged tile (generic writes) is read by the bulk copies
     __syncwarp();
     if (trace && threadIdx.x == 0) tr[9] = globaltimer();
@@ -595,13 +600,15 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       // the sender's distance behind it
       for (uint32_t j = 1; j < ks; ++j) {
         const uint32_t owner = (split + j) & (ks - 1);
+        const uint32_t bytes = valid_rows(owner) * TC_BM * 4;
+        if (bytes == 0) continue;
         const uint32_t slot = (split + ks - owner - 1) & (ks - 1);
         uint32_t dst, bar;
         asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(dst) : "r"(su32(recv) + slot * slice), "r"(owner));
         asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(bar) : "r"(su32(rbar)), "r"(owner));
         asm volatile(
             "cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
-            "r"(su32(stage) + owner * slice), "r"(slice), "r"(bar)
+            "r"(su32(stage) + owner * slice), "r"(bytes), "r"(bar)
             : "memory");
       }
     }
