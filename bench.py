@@ -116,7 +116,11 @@ class Dist:
         if self.world > 1:
             import torch.distributed as dist
             os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-            dist.init_process_group("gloo", rank=self.rank, world_size=self.world)
+            import datetime
+            # rank 0 drives every GPU (calibration, five arms, SLO searches) while the
+            # other ranks wait at the barrier: a long timeout
+            dist.init_process_group("gloo", rank=self.rank, world_size=self.world,
+                                    timeout=datetime.timedelta(hours=3))
             self.pg = dist
 
     def barrier(self):
