@@ -492,7 +492,7 @@ def run_gpu(args, ngpus, cores, fake):
         r["dispatcher"] = dstats
         if label == "paella":
             # device-only roofline (summed isolated kernel time), dominant-kernel roofline
-            dev_roof, kinfo = {}, {}
+            dev_roof, dev_cold, kinfo = {}, {}, {}
             for m, nm in enumerate(names):
                 ks = a.e.kernels(a.mids[m])
                 if fake:
@@ -500,9 +500,13 @@ def run_gpu(args, ngpus, cores, fake):
                 else:
                     kt = a.e.time_kernels(a.mids[m], instrumented=False, reps=20)
                     kti = a.e.time_kernels(a.mids[m], instrumented=True, reps=20)
+                    # L2-cold: 2 x L2 overwritten before each launch
+                    dev_cold[nm] = float(a.e.time_kernels(a.mids[m], instrumented=False, reps=7,
+                                                          l2_cold=True).sum()) / 1e3
                 dev_roof[nm] = float(kt.sum()) / 1e3
                 kinfo[nm] = (ks, kt, kti)
             r["dev_roof"] = dev_roof
+            r["dev_roof_l2_cold"] = dev_cold
             r["kinfo"] = kinfo
             # the served kernel table (simulator inputs, tools/sim_delay_sweep.py)
             detail["kernels"] = {nm: [dict(name=k["name"], grid=k["grid"], block=k["block"], regs=k["regs"],
@@ -789,6 +793,10 @@ def main():
                 "jct_p99_us": round(P["e2e"]["jct"]["mix"]["p99_us"])},
         "gpu_launches": int(sum(d["launches"] for d in disp)),
         "dispatcher_busy_frac": [d["busy_frac"] for d in disp],
+        # north star: JCT as a fraction of the device-only roofline (summed isolated
+        # kernel time of the model, L2-warm PDL chain) -- roofline / mean JCT per model
+        "device_roofline_frac": {nm: round(P["dev_roof"][nm] / P["jct"][nm]["mean_us"], 3)
+                                 for nm in names if nm in P["jct"]} if "dev_roof" in P else None,
         "clocks": P["clocks"],
     }
     if ngpus == 1 and not args.fake:

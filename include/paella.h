@@ -421,6 +421,10 @@ int paella_run_isolated(paella_t* p, uint32_t gpu, uint32_t model_id, const void
    elapsed / reps.  Returns 0 or -errno. */
 int paella_time_kernels(paella_t* p, uint32_t gpu, uint32_t model_id, uint32_t instrumented,
                         uint32_t reps, int64_t* kernel_ns);
+#define PAELLA_TIME_L2_COLD 2u   /* `instrumented` bit: L2-cold timing -- before every launch a
+                                    256 MiB buffer (2 x L2) is overwritten on the stream and each
+                                    launch is timed alone (plain launch, median of reps); without
+                                    it the launches run back to back (PDL chain, L2-warm) */
 
 /* X_dev, the device-only saturation throughput: request i runs model
    models[seq[i]] as a CUDA graph of its uninstrumented kernel chain on stream i % streams

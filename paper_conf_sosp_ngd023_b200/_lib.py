@@ -356,10 +356,11 @@ class Engine:
         _check(self.lib.paella_debug_node(self.h, gpu, model, node, _fptr(out)), "paella_debug_node")
         return out.reshape(shape)
 
-    def time_kernels(self, model, instrumented=True, reps=50, gpu=0):
+    def time_kernels(self, model, instrumented=True, reps=50, gpu=0, l2_cold=False):
         n = self.model_info(model)["n_kernels"]
         kt = np.zeros(n, dtype=np.int64)
-        _check(self.lib.paella_time_kernels(self.h, gpu, model, 1 if instrumented else 0, reps,
+        flags = (1 if instrumented else 0) | (2 if l2_cold else 0)
+        _check(self.lib.paella_time_kernels(self.h, gpu, model, flags, reps,
                                             kt.ctypes.data_as(C.POINTER(C.c_int64))), "paella_time_kernels")
         return kt
 

@@ -1485,7 +1485,18 @@ int paella_shutdown(paella_t* p) {
       cudaSetDevice(g->device);
       static_cast<CudaBackend*>(g->be.get())->stop_proxy();
       g->be->sync();
-      if (g->prof_stream) cudaStreamSynchronize((cudaStream_t)g->prof_stream);
+      if (g->prof_stream) {   // isolated-run resources (ensure_iso)
+        cudaStreamSynchronize((cudaStream_t)g->prof_stream);
+        cudaStreamDestroy((cudaStream_t)g->prof_stream);
+        g->prof_stream = nullptr;
+        cudaFreeHost(g->prof_ring_h);
+        cudaFreeHost(g->stage_in);
+        cudaFree(g->prof_tail);
+        cudaFree(g->prof_ctr);
+        cudaFree(g->prof_devring);
+        cudaFree(g->trace_buf);
+      }
+      if (g->flush_buf) cudaFree(g->flush_buf);
     }
   }
   write_route_logs(P);
@@ -1827,6 +1838,45 @@ static int64_t time_layer(Gpu* g, Model* m, uint32_t l, bool instr, uint32_t rep
   }
   cudaEventDestroy(e0);
   cudaEventDestroy(e1);
+  return ns;
+}
+
+// L2-cold device time of kernel l (L2-cold vs L2-warm): before each of
+// `reps` launches a 2 x L2-sized buffer is overwritten on the same stream (the kernel's
+// weights and inputs are evicted), and only the kernel itself is timed (events around
+// each launch); ns per launch (median), -1 on error.
+static int64_t time_layer_cold(Gpu* g, Model* m, uint32_t l, bool instr, uint32_t reps) {
+  cudaSetDevice(g->device);
+  cudaStream_t s = (cudaStream_t)g->prof_stream;
+  auto* cb = static_cast<CudaBackend*>(g->be.get());
+  const uint32_t iso_slot = (uint32_t)m->gpu[g->index].args.size() - 1;
+  const KernelInst& k = m->kernels[l];
+  const size_t flush_bytes = 256ull << 20;
+  if (!g->flush_buf && cudaMalloc(&g->flush_buf, flush_bytes) != cudaSuccess) return -1;
+  reps = std::min(reps, 64u);
+  std::vector<cudaEvent_t> ev(2 * reps);
+  for (auto& e : ev) cudaEventCreate(&e);
+  const void* tm = is_tc(k.kind) ? m->gpu[g->index].tmaps[l].b : nullptr;
+  for (uint32_t r = 0; r < reps; ++r) {
+    cudaMemsetAsync(g->flush_buf, (int)(r & 0xff), flush_bytes, s);
+    InstrArgs ia = iso_instr(g, k.grid_total(), g->P->cfg.group_size, l + 1 == m->kernels.size());
+    void* args[3] = {(void*)&m->gpu[g->index].args[iso_slot][l], (void*)&ia, (void*)tm};
+    cudaEventRecord(ev[2 * r], s);
+    cuda_launch(cb->fn(k.kind, m->dtype, instr), k, args, s, false);
+    cudaEventRecord(ev[2 * r + 1], s);
+  }
+  int64_t ns = -1;
+  if (cudaStreamSynchronize(s) == cudaSuccess) {
+    std::vector<int64_t> t(reps);
+    for (uint32_t r = 0; r < reps; ++r) {
+      float ms = 0;
+      cudaEventElapsedTime(&ms, ev[2 * r], ev[2 * r + 1]);
+      t[r] = (int64_t)((double)ms * 1e6);
+    }
+    std::nth_element(t.begin(), t.begin() + reps / 2, t.end());
+    ns = t[reps / 2];
+  }
+  for (auto& e : ev) cudaEventDestroy(e);
   return ns;
 }
 
@@ -2189,7 +2239,8 @@ int paella_time_kernels(paella_t* p, uint32_t gpu, uint32_t model_id, uint32_t i
   int rc = iso_run(g, m, nullptr, nullptr, nullptr, true);   // materialise valid activations
   if (rc) return rc;
   for (uint32_t l = 0; l < m->kernels.size(); ++l) {
-    kernel_ns[l] = time_layer(g, m, l, instrumented != 0, reps);
+    kernel_ns[l] = (instrumented & PAELLA_TIME_L2_COLD) ? time_layer_cold(g, m, l, instrumented & 1u, reps)
+                                                        : time_layer(g, m, l, instrumented & 1u, reps);
     if (kernel_ns[l] < 0) return -EIO;
   }
   return 0;

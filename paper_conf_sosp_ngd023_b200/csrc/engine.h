@@ -224,6 +224,7 @@ struct Gpu {
   uint32_t* prof_tail = nullptr;
   Rec* prof_devring = nullptr;     // device-memory ring of isolated runs
   void* trace_buf = nullptr;       // debug phase timestamps
+  void* flush_buf = nullptr;       // L2-cold timing: overwritten before each timed launch
   uint32_t* prof_ctr = nullptr;
   std::vector<uint32_t> prof_base;
   uint32_t prof_uid = 0;
