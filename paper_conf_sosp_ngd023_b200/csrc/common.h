@@ -75,10 +75,15 @@ struct InstrArgs {
   uint32_t uid;       // unique launch id (kernel id of the paper)
   uint32_t group;     // G
   uint32_t flags;     // INSTR_*
+  uint32_t ctr_stride;   // counter mode: words between the NCTR_SUB counter tables
 };
 
 constexpr uint32_t NCTR = 4096;   // counter slots; > max in-flight launches (<= P)
 constexpr uint32_t NCTR_M = 256;  // counter-mode slots (free list; > P x (lookahead + 1))
+// counter mode: each launch's {start, end} counts are split over NCTR_SUB tables (block b
+// counts in table b % NCTR_SUB, ctr_stride words apart) so the blocks of one launch do not
+// all reduce into one L2 address; the host sums the tables
+constexpr uint32_t NCTR_SUB = 4;
 
 // Kernel-side arguments of one layer.  Activations are NHWC with an explicit
 // channel stride/offset so that a concat is just producers writing into disjoint

@@ -279,7 +279,7 @@ struct CudaBackend : Backend {
   // forwards to the host ring, so no kernel pays the PCIe write on its exit path
   bool proxy = false;
   bool mirror = false;         // counter mode: kernels only count, k_notify_mirror copies
-  uint32_t* ctr_m = nullptr;   // device: NCTR_M x {start, end}
+  uint32_t* ctr_m = nullptr;   // device: NCTR_SUB tables of NCTR_M x {start, end}
   uint32_t* mirror_h = nullptr;   // pinned, mapped host copy
   uint32_t* mirror_d = nullptr;
   bool pdl = true;             // programmatic dependent launches (off for the naive baseline)
@@ -298,12 +298,13 @@ struct CudaBackend : Backend {
   uint32_t* ctl_d = nullptr;
   int setup_proxy(cudaStream_t s) {
     if (mirror) {
-      if (cudaMalloc(&ctr_m, 2 * NCTR_M * sizeof(uint32_t)) != cudaSuccess) return -ENOMEM;
-      cudaMemsetAsync(ctr_m, 0, 2 * NCTR_M * sizeof(uint32_t), s);
-      if (cudaHostAlloc((void**)&mirror_h, 2 * NCTR_M * sizeof(uint32_t), cudaHostAllocMapped | cudaHostAllocPortable) !=
+      if (cudaMalloc(&ctr_m, NCTR_SUB * 2 * NCTR_M * sizeof(uint32_t)) != cudaSuccess) return -ENOMEM;
+      cudaMemsetAsync(ctr_m, 0, NCTR_SUB * 2 * NCTR_M * sizeof(uint32_t), s);
+      if (cudaHostAlloc((void**)&mirror_h, NCTR_SUB * 2 * NCTR_M * sizeof(uint32_t),
+                        cudaHostAllocMapped | cudaHostAllocPortable) !=
           cudaSuccess)
         return -ENOMEM;
-      std::memset(mirror_h, 0, 2 * NCTR_M * sizeof(uint32_t));
+      std::memset(mirror_h, 0, NCTR_SUB * 2 * NCTR_M * sizeof(uint32_t));
       cudaHostGetDevicePointer((void**)&mirror_d, mirror_h, 0);
     } else {
       if (cudaMalloc(&dev_ring, (size_t)cap * sizeof(Rec)) != cudaSuccess) return -ENOMEM;
@@ -457,6 +458,7 @@ static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last, bool
     uint32_t slot = g->ctr_free.back();
     g->ctr_free.pop_back();
     ia.ctr = static_cast<CudaBackend*>(g->be.get())->ctr_m + 2 * slot;
+    ia.ctr_stride = 2 * NCTR_M;
     ia.base = g->ctr_mbase[slot];
     g->ctr_mbase[slot] += grid;
     if (last && std::getenv("PAELLA_LAST_SYS")) ia.flags |= INSTR_SYSREL;
@@ -757,8 +759,13 @@ static uint32_t drain_counters(Gpu* g) {
   uint32_t n = 0;
   for (size_t i = 0; i < g->ctr_live.size();) {
     Gpu::CtrLive& L = g->ctr_live[i];
-    const uint64_t v = *reinterpret_cast<volatile uint64_t*>(cb->mirror_h + 2 * L.slot);
-    uint32_t cnt[2] = {(uint32_t)v - L.base, (uint32_t)(v >> 32) - L.base};
+    uint32_t st = 0, en = 0;   // the launch's counts, summed over the NCTR_SUB tables
+    for (uint32_t t = 0; t < NCTR_SUB; ++t) {
+      const uint64_t v = *reinterpret_cast<volatile uint64_t*>(cb->mirror_h + t * 2 * NCTR_M + 2 * L.slot);
+      st += (uint32_t)v;
+      en += (uint32_t)(v >> 32);
+    }
+    uint32_t cnt[2] = {st - L.base, en - L.base};
     uint32_t* seen[2] = {&L.p, &L.f};
     bool finished = false;
     for (int t = 0; t < 2; ++t) {
@@ -1291,8 +1298,8 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     for (int r = 0; r < NRES; ++r) pc.capacity[r] = P->capacity[r];
     if (cfg.device == PAELLA_DEVICE_CUDA &&
         (static_cast<CudaBackend*>(g->be.get())->proxy || static_cast<CudaBackend*>(g->be.get())->mirror)) {
-      // the resident proxy warp: 1 block, 1 warp, <= 64 regs/thread, the 1 KB reservation
-      const int64_t proxy[NRES] = {1, 1, 64 * 32, 1024, 0};
+      // the resident proxy / mirror warp: 1 block, 1 warp, its registers, the 1 KB reservation
+      const int64_t proxy[NRES] = {1, 1, 160 * 32, 1024, 0};   // mirror warp: <= 160 regs/thread
       for (int r = 0; r < NRES; ++r) pc.capacity[r] -= proxy[r];
     }
     g->policy.reset(new Policy(pc));
@@ -1597,7 +1604,7 @@ int paella_check_counters(paella_t* p, uint32_t gpu, uint32_t* slots_checked) {
   if (!g->ctr_mode) return -ENOTSUP;
   if (g->policy->live_jobs() != 0 || !g->ctr_live.empty()) return -EBUSY;
   auto* cb = static_cast<CudaBackend*>(g->be.get());
-  std::vector<uint32_t> dev(2 * NCTR_M), mir(2 * NCTR_M);
+  std::vector<uint32_t> dev(NCTR_SUB * 2 * NCTR_M), mir(NCTR_SUB * 2 * NCTR_M);
   cudaSetDevice(g->device);
   if (cudaMemcpy(dev.data(), cb->ctr_m, dev.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess) return -EIO;
   std::memcpy(mir.data(), (const void*)cb->mirror_h, mir.size() * 4);
@@ -1606,8 +1613,15 @@ int paella_check_counters(paella_t* p, uint32_t gpu, uint32_t* slots_checked) {
   for (uint32_t s = 0; s < NCTR_M; ++s) {
     const uint32_t want = g->ctr_mbase[s];   // sum of the grids of every launch counted on slot s
     if (want) ++used;
+    uint32_t d0 = 0, d1 = 0, m0 = 0, m1 = 0;
+    for (uint32_t t = 0; t < NCTR_SUB; ++t) {
+      d0 += dev[t * 2 * NCTR_M + 2 * s];
+      d1 += dev[t * 2 * NCTR_M + 2 * s + 1];
+      m0 += mir[t * 2 * NCTR_M + 2 * s];
+      m1 += mir[t * 2 * NCTR_M + 2 * s + 1];
+    }
     // device counters AND their host mirror: every block entered and exited exactly once
-    if (dev[2 * s] != want || dev[2 * s + 1] != want || mir[2 * s] != want || mir[2 * s + 1] != want) ++bad;
+    if (d0 != want || d1 != want || m0 != want || m1 != want) ++bad;
   }
   if (slots_checked) *slots_checked = used;
   return bad;
@@ -1673,13 +1687,13 @@ static int ensure_iso(Gpu* g) {
     return -ENOMEM;
   std::memset(g->prof_ring_h, 0, cap * sizeof(Rec));
   cudaHostGetDevicePointer(&g->prof_ring_d, g->prof_ring_h, 0);
-  if (cudaMalloc(&g->prof_tail, 256) || cudaMalloc(&g->prof_ctr, 2 * NCTR * sizeof(uint32_t))) return -ENOMEM;
+  if (cudaMalloc(&g->prof_tail, 256) || cudaMalloc(&g->prof_ctr, NCTR_SUB * 2 * NCTR * sizeof(uint32_t))) return -ENOMEM;
   g->prof_base.assign(NCTR, 0);
   cudaStream_t s;
   cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
   g->prof_stream = s;
   cudaMemsetAsync(g->prof_tail, 0, 256, s);
-  cudaMemsetAsync(g->prof_ctr, 0, 2 * NCTR * sizeof(uint32_t), s);
+  cudaMemsetAsync(g->prof_ctr, 0, NCTR_SUB * 2 * NCTR * sizeof(uint32_t), s);
   // isolated runs write their records to device memory (as served kernels do through
   // the proxy); nobody consumes them except the round-trip benchmark's direct ring
   if (cudaMalloc(&g->prof_devring, cap * sizeof(Rec))) return -ENOMEM;
@@ -2130,6 +2144,7 @@ static InstrArgs iso_instr(Gpu* g, uint32_t grid, uint32_t group, bool last) {
   uint32_t uid = g->prof_uid++;
   uint32_t slot = uid % NCTR;
   ia.ctr = g->prof_ctr + 2 * slot;
+  ia.ctr_stride = 2 * NCTR;
   ia.mask = (1u << 16) - 1;
   ia.log2cap = 16;
   ia.base = g->prof_base[slot];

@@ -54,6 +54,12 @@ __device__ __forceinline__ void maybe_record(const InstrArgs& ia, uint32_t type,
   }
 }
 
+// counter mode: this block's {start, end} counter pair (table blockid % NCTR_SUB)
+__device__ __forceinline__ uint32_t* ctr_of_block(const InstrArgs& ia) {
+  const uint32_t b = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
+  return ia.ctr + (b % NCTR_SUB) * ia.ctr_stride;
+}
+
 // T = the (1-D) thread that does the bookkeeping; kernels pick an otherwise idle
 // thread so that compute never waits on the counter atomics
 template <bool INSTR, uint32_t T = 0>
@@ -61,7 +67,7 @@ __device__ __forceinline__ void instr_enter(const InstrArgs& ia) {
   if constexpr (INSTR) {
     if (threadIdx.x == T && threadIdx.y == 0 && threadIdx.z == 0) {
       if (ia.flags & INSTR_CTR) {
-        asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[0]) : "memory");
+        asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(ctr_of_block(ia)) : "memory");
       } else {
         uint32_t total = gridDim.x * gridDim.y * gridDim.z;
         uint32_t c = atomicAdd(&ia.ctr[0], 1u) + 1u - ia.base;
@@ -100,9 +106,9 @@ __device__ __forceinline__ void kernel_begin(const InstrArgs& ia) {
 // system-scope release.
 __device__ __forceinline__ void last_kernel_exit(const InstrArgs& ia) {
   if (ia.flags & INSTR_SYSREL)
-    asm volatile("red.release.sys.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+    asm volatile("red.release.sys.global.add.u32 [%0], 1;" ::"l"(ctr_of_block(ia) + 1) : "memory");
   else
-    asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+    asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(ctr_of_block(ia) + 1) : "memory");
 }
 
 // exit count of a block whose every other thread is already past a CTA barrier (the
@@ -114,9 +120,9 @@ __device__ __forceinline__ void instr_exit_last_thread(const InstrArgs& ia) {
       if (ia.flags & INSTR_LAST)
         last_kernel_exit(ia);
       else if (ia.flags & INSTR_RELAXED)
-        asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+        asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(ctr_of_block(ia) + 1) : "memory");
       else
-        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(ctr_of_block(ia) + 1) : "memory");
     } else {
       uint32_t old;
       if (ia.flags & INSTR_LAST)
@@ -139,7 +145,7 @@ __device__ __forceinline__ void instr_exit(const InstrArgs& ia) {
       // the block finished a few hundred ns before its last warp retires, which only
       // shifts the occupancy estimate
       if (threadIdx.x == T && threadIdx.y == 0 && threadIdx.z == 0)
-        asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+        asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(ctr_of_block(ia) + 1) : "memory");
       return;
     }
     __syncthreads();
@@ -150,9 +156,9 @@ __device__ __forceinline__ void instr_exit(const InstrArgs& ia) {
       if (ia.flags & INSTR_LAST)
         last_kernel_exit(ia);
       else if (ia.flags & INSTR_RELAXED)   // data dependencies ride on stream order
-        asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+        asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(ctr_of_block(ia) + 1) : "memory");
       else
-        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(ctr_of_block(ia) + 1) : "memory");
     } else if (threadIdx.x == T && threadIdx.y == 0 && threadIdx.z == 0) {
       // acq_rel atomic: releases this block's outputs (ordered before by the barrier,
       // release is cumulative) and acquires the earlier blocks' before the record is

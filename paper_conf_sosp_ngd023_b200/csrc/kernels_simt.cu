@@ -682,7 +682,7 @@ KernelFn proxy_kernel() { return (KernelFn)k_notify_proxy; }
 // ---------------------------------------------------------------------------
 __global__ void __launch_bounds__(32, 1) k_notify_mirror(const uint4* ctrs, uint4* host, volatile uint32_t* state) {
   const uint32_t lane = threadIdx.x;
-  constexpr uint32_t NQ = NCTR_M * 2 / 4 / 32;   // 16-byte chunks per lane
+  constexpr uint32_t NQ = NCTR_SUB * NCTR_M * 2 / 4 / 32;   // 16-byte chunks per lane (all tables)
   uint4 prev[NQ];
 #pragma unroll
   for (uint32_t i = 0; i < NQ; ++i) prev[i] = make_uint4(~0u, ~0u, ~0u, ~0u);   // publish everything once

@@ -507,7 +507,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     // counts the block as soon as its MMAs are complete -- the count travels while the
     // epilogue runs instead of trailing the block's last store
     if (warp == 5 && lane == 0 && (ia.flags & RELAXED_CTR) == RELAXED_CTR)
-      asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(&ia.ctr[1]) : "memory");
+      asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(ctr_of_block(ia) + 1) : "memory");
   }
   if (warp < 4) {
     const uint32_t row = warp * 32 + lane;
