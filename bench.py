@@ -78,10 +78,10 @@ def parse():
                     help="arms to run on the step traces (paella always runs)")
     ap.add_argument("--no-baselines", action="store_true", help="only the paella arm")
     ap.add_argument("--max-active", type=int, default=8, help="job cap K of the paella arms (B200-Q6); 0 = none")
-    ap.add_argument("--lookahead", type=int, default=3, help="NEXT-1 launch-ahead depth of the paella arms")
-    ap.add_argument("--slack", type=int, default=1184,
-                    help="B, blocks issued beyond full utilisation (P1300-1304); 8 x 148 SMs covers the "
-                         "measured dispatch loop delay (DESIGN.md B200-Q1)")
+    ap.add_argument("--lookahead", type=int, default=6, help="NEXT-1 launch-ahead depth of the paella arms")
+    ap.add_argument("--slack", type=int, default=3552,
+                    help="B, blocks issued beyond full utilisation (P1300-1304); 24 x 148 SMs covers the "
+                         "measured dispatch loop delay with launch-ahead 6 (DESIGN.md B200-Q1)")
     ap.add_argument("--policy", default="srpt", choices=["srpt", "fifo", "sjf", "rr"],
                     help="policy of the paella arm (sjf/rr: Table 3 ablations, NEXT-2)")
     ap.add_argument("--theta", type=int, default=100, help="fairness threshold (kernel dispatches, P1296-1297)")
@@ -643,7 +643,7 @@ def cpu_baseline(cfg, seconds=20.0, reserve=0):
             "host": hi}
 
 
-def simulator_timing(kinfo, cfg, names, lam, n=20):
+def simulator_timing(kinfo, cfg, names, lam, args_slack, args_lookahead, n=20):
     """The oracle's discrete-event simulator (synthetic mode) on a trace of the config:
     wall time and simulated events per second on one core."""
     from oracle import sim
@@ -660,7 +660,7 @@ def simulator_timing(kinfo, cfg, names, lam, n=20):
         models.append(ls)
     t, mm, _ = make_trace(n, lam, cfg, len(names), seed=31)
     trace = [(int(t[i]), int(mm[i]), int(mm[i])) for i in range(n)]
-    c = sim.Config(num_clients=len(names), slack=1184, lookahead=3, max_active=8)
+    c = sim.Config(num_clients=len(names), slack=args_slack, lookahead=args_lookahead, max_active=8)
     t0 = time.perf_counter()
     r = sim.simulate(c, models, trace, sim.GPUModel(), check=False)
     el = time.perf_counter() - t0
@@ -808,7 +808,8 @@ def main():
         line["cpu_baseline"] = {k: v for k, v in cb.items() if k != "host"}
         detail["cpu_baseline"] = cb
         try:
-            detail["simulator"] = simulator_timing(P["kinfo"], dict(cfg, weights=detail["mix_weights"]), names, lam)
+            detail["simulator"] = simulator_timing(P["kinfo"], dict(cfg, weights=detail["mix_weights"]), names, lam,
+                                                  args.slack, args.lookahead)
         except Exception as ex:
             detail["simulator"] = {"error": str(ex)[:200]}
     if args.fake:

@@ -113,7 +113,7 @@ typedef struct {
                                     the durations (paella_stats ev_*): the live roofline */
   uint32_t lookahead;            /* NEXT-1 launch-ahead depth: 0 = the paper's semantics (a
                                     job's next kernel is dispatched after the previous one's
-                                    final COMPLETION); D in 1..4 = once the job's OLDEST
+                                    final COMPLETION); D in 1..7 = once the job's OLDEST
                                     in-flight kernel is fully placed (running) and <= D are in
                                     flight, the next kernel is queued behind it on the same
                                     stream (with PDL it starts ~0.6 us after its predecessor) */

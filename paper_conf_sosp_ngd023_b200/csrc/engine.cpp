@@ -81,7 +81,7 @@ static double ns_per_tick() {
 // event log (replay input for oracle/sim.py::replay; format in DESIGN.md)
 // ---------------------------------------------------------------------------
 enum : uint32_t { EV_ARRIVAL = 1, EV_RECORD = 2, EV_BATCH_END = 3, EV_ISSUE = 4, EV_COMPLETE = 5, EV_OBSERVE = 6, EV_ROUTE = 7,
-                  EV_CLOCK = 8,
+                  EV_CLOCK = 8, EV_TIME = 9,
                   EV_CONFIG = 100, EV_CAPACITY = 101, EV_MODEL = 110, EV_LAYER = 111, EV_DEMAND = 112, EV_DEP = 113,
                   EV_VS = 114 };
 
@@ -821,6 +821,7 @@ static void decide_and_launch(Gpu* g) {
     JobRec& j = g->jobs[is.job];
     Model* m = g->P->models[j.model].get();
     logev(g, EV_ISSUE, is.stream, is.uid, is.job, is.layer);
+    if (g->log_times) logev(g, EV_TIME, 0, is.uid, (uint64_t)now_ns(), 0);   // decision time (host)
     const uint32_t v = g->policy->model(j.model)[is.layer].vs;
     if (j.rel_stream[v] >= 0) {
       if ((uint32_t)j.rel_stream[v] != is.stream) {   // moved: wait for the previous stream's release
@@ -1015,6 +1016,7 @@ static void dispatch_loop(Gpu* g) {
     // 3. decide (the batch boundary is logged for replay, C2-Q17)
     if (nev) {
       logev(g, EV_BATCH_END, 0, 0, 0, 0);
+      if (g->log_times) logev(g, EV_TIME, 1, 0, (uint64_t)now_ns(), 0);   // records consumed (host)
       decide_and_launch(g);
       g->pub->work.store(g->policy->outstanding_work(), std::memory_order_release);
       busy_ticks += ticks() - it0;
@@ -1178,7 +1180,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
   if (cfg.client_region_bytes == 0) cfg.client_region_bytes = 64ull << 20;
   if (cfg.fake_time_scale_ns == 0) cfg.fake_time_scale_ns = 500;
   if (cfg.fairness_threshold < 0) return -EINVAL;
-  if (cfg.lookahead > 4) return -EINVAL;
+  if (cfg.lookahead > 7) return -EINVAL;   // in-flight uid list per virtual stream: 8
   if (cfg.prio_classes == 0) cfg.prio_classes = 1;
   if (cfg.notify_mode > PAELLA_NOTIFY_RING) return -EINVAL;
   // counter mode: in-flight launches (<= P x (lookahead + 1)) must fit the slot table
@@ -1312,6 +1314,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
       char path[4096];
       snprintf(path, sizeof path, cfg.event_log_path, gi);
       g->log = fopen(path, "wb");
+      g->log_times = std::getenv("PAELLA_TRACE_TIMES") != nullptr;
       if (!g->log) return -EINVAL;
       setvbuf(g->log, nullptr, _IOFBF, 1 << 20);
       logev(g.get(), EV_CONFIG, cfg.num_clients, cfg.policy, (uint64_t)cfg.fairness_threshold,

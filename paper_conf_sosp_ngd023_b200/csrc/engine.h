@@ -215,6 +215,7 @@ struct Gpu {
   int64_t clk_new[4] = {0, 0, 0, 0};
   std::atomic<uint64_t> clk_req{0}, clk_applied{0};
   FILE* log = nullptr;
+  bool log_times = false;   // PAELLA_TRACE_TIMES: host-time events (EV_TIME) for timelines
   std::mutex log_mu;
   paella_stats_t stats{};
   std::vector<Issue> issues;

@@ -117,7 +117,8 @@ def _serve(e, mids, n, n_clients, seed, stride=16384, timeout=60):
     (L.POLICY_SJF, 100, 16, 8, 0, 1), (L.POLICY_SJF, 100, 4, 4, 2, 2),
     (L.POLICY_RR, 100, 16, 8, 0, 1), (L.POLICY_RR, 100, 4, 12, 1, 3),
     (L.POLICY_SRPT_DEFICIT, 100, 16, 8, 0, -1), (L.POLICY_SRPT_DEFICIT, None, 4, 12, 2, -3),
-    (L.POLICY_SJF, 3, 16, 8, 1, -1)])
+    (L.POLICY_SJF, 3, 16, 8, 1, -1), (L.POLICY_SRPT_DEFICIT, 100, 16, 8, 6, 1),
+    (L.POLICY_FIFO, 100, 1, 16, 7, 1)])
 def test_fake_device_replay_parity(tmp_path, policy, theta, group, streams, look, prio):
     """prio < 0: |prio| classes with NEXT-4 online T-bar refinement (OBSERVE events)."""
     log = str(tmp_path / "ev_%u.log")
@@ -261,7 +262,8 @@ def test_route_pair_matches_oracle():
 
 @pytest.mark.parametrize("policy,theta,K,look", [
     (L.POLICY_SRPT_DEFICIT, 100, 2, 0), (L.POLICY_SRPT_DEFICIT, None, 3, 2), (L.POLICY_SRPT_DEFICIT, 0, 1, 1),
-    (L.POLICY_FIFO, 100, 2, 3), (L.POLICY_SJF, 100, 4, 1), (L.POLICY_RR, 100, 2, 0)])
+    (L.POLICY_FIFO, 100, 2, 3), (L.POLICY_SJF, 100, 4, 1), (L.POLICY_RR, 100, 2, 0),
+    (L.POLICY_SRPT_DEFICIT, 100, 3, 6)])
 def test_fake_replay_max_active(tmp_path, policy, theta, K, look):
     """B200-Q6 (max_active = K): the C++ dispatcher's decisions with the job cap replay
     bit-exactly through the oracle policy; at most K capped jobs (plus deficit

@@ -55,5 +55,8 @@ for v in variants:
            "stop": st["stop_reason"], "avg_ready": round(st["sum_ready"] / dc, 2),
            "avg_live": round(st["sum_live_jobs"] / dc, 2), "avg_Q": round(st["sum_Q"] / dc, 1),
            "launches": st["launches"], "decides": st["decide_calls"]}
+    if st.get("ev_launches"):   # event_time_kind: mean CUDA-event duration of that kernel kind
+        res["ev_mean_us"] = round(st["ev_ns"] / st["ev_launches"] / 1e3, 3)
+        res["ev_launches"] = st["ev_launches"]
     print(json.dumps(res), flush=True)
     e.shutdown()
