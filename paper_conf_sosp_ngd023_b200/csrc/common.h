@@ -93,7 +93,11 @@ enum : uint32_t {
   LF_CEIL = 2u,       // maxpool ceil mode
   LF_FINAL = 4u,      // output is the fp32 logits in client memory
   LF_RESIDUAL = 8u,
-  LF_TRACE = 16u,     // debug: per-CTA phase timestamps (globaltimer) into ws
+  LF_TRACE = 16u,     // debug: per-CTA phase timestamps (globaltimer) into trace
+  LF_SPLIT_DSMEM = 32u,   // split-K reduced over DSMEM (round-2 design, A/B) instead of in L2
+  LF_SPLIT_NOROT = 64u,   // (A/B) L2 split-K: every CTA reduces its rows in tile order
+  LF_SPLIT_RELBAR = 128u, // (A/B) L2 split-K: release/acquire cluster barrier instead of a
+                          // relaxed one after the reducing thread's own fence
 };
 
 struct LayerArgs {
@@ -115,8 +119,8 @@ struct LayerArgs {
   uint32_t tiles_m, tiles_n;// tcgen05 conv: tile grid
   uint32_t ksplit;          // split-K factor (1 = none)
   uint32_t a_rows;          // tcgen05 conv: weight rows fetched per stage (TMA box), <= 128
-  float* ws;                // fp32 split-K workspace
-  uint32_t* ws_ctr;         // split-K arrival counters (one per output tile)
+  float* ws;                // split-K: fp32 partial sums, 64 x 128 per output tile, all zero between uses
+  uint64_t* trace;          // debug (LF_TRACE): per-CTA phase timestamps
 };
 
 }  // namespace paella

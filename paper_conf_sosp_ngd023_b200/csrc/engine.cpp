@@ -1535,8 +1535,8 @@ int paella_shutdown(paella_t* p) {
         cudaSetDevice(P->gpus[gi]->device);
         cudaFree(m->gpu[gi].weights);
         cudaFree(m->gpu[gi].workspace);
-        if (m->gpu[gi].splitk_ws) cudaFree(m->gpu[gi].splitk_ws);
-        if (m->gpu[gi].splitk_ctr) cudaFree(m->gpu[gi].splitk_ctr);
+        if (m->gpu[gi].splitk_iso) cudaFree(m->gpu[gi].splitk_iso);
+        if (m->gpu[gi].splitk_slots) cudaFree(m->gpu[gi].splitk_slots);
       } else {
         free(m->gpu[gi].weights);
         free(m->gpu[gi].workspace);
@@ -1764,7 +1764,7 @@ static int iso_run(Gpu* g, Model* m, const void* input, void* output, int64_t* k
     cudaMemsetAsync(trbuf, 0, 16 * 8 * m->kernels[trace_k].grid_total(), s);
     saved = args[trace_k];
     args[trace_k].flags |= LF_TRACE;
-    args[trace_k].ws = (float*)trbuf;
+    args[trace_k].trace = trbuf;
   } else {
     trace_k = -1;
   }
@@ -1900,25 +1900,33 @@ static int64_t time_layer_cold(Gpu* g, Model* m, uint32_t l, bool instr, uint32_
 // Split-K autotuning of the tcgen05 convs (GPU 0, at registration, before T-bar is
 // profiled): every admissible split (power of two, <= 16 = the cluster limit, >= 1
 // k-block per split, <= one wave at 2 CTAs/SM) is timed as served (instrumented, PDL
-// chain); a larger split must win by >= 5 % (it occupies more SMs under load).
-// PAELLA_SPLITS_FILE: a cache of the choices ("model layer split" lines): read if it
-// exists (profiling runs reuse the served configuration without re-timing), appended to
-// otherwise.
+// chain) with each split-K reduction (in L2, or over DSMEM: neither wins on every layer,
+// profiles/r2/splitk_*); a larger split must win by >= 5 % (it occupies more SMs under
+// load).  PAELLA_SPLITS_FILE: a cache of the choices ("model layer split [dsmem]"
+// lines): read if it exists (profiling runs reuse the served configuration without
+// re-timing), appended to otherwise.
 static int autotune_splits(Gpu* g, Model* m) {
   if (std::getenv("PAELLA_NO_AUTOTUNE") || std::getenv("PAELLA_NOSPLIT")) return 0;
   auto& mg = m->gpu[g->index];
   const char* cache = std::getenv("PAELLA_SPLITS_FILE");
   if (cache) {
     if (FILE* f = std::fopen(cache, "r")) {
-      char name[256];
-      unsigned l, sp;
+      char line[512], name[256];
+      unsigned l, sp, dsm;
       bool any = false;
-      while (std::fscanf(f, "%255s %u %u", name, &l, &sp) == 3) {
+      while (std::fgets(line, sizeof line, f)) {
+        const int n = std::sscanf(line, "%255s %u %u %u", name, &l, &sp, &dsm);
+        if (n < 3) continue;
         if (m->name != name || l >= m->kernels.size() || !is_tc(m->kernels[l].kind)) continue;
         KernelInst& k = m->kernels[l];
+        const uint32_t fl = (n == 4 && dsm) ? (k.proto.flags | LF_SPLIT_DSMEM) : (k.proto.flags & ~LF_SPLIT_DSMEM);
         k.proto.ksplit = sp;
+        k.proto.flags = fl;
         k.grid[2] = sp;
-        for (auto& A : mg.args) A[l].ksplit = sp;
+        for (auto& A : mg.args) {
+          A[l].ksplit = sp;
+          A[l].flags = fl;
+        }
         any = true;
       }
       std::fclose(f);
@@ -1930,34 +1938,85 @@ static int autotune_splits(Gpu* g, Model* m) {
     KernelInst& k = m->kernels[l];
     if (!is_tc(k.kind)) continue;
     const uint32_t nk = k.proto.kpad / TC_BK, tiles = k.proto.tiles_m * k.proto.tiles_n;
-    auto set = [&](uint32_t sp) {
+    auto set = [&](uint32_t sp, bool dsm) {
       k.proto.ksplit = sp;
+      k.proto.flags = dsm ? (k.proto.flags | LF_SPLIT_DSMEM) : (k.proto.flags & ~LF_SPLIT_DSMEM);
       k.grid[2] = sp;
-      for (auto& A : mg.args) A[l].ksplit = sp;
+      for (auto& A : mg.args) {
+        A[l].ksplit = sp;
+        A[l].flags = k.proto.flags;
+      }
     };
     const uint32_t orig = k.proto.ksplit;
+    // PAELLA_SPLIT_DSMEM forces the DSMEM reduction, PAELLA_SPLIT_L2 the L2 one
+    const bool only_dsm = std::getenv("PAELLA_SPLIT_DSMEM") != nullptr, only_l2 = std::getenv("PAELLA_SPLIT_L2") != nullptr;
     uint32_t best = orig;
+    bool best_dsm = (k.proto.flags & LF_SPLIT_DSMEM) != 0;
     int64_t best_t = INT64_MAX;
     for (uint32_t sp = 1; sp <= 16 && sp <= nk && tiles * sp <= 2 * g->P->sms; sp *= 2) {
-      set(sp);
-      time_layer(g, m, l, true, 8);   // warm
-      const int64_t t = time_layer(g, m, l, true, 40);
-      if (t < 0) return -EIO;
-      if (best_t == INT64_MAX || t * 100 < best_t * 95) {
-        best_t = t;
+      int64_t t_sp = INT64_MAX;
+      bool dsm_sp = false;
+      for (int dsm = 0; dsm < 2; ++dsm) {
+        if ((dsm && only_l2) || (!dsm && only_dsm) || (dsm && sp == 1)) continue;
+        set(sp, dsm != 0);
+        time_layer(g, m, l, true, 8);   // warm
+        const int64_t t = time_layer(g, m, l, true, 40);
+        if (t < 0) return -EIO;
+        if (t < t_sp) {
+          t_sp = t;
+          dsm_sp = dsm != 0;
+        }
+      }
+      if (t_sp == INT64_MAX) continue;
+      if (best_t == INT64_MAX || t_sp * 100 < best_t * 95) {
+        best_t = t_sp;
         best = sp;
+        best_dsm = dsm_sp;
       }
     }
-    set(best);
+    set(best, best_dsm && best > 1);
     if (cache)
       if (FILE* f = std::fopen(cache, "a")) {
-        std::fprintf(f, "%s %u %u\n", m->name.c_str(), l, best);
+        std::fprintf(f, "%s %u %u %u\n", m->name.c_str(), l, best, best_dsm && best > 1 ? 1u : 0u);
         std::fclose(f);
       }
     if (std::getenv("PAELLA_AUTOTUNE_LOG"))
-      fprintf(stderr, "autotune %s layer %u: nk %u tiles %u split %u -> %u (%lld ns)\n", m->name.c_str(), l, nk,
-              tiles, orig, best, (long long)best_t);
+      fprintf(stderr, "autotune %s layer %u: nk %u tiles %u split %u -> %u%s (%lld ns)\n", m->name.c_str(), l, nk,
+              tiles, orig, best, best_dsm && best > 1 ? " dsmem" : "", (long long)best_t);
   }
+  return 0;
+}
+
+// Split-K partial-sum workspaces (ModelGpu::splitk_*; the tcgen05 conv reduces its
+// split-K partials in L2 with bulk fp32 reductions): per virtual stream, room for the
+// largest tile grid among the layers that may split there (iso: any tcgen05 layer --
+// autotuning and forced splits run in the isolated slot; else the layers whose chosen
+// split is > 1), TC_BN x TC_BM floats per output tile.  Zeroed once; every owner CTA
+// re-zeroes the sums it consumed, so the region is all zero between launches.
+static int splitk_workspace(Model* m, ModelGpu& mg, bool iso) {
+  constexpr size_t kTile = (size_t)TC_BN * TC_BM;
+  uint32_t nvs = 1;
+  for (const auto& k : m->kernels)
+    if (is_tc(k.kind)) nvs = std::max(nvs, k.vs + 1);
+  std::vector<size_t> off(nvs, 0), tiles(nvs, 0);
+  for (const auto& k : m->kernels)
+    if (is_tc(k.kind) && (iso || k.proto.ksplit > 1))
+      tiles[k.vs] = std::max<size_t>(tiles[k.vs], (size_t)k.proto.tiles_m * k.proto.tiles_n);
+  size_t per = 0;
+  for (uint32_t v = 0; v < nvs; ++v) {
+    off[v] = per;
+    per += tiles[v] * kTile;
+  }
+  if (per == 0) return 0;
+  const size_t first = iso ? mg.args.size() - 1 : 0, nsl = iso ? 1 : mg.args.size() - 1;
+  float* ws = nullptr;
+  if (cudaMalloc((void**)&ws, nsl * per * sizeof(float))) return -ENOMEM;
+  cudaMemset(ws, 0, nsl * per * sizeof(float));
+  if (cudaStreamSynchronize(0) != cudaSuccess) return -EIO;   // legacy-stream memset vs. our streams
+  (iso ? mg.splitk_iso : mg.splitk_slots) = ws;
+  for (size_t s = 0; s < nsl; ++s)
+    for (uint32_t l = 0; l < m->kernels.size(); ++l)
+      if (is_tc(m->kernels[l].kind)) mg.args[first + s][l].ws = ws + s * per + off[m->kernels[l].vs];
   return 0;
 }
 
@@ -1975,12 +2034,6 @@ static int setup_model_gpu(Paella* P, Model* m, Gpu* g) {
     if (cudaMalloc((void**)&wsp, nslot * m->slot_bytes)) return -ENOMEM;
     cudaMemset(wsp, 0, nslot * m->slot_bytes);
     cudaStreamSynchronize(0);   // legacy-stream memset vs. our non-blocking streams
-    if (m->splitk_floats) {
-      if (cudaMalloc((void**)&mg.splitk_ws, nslot * m->splitk_floats * 4)) return -ENOMEM;
-      if (cudaMalloc((void**)&mg.splitk_ctr, nslot * m->splitk_ctrs * 4)) return -ENOMEM;
-      cudaMemset(mg.splitk_ctr, 0, nslot * m->splitk_ctrs * 4);
-      cudaStreamSynchronize(0);
-    }
   } else {
     wdev = (uint8_t*)malloc(m->blob.size() + 256);
     wsp = (uint8_t*)calloc(1, 256);   // the fake device never touches activations
@@ -2046,19 +2099,25 @@ static int setup_model_gpu(Paella* P, Model* m, Gpu* g) {
       a.bias = (const float*)(wdev + k.b_off);
       a.pro_scale = k.has_pro ? (const float*)(wdev + k.ps_off) : nullptr;
       a.pro_shift = k.has_pro ? (const float*)(wdev + k.pz_off) : nullptr;
-      if (cuda && mg.splitk_ws) {
-        a.ws = mg.splitk_ws + s * m->splitk_floats;
-        a.ws_ctr = mg.splitk_ctr + s * m->splitk_ctrs;
-      }
       A[l] = a;
     }
   }
   mg.free_slots.clear();
   for (uint32_t s = slots; s-- > 0;) mg.free_slots.push_back(s);
+  if (cuda) {
+    const int rc = splitk_workspace(m, mg, true);
+    if (rc) return rc;
+  }
+  // split factors: GPU 0 tunes them (the other GPUs are set up afterwards from the
+  // tuned prototypes), then the serving slots' workspaces are sized for them
+  if (g->index == 0 && cuda && autotune_splits(g, m)) return -EIO;
+  if (cuda) {
+    const int rc = splitk_workspace(m, mg, false);
+    if (rc) return rc;
+  }
   // profile T-bar (P1249-1254; reading C2-Q15): GPU 0 measures, others copy
   if (g->index == 0) {
     uint32_t runs = 20;
-    if (cuda && autotune_splits(g, m)) return -EIO;
     if (cuda) {
       std::vector<int64_t> t(m->kernels.size()), acc(m->kernels.size(), 0);
       for (int w = 0; w < 5; ++w)

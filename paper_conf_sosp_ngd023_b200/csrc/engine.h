@@ -57,8 +57,12 @@ struct TmapStore {           // CUtensorMap storage (64-byte aligned, 128 bytes)
 struct ModelGpu {
   void* weights = nullptr;     // device blob (packed weights + fp32 vectors)
   void* workspace = nullptr;   // slots * slot_bytes (+1 isolated slot)
-  float* splitk_ws = nullptr;  // split-K fp32 partials, per slot
-  uint32_t* splitk_ctr = nullptr;
+  // split-K partial sums (fp32, TC_BN x TC_BM per output tile, all zero between uses):
+  // the isolated slot's (sized for any split of any layer: autotuning, forced splits)
+  // and the serving slots' (sized for the chosen splits); per virtual stream (NEXT-4
+  // branches of one job run concurrently)
+  float* splitk_iso = nullptr;
+  float* splitk_slots = nullptr;
   std::vector<std::vector<LayerArgs>> args;   // [slot][kernel]
   std::vector<uint32_t> free_slots;
   std::vector<TmapStore> tmaps;   // per kernel (tcgen05 conv weights)
@@ -73,7 +77,6 @@ struct Model {
   std::vector<uint32_t> coff;             // node -> channel offset in its buffer
   std::vector<Buffer> bufs;
   size_t slot_bytes = 0;
-  size_t splitk_floats = 0, splitk_ctrs = 0;
   std::vector<KernelInst> kernels;
   std::vector<uint8_t> blob;              // host copy of the packed parameters
   size_t input_bytes = 0, output_bytes = 0;

@@ -18,8 +18,10 @@
 //    owns TMEM lanes 32w..32w+31 = 32 output channels), add bias, residual (fp32),
 //    activation, round once to bf16 (reading C1-Q7) and store NHWC;
 //  * split-K over blockIdx.z for the deep, narrow late layers: the ksplit CTAs of a
-//    tile form a thread-block cluster; partial tiles stay in shared memory and are
-//    reduced over DSMEM, each CTA finishing a 1/ksplit slice of the tile.
+//    tile form a thread-block cluster; each adds its partial tile into an fp32 workspace
+//    with one bulk L2 reduction, and after a cluster barrier each CTA finishes a
+//    1/ksplit slice of the tile from the sums (LF_SPLIT_DSMEM: the previous reduction
+//    over DSMEM, kept for A/B measurements).
 //
 // Block instrumentation (K1) wraps the whole CTA (instr.cuh).
 #include <cuda.h>
@@ -74,6 +76,7 @@ __device__ __forceinline__ void cp_async_wait() {
   asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
 }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async_global() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 
@@ -218,7 +221,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     k_conv_tc(const __grid_constant__ LayerArgs a, const __grid_constant__ InstrArgs ia,
               const __grid_constant__ CUtensorMap wmap) {
   const bool trace = (a.flags & LF_TRACE) != 0;
-  uint64_t* tr = trace ? reinterpret_cast<uint64_t*>(a.ws) +
+  uint64_t* tr = trace ? a.trace +
                              16 * ((blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x)
                        : nullptr;
   if (trace && threadIdx.x == 0) tr[0] = globaltimer();
@@ -550,8 +553,95 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
         }
       }
     }
+  } else if (!(a.flags & LF_SPLIT_DSMEM)) {
+    // split-K across the CTAs of a cluster (1 x 1 x ksplit), reduced in L2: every CTA
+    // adds its staged partial tile (only the rows holding pixels) into the tile's fp32
+    // workspace with ONE bulk reduction (cp.reduce.async.bulk .add.f32: the adds run in
+    // the L2, the SM streams the tile out at its store bandwidth instead of pushing it
+    // over DSMEM at ~20 B/cycle and summing ks slices itself); after one cluster barrier
+    // CTA r reads the sums of its 1/ksplit slice of pixel rows from L2, writes zeros back
+    // (the workspace is all zero between launches) and runs the epilogue for them.  The
+    // fp32 additions happen in L2 in arrival order (one bf16 rounding afterwards).
+    // Items of thread t: pixel rows px0 + (t + 128 i) / 16 (i < 4), channel group t % 16.
+    constexpr uint32_t MAXI = TC_BN * (TC_BM / 8) / (2 * NPROD);   // 4 items at ksplit 2
+    const uint32_t ks = a.ksplit;
+    const uint32_t rows = TC_BN / ks;
+    const uint32_t px0 = split * rows;
+    const uint32_t g = threadIdx.x % (TC_BM / 8), co = m0 + g * 8;
+    const uint32_t nitems = rows * (TC_BM / 8);
+    const uint32_t rv = n0 >= P ? 0u : min(TC_BN, P - n0);   // pixel rows of the tile that exist
+    float* wt = a.ws + (size_t)(tile_m * gridDim.x + tile_n) * (TC_BN * TC_BM);
+    float bias[8];
+    uint4 rres[MAXI];
+    if (warp < 4 && co < a.cout) {
+      load_bias8(a, co, bias);
+      if (a.flags & LF_RESIDUAL) {
+#pragma unroll
+        for (uint32_t i = 0; i < MAXI; ++i) {
+          const uint32_t item = threadIdx.x + i * NPROD;
+          const uint32_t p = n0 + px0 + item / (TC_BM / 8);
+          if (item < nitems && p < P) rres[i] = load_res8(a, p, co);
+        }
+      }
+    }
+    if (warp < 4) {
+      fence_proxy_async();                                 // staged rows -> the async proxy
+      asm volatile("bar.sync 1, 128;" ::: "memory");      // all 4 staging warps are done
+      if (threadIdx.x == 0 && nkl > 0 && rv > 0) {
+        // rotated by the CTA's own slice (two bulk ranges) so that the ks CTAs of the
+        // cluster start on different L2 lines instead of all adding into row 0 first
+        const uint32_t r0 = (a.flags & LF_SPLIT_NOROT) ? 0u : min(px0, rv);
+        const uint32_t sb = su32(stage);
+        if (rv > r0)
+          asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.add.f32 [%0], [%1], %2;" ::"l"(
+                           wt + r0 * TC_BM),
+                       "r"(sb + r0 * TC_BM * 4), "r"((rv - r0) * TC_BM * 4)
+                       : "memory");
+        if (r0 > 0)
+          asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.add.f32 [%0], [%1], %2;" ::"l"(wt),
+                       "r"(sb), "r"(r0 * TC_BM * 4)
+                       : "memory");
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // the adds are performed
+        asm volatile("fence.proxy.async.global;" ::: "memory");      // ... before the generic release
+        if (!(a.flags & LF_SPLIT_RELBAR)) asm volatile("fence.acq_rel.cluster;" ::: "memory");
+      }
+    }
+    if (trace && threadIdx.x == 0) tr[9] = globaltimer();
+    __syncwarp();
+    // every CTA's additions are complete and visible cluster-wide: the one thread that
+    // issued them released them with its fence; the barrier then only needs to order
+    // (relaxed arrive) and every reader acquires after it
+    if (a.flags & LF_SPLIT_RELBAR)
+      asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    else
+      asm volatile("barrier.cluster.arrive.relaxed.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    if (trace && threadIdx.x == 0) tr[10] = globaltimer();
+    if (warp < 4 && co < a.cout) {
+#pragma unroll
+      for (uint32_t i = 0; i < MAXI; ++i) {
+        const uint32_t item = threadIdx.x + i * NPROD;
+        const uint32_t r = item / (TC_BM / 8), p = n0 + px0 + r;
+        if (item < nitems && p < P) {
+          float* q = wt + (px0 + r) * TC_BM + g * 8;
+          float v[8];
+          asm volatile("ld.relaxed.gpu.global.L1::no_allocate.v4.f32 {%0, %1, %2, %3}, [%4];"
+                       : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3])
+                       : "l"(q));
+          asm volatile("ld.relaxed.gpu.global.L1::no_allocate.v4.f32 {%0, %1, %2, %3}, [%4];"
+                       : "=f"(v[4]), "=f"(v[5]), "=f"(v[6]), "=f"(v[7])
+                       : "l"(q + 4));
+          asm volatile("st.global.v4.f32 [%0], {%1, %1, %1, %1};\n\tst.global.v4.f32 [%2], {%1, %1, %1, %1};" ::"l"(q),
+                       "f"(0.f), "l"(q + 4)
+                       : "memory");
+          epi_store8(a, p, co, v, bias, rres[i]);
+        }
+      }
+      fence_proxy_async_global();   // the zeros, before a later grid's bulk reductions
+    }
+    if (trace && threadIdx.x == 0) tr[14] = globaltimer();
   } else {
-    // split-K across the CTAs of a cluster (1 x 1 x ksplit): CTA r owns a 1/ksplit
+    // (A/B, LF_SPLIT_DSMEM) split-K across the CTAs of a cluster (1 x 1 x ksplit): CTA r owns a 1/ksplit
     // slice of the tile's pixel rows.  Every CTA PUSHES the other slices of its staged
     // partial tile to their owners with one bulk DSMEM copy each (cp.async.bulk
     // shared::cta -> shared::cluster, completing on the owner's mbarrier); the owner

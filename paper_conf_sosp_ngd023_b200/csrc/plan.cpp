@@ -167,7 +167,6 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
     m->kernels.push_back(k);
   }
 
-  size_t max_splitk = 0, max_tiles = 0;
   // GAP whose only consumer is an FC: fused into one gap_fc kernel
   std::vector<uint32_t> consumers(n, 0);
   for (uint32_t i = 0; i < n; ++i) {
@@ -286,6 +285,9 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
                 while (split < 16 && tiles * split * 2 <= P->sms && nk / (split * 2) >= min_st) split *= 2;
             }
             a.ksplit = split;
+            if (std::getenv("PAELLA_SPLIT_DSMEM")) a.flags |= LF_SPLIT_DSMEM;   // A/B: the DSMEM reduction
+            if (std::getenv("PAELLA_SPLIT_NOROT")) a.flags |= LF_SPLIT_NOROT;
+            if (std::getenv("PAELLA_SPLIT_RELBAR")) a.flags |= LF_SPLIT_RELBAR;
             // narrow layers: fetch only the live weight rows (SW128 atoms are 8 rows)
             a.a_rows = nd.c < TC_BM ? (uint32_t)align_up(nd.c, 8) : TC_BM;
             k.grid[0] = a.tiles_n;
@@ -431,8 +433,6 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
     m->kernels.push_back(k);
   }
   if (!exact && es == 2) return -EINVAL;   // bf16 path requires bf16-representable weights
-  m->splitk_floats = max_splitk;
-  m->splitk_ctrs = max_tiles;
 
   // ---- NEXT-4: the kernel DAG and its virtual streams (Fig. 7 waitlists) ----
   // producers(node) = the kernels that write node's tensor: its own kernel, or through a

@@ -76,16 +76,17 @@ def test_isolated_fp32_parity(engine, name):
 
 @pytest.mark.parametrize("name", ["resnet18", "densenet121"])
 def test_forced_split_k_parity(engine, name, tmp_path, monkeypatch):
-    """Every cluster split-K factor the autotuner may pick (1..16, DSMEM reduction,
-    including splits with empty k-ranges), forced on every tcgen05 layer through the
-    split cache (PAELLA_SPLITS_FILE), stays within the bf16 tolerance."""
+    """Every cluster split-K factor the autotuner may pick (1..16, including splits with
+    empty k-ranges) with either split-K reduction (bulk fp32 adds in L2, or pushes over
+    DSMEM), forced on every tcgen05 layer through the split cache (PAELLA_SPLITS_FILE),
+    stays within the bf16 tolerance."""
     g = archs.build(name)
     P = rng.model_params(g)
     ref = oracle_out(name, 0, "bf16")
-    for sp in (1, 2, 4, 8, 16):
-        mname = f"{name}-split{sp}"
-        f = tmp_path / f"splits{sp}.txt"
-        f.write_text("".join(f"{mname} {l} {sp}\n" for l in range(len(g.nodes) + 2)))
+    for sp, dsm in ((1, 0), (2, 0), (4, 0), (8, 0), (16, 0), (2, 1), (4, 1), (8, 1), (16, 1)):
+        mname = f"{name}-split{sp}-{dsm}"
+        f = tmp_path / f"splits{sp}-{dsm}.txt"
+        f.write_text("".join(f"{mname} {l} {sp} {dsm}\n" for l in range(len(g.nodes) + 2)))
         monkeypatch.setenv("PAELLA_SPLITS_FILE", str(f))
         mid = engine.register_model(g, P, dtype=L.DTYPE_BF16, name=mname)
         monkeypatch.delenv("PAELLA_SPLITS_FILE")
@@ -93,7 +94,9 @@ def test_forced_split_k_parity(engine, name, tmp_path, monkeypatch):
         assert any(k["name"].startswith("conv_tcgen05") and k["grid"] % sp == 0 for k in ks)
         out = engine.run_isolated(mid, rng.image(g, 0))
         ok = within(out, ref, BF16_TOL)
-        assert ok.all(), f"{name} split {sp}: max err {np.abs(out - ref).max()}"
+        assert ok.all(), f"{name} split {sp} dsmem {dsm}: max err {np.abs(out - ref).max()}"
+        out2 = engine.run_isolated(mid, rng.image(g, 0))   # the workspace is zero again
+        assert within(out2, ref, BF16_TOL).all(), f"{name} split {sp} dsmem {dsm}: second run"
 
 
 def _serve_and_check(e, specs, n, n_clients, seed, rate_us=30.0):
