@@ -95,7 +95,11 @@ def parse():
     ap.add_argument("--dispatcher-cpu", type=int, default=-2,
                     help="first dispatcher core (-1 = unpinned; default: NUMA-local cores of each GPU, "
                          "else 2, 3, ...)")
-    ap.add_argument("--launch-threads", type=int, default=4, help="launcher helper threads per GPU")
+    ap.add_argument("--launch-threads", type=int, default=8,
+                    help="launcher helper threads per GPU of the paella arms (B200 sweep, profiles/r2/diag/lt_*: "
+                         "8 serve C-3 at 6-8k req/s with 16-35 %% lower mean JCT than 4)")
+    ap.add_argument("--naive-launch-threads", type=int, default=4,
+                    help="launcher helper threads per GPU of the naive arms (their best: 8 is 1.5-3x worse)")
     ap.add_argument("--slo-reqs", type=int, default=1500, help="requests per point of the SLO search")
     ap.add_argument("--no-slo", action="store_true", help="skip the req/s-at-SLO search (value = served req/s)")
     ap.add_argument("--no-c5", action="store_true", help="skip the notification microbenchmarks")
@@ -406,8 +410,10 @@ def run_gpu(args, ngpus, cores, fake):
     pol = {"srpt": L.POLICY_SRPT_DEFICIT, "fifo": L.POLICY_FIFO, "sjf": L.POLICY_SJF, "rr": L.POLICY_RR}
     # launcher helper threads spin on their queues: keep dispatchers + helpers within the host
     ncores = len(os.sched_getaffinity(0))
-    lt = min(args.launch_threads, max(1, (ncores - 2 - ngpus) // max(1, ngpus)))
-    common = dict(launch_threads=0 if fake else lt, max_jobs_per_model=128)
+    lt_cap = max(1, (ncores - 2 - ngpus) // max(1, ngpus))
+    lt = min(args.launch_threads, lt_cap)
+    lt_naive = min(args.naive_launch_threads, lt_cap)
+    common = dict(max_jobs_per_model=128)
     if cores:
         common["dispatcher_cpus"] = cores
     paella_kw = dict(policy=pol[args.policy], theta=args.theta, decide_delay_ns=args.decide_delay_ns,
@@ -433,10 +439,12 @@ def run_gpu(args, ngpus, cores, fake):
                          [a for a in args.arms.split(",") if a and a != "paella" and a in arms_kw])
 
     def arm(label, n=ngpus):
-        return Arm(L, label, specs, pool, n, region, stride, slots, fake, **common, **arms_kw[label])
+        kw = dict(arms_kw[label])
+        kw["launch_threads"] = 0 if fake else (lt_naive if kw.get("naive") else lt)
+        return Arm(L, label, specs, pool, n, region, stride, slots, fake, **common, **kw)
 
     detail = {"config": args.config, "models": names, "n_gpus": ngpus, "dispatcher_cpus": cores,
-              "launch_threads_per_gpu": common["launch_threads"], "host_cores": ncores}
+              "launch_threads_per_gpu": {"paella_arms": lt, "naive_arms": lt_naive}, "host_cores": ncores}
     # --- calibration (untimed): naive X_sat on ONE GPU, unloaded JCT -> SLO ---------------
     t_cal = time.time()
     a1 = arm("naive", 1)
