@@ -30,10 +30,10 @@ slots = 64
 region = slots * stride + (1 << 20)
 cuda = ctypes.CDLL("libcuda.so.1")
 t, mm, ii = bench.make_trace(n, rate, cfg, len(names), seed=77)
-for label, kw in (("paella", dict(policy=L.POLICY_SRPT_DEFICIT, slack=1184, lookahead=3, max_active=8)),
+for label, kw in (("paella", dict(policy=L.POLICY_SRPT_DEFICIT, slack=3552, lookahead=6, max_active=8, launch_threads=8)),
                   ("naive", dict(naive=True, instrument=False))):
-    a = bench.Arm(L, label, specs, pool, 1, region, stride, slots, False, launch_threads=4, max_jobs_per_model=64,
-                  **kw)
+    a = bench.Arm(L, label, specs, pool, 1, region, stride, slots, False,
+                  **dict(dict(launch_threads=4, max_jobs_per_model=64), **kw))
     a.serve(*bench.make_trace(40, rate, cfg, len(names), seed=5))   # warm, unprofiled
     ctx = ctypes.c_void_p()
     cuda.cuDevicePrimaryCtxRetain(ctypes.byref(ctx), 0)

@@ -31,12 +31,13 @@ sizes = [int(np.prod(g.nodes[0]["out"])) * 4 + g.num_classes * 4 for (g, _) in s
 stride = (max(sizes) + 4095) // 4096 * 4096
 slots = 256
 region = slots * stride + (1 << 20)
-common = dict(launch_threads=4, max_jobs_per_model=128, dispatcher_cpus=[2])
+common = dict(max_jobs_per_model=128, dispatcher_cpus=[2])
+# the bench's arm configurations (bench.py defaults: each arm with its best launcher count)
 arms = {
-    "naive": dict(naive=True, instrument=False),
-    "naive_pdl": dict(naive=True, instrument=False, naive_pdl=True),
-    "paella": dict(policy=L.POLICY_SRPT_DEFICIT, theta=100, slack=1184, lookahead=3, max_active=8),
-    "paella_fifo": dict(policy=L.POLICY_FIFO, slack=1184, lookahead=3, max_active=8),
+    "naive": dict(naive=True, instrument=False, launch_threads=4),
+    "naive_pdl": dict(naive=True, instrument=False, naive_pdl=True, launch_threads=4),
+    "paella": dict(policy=L.POLICY_SRPT_DEFICIT, theta=100, slack=3552, lookahead=6, max_active=8, launch_threads=8),
+    "paella_fifo": dict(policy=L.POLICY_FIFO, slack=3552, lookahead=6, max_active=8, launch_threads=8),
 }
 out = open(f"gpurun_out/rho_sweep_{tag}.jsonl", "w")
 # calibration per config on the naive arm: unloaded medians (mix weights), X_sat bisection
