@@ -296,6 +296,7 @@ def test_serving_parity_c3_models_bench_arm(tmp_path):
     ok, msg, n = sim.replay(cfg, ms, events)
     assert ok, msg
     assert n == len(ex["issues"]) == st["launches"]
+    assert sim.check_inflight_bound(events, ms, 6) == []
 
 
 @pytest.mark.parametrize("name", ["resnet18", "inception_v3"])

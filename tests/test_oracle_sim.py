@@ -492,7 +492,7 @@ def _chain(L, d):
     return [[Layer(1, (1, 1, 1, 1, 0), d, d) for _ in range(L)]]
 
 
-@pytest.mark.parametrize("D", [0, 1, 2, 3])
+@pytest.mark.parametrize("D", [0, 1, 2, 3, 6, 7])
 def test_launch_ahead_closed_form_zero_delay(D):
     """One job of L single-block kernels of duration d, zero launch/notification delay:
     at t = 0 kernels 0..D are issued (each new one is queued behind a fully placed
@@ -500,7 +500,7 @@ def test_launch_ahead_closed_form_zero_delay(D):
     is issued.  So kernel k is issued at max(0, (k - D) d), and JCT = L d for every D.
     A rule that looked at the NEWEST in-flight kernel instead of the oldest would issue
     only one kernel ahead; one that ignored D would issue all L at t = 0."""
-    Lk, d = 6, 1000
+    Lk, d = 10, 1000   # longer than D + 1 for every D tested (the bench runs D = 6)
     cfg = Config(num_clients=1, theta=sim.INF_THETA, slack=10**6, lookahead=D,
                  capacity=(10**6, 10**9, 10**12, 10**12, 10**9))
     res = sim.simulate(cfg, _chain(Lk, d), [(0, 0, 0)], GPUModel(sms=1, per_sm=(1, 64, 65536, 233472, 512)))
@@ -528,7 +528,7 @@ def test_launch_ahead_closed_form_with_delays():
         assert res.jct()[0] == want_jct * u
 
 
-@pytest.mark.parametrize("D", [0, 1, 3])
+@pytest.mark.parametrize("D", [0, 1, 3, 6])
 def test_inflight_bound_checker(D):
     """check_inflight_bound accepts every simulator log at its own depth; on the chain of
     test_launch_ahead_closed_form_zero_delay (depth D + 1 reached at t = 0) it rejects
@@ -541,7 +541,7 @@ def test_inflight_bound_checker(D):
     trace = random_trace(r, 30, 2, len(models), rate_ns=3000)
     res = _run_policy_with_log(cfg, models, trace, gpu)
     assert sim.check_inflight_bound(res.policy.log, models, D) == []
-    chain = _chain(6, 1000)
+    chain = _chain(10, 1000)
     cfg1 = Config(num_clients=1, theta=sim.INF_THETA, slack=10**6, lookahead=D,
                   capacity=(10**6, 10**9, 10**12, 10**12, 10**9))
     res1 = _run_policy_with_log(cfg1, chain, [(0, 0, 0)], GPUModel(sms=1, per_sm=(1, 64, 65536, 233472, 512)))
