@@ -2,8 +2,6 @@
 #pragma once
 #include <stdint.h>
 
-#include "common.h"
-
 namespace paella {
 
 enum KernelKind : uint32_t {
@@ -37,18 +35,7 @@ void tc_kernel_table(KernelFn* instr, KernelFn* plain);
 constexpr uint32_t TC_BM = 128;       // Cout rows per CTA (UMMA M, TMEM lanes)
 constexpr uint32_t TC_BN = 64;        // output pixels per CTA (UMMA N)
 constexpr uint32_t TC_BK = 64;        // K per pipeline stage (128 B of bf16 = one swizzle row)
-constexpr uint32_t TC_STAGES = 4;         // pipeline depth of full-width (Cout >= 128) layers
-constexpr uint32_t TC_MAXSTAGES = 8;      // ... of narrow layers (fewer weight rows per stage)
-constexpr uint32_t TC_RING = TC_STAGES * (TC_BM * TC_BK * 2 + TC_BN * TC_BK * 2);   // 96 KiB of stages
-// Stages of a layer fetching a_rows weight rows: A stages are a_rows x 128 B apart (the
-// UMMA still reads 128 rows from each stage base: rows past a_rows are the next stages'
-// data -- accumulator lanes that are never stored), so narrow layers fit deeper rings in
-// the same 96 KiB: 4 (128 rows), 5 (64), 7 (32), 8 (<= 16).
-PAELLA_HD constexpr uint32_t tc_stages(uint32_t a_rows) {
-  return (TC_RING - (TC_BM - a_rows) * 128) / (a_rows * 128 + TC_BN * TC_BK * 2) < TC_MAXSTAGES
-             ? (TC_RING - (TC_BM - a_rows) * 128) / (a_rows * 128 + TC_BN * TC_BK * 2)
-             : TC_MAXSTAGES;
-}
+constexpr uint32_t TC_STAGES = 4;
 constexpr uint32_t GAPFC_CLUSTER = 8;   // fused GAP+FC head: CTAs per cluster (pooling split)
 constexpr uint32_t TC_THREADS = 192;    // 4 producer/epilogue warps + 1 MMA warp + 1 bookkeeping warp
 uint32_t tc_smem_bytes();

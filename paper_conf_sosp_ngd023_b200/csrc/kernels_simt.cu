@@ -454,36 +454,17 @@ __global__ void __launch_bounds__(256) k_fc(const __grid_constant__ LayerArgs a,
 // between the two, reading C1-Q7: one rounding per fused layer).
 // ---------------------------------------------------------------------------
 template <typename T, bool INSTR>
-__global__ void __launch_bounds__(256, 1) k_gapfc(const __grid_constant__ LayerArgs a,
+__global__ void __launch_bounds__(256) k_gapfc(const __grid_constant__ LayerArgs a,
                                                const __grid_constant__ InstrArgs ia) {
   // Batch-1 latency layout: clusters of GAPFC_CLUSTER CTAs; the CTAs of a cluster
   // pool 1/GAPFC_CLUSTER of the channels each, exchange the pooled slices over DSMEM,
   // then every warp computes one FC row (8 rows per CTA, ~128 CTAs for 1000 classes:
-  // the weight stream is spread over many SMs).  The weights do not depend on the
-  // predecessor: each warp fetches its row (bf16, up to 2,048 columns) into registers
-  // BEFORE the programmatic-dependent-launch wait, so the weight stream overlaps the
-  // predecessor's tail instead of following the pooling.
-  instr_enter<INSTR>(ia);
+  // the weight stream is spread over many SMs).
+  kernel_begin<INSTR>(ia);
   extern __shared__ float pooled[];   // [C], every CTA ends up with all of it
   const T* X = static_cast<const T*>(a.in);
   const T* W = static_cast<const T*>(a.w);
   const uint32_t C = a.cin, HW = a.h * a.w_, NG = C / 8;
-  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-  const int row = blockIdx.x * (blockDim.x / 32) + warp;
-  constexpr uint32_t PF = sizeof(T) == 2 ? 8 : 0;   // prefetched 8-column chunks per lane
-  uint4 wpf[PF > 0 ? PF : 1];
-  if constexpr (PF > 0) {
-    // unpredicated (columns past C re-read column 0; rows past cout read row 0): the
-    // registers stay registers
-    const T* wr = W + (size_t)(row < (int)a.cout ? row : 0) * a.kpad;
-#pragma unroll
-    for (uint32_t j = 0; j < PF; ++j) {
-      const uint32_t k = lane * 8 + j * 256;
-      wpf[j] = __ldg(reinterpret_cast<const uint4*>(wr + (k < C ? k : 0u)));
-    }
-  }
-  pdl_wait();
-  pdl_trigger();
   const float inv = 1.f / (float)HW;
   uint32_t rank;
   asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
@@ -546,26 +527,13 @@ __global__ void __launch_bounds__(256, 1) k_gapfc(const __grid_constant__ LayerA
   // done reading the peers; the matching wait (peers stay resident) is at the end
   asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
   __syncthreads();
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int row = blockIdx.x * (blockDim.x / 32) + warp;
   if (row < (int)a.cout) {
     const T* wr = W + (size_t)row * a.kpad;
     float acc = 0.f;
-    if constexpr (PF > 0) {
-#pragma unroll
-      for (uint32_t j = 0; j < PF; ++j) {
-        const uint32_t k = lane * 8 + j * 256;
-        if (k < C) {
-          const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&wpf[j]);
-#pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            const float2 f = __bfloat1622float2(h[i]);
-            acc = fmaf(f.x, pooled[k + 2 * i], acc);
-            acc = fmaf(f.y, pooled[k + 2 * i + 1], acc);
-          }
-        }
-      }
-    }
 #pragma unroll 8
-    for (uint32_t k = lane * 8 + PF * 256; k < C; k += 32 * 8) {
+    for (uint32_t k = lane * 8; k < C; k += 32 * 8) {
       float wv[8];
       load8(wr + k, wv);
 #pragma unroll

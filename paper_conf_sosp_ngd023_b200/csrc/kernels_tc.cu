@@ -231,16 +231,11 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   // cast) keeps the shared address space visible to the compiler: LDS/STS, no
   // aliasing with global stores
   uint8_t* smem = smem_raw + ((1024u - (su32(smem_raw) & 1023u)) & 1023u);
-  // nst stages: A stage s at sA + s * abytes (a_rows weight rows; the UMMA reads 128 rows
-  // from there, rows past a_rows belong to the next stages: accumulator lanes >= a_rows
-  // are garbage and never stored), then nst B stages of 8 KiB; 96 KiB in all
-  const uint32_t abytes = a.a_rows * 128;
-  const uint32_t nst = tc_stages(a.a_rows);
-  uint8_t* sA = smem;
-  uint8_t* sB = smem + nst * abytes + (A_BYTES - abytes);
-  uint64_t* full = (uint64_t*)(smem + TC_RING);
-  uint64_t* empty = full + TC_MAXSTAGES;
-  uint64_t* accb = empty + TC_MAXSTAGES;
+  uint8_t* sA = smem;                                  // STAGES x 16 KiB
+  uint8_t* sB = smem + TC_STAGES * A_BYTES;            // STAGES x 8 KiB
+  uint64_t* full = (uint64_t*)(sB + TC_STAGES * B_BYTES);
+  uint64_t* empty = full + TC_STAGES;
+  uint64_t* accb = empty + TC_STAGES;
   uint64_t* rbar = accb + 1;                           // split-K: peers' slices landed
   uint32_t* tmem_slot = (uint32_t*)(rbar + 1);
   float* stage = reinterpret_cast<float*>(smem);       // epilogue tile [64 px][128 ch] fp32 (reuses sA)
@@ -255,11 +250,14 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   const uint32_t kb1 = min(nk, kb0 + per);
   const uint32_t nkl = kb1 > kb0 ? kb1 - kb0 : 0;
 
-  const uint32_t pre = nkl < nst ? nkl : nst;
+  const uint32_t pre = nkl < TC_STAGES ? nkl : TC_STAGES;
+  // narrow layers (Cout < 128) fetch only a_rows weight rows per stage; rows a_rows..127
+  // of every A stage are zeroed once below (the UMMA still runs M = 128)
+  const uint32_t abytes = a.a_rows * 128;
   if (warp == 4 && lane == 0) {
     // the MMA warp's leader sets up the barriers and starts the weight stream while
     // the gather warps compute their addresses
-    for (uint32_t s = 0; s < nst; ++s) {
+    for (uint32_t s = 0; s < TC_STAGES; ++s) {
       mbar_init(&full[s], NPROD + 1);
       mbar_init(&empty[s], 1);
     }
@@ -269,7 +267,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     if (trace) tr[11] = globaltimer();
     for (uint32_t it = 0; it < pre; ++it) {   // the first stages need no empty-wait
       mbar_arrive_tx(&full[it], abytes);
-      tma_load_2d(sA + it * abytes, &wmap, &full[it], (int)((kb0 + it) * TC_BK), (int)m0);
+      tma_load_2d(sA + it * A_BYTES, &wmap, &full[it], (int)((kb0 + it) * TC_BK), (int)m0);
     }
     if (trace) tr[12] = globaltimer();
   }
@@ -296,7 +294,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   int kr = 0, ks_ = 0, kci = 0;
   uint32_t kcur = 0;
   auto issue_B = [&](uint32_t it, bool arrive) {
-    const uint32_t s = it % nst;
+    const uint32_t s = it % TC_STAGES;
     const bool kv = kcur < K;
     const int dk = (kr * (int)a.w_ + ks_) * (int)a.in_cs + kci;
     const uint32_t bstage = su32(sB + s * B_BYTES) + dst0;
@@ -337,7 +335,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   int tr_r = 0, tr_s = 0, tr_ci = 0;
   uint32_t tr_k = 0;
   auto transform_B = [&](uint32_t it) {
-    const uint32_t bstage = su32(sB + (it % nst) * B_BYTES) + dst0;
+    const uint32_t bstage = su32(sB + (it % TC_STAGES) * B_BYTES) + dst0;
     if (tr_k < K) {
       const float4 s0 = __ldg(reinterpret_cast<const float4*>(a.pro_scale + tr_ci));
       const float4 s1 = __ldg(reinterpret_cast<const float4*>(a.pro_scale + tr_ci + 4));
@@ -396,6 +394,16 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       kr = rs / (int)a.kw;
       tr_k = kcur, tr_ci = kci, tr_s = ks_, tr_r = kr;
     }
+    if (a.a_rows < TC_BM) {
+      const uint32_t zb = A_BYTES - abytes;   // bytes per stage, multiple of 1024
+      for (uint32_t o = t * 16; o < TC_STAGES * zb; o += NPROD * 16) {
+        const uint32_t st = o / zb;
+        asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(su32(sA + st * A_BYTES + abytes + (o - st * zb))),
+                     "r"(0u)
+                     : "memory");
+      }
+      fence_proxy_async();   // visible to the tensor core (async proxy) after the CTA barrier
+    }
     // ... and the first activation gathers, before the CTA-wide barrier, once the
     // predecessor kernel's output is complete (PDL; the weight TMA above needs no wait)
     pdl_wait();
@@ -420,12 +428,12 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     if constexpr (!PRO) {
       for (uint32_t it = 0; it < pre; ++it)
         asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(su32(&full[it])) : "memory");
-      for (uint32_t nxt = nst; nxt < nkl; ++nxt) {
-        const uint32_t s = nxt % nst;
-        mbar_wait(&empty[s], ((nxt / nst) & 1) ^ 1);   // MMA of stage nxt - nst retired
+      for (uint32_t nxt = TC_STAGES; nxt < nkl; ++nxt) {
+        const uint32_t s = nxt % TC_STAGES;
+        mbar_wait(&empty[s], ((nxt / TC_STAGES) & 1) ^ 1);   // MMA of stage nxt - STAGES retired
         if (t == 0) {
           mbar_arrive_tx(&full[s], abytes);
-          tma_load_2d(sA + s * abytes, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
+          tma_load_2d(sA + s * A_BYTES, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
         }
         issue_B(nxt, true);
       }
@@ -433,27 +441,23 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       // prologue path: wait for this thread's own copies of stage it (cp.async groups,
       // STAGES in flight), transform them in place, publish to the async proxy, arrive
       for (uint32_t it = 0; it < nkl; ++it) {
-        const uint32_t issued = min(nkl, it + nst);
+        const uint32_t issued = min(nkl, it + TC_STAGES);
         switch (issued - it - 1) {
           case 0: cp_async_wait<0>(); break;
           case 1: cp_async_wait<1>(); break;
           case 2: cp_async_wait<2>(); break;
-          case 3: cp_async_wait<3>(); break;
-          case 4: cp_async_wait<4>(); break;
-          case 5: cp_async_wait<5>(); break;
-          case 6: cp_async_wait<6>(); break;
-          default: cp_async_wait<7>(); break;
+          default: cp_async_wait<3>(); break;
         }
         transform_B(it);
         fence_proxy_async();
-        mbar_arrive(&full[it % nst]);
-        const uint32_t nxt = it + nst;
+        mbar_arrive(&full[it % TC_STAGES]);
+        const uint32_t nxt = it + TC_STAGES;
         if (nxt < nkl) {
-          const uint32_t s = nxt % nst;
-          mbar_wait(&empty[s], ((nxt / nst) & 1) ^ 1);
+          const uint32_t s = nxt % TC_STAGES;
+          mbar_wait(&empty[s], ((nxt / TC_STAGES) & 1) ^ 1);
           if (t == 0) {
             mbar_arrive_tx(&full[s], abytes);
-            tma_load_2d(sA + s * abytes, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
+            tma_load_2d(sA + s * A_BYTES, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
           }
           issue_B(nxt, false);
           cp_async_commit();
@@ -473,12 +477,12 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     if (lane == 0) {
       constexpr uint32_t IDESC = idesc_bf16(TC_BM, TC_BN);
       for (uint32_t it = 0; it < nkl; ++it) {
-        const uint32_t s = it % nst;
-        mbar_wait(&full[s], (it / nst) & 1);
+        const uint32_t s = it % TC_STAGES;
+        mbar_wait(&full[s], (it / TC_STAGES) & 1);
         if (trace && it == 0) tr[2] = globaltimer();
         fence_proxy_async();   // the gathered B tile was written through the generic proxy
         tc_fence_after();
-        const uint32_t abase = su32(sA + s * abytes), bbase = su32(sB + s * B_BYTES);
+        const uint32_t abase = su32(sA + s * A_BYTES), bbase = su32(sB + s * B_BYTES);
 #pragma unroll
         for (uint32_t kk = 0; kk < TC_BK / 16; ++kk) {
           umma_bf16(tmem, sdesc_sw128(abase + kk * 32), sdesc_sw128(bbase + kk * 32), IDESC,
@@ -520,7 +524,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
         float v[16];
         tmem_ld16(taddr + c * 16, v);
 #pragma unroll
-        for (int i = 0; i < 16; ++i) stage[(c * 16 + i) * TC_BM + row] = row < a.cout ? v[i] : 0.f;   // lanes >= a_rows: garbage
+        for (int i = 0; i < 16; ++i) stage[(c * 16 + i) * TC_BM + row] = v[i];
       }
       if (trace && threadIdx.x == 0) tr[8] = globaltimer();
     } else {
@@ -738,9 +742,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   }
 }
 
-uint32_t tc_smem_bytes() { return 1024 + TC_RING + 256; }   // align pad + stages + barriers
-static_assert(TC_RING == TC_STAGES * (A_BYTES + B_BYTES), "ring");
-static_assert(tc_stages(TC_BM) == TC_STAGES, "full-width layers keep the 4-stage ring");
+uint32_t tc_smem_bytes() { return 1024 + TC_STAGES * (A_BYTES + B_BYTES) + 128; }
 
 void tc_kernel_table(KernelFn* instr, KernelFn* plain) {
   instr[0] = (KernelFn)k_conv_tc<true, false>;

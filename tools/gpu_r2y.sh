@@ -1,0 +1,7 @@
+#!/bin/bash
+# Full GPU suite + smoke + bench line after the split-K change.
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1; echo "build rc=$?"
+timeout 1800 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu_r2y.log 2>&1; echo "pytest rc=$?"; tail -3 gpurun_out/pytest_gpu_r2y.log
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke_r2y.log 2>&1; echo "smoke rc=$?"; tail -1 gpurun_out/smoke_r2y.log
+( time timeout 1500 python bench.py --steps 10 --warmup 3 > gpurun_out/bench_r2y.json 2> gpurun_out/bench_r2y.err ) 2> gpurun_out/bench_r2y.time; echo "bench rc=$?"; head -c 1500 gpurun_out/bench_r2y.json; cat gpurun_out/bench_r2y.time
+cp gpurun_out/bench_detail_c3_dispersion_n1.json gpurun_out/bench_detail_c3_r2y.json

@@ -7,13 +7,13 @@ import sys
 
 err, out = sys.argv[1], sys.argv[2]
 layers = [json.loads(l) for l in open(out) if l.startswith("{")]
-blocks = {}
+seq = []   # traced blocks in file order: 2 runs per layer, layers in stdout order
 cur = None
 for line in open(err):
     m = re.match(r"trace kernel (\d+) grid (\d+)", line)
     if m:
         cur = {}
-        blocks.setdefault(int(m.group(1)), []).append(cur)
+        seq.append((int(m.group(1)), cur))
         continue
     m = re.match(r"\s+(\w+)\s+(-?\d+)\s+(-?\d+)\s+(-?\d+)", line)
     if m and cur is not None:
@@ -21,8 +21,12 @@ for line in open(err):
 print(f"{'model':12s} {'k':>3s} {'grid':>4s} {'MB':>5s} {'GF':>6s} | {'b_iss':>6s} {'full0':>6s} {'mma':>6s} "
       f"{'epi':>6s} {'exit':>6s} | {'data':>5s} {'loop':>5s} {'tail':>5s} {'span':>5s}")
 tot = {}
+pos = 0
 for L in layers:
-    bl = blocks.get(L["k"])
+    bl = []
+    while pos < len(seq) and seq[pos][0] == L["k"]:
+        bl.append(seq[pos][1])
+        pos += 1
     if not bl:
         continue
     b = bl[-1]
