@@ -47,6 +47,12 @@ static bool profiled() {
 }
 static bool no_gate() { return profiled() || std::getenv("PAELLA_NO_GATE") != nullptr; }
 static bool no_proxy_env() { return profiled() || std::getenv("PAELLA_NO_PROXY") != nullptr; }
+// diagnosis: run the counter mirror warp next to the naive baseline (its cost alone)
+static bool naive_mirror_env() { return std::getenv("PAELLA_NAIVE_MIRROR") != nullptr; }
+// diagnosis: the naive baseline launches the INSTRUMENTED kernels, counting into a scratch
+// counter table laid out like counter mode's (nobody reads it): the device-side cost of
+// the instrumentation alone, without the dispatcher
+static bool naive_instr_env() { return std::getenv("PAELLA_NAIVE_INSTR") != nullptr; }
 
 int64_t now_ns() {
   timespec ts;
@@ -327,6 +333,8 @@ struct CudaBackend : Backend {
       proxy_running = false;   // it left after an idle spell
     }
     __atomic_store_n(&proxy_ctl[32], 0u, __ATOMIC_RELEASE);
+    if (const char* pace = std::getenv("PAELLA_MIRROR_PACE_NS"))
+      __atomic_store_n(&proxy_ctl[8], (uint32_t)atoi(pace), __ATOMIC_RELEASE);
     const Rec* src = dev_ring;
     Rec* dst = ring_d;
     uint32_t mask = cap - 1, l2 = 0;
@@ -370,6 +378,8 @@ struct CudaBackend : Backend {
       }
       if (cudaStreamCreateWithPriority(&streams[i], cudaStreamNonBlocking, prio) != cudaSuccess) return -EIO;
     }
+    if (const char* rot = std::getenv("PAELLA_STREAM_ROT"))   // diagnosis: logical -> physical stream
+      if (nstreams) std::rotate(streams.begin(), streams.begin() + (atoi(rot) % nstreams), streams.end());
     cudaMemsetAsync(tail, 0, 256, streams[0]);
     cudaMemsetAsync(ctr, 0, 2 * NCTR * sizeof(uint32_t), streams[0]);
     KernelFn tc_i[2], tc_p[2];
@@ -452,6 +462,12 @@ static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last, bool
   ia.uid = uid;
   ia.group = g->P->cfg.group_size;
   ia.flags = INSTR_ON | (last ? INSTR_LAST : 0);
+  if (g->P->cfg.naive && instr) {   // PAELLA_NAIVE_INSTR (diagnosis)
+    ia.ctr = g->be->ctr_dev() + 2 * (uid % NCTR_M);
+    ia.ctr_stride = 2 * NCTR_M;
+    ia.flags |= INSTR_CTR | (last ? 0u : INSTR_RELAXED);
+    return ia;
+  }
   if (g->ctr_mode && instr) {
     // counter mode: a free slot of the mirrored counter table (> P x (lookahead + 1)
     // slots, so one is always free); the slot returns when its last block has exited
@@ -476,9 +492,34 @@ static InstrArgs make_instr(Gpu* g, uint32_t uid, uint32_t grid, bool last, bool
   return ia;
 }
 
-static void launcher_push(Gpu* g, const LaunchDesc& d) {
-  Launcher* L = g->launchers[d.stream % g->launchers.size()].get();
+static bool launch_stats_env() {
+  static const bool on = std::getenv("PAELLA_LAUNCH_STATS") != nullptr;
+  return on;
+}
+
+static void launcher_push(Gpu* g, const LaunchDesc& d0) {
+  Launcher* L = g->launchers[d0.stream % g->launchers.size()].get();
+  LaunchDesc d = d0;
+  d.t_push = launch_stats_env() ? now_ns() : 0;
   while (!L->q.push(d)) {
+  }
+}
+
+static void launch_stats_print(Gpu* g) {
+  auto pct = [](const std::vector<uint64_t>& h, uint64_t n, double q) {
+    uint64_t c = 0;
+    for (size_t i = 0; i < h.size(); ++i) {
+      c += h[i];
+      if (c >= q * n) return 0.5 * (double)i;
+    }
+    return 100.0;
+  };
+  for (size_t i = 0; i < g->launchers.size(); ++i) {
+    const Launcher* L = g->launchers[i].get();
+    if (!L->n) continue;
+    fprintf(stderr, "[paella] gpu %u launcher %zu: %llu launches, queued p50 %.1f p99 %.1f us, call p50 %.1f p90 %.1f p99 %.1f us\n",
+            g->index, i, (unsigned long long)L->n, pct(L->h_queue, L->n, 0.5), pct(L->h_queue, L->n, 0.99),
+            pct(L->h_call, L->n, 0.5), pct(L->h_call, L->n, 0.9), pct(L->h_call, L->n, 0.99));
   }
 }
 
@@ -494,8 +535,15 @@ static void launcher_main(Gpu* g, Launcher* L) {
     }
     if (d->kind == 0) {
       void* args[3] = {(void*)&d->a, (void*)&d->ia, (void*)d->tmap};
+      const int64_t t0 = d->t_push ? now_ns() : 0;
       cudaError_t e = cuda_launch(cb->fn(d->k->kind, d->dtype, d->instr != 0), *d->k, args, cb->streams[d->stream], cb->pdl);
       if (e != cudaSuccess) g->launch_err.store((int)e);
+      if (d->t_push) {
+        const int64_t t1 = now_ns();
+        L->n++;
+        L->h_queue[std::min<int64_t>(200, (t0 - d->t_push) / 500)]++;
+        L->h_call[std::min<int64_t>(200, (t1 - t0) / 500)]++;
+      }
     } else if (d->kind == 1) {
       cudaEventRecord((cudaEvent_t)d->event, cb->streams[d->stream]);
       __atomic_store_n(d->recorded, (uint8_t)1, __ATOMIC_RELEASE);
@@ -648,8 +696,9 @@ static bool admit(Gpu* g, uint32_t client, const SubmitSlot& s) {
     // CUDA-MS baseline: every kernel of the job enters stream jid % P now
     uint32_t st = jid % P->cfg.stream_pool;
     j.stream = st;
+    const bool ninstr = naive_instr_env();
     for (uint32_t l = 0; l < m->kernels.size(); ++l) {
-      do_launch(g, m, slot, l, 0, st, false);
+      do_launch(g, m, slot, l, ninstr ? g->naive_uid++ : 0, st, ninstr);
       g->stats.launches++;
     }
     if (!g->launchers.empty()) {
@@ -782,6 +831,7 @@ static uint32_t drain_counters(Gpu* g) {
         g->stats.records++;
         observe_before_record(g, type, L.uid, cnt_g);   // OBSERVE precedes its RECORD in the log
         logev(g, EV_RECORD, type, L.uid, cnt_g, ((uint64_t)grp << 40) | (0xFFull << 56));
+        if (g->log_times) logev(g, EV_TIME, 1 + type, L.uid, (uint64_t)now_ns(), end);   // count seen (host)
         int64_t done = -1;
         const bool complete = g->policy->record(type, L.uid, cnt_g, &done);
         if (done >= 0)
@@ -999,6 +1049,8 @@ static void dispatch_loop(Gpu* g) {
       }
       if (progressed || nev) busy_ticks += ticks() - it0;
       if (stopping && g->naive_inflight.empty()) return;
+      if (naive_mirror_env() && (g->stats.loop_iters & 1023) == 0 && !g->naive_inflight.empty())
+        static_cast<CudaBackend*>(g->be.get())->ensure_proxy();
       continue;
     }
     // 2. notification ring (keep the forwarding warp alive while records are due)
@@ -1269,7 +1321,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
       g->be.reset(new CudaBackend(g->device, g->cap, cfg.stream_pool,
                                   cfg.no_proxy == 0 && !no_proxy_env(),
                                   cfg.no_proxy == 0 && cfg.notify_mode == PAELLA_NOTIFY_COUNTERS &&
-                                      !cfg.naive && !no_proxy_env()));
+                                      (!cfg.naive || naive_mirror_env()) && !no_proxy_env()));
     if (cfg.device == PAELLA_DEVICE_CUDA) {
       auto* cb = static_cast<CudaBackend*>(g->be.get());
       cb->pdl = (!cfg.naive || cfg.naive_pdl) && !cfg.no_pdl && !std::getenv("PAELLA_NO_PDL");
@@ -1342,6 +1394,31 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
         g->launchers.push_back(std::move(L));
       }
       for (auto& L : g->launchers) L->th = std::thread(launcher_main, g.get(), L.get());
+    }
+    if (cfg.device == PAELLA_DEVICE_CUDA && std::getenv("PAELLA_LAUNCH_NOISE_US")) {
+      // diagnosis: host launches during kernel execution -- an empty 1-block kernel on its
+      // own stream every N us until shutdown
+      const int64_t period = (int64_t)(atof(std::getenv("PAELLA_LAUNCH_NOISE_US")) * 1000);
+      Gpu* gp = g.get();
+      gp->noise = std::thread([gp, period] {
+        cudaSetDevice(gp->device);
+        cudaStream_t s;
+        cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
+        auto* cb = static_cast<CudaBackend*>(gp->be.get());
+        KernelFn f = cb->fn(KIND_EMPTY, 0, false);
+        LayerArgs la{};
+        InstrArgs ia{};
+        void* args[2] = {(void*)&la, (void*)&ia};
+        int64_t next = now_ns();
+        while (!gp->launchers_stop.load(std::memory_order_acquire) && !gp->stop.load(std::memory_order_acquire)) {
+          cudaLaunchKernel((const void*)f, dim3(1), dim3(32), args, 0, s);
+          next += period;
+          while (now_ns() < next) {
+          }
+        }
+        cudaStreamSynchronize(s);
+        cudaStreamDestroy(s);
+      });
     }
     g->thread = std::thread(dispatcher_main, g.get());
   }
@@ -1491,6 +1568,8 @@ int paella_shutdown(paella_t* p) {
     g->launchers_stop.store(true, std::memory_order_release);
     for (auto& L : g->launchers)
       if (L->th.joinable()) L->th.join();
+    if (g->noise.joinable()) g->noise.join();
+    if (launch_stats_env()) launch_stats_print(g.get());
     if (P->cfg.device == PAELLA_DEVICE_CUDA) {
       cudaSetDevice(g->device);
       static_cast<CudaBackend*>(g->be.get())->stop_proxy();

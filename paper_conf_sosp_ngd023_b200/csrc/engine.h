@@ -118,6 +118,7 @@ struct LaunchDesc {
   uint8_t* recorded;
   uint32_t stream, dtype;
   uint8_t instr, kind;         // kind 0 = kernel, 1 = event record, 2 = wait for a recorded event
+  int64_t t_push;              // PAELLA_LAUNCH_STATS: host time the dispatcher queued it
 };
 
 // plain (in-process) single-producer / single-consumer queue
@@ -149,6 +150,10 @@ struct SpscQ {
 struct Launcher {
   SpscQ<LaunchDesc> q;
   std::thread th;
+  // PAELLA_LAUNCH_STATS (diagnosis): kernel launches, time queued before the call and
+  // time inside cudaLaunchKernelExC, histograms in 0.5 us bins (last bin: >= 100 us)
+  uint64_t n = 0;
+  std::vector<uint64_t> h_queue = std::vector<uint64_t>(201, 0), h_call = std::vector<uint64_t>(201, 0);
 };
 
 // device backend: real CUDA GPU or CPU fake
@@ -218,7 +223,8 @@ struct Gpu {
   int64_t clk_new[4] = {0, 0, 0, 0};
   std::atomic<uint64_t> clk_req{0}, clk_applied{0};
   FILE* log = nullptr;
-  bool log_times = false;   // PAELLA_TRACE_TIMES: host-time events (EV_TIME) for timelines
+  bool log_times = false;
+  uint32_t naive_uid = 0;   // PAELLA_NAIVE_INSTR diagnosis: launch counter of the naive path   // PAELLA_TRACE_TIMES: host-time events (EV_TIME) for timelines
   std::mutex log_mu;
   paella_stats_t stats{};
   std::vector<Issue> issues;
@@ -249,6 +255,7 @@ struct Gpu {
   // launcher threads (cfg.launch_threads)
   std::vector<std::unique_ptr<Launcher>> launchers;
   std::atomic<bool> launchers_stop{false};
+  std::thread noise;   // PAELLA_LAUNCH_NOISE_US (diagnosis): background launches of an empty kernel
   std::atomic<int> launch_err{0};
 };
 

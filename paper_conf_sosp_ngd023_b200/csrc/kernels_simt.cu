@@ -681,6 +681,7 @@ KernelFn proxy_kernel() { return (KernelFn)k_notify_proxy; }
 // flight (the counters are the state, so nothing is lost across a relaunch).
 // ---------------------------------------------------------------------------
 __global__ void __launch_bounds__(32, 1) k_notify_mirror(const uint4* ctrs, uint4* host, volatile uint32_t* state) {
+  const uint32_t pace = state[8];   // diagnosis (PAELLA_MIRROR_PACE_NS): extra pause per scan
   const uint32_t lane = threadIdx.x;
   constexpr uint32_t NQ = NCTR_SUB * NCTR_M * 2 / 4 / 32;   // 16-byte chunks per lane (all tables)
   uint4 prev[NQ];
@@ -722,6 +723,7 @@ __global__ void __launch_bounds__(32, 1) k_notify_mirror(const uint4* ctrs, uint
       }
       __nanosleep(64);
     }
+    if (pace) __nanosleep(pace);
   }
   if (lane == 0) {
     __threadfence_system();

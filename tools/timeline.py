@@ -46,6 +46,13 @@ def parse(path):
             jobs[life]["uids"].append(b)
         elif t == EV_TIME and a == 0:
             launches[b]["t_issue"] = c
+        elif t == EV_TIME and a in (2, 3) and b in launches:   # counter mode: counts seen by the host
+            L = launches[b]
+            key = "seen_place" if a == 2 else "seen_done"
+            if a == 2 and L.get("seen_place") is None:
+                L["seen_place"] = c
+            if a == 3:
+                L["seen_done"] = c      # the last one is the final count
         elif t == EV_RECORD:
             L = launches.get(b)
             if L is None:
@@ -117,6 +124,39 @@ def summarize(jobs, launches, names):
     return out
 
 
+def summarize_seen(jobs, launches, names):
+    """Counter mode (no device timestamps): host-observed times.  Per job: arrival ->
+    first issue, and the completion-to-completion intervals of consecutive kernels as
+    the host saw them (the notification latency cancels out in the differences), plus
+    how far ahead each kernel was decided relative to its predecessor's completion seen."""
+    per_model = {}
+    lead = []
+    for jb in jobs.values():
+        ks = sorted((launches[u] for u in jb["uids"]), key=lambda k: k["layer"])
+        if not ks or any(k.get("seen_done") is None or k.get("t_issue") is None for k in ks):
+            continue
+        pm = per_model.setdefault(names[jb["model"]], dict(n=0, admit=0.0, first_done=0.0, chain=0.0, tail=0.0,
+                                                            late=0))
+        pm["n"] += 1
+        pm["admit"] += ks[0]["t_issue"] - jb["t_sched"]
+        pm["first_done"] += ks[0]["seen_done"] - ks[0]["t_issue"]
+        pm["chain"] += ks[-1]["seen_done"] - ks[0]["seen_done"]
+        if jb["t_complete"] is not None:
+            pm["tail"] += jb["t_complete"] - ks[-1]["seen_done"]
+        for p, q in zip(ks, ks[1:]):
+            lead.append(p["seen_done"] - q["t_issue"])
+            if q["t_issue"] > p["seen_done"]:
+                pm["late"] += 1
+    pct = lambda v, p: round(float(np.percentile(v, p)) / 1e3, 2) if len(v) else None   # noqa: E731
+    return dict(issue_lead_vs_pred_done_seen_us=dict(p10=pct(lead, 10), p50=pct(lead, 50)),
+                per_model={m: dict(jobs=v["n"], admit_to_first_issue_us=round(v["admit"] / v["n"] / 1e3, 1),
+                                   first_issue_to_first_done_seen_us=round(v["first_done"] / v["n"] / 1e3, 1),
+                                   chain_done_seen_us=round(v["chain"] / v["n"] / 1e3, 1),
+                                   last_done_seen_to_complete_us=round(v["tail"] / v["n"] / 1e3, 1),
+                                   late_issues_per_job=round(v["late"] / v["n"], 2))
+                           for m, v in per_model.items()})
+
+
 def chrome(jobs, launches, names, path):
     ev = []
     t0 = min(L["start"] for L in launches.values() if L["start"] is not None)
@@ -152,7 +192,7 @@ def main():
     specs = [(g, rng.model_params(g)) for g in (archs.build(n) for n in names)]
     slots, stride = 64, 1 << 21
     log = out + ".evlog"
-    kw = dict(launch_threads=4, dispatcher_cpus=[2], notify="ring", group=1, slack=2368, lookahead=6,
+    kw = dict(launch_threads=8, dispatcher_cpus=[2], notify="counters", group=16, slack=3552, lookahead=6,
               max_active=8)
     kw.update(variant)
     e = L.Engine(num_clients=len(specs), region_bytes=slots * stride + (1 << 20), max_jobs_per_model=64,
@@ -168,12 +208,16 @@ def main():
     jct, _ = e.loadgen(t, mm, mm, ii, stride, slots)
     e.shutdown()
     jobs, launches, _ = parse(log)
-    s = summarize(jobs, launches, names)
+    if kw.get("notify", "counters") == "counters":
+        s = summarize_seen(jobs, launches, names)
+    else:
+        s = summarize(jobs, launches, names)
     s["variant"] = kw
     s["jct_mean_us"] = round(float(jct.mean()) / 1e3, 1)
     s["jct_per_model_us"] = {n: round(float(jct[mm == i].mean()) / 1e3, 1) for i, n in enumerate(names)
                              if (mm == i).any()}
-    chrome(jobs, launches, names, out + ".trace.json")
+    if kw.get("notify", "counters") != "counters":
+        chrome(jobs, launches, names, out + ".trace.json")
     print(json.dumps(s))
 
 
