@@ -79,6 +79,9 @@ def parse():
     ap.add_argument("--no-baselines", action="store_true", help="only the paella arm")
     ap.add_argument("--max-active", type=int, default=8, help="job cap K of the paella arms (B200-Q6); 0 = none")
     ap.add_argument("--lookahead", type=int, default=6, help="NEXT-1 launch-ahead depth of the paella arms")
+    ap.add_argument("--lookahead-placed", action="store_true",
+                    help="launch-ahead waits for the oldest in-flight kernel's placement (the round-2 rule); "
+                         "default: lookahead_unplaced (profiles/r2/diag/un_*)")
     ap.add_argument("--slack", type=int, default=3552,
                     help="B, blocks issued beyond full utilisation (P1300-1304); 24 x 148 SMs covers the "
                          "measured dispatch loop delay with launch-ahead 6 (DESIGN.md B200-Q1)")
@@ -418,7 +421,8 @@ def run_gpu(args, ngpus, cores, fake):
         common["dispatcher_cpus"] = cores
     paella_kw = dict(policy=pol[args.policy], theta=args.theta, decide_delay_ns=args.decide_delay_ns,
                      online_tbar=args.online_tbar, slack=args.slack, prio_classes=args.prio_classes,
-                     lookahead=args.lookahead, max_active=args.max_active, instrument=True,
+                     lookahead=args.lookahead, lookahead_unplaced=not args.lookahead_placed,
+                     max_active=args.max_active, instrument=True,
                      route=L.ROUTE_LEAST_WORK, branches=bool(args.branches))
     arms_kw = {
         "paella": paella_kw,
@@ -651,7 +655,7 @@ def cpu_baseline(cfg, seconds=20.0, reserve=0):
             "host": hi}
 
 
-def simulator_timing(kinfo, cfg, names, lam, args_slack, args_lookahead, n=20):
+def simulator_timing(kinfo, cfg, names, lam, args_slack, args_lookahead, n=20, unplaced=1):
     """The oracle's discrete-event simulator (synthetic mode) on a trace of the config:
     wall time and simulated events per second on one core."""
     from oracle import sim
@@ -668,7 +672,8 @@ def simulator_timing(kinfo, cfg, names, lam, args_slack, args_lookahead, n=20):
         models.append(ls)
     t, mm, _ = make_trace(n, lam, cfg, len(names), seed=31)
     trace = [(int(t[i]), int(mm[i]), int(mm[i])) for i in range(n)]
-    c = sim.Config(num_clients=len(names), slack=args_slack, lookahead=args_lookahead, max_active=8)
+    c = sim.Config(num_clients=len(names), slack=args_slack, lookahead=args_lookahead, max_active=8,
+                   lookahead_unplaced=unplaced)
     t0 = time.perf_counter()
     r = sim.simulate(c, models, trace, sim.GPUModel(), check=False)
     el = time.perf_counter() - t0
@@ -789,7 +794,8 @@ def main():
                    "requests_per_step": args.reqs * ngpus,
                    "parallelism": f"{ngpus} GPU dispatchers, least-work router" if ngpus > 1 else "1 GPU dispatcher",
                    "paella": (f"srpt+deficit th{args.theta}" if args.policy == "srpt" else args.policy)
-                   + f" K{args.max_active} la{args.lookahead} B{args.slack} pdl" + (" branches" if args.branches else ""),
+                   + f" K{args.max_active} la{args.lookahead}{'' if args.lookahead_placed else 'u'} B{args.slack} pdl"
+                   + (" branches" if args.branches else ""),
                    "l2": "not flushed: weights (~120 MB bf16) largely L2-resident as in serving; inputs stream "
                          "from pinned host memory every request"},
         "roofline": roofline_entry(dict(P, config=args.config), peaks) if "kinfo" in P else None,
@@ -817,7 +823,7 @@ def main():
         detail["cpu_baseline"] = cb
         try:
             detail["simulator"] = simulator_timing(P["kinfo"], dict(cfg, weights=detail["mix_weights"]), names, lam,
-                                                  args.slack, args.lookahead)
+                                                  args.slack, args.lookahead, unplaced=int(not args.lookahead_placed))
         except Exception as ex:
             detail["simulator"] = {"error": str(ex)[:200]}
     if args.fake:

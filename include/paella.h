@@ -185,6 +185,13 @@ typedef struct {
                                     override is exempt).  Preemption stays kernel-granular: a
                                     job pushed out of the K first stops issuing, its in-flight
                                     kernels drain */
+  uint32_t lookahead_unplaced;    /* NEXT-1 variant: 1 = launch-ahead queues the next kernel of a
+                                    (virtual) stream as soon as <= D are in flight, without
+                                    waiting for the oldest in-flight kernel's placement to be
+                                    seen (the occupancy predicate's slack B still bounds the
+                                    queued blocks).  Kernels shorter than the notification
+                                    round trip otherwise complete before their placement is
+                                    seen and launch-ahead degenerates to one kernel at a time */
 } paella_config_t;
 
 /* One routing decision.  W_g = work[g] + pending[g] * tbar_model:

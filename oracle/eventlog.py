@@ -6,7 +6,8 @@ Format (DESIGN.md §"Event log"): a sequence of 32-byte little-endian records
 
   100 CONFIG    a=N clients, b=policy, c=theta, d=(B << 32) | G
   100 CONFIG    a=0xFFFFFFFF, b=ring capacity, c=stream pool P, d=(priority classes << 32) | launch-ahead depth
-  100 CONFIG    a=0xFFFFFFFE, b=online T-bar refinement (NEXT-4), c=max_active K (B200-Q6)
+  100 CONFIG    a=0xFFFFFFFE, b=online T-bar refinement (NEXT-4), c=max_active K (B200-Q6),
+                d=branches | lookahead_unplaced << 8 (NEXT-1 variant)
   101 CAPACITY  a=resource r, b=C_r
   110 MODEL     a=model, b=#kernels
   111 LAYER     a=model, b=layer, c=grid, d=T-bar ns
@@ -19,6 +20,8 @@ Format (DESIGN.md §"Event log"): a sequence of 32-byte little-endian records
     4 ISSUE     a=stream, b=uid, c=job, d=layer
     5 COMPLETE  b=job, c=t ns
     6 OBSERVE   b=uid, c=observed duration ns (NEXT-4; precedes the final COMPLETION)
+    9 TIME      (PAELLA_TRACE_TIMES only; ignored here) a=0 decision of launch b, 1 batch end,
+                2/3 placement/completion count of launch b seen; c = host ns (tools/timeline.py)
     8 CLOCK     a=gpu | resolution ns << 8, b=offset (globaltimer - host CLOCK_MONOTONIC, ns),
                 c=round trip ns, d=host time of the calibration sample (at init and at every
                 paella_clock_sync)
@@ -58,6 +61,7 @@ def read(path):
             if a == 0xFFFFFFFE:
                 cfg_kw["online_tbar"] = b
                 cfg_kw["max_active"] = c
+                cfg_kw["lookahead_unplaced"] = (d >> 8) & 1
             elif a == 0xFFFFFFFF:
                 cfg_kw["ring_capacity"] = b
                 cfg_kw["streams"] = c

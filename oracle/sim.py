@@ -79,6 +79,7 @@ class Config:
     online_tbar: int = 0              # NEXT-4: refine T-bar online (running average, P1252-1254)
     max_active: int = 0               # K: only the K first jobs in the policy's order that still
                                       # have kernels to issue may issue (0 = no cap); B200-Q6
+    lookahead_unplaced: int = 0       # NEXT-1 variant: launch-ahead without the oldest-placed test
 
 
 # NEXT-4 (P1249-1266: "x-bar is the average of all previous observations of x"; "these
@@ -260,7 +261,8 @@ class Policy:
         """The job's lowest-index active kernel that may be dispatched now, or None:
         the next kernel of a virtual stream whose cross-stream dependencies have all
         completed, and whose stream is idle -- or, with launch-ahead D > 0, whose oldest
-        in-flight kernel is fully placed (running) with at most D in flight."""
+        in-flight kernel is fully placed (running) with at most D in flight (with
+        lookahead_unplaced: at most D in flight, whether or not the oldest is placed)."""
         T = self.topo[j.model]
         best = None
         for v, ks in enumerate(T.vs_kernels):
@@ -274,7 +276,7 @@ class Policy:
                 if self.cfg.lookahead <= 0 or infl > self.cfg.lookahead:
                     continue
                 L = self.launches[j.vs_uids[v][0]]          # the oldest kernel in flight
-                if max(L.p, L.f) < L.grid:
+                if not self.cfg.lookahead_unplaced and max(L.p, L.f) < L.grid:
                     continue
             if best is None or k < best:
                 best = k

@@ -64,7 +64,8 @@ int Policy::lowest_free_in_class(uint32_t c) const {
 // The job's lowest-index active kernel that may be dispatched now, or -1 (identical to
 // oracle Policy.head): the next kernel of a virtual stream whose cross-stream
 // dependencies have completed and whose stream is idle -- or, with launch-ahead D > 0,
-// whose oldest in-flight kernel is fully placed (running) with at most D in flight.
+// whose oldest in-flight kernel is fully placed (running) with at most D in flight
+// (la_unplaced: at most D in flight, placement not required).
 int64_t Policy::head(const PolicyJob& j) const {
   if (!j.live || j.cursor >= models_[j.model].size()) return -1;
   const auto& ml = models_[j.model];
@@ -79,6 +80,10 @@ int64_t Policy::head(const PolicyJob& j) const {
     const uint32_t infl = j.vs_infl[v];
     if (infl > 0) {
       if (cfg_.lookahead == 0 || infl > cfg_.lookahead) continue;
+      if (cfg_.la_unplaced) {
+        if (best < 0 || (int64_t)k < best) best = k;
+        continue;
+      }
       const uint32_t oldest = j.vs_uid[v][0];
       const PolicyLaunch& L = launches_[oldest % kLaunchSlots];
       if (!L.live || L.uid != oldest || (L.p > L.f ? L.p : L.f) < L.grid) continue;

@@ -156,7 +156,8 @@ def _serve_and_check(e, specs, n, n_clients, seed, rate_us=30.0):
     (L.POLICY_SRPT_DEFICIT, 16, 32, 2048, 1, 2, "direct", 1),  # direct record writes (the paper's path)
     (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 3, 4, "counters", -4),  # bench arm + online T-bar (NEXT-4)
     (L.POLICY_SJF, 16, 32, 65536, 3, 4, "counters", 1),
-    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 6, 4, "counters", 108),   # the bench arm: job cap K = 8, launch-ahead 6
+    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, -6, 8, "counters", 108),  # the bench arm: K = 8, launch-ahead 6 unplaced
+    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 6, 4, "counters", 108),
     (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 3, 4, "counters", 108),
     (L.POLICY_FIFO, 16, 32, 65536, 3, 4, "counters", 104),           # FIFO arm, K = 4
     (L.POLICY_RR, 16, 8, 4096, 0, 0, "counters", 1),
@@ -165,12 +166,13 @@ def test_serving_parity_and_replay(tmp_path, policy, group, streams, ring, look,
     log = str(tmp_path / "gpu_%u.log")
     names = ["toy", "resnet18", "mobilenet_v2", "squeezenet1_1"]
     online, prio = prio < 0, abs(prio)
+    unpl, look = look < 0, abs(look)          # look < 0: launch-ahead without the placement test
     K = prio - 100 if prio > 100 else 0       # 1xx: job cap K = xx (B200-Q6), one priority class
     prio = 1 if K else prio
     with L.Engine(num_clients=3, policy=policy, group=group, streams=streams, ring_capacity=ring,
                   event_log=log, max_jobs_per_model=32, lookahead=look, launch_threads=lt, notify=notify,
                   prio_classes=prio, slack=(3552 if K else 1184) if (prio > 1 or K) else 0, online_tbar=online,
-                  max_active=K) as e:
+                  max_active=K, lookahead_unplaced=unpl) as e:
         specs = []
         for nm in names:
             g = archs.build(nm)
@@ -273,8 +275,9 @@ def test_per_sm_capacity_from_g1_records(tmp_path):
 @pytest.mark.gpu
 def test_serving_parity_c3_models_bench_arm(tmp_path):
     """C-3's models (ResNet-50, DenseNet-121, Inception-v3, MobileNetV2) served
-    concurrently in the launch configuration bench.py times (launch-ahead 6, job cap 8, 4
-    launcher threads, counter notification, B = 24x148, dispatcher on its own core): every output
+    concurrently in the launch configuration bench.py times (launch-ahead 6 without the
+    placement test, job cap 8, 8 launcher threads, counter notification, B = 24x148,
+    dispatcher on its own core): every output
     within the bf16 tolerance of the float64 oracle and the issue order replayed."""
     log = str(tmp_path / "gpu_%u.log")
     names = ["resnet50", "densenet121", "inception_v3", "mobilenet_v2"]
@@ -282,8 +285,9 @@ def test_serving_parity_c3_models_bench_arm(tmp_path):
         for i in range(4):
             oracle_out(nm, i, "bf16")
     cpus = sorted(os.sched_getaffinity(0))
-    with L.Engine(num_clients=4, event_log=log, max_jobs_per_model=32, lookahead=6, launch_threads=4,
-                  slack=3552, max_active=8, region_bytes=96 << 20,   # 64 slots of Inception-v3's 1.08 MB io buffer
+    with L.Engine(num_clients=4, event_log=log, max_jobs_per_model=32, lookahead=6, launch_threads=8,
+                  slack=3552, max_active=8, lookahead_unplaced=True,
+                  region_bytes=96 << 20,   # 64 slots of Inception-v3's 1.08 MB io buffer
                   dispatcher_cpus=[cpus[min(2, len(cpus) - 1)]]) as e:
         specs = []
         for nm in names:

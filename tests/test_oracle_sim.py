@@ -214,15 +214,17 @@ def _run_policy_with_log(cfg, models, trace, gpu):
         sim.Policy.__init__ = orig
 
 
-@pytest.mark.parametrize("lookahead", [0, 1, 2])
+@pytest.mark.parametrize("lookahead", [0, 1, 2, -2])
 @pytest.mark.parametrize("seed", range(8))
 def test_S6_replay_reproduces_issue_order(seed, lookahead):
+    """lookahead < 0: depth |lookahead| with lookahead_unplaced (NEXT-1 variant)."""
+    unplaced, lookahead = lookahead < 0, abs(lookahead)
     r = random.Random(50 + seed)
     models = random_models(r)
     gpu = GPUModel(sms=4, per_sm=(32, 64, 65536, 233472, 512), launch_delay=300, notif_delay=1100)
     cfg = Config(num_clients=4, theta=r.choice([0, 3, 100]), slack=4, group=r.choice([1, 16]),
                  ring_capacity=128, streams=8, capacity=tuple(4 * x for x in (32, 64, 65536, 233472, 512)),
-                 lookahead=lookahead)
+                 lookahead=lookahead, lookahead_unplaced=int(unplaced))
     trace = random_trace(r, 120, 4, len(models), rate_ns=2000)
     res = _run_policy_with_log(cfg, models, trace, gpu)
     log = res.policy.log
@@ -510,6 +512,46 @@ def test_launch_ahead_closed_form_zero_delay(D):
     assert len({s for (_, _, _, _, s) in res.issues}) == (1 if D > 0 else 1)
 
 
+@pytest.mark.parametrize("D", [1, 2, 3, 6])
+def test_launch_ahead_unplaced_closed_form_zero_delay(D):
+    """The NEXT-1 variant without the placement test gives the same schedule as the
+    original rule when placement is seen instantly: kernel k issued at max(0, (k - D) d),
+    JCT = L d."""
+    Lk, d = 10, 1000
+    cfg = Config(num_clients=1, theta=sim.INF_THETA, slack=10**6, lookahead=D, lookahead_unplaced=1,
+                 capacity=(10**6, 10**9, 10**12, 10**12, 10**9))
+    res = sim.simulate(cfg, _chain(Lk, d), [(0, 0, 0)], GPUModel(sms=1, per_sm=(1, 64, 65536, 233472, 512)))
+    issue_t = [t for (t, uid, jid, layer, stream) in sorted(res.issues, key=lambda x: x[3])]
+    assert issue_t == [max(0, (k - D) * d) for k in range(Lk)]
+    assert res.jct()[0] == Lk * d
+
+
+def test_launch_ahead_unplaced_closed_form_with_delays():
+    """Launch delay 2, notification delay 3 (units of 1 us), derived by hand.
+    (a) d = 10, L = 4.  Original rule D = 1: issues 0, 5, 15, 25 (test below).  Without
+        the placement test, D = 1: k0 and k1 are both issued at 0 (k1 queued behind k0);
+        k0 ends 12, its completion is seen 15 -> k2 issued 15; k1 ends 22, seen 25 -> k3
+        issued 25, runs 32..42, seen 45: issues 0, 0, 15, 25, JCT 45.  D = 2: k0..k2 at
+        0, k3 when k0's completion is seen (15): issues 0, 0, 0, 15, JCT 45.
+    (b) d = 2 (shorter than the notification round trip), L = 4, D = 3.  Original rule:
+        k0 issued 0, launched 2, runs 2..4; its placement is seen 5 -> k1, k2, k3 issued
+        5, launched 7, run 7..9, 9..11, 11..13; seen 16: JCT 16.  Without the placement
+        test all four are issued at 0, launched 2, run 2..4, 4..6, 6..8, 8..10, the last
+        completion is seen 13: JCT 13."""
+    u = 1000
+    gpu = GPUModel(sms=1, per_sm=(1, 64, 65536, 233472, 512), launch_delay=2 * u, notif_delay=3 * u)
+    for d, L, D, unpl, want_issue, want_jct in ((10, 4, 1, 1, [0, 0, 15, 25], 45),
+                                                (10, 4, 2, 1, [0, 0, 0, 15], 45),
+                                                (2, 4, 3, 0, [0, 5, 5, 5], 16),
+                                                (2, 4, 3, 1, [0, 0, 0, 0], 13)):
+        cfg = Config(num_clients=1, theta=sim.INF_THETA, slack=10**6, lookahead=D, lookahead_unplaced=unpl,
+                     capacity=(10**6, 10**9, 10**12, 10**12, 10**9))
+        res = sim.simulate(cfg, _chain(L, d * u), [(0, 0, 0)], gpu)
+        got = [t for (t, *_r) in sorted(res.issues, key=lambda x: x[3])]
+        assert got == [x * u for x in want_issue], (d, D, unpl, got)
+        assert res.jct()[0] == want_jct * u, (d, D, unpl, res.jct()[0])
+
+
 def test_launch_ahead_closed_form_with_delays():
     """d = 10, launch delay 2, notification delay 3, L = 4 (times in units of 1 us),
     derived step by step in the test docstring's notation:
@@ -528,21 +570,22 @@ def test_launch_ahead_closed_form_with_delays():
         assert res.jct()[0] == want_jct * u
 
 
-@pytest.mark.parametrize("D", [0, 1, 3, 6])
+@pytest.mark.parametrize("D", [0, 1, 3, 6, -3])
 def test_inflight_bound_checker(D):
     """check_inflight_bound accepts every simulator log at its own depth; on the chain of
     test_launch_ahead_closed_form_zero_delay (depth D + 1 reached at t = 0) it rejects
-    the log when checked against depth D - 1."""
+    the log when checked against depth D - 1.  D < 0: depth |D| with lookahead_unplaced."""
+    unpl, D = int(D < 0), abs(D)
     r = random.Random(900 + D)
     models = random_models(r)
     gpu = GPUModel(sms=4, per_sm=(32, 64, 65536, 233472, 512), launch_delay=300, notif_delay=400)
-    cfg = Config(num_clients=2, slack=64, group=4, streams=8, lookahead=D,
+    cfg = Config(num_clients=2, slack=64, group=4, streams=8, lookahead=D, lookahead_unplaced=unpl,
                  capacity=tuple(4 * x for x in (32, 64, 65536, 233472, 512)))
     trace = random_trace(r, 30, 2, len(models), rate_ns=3000)
     res = _run_policy_with_log(cfg, models, trace, gpu)
     assert sim.check_inflight_bound(res.policy.log, models, D) == []
     chain = _chain(10, 1000)
-    cfg1 = Config(num_clients=1, theta=sim.INF_THETA, slack=10**6, lookahead=D,
+    cfg1 = Config(num_clients=1, theta=sim.INF_THETA, slack=10**6, lookahead=D, lookahead_unplaced=unpl,
                   capacity=(10**6, 10**9, 10**12, 10**12, 10**9))
     res1 = _run_policy_with_log(cfg1, chain, [(0, 0, 0)], GPUModel(sms=1, per_sm=(1, 64, 65536, 233472, 512)))
     assert sim.check_inflight_bound(res1.policy.log, chain, D) == []

@@ -30,7 +30,8 @@ slots = 64
 region = slots * stride + (1 << 20)
 cuda = ctypes.CDLL("libcuda.so.1")
 t, mm, ii = bench.make_trace(n, rate, cfg, len(names), seed=77)
-for label, kw in (("paella", dict(policy=L.POLICY_SRPT_DEFICIT, slack=3552, lookahead=6, max_active=8, launch_threads=8)),
+for label, kw in (("paella", dict(policy=L.POLICY_SRPT_DEFICIT, slack=3552, lookahead=6, max_active=8, launch_threads=8,
+                                lookahead_unplaced=True)),
                   ("naive", dict(naive=True, instrument=False))):
     a = bench.Arm(L, label, specs, pool, 1, region, stride, slots, False,
                   **dict(dict(launch_threads=4, max_jobs_per_model=64), **kw))

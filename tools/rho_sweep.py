@@ -36,8 +36,10 @@ common = dict(max_jobs_per_model=128, dispatcher_cpus=[2])
 arms = {
     "naive": dict(naive=True, instrument=False, launch_threads=4),
     "naive_pdl": dict(naive=True, instrument=False, naive_pdl=True, launch_threads=4),
-    "paella": dict(policy=L.POLICY_SRPT_DEFICIT, theta=100, slack=3552, lookahead=6, max_active=8, launch_threads=8),
-    "paella_fifo": dict(policy=L.POLICY_FIFO, slack=3552, lookahead=6, max_active=8, launch_threads=8),
+    "paella": dict(policy=L.POLICY_SRPT_DEFICIT, theta=100, slack=3552, lookahead=6, max_active=8, launch_threads=8,
+                   lookahead_unplaced=True),
+    "paella_fifo": dict(policy=L.POLICY_FIFO, slack=3552, lookahead=6, max_active=8, launch_threads=8,
+                        lookahead_unplaced=True),
 }
 out = open(f"gpurun_out/rho_sweep_{tag}.jsonl", "w")
 # calibration per config on the naive arm: unloaded medians (mix weights), X_sat bisection

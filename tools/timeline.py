@@ -193,7 +193,7 @@ def main():
     slots, stride = 64, 1 << 21
     log = out + ".evlog"
     kw = dict(launch_threads=8, dispatcher_cpus=[2], notify="counters", group=16, slack=3552, lookahead=6,
-              max_active=8)
+              max_active=8, lookahead_unplaced=True)
     kw.update(variant)
     e = L.Engine(num_clients=len(specs), region_bytes=slots * stride + (1 << 20), max_jobs_per_model=64,
                  event_log=log, **kw)
@@ -223,3 +223,17 @@ def main():
 
 if __name__ == "__main__":
     main()
+
+
+def dump_jobs(path, names, n=5):
+    """Print the first n jobs' launches: layer, issue / placement seen / completion seen
+    (us after the job's scheduled arrival)."""
+    jobs, launches, _ = parse(path)
+    for li in list(jobs)[:n]:
+        jb = jobs[li]
+        t0 = jb["t_sched"]
+        print(f"job {li} {names[jb['model']]}: complete {((jb['t_complete'] or t0) - t0) / 1e3:.1f}")
+        for u in jb["uids"]:
+            L = launches[u]
+            f = lambda x: f"{(x - t0) / 1e3:7.1f}" if x is not None else "      -"   # noqa: E731
+            print(f"   L{L['layer']:3d} issue {f(L['t_issue'])} placed {f(L.get('seen_place'))} done {f(L.get('seen_done'))}")
