@@ -1401,8 +1401,9 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
       // diagnosis: host launches during kernel execution -- an empty 1-block kernel on its
       // own stream every N us until shutdown
       const int64_t period = (int64_t)(atof(std::getenv("PAELLA_LAUNCH_NOISE_US")) * 1000);
+      const int burst = std::getenv("PAELLA_LAUNCH_NOISE_BURST") ? atoi(std::getenv("PAELLA_LAUNCH_NOISE_BURST")) : 1;
       Gpu* gp = g.get();
-      gp->noise = std::thread([gp, period] {
+      gp->noise = std::thread([gp, period, burst] {
         cudaSetDevice(gp->device);
         cudaStream_t s;
         cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
@@ -1413,7 +1414,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
         void* args[2] = {(void*)&la, (void*)&ia};
         int64_t next = now_ns();
         while (!gp->launchers_stop.load(std::memory_order_acquire) && !gp->stop.load(std::memory_order_acquire)) {
-          cudaLaunchKernel((const void*)f, dim3(1), dim3(32), args, 0, s);
+          for (int b = 0; b < burst; ++b) cudaLaunchKernel((const void*)f, dim3(1), dim3(32), args, 0, s);
           next += period;
           while (now_ns() < next) {
           }
