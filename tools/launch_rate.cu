@@ -8,6 +8,7 @@
 //   2 cuLaunchKernelEx (driver API) + PDL
 //   3 cudaLaunchKernelExC + PDL + cluster (1,1,16), grid 64
 //   4 cuLaunchKernelEx + PDL + cluster (1,1,16), grid 64
+//   5 cudaLaunchKernelExC + PDL, 64 B parameter block
 //   nvcc -gencode arch=compute_100a,code=sm_100a -O2 -o /tmp/lr tools/launch_rate.cu -lcuda -lpthread
 #include <cuda.h>
 #include <cuda_runtime.h>
@@ -22,8 +23,15 @@
 struct Params {
   unsigned char b[352];
 };
+struct Small {
+  unsigned char b[64];
+};
 
 __global__ void empty_k(const __grid_constant__ Params p) {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  if (p.b[0] == 255 && threadIdx.x == 9999) printf("x");
+}
+__global__ void empty_small(const __grid_constant__ Small p) {
   asm volatile("griddepcontrol.wait;" ::: "memory");
   if (p.b[0] == 255 && threadIdx.x == 9999) printf("x");
 }
@@ -44,7 +52,9 @@ static double run(int mode, int T, int S, int per_thread) {
   auto body = [&](int t) {
     cudaSetDevice(0);
     Params p{};
+    Small ps{};
     void* args[1] = {&p};
+    void* args_s[1] = {&ps};
     while (!go.load()) {
     }
     for (int i = 0; i < per_thread; ++i) {
@@ -53,6 +63,17 @@ static double run(int mode, int T, int S, int per_thread) {
       const unsigned gz = cl ? 64 : 1;
       if (mode == 0) {
         cudaLaunchKernel((const void*)empty_k, dim3(1, 1, gz), dim3(128), args, 0, s);
+      } else if (mode == 5) {   // PDL, 64 B parameter block
+        cudaLaunchConfig_t cfg{};
+        cfg.gridDim = dim3(1, 1, 1);
+        cfg.blockDim = dim3(128);
+        cfg.stream = s;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        at[0].val.programmaticStreamSerializationAllowed = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        cudaLaunchKernelExC(&cfg, (const void*)empty_small, args_s);
       } else if (mode == 1 || mode == 3) {
         cudaLaunchConfig_t cfg{};
         cfg.gridDim = dim3(1, 1, gz);
@@ -121,7 +142,7 @@ int main(int argc, char** argv) {
   cudaFree(0);
   run(1, 1, 8, 2000);   // warm-up
   printf("mode threads streams_per_thread launches_per_s us_per_launch_per_thread\n");
-  for (int mode = 0; mode < 5; ++mode)
+  for (int mode : {1, 5, 0, 2})
     for (int T : {1, 2, 4, 8}) {
       const double r = run(mode, T, 8, per);
       printf("%d %d %d %.0f %.3f\n", mode, T, 8, r, 1e6 * T / r);
