@@ -1841,7 +1841,8 @@ static int iso_run(Gpu* g, Model* m, const void* input, void* output, int64_t* k
   int trace_k = std::getenv("PAELLA_TRACE_KERNEL") ? atoi(std::getenv("PAELLA_TRACE_KERNEL")) : -1;
   uint64_t* trbuf = nullptr;
   LayerArgs saved{};
-  if (trace_k >= 0 && trace_k < (int)m->kernels.size() && is_tc(m->kernels[trace_k].kind)) {
+  if (trace_k >= 0 && trace_k < (int)m->kernels.size() &&
+      (is_tc(m->kernels[trace_k].kind) || m->kernels[trace_k].kind == KIND_GAPFC)) {
     trbuf = (uint64_t*)g->trace_buf;
     cudaMemsetAsync(trbuf, 0, 16 * 8 * m->kernels[trace_k].grid_total(), s);
     saved = args[trace_k];
@@ -1872,10 +1873,16 @@ static int iso_run(Gpu* g, Model* m, const void* input, void* output, int64_t* k
     args[trace_k] = saved;
     uint64_t t0 = UINT64_MAX;
     for (uint32_t b = 0; b < nb; ++b) t0 = std::min(t0, h[16 * b]);
-    const char* names[16] = {"entry", "setup", "full0", "mma_done", "accb", "epi_done", "pre_exit", "exit",
-                             "tmem2smem", "pre_bar", "post_bar", "inited", "tma_issued", "b_issued", "reduced", "peers01"};
+    const bool head = m->kernels[trace_k].kind == KIND_GAPFC;
+    const char* names_tc[16] = {"entry", "setup", "full0", "mma_done", "accb", "epi_done", "pre_exit", "exit",
+                                "tmem2smem", "pre_bar", "post_bar", "inited", "tma_issued", "b_issued", "reduced", "peers01"};
+    const char* names_head[16] = {"entry", "pdl_done", "pooled", "bar1", "gathered", "fc_done", "stored", "exit",
+                                  "-", "-", "-", "-", "-", "-", "-", "-"};
+    const char* const* names = head ? names_head : names_tc;
     fprintf(stderr, "trace kernel %d grid %u (ns from first CTA entry): phase min/med/max\n", trace_k, nb);
-    const int order[16] = {0, 11, 12, 13, 1, 2, 3, 4, 8, 9, 10, 15, 14, 5, 6, 7};
+    const int order_tc[16] = {0, 11, 12, 13, 1, 2, 3, 4, 8, 9, 10, 15, 14, 5, 6, 7};
+    const int order_head[16] = {0, 1, 2, 3, 4, 5, 6, 7, 8, 8, 8, 8, 8, 8, 8, 8};
+    const int* order = head ? order_head : order_tc;
     for (int oi = 0; oi < 16; ++oi) {
       int ph = order[oi];
       std::vector<int64_t> v;

@@ -460,7 +460,14 @@ __global__ void __launch_bounds__(256) k_gapfc(const __grid_constant__ LayerArgs
   // pool 1/GAPFC_CLUSTER of the channels each, exchange the pooled slices over DSMEM,
   // then every warp computes one FC row (8 rows per CTA, ~128 CTAs for 1000 classes:
   // the weight stream is spread over many SMs).
+  const bool trace = (a.flags & LF_TRACE) != 0;   // debug: per-CTA phase timestamps (thread 0)
+  uint64_t* tr = trace ? a.trace + 16 * blockIdx.x : nullptr;
+  auto mark = [&](int k) {
+    if (trace && threadIdx.x == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tr[k]));
+  };
+  mark(0);
   kernel_begin<INSTR>(ia);
+  mark(1);
   extern __shared__ float pooled[];   // [C], every CTA ends up with all of it
   const T* X = static_cast<const T*>(a.in);
   const T* W = static_cast<const T*>(a.w);
@@ -507,11 +514,13 @@ __global__ void __launch_bounds__(256) k_gapfc(const __grid_constant__ LayerArgs
       for (int i = 0; i < 8; ++i) pooled[g * 8 + i] = acc[i] * inv;
     }
   }
+  mark(2);
   // publish the slice to the cluster (restricted release: MEMBAR.CTA), then gather the
   // peers' slices (16-byte DSMEM loads) into the local copy
   asm volatile(
       "fence.release.sync_restrict::shared::cta.cluster;\n\t"
       "barrier.cluster.arrive.relaxed.aligned;\n\tbarrier.cluster.wait.aligned;" ::: "memory");
+  mark(3);
   const uint32_t base = (uint32_t)__cvta_generic_to_shared(pooled);
   for (uint32_t q = threadIdx.x; q < C / 4; q += blockDim.x) {
     const uint32_t owner = (q * 4 / 8) / per;
@@ -527,6 +536,7 @@ __global__ void __launch_bounds__(256) k_gapfc(const __grid_constant__ LayerArgs
   // done reading the peers; the matching wait (peers stay resident) is at the end
   asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
   __syncthreads();
+  mark(4);
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const int row = blockIdx.x * (blockDim.x / 32) + warp;
   if (row < (int)a.cout) {
@@ -549,8 +559,11 @@ __global__ void __launch_bounds__(256) k_gapfc(const __grid_constant__ LayerArgs
         static_cast<T*>(a.out)[a.out_co + row] = (T)v;
     }
   }
+  mark(5);
   asm volatile("barrier.cluster.wait.aligned;" ::: "memory");
+  mark(6);
   instr_exit<INSTR>(ia);
+  mark(7);
 }
 
 // ---------------------------------------------------------------------------
