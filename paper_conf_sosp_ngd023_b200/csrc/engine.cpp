@@ -808,12 +808,9 @@ static uint32_t drain_counters(Gpu* g) {
   uint32_t n = 0;
   for (size_t i = 0; i < g->ctr_live.size();) {
     Gpu::CtrLive& L = g->ctr_live[i];
-    uint32_t st = 0, en = 0;   // the launch's counts, summed over the NCTR_SUB tables
-    for (uint32_t t = 0; t < NCTR_SUB; ++t) {
-      const uint64_t v = *reinterpret_cast<volatile uint64_t*>(cb->mirror_h + t * 2 * NCTR_M + 2 * L.slot);
-      st += (uint32_t)v;
-      en += (uint32_t)(v >> 32);
-    }
+    // the launch's counts (the mirror warp publishes them summed over the NCTR_SUB tables)
+    const uint64_t v = *reinterpret_cast<volatile uint64_t*>(cb->mirror_h + 2 * L.slot);
+    const uint32_t st = (uint32_t)v, en = (uint32_t)(v >> 32);
     uint32_t cnt[2] = {st - L.base, en - L.base};
     uint32_t* seen[2] = {&L.p, &L.f};
     bool finished = false;
@@ -1698,13 +1695,12 @@ int paella_check_counters(paella_t* p, uint32_t gpu, uint32_t* slots_checked) {
   for (uint32_t s = 0; s < NCTR_M; ++s) {
     const uint32_t want = g->ctr_mbase[s];   // sum of the grids of every launch counted on slot s
     if (want) ++used;
-    uint32_t d0 = 0, d1 = 0, m0 = 0, m1 = 0;
+    uint32_t d0 = 0, d1 = 0;
     for (uint32_t t = 0; t < NCTR_SUB; ++t) {
       d0 += dev[t * 2 * NCTR_M + 2 * s];
       d1 += dev[t * 2 * NCTR_M + 2 * s + 1];
-      m0 += mir[t * 2 * NCTR_M + 2 * s];
-      m1 += mir[t * 2 * NCTR_M + 2 * s + 1];
     }
+    const uint32_t m0 = mir[2 * s], m1 = mir[2 * s + 1];   // the mirror holds the sums
     // device counters AND their host mirror: every block entered and exited exactly once
     if (d0 != want || d1 != want || m0 != want || m1 != want) ++bad;
   }

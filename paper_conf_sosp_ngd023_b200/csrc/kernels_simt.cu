@@ -722,30 +722,45 @@ KernelFn proxy_kernel() { return (KernelFn)k_notify_proxy; }
 
 // ---------------------------------------------------------------------------
 // Counter mirror (counter-mode notification): one resident warp copies
-// the NCTR_M {start, end} launch counters (2 KiB of device memory) to pinned host
-// memory whenever they change.  Lane i owns 16-byte chunks i, i+32, i+64, i+96 (two
-// slots each).  A changed chunk is copied as loaded (acquire loads), so the host sees
-// a block's outputs no later than the count that covers the block.  The warp leaves
+// the NCTR_M {start, end} launch counters (NCTR_SUB tables of 2 KiB in device memory,
+// summed) to one 2 KiB table in pinned host memory whenever they change.  Lane i owns
+// 16-byte chunks i, i+32, i+64, i+96 of every table (two slots each).  A changed sum is
+// published after the acquire loads of its parts, so the host sees a block's outputs
+// no later than the count that covers the block.  The warp leaves
 // after ~35 ms without changes; the dispatcher relaunches it while launches are in
 // flight (the counters are the state, so nothing is lost across a relaunch).
 // ---------------------------------------------------------------------------
 __global__ void __launch_bounds__(32, 1) k_notify_mirror(const uint4* ctrs, uint4* host, volatile uint32_t* state) {
   const uint32_t pace = state[8];   // diagnosis (PAELLA_MIRROR_PACE_NS): extra pause per scan
   const uint32_t lane = threadIdx.x;
-  constexpr uint32_t NQ = NCTR_SUB * NCTR_M * 2 / 4 / 32;   // 16-byte chunks per lane (all tables)
-  uint4 prev[NQ];
+  // the NCTR_SUB device tables are summed here, so the host reads ONE table of NCTR_M
+  // {start, end} pairs (a quarter of the cache lines its drain loop misses on)
+  constexpr uint32_t NT = NCTR_M * 2 / 4 / 32;   // 16-byte chunks per lane of one table
+  constexpr uint32_t NQ = NCTR_SUB * NT;          // ... of all tables
+  uint4 prev[NT];
 #pragma unroll
-  for (uint32_t i = 0; i < NQ; ++i) prev[i] = make_uint4(~0u, ~0u, ~0u, ~0u);   // publish everything once
+  for (uint32_t i = 0; i < NT; ++i) prev[i] = make_uint4(~0u, ~0u, ~0u, ~0u);   // publish everything once
   uint32_t idle = 0;
   for (;;) {
-    uint4 cur[NQ];
+    uint4 raw[NQ];
+#pragma unroll
+    for (uint32_t i = 0; i < NQ; ++i)
+      asm volatile("ld.acquire.gpu.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+                   : "=r"(raw[i].x), "=r"(raw[i].y), "=r"(raw[i].z), "=r"(raw[i].w)
+                   : "l"(ctrs + lane + 32 * i));
+    uint4 cur[NT];
     bool ch = false;
 #pragma unroll
-    for (uint32_t i = 0; i < NQ; ++i) {
-      asm volatile("ld.acquire.gpu.global.v4.u32 {%0, %1, %2, %3}, [%4];"
-                   : "=r"(cur[i].x), "=r"(cur[i].y), "=r"(cur[i].z), "=r"(cur[i].w)
-                   : "l"(ctrs + lane + 32 * i));
-      ch |= cur[i].x != prev[i].x || cur[i].y != prev[i].y || cur[i].z != prev[i].z || cur[i].w != prev[i].w;
+    for (uint32_t q = 0; q < NT; ++q) {
+      cur[q] = raw[q];
+#pragma unroll
+      for (uint32_t t = 1; t < NCTR_SUB; ++t) {
+        cur[q].x += raw[t * NT + q].x;
+        cur[q].y += raw[t * NT + q].y;
+        cur[q].z += raw[t * NT + q].z;
+        cur[q].w += raw[t * NT + q].w;
+      }
+      ch |= cur[q].x != prev[q].x || cur[q].y != prev[q].y || cur[q].z != prev[q].z || cur[q].w != prev[q].w;
     }
     if (__any_sync(0xffffffffu, ch)) {
       // A block's release reduction made its outputs visible (at system scope for a
@@ -755,7 +770,7 @@ __global__ void __launch_bounds__(32, 1) k_notify_mirror(const uint4* ctrs, uint
       // publish the counts to the host (cumulativity of fence.acq_rel.sys)
       asm volatile("fence.acq_rel.sys;" ::: "memory");
 #pragma unroll
-      for (uint32_t i = 0; i < NQ; ++i) {
+      for (uint32_t i = 0; i < NT; ++i) {
         if (cur[i].x != prev[i].x || cur[i].y != prev[i].y || cur[i].z != prev[i].z || cur[i].w != prev[i].w) {
           asm volatile("st.relaxed.sys.global.v4.u32 [%0], {%1, %2, %3, %4};" ::"l"(host + lane + 32 * i),
                        "r"(cur[i].x), "r"(cur[i].y), "r"(cur[i].z), "r"(cur[i].w)
