@@ -235,7 +235,8 @@ struct FakeBackend : Backend {
 // CUDA backend
 // ---------------------------------------------------------------------------
 // one launch of kernel k: split-K tcgen05 convs are thread-block clusters
-static bool is_tc(uint32_t kind) { return kind == KIND_CONV_TC || kind == KIND_CONV_TC_PRO; }
+static bool is_tc(uint32_t kind) { return kind == KIND_CONV_TC || kind == KIND_CONV_TC_PRO || kind == KIND_CONV_TC128; }
+static uint32_t tc_bn(uint32_t kind) { return kind == KIND_CONV_TC128 ? TC_BN_WIDE : TC_BN; }
 
 // pdl: programmatic dependent launch (programmatic stream serialization).  Measured on
 // B200 (tools/launch_quantum.cu, profiles/launch_quantum_r1.txt): a kernel queued
@@ -382,14 +383,16 @@ struct CudaBackend : Backend {
       if (nstreams) std::rotate(streams.begin(), streams.begin() + (atoi(rot) % nstreams), streams.end());
     cudaMemsetAsync(tail, 0, 256, streams[0]);
     cudaMemsetAsync(ctr, 0, 2 * NCTR * sizeof(uint32_t), streams[0]);
-    KernelFn tc_i[2], tc_p[2];
+    KernelFn tc_i[3], tc_p[3];
     simt_kernel_table(tab[0][1], tab[0][0], tab[1][1], tab[1][0]);
     tc_kernel_table(tc_i, tc_p);
     tab[0][1][KIND_CONV_TC] = tc_i[0];
     tab[0][0][KIND_CONV_TC] = tc_p[0];
     tab[0][1][KIND_CONV_TC_PRO] = tc_i[1];
     tab[0][0][KIND_CONV_TC_PRO] = tc_p[1];
-    for (int i = 0; i < 2; ++i) tab[1][i][KIND_CONV_TC] = tab[1][i][KIND_CONV_TC_PRO] = nullptr;
+    tab[0][1][KIND_CONV_TC128] = tc_i[2];
+    tab[0][0][KIND_CONV_TC128] = tc_p[2];
+    for (int i = 0; i < 2; ++i) tab[1][i][KIND_CONV_TC] = tab[1][i][KIND_CONV_TC_PRO] = tab[1][i][KIND_CONV_TC128] = nullptr;
     if (proxy || mirror) {
       int rc = setup_proxy(streams[0]);
       if (rc) return rc;
@@ -1674,7 +1677,8 @@ int paella_kernel_info(paella_t* p, uint32_t model_id, uint32_t k, paella_kernel
 
 const char* paella_kernel_name(uint32_t kind) {
   static const char* names[] = {"ingest", "conv_simt", "conv_tcgen05", "dwconv", "maxpool",
-                                "avgpool", "gap", "fc_gemv", "empty", "conv_tcgen05_pro", "gap_fc", "spin"};
+                                "avgpool", "gap", "fc_gemv", "empty", "conv_tcgen05_pro", "gap_fc", "spin",
+                                "conv_tcgen05_n128"};
   return kind < KIND_COUNT ? names[kind] : "?";
 }
 
@@ -2003,6 +2007,7 @@ static int autotune_splits(Gpu* g, Model* m) {
         const int n = std::sscanf(line, "%255s %u %u %u", name, &l, &sp, &dsm);
         if (n < 3) continue;
         if (m->name != name || l >= m->kernels.size() || !is_tc(m->kernels[l].kind)) continue;
+        if (m->kernels[l].kind == KIND_CONV_TC128) continue;   // 128-pixel tiles never split
         KernelInst& k = m->kernels[l];
         const uint32_t fl = (n == 4 && dsm) ? (k.proto.flags | LF_SPLIT_DSMEM) : (k.proto.flags & ~LF_SPLIT_DSMEM);
         k.proto.ksplit = sp;
@@ -2021,7 +2026,7 @@ static int autotune_splits(Gpu* g, Model* m) {
   if (iso_run(g, m, nullptr, nullptr, nullptr, true)) return -EIO;
   for (uint32_t l = 0; l < m->kernels.size(); ++l) {
     KernelInst& k = m->kernels[l];
-    if (!is_tc(k.kind)) continue;
+    if (!is_tc(k.kind) || k.kind == KIND_CONV_TC128) continue;   // 128-pixel tiles never split
     const uint32_t nk = k.proto.kpad / TC_BK, tiles = k.proto.tiles_m * k.proto.tiles_n;
     auto set = [&](uint32_t sp, bool dsm) {
       k.proto.ksplit = sp;
@@ -2079,13 +2084,13 @@ static int autotune_splits(Gpu* g, Model* m) {
 // split is > 1), TC_BN x TC_BM floats per output tile.  Zeroed once; every owner CTA
 // re-zeroes the sums it consumed, so the region is all zero between launches.
 static int splitk_workspace(Model* m, ModelGpu& mg, bool iso) {
-  constexpr size_t kTile = (size_t)TC_BN * TC_BM;
+  constexpr size_t kTile = (size_t)TC_BN * TC_BM;   // (KIND_CONV_TC128 never splits)
   uint32_t nvs = 1;
   for (const auto& k : m->kernels)
     if (is_tc(k.kind)) nvs = std::max(nvs, k.vs + 1);
   std::vector<size_t> off(nvs, 0), tiles(nvs, 0);
   for (const auto& k : m->kernels)
-    if (is_tc(k.kind) && (iso || k.proto.ksplit > 1))
+    if (is_tc(k.kind) && k.kind != KIND_CONV_TC128 && (iso || k.proto.ksplit > 1))
       tiles[k.vs] = std::max<size_t>(tiles[k.vs], (size_t)k.proto.tiles_m * k.proto.tiles_n);
   size_t per = 0;
   for (uint32_t v = 0; v < nvs; ++v) {

@@ -17,7 +17,8 @@ enum KernelKind : uint32_t {
   KIND_CONV_TC_PRO = 9, // tcgen05 conv with the per-channel affine+ReLU input prologue
   KIND_GAPFC = 10,      // fused global average pool + FC classifier head
   KIND_SPIN = 11,       // synthetic HoL-microbenchmark kernel (Fig. 2): one resident block
-  KIND_COUNT = 12,
+  KIND_CONV_TC128 = 12, // tcgen05 conv with 128-pixel tiles (saturating shapes, no split-K)
+  KIND_COUNT = 13,
 };
 
 typedef void (*KernelFn)();
@@ -36,6 +37,8 @@ constexpr uint32_t TC_BM = 128;       // Cout rows per CTA (UMMA M, TMEM lanes)
 constexpr uint32_t TC_BN = 64;        // output pixels per CTA (UMMA N)
 constexpr uint32_t TC_BK = 64;        // K per pipeline stage (128 B of bf16 = one swizzle row)
 constexpr uint32_t TC_STAGES = 4;
+constexpr uint32_t TC_RING = TC_STAGES * (TC_BM * TC_BK * 2 + TC_BN * TC_BK * 2);   // 96 KiB stage ring
+constexpr uint32_t TC_BN_WIDE = 128;   // KIND_CONV_TC128: 3 stages of 16 + 16 KiB in the same ring
 constexpr uint32_t GAPFC_CLUSTER = 8;   // fused GAP+FC head: CTAs per cluster (pooling split)
 constexpr uint32_t TC_THREADS = 192;    // 4 producer/epilogue warps + 1 MMA warp + 1 bookkeeping warp
 uint32_t tc_smem_bytes();

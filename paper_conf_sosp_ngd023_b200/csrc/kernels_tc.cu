@@ -216,7 +216,7 @@ __device__ __forceinline__ void epi_tile(const LayerArgs& a, const float* stage,
 // only the block bookkeeping (instrumentation), so no compute warp waits on its
 // atomics at entry.
 constexpr uint32_t TBOOK = NPROD + 32;   // warp 5, lane 0
-template <bool INSTR, bool PRO>
+template <bool INSTR, bool PRO, uint32_t BN>
 __global__ void __launch_bounds__(TC_THREADS, 2)
     k_conv_tc(const __grid_constant__ LayerArgs a, const __grid_constant__ InstrArgs ia,
               const __grid_constant__ CUtensorMap wmap) {
@@ -232,8 +232,11 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   // aliasing with global stores
   uint8_t* smem = smem_raw + ((1024u - (su32(smem_raw) & 1023u)) & 1023u);
   uint8_t* sA = smem;                                  // STAGES x 16 KiB
-  uint8_t* sB = smem + TC_STAGES * A_BYTES;            // STAGES x 8 KiB
-  uint64_t* full = (uint64_t*)(sB + TC_STAGES * B_BYTES);
+  constexpr uint32_t BNB = BN * TC_BK * 2;                      // B stage bytes: 8 / 16 KiB
+  constexpr uint32_t NST = TC_RING / (A_BYTES + BNB);           // 4 stages (BN 64) / 3 (BN 128)
+  constexpr uint32_t RPT = BN / 16;                             // B pixel rows per gather thread
+  uint8_t* sB = smem + NST * A_BYTES;
+  uint64_t* full = (uint64_t*)(smem + TC_RING);
   uint64_t* empty = full + TC_STAGES;
   uint64_t* accb = empty + TC_STAGES;
   uint64_t* rbar = accb + 1;                           // split-K: peers' slices landed
@@ -243,21 +246,21 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   const uint32_t warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const uint32_t tile_n = blockIdx.x, tile_m = blockIdx.y, split = blockIdx.z;
   const uint32_t P = a.oh * a.ow;
-  const uint32_t n0 = tile_n * TC_BN, m0 = tile_m * TC_BM;
+  const uint32_t n0 = tile_n * BN, m0 = tile_m * TC_BM;
   const uint32_t nk = a.kpad / TC_BK;
   const uint32_t per = (nk + a.ksplit - 1) / a.ksplit;
   const uint32_t kb0 = split * per;
   const uint32_t kb1 = min(nk, kb0 + per);
   const uint32_t nkl = kb1 > kb0 ? kb1 - kb0 : 0;
 
-  const uint32_t pre = nkl < TC_STAGES ? nkl : TC_STAGES;
+  const uint32_t pre = nkl < NST ? nkl : NST;
   // narrow layers (Cout < 128) fetch only a_rows weight rows per stage; rows a_rows..127
   // of every A stage are zeroed once below (the UMMA still runs M = 128)
   const uint32_t abytes = a.a_rows * 128;
   if (warp == 4 && lane == 0) {
     // the MMA warp's leader sets up the barriers and starts the weight stream while
     // the gather warps compute their addresses
-    for (uint32_t s = 0; s < TC_STAGES; ++s) {
+    for (uint32_t s = 0; s < NST; ++s) {
       mbar_init(&full[s], NPROD + 1);
       mbar_init(&empty[s], 1);
     }
@@ -275,31 +278,31 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   // fetched before the PDL wait, the residual right after it, both hidden behind the
   // main loop.  Thread t owns channel group eg = t % 16 and pixels t / 16 + 8 i.
   const uint32_t eg = threadIdx.x % (TC_BM / 8), eco = m0 + eg * 8;
-  constexpr uint32_t NIT = TC_BN * (TC_BM / 8) / NPROD;   // 8 items per thread
+  constexpr uint32_t NIT = BN * (TC_BM / 8) / NPROD;   // 8 items per thread (BN 64)
   float ebias[8];
   uint4 eres[NIT];
   if (warp < 4 && a.ksplit == 1) load_bias8(a, eco, ebias);
   // ---- producer state (warps 0-3): this thread gathers 16-byte chunk `chunk` of
-  // pixel rows n = t/8 + 16 j (j < 4) of every B stage
+  // pixel rows n = t/8 + 16 j (j < RPT) of every B stage
   const __nv_bfloat16* X = static_cast<const __nv_bfloat16*>(a.in);
   const uint32_t t = threadIdx.x;
   const uint32_t chunk = t % 8;
   // per pixel row j: top-left input coordinate of its window (invalid pixels get a
   // coordinate that fails every bounds check) and its element offset; per stage only
   // the (r, s, ci) offset `dk`, common to the 4 rows, changes
-  int ih0[4], iw0[4], off0[4];
+  int ih0[RPT], iw0[RPT], off0[RPT];
   const uint32_t K = a.kh * a.kw * a.cin;
   const uint32_t dst0 = (t / 8) * 128 + ((chunk ^ ((t / 8) & 7)) << 4);   // row t/8 of the SW128 atom
   // (r, s, ci) of k = kbase + 8*chunk, advanced incrementally by TC_BK per stage
   int kr = 0, ks_ = 0, kci = 0;
   uint32_t kcur = 0;
   auto issue_B = [&](uint32_t it, bool arrive) {
-    const uint32_t s = it % TC_STAGES;
+    const uint32_t s = it % NST;
     const bool kv = kcur < K;
     const int dk = (kr * (int)a.w_ + ks_) * (int)a.in_cs + kci;
-    const uint32_t bstage = su32(sB + s * B_BYTES) + dst0;
+    const uint32_t bstage = su32(sB + s * BNB) + dst0;
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
+    for (uint32_t j = 0; j < RPT; ++j) {
       const bool ok = kv && (uint32_t)(ih0[j] + kr) < a.h && (uint32_t)(iw0[j] + ks_) < a.w_;
       const __nv_bfloat16* src = ok ? X + (off0[j] + dk) : X;
       const uint32_t dst = bstage + j * 2048;   // pixel row n = t/8 + 16 j
@@ -335,7 +338,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   int tr_r = 0, tr_s = 0, tr_ci = 0;
   uint32_t tr_k = 0;
   auto transform_B = [&](uint32_t it) {
-    const uint32_t bstage = su32(sB + (it % TC_STAGES) * B_BYTES) + dst0;
+    const uint32_t bstage = su32(sB + (it % NST) * BNB) + dst0;
     if (tr_k < K) {
       const float4 s0 = __ldg(reinterpret_cast<const float4*>(a.pro_scale + tr_ci));
       const float4 s1 = __ldg(reinterpret_cast<const float4*>(a.pro_scale + tr_ci + 4));
@@ -344,7 +347,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       const float sc[8] = {s0.x, s0.y, s0.z, s0.w, s1.x, s1.y, s1.z, s1.w};
       const float sh[8] = {z0.x, z0.y, z0.z, z0.w, z1.x, z1.y, z1.z, z1.w};
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
+      for (uint32_t j = 0; j < RPT; ++j) {
         // padding and empty pixels stay zero (padding pads the activated tensor)
         if ((uint32_t)(ih0[j] + tr_r) < a.h && (uint32_t)(iw0[j] + tr_s) < a.w_) {
           const uint32_t adr = bstage + j * 2048;
@@ -377,7 +380,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   };
   if (warp < 4) {
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
+    for (uint32_t j = 0; j < RPT; ++j) {
       const uint32_t p = n0 + t / 8 + 16 * j;
       const bool pv = p < P;
       const int oh = (int)(p / a.ow), ow = (int)(p - (uint32_t)oh * a.ow);
@@ -396,7 +399,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     }
     if (a.a_rows < TC_BM) {
       const uint32_t zb = A_BYTES - abytes;   // bytes per stage, multiple of 1024
-      for (uint32_t o = t * 16; o < TC_STAGES * zb; o += NPROD * 16) {
+      for (uint32_t o = t * 16; o < NST * zb; o += NPROD * 16) {
         const uint32_t st = o / zb;
         asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(su32(sA + st * A_BYTES + abytes + (o - st * zb))),
                      "r"(0u)
@@ -428,9 +431,9 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     if constexpr (!PRO) {
       for (uint32_t it = 0; it < pre; ++it)
         asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(su32(&full[it])) : "memory");
-      for (uint32_t nxt = TC_STAGES; nxt < nkl; ++nxt) {
-        const uint32_t s = nxt % TC_STAGES;
-        mbar_wait(&empty[s], ((nxt / TC_STAGES) & 1) ^ 1);   // MMA of stage nxt - STAGES retired
+      for (uint32_t nxt = NST; nxt < nkl; ++nxt) {
+        const uint32_t s = nxt % NST;
+        mbar_wait(&empty[s], ((nxt / NST) & 1) ^ 1);   // MMA of stage nxt - NST retired
         if (t == 0) {
           mbar_arrive_tx(&full[s], abytes);
           tma_load_2d(sA + s * A_BYTES, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
@@ -441,7 +444,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       // prologue path: wait for this thread's own copies of stage it (cp.async groups,
       // STAGES in flight), transform them in place, publish to the async proxy, arrive
       for (uint32_t it = 0; it < nkl; ++it) {
-        const uint32_t issued = min(nkl, it + TC_STAGES);
+        const uint32_t issued = min(nkl, it + NST);
         switch (issued - it - 1) {
           case 0: cp_async_wait<0>(); break;
           case 1: cp_async_wait<1>(); break;
@@ -450,11 +453,11 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
         }
         transform_B(it);
         fence_proxy_async();
-        mbar_arrive(&full[it % TC_STAGES]);
-        const uint32_t nxt = it + TC_STAGES;
+        mbar_arrive(&full[it % NST]);
+        const uint32_t nxt = it + NST;
         if (nxt < nkl) {
-          const uint32_t s = nxt % TC_STAGES;
-          mbar_wait(&empty[s], ((nxt / TC_STAGES) & 1) ^ 1);
+          const uint32_t s = nxt % NST;
+          mbar_wait(&empty[s], ((nxt / NST) & 1) ^ 1);
           if (t == 0) {
             mbar_arrive_tx(&full[s], abytes);
             tma_load_2d(sA + s * A_BYTES, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
@@ -467,7 +470,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   } else if (warp == 4) {
     // ------------------------------------------------------------ MMA warp
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(su32(tmem_slot)),
-                 "r"(64u)
+                 "r"(BN)
                  : "memory");
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
     tc_fence_before();
@@ -475,14 +478,14 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     tc_fence_after();
     const uint32_t tmem = *tmem_slot;
     if (lane == 0) {
-      constexpr uint32_t IDESC = idesc_bf16(TC_BM, TC_BN);
+      constexpr uint32_t IDESC = idesc_bf16(TC_BM, BN);
       for (uint32_t it = 0; it < nkl; ++it) {
-        const uint32_t s = it % TC_STAGES;
-        mbar_wait(&full[s], (it / TC_STAGES) & 1);
+        const uint32_t s = it % NST;
+        mbar_wait(&full[s], (it / NST) & 1);
         if (trace && it == 0) tr[2] = globaltimer();
         fence_proxy_async();   // the gathered B tile was written through the generic proxy
         tc_fence_after();
-        const uint32_t abase = su32(sA + s * A_BYTES), bbase = su32(sB + s * B_BYTES);
+        const uint32_t abase = su32(sA + s * A_BYTES), bbase = su32(sB + s * BNB);
 #pragma unroll
         for (uint32_t kk = 0; kk < TC_BK / 16; ++kk) {
           umma_bf16(tmem, sdesc_sw128(abase + kk * 32), sdesc_sw128(bbase + kk * 32), IDESC,
@@ -520,7 +523,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       tc_fence_after();
       const uint32_t taddr = *tmem_slot + ((warp * 32) << 16);
 #pragma unroll
-      for (int c = 0; c < 4; ++c) {
+      for (uint32_t c = 0; c < BN / 16; ++c) {
         float v[16];
         tmem_ld16(taddr + c * 16, v);
 #pragma unroll
@@ -529,7 +532,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       if (trace && threadIdx.x == 0) tr[8] = globaltimer();
     } else {
 #pragma unroll 8
-      for (int j = 0; j < 64; ++j) stage[j * TC_BM + row] = 0.f;
+      for (uint32_t j = 0; j < BN; ++j) stage[j * TC_BM + row] = 0.f;
     }
   }
   if (a.ksplit == 1) {
@@ -563,14 +566,14 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     // (the workspace is all zero between launches) and runs the epilogue for them.  The
     // fp32 additions happen in L2 in arrival order (one bf16 rounding afterwards).
     // Items of thread t: pixel rows px0 + (t + 128 i) / 16 (i < 4), channel group t % 16.
-    constexpr uint32_t MAXI = TC_BN * (TC_BM / 8) / (2 * NPROD);   // 4 items at ksplit 2
+    constexpr uint32_t MAXI = BN * (TC_BM / 8) / (2 * NPROD);   // 4 items at ksplit 2 (BN 64)
     const uint32_t ks = a.ksplit;
-    const uint32_t rows = TC_BN / ks;
+    const uint32_t rows = BN / ks;
     const uint32_t px0 = split * rows;
     const uint32_t g = threadIdx.x % (TC_BM / 8), co = m0 + g * 8;
     const uint32_t nitems = rows * (TC_BM / 8);
-    const uint32_t rv = n0 >= P ? 0u : min(TC_BN, P - n0);   // pixel rows of the tile that exist
-    float* wt = a.ws + (size_t)(tile_m * gridDim.x + tile_n) * (TC_BN * TC_BM);
+    const uint32_t rv = n0 >= P ? 0u : min(BN, P - n0);   // pixel rows of the tile that exist
+    float* wt = a.ws + (size_t)(tile_m * gridDim.x + tile_n) * (BN * TC_BM);
     float bias[8];
     uint4 rres[MAXI];
     if (warp < 4 && co < a.cout) {
@@ -649,14 +652,14 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     // epilogue for it -- no global workspace, no atomics, no per-element remote loads
     // (those were bound at ~17 GB/s per SM: 1.7 us for ksplit 8).
     // Items of thread t: pixel rows px0 + (t + 128 i) / 16 (i < 4), channel group t % 16.
-    constexpr uint32_t MAXI = TC_BN * (TC_BM / 8) / (2 * NPROD);   // 4 items at ksplit 2
+    constexpr uint32_t MAXI = BN * (TC_BM / 8) / (2 * NPROD);   // 4 items at ksplit 2 (BN 64)
     const uint32_t ks = a.ksplit;
-    const uint32_t rows = TC_BN / ks;
+    const uint32_t rows = BN / ks;
     const uint32_t px0 = split * rows;
     const uint32_t g = threadIdx.x % (TC_BM / 8), co = m0 + g * 8;
     const uint32_t nitems = rows * (TC_BM / 8);
     const uint32_t slice = rows * TC_BM * 4;                // bytes of one slice (slot pitch)
-    float* recv = stage + TC_BN * TC_BM;                    // ks - 1 received slices (free A stages)
+    float* recv = stage + BN * TC_BM;                       // ks - 1 received slices (free A stages)
     // only the slice rows that hold real pixels travel (the tile tail past P does not)
     auto valid_rows = [&](uint32_t owner) -> uint32_t {
       const uint32_t r0 = n0 + owner * rows;
@@ -733,7 +736,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   __syncthreads();
   if (warp == 4) {
     tc_fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tmem_slot), "r"(64u) : "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tmem_slot), "r"(BN) : "memory");
     // every other thread is past the barrier above: the MMA warp, last to finish, counts
     // the block's exit itself (no second block barrier)
     if (trace && lane == 0) tr[6] = globaltimer();
@@ -742,13 +745,16 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   }
 }
 
-uint32_t tc_smem_bytes() { return 1024 + TC_STAGES * (A_BYTES + B_BYTES) + 128; }
+uint32_t tc_smem_bytes() { return 1024 + TC_RING + 128; }   // align pad + stage ring + barriers
+static_assert(TC_RING == TC_STAGES * (A_BYTES + B_BYTES), "ring");
 
 void tc_kernel_table(KernelFn* instr, KernelFn* plain) {
-  instr[0] = (KernelFn)k_conv_tc<true, false>;
-  plain[0] = (KernelFn)k_conv_tc<false, false>;
-  instr[1] = (KernelFn)k_conv_tc<true, true>;     // with the DenseNet prologue
-  plain[1] = (KernelFn)k_conv_tc<false, true>;
+  instr[0] = (KernelFn)k_conv_tc<true, false, TC_BN>;
+  plain[0] = (KernelFn)k_conv_tc<false, false, TC_BN>;
+  instr[1] = (KernelFn)k_conv_tc<true, true, TC_BN>;     // with the DenseNet prologue
+  plain[1] = (KernelFn)k_conv_tc<false, true, TC_BN>;
+  instr[2] = (KernelFn)k_conv_tc<true, false, TC_BN_WIDE>;   // 128-pixel tiles
+  plain[2] = (KernelFn)k_conv_tc<false, false, TC_BN_WIDE>;
 }
 
 // Host: tensor map for the packed weights [rows][kpad] bf16, box 64 x box_rows

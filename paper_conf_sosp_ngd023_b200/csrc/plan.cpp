@@ -290,12 +290,20 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
             if (std::getenv("PAELLA_SPLIT_RELBAR")) a.flags |= LF_SPLIT_RELBAR;
             // narrow layers: fetch only the live weight rows (SW128 atoms are 8 rows)
             a.a_rows = nd.c < TC_BM ? (uint32_t)align_up(nd.c, 8) : TC_BM;
+            k.tmem_cols = tc_tmem_cols();
+            // saturating shapes (>= 2 waves of 64-pixel tiles at 2 CTAs/SM, no split, no
+            // prologue): 128-pixel tiles halve the weight traffic per flop.  Batch-1
+            // serving layers stay below this (at most 196 tiles of 64 pixels at 224^2).
+            if (k.kind == KIND_CONV_TC && split == 1 && tiles >= 4 * P->sms && !std::getenv("PAELLA_NO_WIDE")) {
+              k.kind = KIND_CONV_TC128;
+              a.tiles_n = (P_out + TC_BN_WIDE - 1) / TC_BN_WIDE;
+              k.tmem_cols = TC_BN_WIDE;
+            }
             k.grid[0] = a.tiles_n;
             k.grid[1] = a.tiles_m;
             k.grid[2] = split;
             k.block = TC_THREADS;
             k.smem = tc_smem_bytes();
-            k.tmem_cols = tc_tmem_cols();
 
           } else {
             k.kind = KIND_CONV_SIMT;

@@ -552,3 +552,34 @@ def test_bench_xdev_graph_replay():
         r32 = e.bench_xdev(mids, seq, streams=32)
         r1 = e.bench_xdev(mids, seq, streams=1)
     assert 0 < r1 < r32 < 1e6, (r1, r32)
+
+
+def test_wide_tile_conv_parity(engine):
+    """KIND_CONV_TC128 (128-pixel tiles, chosen for saturating shapes: >= 2 waves of
+    64-pixel tiles): a 3x3 64->64 conv over 200x200 pixels (625 tiles of 64) and the
+    logits behind it match the float64 oracle -- the conv's own output element by
+    element (bf16 tolerance), with the ragged last tile (40,000 = 312 x 128 + 64)."""
+    from oracle.bf16 import round_bf16
+    g = archs.Graph("wide200", (3, 200, 200), 10)
+    x = g.conv(g.input, 64, 1, name="stem")
+    y = g.conv(x, 64, 3, 1, 1, name="big")
+    z = g.gap(y, name="gap")
+    g.fc(z, 10, name="fc")
+    r = np.random.default_rng(5)
+    P = {}
+    for nd in g.weight_nodes():
+        shp = g.param_shapes()[nd["name"] + ".weight"]
+        P[nd["name"] + ".weight"] = round_bf16((r.standard_normal(shp) / np.sqrt(np.prod(shp[1:]))).astype(np.float32))
+        P[nd["name"] + ".bias"] = (0.01 * r.standard_normal(shp[0])).astype(np.float32)
+    mid = engine.register_model(g, P, dtype=L.DTYPE_BF16, name="wide200")
+    names = [k["name"] for k in engine.kernels(mid)]
+    assert "conv_tcgen05_n128" in names, names
+    img = r.standard_normal((1, 3, 200, 200)).astype(np.float32)
+    out = engine.run_isolated(mid, img)
+    vals = infer.forward(g, P, img, dtype="bf16", return_all=True)
+    big = next(nd["id"] for nd in g.nodes if nd["name"] == "big")
+    got = engine.debug_node(mid, big, (64, 200, 200))
+    want = vals[big]
+    ok = within(got, want, BF16_TOL)
+    assert ok.all(), (int((~ok).sum()), float(np.abs(got - want).max()))
+    assert within(out, vals[g.output].reshape(-1), BF16_TOL).all()
