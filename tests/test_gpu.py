@@ -573,7 +573,7 @@ def test_wide_tile_conv_parity(engine):
         P[nd["name"] + ".bias"] = (0.01 * r.standard_normal(shp[0])).astype(np.float32)
     mid = engine.register_model(g, P, dtype=L.DTYPE_BF16, name="wide200")
     names = [k["name"] for k in engine.kernels(mid)]
-    assert "conv_tcgen05_n128" in names, names
+    assert any(n.startswith("conv_tcgen05_n") for n in names), names   # n128 (or n256: PAELLA_WIDE=256)
     img = r.standard_normal((1, 3, 200, 200)).astype(np.float32)
     out = engine.run_isolated(mid, img)
     vals = infer.forward(g, P, img, dtype="bf16", return_all=True)
