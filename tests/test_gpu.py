@@ -428,20 +428,22 @@ def test_hybrid_completion_serving(tmp_path):
     assert cpu < 0.7 * wall, (cpu, wall)
 
 
-@pytest.mark.parametrize("look,K", [(3, 8), (0, 0)])
+@pytest.mark.parametrize("look,K", [(3, 8), (0, 0), (-6, 8)])
 def test_serving_branches_c3_models(tmp_path, look, K):
     """NEXT-4 intra-job branch concurrency on the GPU: C-3's models served with their
     kernel DAGs over virtual streams (Inception / ResNet-50 branches on several CUDA
     streams at once; a consumer on another stream is issued after its inputs' final
     COMPLETION, whose exit count is a release): every output within the bf16 tolerance,
-    the issue order replayed bit-exactly, launch-ahead depth respected per stream."""
+    the issue order replayed bit-exactly, launch-ahead depth respected per stream.
+    look < 0: launch-ahead |look| without the placement test (the bench arms' rule)."""
     log = str(tmp_path / "br_%u.log")
+    unpl, look = look < 0, abs(look)
     names = ["resnet50", "inception_v3", "mobilenet_v2", "squeezenet1_1"]
     for nm in names:
         for i in range(4):
             oracle_out(nm, i, "bf16")
     with L.Engine(num_clients=4, event_log=log, max_jobs_per_model=32, lookahead=look, launch_threads=4,
-                  slack=1184, region_bytes=96 << 20, branches=True, max_active=K) as e:
+                  slack=1184, region_bytes=96 << 20, branches=True, max_active=K, lookahead_unplaced=unpl) as e:
         specs = []
         for nm in names:
             g = archs.build(nm)

@@ -354,14 +354,17 @@ def test_planner_dag_matches_graph(name):
 
 
 @pytest.mark.parametrize("policy,look,K", [(L.POLICY_SRPT_DEFICIT, 0, 0), (L.POLICY_SRPT_DEFICIT, 2, 0),
-                                           (L.POLICY_FIFO, 3, 2), (L.POLICY_SRPT_DEFICIT, 3, 3)])
+                                           (L.POLICY_FIFO, 3, 2), (L.POLICY_SRPT_DEFICIT, 3, 3),
+                                           (L.POLICY_SRPT_DEFICIT, -6, 3)])
 def test_fake_replay_branches(tmp_path, policy, look, K):
     """NEXT-4: jobs whose kernels form a DAG over virtual streams (several CUDA streams
-    per job) replay bit-exactly through the oracle policy (Topo / head)."""
+    per job) replay bit-exactly through the oracle policy (Topo / head).  look < 0:
+    launch-ahead |look| without the placement test."""
     log = str(tmp_path / "ev_%u.log")
     models = [archs.squeezenet1_1(), archs.inception_v3()]
+    unpl, look = look < 0, abs(look)
     with _toy_engine(num_clients=2, policy=policy, streams=12, event_log=log, ring_capacity=4096, slack=8,
-                     lookahead=look, branches=True, max_active=K, fake_sms=8) as e:
+                     lookahead=look, branches=True, max_active=K, fake_sms=8, lookahead_unplaced=unpl) as e:
         mids = [e.register_model(g, rng.model_params(g)) for g in models]
         _serve(e, mids, 60, 2, seed=17 + look)
     cfg, ms, events, ex = eventlog.read(log % 0)
