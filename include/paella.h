@@ -45,7 +45,7 @@
 extern "C" {
 #endif
 
-#define PAELLA_ABI_VERSION 1u
+#define PAELLA_ABI_VERSION 2u   /* 2: paella_config_t.lookahead_unplaced */
 #define PAELLA_NOTIFY_COUNTERS 0u
 #define PAELLA_NOTIFY_RING     1u
 

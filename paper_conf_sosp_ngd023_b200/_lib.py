@@ -16,7 +16,7 @@ import numpy as np
 HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "libpaella.so")
 
-ABI_VERSION = 1
+ABI_VERSION = 2
 NOTIFY_COUNTERS, NOTIFY_RING = 0, 1
 POLICY_SRPT_DEFICIT, POLICY_FIFO, POLICY_SJF, POLICY_RR = 0, 1, 2, 3
 ROUTE_LEAST_WORK, ROUTE_ROUND_ROBIN, ROUTE_POWER_OF_TWO = 0, 1, 2
