@@ -45,7 +45,7 @@
 extern "C" {
 #endif
 
-#define PAELLA_ABI_VERSION 2u   /* 2: paella_config_t.lookahead_unplaced */
+#define PAELLA_ABI_VERSION 2u   /* 2: paella_config_t.lookahead_unplaced, cap_arrival_order */
 #define PAELLA_NOTIFY_COUNTERS 0u
 #define PAELLA_NOTIFY_RING     1u
 
@@ -192,6 +192,11 @@ typedef struct {
                                     queued blocks).  Kernels shorter than the notification
                                     round trip otherwise complete before their placement is
                                     seen and launch-ahead degenerates to one kernel at a time */
+  uint32_t cap_arrival_order;     /* with max_active_jobs = K: 0 = the K first live jobs in the
+                                    policy's order (SRPT: remaining time) may issue; 1 = the K
+                                    first in ARRIVAL order (the policy still orders the ready
+                                    jobs among them): a long job cannot be kept out of the cap
+                                    by a stream of shorter arrivals */
 } paella_config_t;
 
 /* One routing decision.  W_g = work[g] + pending[g] * tbar_model:

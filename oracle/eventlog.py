@@ -7,7 +7,7 @@ Format (DESIGN.md §"Event log"): a sequence of 32-byte little-endian records
   100 CONFIG    a=N clients, b=policy, c=theta, d=(B << 32) | G
   100 CONFIG    a=0xFFFFFFFF, b=ring capacity, c=stream pool P, d=(priority classes << 32) | launch-ahead depth
   100 CONFIG    a=0xFFFFFFFE, b=online T-bar refinement (NEXT-4), c=max_active K (B200-Q6),
-                d=branches | lookahead_unplaced << 8 (NEXT-1 variant)
+                d=branches | lookahead_unplaced << 8 (NEXT-1 variant) | cap_fifo << 9 (B200-Q6 variant)
   101 CAPACITY  a=resource r, b=C_r
   110 MODEL     a=model, b=#kernels
   111 LAYER     a=model, b=layer, c=grid, d=T-bar ns
@@ -62,6 +62,7 @@ def read(path):
                 cfg_kw["online_tbar"] = b
                 cfg_kw["max_active"] = c
                 cfg_kw["lookahead_unplaced"] = (d >> 8) & 1
+                cfg_kw["cap_fifo"] = (d >> 9) & 1
             elif a == 0xFFFFFFFF:
                 cfg_kw["ring_capacity"] = b
                 cfg_kw["streams"] = c

@@ -80,6 +80,7 @@ class Config:
     max_active: int = 0               # K: only the K first jobs in the policy's order that still
                                       # have kernels to issue may issue (0 = no cap); B200-Q6
     lookahead_unplaced: int = 0       # NEXT-1 variant: launch-ahead without the oldest-placed test
+    cap_fifo: int = 0                 # B200-Q6 variant: the job cap admits in arrival order
 
 
 # NEXT-4 (P1249-1266: "x-bar is the average of all previous observations of x"; "these
@@ -301,12 +302,14 @@ class Policy:
 
     def eligible(self):
         """B200-Q6: with max_active = K > 0, the ids of the K first jobs, in the
-        policy's order, among the live jobs that still have kernels to issue; None = no cap."""
+        policy's order (cap_fifo: in arrival order), among the live jobs that still have
+        kernels to issue; None = no cap."""
         K = self.cfg.max_active
         if K <= 0:
             return None
         left = [j for j in self.jobs.values() if j.cursor < len(self.models[j.model])]
-        return {j.id for j in sorted(left, key=self.order)[:K]}
+        key = (lambda j: (j.seq, j.id)) if self.cfg.cap_fifo else self.order
+        return {j.id for j in sorted(left, key=key)[:K]}
 
     def pick(self, rdy):
         cfg = self.cfg

@@ -56,7 +56,8 @@ class Config(C.Structure):
                 ("decide_delay_ns", C.c_uint32), ("naive_pdl", C.c_uint32), ("watchdog_ms", C.c_uint32),
                 ("fake_fault", C.c_uint32), ("fake_fault_arg", C.c_uint32), ("branches", C.c_uint32),
                 ("route_log_path", C.c_char_p),
-                ("max_active_jobs", C.c_uint32), ("lookahead_unplaced", C.c_uint32)]
+                ("max_active_jobs", C.c_uint32), ("lookahead_unplaced", C.c_uint32),
+                ("cap_arrival_order", C.c_uint32)]
 
 
 class Node(C.Structure):
@@ -190,7 +191,7 @@ class Engine:
                  launch_threads=0, proxy=True, pdl=True, prio_classes=1,
                  notify="counters", decide_delay_ns=0, online_tbar=False, naive_pdl=False, watchdog_ms=0,
                  fake_fault=0, fake_fault_arg=0, route_log=None, max_active=0, branches=False,
-                 lookahead_unplaced=False):
+                 lookahead_unplaced=False, cap_fifo=False):
         self.lib = load()
         cfg = Config()
         cfg.abi_version = ABI_VERSION
@@ -234,6 +235,7 @@ class Engine:
         cfg.route_log_path = self._rlog
         cfg.max_active_jobs = max_active
         cfg.lookahead_unplaced = 1 if lookahead_unplaced else 0
+        cfg.cap_arrival_order = 1 if cap_fifo else 0
         cfg.branches = 1 if branches else 0
         # notification path: "counters" (default), "ring" (device ring + forwarding warp),
         # "direct" (the paper's direct ring writes; same as proxy=False)

@@ -1242,7 +1242,9 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
   if (cfg.prio_classes > cfg.stream_pool && cfg.stream_pool != 0) return -EINVAL;
   if (cfg.launch_threads > 16) return -EINVAL;
   if (cfg.max_jobs_per_model > 4096) return -EINVAL;   // job ids: 65,536 per GPU
-  if (cfg.fake_fault > PAELLA_FAULT_CORRUPT || cfg.branches > 1 || cfg.lookahead_unplaced > 1) return -EINVAL;
+  if (cfg.fake_fault > PAELLA_FAULT_CORRUPT || cfg.branches > 1 || cfg.lookahead_unplaced > 1 ||
+      cfg.cap_arrival_order > 1)
+    return -EINVAL;
 
   auto P = std::make_unique<Paella>();
   P->cfg = cfg;
@@ -1350,6 +1352,7 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
     pc.online_tbar = cfg.online_tbar;
     pc.max_active = cfg.max_active_jobs;
     pc.la_unplaced = cfg.lookahead_unplaced ? 1u : 0u;
+    pc.cap_fifo = cfg.cap_arrival_order ? 1u : 0u;
     for (int r = 0; r < NRES; ++r) pc.capacity[r] = P->capacity[r];
     if (cfg.device == PAELLA_DEVICE_CUDA &&
         (static_cast<CudaBackend*>(g->be.get())->proxy || static_cast<CudaBackend*>(g->be.get())->mirror)) {
@@ -1375,7 +1378,8 @@ int paella_init(const paella_config_t* cfg_in, paella_t** out) {
       logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFFu, cfg.ring_capacity, cfg.stream_pool,
             ((uint64_t)pc.prio_classes << 32) | cfg.lookahead);
       logev(g.get(), EV_CONFIG + 0, 0xFFFFFFFEu, cfg.online_tbar, cfg.max_active_jobs,
-            cfg.branches | ((uint64_t)(cfg.lookahead_unplaced ? 1 : 0) << 8));
+            cfg.branches | ((uint64_t)(cfg.lookahead_unplaced ? 1 : 0) << 8) |
+                ((uint64_t)(cfg.cap_arrival_order ? 1 : 0) << 9));
       for (int r = 0; r < NRES; ++r) logev(g.get(), EV_CAPACITY, (uint32_t)r, (uint64_t)pc.capacity[r], 0, 0);
     }
     if (cfg.device == PAELLA_DEVICE_CUDA &&

@@ -140,10 +140,11 @@ int64_t Policy::order_key(const PolicyJob& j) const {
   return j.R;
 }
 
-// the policy's total order (oracle Policy.order): SRPT R_j, SJF model T-bar sum, RR last
-// issued uid, FIFO arrival only; ties (seq, id)
+// the order of the job cap (oracle Policy.eligible): the policy's total order (SRPT R_j,
+// SJF model T-bar sum, RR last issued uid, FIFO arrival only), or arrival only with
+// cap_fifo; ties (seq, id)
 int64_t Policy::active_key(const PolicyJob& j) const {
-  return cfg_.policy == POL_FIFO ? 0 : order_key(j);
+  return (cfg_.policy == POL_FIFO || cfg_.cap_fifo) ? 0 : order_key(j);
 }
 void Policy::active_erase(const PolicyJob& j) {
   if (cfg_.max_active) active_.erase(std::make_tuple(active_key(j), j.seq, j.id));
@@ -259,6 +260,22 @@ int Policy::lowest_free() const {
 // policy's order over live jobs with kernels left to issue); false if none is ready
 bool Policy::pick_capped(uint32_t* job_id) const {
   uint32_t k = 0;
+  if (cfg_.cap_fifo && cfg_.policy != POL_FIFO) {
+    // the cap admits in arrival order; among its ready jobs the policy's order decides
+    bool found = false;
+    std::tuple<int64_t, uint64_t, uint32_t> best{};
+    for (auto it = active_.begin(); it != active_.end() && k < cfg_.max_active; ++it, ++k) {
+      const PolicyJob& j = jobs_[std::get<2>(*it)];
+      if (!j.in_ready) continue;
+      const auto key = std::make_tuple(order_key(j), j.seq, j.id);
+      if (!found || key < best) {
+        best = key;
+        found = true;
+      }
+    }
+    if (found) *job_id = std::get<2>(best);
+    return found;
+  }
   for (auto it = active_.begin(); it != active_.end() && k < cfg_.max_active; ++it, ++k) {
     const uint32_t id = std::get<2>(*it);
     if (jobs_[id].in_ready) {

@@ -93,6 +93,7 @@ class Policy {
     uint32_t max_active = 0;     // K: only the K first jobs in the policy's order that still
                                  // have kernels to issue may issue (0 = no cap); B200-Q6
     uint32_t la_unplaced = 0;    // NEXT-1 variant: launch-ahead without the oldest-placed test
+    uint32_t cap_fifo = 0;       // B200-Q6 variant: the job cap admits in arrival order
   };
   static constexpr int64_t kProfileRuns = 20;   // observations behind the profiled T-bar
   // class of stream s: consecutive index ranges, class 0 = highest hardware priority

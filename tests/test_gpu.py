@@ -157,6 +157,7 @@ def _serve_and_check(e, specs, n, n_clients, seed, rate_us=30.0):
     (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 3, 4, "counters", -4),  # bench arm + online T-bar (NEXT-4)
     (L.POLICY_SJF, 16, 32, 65536, 3, 4, "counters", 1),
     (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, -6, 8, "counters", 108),  # the bench arm: K = 8, launch-ahead 6 unplaced
+    (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, -6, 8, "counters", 208),  # ... with the cap admitting in arrival order
     (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 6, 4, "counters", 108),
     (L.POLICY_SRPT_DEFICIT, 16, 32, 65536, 3, 4, "counters", 108),
     (L.POLICY_FIFO, 16, 32, 65536, 3, 4, "counters", 104),           # FIFO arm, K = 4
@@ -167,12 +168,13 @@ def test_serving_parity_and_replay(tmp_path, policy, group, streams, ring, look,
     names = ["toy", "resnet18", "mobilenet_v2", "squeezenet1_1"]
     online, prio = prio < 0, abs(prio)
     unpl, look = look < 0, abs(look)          # look < 0: launch-ahead without the placement test
-    K = prio - 100 if prio > 100 else 0       # 1xx: job cap K = xx (B200-Q6), one priority class
+    cap_fifo = prio > 200                     # 2xx: job cap K = xx admitting in arrival order
+    K = prio % 100 if prio > 100 else 0       # 1xx: job cap K = xx (B200-Q6), one priority class
     prio = 1 if K else prio
     with L.Engine(num_clients=3, policy=policy, group=group, streams=streams, ring_capacity=ring,
                   event_log=log, max_jobs_per_model=32, lookahead=look, launch_threads=lt, notify=notify,
                   prio_classes=prio, slack=(3552 if K else 1184) if (prio > 1 or K) else 0, online_tbar=online,
-                  max_active=K, lookahead_unplaced=unpl) as e:
+                  max_active=K, lookahead_unplaced=unpl, cap_fifo=cap_fifo) as e:
         specs = []
         for nm in names:
             g = archs.build(nm)

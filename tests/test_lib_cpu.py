@@ -264,21 +264,23 @@ def test_route_pair_matches_oracle():
     (L.POLICY_SRPT_DEFICIT, 100, 2, 0), (L.POLICY_SRPT_DEFICIT, None, 3, 2), (L.POLICY_SRPT_DEFICIT, 0, 1, 1),
     (L.POLICY_FIFO, 100, 2, 3), (L.POLICY_SJF, 100, 4, 1), (L.POLICY_RR, 100, 2, 0),
     (L.POLICY_SRPT_DEFICIT, 100, 3, 6), (L.POLICY_SRPT_DEFICIT, 100, 3, -6), (L.POLICY_FIFO, 100, 2, -2),
-    (L.POLICY_SRPT_DEFICIT, None, 0, -3)])
+    (L.POLICY_SRPT_DEFICIT, None, 0, -3), (L.POLICY_SRPT_DEFICIT, 100, 103, -6), (L.POLICY_SRPT_DEFICIT, None, 101, 0)])
 def test_fake_replay_max_active(tmp_path, policy, theta, K, look):
     """B200-Q6 (max_active = K): the C++ dispatcher's decisions with the job cap replay
     bit-exactly through the oracle policy; at most K capped jobs (plus deficit
     overrides) ever have kernels in flight.  look < 0: launch-ahead |look| without the
-    placement test (lookahead_unplaced, the bench arms' NEXT-1 variant)."""
+    placement test (lookahead_unplaced, the bench arms' NEXT-1 variant); K > 100: cap
+    K - 100 admitting in arrival order (cap_fifo)."""
     log = str(tmp_path / "ev_%u.log")
     models = [archs.toy(), archs.squeezenet1_1()]
     unpl, look = look < 0, abs(look)
+    cap_fifo, K = K > 100, K - 100 if K > 100 else K
     with _toy_engine(num_clients=3, policy=policy, theta=theta, streams=8, event_log=log, ring_capacity=1024,
-                     slack=8, lookahead=look, max_active=K, lookahead_unplaced=unpl) as e:
+                     slack=8, lookahead=look, max_active=K, lookahead_unplaced=unpl, cap_fifo=cap_fifo) as e:
         mids = [e.register_model(g, rng.model_params(g)) for g in models]
         _serve(e, mids, 200, 3, seed=K * 3 + policy)
     cfg, ms, events, ex = eventlog.read(log % 0)
-    assert cfg.max_active == K and cfg.lookahead_unplaced == int(unpl)
+    assert cfg.max_active == K and cfg.lookahead_unplaced == int(unpl) and cfg.cap_fifo == int(cap_fifo)
     assert sim.check_inflight_bound(events, ms, look) == []
     ok, msg, n = sim.replay(cfg, ms, events)
     assert ok, msg

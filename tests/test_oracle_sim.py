@@ -689,6 +689,27 @@ def test_max_active_fifo_order_and_override():
     assert pol2.over
 
 
+def test_cap_arrival_order_worked_example():
+    """K = 1, SRPT, theta = inf, no launch-ahead; A (2 kernels x 15 ns, R = 30) arrives
+    before B (1 kernel, 10 ns).  Cap in SRPT order: B is the cap's job, issues, leaves the
+    set (nothing left), then A issues its first kernel: [B, A.0]; after A.0 completes:
+    [A.1].  Cap in arrival order (cap_fifo): A holds the cap until it has issued its LAST
+    kernel: [A.0]; after A.0 completes: [A.1, B]."""
+    big = (10**6, 10**9, 10**12, 10**12, 10**9)
+    m = [[Layer(1, (1, 1, 1, 1, 0), 15, 15)] * 2, [Layer(1, (1, 1, 1, 1, 0), 10, 10)]]
+    for cf, want1, want2 in ((0, [(1, 0), (0, 0)], [(0, 1)]), (1, [(0, 0)], [(0, 1), (1, 0)])):
+        pol = sim.Policy(Config(num_clients=1, theta=sim.INF_THETA, slack=10**6, streams=8, max_active=1,
+                                cap_fifo=cf, capacity=big), m)
+        pol.arrival(0, 0, 0)
+        pol.arrival(1, 0, 1)
+        iss = pol.decide()
+        assert [(j, l) for (_, j, l, _) in iss] == want1, cf
+        ua = next(u for (u, j, l, _) in iss if j == 0)
+        pol.record(sim.PLACEMENT, ua, 1)
+        pol.record(sim.COMPLETION, ua, 1)
+        assert [(j, l) for (_, j, l, _) in pol.decide()] == want2, cf
+
+
 # --- S5 (b) exactly-once checker on bad logs ------------------------------------------
 
 def test_exactly_once_checker_rejects_bad_logs():
