@@ -79,6 +79,8 @@ def parse():
     ap.add_argument("--no-baselines", action="store_true", help="only the paella arm")
     ap.add_argument("--max-active", type=int, default=8, help="job cap K of the paella arms (B200-Q6); 0 = none")
     ap.add_argument("--lookahead", type=int, default=6, help="NEXT-1 launch-ahead depth of the paella arms")
+    ap.add_argument("--cap-fifo", action="store_true",
+                    help="the job cap admits in arrival order (cap_arrival_order, DESIGN.md B200-Q6)")
     ap.add_argument("--lookahead-placed", action="store_true",
                     help="launch-ahead waits for the oldest in-flight kernel's placement (the round-2 rule); "
                          "default: lookahead_unplaced (profiles/r2/diag/un_*)")
@@ -422,6 +424,7 @@ def run_gpu(args, ngpus, cores, fake):
     paella_kw = dict(policy=pol[args.policy], theta=args.theta, decide_delay_ns=args.decide_delay_ns,
                      online_tbar=args.online_tbar, slack=args.slack, prio_classes=args.prio_classes,
                      lookahead=args.lookahead, lookahead_unplaced=not args.lookahead_placed,
+                     cap_fifo=args.cap_fifo,
                      max_active=args.max_active, instrument=True,
                      route=L.ROUTE_LEAST_WORK, branches=bool(args.branches))
     arms_kw = {
@@ -794,7 +797,8 @@ def main():
                    "requests_per_step": args.reqs * ngpus,
                    "parallelism": f"{ngpus} GPU dispatchers, least-work router" if ngpus > 1 else "1 GPU dispatcher",
                    "paella": (f"srpt+deficit th{args.theta}" if args.policy == "srpt" else args.policy)
-                   + f" K{args.max_active} la{args.lookahead}{'' if args.lookahead_placed else 'u'} B{args.slack} pdl"
+                   + f" K{args.max_active}{'a' if args.cap_fifo else ''} la{args.lookahead}{'' if args.lookahead_placed else 'u'}"
+                   + f" B{args.slack} pdl"
                    + (" branches" if args.branches else ""),
                    "l2": "not flushed: weights (~120 MB bf16) largely L2-resident as in serving; inputs stream "
                          "from pinned host memory every request"},
