@@ -235,7 +235,9 @@ struct FakeBackend : Backend {
 // CUDA backend
 // ---------------------------------------------------------------------------
 // one launch of kernel k: split-K tcgen05 convs are thread-block clusters
-static bool is_tc(uint32_t kind) { return kind == KIND_CONV_TC || kind == KIND_CONV_TC_PRO || kind == KIND_CONV_TC128; }
+static bool is_tc(uint32_t kind) {
+  return kind == KIND_CONV_TC || kind == KIND_CONV_TC_PRO || kind == KIND_CONV_TC128 || kind == KIND_CONV_TC_M64;
+}
 static uint32_t tc_bn(uint32_t kind) { return kind == KIND_CONV_TC128 ? TC_BN_WIDE : TC_BN; }
 
 // pdl: programmatic dependent launch (programmatic stream serialization).  Measured on
@@ -383,7 +385,7 @@ struct CudaBackend : Backend {
       if (nstreams) std::rotate(streams.begin(), streams.begin() + (atoi(rot) % nstreams), streams.end());
     cudaMemsetAsync(tail, 0, 256, streams[0]);
     cudaMemsetAsync(ctr, 0, 2 * NCTR * sizeof(uint32_t), streams[0]);
-    KernelFn tc_i[3], tc_p[3];
+    KernelFn tc_i[4], tc_p[4];
     simt_kernel_table(tab[0][1], tab[0][0], tab[1][1], tab[1][0]);
     tc_kernel_table(tc_i, tc_p);
     tab[0][1][KIND_CONV_TC] = tc_i[0];
@@ -392,7 +394,11 @@ struct CudaBackend : Backend {
     tab[0][0][KIND_CONV_TC_PRO] = tc_p[1];
     tab[0][1][KIND_CONV_TC128] = tc_i[2];
     tab[0][0][KIND_CONV_TC128] = tc_p[2];
-    for (int i = 0; i < 2; ++i) tab[1][i][KIND_CONV_TC] = tab[1][i][KIND_CONV_TC_PRO] = tab[1][i][KIND_CONV_TC128] = nullptr;
+    tab[0][1][KIND_CONV_TC_M64] = tc_i[3];
+    tab[0][0][KIND_CONV_TC_M64] = tc_p[3];
+    for (int i = 0; i < 2; ++i)
+      tab[1][i][KIND_CONV_TC] = tab[1][i][KIND_CONV_TC_PRO] = tab[1][i][KIND_CONV_TC128] = tab[1][i][KIND_CONV_TC_M64] =
+          nullptr;
     if (proxy || mirror) {
       int rc = setup_proxy(streams[0]);
       if (rc) return rc;
@@ -1682,7 +1688,7 @@ int paella_kernel_info(paella_t* p, uint32_t model_id, uint32_t k, paella_kernel
 const char* paella_kernel_name(uint32_t kind) {
   static const char* names[] = {"ingest", "conv_simt", "conv_tcgen05", "dwconv", "maxpool",
                                 "avgpool", "gap", "fc_gemv", "empty", "conv_tcgen05_pro", "gap_fc", "spin",
-                                "conv_tcgen05_n128"};
+                                "conv_tcgen05_n128", "conv_tcgen05_m64"};
   return kind < KIND_COUNT ? names[kind] : "?";
 }
 

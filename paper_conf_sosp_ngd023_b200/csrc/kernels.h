@@ -18,7 +18,8 @@ enum KernelKind : uint32_t {
   KIND_GAPFC = 10,      // fused global average pool + FC classifier head
   KIND_SPIN = 11,       // synthetic HoL-microbenchmark kernel (Fig. 2): one resident block
   KIND_CONV_TC128 = 12, // tcgen05 conv with 128-pixel tiles (saturating shapes, no split-K)
-  KIND_COUNT = 13,
+  KIND_CONV_TC_M64 = 13,  // tcgen05 conv with UMMA M = 64 (layers with <= 64 output channels)
+  KIND_COUNT = 14,
 };
 
 typedef void (*KernelFn)();

@@ -173,19 +173,19 @@ __device__ __forceinline__ uint4 load_res8(const LayerArgs& a, uint32_t p, uint3
 // activation and residual fixed at compile time so the unrolled items carry no
 // branches and interleave (a single warp per SM sub-partition runs this: its speed
 // is instruction latency, not bandwidth); one output pointer advanced by 8 pixels.
-template <uint32_t ACT, bool RES, uint32_t NIT>
+template <uint32_t ACT, bool RES, uint32_t NIT, uint32_t BM>
 __device__ __forceinline__ void epi_tile(const LayerArgs& a, const float* stage, uint32_t n0, uint32_t P,
                                          uint32_t g, uint32_t co, const float (&bias)[8],
                                          const uint4 (&res)[NIT]) {
-  const uint32_t px0 = threadIdx.x / (TC_BM / 8);
+  const uint32_t px0 = threadIdx.x / (BM / 8);
   __nv_bfloat16* out = static_cast<__nv_bfloat16*>(a.out) + (size_t)(n0 + px0) * a.out_cs + a.out_co + co;
-  const size_t ostep = (size_t)(NPROD / (TC_BM / 8)) * a.out_cs;
+  const size_t ostep = (size_t)(NPROD / (BM / 8)) * a.out_cs;
   // all items are computed (the staged tile has 64 pixel rows), only the stores are
   // predicated: no branches around the item bodies, so the compiler interleaves them
 #pragma unroll
   for (uint32_t i = 0; i < NIT; ++i) {
-    const uint32_t px = px0 + i * (NPROD / (TC_BM / 8));
-    const float4* q = reinterpret_cast<const float4*>(stage + px * TC_BM + g * 8);
+    const uint32_t px = px0 + i * (NPROD / (BM / 8));
+    const float4* q = reinterpret_cast<const float4*>(stage + px * BM + g * 8);
     const float4 u0 = q[0], u1 = q[1];
     float x[8] = {u0.x + bias[0], u0.y + bias[1], u0.z + bias[2], u0.w + bias[3],
                   u1.x + bias[4], u1.y + bias[5], u1.z + bias[6], u1.w + bias[7]};
@@ -216,7 +216,7 @@ __device__ __forceinline__ void epi_tile(const LayerArgs& a, const float* stage,
 // only the block bookkeeping (instrumentation), so no compute warp waits on its
 // atomics at entry.
 constexpr uint32_t TBOOK = NPROD + 32;   // warp 5, lane 0
-template <bool INSTR, bool PRO, uint32_t BN>
+template <bool INSTR, bool PRO, uint32_t BN, uint32_t BM = TC_BM>
 __global__ void __launch_bounds__(TC_THREADS, 2)
     k_conv_tc(const __grid_constant__ LayerArgs a, const __grid_constant__ InstrArgs ia,
               const __grid_constant__ CUtensorMap wmap) {
@@ -233,12 +233,13 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   uint8_t* smem = smem_raw + ((1024u - (su32(smem_raw) & 1023u)) & 1023u);
   uint8_t* sA = smem;                                  // STAGES x 16 KiB
   constexpr uint32_t BNB = BN * TC_BK * 2;                      // B stage bytes: 8 / 16 KiB
-  constexpr uint32_t NST = TC_RING / (A_BYTES + BNB);           // 4 stages (BN 64) / 3 (BN 128)
+  constexpr uint32_t ABY = BM * TC_BK * 2;                      // A stage bytes: 16 / 8 KiB (M 128 / 64)
+  constexpr uint32_t NST = TC_RING / (ABY + BNB);           // 4 stages (BN 64) / 3 (BN 128) / 6 (M 64)
   constexpr uint32_t RPT = BN / 16;                             // B pixel rows per gather thread
-  uint8_t* sB = smem + NST * A_BYTES;
+  uint8_t* sB = smem + NST * ABY;
   uint64_t* full = (uint64_t*)(smem + TC_RING);
-  uint64_t* empty = full + TC_STAGES;
-  uint64_t* accb = empty + TC_STAGES;
+  uint64_t* empty = full + 8;
+  uint64_t* accb = empty + 8;
   uint64_t* rbar = accb + 1;                           // split-K: peers' slices landed
   uint32_t* tmem_slot = (uint32_t*)(rbar + 1);
   float* stage = reinterpret_cast<float*>(smem);       // epilogue tile [64 px][128 ch] fp32 (reuses sA)
@@ -246,7 +247,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   const uint32_t warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const uint32_t tile_n = blockIdx.x, tile_m = blockIdx.y, split = blockIdx.z;
   const uint32_t P = a.oh * a.ow;
-  const uint32_t n0 = tile_n * BN, m0 = tile_m * TC_BM;
+  const uint32_t n0 = tile_n * BN, m0 = tile_m * BM;
   const uint32_t nk = a.kpad / TC_BK;
   const uint32_t per = (nk + a.ksplit - 1) / a.ksplit;
   const uint32_t kb0 = split * per;
@@ -270,15 +271,15 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     if (trace) tr[11] = globaltimer();
     for (uint32_t it = 0; it < pre; ++it) {   // the first stages need no empty-wait
       mbar_arrive_tx(&full[it], abytes);
-      tma_load_2d(sA + it * A_BYTES, &wmap, &full[it], (int)((kb0 + it) * TC_BK), (int)m0);
+      tma_load_2d(sA + it * ABY, &wmap, &full[it], (int)((kb0 + it) * TC_BK), (int)m0);
     }
     if (trace) tr[12] = globaltimer();
   }
   // epilogue operands that do not depend on the accumulator: the bias (a weight) is
   // fetched before the PDL wait, the residual right after it, both hidden behind the
   // main loop.  Thread t owns channel group eg = t % 16 and pixels t / 16 + 8 i.
-  const uint32_t eg = threadIdx.x % (TC_BM / 8), eco = m0 + eg * 8;
-  constexpr uint32_t NIT = BN * (TC_BM / 8) / NPROD;   // 8 items per thread (BN 64)
+  const uint32_t eg = threadIdx.x % (BM / 8), eco = m0 + eg * 8;
+  constexpr uint32_t NIT = BN * (BM / 8) / NPROD;   // 8 items per thread (BN 64)
   float ebias[8];
   uint4 eres[NIT];
   if (warp < 4 && a.ksplit == 1) load_bias8(a, eco, ebias);
@@ -397,11 +398,11 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       kr = rs / (int)a.kw;
       tr_k = kcur, tr_ci = kci, tr_s = ks_, tr_r = kr;
     }
-    if (a.a_rows < TC_BM) {
-      const uint32_t zb = A_BYTES - abytes;   // bytes per stage, multiple of 1024
+    if (a.a_rows < BM) {
+      const uint32_t zb = ABY - abytes;   // bytes per stage, multiple of 1024
       for (uint32_t o = t * 16; o < NST * zb; o += NPROD * 16) {
         const uint32_t st = o / zb;
-        asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(su32(sA + st * A_BYTES + abytes + (o - st * zb))),
+        asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(su32(sA + st * ABY + abytes + (o - st * zb))),
                      "r"(0u)
                      : "memory");
       }
@@ -417,7 +418,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     if (a.ksplit == 1 && (a.flags & LF_RESIDUAL) && eco < a.cout) {
 #pragma unroll
       for (uint32_t i = 0; i < NIT; ++i) {
-        const uint32_t p = n0 + t / (TC_BM / 8) + i * (NPROD / (TC_BM / 8));
+        const uint32_t p = n0 + t / (BM / 8) + i * (NPROD / (BM / 8));
         if (p < P) eres[i] = load_res8(a, p, eco);
       }
     }
@@ -436,7 +437,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
         mbar_wait(&empty[s], ((nxt / NST) & 1) ^ 1);   // MMA of stage nxt - NST retired
         if (t == 0) {
           mbar_arrive_tx(&full[s], abytes);
-          tma_load_2d(sA + s * A_BYTES, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
+          tma_load_2d(sA + s * ABY, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
         }
         issue_B(nxt, true);
       }
@@ -460,7 +461,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
           mbar_wait(&empty[s], ((nxt / NST) & 1) ^ 1);
           if (t == 0) {
             mbar_arrive_tx(&full[s], abytes);
-            tma_load_2d(sA + s * A_BYTES, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
+            tma_load_2d(sA + s * ABY, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
           }
           issue_B(nxt, false);
           cp_async_commit();
@@ -478,14 +479,14 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     tc_fence_after();
     const uint32_t tmem = *tmem_slot;
     if (lane == 0) {
-      constexpr uint32_t IDESC = idesc_bf16(TC_BM, BN);
+      constexpr uint32_t IDESC = idesc_bf16(BM, BN);
       for (uint32_t it = 0; it < nkl; ++it) {
         const uint32_t s = it % NST;
         mbar_wait(&full[s], (it / NST) & 1);
         if (trace && it == 0) tr[2] = globaltimer();
         fence_proxy_async();   // the gathered B tile was written through the generic proxy
         tc_fence_after();
-        const uint32_t abase = su32(sA + s * A_BYTES), bbase = su32(sB + s * BNB);
+        const uint32_t abase = su32(sA + s * ABY), bbase = su32(sB + s * BNB);
 #pragma unroll
         for (uint32_t kk = 0; kk < TC_BK / 16; ++kk) {
           umma_bf16(tmem, sdesc_sw128(abase + kk * 32), sdesc_sw128(bbase + kk * 32), IDESC,
@@ -516,7 +517,11 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(ctr_of_block(ia) + 1) : "memory");
   }
   if (warp < 4) {
-    const uint32_t row = warp * 32 + lane;
+    // M = 128: accumulator row r in TMEM lane r (warp w reads lanes 32w..32w+31).  M = 64:
+    // rows 16w..16w+15 in lanes 32w..32w+15 of each sub-partition (CUTLASS tmem_frg_1sm,
+    // M_MMA = 64); the other half of the warp's lanes holds no row
+    const uint32_t row = BM == 128 ? warp * 32 + lane : warp * 16 + (lane & 15);
+    const bool owns = BM == 128 || lane < 16;
     if (nkl > 0) {
       mbar_wait(accb, 0);
       if (trace && threadIdx.x == 0) tr[4] = globaltimer();
@@ -527,12 +532,14 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
         float v[16];
         tmem_ld16(taddr + c * 16, v);
 #pragma unroll
-        for (int i = 0; i < 16; ++i) stage[(c * 16 + i) * TC_BM + row] = v[i];
+        for (int i = 0; i < 16; ++i)
+          if (owns) stage[(c * 16 + i) * BM + row] = v[i];
       }
       if (trace && threadIdx.x == 0) tr[8] = globaltimer();
     } else {
 #pragma unroll 8
-      for (uint32_t j = 0; j < BN; ++j) stage[j * TC_BM + row] = 0.f;
+      for (uint32_t j = 0; j < BN; ++j)
+        if (owns) stage[j * BM + row] = 0.f;
     }
   }
   if (a.ksplit == 1) {
@@ -545,14 +552,14 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       if (co < a.cout) {
         const bool rf = (a.flags & LF_RESIDUAL) != 0;
         if (a.act == 1) {
-          if (rf) epi_tile<1, true>(a, stage, n0, P, g, co, ebias, eres);
-          else epi_tile<1, false>(a, stage, n0, P, g, co, ebias, eres);
+          if (rf) epi_tile<1, true, NIT, BM>(a, stage, n0, P, g, co, ebias, eres);
+          else epi_tile<1, false, NIT, BM>(a, stage, n0, P, g, co, ebias, eres);
         } else if (a.act == 2) {
-          if (rf) epi_tile<2, true>(a, stage, n0, P, g, co, ebias, eres);
-          else epi_tile<2, false>(a, stage, n0, P, g, co, ebias, eres);
+          if (rf) epi_tile<2, true, NIT, BM>(a, stage, n0, P, g, co, ebias, eres);
+          else epi_tile<2, false, NIT, BM>(a, stage, n0, P, g, co, ebias, eres);
         } else {
-          if (rf) epi_tile<0, true>(a, stage, n0, P, g, co, ebias, eres);
-          else epi_tile<0, false>(a, stage, n0, P, g, co, ebias, eres);
+          if (rf) epi_tile<0, true, NIT, BM>(a, stage, n0, P, g, co, ebias, eres);
+          else epi_tile<0, false, NIT, BM>(a, stage, n0, P, g, co, ebias, eres);
         }
       }
     }
@@ -566,14 +573,14 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     // (the workspace is all zero between launches) and runs the epilogue for them.  The
     // fp32 additions happen in L2 in arrival order (one bf16 rounding afterwards).
     // Items of thread t: pixel rows px0 + (t + 128 i) / 16 (i < 4), channel group t % 16.
-    constexpr uint32_t MAXI = BN * (TC_BM / 8) / (2 * NPROD);   // 4 items at ksplit 2 (BN 64)
+    constexpr uint32_t MAXI = BN * (BM / 8) / (2 * NPROD);   // 4 items at ksplit 2 (BN 64)
     const uint32_t ks = a.ksplit;
     const uint32_t rows = BN / ks;
     const uint32_t px0 = split * rows;
-    const uint32_t g = threadIdx.x % (TC_BM / 8), co = m0 + g * 8;
-    const uint32_t nitems = rows * (TC_BM / 8);
+    const uint32_t g = threadIdx.x % (BM / 8), co = m0 + g * 8;
+    const uint32_t nitems = rows * (BM / 8);
     const uint32_t rv = n0 >= P ? 0u : min(BN, P - n0);   // pixel rows of the tile that exist
-    float* wt = a.ws + (size_t)(tile_m * gridDim.x + tile_n) * (BN * TC_BM);
+    float* wt = a.ws + (size_t)(tile_m * gridDim.x + tile_n) * (BN * BM);
     float bias[8];
     uint4 rres[MAXI];
     if (warp < 4 && co < a.cout) {
@@ -582,7 +589,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
 #pragma unroll
         for (uint32_t i = 0; i < MAXI; ++i) {
           const uint32_t item = threadIdx.x + i * NPROD;
-          const uint32_t p = n0 + px0 + item / (TC_BM / 8);
+          const uint32_t p = n0 + px0 + item / (BM / 8);
           if (item < nitems && p < P) rres[i] = load_res8(a, p, co);
         }
       }
@@ -597,12 +604,12 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
         const uint32_t sb = su32(stage);
         if (rv > r0)
           asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.add.f32 [%0], [%1], %2;" ::"l"(
-                           wt + r0 * TC_BM),
-                       "r"(sb + r0 * TC_BM * 4), "r"((rv - r0) * TC_BM * 4)
+                           wt + r0 * BM),
+                       "r"(sb + r0 * BM * 4), "r"((rv - r0) * BM * 4)
                        : "memory");
         if (r0 > 0)
           asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.add.f32 [%0], [%1], %2;" ::"l"(wt),
-                       "r"(sb), "r"(r0 * TC_BM * 4)
+                       "r"(sb), "r"(r0 * BM * 4)
                        : "memory");
         asm volatile("cp.async.bulk.commit_group;" ::: "memory");
         asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // the adds are performed
@@ -624,9 +631,9 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
 #pragma unroll
       for (uint32_t i = 0; i < MAXI; ++i) {
         const uint32_t item = threadIdx.x + i * NPROD;
-        const uint32_t r = item / (TC_BM / 8), p = n0 + px0 + r;
+        const uint32_t r = item / (BM / 8), p = n0 + px0 + r;
         if (item < nitems && p < P) {
-          float* q = wt + (px0 + r) * TC_BM + g * 8;
+          float* q = wt + (px0 + r) * BM + g * 8;
           float v[8];
           asm volatile("ld.relaxed.gpu.global.L1::no_allocate.v4.f32 {%0, %1, %2, %3}, [%4];"
                        : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3])
@@ -652,14 +659,14 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     // epilogue for it -- no global workspace, no atomics, no per-element remote loads
     // (those were bound at ~17 GB/s per SM: 1.7 us for ksplit 8).
     // Items of thread t: pixel rows px0 + (t + 128 i) / 16 (i < 4), channel group t % 16.
-    constexpr uint32_t MAXI = BN * (TC_BM / 8) / (2 * NPROD);   // 4 items at ksplit 2 (BN 64)
+    constexpr uint32_t MAXI = BN * (BM / 8) / (2 * NPROD);   // 4 items at ksplit 2 (BN 64)
     const uint32_t ks = a.ksplit;
     const uint32_t rows = BN / ks;
     const uint32_t px0 = split * rows;
-    const uint32_t g = threadIdx.x % (TC_BM / 8), co = m0 + g * 8;
-    const uint32_t nitems = rows * (TC_BM / 8);
-    const uint32_t slice = rows * TC_BM * 4;                // bytes of one slice (slot pitch)
-    float* recv = stage + BN * TC_BM;                       // ks - 1 received slices (free A stages)
+    const uint32_t g = threadIdx.x % (BM / 8), co = m0 + g * 8;
+    const uint32_t nitems = rows * (BM / 8);
+    const uint32_t slice = rows * BM * 4;                // bytes of one slice (slot pitch)
+    float* recv = stage + BN * BM;                       // ks - 1 received slices (free A stages)
     // only the slice rows that hold real pixels travel (the tile tail past P does not)
     auto valid_rows = [&](uint32_t owner) -> uint32_t {
       const uint32_t r0 = n0 + owner * rows;
@@ -673,12 +680,12 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
 #pragma unroll
         for (uint32_t i = 0; i < MAXI; ++i) {
           const uint32_t item = threadIdx.x + i * NPROD;
-          const uint32_t p = n0 + px0 + item / (TC_BM / 8);
+          const uint32_t p = n0 + px0 + item / (BM / 8);
           if (item < nitems && p < P) rres[i] = load_res8(a, p, co);
         }
       }
     }
-    if (threadIdx.x == 0) mbar_arrive_tx(rbar, (ks - 1) * valid_rows(split) * TC_BM * 4);   // before any push
+    if (threadIdx.x == 0) mbar_arrive_tx(rbar, (ks - 1) * valid_rows(split) * BM * 4);   // before any push
     if (warp < 4) fence_proxy_async();   // the staged tile (generic writes) is read by the bulk copies
     __syncwarp();
     if (trace && threadIdx.x == 0) tr[9] = globaltimer();
@@ -693,7 +700,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       // the sender's distance behind it
       for (uint32_t j = 1; j < ks; ++j) {
         const uint32_t owner = (split + j) & (ks - 1);
-        const uint32_t bytes = valid_rows(owner) * TC_BM * 4;
+        const uint32_t bytes = valid_rows(owner) * BM * 4;
         if (bytes == 0) continue;
         const uint32_t slot = (split + ks - owner - 1) & (ks - 1);
         uint32_t dst, bar;
@@ -711,12 +718,12 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
 #pragma unroll
       for (uint32_t i = 0; i < MAXI; ++i) {
         const uint32_t item = threadIdx.x + i * NPROD;
-        const uint32_t r = item / (TC_BM / 8), p = n0 + px0 + r;
+        const uint32_t r = item / (BM / 8), p = n0 + px0 + r;
         if (item < nitems && p < P) {
-          const float4* own = reinterpret_cast<const float4*>(stage + (px0 + r) * TC_BM + g * 8);
+          const float4* own = reinterpret_cast<const float4*>(stage + (px0 + r) * BM + g * 8);
           float4 x0 = own[0], x1 = own[1];
           for (uint32_t q = 0; q + 1 < ks; ++q) {
-            const float4* o = reinterpret_cast<const float4*>(recv + (q * rows + r) * TC_BM + g * 8);
+            const float4* o = reinterpret_cast<const float4*>(recv + (q * rows + r) * BM + g * 8);
             const float4 y0 = o[0], y1 = o[1];
             x0.x += y0.x; x0.y += y0.y; x0.z += y0.z; x0.w += y0.w;
             x1.x += y1.x; x1.y += y1.y; x1.z += y1.z; x1.w += y1.w;
@@ -745,7 +752,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   }
 }
 
-uint32_t tc_smem_bytes() { return 1024 + TC_RING + 128; }   // align pad + stage ring + barriers
+uint32_t tc_smem_bytes() { return 1024 + TC_RING + 256; }   // align pad + stage ring + barriers
 static_assert(TC_RING == TC_STAGES * (A_BYTES + B_BYTES), "ring");
 
 void tc_kernel_table(KernelFn* instr, KernelFn* plain) {
@@ -755,6 +762,8 @@ void tc_kernel_table(KernelFn* instr, KernelFn* plain) {
   plain[1] = (KernelFn)k_conv_tc<false, true, TC_BN>;
   instr[2] = (KernelFn)k_conv_tc<true, false, TC_BN_WIDE>;   // 128-pixel tiles
   plain[2] = (KernelFn)k_conv_tc<false, false, TC_BN_WIDE>;
+  instr[3] = (KernelFn)k_conv_tc<true, false, TC_BN, 64>;    // narrow layers: UMMA M = 64
+  plain[3] = (KernelFn)k_conv_tc<false, false, TC_BN, 64>;
 }
 
 // Host: tensor map for the packed weights [rows][kpad] bf16, box 64 x box_rows

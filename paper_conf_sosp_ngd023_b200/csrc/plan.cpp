@@ -299,6 +299,9 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
               a.tiles_n = (P_out + TC_BN_WIDE - 1) / TC_BN_WIDE;
               k.tmem_cols = TC_BN_WIDE;
             }
+            // narrow layers (<= 64 output channels, no prologue): UMMA M = 64, so the tensor
+            // core reads 64 weight rows per k-block instead of 128 (half of them zero)
+            if (k.kind == KIND_CONV_TC && a.a_rows <= 64 && !std::getenv("PAELLA_NO_M64")) k.kind = KIND_CONV_TC_M64;
             k.grid[0] = a.tiles_n;
             k.grid[1] = a.tiles_m;
             k.grid[2] = split;
