@@ -14,7 +14,8 @@ import os
 import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libpaella.so")
+# PAELLA_LIB: another build of the same library (the ThreadSanitizer build, build.py --tsan)
+LIB_PATH = os.environ.get("PAELLA_LIB") or os.path.join(HERE, "libpaella.so")
 
 ABI_VERSION = 2
 NOTIFY_COUNTERS, NOTIFY_RING = 0, 1

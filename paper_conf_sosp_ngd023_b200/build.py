@@ -6,6 +6,12 @@ Host C++ (runtime, dispatcher, planner, policy) is compiled with g++; kernels wi
 nvcc ``-gencode arch=compute_100a,code=sm_100a -lineinfo``; everything is linked by
 nvcc into one shared library with the static CUDA runtime.  Incremental: objects
 are rebuilt when their source or any header is newer.
+
+    python -m paper_conf_sosp_ngd023_b200.build --tsan
+
+builds ``libpaella_tsan.so`` (host objects with ``-fsanitize=thread``, own build
+directory) for the ThreadSanitizer run of the dispatcher (tools/sanitize.sh); load it
+with ``PAELLA_LIB=<path>`` and ``LD_PRELOAD=<libtsan.so>``.
 """
 from __future__ import annotations
 
@@ -42,32 +48,35 @@ def _run(cmd, verbose):
         sys.stderr.write(r.stdout + r.stderr)
 
 
-def build(verbose=False, ptxas_v=False):
-    os.makedirs(BUILD, exist_ok=True)
+def build(verbose=False, ptxas_v=False, tsan=False):
+    build_dir = BUILD + ("_tsan" if tsan else "")
+    out = os.path.join(HERE, "libpaella_tsan.so") if tsan else OUT
+    san = ["-fsanitize=thread"] if tsan else []
+    os.makedirs(build_dir, exist_ok=True)
     headers = glob.glob(os.path.join(CSRC, "*.h")) + glob.glob(os.path.join(CSRC, "*.cuh")) + \
         [os.path.join(ROOT, "include", "paella.h")]
     objs = []
     inc = ["-I", CSRC, "-I", os.path.join(ROOT, "include"), "-I", os.path.join(CUDA, "include")]
     for src in sorted(glob.glob(os.path.join(CSRC, "*.cpp"))):
-        obj = os.path.join(BUILD, os.path.basename(src) + ".o")
+        obj = os.path.join(build_dir, os.path.basename(src) + ".o")
         objs.append(obj)
         if _newer(src, obj, headers):
-            _run(["g++", "-O2", "-g", "-fPIC", "-std=c++17", "-Wall", "-Wno-unused-function",
+            _run(["g++", "-O2", "-g", "-fPIC", *san, "-std=c++17", "-Wall", "-Wno-unused-function",
                   "-Wno-sign-compare", *inc, "-c", src, "-o", obj], verbose)
     for src in sorted(glob.glob(os.path.join(CSRC, "*.cu"))):
-        obj = os.path.join(BUILD, os.path.basename(src) + ".o")
+        obj = os.path.join(build_dir, os.path.basename(src) + ".o")
         objs.append(obj)
         if _newer(src, obj, headers):
             extra = ["-Xptxas", "-v"] if ptxas_v else []
             _run([NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", *inc, *extra,
                   "-c", src, "-o", obj], verbose or ptxas_v)
-    if not os.path.exists(OUT) or any(os.path.getmtime(o) > os.path.getmtime(OUT) for o in objs):
-        tmp = OUT + ".tmp"
-        _run([NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lpthread", "-lrt", "-ldl"], verbose)
-        os.replace(tmp, OUT)
-    return OUT
+    if not os.path.exists(out) or any(os.path.getmtime(o) > os.path.getmtime(out) for o in objs):
+        tmp = out + ".tmp"
+        _run([NVCC, *ARCH, "-shared", "-o", tmp, *objs, *(["-Xcompiler", "-fsanitize=thread"] if tsan else []),
+              "-lpthread", "-lrt", "-ldl"], verbose)
+        os.replace(tmp, out)
+    return out
 
 
 if __name__ == "__main__":
-    build(verbose="-v" in sys.argv, ptxas_v="--ptxas" in sys.argv)
-    print(OUT)
+    print(build(verbose="-v" in sys.argv, ptxas_v="--ptxas" in sys.argv, tsan="--tsan" in sys.argv))

@@ -98,6 +98,7 @@ enum : uint32_t {
   LF_SPLIT_NOROT = 64u,   // (A/B) L2 split-K: every CTA reduces its rows in tile order
   LF_SPLIT_RELBAR = 128u, // (A/B) L2 split-K: release/acquire cluster barrier instead of a
                           // relaxed one after the reducing thread's own fence
+  LF_MBAR_SPIN = 256u,    // (A/B) conv k-block loop: mbarrier.test_wait spin instead of try_wait
 };
 
 struct LayerArgs {

@@ -904,6 +904,14 @@ static void decide_and_launch(Gpu* g) {
 // Models posted by paella_register_model: added to this GPU's policy and logged by the
 // dispatcher thread itself, between two loop iterations.
 static void apply_inbox(Gpu* g) {
+  if (g->st_req.load(std::memory_order_acquire) != g->st_ack.load(std::memory_order_relaxed)) {
+    const uint64_t req = g->st_req.load(std::memory_order_acquire);
+    {
+      std::lock_guard<std::mutex> lk(g->st_mu);
+      g->st_snap = g->stats;
+    }
+    g->st_ack.store(req, std::memory_order_release);
+  }
   if (g->clk_req.load(std::memory_order_acquire) != g->clk_applied.load(std::memory_order_relaxed)) {
     std::lock_guard<std::mutex> lk(g->inbox_mu);
     if (g->clk_pending) {
@@ -1124,6 +1132,7 @@ static void dispatcher_main(Gpu* g) {
     fail_gpu(g, -EIO, ex.what());
   }
   if (g->pub->err.load(std::memory_order_acquire)) dead_loop(g);
+  g->loop_done.store(true, std::memory_order_release);
 }
 
 // globaltimer -> host clock calibration: n ping-pongs with
@@ -1762,8 +1771,22 @@ int paella_clock_info(paella_t* p, uint32_t gpu, int64_t* offset_ns, int64_t* rt
 int paella_stats(paella_t* p, uint32_t gpu, paella_stats_t* st) {
   Paella* P = (Paella*)p;
   if (!P || !st || gpu >= P->gpus.size()) return -EINVAL;
-  *st = P->gpus[gpu]->stats;   // racy snapshot of counters, fine for reporting
-  st->outstanding_work_ns = P->gpus[gpu]->pub->work.load();
+  Gpu* g = P->gpus[gpu].get();
+  // ask the dispatcher thread for a snapshot (apply_inbox runs every 64 loop iterations)
+  // unless it has finished; a thread that was never started has written nothing
+  if (g->thread.joinable() && !g->loop_done.load(std::memory_order_acquire)) {
+    const uint64_t seen = g->st_ack.load(std::memory_order_acquire);
+    g->st_req.fetch_add(1, std::memory_order_release);
+    while (g->st_ack.load(std::memory_order_acquire) == seen && !g->loop_done.load(std::memory_order_acquire))
+      std::this_thread::yield();
+  }
+  if (g->loop_done.load(std::memory_order_acquire) || !g->thread.joinable()) {
+    *st = g->stats;
+  } else {
+    std::lock_guard<std::mutex> lk(g->st_mu);
+    *st = g->st_snap;
+  }
+  st->outstanding_work_ns = g->pub->work.load();
   return 0;
 }
 

@@ -226,7 +226,14 @@ struct Gpu {
   bool log_times = false;
   uint32_t naive_uid = 0;   // PAELLA_NAIVE_INSTR diagnosis: launch counter of the naive path   // PAELLA_TRACE_TIMES: host-time events (EV_TIME) for timelines
   std::mutex log_mu;
-  paella_stats_t stats{};
+  paella_stats_t stats{};   // written by the dispatcher thread only
+  // paella_stats: a caller bumps st_req; the dispatcher copies stats into st_snap (under
+  // st_mu) and publishes st_ack; after the thread's last write it sets loop_done, so a
+  // caller can read stats directly (release/acquire, no data race -- ThreadSanitizer run)
+  std::atomic<uint64_t> st_req{0}, st_ack{0};
+  std::atomic<bool> loop_done{false};
+  std::mutex st_mu;
+  paella_stats_t st_snap{};
   std::vector<Issue> issues;
   // isolated runs (profiling, parity tests): private ring, counters and stream
   Rec* prof_ring_h = nullptr;

@@ -60,6 +60,16 @@ __device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
       "r"(parity)
       : "memory");
 }
+// non-suspending poll (A/B against try_wait's potentially-suspending wait)
+__device__ __forceinline__ void mbar_wait_spin(uint64_t* b, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "SPIN_%=:\n\t"
+      "mbarrier.test_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra SPIN_%=;\n}" ::"r"(su32(b)),
+      "r"(parity)
+      : "memory");
+}
 __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, uint64_t* bar, int x, int y) {
   asm volatile(
       "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(
@@ -221,6 +231,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     k_conv_tc(const __grid_constant__ LayerArgs a, const __grid_constant__ InstrArgs ia,
               const __grid_constant__ CUtensorMap wmap) {
   const bool trace = (a.flags & LF_TRACE) != 0;
+  const bool spin = (a.flags & LF_MBAR_SPIN) != 0;
   uint64_t* tr = trace ? a.trace +
                              16 * ((blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x)
                        : nullptr;
@@ -434,7 +445,8 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
         asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(su32(&full[it])) : "memory");
       for (uint32_t nxt = NST; nxt < nkl; ++nxt) {
         const uint32_t s = nxt % NST;
-        mbar_wait(&empty[s], ((nxt / NST) & 1) ^ 1);   // MMA of stage nxt - NST retired
+        if (spin) mbar_wait_spin(&empty[s], ((nxt / NST) & 1) ^ 1);
+        else mbar_wait(&empty[s], ((nxt / NST) & 1) ^ 1);   // MMA of stage nxt - NST retired
         if (t == 0) {
           mbar_arrive_tx(&full[s], abytes);
           tma_load_2d(sA + s * ABY, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
@@ -482,7 +494,8 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       constexpr uint32_t IDESC = idesc_bf16(BM, BN);
       for (uint32_t it = 0; it < nkl; ++it) {
         const uint32_t s = it % NST;
-        mbar_wait(&full[s], (it / NST) & 1);
+        if (spin) mbar_wait_spin(&full[s], (it / NST) & 1);
+        else mbar_wait(&full[s], (it / NST) & 1);
         if (trace && it == 0) tr[2] = globaltimer();
         fence_proxy_async();   // the gathered B tile was written through the generic proxy
         tc_fence_after();

@@ -288,6 +288,7 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
             if (std::getenv("PAELLA_SPLIT_DSMEM")) a.flags |= LF_SPLIT_DSMEM;   // A/B: the DSMEM reduction
             if (std::getenv("PAELLA_SPLIT_NOROT")) a.flags |= LF_SPLIT_NOROT;
             if (std::getenv("PAELLA_SPLIT_RELBAR")) a.flags |= LF_SPLIT_RELBAR;
+            if (std::getenv("PAELLA_MBAR_SPIN")) a.flags |= LF_MBAR_SPIN;
             // narrow layers: fetch only the live weight rows (SW128 atoms are 8 rows)
             a.a_rows = nd.c < TC_BM ? (uint32_t)align_up(nd.c, 8) : TC_BM;
             k.tmem_cols = tc_tmem_cols();
