@@ -2073,6 +2073,9 @@ static int autotune_splits(Gpu* g, Model* m) {
     const uint32_t orig = k.proto.ksplit;
     // PAELLA_SPLIT_DSMEM forces the DSMEM reduction, PAELLA_SPLIT_L2 the L2 one
     const bool only_dsm = std::getenv("PAELLA_SPLIT_DSMEM") != nullptr, only_l2 = std::getenv("PAELLA_SPLIT_L2") != nullptr;
+    // a doubled split must beat the best so far by this factor (percent of its time):
+    // it doubles the CTAs (device work) of the layer, which serving under load pays for
+    static const int64_t gain = std::getenv("PAELLA_SPLIT_GAIN") ? atoi(std::getenv("PAELLA_SPLIT_GAIN")) : 95;
     uint32_t best = orig;
     bool best_dsm = (k.proto.flags & LF_SPLIT_DSMEM) != 0;
     int64_t best_t = INT64_MAX;
@@ -2091,7 +2094,7 @@ static int autotune_splits(Gpu* g, Model* m) {
         }
       }
       if (t_sp == INT64_MAX) continue;
-      if (best_t == INT64_MAX || t_sp * 100 < best_t * 95) {
+      if (best_t == INT64_MAX || t_sp * 100 < best_t * gain) {
         best_t = t_sp;
         best = sp;
         best_dsm = dsm_sp;

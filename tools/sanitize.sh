@@ -3,8 +3,7 @@
 #  tsan: the host runtime (dispatcher, launchers, router, channels, policy) built with
 #        -fsanitize=thread, driven by the CPU library tests on the fake device -- runs
 #        here, no GPU.  Reports go to $OUT/tsan.*; the run fails if any report exists.
-#  cuda: compute-sanitizer memcheck / racecheck / synccheck on the isolated parity tests
-#        and smoke (GPU box only).
+#  cuda: compute-sanitizer -- closed on this GPU pool (see below).
 set -u
 OUT=${OUT:-gpurun_out/sanitize}
 mkdir -p "$OUT"
@@ -20,14 +19,8 @@ if [ "$mode" = tsan ]; then
   echo "tsan reports: $n"
   [ "$n" = 0 ]
 else
-  for tool in memcheck racecheck synccheck; do
-    sel="isolated_bf16_parity and (toy or resnet18 or mobilenet_v2 or densenet121)"
-    [ $tool = memcheck ] && sel="isolated or wide_tile or forced_split_k"
-    timeout 1500 compute-sanitizer --tool $tool --error-exitcode 9 --print-limit 20 \
-      python -m pytest tests/test_gpu.py -x -q -k "$sel" -p no:cacheprovider \
-      > "$OUT/cs_$tool.log" 2>&1
-    echo "$tool tests rc=$?"; tail -3 "$OUT/cs_$tool.log"
-  done
-  timeout 900 compute-sanitizer --tool memcheck --error-exitcode 9 python -c "import __graft_entry__ as g; g.smoke()" \
-    > "$OUT/cs_smoke.log" 2>&1; echo "memcheck smoke rc=$?"; tail -3 "$OUT/cs_smoke.log"
+  # compute-sanitizer is closed on this GPU pool (gpurun answers rc 86: runs under it have
+  # left GPUs needing a reset); kernel memory safety is covered by the bounds asserts and
+  # the element-by-element parity tests instead (tests/test_gpu.py)
+  echo "compute-sanitizer unavailable on this pool"; exit 2
 fi
