@@ -302,7 +302,15 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
             }
             // narrow layers (<= 64 output channels, no prologue): UMMA M = 64, so the tensor
             // core reads 64 weight rows per k-block instead of 128 (half of them zero)
-            if (k.kind == KIND_CONV_TC && a.a_rows <= 64 && !std::getenv("PAELLA_NO_M64")) k.kind = KIND_CONV_TC_M64;
+            // Opt-in (PAELLA_M64): faster in isolation (DenseNet-121 -3.7 %) but the C-3 mix's
+            // device-only saturation rate drops ~5 % (profiles/r2/diag/split_gain)
+            if (k.kind == KIND_CONV_TC && a.a_rows <= 64 && std::getenv("PAELLA_M64")) k.kind = KIND_CONV_TC_M64;
+            // activations by TMA im2col: one 64-channel slice of one filter tap per k-block
+            // (cin % 64 == 0), 16-byte aligned pixel rows, no in-place prologue
+            if (k.kind != KIND_CONV_TC_PRO && a.cin % 64 == 0 && a.in_cs % 8 == 0 && a.in_co % 8 == 0 &&
+                a.sh <= 8 && a.sw <= 8 && a.ph < 128 && a.pw < 128 && a.kh <= 128 && a.kw <= 128 &&
+                !std::getenv("PAELLA_NO_TMA_B"))
+              a.flags |= LF_TMA_B;
             k.grid[0] = a.tiles_n;
             k.grid[1] = a.tiles_m;
             k.grid[2] = split;

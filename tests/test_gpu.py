@@ -64,6 +64,20 @@ def test_isolated_bf16_parity(engine, name):
         assert ok.all(), f"{name} input {i}: {np.sum(~ok)} logits out of tolerance, max err {np.abs(out-ref).max()}"
 
 
+@pytest.mark.parametrize("name", ["mobilenet_v2", "densenet121", "inception_v3"])
+def test_isolated_bf16_parity_m64(engine, name, monkeypatch):
+    """The opt-in UMMA M = 64 conv (PAELLA_M64, layers with <= 64 output channels),
+    planned at registration, against the same float64 oracle as the default kernels."""
+    monkeypatch.setenv("PAELLA_M64", "1")
+    g = archs.build(name)
+    mid = engine.register_model(g, rng.model_params(g), dtype=L.DTYPE_BF16, name=name + "-m64")
+    assert any(k["name"].startswith("conv_tcgen05") for k in engine.kernels(mid))
+    out = engine.run_isolated(mid, rng.image(g, 0))
+    ref = oracle_out(name, 0, "bf16")
+    ok = within(out, ref, BF16_TOL)
+    assert ok.all(), f"{name}: {np.sum(~ok)} logits out of tolerance, max err {np.abs(out-ref).max()}"
+
+
 @pytest.mark.parametrize("name", ["toy", "resnet18", "mobilenet_v2", "squeezenet1_1", "densenet121", "resnet50",
                                   "inception_v3"])
 def test_isolated_fp32_parity(engine, name):

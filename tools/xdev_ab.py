@@ -1,7 +1,7 @@
 """Diagnosis: the C-3 mix's device-only saturation rate (X_dev: CUDA graphs of the mix on
 32 streams, no dispatcher) next to its isolated latency (summed instrumented kernel
 times) and device work (summed CTAs), for the current environment's planner/autotuner
-switches (PAELLA_NO_M64, PAELLA_SPLIT_GAIN, ...).  One JSON line.  No oracle."""
+switches (PAELLA_M64, PAELLA_NO_TMA_B, PAELLA_SPLIT_GAIN, ...).  One JSON line.  No oracle."""
 import json
 import os
 os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
