@@ -99,6 +99,8 @@ enum : uint32_t {
   LF_SPLIT_RELBAR = 128u, // (A/B) L2 split-K: release/acquire cluster barrier instead of a
                           // relaxed one after the reducing thread's own fence
   LF_MBAR_SPIN = 256u,    // (A/B) conv k-block loop: mbarrier.test_wait spin instead of try_wait
+  LF_TMA_B = 512u,        // tcgen05 conv: B (activations) by TMA im2col (bmap) instead of the
+                          // LDGSTS gather (cin % 64 == 0, no prologue)
 };
 
 struct LayerArgs {
@@ -122,6 +124,7 @@ struct LayerArgs {
   uint32_t a_rows;          // tcgen05 conv: weight rows fetched per stage (TMA box), <= 128
   float* ws;                // split-K: fp32 partial sums, 64 x 128 per output tile, all zero between uses
   uint64_t* trace;          // debug (LF_TRACE): per-CTA phase timestamps
+  const void* bmap;         // LF_TMA_B: device address of this slot's im2col CUtensorMap (128 B)
 };
 
 }  // namespace paella

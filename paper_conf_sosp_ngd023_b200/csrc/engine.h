@@ -66,6 +66,7 @@ struct ModelGpu {
   std::vector<std::vector<LayerArgs>> args;   // [slot][kernel]
   std::vector<uint32_t> free_slots;
   std::vector<TmapStore> tmaps;   // per kernel (tcgen05 conv weights)
+  uint8_t* bmaps = nullptr;       // device: [slot][kernel] im2col tensor maps (LF_TMA_B), 128 B each
 };
 
 struct Model {

@@ -77,6 +77,16 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, u
       "l"(map), "r"(su32(bar)), "r"(x), "r"(y)
       : "memory");
 }
+// B tile by TMA im2col: BN output pixels from linear pixel (w, h) onwards (traversal in
+// W, H order with the map's conv strides), 64 channels from c of filter tap (s, r)
+__device__ __forceinline__ void tma_im2col_4d(void* dst, const void* map, uint64_t* bar, int c, int w, int h,
+                                              uint16_t s, uint16_t r) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.shared::cluster.global.im2col.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4, %5, %6}], [%2], {%7, %8};" ::"r"(su32(dst)),
+      "l"(map), "r"(su32(bar)), "r"(c), "r"(w), "r"(h), "r"(0), "h"(s), "h"(r)
+      : "memory");
+}
 __device__ __forceinline__ void cp_async16(uint32_t dst, const void* src, uint32_t src_bytes) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
 }
@@ -232,6 +242,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
               const __grid_constant__ CUtensorMap wmap) {
   const bool trace = (a.flags & LF_TRACE) != 0;
   const bool spin = (a.flags & LF_MBAR_SPIN) != 0;
+  const bool tmab = !PRO && (a.flags & LF_TMA_B) && a.bmap != nullptr;
   uint64_t* tr = trace ? a.trace +
                              16 * ((blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x)
                        : nullptr;
@@ -269,11 +280,19 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   // narrow layers (Cout < 128) fetch only a_rows weight rows per stage; rows a_rows..127
   // of every A stage are zeroed once below (the UMMA still runs M = 128)
   const uint32_t abytes = a.a_rows * 128;
+  // LF_TMA_B: k-block kb is filter tap (r, s) = divmod(kb * 64 / cin, kw), channels
+  // kb * 64 % cin onwards; the tile's first output pixel's window starts at (tw0, th0)
+  const int tw0 = (int)((n0 % a.ow) * a.sw) - (int)a.pw, th0 = (int)((n0 / a.ow) * a.sh) - (int)a.ph;
+  auto tma_B = [&](uint32_t it) {
+    const uint32_t k0 = (kb0 + it) * TC_BK, tap = k0 / a.cin, c0 = k0 - tap * a.cin;
+    const uint32_t r = tap / a.kw, sx = tap - r * a.kw;
+    tma_im2col_4d(sB + (it % NST) * BNB, a.bmap, &full[it % NST], (int)c0, tw0, th0, (uint16_t)sx, (uint16_t)r);
+  };
   if (warp == 4 && lane == 0) {
     // the MMA warp's leader sets up the barriers and starts the weight stream while
     // the gather warps compute their addresses
     for (uint32_t s = 0; s < NST; ++s) {
-      mbar_init(&full[s], NPROD + 1);
+      mbar_init(&full[s], tmab ? 1 : NPROD + 1);
       mbar_init(&empty[s], 1);
     }
     mbar_init(accb, 1);
@@ -281,8 +300,12 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     if (trace) tr[11] = globaltimer();
     for (uint32_t it = 0; it < pre; ++it) {   // the first stages need no empty-wait
-      mbar_arrive_tx(&full[it], abytes);
+      mbar_arrive_tx(&full[it], abytes + (tmab ? BNB : 0u));
       tma_load_2d(sA + it * ABY, &wmap, &full[it], (int)((kb0 + it) * TC_BK), (int)m0);
+    }
+    if (tmab) {   // the activations once the predecessor's output is complete (PDL)
+      pdl_wait();
+      for (uint32_t it = 0; it < pre; ++it) tma_B(it);
     }
     if (trace) tr[12] = globaltimer();
   }
@@ -422,10 +445,11 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
     // ... and the first activation gathers, before the CTA-wide barrier, once the
     // predecessor kernel's output is complete (PDL; the weight TMA above needs no wait)
     pdl_wait();
-    for (uint32_t it = 0; it < pre; ++it) {   // barriers not initialised yet
-      issue_B(it, false);
-      if constexpr (PRO) cp_async_commit();   // one group per stage
-    }
+    if (!tmab)
+      for (uint32_t it = 0; it < pre; ++it) {   // barriers not initialised yet
+        issue_B(it, false);
+        if constexpr (PRO) cp_async_commit();   // one group per stage
+      }
     if (a.ksplit == 1 && (a.flags & LF_RESIDUAL) && eco < a.cout) {
 #pragma unroll
       for (uint32_t i = 0; i < NIT; ++i) {
@@ -441,6 +465,17 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   if (warp < 4) {
     // ------------------------------------------------------------ producers
     if constexpr (!PRO) {
+      if (tmab) {
+        // one thread streams both operands by TMA (A + B bytes on one full barrier)
+        if (t == 0)
+          for (uint32_t nxt = NST; nxt < nkl; ++nxt) {
+            const uint32_t s = nxt % NST;
+            mbar_wait(&empty[s], ((nxt / NST) & 1) ^ 1);
+            mbar_arrive_tx(&full[s], abytes + BNB);
+            tma_load_2d(sA + s * ABY, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
+            tma_B(nxt);
+          }
+      } else {
       for (uint32_t it = 0; it < pre; ++it)
         asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(su32(&full[it])) : "memory");
       for (uint32_t nxt = NST; nxt < nkl; ++nxt) {
@@ -452,6 +487,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
           tma_load_2d(sA + s * ABY, &wmap, &full[s], (int)((kb0 + nxt) * TC_BK), (int)m0);
         }
         issue_B(nxt, true);
+      }
       }
     } else {
       // prologue path: wait for this thread's own copies of stage it (cp.async groups,
@@ -801,6 +837,39 @@ int make_weight_tmap(void* weights, uint32_t rows, uint32_t kpad, uint32_t box_r
   cuuint32_t estr[2] = {1, 1};
   CUresult r = enc((CUtensorMap*)out128, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, weights, dims, strides, box, estr,
                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? 0 : -1;
+}
+
+
+// Host: im2col tensor map of a conv's NHWC bf16 input (batch 1) for LF_TMA_B: channels
+// [in_co, in_co + cin) of a buffer with channel stride in_cs, BN pixels x 64 channels per
+// load, SW128 (the B operand's K-major layout), conv strides as traversal strides, the
+// padded window range as the pixel bounding box (out of bounds -> zero = padding).
+typedef CUresult (*EncodeIm2colFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                   const cuuint64_t*, const int*, const int*, cuuint32_t, cuuint32_t,
+                                   const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                   CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+int make_im2col_tmap(const void* in, const LayerArgs& a, uint32_t bn, void* out128) {
+  static EncodeIm2colFn enc = nullptr;
+  if (!enc) {
+    cudaDriverEntryPointQueryResult q;
+    void* fn = nullptr;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeIm2col", &fn, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess || !fn)
+      return -1;
+    enc = (EncodeIm2colFn)fn;
+  }
+  const cuuint64_t px = (cuuint64_t)a.in_cs * 2;
+  cuuint64_t dims[4] = {a.cin, a.w_, a.h, 1};
+  cuuint64_t strides[3] = {px, px * a.w_, px * a.w_ * a.h};
+  int lower[2] = {-(int)a.pw, -(int)a.ph};                                     // {W, H}
+  int upper[2] = {(int)a.pw - ((int)a.kw - 1), (int)a.ph - ((int)a.kh - 1)};
+  cuuint32_t estr[4] = {1, a.sw, a.sh, 1};
+  CUresult r = enc((CUtensorMap*)out128, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4,
+                   (void*)((const uint8_t*)in + (size_t)a.in_co * 2), dims, strides, lower, upper, TC_BK, bn, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS ? 0 : -1;
 }
