@@ -49,8 +49,12 @@ def _run(cmd, verbose):
 
 
 def build(verbose=False, ptxas_v=False, tsan=False):
-    build_dir = BUILD + ("_tsan" if tsan else "")
-    out = os.path.join(HERE, "libpaella_tsan.so") if tsan else OUT
+    # A/B build variants: PAELLA_BUILD_VARIANT=<name> builds libpaella_<name>.so in its own
+    # directory with the extra -D flags of PAELLA_DEFINES (load it with PAELLA_LIB)
+    variant = os.environ.get("PAELLA_BUILD_VARIANT", "") or ("tsan" if tsan else "")
+    defines = os.environ.get("PAELLA_DEFINES", "").split() if variant else []
+    build_dir = BUILD + ("_" + variant if variant else "")
+    out = os.path.join(HERE, f"libpaella_{variant}.so") if variant else OUT
     san = ["-fsanitize=thread"] if tsan else []
     os.makedirs(build_dir, exist_ok=True)
     headers = glob.glob(os.path.join(CSRC, "*.h")) + glob.glob(os.path.join(CSRC, "*.cuh")) + \
@@ -61,14 +65,14 @@ def build(verbose=False, ptxas_v=False, tsan=False):
         obj = os.path.join(build_dir, os.path.basename(src) + ".o")
         objs.append(obj)
         if _newer(src, obj, headers):
-            _run(["g++", "-O2", "-g", "-fPIC", *san, "-std=c++17", "-Wall", "-Wno-unused-function",
+            _run(["g++", "-O2", "-g", "-fPIC", *san, *defines, "-std=c++17", "-Wall", "-Wno-unused-function",
                   "-Wno-sign-compare", *inc, "-c", src, "-o", obj], verbose)
     for src in sorted(glob.glob(os.path.join(CSRC, "*.cu"))):
         obj = os.path.join(build_dir, os.path.basename(src) + ".o")
         objs.append(obj)
         if _newer(src, obj, headers):
             extra = ["-Xptxas", "-v"] if ptxas_v else []
-            _run([NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", *inc, *extra,
+            _run([NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", *inc, *extra, *defines,
                   "-c", src, "-o", obj], verbose or ptxas_v)
     if not os.path.exists(out) or any(os.path.getmtime(o) > os.path.getmtime(out) for o in objs):
         tmp = out + ".tmp"

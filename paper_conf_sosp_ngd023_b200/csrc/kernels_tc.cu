@@ -257,11 +257,12 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   constexpr uint32_t BNB = BN * TC_BK * 2;                      // B stage bytes: 8 / 16 KiB
   constexpr uint32_t ABY = BM * TC_BK * 2;                      // A stage bytes: 16 / 8 KiB (M 128 / 64)
   constexpr uint32_t NST = TC_RING / (ABY + BNB);           // 4 stages (BN 64) / 3 (BN 128) / 6 (M 64)
+  static_assert(NST <= 16, "barrier arrays hold 16 stages");
   constexpr uint32_t RPT = BN / 16;                             // B pixel rows per gather thread
   uint8_t* sB = smem + NST * ABY;
   uint64_t* full = (uint64_t*)(smem + TC_RING);
-  uint64_t* empty = full + 8;
-  uint64_t* accb = empty + 8;
+  uint64_t* empty = full + 16;
+  uint64_t* accb = empty + 16;
   uint64_t* rbar = accb + 1;                           // split-K: peers' slices landed
   uint32_t* tmem_slot = (uint32_t*)(rbar + 1);
   float* stage = reinterpret_cast<float*>(smem);       // epilogue tile [64 px][128 ch] fp32 (reuses sA)
@@ -801,7 +802,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   }
 }
 
-uint32_t tc_smem_bytes() { return 1024 + TC_RING + 256; }   // align pad + stage ring + barriers
+uint32_t tc_smem_bytes() { return 1024 + TC_RING + 512; }   // align pad + stage ring + barriers
 static_assert(TC_RING == TC_STAGES * (A_BYTES + B_BYTES), "ring");
 
 void tc_kernel_table(KernelFn* instr, KernelFn* plain) {
