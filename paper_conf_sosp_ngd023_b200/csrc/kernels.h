@@ -41,6 +41,10 @@ constexpr uint32_t TC_BK = 64;        // K per pipeline stage (128 B of bf16 = o
 #define PAELLA_TC_STAGES 4   // (A/B build variant: build.py PAELLA_DEFINES=-DPAELLA_TC_STAGES=8)
 #endif
 constexpr uint32_t TC_STAGES = PAELLA_TC_STAGES;
+#ifndef PAELLA_TC_ACCS
+#define PAELLA_TC_ACCS 1     // (A/B build variant) TMEM accumulators alternated over k-blocks
+#endif
+constexpr uint32_t TC_ACCS = PAELLA_TC_ACCS;
 constexpr uint32_t TC_RING = TC_STAGES * (TC_BM * TC_BK * 2 + TC_BN * TC_BK * 2);   // 96 KiB stage ring
 constexpr uint32_t TC_BN_WIDE = 128;   // KIND_CONV_TC128: 3 stages of 16 + 16 KiB in the same ring
 constexpr uint32_t GAPFC_CLUSTER = 8;   // fused GAP+FC head: CTAs per cluster (pooling split)

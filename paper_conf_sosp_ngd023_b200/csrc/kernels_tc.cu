@@ -520,7 +520,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   } else if (warp == 4) {
     // ------------------------------------------------------------ MMA warp
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(su32(tmem_slot)),
-                 "r"(BN)
+                 "r"(BN * TC_ACCS)
                  : "memory");
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
     tc_fence_before();
@@ -539,8 +539,10 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
         const uint32_t abase = su32(sA + s * ABY), bbase = su32(sB + s * BNB);
 #pragma unroll
         for (uint32_t kk = 0; kk < TC_BK / 16; ++kk) {
-          umma_bf16(tmem, sdesc_sw128(abase + kk * 32), sdesc_sw128(bbase + kk * 32), IDESC,
-                    (it | kk) != 0 ? 1u : 0u);
+          // TC_ACCS > 1: k-block it accumulates into accumulator it % TC_ACCS (independent
+          // accumulation chains), summed by the epilogue
+          umma_bf16(tmem + (it % TC_ACCS) * BN, sdesc_sw128(abase + kk * 32), sdesc_sw128(bbase + kk * 32), IDESC,
+                    ((it / TC_ACCS) | kk) != 0 ? 1u : 0u);
         }
         umma_commit(&empty[s]);
       }
@@ -581,6 +583,14 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
       for (uint32_t c = 0; c < BN / 16; ++c) {
         float v[16];
         tmem_ld16(taddr + c * 16, v);
+#pragma unroll
+        for (uint32_t q = 1; q < TC_ACCS; ++q)
+          if (q < nkl) {
+            float u[16];
+            tmem_ld16(taddr + q * BN + c * 16, u);
+#pragma unroll
+            for (int i = 0; i < 16; ++i) v[i] += u[i];
+          }
 #pragma unroll
         for (int i = 0; i < 16; ++i)
           if (owns) stage[(c * 16 + i) * BM + row] = v[i];
@@ -793,7 +803,7 @@ __global__ void __launch_bounds__(TC_THREADS, 2)
   __syncthreads();
   if (warp == 4) {
     tc_fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tmem_slot), "r"(BN) : "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(*tmem_slot), "r"(BN * TC_ACCS) : "memory");
     // every other thread is past the barrier above: the MMA warp, last to finish, counts
     // the block's exit itself (no second block barrier)
     if (trace && lane == 0) tr[6] = globaltimer();

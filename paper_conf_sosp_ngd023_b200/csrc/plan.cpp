@@ -49,7 +49,7 @@ static bool use_tc() {
   return !(e && std::string(e) == "simt");
 }
 
-uint32_t tc_tmem_cols() { return TC_BN < 32 ? 32 : TC_BN; }
+uint32_t tc_tmem_cols() { return (TC_BN < 32 ? 32 : TC_BN) * TC_ACCS; }
 
 int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
   const uint32_t n = d->n_nodes;
@@ -298,7 +298,7 @@ int plan_model(Paella* P, const paella_model_desc_t* d, Model* m) {
             if (k.kind == KIND_CONV_TC && split == 1 && tiles >= 4 * P->sms && !std::getenv("PAELLA_NO_WIDE")) {
               k.kind = KIND_CONV_TC128;
               a.tiles_n = (P_out + TC_BN_WIDE - 1) / TC_BN_WIDE;
-              k.tmem_cols = TC_BN_WIDE;
+              k.tmem_cols = TC_BN_WIDE * TC_ACCS;
             }
             // narrow layers (<= 64 output channels, no prologue): UMMA M = 64, so the tensor
             // core reads 64 weight rows per k-block instead of 128 (half of them zero)
