@@ -800,6 +800,9 @@ def main():
                    + f" K{args.max_active}{'a' if args.cap_fifo else ''} la{args.lookahead}{'' if args.lookahead_placed else 'u'}"
                    + f" B{args.slack} pdl"
                    + (" branches" if args.branches else ""),
+                   "kernels": "tcgen05 conv, split-K gain " + os.environ.get("PAELLA_SPLIT_GAIN", "65") + "%"
+                   + (", LDGSTS gather" if os.environ.get("PAELLA_NO_TMA_B") else ", TMA im2col B")
+                   + (", M64" if os.environ.get("PAELLA_M64") else ""),
                    "l2": "not flushed: weights (~120 MB bf16) largely L2-resident as in serving; inputs stream "
                          "from pinned host memory every request"},
         "roofline": roofline_entry(dict(P, config=args.config), peaks) if "kinfo" in P else None,
